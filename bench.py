@@ -1,0 +1,461 @@
+#!/usr/bin/env python
+"""bench.py -- Betty's micro-batch GNN training step on B200 (the metric of
+BASELINE.json: epoch time & aggregated edges/s, SAGE, products-shape).
+
+One step (= one epoch of the paper, Table 6 "training time per epoch",
+PAPER.md:1668-1679) is the whole hot path over one batch: the REG rebuild
+(a1), extraction of every micro-batch (a2), SAGE forward (a3), loss (a4),
+backward (a5) with fused gradient accumulation (a6), the all-reduce across
+ranks and the Adam update (a7).  Sampling and the host partitioner are
+outside (the paper also excludes "data preparing").
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+
+For N > 1 it runs under torchrun, one rank per GPU over NCCL; micro-batches
+are LPT-assigned to ranks and K (micro-batches per batch) is fixed across N
+(the total work is the same batch), so the scaling is STRONG.
+Prints ONE JSON line on rank 0.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+
+def parse():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=20)
+    p.add_argument("--warmup", type=int, default=3)
+    p.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    p.add_argument("--config", default="C3")
+    p.add_argument("--K", type=int, default=32, help="micro-batches per batch (fixed across GPU counts)")
+    p.add_argument("--mode", default="bf16", choices=["fp32", "bf16"], help="GEMM operand precision")
+    p.add_argument("--group", type=int, default=0, help="micro-batches per launch group (0 = all of a rank's)")
+    p.add_argument("--partition", default="reg", choices=["reg", "range", "random"])
+    p.add_argument("--no-graph", action="store_true")
+    p.add_argument("--no-reg", action="store_true", help="exclude the REG rebuild (a1) from the step")
+    p.add_argument("--probe", default="auto")
+    p.add_argument("--e2e-steps", type=int, default=5)
+    p.add_argument("--cpu-sample-outputs", type=int, default=4096, help="cpu_baseline sample (~10 s)")
+    p.add_argument("--ref-sample-outputs", type=int, default=1024, help="--impl reference per-step sample")
+    p.add_argument("--scale", type=float, default=1.0, help="shrink the graph (debug only)")
+    p.add_argument("--json-out", default=None)
+    return p.parse_args()
+
+
+# ------------------------------------------------------------------ helpers
+def dist_env():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return ws, rank, local
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled DURING the timed region."""
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device: int):
+        self.device = device
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                                          "-lms", "200", "-i", str(self.device)], stdout=subprocess.PIPE,
+                                         stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if not self.proc:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1]))
+                mx = float(f[2])
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[5:9]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return d, "measured (MEASURED_PEAKS.json)"
+    return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0}, \
+        "fallback (B200_PROFILING.md)"
+
+
+def load_traffic(kernel: str, key: str):
+    """ncu dram bytes per launch from a committed capture (profiles/), or None."""
+    p = os.path.join(ROOT, "profiles", "traffic.json")
+    if not os.path.exists(p):
+        return None
+    with open(p) as f:
+        d = json.load(f)
+    return d.get(key, {}).get(kernel)
+
+
+# -------------------------------------------------------------- the workload
+def build_inputs(args, rank, ws, device):
+    """Rank 0 generates the synthetic products-shaped batch (C + OpenMP) and
+    broadcasts it; every rank ends with the same host arrays."""
+    import torch
+    import torch.distributed as dist
+    import synth
+    cfg = synth.CONFIGS[args.config]
+    if args.scale != 1.0:
+        cfg = synth.scaled(cfg, args.scale)
+    t0 = time.time()
+    if rank == 0:
+        ds = synth.make(cfg)
+        arrays = [ds.feats, ds.labels, ds.seeds]
+        for b in ds.blocks:
+            arrays += [b.indptr, b.nbr_pos, b.src_gid]
+    else:
+        ds, arrays = None, None
+    if ws > 1:
+        meta = [None]
+        if rank == 0:
+            meta = [[(a.shape, str(a.dtype)) for a in arrays]]
+        dist.broadcast_object_list(meta, src=0)
+        out = []
+        for i, (shape, dt) in enumerate(meta[0]):
+            t = torch.from_numpy(arrays[i]).to(device) if rank == 0 else \
+                torch.empty(shape, dtype=getattr(torch, dt), device=device)
+            dist.broadcast(t, src=0)
+            out.append(t.cpu().numpy())
+        arrays = out
+        if rank != 0:
+            blocks = []
+            for l in range(cfg.L):
+                ip, nb, sg = arrays[3 + 3 * l: 6 + 3 * l]
+                blocks.append(synth.Block(len(ip) - 1, len(sg), ip, nb, sg))
+            ds = synth.Dataset(cfg, None, arrays[0], arrays[1], arrays[2], blocks)
+    return cfg, ds, time.time() - t0
+
+
+def make_partition(args, B, ctx, cfg, ds, dev_blocks, rank, ws, device):
+    import torch
+    import torch.distributed as dist
+    import synth
+    if args.partition == "range":
+        part = synth.range_partition(cfg.n_out, args.K)
+    elif args.partition == "random":
+        part = synth.random_partition(cfg.n_out, args.K, cfg.seeds["part"])
+    else:
+        part = None
+        if rank == 0:
+            ip, col, w = B.betty_reg_build(ctx, dev_blocks[-1])
+            part = B.betty_reg_partition(ip.cpu().numpy(), col.cpu().numpy(), w.cpu().numpy(), args.K)
+        if ws > 1:
+            t = torch.as_tensor(part if rank == 0 else np.zeros(cfg.n_out, np.int32)).to(device)
+            dist.broadcast(t, src=0)
+            part = t.cpu().numpy()
+    return np.ascontiguousarray(part, dtype=np.int32)
+
+
+def alg_bytes(site: str, info: dict, cfg, mode: str, n_groups: int):
+    """Algorithmic (compulsory) bytes of ONE launch of a kernel site, from the
+    plan's per-layer totals.  Totals / n_groups = per launch."""
+    s_feat = 2 if mode == "bf16" else 4
+    s_act = 2 if mode == "bf16" else 4
+    E, ns, nd = info["edges"], info["n_src"], info["n_dst"]
+    F = cfg.F
+    Fp = (F + 7) // 8 * 8
+    ld_xa = (2 * Fp + 1 + 7) // 8 * 8
+    if site == "agg_l0":
+        b = 8 * (nd[0] + 1) + 4 * E[0] + 4 * ns[0] + s_feat * F * ns[0] + s_act * ld_xa * nd[0]
+    elif site == "gemm_fwd_l0":
+        H = cfg.hidden
+        b = s_act * ld_xa * nd[0] + s_act * (2 * Fp + 1) * H + s_act * ((H + 1 + 7) // 8 * 8) * nd[0]
+    else:
+        return None
+    return b / max(n_groups, 1)
+
+
+# ------------------------------------------------------------ reference arm
+def run_reference(args, ws, rank):
+    """The CPU oracle, as it stands, on a bounded sample of the same workload
+    (micro-batch 0 of the bench's partition, its first S outputs)."""
+    if rank != 0:
+        return
+    import synth
+    import oracle
+    cfg = synth.CONFIGS[args.config]
+    if args.scale != 1.0:
+        cfg = synth.scaled(cfg, args.scale)
+    ds = synth.make(cfg)
+    part, sample_desc, edges = reference_sample(args, cfg, ds, args.ref_sample_outputs)
+    params = synth.init_params(cfg.dims, cfg.aggr, seed=cfg.seeds["init"])
+    times = []
+    for it in range(args.warmup + args.steps):
+        t0 = time.perf_counter()
+        oracle.step(cfg.dims, cfg.aggr, args.mode == "bf16", ds.blocks, part, 2, [0], params, ds.feats, ds.labels,
+                    1.0 / cfg.n_out)
+        if it >= args.warmup:
+            times.append(time.perf_counter() - t0)
+    t = float(np.mean(times))
+    val = edges / t
+    line = {"impl": "reference", "metric": "aggregated edges/s (SAGE, products-shape)", "value": val,
+            "unit": "edges/s", "higher_is_better": True, "n_gpus": args.gpus, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": t * 1e3, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": f"{args.config} {cfg.name}-shaped, bounded sample", "sample": sample_desc},
+            "cpu_baseline": {"value": val, "unit": "edges/s", "cores": 1, "kind": "oracle", "sample": sample_desc},
+            "e2e": {"value": val, "unit": "edges/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def reference_sample(args, cfg, ds, n_outputs):
+    """Outputs: the first S outputs (ascending) of micro-batch 0 of a range
+    partition into K parts -> a 2-way partition {sample, rest}."""
+    import synth
+    import oracle
+    base = synth.range_partition(cfg.n_out, args.K)
+    idx = np.nonzero(base == 0)[0][:n_outputs]
+    part = np.ones(cfg.n_out, dtype=np.int32)
+    part[idx] = 0
+    mb = oracle.extract(ds.blocks, part, 2, 0)
+    edges = sum(b.n_edges for b in mb)
+    desc = (f"{len(idx)} outputs (first of micro-batch 0, K={args.K}); {edges} edges through "
+            f"{cfg.L} layers; extraction+fwd+bwd in float64, 1 thread")
+    return part, desc, edges
+
+
+# -------------------------------------------------------------------- main
+def main():
+    args = parse()
+    ws, rank, local = dist_env()
+    if args.impl == "reference":
+        run_reference(args, ws, rank)
+        return
+    import torch
+    import torch.distributed as dist
+    import paper_conf_asplos_yangzd023_b200 as B
+    from paper_conf_asplos_yangzd023_b200.dist import allreduce_grad, lpt_assign, micro_batch_costs
+
+    torch.cuda.set_device(local)
+    device = torch.device("cuda", local)
+    if ws > 1:
+        dist.init_process_group("nccl", device_id=device)
+    cfg, ds, t_gen = build_inputs(args, rank, ws, device)
+    ctx = B.betty_ctx_create(local)
+    dev_blocks = B.blocks_to_device(ds.blocks, local)
+    part = make_partition(args, B, ctx, cfg, ds, dev_blocks, rank, ws, device)
+    dpart = torch.as_tensor(part).to(device)
+    costs = micro_batch_costs(part, args.K, ds.blocks[-1].indptr)
+    my_k = lpt_assign(costs, ws)[rank]
+
+    feats = torch.as_tensor(ds.feats).to(device)
+    if args.mode == "bf16":
+        feats = feats.to(torch.bfloat16).contiguous()       # bf16 feature table (reading #17)
+    labels = torch.as_tensor(ds.labels).to(device)
+    model = B.Model(cfg.dims, cfg.aggr, args.mode, args.mode)
+    params = torch.as_tensor(synth_params(cfg)).to(device)
+    grad = torch.zeros_like(params)
+    m = torch.zeros_like(params)
+    v = torch.zeros_like(params)
+    loss = torch.zeros(1, device=device)
+    flags = (0 if args.no_graph else B.PLAN_GRAPH) | (0 if args.no_reg else B.PLAN_REG)
+    t0 = time.time()
+    plan = B.betty_plan_create(ctx, model, dev_blocks, dpart, args.K, my_k, group=args.group, flags=flags)
+    t_plan = time.time() - t0
+    info = plan.info()
+    scale = 1.0 / cfg.n_out
+    stream = torch.cuda.current_stream()
+    t_opt = [0]
+
+    def step():
+        loss.zero_()
+        B.betty_step(ctx, plan, params, feats, labels, scale, grad, loss)
+        allreduce_grad(grad)
+        t_opt[0] += 1
+        B.betty_adam(ctx, params, grad, m, v, t_opt[0], zero_grad=True)
+
+    for _ in range(args.warmup):
+        step()
+    B.betty_sync_check(ctx)
+
+    # ------------------------------------------------------ timed region
+    clocks = ClockSampler(local)
+    if ws > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    clocks.start()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for _ in range(args.steps):
+        step()
+    e1.record(stream)
+    torch.cuda.synchronize()
+    if ws > 1:
+        dist.barrier()
+    clk = clocks.stop()
+    ms = e0.elapsed_time(e1) / args.steps
+    t = torch.tensor([ms, float(sum(info["edges"])), float(info["kernels_per_step"])], device=device,
+                     dtype=torch.float64)
+    if ws > 1:
+        tmax = t.clone()
+        dist.all_reduce(tmax, op=dist.ReduceOp.MAX)
+        tsum = t.clone()
+        dist.all_reduce(tsum, op=dist.ReduceOp.SUM)
+        ms_step, edges_all = float(tmax[0]), float(tsum[1])
+    else:
+        ms_step, edges_all = ms, float(t[1])
+    value = edges_all / (ms_step * 1e-3)
+    launches = args.steps * (info["kernels_per_step"] + 1)
+
+    # ------------------------------------- e2e: host buffers through the ABI
+    host = []
+    for b in ds.blocks:
+        host += [torch.from_numpy(b.indptr).pin_memory(), torch.from_numpy(b.nbr_pos).pin_memory(),
+                 torch.from_numpy(b.src_gid).pin_memory()]
+    host.append(torch.from_numpy(part).pin_memory())
+    devs = []
+    for db in dev_blocks:
+        devs += [db.indptr, db.indices, db.src_gid]
+    devs.append(dpart)
+    h2d = sum(x.numel() * x.element_size() for x in host)
+    loss_host = torch.zeros(1).pin_memory()
+    if ws > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    f0.record(stream)
+    for _ in range(args.e2e_steps):
+        for hsrc, ddst in zip(host, devs):
+            ddst.copy_(hsrc, non_blocking=True)
+        step()
+        loss_host.copy_(loss, non_blocking=True)
+        stream.synchronize()
+        _ = float(loss_host[0])
+    f1.record(stream)
+    torch.cuda.synchronize()
+    e2e_ms = f0.elapsed_time(f1) / args.e2e_steps
+    if ws > 1:
+        te = torch.tensor([e2e_ms], device=device, dtype=torch.float64)
+        dist.all_reduce(te, op=dist.ReduceOp.MAX)
+        e2e_ms = float(te[0])
+
+    # ---------------------------------- roofline of the dominant kernel
+    sites = {"agg_l0": 1, "gemm_fwd_l0": 2, "gemm_red_l0": 3, "extract": 4, "reg": 5}
+    probe_ms = {}
+    for name, sid in sites.items():
+        plan.probe(sid)
+        tot, n = 0.0, 0
+        for _ in range(3):
+            step()
+            ms_k, nl = plan.probe_read()
+            tot += ms_k
+            n += nl
+        probe_ms[name] = (tot / max(n, 1), n / 3)
+    plan.probe(0)
+    peaks, peak_src = measured_peaks()
+    key = f"{args.config}:K{args.K}:{args.mode}:n{ws}"
+    dom = "agg_l0"
+    per_launch_ms, launches_per_step = probe_ms[dom]
+    ab = alg_bytes(dom, info, cfg, args.mode, info["n_groups"])
+    achieved = ab / (per_launch_ms * 1e-3) / 1e9
+    roof = {"kernel": "k_agg_mean_xa (layer-0 mean aggregation)", "bound": "hbm", "achieved": achieved,
+            "peak": peaks["hbm_gbs"], "unit": "GB/s", "frac": achieved / peaks["hbm_gbs"],
+            "traffic": load_traffic(dom, key), "alg_bytes_per_launch": ab, "avg_launch_ms": per_launch_ms,
+            "launches_per_step": launches_per_step, "peak_source": peak_src,
+            "share_of_step": per_launch_ms * launches_per_step / ms,
+            "other_sites_ms_per_step": {k: v[0] * v[1] for k, v in probe_ms.items()}}
+
+    # ------------------------------------------------------- cpu baseline
+    cpu = None
+    if rank == 0 and ws == 1:
+        import oracle
+        rpart, desc, redges = reference_sample(args, cfg, ds, args.cpu_sample_outputs)
+        pr = synth_params(cfg).astype(np.float64)
+        tc = time.perf_counter()
+        oracle.step(cfg.dims, cfg.aggr, args.mode == "bf16", ds.blocks, rpart, 2, [0], pr, ds.feats, ds.labels,
+                    scale)
+        dt = time.perf_counter() - tc
+        cpu = {"value": redges / dt, "unit": "edges/s", "cores": 1, "kind": "oracle", "sample": desc,
+               "seconds": dt}
+
+    if rank == 0:
+        line = {
+            "metric": "aggregated edges/s (SAGE, products-shape); epoch time = ms_per_step",
+            "value": value, "unit": "edges/s", "n_gpus": ws, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": ms_step, "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+            "dtype": "bf16-gemm/fp32-accum" if args.mode == "bf16" else "fp32",
+            "data": "synthetic",
+            "config": {"workload": f"{args.config}: {cfg.name}-shaped DC-SBM ({cfg.n} nodes, "
+                                   f"{len(ds.feats)}x{cfg.F} feats), {cfg.L}-layer SAGE-{cfg.aggr} "
+                                   f"{cfg.dims}, fanout {tuple(cfg.fanouts)}, {cfg.n_out} outputs",
+                       "K": args.K, "partition": args.partition, "group": args.group or "all",
+                       "micro_batches_per_rank": len(my_k), "step": ("REG + " if not args.no_reg else "") +
+                       "extract + fwd + loss + bwd + allreduce + adam", "graph": not args.no_graph,
+                       "parallelism": f"dp{ws} over micro-batches",
+                       "l2": "inputs > L2 (feature table %.2f GB + blocks)" % (feats.numel() * feats.element_size()
+                                                                           / 1e9)},
+            "edges_per_step": edges_all,
+            "full_batch_edges": int(sum(b.n_edges for b in ds.blocks)),
+            "plan": {k: info[k] for k in ("n_groups", "edges", "n_src", "n_dst", "reg_nnz", "arena_bytes",
+                                          "kernels_per_step")},
+            "e2e": {"value": edges_all / (e2e_ms * 1e-3), "unit": "edges/s", "ms_per_step": e2e_ms,
+                    "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": 4},
+            "gpu_launches": launches,
+            "clocks": clk,
+            "roofline": roof,
+            "cpu_baseline": cpu,
+            "paper_context": "Table 6 (RTX 6000, real ogbn-products, fp32): 0.85 s/epoch at K=8, 2.55 s at K=64",
+            "setup_s": {"generate": t_gen, "plan": t_plan},
+        }
+        s = json.dumps(line)
+        print(s, flush=True)
+        if args.json_out:
+            with open(args.json_out, "w") as f:
+                f.write(s + "\n")
+    plan.free()
+    if ws > 1:
+        dist.destroy_process_group()
+
+
+def synth_params(cfg):
+    import synth
+    return synth.init_params(cfg.dims, cfg.aggr, seed=cfg.seeds["init"])
+
+
+if __name__ == "__main__":
+    main()

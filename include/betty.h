@@ -1,0 +1,226 @@
+/*
+ * betty.h -- C ABI of the B200-native hot path of Betty's batch-level
+ * partitioned GNN training step (Yang et al., ASPLOS '23; PAPER.md).
+ *
+ * The library (paper_conf_asplos_yangzd023_b200/libbetty.so) is hand-written
+ * CUDA for sm_100a.  Every entry point takes plain pointers and sizes; no torch
+ * types cross this boundary.  Unless noted, pointers are DEVICE pointers on
+ * the ctx's device, calls are stream-ordered on `stream` (a cudaStream_t,
+ * passed as void* so this header needs no CUDA include) and asynchronous.
+ * No exceptions cross the ABI; every failure is a betty_status, with a message
+ * from betty_last_error().
+ *
+ * Terminology (§4.2.2-4.2.3).  A batch is a multi-level
+ * bipartite graph: block l (l = 0 input ... L-1 output) has dst nodes V and
+ * src nodes U with dst ids == src ids [0, n_dst) (the dst list is a prefix of
+ * the src list).  Betty partitions the output nodes into K micro-batches; the
+ * micro-batch k of every layer is the sub-bipartite reachable from its
+ * outputs.  Gradients of the K micro-batches are summed and give the
+ * full-batch gradient.
+ */
+#ifndef BETTY_H
+#define BETTY_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define BETTY_API __attribute__((visibility("default")))
+#else
+#define BETTY_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    BETTY_OK = 0,
+    BETTY_EINVAL = 1,       /* bad argument (null pointer, k out of range, part[] out of range, duplicate edge ...) */
+    BETTY_ENOMEM = 2,       /* the allocator returned null */
+    BETTY_ECUDA = 3,        /* a CUDA runtime error; message in betty_last_error */
+    BETTY_EOVERFLOW = 4,    /* a size exceeds int32 local ids or a plan capacity */
+    BETTY_EUNSUPPORTED = 5  /* a configuration this build does not implement */
+} betty_status;
+
+typedef struct betty_ctx betty_ctx;
+typedef void* betty_stream;                                          /* cudaStream_t */
+typedef void* (*betty_alloc_fn)(size_t bytes, betty_stream stream, void* user);
+typedef void (*betty_free_fn)(void* ptr, betty_stream stream, void* user);
+
+/* One context per device (per rank).  alloc/free may be NULL: the library
+ * then uses the CUDA stream-ordered allocator (cudaMallocAsync).  Outputs of
+ * betty_extract_blocks / betty_reg_build / betty_sage_fwd and plan arenas come
+ * from this allocator and are released with the matching *_free call. */
+BETTY_API betty_status betty_ctx_create(int device, betty_alloc_fn alloc, betty_free_fn dealloc, void* user, betty_ctx** out);
+BETTY_API void betty_ctx_destroy(betty_ctx* ctx);
+BETTY_API const char* betty_last_error(const betty_ctx* ctx);
+BETTY_API const char* betty_version(void);
+
+/* One bipartite layer, CSR by dst.
+ *   indptr    [n_dst+1] int64    row offsets
+ *   indices   [n_edges] int32    src ids: local ids for a micro-batch; for the FULL batch given to
+ *                                betty_extract_blocks, positions in the full-batch src list
+ *   src_pos   [n_src]   int32    position of each src in the full-batch src list of this layer
+ *                                (NULL for the full batch = identity)
+ *   src_gid   [n_src]   int32    global node id (row of the feature / label tables)
+ *   t_indptr  [n_src+1] int64    CSC (dst ids per src), may be NULL on input
+ *   t_indices [n_edges] int32    dst ids, ascending per column
+ * Canonical order (readings #9/#10): outputs ascending; src =
+ * dst ++ (new sources ascending full-batch src position); rows keep the
+ * full-batch order.  Sizes are host values. */
+typedef struct {
+    int64_t n_dst, n_src, n_edges;
+    int64_t* indptr;
+    int32_t* indices;
+    int32_t* src_pos;
+    int32_t* src_gid;
+    int64_t* t_indptr;
+    int32_t* t_indices;
+} betty_block;
+
+/* Symmetric weighted CSR (the REG): n rows, nnz entries, int64 indptr[n+1],
+ * int32 col[nnz] ascending per row, int32 w[nnz] >= 1, no diagonal. */
+typedef struct {
+    int64_t n, nnz;
+    int64_t* indptr;
+    int32_t* col;
+    int32_t* w;
+} betty_csr;
+
+enum { BETTY_AGGR_MEAN = 0, BETTY_AGGR_POOL = 1 };
+enum { BETTY_GEMM_FP32 = 0, BETTY_GEMM_BF16 = 1 };
+enum { BETTY_FEAT_FP32 = 0, BETTY_FEAT_BF16 = 1 };
+
+/* GraphSAGE model (Table 1; Eq. 1; DGL SAGEConv
+ * form, reading #11): L layers of widths dims[0..L] (host array).
+ * Parameters are one flat fp32 vector; per layer l (Fi = dims[l], Fo = dims[l+1]):
+ *   pool only: W_pool [Fi x Fi], b_pool [Fi]
+ *   W_self [Fi x Fo], W_neigh [Fi x Fo], b [Fo]          (row-major, x . W)
+ * gemm: FP32 = fp32 SIMT everywhere (no TF32); BF16 = GEMM operands in bf16,
+ * fp32 accumulation, aggregation / loss / gradients fp32, hidden activations
+ * stored bf16 (reading #17).  feat_dtype says how `feats` is stored. */
+typedef struct {
+    int32_t L;
+    int32_t aggr;
+    int32_t gemm;
+    int32_t feat_dtype;
+    const int32_t* dims;
+} betty_model;
+
+BETTY_API int64_t betty_num_params(const betty_model* model);
+
+/* a1 -- REG (§4.3.2, Eq. 2-4, Alg. 1 lines 1-7 PAPER.md:934-940).
+ * out_layer: the output block of the FULL batch (n_dst = n_out rows, indices =
+ * full-batch src positions in [0, n_src)).  Computes c_ij = #shared sources of
+ * outputs i != j as an integer SpGEMM B.B^T (B[i,u] = 1 iff u -> i); zero
+ * entries dropped, diagonal removed.  Rows must not repeat a source (binary A,
+ * reading #2): a repeat returns EINVAL.  Allocates reg's arrays; synchronizes
+ * the stream once to learn nnz.  Result is bit-exact (integer). */
+BETTY_API betty_status betty_reg_build(betty_ctx* ctx, const betty_block* out_layer, betty_csr* reg, betty_stream stream);
+BETTY_API void betty_csr_free(betty_ctx* ctx, betty_csr* reg);
+
+/* a2 -- micro-batch extraction (batch-level partition, PAPER.md:535-547;
+ * block generation and the local<->global index map).
+ * full[L]: full-batch blocks (indices = full-batch src positions; src_pos may
+ * be NULL).  part[n_out] (device) assigns each output position to [0,K).
+ * Fills mb[L] with micro-batch k (all arrays allocated, CSC included,
+ * sizes written on the host after one stream synchronisation).  part values
+ * out of range return EINVAL.  An empty micro-batch yields zero-sized blocks. */
+BETTY_API betty_status betty_extract_blocks(betty_ctx* ctx, const betty_block* full, int32_t L, const int32_t* part,
+                                  int64_t n_out, int32_t K, int32_t k, betty_block* mb, betty_stream stream);
+BETTY_API void betty_block_free(betty_ctx* ctx, betty_block* blocks, int32_t L);
+
+/* a3 -- forward of one micro-batch (mean: h_N = (1/D_v) sum h_u, or pool:
+ * max_u ReLU(W_pool h_u + b_pool); then h_v W_self + h_N W_neigh + b; ReLU
+ * between layers).  mb[L] as returned by betty_extract_blocks (host sizes,
+ * CSC present).  feats: [N x ld_feats] table indexed by src_gid of layer 0.
+ * logits (optional) [n_dst(L-1) x dims[L]] fp32.  *saved receives the
+ * activations the backward needs (free with betty_saved_free). */
+typedef struct betty_saved betty_saved;
+BETTY_API betty_status betty_sage_fwd(betty_ctx* ctx, const betty_model* model, const float* params, const betty_block* mb,
+                            const void* feats, int64_t ld_feats, betty_saved** saved, float* logits,
+                            betty_stream stream);
+/* a4+a5+a6 -- softmax cross-entropy on the micro-batch's outputs (labels[gid],
+ * int32), scaled by loss_scale (1/n_out of the full batch, so that the K
+ * micro-batch losses sum to the full-batch mean loss, reading #15), and the
+ * backward, ADDING the gradient into grad_accum[num_params] (fused
+ * accumulation across micro-batches) and the loss into
+ * loss_accum[0]. */
+BETTY_API betty_status betty_sage_bwd(betty_ctx* ctx, const betty_model* model, const float* params, const betty_block* mb,
+                            const betty_saved* saved, const int32_t* labels, float loss_scale, float* grad_accum,
+                            float* loss_accum, betty_stream stream);
+BETTY_API void betty_saved_free(betty_ctx* ctx, betty_saved* saved);
+
+/* The fused per-step path.  A plan binds the full batch, the partition and
+ * this rank's micro-batches my_k[n_my] (host array); it runs one extraction
+ * pass (synchronising) to size device arenas, so that betty_step itself never
+ * synchronises and can be captured in / replayed as a CUDA graph.
+ * group: micro-batches executed together per launch (>= 1; <= 0 means all of
+ * this rank's).  A group is the block-diagonal union of its micro-batches:
+ * per-micro-batch dedupe / relabel / numerics are unchanged; memory grows
+ * with the group.  flags: BETTY_PLAN_GRAPH captures the step as a CUDA graph
+ * on first use; BETTY_PLAN_REG rebuilds the REG (a1) inside every step. */
+typedef struct betty_plan betty_plan;
+enum { BETTY_PLAN_GRAPH = 1, BETTY_PLAN_REG = 2 };
+typedef struct {
+    int32_t n_groups;            /* launch groups per step */
+    int32_t L;
+    int64_t edges[16];           /* sum over this rank's micro-batches of E_l   (l = 0..L-1) */
+    int64_t n_src[16];           /* sum of n_src,l */
+    int64_t n_dst[16];           /* sum of n_dst,l */
+    int64_t max_group_edges[16]; /* capacity used for layer l */
+    int64_t reg_nnz;             /* last REG nnz (BETTY_PLAN_REG) */
+    int64_t arena_bytes;         /* device bytes held by the plan */
+    int32_t kernels_per_step;    /* library kernel launches per betty_step */
+} betty_plan_info;
+BETTY_API betty_status betty_plan_create(betty_ctx* ctx, const betty_model* model, const betty_block* full, int32_t L,
+                               const int32_t* part, int64_t n_out, int32_t K, const int32_t* my_k, int32_t n_my,
+                               int32_t group, int32_t flags, betty_plan** out, betty_stream stream);
+BETTY_API betty_status betty_plan_info_get(const betty_plan* plan, betty_plan_info* info);
+BETTY_API void betty_plan_destroy(betty_ctx* ctx, betty_plan* plan);
+
+/* One training step on this rank: for every micro-batch of the plan,
+ * extraction (a2) -> forward (a3) -> loss (a4) -> backward (a5) with the
+ * gradient ADDED into grad_accum (a6).  The caller then all-reduces
+ * grad_accum across ranks (NCCL) and applies betty_adam (a7). */
+BETTY_API betty_status betty_step(betty_ctx* ctx, betty_plan* plan, const float* params, const void* feats,
+                        int64_t ld_feats, const int32_t* labels, float loss_scale, float* grad_accum,
+                        float* loss_accum, betty_stream stream);
+
+/* a7 -- Adam (PyTorch semantics; PAPER.md:1115-1118 names Adam), one fused
+ * kernel over the flat parameter vector: m = b1 m + (1-b1) g;
+ * v = b2 v + (1-b2) g^2; p -= lr * (m / (1-b1^t)) / (sqrt(v / (1-b2^t)) + eps).
+ * zero_grad != 0 also clears g for the next step. */
+BETTY_API betty_status betty_adam(betty_ctx* ctx, float* params, float* grad, float* m, float* v, int64_t n, int32_t t,
+                        float lr, float b1, float b2, float eps, int32_t zero_grad, betty_stream stream);
+
+/* Measurement hook: bracket every launch of one kernel site with CUDA events
+ * on the step's stream in subsequent betty_step calls (graph replays
+ * included; changing the site re-captures the graph).  Sites: 0 off,
+ * 1 layer-0 aggregation, 2 layer-0 forward GEMM, 3 layer-0 dW GEMM,
+ * 4 extraction (whole group), 5 REG, 6 layer-1 aggregation, 7 layer-1
+ * forward GEMM.  probe_read synchronises and returns the summed elapsed time
+ * of the last step's bracketed launches and their number. */
+enum { BETTY_PROBE_OFF = 0, BETTY_PROBE_AGG_L0 = 1, BETTY_PROBE_GEMM_FWD_L0 = 2, BETTY_PROBE_GEMM_RED_L0 = 3,
+       BETTY_PROBE_EXTRACT = 4, BETTY_PROBE_REG = 5, BETTY_PROBE_AGG_L1 = 6, BETTY_PROBE_GEMM_FWD_L1 = 7 };
+BETTY_API betty_status betty_plan_probe(betty_plan* plan, int32_t site);
+BETTY_API betty_status betty_plan_probe_read(betty_plan* plan, float* total_ms, int32_t* launches);
+
+/* HOST function, outside the hot path (Alg. 1 line 8, where
+ * the paper calls METIS): K-way partition of a REG given as HOST arrays
+ * (indptr[n+1], col[nnz], w[nnz] or NULL for unit weights) by greedy graph
+ * growing on the REG weights (the most shared inputs stay together), with
+ * balanced part sizes floor/ceil(n/K).  Writes part[n] (host).  Deterministic. */
+BETTY_API betty_status betty_reg_partition(const int64_t* indptr, const int32_t* col, const int32_t* w, int64_t n,
+                                           int32_t K, int32_t* part);
+
+/* Synchronise `stream` and report device-side errors of earlier
+ * asynchronous calls (part[] out of range -> EINVAL, capacity exceeded ->
+ * EOVERFLOW, CUDA faults -> ECUDA). */
+BETTY_API betty_status betty_sync_check(betty_ctx* ctx, betty_stream stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* BETTY_H */

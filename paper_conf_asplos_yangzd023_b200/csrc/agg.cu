@@ -1,0 +1,372 @@
+// agg.cu -- a3/a5: GraphSAGE aggregation forward and backward (HBM-bound
+// CSR segment reductions), Table 1, Eq. 1 PAPER.md:269.
+//
+// Forward kernels write the A operand of the following dense GEMM directly
+// (fusing the concat and the bias "ones" column):
+//   mean, aggregate-first:  XA[v] = [ h_v | (1/D_v) sum_{u in N(v)} h_u | 1 ]
+//   mean, project-first:    S[v]  = Y[v, self] + (1/D_v) sum_u Y[u, neigh]
+//                           (Y = [H|1] [W_n | W_s ; 0 | b] from the GEMM)
+//   pool:                   XA[v] = [ h_v | max_u ReLU(Zp[u]) | 1 ], argmax
+// Backward kernels gather through the CSC (deterministic, no float atomics).
+// Feature rows are read with 128-bit vector loads; one warp owns a dst row
+// and its lanes cover the row's 16-byte vectors; edge indices are loaded 32
+// at a time and broadcast with shuffles, and up to 4 neighbour rows are in
+// flight per lane.
+#include "common.cuh"
+#include "internal.h"
+#include "sage.h"
+
+namespace betty {
+
+template <typename T> __device__ __forceinline__ const T* row_ptr(const T* X, int64_t ld, const int32_t* xrow, int64_t r) {
+    return X + (int64_t)(xrow ? xrow[r] : (int32_t)r) * ld;
+}
+
+// ------------------------------------------------ mean, aggregate-first fwd
+template <typename Tin, typename Tout>
+__global__ void __launch_bounds__(256) k_agg_mean_xa(const Tin* __restrict__ X, int64_t ldx,
+                                                     const int32_t* __restrict__ xrow,
+                                                     const int64_t* __restrict__ indptr,
+                                                     const int32_t* __restrict__ idx, const int64_t* cnt, int Fi,
+                                                     int Fp, Tout* __restrict__ XA, int64_t ldxa) {
+    using VI = Vec<Tin>;
+    constexpr int VW = VI::N;
+    const int64_t nd = cnt[0];
+    const int NV = (Fi + VW - 1) / VW;
+    const int lane = lane_id();
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t v = gw; v < nd; v += nw) {
+        const int64_t b = indptr[v], e = indptr[v + 1];
+        const float inv = e > b ? 1.0f / (float)(e - b) : 0.0f;
+        Tout* out = XA + v * ldxa;
+        for (int vb = 0; vb < NV; vb += 32) {
+            const int vi = vb + lane;
+            const bool act = vi < NV;
+            float acc[VW];
+#pragma unroll
+            for (int t = 0; t < VW; ++t) acc[t] = 0.f;
+            for (int64_t e0 = b; e0 < e; e0 += 32) {
+                const int n = (int)mn64(32, e - e0);
+                const int32_t my = lane < n ? idx[e0 + lane] : 0;
+                int j = 0;
+                for (; j + 4 <= n; j += 4) {
+                    VI x0, x1, x2, x3;
+                    const int32_t u0 = __shfl_sync(0xffffffffu, my, j);
+                    const int32_t u1 = __shfl_sync(0xffffffffu, my, j + 1);
+                    const int32_t u2 = __shfl_sync(0xffffffffu, my, j + 2);
+                    const int32_t u3 = __shfl_sync(0xffffffffu, my, j + 3);
+                    if (act) {
+                        x0.load(row_ptr(X, ldx, xrow, u0) + vi * VW);
+                        x1.load(row_ptr(X, ldx, xrow, u1) + vi * VW);
+                        x2.load(row_ptr(X, ldx, xrow, u2) + vi * VW);
+                        x3.load(row_ptr(X, ldx, xrow, u3) + vi * VW);
+#pragma unroll
+                        for (int t = 0; t < VW; ++t) acc[t] += (x0.v[t] + x1.v[t]) + (x2.v[t] + x3.v[t]);
+                    }
+                }
+                for (; j < n; ++j) {
+                    const int32_t u = __shfl_sync(0xffffffffu, my, j);
+                    if (act) {
+                        VI x;
+                        x.load(row_ptr(X, ldx, xrow, u) + vi * VW);
+#pragma unroll
+                        for (int t = 0; t < VW; ++t) acc[t] += x.v[t];
+                    }
+                }
+            }
+            if (act) {
+                VI self;
+                self.load(row_ptr(X, ldx, xrow, v) + vi * VW);
+#pragma unroll
+                for (int t = 0; t < VW; ++t) {
+                    const int col = vi * VW + t;
+                    if (col < Fi) {
+                        st_act(out + col, self.v[t]);
+                        st_act(out + Fp + col, acc[t] * inv);
+                    }
+                }
+            }
+        }
+        // pad columns of both halves, the ones column (bias), trailing pad
+        for (int col = Fi + lane; col < Fp; col += 32) { st_act(out + col, 0.f); st_act(out + Fp + col, 0.f); }
+        for (int col = 2 * Fp + lane; col < ldxa; col += 32) st_act(out + col, col == 2 * Fp ? 1.f : 0.f);
+    }
+}
+
+// ------------------------------------------------ mean, project-first fwd
+// S[v,c] = Y[v, Fop + c] + (1/D_v) sum_u Y[u, c];  out = logits (fp32) or ReLU -> H (+ones col)
+template <typename Tout>
+__global__ void __launch_bounds__(256) k_agg_mean_pf(const float* __restrict__ Y, int64_t ldy,
+                                                     const int64_t* __restrict__ indptr,
+                                                     const int32_t* __restrict__ idx, const int64_t* cnt, int Fo,
+                                                     int Fop, int relu, Tout* __restrict__ out, int64_t ldo) {
+    const int64_t nd = cnt[0];
+    const int lane = lane_id();
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t v = gw; v < nd; v += nw) {
+        const int64_t b = indptr[v], e = indptr[v + 1];
+        const float inv = e > b ? 1.0f / (float)(e - b) : 0.0f;
+        for (int c0 = 0; c0 < Fo; c0 += 32) {
+            const int c = c0 + lane;
+            const bool act = c < Fo;
+            float acc = 0.f;
+            for (int64_t e0 = b; e0 < e; e0 += 32) {
+                const int n = (int)mn64(32, e - e0);
+                const int32_t my = lane < n ? idx[e0 + lane] : 0;
+                for (int j = 0; j < n; ++j) {
+                    const int32_t u = __shfl_sync(0xffffffffu, my, j);
+                    if (act) acc += Y[(int64_t)u * ldy + c];
+                }
+            }
+            if (act) {
+                float sv = Y[v * ldy + Fop + c] + acc * inv;
+                if (relu) sv = fmaxf(sv, 0.f);
+                st_act(out + v * ldo + c, sv);
+            }
+        }
+        if (relu)
+            for (int col = Fo + lane; col < ldo; col += 32) st_act(out + v * ldo + col, col == Fo ? 1.f : 0.f);
+    }
+}
+
+// ----------------------------------------------- A = [X[xrow] | 1 | 0] rows
+template <typename Tin, typename Tout>
+__global__ void k_gather_ones(const Tin* __restrict__ X, int64_t ldx, const int32_t* __restrict__ xrow,
+                              const int64_t* cnt_rows, int Fi, Tout* __restrict__ out, int64_t ldo) {
+    const int64_t n = cnt_rows[0];
+    const int lane = lane_id();
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t r = gw; r < n; r += nw) {
+        const Tin* x = row_ptr(X, ldx, xrow, r);
+        for (int col = lane; col < ldo; col += 32)
+            st_act(out + r * ldo + col, col < Fi ? ld_act(x + col) : (col == Fi ? 1.f : 0.f));
+    }
+}
+
+// ------------------------------------ mean, aggregate-first bwd (via CSC)
+// dS_prev[u,f] = ( [u < nd] dXA[u, f] + sum_{v in CSC(u)} dXA[v, Fp + f] / D_v ) * [H[u,f] > 0]
+template <typename Tm, typename Tout>
+__global__ void __launch_bounds__(256) k_csc_mean(const float* __restrict__ dXA, int64_t ldd,
+                                                  const int64_t* __restrict__ indptr,
+                                                  const int64_t* __restrict__ t_indptr,
+                                                  const int32_t* __restrict__ t_idx, const int64_t* cnt, int Fi,
+                                                  int Fp, const Tm* __restrict__ H, int64_t ldh,
+                                                  Tout* __restrict__ out, int64_t ldo) {
+    const int64_t nd = cnt[0], ns = cnt[1];
+    const int lane = lane_id();
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t u = gw; u < ns; u += nw) {
+        const int64_t b = t_indptr[u], e = t_indptr[u + 1];
+        for (int c0 = 0; c0 < Fi; c0 += 32) {
+            const int c = c0 + lane;
+            const bool act = c < Fi;
+            float acc = 0.f;
+            for (int64_t e0 = b; e0 < e; e0 += 32) {
+                const int n = (int)mn64(32, e - e0);
+                int32_t my = 0;
+                float myinv = 0.f;
+                if (lane < n) {
+                    my = t_idx[e0 + lane];
+                    myinv = 1.0f / (float)(indptr[my + 1] - indptr[my]);
+                }
+                for (int j = 0; j < n; ++j) {
+                    const int32_t v = __shfl_sync(0xffffffffu, my, j);
+                    const float iv = __shfl_sync(0xffffffffu, myinv, j);
+                    if (act) acc += dXA[(int64_t)v * ldd + Fp + c] * iv;
+                }
+            }
+            if (act) {
+                float g = acc + (u < nd ? dXA[u * ldd + c] : 0.f);
+                if (!(ld_act(H + u * ldh + c) > 0.f)) g = 0.f;
+                st_act(out + u * ldo + c, g);
+            }
+        }
+        for (int col = Fi + lane; col < ldo; col += 32) st_act(out + u * ldo + col, 0.f);
+    }
+}
+
+// --------------------------------------- mean, project-first bwd (via CSC)
+// G[u] = [ sum_{v in CSC(u)} dS[v]/D_v (Fo) | 0 | [u < nd] dS[u] (Fo) | 0 ]
+template <typename Tin, typename Tout>
+__global__ void __launch_bounds__(256) k_csc_pf(const Tin* __restrict__ dS, int64_t ldds,
+                                                const int64_t* __restrict__ indptr,
+                                                const int64_t* __restrict__ t_indptr,
+                                                const int32_t* __restrict__ t_idx, const int64_t* cnt, int Fo,
+                                                int Fop, Tout* __restrict__ G, int64_t ldg) {
+    const int64_t nd = cnt[0], ns = cnt[1];
+    const int lane = lane_id();
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t u = gw; u < ns; u += nw) {
+        const int64_t b = t_indptr[u], e = t_indptr[u + 1];
+        for (int c0 = 0; c0 < Fop; c0 += 32) {
+            const int c = c0 + lane;
+            const bool act = c < Fo;
+            float acc = 0.f;
+            for (int64_t e0 = b; e0 < e; e0 += 32) {
+                const int n = (int)mn64(32, e - e0);
+                int32_t my = 0;
+                float myinv = 0.f;
+                if (lane < n) {
+                    my = t_idx[e0 + lane];
+                    myinv = 1.0f / (float)(indptr[my + 1] - indptr[my]);
+                }
+                for (int j = 0; j < n; ++j) {
+                    const int32_t v = __shfl_sync(0xffffffffu, my, j);
+                    const float iv = __shfl_sync(0xffffffffu, myinv, j);
+                    if (act) acc += ld_act(dS + (int64_t)v * ldds + c) * iv;
+                }
+            }
+            if (c < Fop) {
+                st_act(G + u * ldg + c, act ? acc : 0.f);
+                st_act(G + u * ldg + Fop + c, (act && u < nd) ? ld_act(dS + u * ldds + c) : 0.f);
+            }
+        }
+    }
+}
+
+// ------------------------------------------------------------ pool fwd
+// XA[v] = [ h_v | max_{u in N(v)} ReLU(Zp[u]) | 1 ]; arg[v,f] = first u attaining the max (-1: empty row)
+template <typename Tin, typename Tout>
+__global__ void __launch_bounds__(256) k_agg_pool(const Tin* __restrict__ X, int64_t ldx,
+                                                  const int32_t* __restrict__ xrow, const float* __restrict__ Zp,
+                                                  int64_t ldz, const int64_t* __restrict__ indptr,
+                                                  const int32_t* __restrict__ idx, const int64_t* cnt, int Fi, int Fp,
+                                                  Tout* __restrict__ XA, int64_t ldxa, int32_t* __restrict__ arg,
+                                                  int64_t ldarg) {
+    const int64_t nd = cnt[0];
+    const int lane = lane_id();
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t v = gw; v < nd; v += nw) {
+        const int64_t b = indptr[v], e = indptr[v + 1];
+        const Tin* xv = row_ptr(X, ldx, xrow, v);
+        for (int c0 = 0; c0 < Fi; c0 += 32) {
+            const int c = c0 + lane;
+            const bool act = c < Fi;
+            float best = 0.f;
+            int32_t a = -1;
+            for (int64_t e0 = b; e0 < e; e0 += 32) {
+                const int n = (int)mn64(32, e - e0);
+                const int32_t my = lane < n ? idx[e0 + lane] : 0;
+                for (int j = 0; j < n; ++j) {
+                    const int32_t u = __shfl_sync(0xffffffffu, my, j);
+                    if (act) {
+                        const float z = fmaxf(Zp[(int64_t)u * ldz + c], 0.f);
+                        if (a < 0 || z > best) { best = z; a = u; }
+                    }
+                }
+            }
+            if (act) {
+                st_act(XA + v * ldxa + c, ld_act(xv + c));
+                st_act(XA + v * ldxa + Fp + c, best);
+                arg[v * ldarg + c] = a;
+            }
+        }
+        for (int col = Fi + lane; col < Fp; col += 32) { st_act(XA + v * ldxa + col, 0.f); st_act(XA + v * ldxa + Fp + col, 0.f); }
+        for (int col = 2 * Fp + lane; col < ldxa; col += 32) st_act(XA + v * ldxa + col, col == 2 * Fp ? 1.f : 0.f);
+    }
+}
+
+// ------------------------------------------------------------ pool bwd
+// dZp[u,f] = ( sum_{v in CSC(u), arg[v,f] == u} dXA[v, Fp + f] ) * [Zp[u,f] > 0]
+template <typename Tout>
+__global__ void __launch_bounds__(256) k_route_pool(const float* __restrict__ dXA, int64_t ldd,
+                                                    const int32_t* __restrict__ arg, int64_t ldarg,
+                                                    const int64_t* __restrict__ t_indptr,
+                                                    const int32_t* __restrict__ t_idx, const int64_t* cnt, int Fi,
+                                                    int Fp, const float* __restrict__ Zp, int64_t ldz,
+                                                    Tout* __restrict__ out, int64_t ldo) {
+    const int64_t ns = cnt[1];
+    const int lane = lane_id();
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t u = gw; u < ns; u += nw) {
+        const int64_t b = t_indptr[u], e = t_indptr[u + 1];
+        for (int c0 = 0; c0 < Fi; c0 += 32) {
+            const int c = c0 + lane;
+            const bool act = c < Fi;
+            float acc = 0.f;
+            for (int64_t e0 = b; e0 < e; e0 += 32) {
+                const int n = (int)mn64(32, e - e0);
+                const int32_t my = lane < n ? t_idx[e0 + lane] : 0;
+                for (int j = 0; j < n; ++j) {
+                    const int32_t v = __shfl_sync(0xffffffffu, my, j);
+                    if (act && arg[(int64_t)v * ldarg + c] == (int32_t)u) acc += dXA[(int64_t)v * ldd + Fp + c];
+                }
+            }
+            if (act) st_act(out + u * ldo + c, Zp[u * ldz + c] > 0.f ? acc : 0.f);
+        }
+        for (int col = Fi + lane; col < ldo; col += 32) st_act(out + u * ldo + col, 0.f);
+    }
+}
+
+// ----------------------------------------------------------- launchers
+static inline int warps_grid(betty_ctx* c, int64_t rows_cap) {
+    return (int)std::max<int64_t>(1, std::min<int64_t>((rows_cap * 32 + 255) / 256, (int64_t)c->num_sms * 16));
+}
+
+#define DISPATCH_ACT(bf, T, ...)                              \
+    if (bf) { using T = __nv_bfloat16; __VA_ARGS__; }          \
+    else { using T = float; __VA_ARGS__; }
+
+void agg_mean_xa(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const int32_t* xrow, const int64_t* indptr,
+                 const int32_t* idx, const int64_t* cnt, int64_t rows_cap, int Fi, int Fp, void* XA, bool xa_bf16,
+                 int64_t ldxa, cudaStream_t s) {
+    DISPATCH_ACT(x_bf16, TI, DISPATCH_ACT(xa_bf16, TO,
+        k_agg_mean_xa<TI, TO><<<warps_grid(c, rows_cap), 256, 0, s>>>((const TI*)X, ldx, xrow, indptr, idx, cnt, Fi,
+                                                                      Fp, (TO*)XA, ldxa)));
+}
+
+void agg_mean_pf(betty_ctx* c, const float* Y, int64_t ldy, const int64_t* indptr, const int32_t* idx,
+                 const int64_t* cnt, int64_t rows_cap, int Fo, int Fop, bool relu, void* out, bool out_bf16,
+                 int64_t ldo, cudaStream_t s) {
+    DISPATCH_ACT(out_bf16, TO,
+        k_agg_mean_pf<TO><<<warps_grid(c, rows_cap), 256, 0, s>>>(Y, ldy, indptr, idx, cnt, Fo, Fop, relu ? 1 : 0,
+                                                                  (TO*)out, ldo));
+}
+
+void gather_ones(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const int32_t* xrow, const int64_t* cnt_rows,
+                 int64_t rows_cap, int Fi, void* out, bool out_bf16, int64_t ldo, cudaStream_t s) {
+    DISPATCH_ACT(x_bf16, TI, DISPATCH_ACT(out_bf16, TO,
+        k_gather_ones<TI, TO><<<warps_grid(c, rows_cap), 256, 0, s>>>((const TI*)X, ldx, xrow, cnt_rows, Fi, (TO*)out,
+                                                                      ldo)));
+}
+
+void csc_mean(betty_ctx* c, const float* dXA, int64_t ldd, const int64_t* indptr, const int64_t* t_indptr,
+              const int32_t* t_idx, const int64_t* cnt, int64_t src_cap, int Fi, int Fp, const void* H, bool h_bf16,
+              int64_t ldh, void* out, bool out_bf16, int64_t ldo, cudaStream_t s) {
+    DISPATCH_ACT(h_bf16, TM, DISPATCH_ACT(out_bf16, TO,
+        k_csc_mean<TM, TO><<<warps_grid(c, src_cap), 256, 0, s>>>(dXA, ldd, indptr, t_indptr, t_idx, cnt, Fi, Fp,
+                                                                  (const TM*)H, ldh, (TO*)out, ldo)));
+}
+
+void csc_pf(betty_ctx* c, const void* dS, bool ds_bf16, int64_t ldds, const int64_t* indptr, const int64_t* t_indptr,
+            const int32_t* t_idx, const int64_t* cnt, int64_t src_cap, int Fo, int Fop, void* G, bool g_bf16,
+            int64_t ldg, cudaStream_t s) {
+    DISPATCH_ACT(ds_bf16, TI, DISPATCH_ACT(g_bf16, TO,
+        k_csc_pf<TI, TO><<<warps_grid(c, src_cap), 256, 0, s>>>((const TI*)dS, ldds, indptr, t_indptr, t_idx, cnt, Fo,
+                                                                Fop, (TO*)G, ldg)));
+}
+
+void agg_pool(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const int32_t* xrow, const float* Zp, int64_t ldz,
+              const int64_t* indptr, const int32_t* idx, const int64_t* cnt, int64_t rows_cap, int Fi, int Fp,
+              void* XA, bool xa_bf16, int64_t ldxa, int32_t* arg, int64_t ldarg, cudaStream_t s) {
+    DISPATCH_ACT(x_bf16, TI, DISPATCH_ACT(xa_bf16, TO,
+        k_agg_pool<TI, TO><<<warps_grid(c, rows_cap), 256, 0, s>>>((const TI*)X, ldx, xrow, Zp, ldz, indptr, idx, cnt,
+                                                                   Fi, Fp, (TO*)XA, ldxa, arg, ldarg)));
+}
+
+void route_pool(betty_ctx* c, const float* dXA, int64_t ldd, const int32_t* arg, int64_t ldarg,
+                const int64_t* t_indptr, const int32_t* t_idx, const int64_t* cnt, int64_t src_cap, int Fi, int Fp,
+                const float* Zp, int64_t ldz, void* out, bool out_bf16, int64_t ldo, cudaStream_t s) {
+    DISPATCH_ACT(out_bf16, TO,
+        k_route_pool<TO><<<warps_grid(c, src_cap), 256, 0, s>>>(dXA, ldd, arg, ldarg, t_indptr, t_idx, cnt, Fi, Fp, Zp,
+                                                                ldz, (TO*)out, ldo));
+}
+
+}  // namespace betty

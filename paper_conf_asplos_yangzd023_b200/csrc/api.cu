@@ -1,0 +1,741 @@
+// api.cu -- the C ABI of include/betty.h: validation, allocation, the
+// standalone entry points, plans and the graph-captured fused step.
+#include <algorithm>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <vector>
+#include "internal.h"
+#include "extract.h"
+#include "model.h"
+#include "reg.h"
+
+using namespace betty;
+
+namespace betty {
+void* ctx_alloc(betty_ctx* c, size_t bytes, cudaStream_t s) {
+    if (bytes == 0) bytes = 16;
+    if (c->alloc) return c->alloc(bytes, (betty_stream)s, c->user);
+    void* p = nullptr;
+    if (cudaMallocAsync(&p, bytes, s) != cudaSuccess) return nullptr;
+    return p;
+}
+void ctx_free(betty_ctx* c, void* p, cudaStream_t s) {
+    if (!p) return;
+    if (c->dealloc) c->dealloc(p, (betty_stream)s, c->user);
+    else cudaFreeAsync(p, s);
+}
+size_t extract_scratch_bytes(int64_t c, int64_t max_full_src, int64_t sel_nchunks);
+}  // namespace betty
+
+static betty_status fail(betty_ctx* c, betty_status st, const char* fmt, ...) {
+    if (c) {
+        char buf[512];
+        va_list ap;
+        va_start(ap, fmt);
+        vsnprintf(buf, sizeof buf, fmt, ap);
+        va_end(ap);
+        c->err = buf;
+    }
+    return st;
+}
+
+#define CUDA_OK(ctx, expr)                                                                   \
+    do {                                                                                     \
+        cudaError_t _e = (expr);                                                             \
+        if (_e != cudaSuccess) return fail(ctx, BETTY_ECUDA, "%s: %s", #expr, cudaGetErrorString(_e)); \
+    } while (0)
+
+static betty_status check_launch(betty_ctx* c) {
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return fail(c, BETTY_ECUDA, "kernel launch: %s", cudaGetErrorString(e));
+    return BETTY_OK;
+}
+
+// synchronise and translate device-side error flags
+static betty_status sync_check(betty_ctx* c, cudaStream_t s) {
+    CUDA_OK(c, cudaStreamSynchronize(s));
+    int flags = 0;
+    CUDA_OK(c, cudaMemcpy(&flags, c->dev_err, sizeof(int), cudaMemcpyDeviceToHost));
+    if (flags) {
+        CUDA_OK(c, cudaMemset(c->dev_err, 0, sizeof(int)));
+        if (flags & DEVERR_BAD_PART) return fail(c, BETTY_EINVAL, "part[] has a value outside [0, K)");
+        if (flags & DEVERR_DUP_EDGE) return fail(c, BETTY_EINVAL, "a row repeats a source (A must be binary)");
+        if (flags & DEVERR_OVERFLOW) return fail(c, BETTY_EOVERFLOW, "a size exceeded a capacity / kernel limit");
+    }
+    return check_launch(c);
+}
+
+// ----------------------------------------------------------------- ctx
+extern "C" const char* betty_version(void) { return "betty-b200 0.1 (sm_100a)"; }
+
+extern "C" betty_status betty_ctx_create(int device, betty_alloc_fn alloc, betty_free_fn dealloc, void* user,
+                                         betty_ctx** out) {
+    if (!out) return BETTY_EINVAL;
+    *out = nullptr;
+    if ((alloc == nullptr) != (dealloc == nullptr)) return BETTY_EINVAL;
+    if (cudaSetDevice(device) != cudaSuccess) return BETTY_ECUDA;
+    betty_ctx* c = new (std::nothrow) betty_ctx();
+    if (!c) return BETTY_ENOMEM;
+    c->device = device;
+    c->alloc = alloc;
+    c->dealloc = dealloc;
+    c->user = user;
+    cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, device);
+    // counters [64 unsigned] + loss partials [512 double] ; device error flags ; big-segment list
+    if (cudaMalloc(&c->counters, 64 * 4 + 512 * 8) != cudaSuccess || cudaMalloc(&c->dev_err, 16) != cudaSuccess ||
+        cudaMalloc(&c->big_count, 16) != cudaSuccess) {
+        delete c;
+        return BETTY_ENOMEM;
+    }
+    c->big_list_cap = 1 << 20;
+    if (cudaMalloc(&c->big_list, sizeof(int64_t) * c->big_list_cap) != cudaSuccess) { delete c; return BETTY_ENOMEM; }
+    cudaMemset(c->counters, 0, 64 * 4 + 512 * 8);
+    init_kernel_attrs();
+    cudaMemset(c->dev_err, 0, 16);
+    cudaMemset(c->big_count, 0, 16);
+    cudaDeviceSynchronize();
+    *out = c;
+    return BETTY_OK;
+}
+
+extern "C" void betty_ctx_destroy(betty_ctx* c) {
+    if (!c) return;
+    cudaDeviceSynchronize();
+    if (c->scan_status) ctx_free(c, c->scan_status, 0);
+    cudaFree(c->counters);
+    cudaFree(c->dev_err);
+    cudaFree(c->big_count);
+    cudaFree(c->big_list);
+    cudaDeviceSynchronize();
+    delete c;
+}
+
+extern "C" const char* betty_last_error(const betty_ctx* c) { return c ? c->err.c_str() : "null ctx"; }
+
+extern "C" int64_t betty_num_params(const betty_model* m) {
+    ModelCfg cfg;
+    if (!m || !make_model_cfg(m->L, m->aggr, m->gemm, m->feat_dtype, m->dims, &cfg)) return -1;
+    return cfg.n_params;
+}
+
+// ------------------------------------------------------------ extraction
+struct Arena {
+    betty_ctx* c;
+    cudaStream_t s;
+    std::vector<void*> owned;
+    int64_t bytes = 0;
+    bool ok = true;
+    template <typename T> T* get(int64_t n) {
+        const int64_t b = std::max<int64_t>(n, 1) * (int64_t)sizeof(T);
+        void* p = ctx_alloc(c, (size_t)b, s);
+        if (!p) ok = false; else { owned.push_back(p); bytes += b; }
+        return (T*)p;
+    }
+    void release() { for (void* p : owned) ctx_free(c, p, s); owned.clear(); }
+};
+
+struct ExtractSet {             // arenas of one extraction configuration (c slots, given capacities)
+    std::vector<ExtractLayer> layers;
+    ExtractScratch sc{};
+    int64_t* cnt_all = nullptr; // [L*4]
+};
+
+static bool alloc_extract(Arena& A, int L, const ExtractFull* full, int64_t n_out, int32_t c,
+                          const std::vector<int64_t>& cap_dst, const std::vector<int64_t>& cap_src,
+                          const std::vector<int64_t>& cap_e, uint32_t csc_mask, ExtractSet* X) {
+    X->layers.assign(L, ExtractLayer{});
+    X->cnt_all = A.get<int64_t>(L * 4);
+    int64_t max_src = 1, max_dst = 1;
+    for (int l = 0; l < L; ++l) {
+        ExtractLayer& B = X->layers[l];
+        B.cap_dst = std::max<int64_t>(cap_dst[l], 1);
+        B.cap_src = std::max<int64_t>(cap_src[l], 1);
+        B.cap_e = std::max<int64_t>(cap_e[l], 1);
+        B.indptr = A.get<int64_t>(B.cap_dst + 1);
+        B.indices = A.get<int32_t>(B.cap_e);
+        B.src_pos = A.get<int32_t>(B.cap_src);
+        B.src_gid = A.get<int32_t>(B.cap_src);
+        B.src_mb = A.get<int32_t>(B.cap_src);
+        if (csc_mask >> l & 1) {
+            B.t_indptr = A.get<int64_t>(B.cap_src + 1);
+            B.t_indices = A.get<int32_t>(B.cap_e);
+        }
+        B.cnt = X->cnt_all + 4 * l;
+        B.mb_src_off = A.get<int64_t>(c + 1);
+        max_src = std::max(max_src, std::max(full[l].n_src, B.cap_src));
+        max_dst = std::max(max_dst, B.cap_dst);
+    }
+    int64_t max_full = 1;
+    for (int l = 0; l < L; ++l) max_full = std::max(max_full, full[l].n_src);
+    const int64_t W = (max_full + 31) / 32 + 1;
+    const int64_t nchunks = (n_out + 1023) / 1024 + 1;
+    ExtractScratch& sc = X->sc;
+    sc.dstbits = A.get<uint32_t>(c * W);
+    sc.newbits = A.get<uint32_t>(c * W);
+    sc.map = A.get<int32_t>(c * max_full);
+    sc.map_stride = max_full;
+    sc.wordcnt = A.get<int32_t>(c * W);
+    sc.wordoff = A.get<int64_t>(c * W + 1);
+    sc.deg = A.get<int64_t>(max_dst);
+    sc.tcnt = A.get<int32_t>(max_src);
+    sc.sel_cnt = A.get<int32_t>(c * nchunks);
+    sc.sel_off = A.get<int64_t>(c * nchunks + 1);
+    sc.top_dst_pos = A.get<int32_t>(std::max<int64_t>(n_out, 1));
+    sc.top_row_mb = A.get<int32_t>(std::max<int64_t>(n_out, 1));
+    sc.top_dst_off = A.get<int64_t>(c + 1);
+    if (!A.ok) return false;
+    cudaMemsetAsync(sc.dstbits, 0, sizeof(uint32_t) * c * W, A.s);
+    cudaMemsetAsync(sc.newbits, 0, sizeof(uint32_t) * c * W, A.s);
+    cudaMemsetAsync(X->cnt_all, 0, sizeof(int64_t) * L * 4, A.s);
+    return true;
+}
+
+static betty_status check_full(betty_ctx* c, const betty_block* full, int32_t L) {
+    if (!full || L < 1 || L > 16) return fail(c, BETTY_EINVAL, "full blocks / L invalid");
+    for (int l = 0; l < L; ++l) {
+        const betty_block& b = full[l];
+        if (!b.indptr || (b.n_edges > 0 && !b.indices) || (b.n_src > 0 && !b.src_gid))
+            return fail(c, BETTY_EINVAL, "full block %d: null array", l);
+        if (b.n_dst < 0 || b.n_src < b.n_dst || b.n_edges < 0)
+            return fail(c, BETTY_EINVAL, "full block %d: bad sizes", l);
+        if (b.n_src >= INT32_MAX || b.n_edges >= ((int64_t)1 << 40))
+            return fail(c, BETTY_EOVERFLOW, "full block %d: sizes exceed int32 ids", l);
+        if (l + 1 < L && full[l + 1].n_src != b.n_dst)
+            return fail(c, BETTY_EINVAL, "block %d dst count must equal block %d src count", l, l + 1);
+    }
+    return BETTY_OK;
+}
+
+static std::vector<ExtractFull> to_full(const betty_block* full, int L) {
+    std::vector<ExtractFull> f(L);
+    for (int l = 0; l < L; ++l) f[l] = ExtractFull{full[l].n_dst, full[l].n_src, full[l].n_edges, full[l].indptr,
+                                                   full[l].indices, full[l].src_gid};
+    return f;
+}
+
+extern "C" betty_status betty_extract_blocks(betty_ctx* c, const betty_block* full, int32_t L, const int32_t* part,
+                                             int64_t n_out, int32_t K, int32_t k, betty_block* mb,
+                                             betty_stream stream) {
+    if (!c) return BETTY_EINVAL;
+    cudaStream_t s = (cudaStream_t)stream;
+    betty_status st = check_full(c, full, L);
+    if (st) return st;
+    if (!mb || (n_out > 0 && !part) || K < 1 || k < 0 || k >= K || full[L - 1].n_dst != n_out)
+        return fail(c, BETTY_EINVAL, "extract: bad part / K / k / n_out");
+    std::vector<ExtractFull> F = to_full(full, L);
+    std::vector<int64_t> cd(L), cs(L), ce(L);
+    for (int l = 0; l < L; ++l) { cd[l] = full[l].n_dst; cs[l] = full[l].n_src; ce[l] = full[l].n_edges; }
+    Arena A{c, s};
+    ExtractSet X;
+    int32_t* d_k = A.get<int32_t>(1);
+    if (!d_k || !alloc_extract(A, L, F.data(), n_out, 1, cd, cs, ce, (1u << L) - 1, &X)) {
+        A.release();
+        return fail(c, BETTY_ENOMEM, "extract: allocation failed");
+    }
+    cudaMemcpyAsync(d_k, &k, sizeof(int32_t), cudaMemcpyHostToDevice, s);
+    ExtractArgs a{};
+    a.L = L; a.full = F.data(); a.part = part; a.K = K; a.ks = d_k; a.c = 1;
+    a.layers = X.layers.data(); a.sc = X.sc; a.csc_mask = (1u << L) - 1;
+    extract_group(c, a, s);
+    std::vector<int64_t> cnt(L * 4);
+    cudaMemcpyAsync(cnt.data(), X.cnt_all, sizeof(int64_t) * L * 4, cudaMemcpyDeviceToHost, s);
+    st = sync_check(c, s);
+    if (st) { A.release(); return st; }
+    // exact-size outputs
+    for (int l = 0; l < L; ++l) {
+        betty_block& o = mb[l];
+        memset(&o, 0, sizeof(o));
+        o.n_dst = cnt[4 * l + 0]; o.n_src = cnt[4 * l + 1]; o.n_edges = cnt[4 * l + 2];
+        o.indptr = (int64_t*)ctx_alloc(c, sizeof(int64_t) * (o.n_dst + 1), s);
+        o.indices = (int32_t*)ctx_alloc(c, sizeof(int32_t) * std::max<int64_t>(o.n_edges, 1), s);
+        o.src_pos = (int32_t*)ctx_alloc(c, sizeof(int32_t) * std::max<int64_t>(o.n_src, 1), s);
+        o.src_gid = (int32_t*)ctx_alloc(c, sizeof(int32_t) * std::max<int64_t>(o.n_src, 1), s);
+        o.t_indptr = (int64_t*)ctx_alloc(c, sizeof(int64_t) * (o.n_src + 1), s);
+        o.t_indices = (int32_t*)ctx_alloc(c, sizeof(int32_t) * std::max<int64_t>(o.n_edges, 1), s);
+        if (!o.indptr || !o.indices || !o.src_pos || !o.src_gid || !o.t_indptr || !o.t_indices) {
+            betty_block_free(c, mb, l + 1);
+            A.release();
+            return fail(c, BETTY_ENOMEM, "extract: output allocation failed");
+        }
+        const ExtractLayer& B = X.layers[l];
+        cudaMemcpyAsync(o.indptr, B.indptr, sizeof(int64_t) * (o.n_dst + 1), cudaMemcpyDeviceToDevice, s);
+        cudaMemcpyAsync(o.indices, B.indices, sizeof(int32_t) * o.n_edges, cudaMemcpyDeviceToDevice, s);
+        cudaMemcpyAsync(o.src_pos, B.src_pos, sizeof(int32_t) * o.n_src, cudaMemcpyDeviceToDevice, s);
+        cudaMemcpyAsync(o.src_gid, B.src_gid, sizeof(int32_t) * o.n_src, cudaMemcpyDeviceToDevice, s);
+        cudaMemcpyAsync(o.t_indptr, B.t_indptr, sizeof(int64_t) * (o.n_src + 1), cudaMemcpyDeviceToDevice, s);
+        cudaMemcpyAsync(o.t_indices, B.t_indices, sizeof(int32_t) * o.n_edges, cudaMemcpyDeviceToDevice, s);
+    }
+    A.release();
+    return sync_check(c, s);
+}
+
+extern "C" void betty_block_free(betty_ctx* c, betty_block* b, int32_t L) {
+    if (!c || !b) return;
+    for (int l = 0; l < L; ++l) {
+        ctx_free(c, b[l].indptr, 0); ctx_free(c, b[l].indices, 0); ctx_free(c, b[l].src_pos, 0);
+        ctx_free(c, b[l].src_gid, 0); ctx_free(c, b[l].t_indptr, 0); ctx_free(c, b[l].t_indices, 0);
+        memset(&b[l], 0, sizeof(betty_block));
+    }
+}
+
+// ------------------------------------------------------------------ REG
+struct RegBufs {
+    RegArgs a{};
+    int64_t* cnt = nullptr;     // [3] n_rows, n_cols, n_edges
+    int32_t* col = nullptr;
+    int32_t* w = nullptr;
+    int64_t ub_cap = 0, nnz_cap = 0;
+};
+
+static bool alloc_reg_phase1(Arena& A, const betty_block* ob, RegBufs* R) {
+    const int64_t n = ob->n_dst, ns = ob->n_src, E = ob->n_edges;
+    R->cnt = A.get<int64_t>(4);
+    RegArgs& a = R->a;
+    a.indptr = ob->indptr; a.idx = ob->indices;
+    a.n_rows_dev = R->cnt; a.n_cols_dev = R->cnt + 1; a.n_edges_dev = R->cnt + 2;
+    a.rows_cap = std::max<int64_t>(n, 1); a.cols_cap = std::max<int64_t>(ns, 1); a.edges_cap = std::max<int64_t>(E, 1);
+    a.t_indptr = A.get<int64_t>(ns + 1);
+    a.t_idx = A.get<int32_t>(E);
+    a.tcnt = A.get<int32_t>(ns);
+    a.ub = A.get<int64_t>(n);
+    a.off = A.get<int64_t>(n + 1);
+    a.ub_total_dev = R->cnt + 3;
+    a.row_nnz = A.get<int64_t>(n);
+    return A.ok;
+}
+
+extern "C" betty_status betty_reg_build(betty_ctx* c, const betty_block* ob, betty_csr* reg, betty_stream stream) {
+    if (!c) return BETTY_EINVAL;
+    cudaStream_t s = (cudaStream_t)stream;
+    if (!ob || !reg || !ob->indptr || (ob->n_edges > 0 && !ob->indices) || ob->n_dst < 0)
+        return fail(c, BETTY_EINVAL, "reg: null argument");
+    if (ob->n_src >= INT32_MAX || ob->n_dst >= INT32_MAX) return fail(c, BETTY_EOVERFLOW, "reg: sizes exceed int32");
+    memset(reg, 0, sizeof(*reg));
+    Arena A{c, s};
+    RegBufs R;
+    if (!alloc_reg_phase1(A, ob, &R)) { A.release(); return fail(c, BETTY_ENOMEM, "reg: allocation failed"); }
+    int64_t h[4] = {ob->n_dst, ob->n_src, ob->n_edges, 0};
+    cudaMemcpyAsync(R.cnt, h, sizeof(h), cudaMemcpyHostToDevice, s);
+    reg_phase1(c, R.a, s);
+    int64_t ub_total = 0;
+    cudaMemcpyAsync(&ub_total, R.a.ub_total_dev, sizeof(int64_t), cudaMemcpyDeviceToHost, s);
+    betty_status st = sync_check(c, s);
+    if (st) { A.release(); return st; }
+    R.a.tcol = A.get<int32_t>(ub_total);
+    R.a.tw = A.get<int32_t>(ub_total);
+    reg->indptr = (int64_t*)ctx_alloc(c, sizeof(int64_t) * (ob->n_dst + 1), s);
+    R.a.out_indptr = reg->indptr;
+    int64_t* nnz_dev = A.get<int64_t>(1);
+    R.a.nnz_total_dev = nnz_dev;
+    if (!A.ok || !reg->indptr) { A.release(); ctx_free(c, reg->indptr, s); reg->indptr = nullptr;
+                                 return fail(c, BETTY_ENOMEM, "reg: allocation failed"); }
+    reg_phase2(c, R.a, s);
+    int64_t nnz = 0;
+    cudaMemcpyAsync(&nnz, nnz_dev, sizeof(int64_t), cudaMemcpyDeviceToHost, s);
+    st = sync_check(c, s);
+    if (st) { A.release(); ctx_free(c, reg->indptr, s); reg->indptr = nullptr;
+              return st == BETTY_EOVERFLOW ? fail(c, BETTY_EUNSUPPORTED, "reg: a row has more than 32768 candidate products") : st; }
+    reg->col = (int32_t*)ctx_alloc(c, sizeof(int32_t) * std::max<int64_t>(nnz, 1), s);
+    reg->w = (int32_t*)ctx_alloc(c, sizeof(int32_t) * std::max<int64_t>(nnz, 1), s);
+    if (!reg->col || !reg->w) { A.release(); betty_csr_free(c, reg); return fail(c, BETTY_ENOMEM, "reg: allocation failed"); }
+    reg_phase3(c, R.a, reg->col, reg->w, nnz, s);
+    reg->n = ob->n_dst;
+    reg->nnz = nnz;
+    A.release();
+    return sync_check(c, s);
+}
+
+extern "C" void betty_csr_free(betty_ctx* c, betty_csr* r) {
+    if (!c || !r) return;
+    ctx_free(c, r->indptr, 0); ctx_free(c, r->col, 0); ctx_free(c, r->w, 0);
+    memset(r, 0, sizeof(*r));
+}
+
+// ---------------------------------------------------- standalone SAGE
+struct betty_saved {
+    ModelCfg m;
+    SageBufs b;
+    std::vector<BlockView> v;
+    int64_t* cnt = nullptr;
+    std::vector<int64_t> hcnt;
+};
+
+static betty_status model_from(betty_ctx* c, const betty_model* model, ModelCfg* m) {
+    if (!model || !make_model_cfg(model->L, model->aggr, model->gemm, model->feat_dtype, model->dims, m))
+        return fail(c, BETTY_EINVAL, "invalid betty_model (L in [1,16], dims >= 1, classes <= 256)");
+    return BETTY_OK;
+}
+
+static betty_status check_feats(betty_ctx* c, const ModelCfg& m, const void* feats, int64_t ld) {
+    const int vw = m.feat_bf16 ? 8 : 4;
+    if (!feats) return fail(c, BETTY_EINVAL, "feats is null");
+    if (ld < (m.dims[0] + vw - 1) / vw * vw || ld % vw)
+        return fail(c, BETTY_EINVAL, "ld_feats must be >= dims[0] rounded up to and a multiple of %d", vw);
+    if (((uintptr_t)feats) % 16) return fail(c, BETTY_EINVAL, "feats must be 16-byte aligned");
+    return BETTY_OK;
+}
+
+extern "C" betty_status betty_sage_fwd(betty_ctx* c, const betty_model* model, const float* params,
+                                       const betty_block* mb, const void* feats, int64_t ld_feats,
+                                       betty_saved** saved, float* logits, betty_stream stream) {
+    if (!c) return BETTY_EINVAL;
+    cudaStream_t s = (cudaStream_t)stream;
+    ModelCfg m;
+    betty_status st = model_from(c, model, &m);
+    if (st) return st;
+    if (!params || !mb || !saved) return fail(c, BETTY_EINVAL, "sage_fwd: null argument");
+    if ((st = check_feats(c, m, feats, ld_feats))) return st;
+    for (int l = 0; l < m.L; ++l) {
+        if (!mb[l].indptr || (mb[l].n_edges && !mb[l].indices) || !mb[l].src_gid)
+            return fail(c, BETTY_EINVAL, "sage_fwd: block %d has null arrays", l);
+        if (m.needs_csc(l) && (!mb[l].t_indptr || (mb[l].n_edges && !mb[l].t_indices)))
+            return fail(c, BETTY_EINVAL, "sage_fwd: block %d needs its CSC", l);
+        if (l + 1 < m.L && mb[l + 1].n_src != mb[l].n_dst)
+            return fail(c, BETTY_EINVAL, "sage_fwd: block %d dst count != block %d src count", l, l + 1);
+    }
+    betty_saved* sv = new (std::nothrow) betty_saved();
+    if (!sv) return BETTY_ENOMEM;
+    sv->m = m;
+    sv->hcnt.assign(4 * m.L, 0);
+    std::vector<int64_t> cd(m.L), cs(m.L);
+    for (int l = 0; l < m.L; ++l) {
+        sv->hcnt[4 * l] = mb[l].n_dst; sv->hcnt[4 * l + 1] = mb[l].n_src; sv->hcnt[4 * l + 2] = mb[l].n_edges;
+        cd[l] = mb[l].n_dst; cs[l] = mb[l].n_src;
+    }
+    sv->cnt = (int64_t*)ctx_alloc(c, sizeof(int64_t) * 4 * m.L, s);
+    if (!sv->cnt || !sage_alloc(c, m, cd, cs, &sv->b, s)) {
+        betty_saved_free(c, sv);
+        return fail(c, BETTY_ENOMEM, "sage_fwd: allocation failed");
+    }
+    cudaMemcpyAsync(sv->cnt, sv->hcnt.data(), sizeof(int64_t) * 4 * m.L, cudaMemcpyHostToDevice, s);
+    sv->v.resize(m.L);
+    for (int l = 0; l < m.L; ++l)
+        sv->v[l] = BlockView{mb[l].indptr, mb[l].indices, mb[l].t_indptr, mb[l].t_indices, mb[l].src_gid,
+                             sv->cnt + 4 * l, std::max<int64_t>(mb[l].n_dst, 1), std::max<int64_t>(mb[l].n_src, 1),
+                             std::max<int64_t>(mb[l].n_edges, 1)};
+    sage_prep(c, m, sv->b, params, s);
+    sage_forward(c, m, sv->b, sv->v.data(), feats, ld_feats, s);
+    if (logits && mb[m.L - 1].n_dst > 0)
+        cudaMemcpy2DAsync(logits, sizeof(float) * m.dims[m.L], sv->b.logits, sizeof(float) * m.layers[m.L - 1].ld_out,
+                          sizeof(float) * m.dims[m.L], mb[m.L - 1].n_dst, cudaMemcpyDeviceToDevice, s);
+    if ((st = check_launch(c))) { betty_saved_free(c, sv); return st; }
+    *saved = sv;
+    return BETTY_OK;
+}
+
+extern "C" betty_status betty_sage_bwd(betty_ctx* c, const betty_model* model, const float* params,
+                                       const betty_block* mb, const betty_saved* saved, const int32_t* labels,
+                                       float loss_scale, float* grad_accum, float* loss_accum, betty_stream stream) {
+    if (!c) return BETTY_EINVAL;
+    cudaStream_t s = (cudaStream_t)stream;
+    if (!saved || !params || !labels || !grad_accum || !loss_accum || !mb)
+        return fail(c, BETTY_EINVAL, "sage_bwd: null argument");
+    ModelCfg m;
+    betty_status st = model_from(c, model, &m);
+    if (st) return st;
+    if (m.n_params != saved->m.n_params || m.L != saved->m.L) return fail(c, BETTY_EINVAL, "sage_bwd: model mismatch");
+    betty_saved* sv = const_cast<betty_saved*>(saved);
+    sage_prep(c, sv->m, sv->b, params, s);
+    sage_loss(c, sv->m, sv->b, sv->v.data(), labels, loss_scale, loss_accum, s);
+    sage_backward(c, sv->m, sv->b, sv->v.data(), nullptr, 0, grad_accum, s);
+    return check_launch(c);
+}
+
+extern "C" void betty_saved_free(betty_ctx* c, betty_saved* sv) {
+    if (!c || !sv) return;
+    sage_free(c, &sv->b, 0);
+    ctx_free(c, sv->cnt, 0);
+    delete sv;
+}
+
+// ------------------------------------------------------------- plan / step
+struct betty_plan {
+    ModelCfg m;
+    int L = 0;
+    int32_t K = 0, c = 1;
+    int flags = 0;
+    int64_t n_out = 0;
+    const int32_t* part = nullptr;
+    std::vector<ExtractFull> full;
+    std::vector<std::vector<int32_t>> groups;
+    int32_t* d_ks = nullptr;
+    Arena* arena = nullptr;
+    ExtractSet X;
+    uint32_t csc_mask = 0;
+    SageBufs sb;
+    std::vector<BlockView> views;
+    // REG inside the step
+    bool with_reg = false;
+    RegBufs R;
+    const betty_block* reg_src = nullptr;
+    betty_block reg_block{};
+    // graph
+    cudaGraphExec_t gexec = nullptr;
+    const void* key[9] = {};
+    betty_plan_info info{};
+    Probe probe;
+};
+
+static void step_body(betty_ctx* c, betty_plan* p, const float* params, const void* feats, int64_t ld_feats,
+                      const int32_t* labels, float scale, float* grad, float* loss, cudaStream_t s) {
+    Probe* pr = p->sb.probe;
+    if (pr) pr->used = 0;
+    sage_prep(c, p->m, p->sb, params, s);
+    for (size_t g = 0; g < p->groups.size(); ++g) {
+        ExtractArgs a{};
+        a.L = p->L; a.full = p->full.data(); a.part = p->part; a.K = p->K;
+        a.ks = p->d_ks + g * p->c; a.c = (int32_t)p->groups[g].size();
+        a.layers = p->X.layers.data(); a.sc = p->X.sc; a.csc_mask = p->csc_mask;
+        if (pr) pr->begin(PROBE_EXTRACT, s);
+        extract_group(c, a, s);
+        if (pr) pr->end(PROBE_EXTRACT, s);
+        sage_forward(c, p->m, p->sb, p->views.data(), feats, ld_feats, s);
+        sage_loss(c, p->m, p->sb, p->views.data(), labels, scale, loss, s);
+        sage_backward(c, p->m, p->sb, p->views.data(), feats, ld_feats, grad, s);
+    }
+    if (p->with_reg) {
+        if (pr) pr->begin(PROBE_REG, s);
+        reg_phase1(c, p->R.a, s);
+        reg_phase2(c, p->R.a, s);
+        reg_phase3(c, p->R.a, p->R.col, p->R.w, p->R.nnz_cap, s);
+        if (pr) pr->end(PROBE_REG, s);
+    }
+}
+
+extern "C" betty_status betty_plan_create(betty_ctx* c, const betty_model* model, const betty_block* full, int32_t L,
+                                          const int32_t* part, int64_t n_out, int32_t K, const int32_t* my_k,
+                                          int32_t n_my, int32_t group, int32_t flags, betty_plan** out,
+                                          betty_stream stream) {
+    if (!c) return BETTY_EINVAL;
+    cudaStream_t s = (cudaStream_t)stream;
+    if (!out) return fail(c, BETTY_EINVAL, "plan: out is null");
+    *out = nullptr;
+    ModelCfg m;
+    betty_status st = model_from(c, model, &m);
+    if (st) return st;
+    if ((st = check_full(c, full, L))) return st;
+    if (L != m.L) return fail(c, BETTY_EINVAL, "plan: L != model.L");
+    if (K < 1 || n_my < 0 || (n_my > 0 && !my_k) || full[L - 1].n_dst != n_out || (n_out > 0 && !part))
+        return fail(c, BETTY_EINVAL, "plan: bad K / my_k / n_out / part");
+    for (int i = 0; i < n_my; ++i)
+        if (my_k[i] < 0 || my_k[i] >= K) return fail(c, BETTY_EINVAL, "plan: my_k[%d] out of range", i);
+    betty_plan* p = new (std::nothrow) betty_plan();
+    if (!p) return BETTY_ENOMEM;
+    p->m = m; p->L = L; p->K = K; p->flags = flags; p->n_out = n_out; p->part = part;
+    p->full = to_full(full, L);
+    p->c = group <= 0 ? std::max(1, n_my) : std::min(group, std::max(1, n_my));
+    for (int i = 0; i < n_my; i += p->c)
+        p->groups.emplace_back(my_k + i, my_k + std::min(n_my, i + p->c));
+    p->csc_mask = 0;
+    for (int l = 0; l < L; ++l) if (m.needs_csc(l)) p->csc_mask |= 1u << l;
+
+    // ---- sizing pass: every micro-batch alone, full-batch capacities
+    std::vector<int64_t> fd(L), fs(L), fe(L);
+    for (int l = 0; l < L; ++l) { fd[l] = full[l].n_dst; fs[l] = full[l].n_src; fe[l] = full[l].n_edges; }
+    std::vector<std::vector<int64_t>> sz(n_my, std::vector<int64_t>(3 * L));
+    {
+        Arena A{c, s};
+        ExtractSet X;
+        int32_t* d_k = A.get<int32_t>(std::max(1, n_my));
+        if (!d_k || !alloc_extract(A, L, p->full.data(), n_out, 1, fd, fs, fe, 0, &X)) {
+            A.release(); delete p;
+            return fail(c, BETTY_ENOMEM, "plan: sizing allocation failed");
+        }
+        if (n_my) cudaMemcpyAsync(d_k, my_k, sizeof(int32_t) * n_my, cudaMemcpyHostToDevice, s);
+        std::vector<int64_t> h(4 * L);
+        for (int i = 0; i < n_my; ++i) {
+            ExtractArgs a{};
+            a.L = L; a.full = p->full.data(); a.part = part; a.K = K; a.ks = d_k + i; a.c = 1;
+            a.layers = X.layers.data(); a.sc = X.sc; a.csc_mask = 0;
+            extract_group(c, a, s);
+            cudaMemcpyAsync(h.data(), X.cnt_all, sizeof(int64_t) * 4 * L, cudaMemcpyDeviceToHost, s);
+            if ((st = sync_check(c, s))) { A.release(); delete p; return st; }
+            for (int l = 0; l < L; ++l)
+                for (int q = 0; q < 3; ++q) sz[i][3 * l + q] = h[4 * l + q];
+        }
+        A.release();
+    }
+    std::vector<int64_t> cd(L, 1), cs(L, 1), ce(L, 1);
+    p->info.L = L;
+    p->info.n_groups = (int32_t)p->groups.size();
+    for (size_t g = 0, i0 = 0; g < p->groups.size(); i0 += p->groups[g].size(), ++g) {
+        std::vector<int64_t> sum(3 * L, 0);
+        for (size_t t = 0; t < p->groups[g].size(); ++t)
+            for (int q = 0; q < 3 * L; ++q) sum[q] += sz[i0 + t][q];
+        for (int l = 0; l < L; ++l) {
+            cd[l] = std::max(cd[l], sum[3 * l]); cs[l] = std::max(cs[l], sum[3 * l + 1]);
+            ce[l] = std::max(ce[l], sum[3 * l + 2]);
+            if (l < 16) {
+                p->info.n_dst[l] += sum[3 * l]; p->info.n_src[l] += sum[3 * l + 1]; p->info.edges[l] += sum[3 * l + 2];
+                p->info.max_group_edges[l] = ce[l];
+            }
+        }
+    }
+    for (int l = 0; l < L; ++l)
+        if (cs[l] >= INT32_MAX) { delete p; return fail(c, BETTY_EOVERFLOW, "plan: group exceeds int32 ids"); }
+    for (int l = 0; l + 1 < L; ++l) { cd[l] = std::max(cd[l], cs[l + 1]); cs[l + 1] = cd[l]; }
+
+    // ---- arenas
+    p->arena = new Arena{c, s};
+    Arena& A = *p->arena;
+    p->d_ks = A.get<int32_t>(std::max<int64_t>(1, (int64_t)p->groups.size() * p->c));
+    if (!p->d_ks || !alloc_extract(A, L, p->full.data(), n_out, p->c, cd, cs, ce, p->csc_mask, &p->X) ||
+        !sage_alloc(c, m, cd, cs, &p->sb, s)) {
+        betty_plan_destroy(c, p);
+        return fail(c, BETTY_ENOMEM, "plan: arena allocation failed");
+    }
+    std::vector<int32_t> hk((size_t)p->groups.size() * p->c, 0);
+    for (size_t g = 0; g < p->groups.size(); ++g)
+        for (size_t t = 0; t < p->groups[g].size(); ++t) hk[g * p->c + t] = p->groups[g][t];
+    if (!hk.empty()) cudaMemcpyAsync(p->d_ks, hk.data(), sizeof(int32_t) * hk.size(), cudaMemcpyHostToDevice, s);
+    p->views.resize(L);
+    for (int l = 0; l < L; ++l) {
+        const ExtractLayer& B = p->X.layers[l];
+        p->views[l] = BlockView{B.indptr, B.indices, B.t_indptr, B.t_indices, B.src_gid, B.cnt, B.cap_dst, B.cap_src,
+                                B.cap_e};
+    }
+    // scan scratch for the largest scan of a step (never grows inside a capture)
+    {
+        int64_t mx = 0;
+        for (int l = 0; l < L; ++l) mx = std::max({mx, cd[l], cs[l], ce[l]});
+        int64_t maxfull = 1;
+        for (int l = 0; l < L; ++l) maxfull = std::max(maxfull, full[l].n_src);
+        mx = std::max(mx, (int64_t)p->c * ((maxfull + 31) / 32 + 1));
+        mx = std::max(mx, (int64_t)p->c * ((n_out + 1023) / 1024 + 1));
+        ensure_scan_scratch(c, mx, s);
+    }
+    // ---- REG inside the step (once here to size its buffers)
+    if (flags & BETTY_PLAN_REG) {
+        p->with_reg = true;
+        const betty_block* ob = &full[L - 1];
+        if (!alloc_reg_phase1(A, ob, &p->R)) { betty_plan_destroy(c, p); return fail(c, BETTY_ENOMEM, "plan: REG alloc"); }
+        int64_t h[4] = {ob->n_dst, ob->n_src, ob->n_edges, 0};
+        cudaMemcpyAsync(p->R.cnt, h, sizeof(h), cudaMemcpyHostToDevice, s);
+        reg_phase1(c, p->R.a, s);
+        int64_t ub = 0;
+        cudaMemcpyAsync(&ub, p->R.a.ub_total_dev, sizeof(int64_t), cudaMemcpyDeviceToHost, s);
+        if ((st = sync_check(c, s))) { betty_plan_destroy(c, p); return st; }
+        p->R.ub_cap = ub;
+        p->R.a.tcol = A.get<int32_t>(ub);
+        p->R.a.tw = A.get<int32_t>(ub);
+        p->R.a.out_indptr = A.get<int64_t>(ob->n_dst + 1);
+        p->R.a.nnz_total_dev = A.get<int64_t>(1);
+        if (!A.ok) { betty_plan_destroy(c, p); return fail(c, BETTY_ENOMEM, "plan: REG alloc"); }
+        reg_phase2(c, p->R.a, s);
+        int64_t nnz = 0;
+        cudaMemcpyAsync(&nnz, p->R.a.nnz_total_dev, sizeof(int64_t), cudaMemcpyDeviceToHost, s);
+        if ((st = sync_check(c, s))) { betty_plan_destroy(c, p); return st; }
+        p->R.nnz_cap = nnz;
+        p->R.col = A.get<int32_t>(nnz);
+        p->R.w = A.get<int32_t>(nnz);
+        if (!A.ok) { betty_plan_destroy(c, p); return fail(c, BETTY_ENOMEM, "plan: REG alloc"); }
+        p->info.reg_nnz = nnz;
+    }
+    // ---- launches per step: capture the body once into a throw-away graph
+    {
+        cudaStream_t cs2;
+        cudaStreamCreateWithFlags(&cs2, cudaStreamNonBlocking);
+        cudaGraph_t gr;
+        if (cudaStreamBeginCapture(cs2, cudaStreamCaptureModeThreadLocal) == cudaSuccess) {
+            float* dummy = (float*)p->sb.partials;
+            step_body(c, p, dummy, dummy, m.feat_bf16 ? 8 : 4, (const int32_t*)dummy, 1.f, dummy, dummy, cs2);
+            if (cudaStreamEndCapture(cs2, &gr) == cudaSuccess) {
+                size_t n = 0;
+                cudaGraphGetNodes(gr, nullptr, &n);
+                p->info.kernels_per_step = (int32_t)n;
+                cudaGraphDestroy(gr);
+            }
+        }
+        cudaGetLastError();
+        cudaStreamDestroy(cs2);
+    }
+    p->info.arena_bytes = A.bytes + p->sb.bytes;
+    if ((st = sync_check(c, s))) { betty_plan_destroy(c, p); return st; }
+    *out = p;
+    return BETTY_OK;
+}
+
+extern "C" betty_status betty_plan_info_get(const betty_plan* p, betty_plan_info* info) {
+    if (!p || !info) return BETTY_EINVAL;
+    *info = p->info;
+    return BETTY_OK;
+}
+
+extern "C" void betty_plan_destroy(betty_ctx* c, betty_plan* p) {
+    if (!c || !p) return;
+    cudaDeviceSynchronize();
+    if (p->gexec) cudaGraphExecDestroy(p->gexec);
+    p->probe.destroy();
+    sage_free(c, &p->sb, 0);
+    if (p->arena) { p->arena->s = 0; p->arena->release(); delete p->arena; }
+    cudaDeviceSynchronize();
+    delete p;
+}
+
+extern "C" betty_status betty_step(betty_ctx* c, betty_plan* p, const float* params, const void* feats,
+                                   int64_t ld_feats, const int32_t* labels, float loss_scale, float* grad_accum,
+                                   float* loss_accum, betty_stream stream) {
+    if (!c || !p) return BETTY_EINVAL;
+    cudaStream_t s = (cudaStream_t)stream;
+    if (!params || !labels || !grad_accum || !loss_accum) return fail(c, BETTY_EINVAL, "step: null argument");
+    betty_status st = check_feats(c, p->m, feats, ld_feats);
+    if (st) return st;
+    if (!(p->flags & BETTY_PLAN_GRAPH)) {
+        step_body(c, p, params, feats, ld_feats, labels, loss_scale, grad_accum, loss_accum, s);
+        return check_launch(c);
+    }
+    float sc = loss_scale;
+    int32_t scbits;
+    memcpy(&scbits, &sc, 4);
+    const void* key[9] = {params, feats, (const void*)(intptr_t)ld_feats, labels, grad_accum, loss_accum,
+                          (const void*)(intptr_t)scbits, s, (const void*)(intptr_t)p->probe.site};
+    if (!p->gexec || memcmp(key, p->key, sizeof key) != 0) {
+        if (p->gexec) { cudaGraphExecDestroy(p->gexec); p->gexec = nullptr; }
+        cudaGraph_t g;
+        CUDA_OK(c, cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal));
+        step_body(c, p, params, feats, ld_feats, labels, loss_scale, grad_accum, loss_accum, s);
+        CUDA_OK(c, cudaStreamEndCapture(s, &g));
+        cudaError_t e = cudaGraphInstantiate(&p->gexec, g, 0);
+        cudaGraphDestroy(g);
+        if (e != cudaSuccess) return fail(c, BETTY_ECUDA, "graph instantiate: %s", cudaGetErrorString(e));
+        memcpy(p->key, key, sizeof key);
+    }
+    CUDA_OK(c, cudaGraphLaunch(p->gexec, s));
+    return BETTY_OK;
+}
+
+extern "C" betty_status betty_adam(betty_ctx* c, float* params, float* grad, float* m, float* v, int64_t n, int32_t t,
+                                   float lr, float b1, float b2, float eps, int32_t zero_grad, betty_stream stream) {
+    if (!c) return BETTY_EINVAL;
+    if (!params || !grad || !m || !v || n < 0 || t < 1) return fail(c, BETTY_EINVAL, "adam: bad argument");
+    adam(c, params, grad, m, v, n, t, lr, b1, b2, eps, zero_grad != 0, (cudaStream_t)stream);
+    return check_launch(c);
+}
+
+extern "C" betty_status betty_plan_probe(betty_plan* p, int32_t site) {
+    if (!p || site < 0 || site > PROBE_GEMM_FWD_L1) return BETTY_EINVAL;
+    p->probe.site = site;
+    p->probe.used = 0;
+    p->sb.probe = site ? &p->probe : nullptr;
+    return BETTY_OK;
+}
+
+extern "C" betty_status betty_plan_probe_read(betty_plan* p, float* total_ms, int32_t* launches) {
+    if (!p || !total_ms || !launches) return BETTY_EINVAL;
+    *total_ms = 0.f;
+    *launches = p->probe.used;
+    for (int i = 0; i < p->probe.used; ++i) {
+        if (cudaEventSynchronize(p->probe.ev[2 * i + 1]) != cudaSuccess) return BETTY_ECUDA;
+        float ms = 0.f;
+        if (cudaEventElapsedTime(&ms, p->probe.ev[2 * i], p->probe.ev[2 * i + 1]) != cudaSuccess) return BETTY_ECUDA;
+        *total_ms += ms;
+    }
+    return BETTY_OK;
+}
+
+extern "C" betty_status betty_sync_check(betty_ctx* c, betty_stream stream) {
+    if (!c) return BETTY_EINVAL;
+    return sync_check(c, (cudaStream_t)stream);
+}

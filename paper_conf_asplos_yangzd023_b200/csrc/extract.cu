@@ -1,0 +1,303 @@
+// extract.cu -- a2: micro-batch block extraction on the GPU.
+//
+// Batch-level partitioning (§4.2.3): micro-batch k keeps the
+// outputs V_k = {i : part[i] == k}; layer by layer (output -> input) its dst
+// list is the previous layer's src list and its src list is
+//     U_k = dst ++ (sources of the dst rows not in dst, ascending full-batch
+//            src position)                                 (readings #9/#10)
+// with edges relabelled to local src ids and the local -> global index map
+// (src_pos, src_gid) of PAPER.md:1167-1187.
+//
+// B200 design: a GROUP of c micro-batches is extracted by the same launches
+// (block-diagonal union, each micro-batch with its own dedupe state).  The
+// dedupe uses two bitmaps per micro-batch over the FULL-batch src positions of
+// the layer (n_src_full/8 bytes each: 306 KB for the products shape, L2
+// resident): `dstbits` marks the dst prefix, `newbits` the other sources.
+// The ascending order of new sources then falls out of a popcount scan over
+// the bitmap words -- no sort, no hash, no atomics-order dependence -- and a
+// new source's local id is n_dst + (#set bits before it).  Only dst nodes
+// need an explicit position -> local id map.  All sizes stay on the device.
+#include "common.cuh"
+#include "internal.h"
+#include "extract.h"
+
+namespace betty {
+
+// ----------------------------------------------------------- output select
+constexpr int SEL_CHUNK = 1024;
+
+__global__ void k_sel_count(const int32_t* __restrict__ part, int64_t n_out, int32_t K, const int32_t* __restrict__ ks,
+                            int32_t c, int32_t* __restrict__ chunk_cnt, int64_t nchunks, int* dev_err) {
+    __shared__ int s[32];
+    const int j = blockIdx.y;
+    const int32_t k = ks[j];
+    for (int64_t ch = blockIdx.x; ch < nchunks; ch += gridDim.x) {
+        int local = 0;
+        for (int64_t i = ch * SEL_CHUNK + threadIdx.x; i < mn64((ch + 1) * SEL_CHUNK, n_out); i += blockDim.x) {
+            const int32_t p = part[i];
+            if (j == 0 && (p < 0 || p >= K)) atomicOr(dev_err, DEVERR_BAD_PART);
+            local += (p == k);
+        }
+        int w = warp_sum(local);
+        if (lane_id() == 0) s[warp_id()] = w;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            int t = 0;
+            for (int i = 0; i < (int)(blockDim.x >> 5); ++i) t += s[i];
+            chunk_cnt[(int64_t)j * nchunks + ch] = t;
+        }
+        __syncthreads();
+    }
+}
+
+// each thread handles SEL_CHUNK/blockDim.x consecutive outputs of the chunk
+__global__ void __launch_bounds__(256) k_sel_write(const int32_t* __restrict__ part, int64_t n_out,
+                                                   const int32_t* __restrict__ ks, const int64_t* __restrict__ off,
+                                                   int64_t nchunks, int32_t* __restrict__ dst_pos,
+                                                   int32_t* __restrict__ row_mb) {
+    __shared__ int64_t s_warp[9];
+    const int j = blockIdx.y;
+    const int32_t k = ks[j];
+    constexpr int PER = SEL_CHUNK / 256;
+    for (int64_t ch = blockIdx.x; ch < nchunks; ch += gridDim.x) {
+        const int64_t b = ch * SEL_CHUNK + (int64_t)threadIdx.x * PER;
+        int flags = 0, cnt = 0;
+#pragma unroll
+        for (int t = 0; t < PER; ++t) {
+            const bool f = (b + t < n_out) && part[b + t] == k;
+            flags |= (int)f << t;
+            cnt += f;
+        }
+        int64_t tot;
+        int64_t pos = off[(int64_t)j * nchunks + ch] + block_excl_scan<int64_t>(cnt, s_warp, &tot);
+#pragma unroll
+        for (int t = 0; t < PER; ++t)
+            if (flags >> t & 1) { dst_pos[pos] = (int32_t)(b + t); row_mb[pos] = j; ++pos; }
+    }
+}
+
+// single CTA: per-slot dst offsets of the output layer
+__global__ void k_sel_offsets(const int64_t* __restrict__ off, int64_t nchunks, int32_t c, int64_t* mb_dst_off,
+                              int64_t* cnt) {
+    for (int j = threadIdx.x; j <= c; j += blockDim.x) mb_dst_off[j] = off[(int64_t)j * nchunks];
+    if (threadIdx.x == 0) cnt[0] = off[(int64_t)c * nchunks];
+}
+
+// ------------------------------------------------------------ per layer
+__global__ void k_deg(const int32_t* __restrict__ dst_pos, const int64_t* __restrict__ findptr, const int64_t* cnt,
+                      int64_t* __restrict__ deg) {
+    const int64_t n = cnt[0];
+    for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < n; r += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t p = dst_pos[r];
+        deg[r] = findptr[p + 1] - findptr[p];
+    }
+}
+
+__global__ void k_mark_dst(const int32_t* __restrict__ dst_pos, const int32_t* __restrict__ row_mb,
+                           const int64_t* __restrict__ mb_dst_off, const int64_t* cnt, uint32_t* dstbits, int64_t W,
+                           int32_t* __restrict__ map, int64_t map_stride) {
+    const int64_t n = cnt[0];
+    for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < n; r += (int64_t)gridDim.x * blockDim.x) {
+        const int j = row_mb[r];
+        const int32_t p = dst_pos[r];
+        atomicOr(&dstbits[j * W + (p >> 5)], 1u << (p & 31));
+        map[j * map_stride + p] = (int32_t)(r - mb_dst_off[j]);
+    }
+}
+
+__global__ void k_mark_new(const int32_t* __restrict__ dst_pos, const int32_t* __restrict__ row_mb,
+                           const int64_t* cnt, const int64_t* __restrict__ findptr, const int32_t* __restrict__ fnbr,
+                           const uint32_t* __restrict__ dstbits, uint32_t* newbits, int64_t W) {
+    const int64_t n = cnt[0];
+    const int lane = lane_id();
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t r = gw; r < n; r += nw) {
+        const int j = row_mb[r];
+        const int32_t q = dst_pos[r];
+        const int64_t b = findptr[q], e = findptr[q + 1];
+        const uint32_t* db = dstbits + j * W;
+        uint32_t* nb = newbits + j * W;
+        for (int64_t i = b + lane; i < e; i += 32) {
+            const int32_t p = fnbr[i];
+            const uint32_t bit = 1u << (p & 31);
+            if (!(db[p >> 5] & bit)) atomicOr(&nb[p >> 5], bit);
+        }
+    }
+}
+
+__global__ void k_popc(const uint32_t* __restrict__ newbits, int64_t n, int32_t* __restrict__ wc) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        wc[i] = __popc(newbits[i]);
+}
+
+// single CTA: per micro-batch src counts and offsets; checks capacities
+__global__ void k_counts(const int64_t* __restrict__ mb_dst_off, const int64_t* __restrict__ wordoff, int64_t W,
+                         int32_t c, int64_t* __restrict__ mb_src_off, int64_t* cnt, int64_t cap_src, int64_t cap_e,
+                         int64_t* next_cnt, int* dev_err) {
+    __shared__ int64_t s_warp[33];
+    __shared__ int64_t s_base;
+    if (threadIdx.x == 0) s_base = 0;
+    __syncthreads();
+    for (int j0 = 0; j0 < c; j0 += blockDim.x) {
+        const int j = j0 + threadIdx.x;
+        int64_t ns = 0;
+        if (j < c) ns = (mb_dst_off[j + 1] - mb_dst_off[j]) + (wordoff[(int64_t)(j + 1) * W] - wordoff[(int64_t)j * W]);
+        int64_t tot;
+        const int64_t ex = block_excl_scan(ns, s_warp, &tot);
+        if (j < c) mb_src_off[j] = s_base + ex;
+        __syncthreads();
+        if (threadIdx.x == 0) s_base += tot;
+        __syncthreads();
+    }
+    if (threadIdx.x == 0) {
+        mb_src_off[c] = s_base;
+        cnt[1] = s_base;
+        if (s_base > cap_src || cnt[2] > cap_e) atomicOr(dev_err, DEVERR_OVERFLOW);
+        if (next_cnt) next_cnt[0] = s_base;
+    }
+}
+
+__global__ void k_emit_new(const uint32_t* __restrict__ newbits, int64_t W, int32_t c,
+                           const int64_t* __restrict__ wordoff, const int64_t* __restrict__ mb_dst_off,
+                           const int64_t* __restrict__ mb_src_off, const int32_t* __restrict__ fsrc_gid,
+                           int32_t* __restrict__ src_pos, int32_t* __restrict__ src_gid, int32_t* __restrict__ src_mb,
+                           int64_t cap_src) {
+    const int64_t n = (int64_t)c * W;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        uint32_t bits = newbits[i];
+        if (!bits) continue;
+        const int j = (int)(i / W);
+        const int64_t w = i - (int64_t)j * W;
+        int64_t s = mb_src_off[j] + (mb_dst_off[j + 1] - mb_dst_off[j]) + (wordoff[i] - wordoff[(int64_t)j * W]);
+        while (bits) {
+            const int b = __ffs(bits) - 1;
+            bits &= bits - 1;
+            const int32_t p = (int32_t)(w * 32 + b);
+            if (s < cap_src) { src_pos[s] = p; src_gid[s] = fsrc_gid[p]; src_mb[s] = j; }
+            ++s;
+        }
+    }
+}
+
+__global__ void k_emit_dst(const int32_t* __restrict__ dst_pos, const int32_t* __restrict__ row_mb,
+                           const int64_t* cnt, const int64_t* __restrict__ mb_dst_off,
+                           const int64_t* __restrict__ mb_src_off, const int32_t* __restrict__ fsrc_gid,
+                           int32_t* __restrict__ src_pos, int32_t* __restrict__ src_gid, int32_t* __restrict__ src_mb,
+                           int64_t cap_src) {
+    const int64_t n = cnt[0];
+    for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < n; r += (int64_t)gridDim.x * blockDim.x) {
+        const int j = row_mb[r];
+        const int64_t s = mb_src_off[j] + (r - mb_dst_off[j]);
+        const int32_t p = dst_pos[r];
+        if (s < cap_src) { src_pos[s] = p; src_gid[s] = fsrc_gid[p]; src_mb[s] = j; }
+    }
+}
+
+__global__ void k_relabel(const int32_t* __restrict__ dst_pos, const int32_t* __restrict__ row_mb, const int64_t* cnt,
+                          const int64_t* __restrict__ findptr, const int32_t* __restrict__ fnbr,
+                          const int64_t* __restrict__ indptr, const uint32_t* __restrict__ dstbits,
+                          const uint32_t* __restrict__ newbits, const int64_t* __restrict__ wordoff, int64_t W,
+                          const int32_t* __restrict__ map, int64_t map_stride, const int64_t* __restrict__ mb_dst_off,
+                          const int64_t* __restrict__ mb_src_off, int32_t* __restrict__ indices, int64_t cap_e) {
+    const int64_t n = cnt[0];
+    const int lane = lane_id();
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t r = gw; r < n; r += nw) {
+        const int j = row_mb[r];
+        const int32_t q = dst_pos[r];
+        const int64_t fb = findptr[q], fe = findptr[q + 1];
+        const int64_t ob = indptr[r];
+        const uint32_t* db = dstbits + j * W;
+        const uint32_t* nb = newbits + j * W;
+        const int64_t* wo = wordoff + j * W;
+        const int64_t wo0 = wo[0];
+        const int64_t nd = mb_dst_off[j + 1] - mb_dst_off[j];
+        const int64_t so = mb_src_off[j];
+        for (int64_t i = fb + lane; i < fe; i += 32) {
+            const int32_t p = fnbr[i];
+            const int32_t w = p >> 5;
+            const uint32_t bit = 1u << (p & 31);
+            int64_t local;
+            if (db[w] & bit) local = map[j * map_stride + p];
+            else local = nd + (wo[w] - wo0) + __popc(nb[w] & (bit - 1));
+            const int64_t o = ob + (i - fb);
+            if (o < cap_e) indices[o] = (int32_t)(so + local);
+        }
+    }
+}
+
+__global__ void k_clear_bits(uint32_t* a, uint32_t* b, int64_t n) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        a[i] = 0u;
+        b[i] = 0u;
+    }
+}
+
+static inline int grid_for(betty_ctx* c, int64_t work, int threads, int per_sm = 8) {
+    return (int)std::max<int64_t>(1, std::min<int64_t>((work + threads - 1) / threads, (int64_t)c->num_sms * per_sm));
+}
+
+size_t extract_scratch_bytes(int64_t c, int64_t max_full_src, int64_t sel_nchunks) {
+    const int64_t W = (max_full_src + 31) / 32 + 1;
+    return (size_t)(c * W * 4 * 2 + c * max_full_src * 4 + (c * W + 1) * 8 + c * W * 4 +
+                    (c * sel_nchunks + 1) * 8 + c * sel_nchunks * 4 + 4096);
+}
+
+void extract_group(betty_ctx* ctx, const ExtractArgs& a, cudaStream_t s) {
+    const int32_t c = a.c;
+    const int64_t n_out = a.full[a.L - 1].n_dst;
+    const int64_t nchunks = (n_out + SEL_CHUNK - 1) / SEL_CHUNK;
+    ExtractLayer* top = &a.layers[a.L - 1];
+
+    // ---- V_k: outputs with part == ks[j], ascending, for every slot j
+    {
+        dim3 g((unsigned)std::max<int64_t>(1, std::min<int64_t>(nchunks, 1024)), (unsigned)c);
+        k_sel_count<<<g, 256, 0, s>>>(a.part, n_out, a.K, a.ks, c, a.sc.sel_cnt, nchunks, ctx->dev_err);
+        scan_i32(ctx, a.sc.sel_cnt, a.sc.sel_off, nullptr, (int64_t)c * nchunks, 0, nullptr, s);
+        k_sel_write<<<g, 256, 0, s>>>(a.part, n_out, a.ks, a.sc.sel_off, nchunks, a.sc.top_dst_pos, a.sc.top_row_mb);
+        k_sel_offsets<<<1, 256, 0, s>>>(a.sc.sel_off, nchunks, c, a.sc.top_dst_off, top->cnt);
+    }
+
+    const int32_t* dst_pos = a.sc.top_dst_pos;
+    const int32_t* row_mb = a.sc.top_row_mb;
+    const int64_t* dst_off = a.sc.top_dst_off;
+    for (int l = a.L - 1; l >= 0; --l) {
+        const ExtractFull& F = a.full[l];
+        ExtractLayer& B = a.layers[l];
+        const int64_t W = (F.n_src + 31) / 32;
+        const int64_t cW = (int64_t)c * W;
+        const int64_t cap_d = B.cap_dst, cap_e = B.cap_e, cap_s = B.cap_src;
+        // rows: degree of each dst row in the full batch -> local indptr
+        k_deg<<<grid_for(ctx, cap_d, 256), 256, 0, s>>>(dst_pos, F.indptr, B.cnt, a.sc.deg);
+        scan_i64(ctx, a.sc.deg, B.indptr, B.cnt + 0, 0, cap_d, B.cnt + 2, s);
+        // dedupe: dst bitmap + position map, then new-source bitmap
+        k_mark_dst<<<grid_for(ctx, cap_d, 256), 256, 0, s>>>(dst_pos, row_mb, dst_off, B.cnt, a.sc.dstbits, W,
+                                                             a.sc.map, a.sc.map_stride);
+        k_mark_new<<<grid_for(ctx, cap_d * 32, 256), 256, 0, s>>>(dst_pos, row_mb, B.cnt, F.indptr, F.nbr,
+                                                                  a.sc.dstbits, a.sc.newbits, W);
+        // ascending order of new sources = popcount scan over the bitmap words
+        k_popc<<<grid_for(ctx, cW, 256), 256, 0, s>>>(a.sc.newbits, cW, a.sc.wordcnt);
+        scan_i32(ctx, a.sc.wordcnt, a.sc.wordoff, nullptr, cW, 0, nullptr, s);
+        k_counts<<<1, 1024, 0, s>>>(dst_off, a.sc.wordoff, W, c, B.mb_src_off, B.cnt, cap_s, cap_e,
+                                    l > 0 ? a.layers[l - 1].cnt : nullptr, ctx->dev_err);
+        k_emit_dst<<<grid_for(ctx, cap_d, 256), 256, 0, s>>>(dst_pos, row_mb, B.cnt, dst_off, B.mb_src_off,
+                                                             F.src_gid, B.src_pos, B.src_gid, B.src_mb, cap_s);
+        k_emit_new<<<grid_for(ctx, cW, 256), 256, 0, s>>>(a.sc.newbits, W, c, a.sc.wordoff, dst_off, B.mb_src_off,
+                                                          F.src_gid, B.src_pos, B.src_gid, B.src_mb, cap_s);
+        k_relabel<<<grid_for(ctx, cap_d * 32, 256), 256, 0, s>>>(dst_pos, row_mb, B.cnt, F.indptr, F.nbr, B.indptr,
+                                                                 a.sc.dstbits, a.sc.newbits, a.sc.wordoff, W, a.sc.map,
+                                                                 a.sc.map_stride, dst_off, B.mb_src_off, B.indices,
+                                                                 cap_e);
+        k_clear_bits<<<grid_for(ctx, cW, 256), 256, 0, s>>>(a.sc.dstbits, a.sc.newbits, cW);
+        if (B.t_indptr && (a.csc_mask >> l & 1))
+            csr_transpose(ctx, B.indptr, B.indices, B.cnt + 0, B.cnt + 1, B.cnt + 2, cap_d, cap_s, cap_e,
+                          B.t_indptr, B.t_indices, a.sc.tcnt, false, s);
+        dst_pos = B.src_pos;
+        row_mb = B.src_mb;
+        dst_off = B.mb_src_off;
+    }
+}
+
+}  // namespace betty

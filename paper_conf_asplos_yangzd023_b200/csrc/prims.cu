@@ -1,0 +1,298 @@
+// prims.cu -- device-wide primitives with DEVICE-resident sizes, so that a
+// whole training step runs without host synchronisation (graph-capturable):
+//   * single-pass exclusive scan (decoupled look-back, persistent CTAs)
+//   * segmented sort of short int32 segments (warp / CTA bitonic)
+//   * CSR -> CSC transpose with ascending row ids per column
+#include <climits>
+#include "common.cuh"
+#include "internal.h"
+
+namespace betty {
+
+// ------------------------------------------------------------------ scan
+constexpr int SCAN_THREADS = 256;
+constexpr int SCAN_ITEMS = 8;
+constexpr int SCAN_TILE = SCAN_THREADS * SCAN_ITEMS;
+constexpr unsigned long long ST_AGG = 1ull << 62, ST_PRE = 2ull << 62, ST_VAL = (1ull << 62) - 1;
+
+__device__ __forceinline__ unsigned long long ld_acquire(const unsigned long long* p) {
+    unsigned long long v;
+    asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release(unsigned long long* p, unsigned long long v) {
+    asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+template <typename Tin>
+__global__ void __launch_bounds__(SCAN_THREADS) k_scan(const Tin* __restrict__ in, int64_t* __restrict__ out,
+                                                       const int64_t* n_dev, int64_t n_fixed, int64_t* total_dev,
+                                                       unsigned long long* status, unsigned* ctr) {
+    __shared__ int64_t s_warp[SCAN_THREADS / 32 + 1];
+    __shared__ int64_t s_tile, s_prefix;
+    __shared__ int s_last;
+    const int64_t n = n_dev ? *n_dev : n_fixed;
+    const int64_t n_tiles = (n + SCAN_TILE - 1) / SCAN_TILE;
+    for (;;) {
+        if (threadIdx.x == 0) s_tile = atomicAdd(&ctr[0], 1u);
+        __syncthreads();
+        const int64_t t = s_tile;
+        if (t >= n_tiles) break;
+        const int64_t base = t * SCAN_TILE + (int64_t)threadIdx.x * SCAN_ITEMS;
+        int64_t v[SCAN_ITEMS];
+        int64_t sum = 0;
+#pragma unroll
+        for (int i = 0; i < SCAN_ITEMS; ++i) {
+            const int64_t idx = base + i;
+            v[i] = idx < n ? (int64_t)in[idx] : 0;
+            sum += v[i];
+        }
+        int64_t agg;
+        const int64_t ex = block_excl_scan(sum, s_warp, &agg);
+        if (threadIdx.x == 0) {
+            int64_t prefix = 0;
+            if (t == 0) {
+                st_release(&status[0], ST_PRE | (unsigned long long)agg);
+            } else {
+                st_release(&status[t], ST_AGG | (unsigned long long)agg);
+                for (int64_t j = t - 1;;) {
+                    const unsigned long long s = ld_acquire(&status[j]);
+                    const unsigned long long f = s >> 62;
+                    if (f == 0) continue;                     // predecessor not published yet
+                    prefix += (int64_t)(s & ST_VAL);
+                    if (f == 2) break;
+                    --j;
+                }
+                st_release(&status[t], ST_PRE | (unsigned long long)(prefix + agg));
+            }
+            s_prefix = prefix;
+            if (t == n_tiles - 1 && total_dev) *total_dev = prefix + agg;
+            if (t == 0) out[0] = 0;
+        }
+        __syncthreads();
+        int64_t run = s_prefix + ex;
+#pragma unroll
+        for (int i = 0; i < SCAN_ITEMS; ++i) {
+            const int64_t idx = base + i;
+            run += v[i];
+            if (idx < n) out[idx + 1] = run;
+        }
+        __syncthreads();
+    }
+    if (n_tiles == 0 && blockIdx.x == 0 && threadIdx.x == 0) {
+        out[0] = 0;
+        if (total_dev) *total_dev = 0;
+    }
+    // the last CTA to finish clears the tile status and the counters
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence();
+        s_last = (atomicAdd(&ctr[1], 1u) == gridDim.x - 1);
+    }
+    __syncthreads();
+    if (s_last) {
+        for (int64_t j = threadIdx.x; j < n_tiles; j += blockDim.x) status[j] = 0;
+        if (threadIdx.x == 0) { ctr[0] = 0; ctr[1] = 0; }
+        __threadfence();
+    }
+}
+
+void ensure_scan_scratch(betty_ctx* c, int64_t n_cap, cudaStream_t s) {
+    const int64_t tiles = (n_cap + SCAN_TILE - 1) / SCAN_TILE + 1;
+    if (tiles > c->scan_status_cap) {
+        // growing is only legal outside graph capture; plan creation sizes it first
+        if (c->scan_status) ctx_free(c, c->scan_status, s);
+        const int64_t cap = tiles * 2 + 1024;
+        c->scan_status = (unsigned long long*)ctx_alloc(c, sizeof(unsigned long long) * cap, s);
+        cudaMemsetAsync(c->scan_status, 0, sizeof(unsigned long long) * cap, s);
+        c->scan_status_cap = cap;
+    }
+}
+
+template <typename Tin>
+static void scan_impl(betty_ctx* c, const Tin* in, int64_t* out, const int64_t* n_dev, int64_t n_fixed, int64_t n_cap,
+                      int64_t* total_dev, cudaStream_t s) {
+    if (!n_dev) n_cap = n_fixed;
+    ensure_scan_scratch(c, n_cap, s);
+    int64_t tiles = (n_cap + SCAN_TILE - 1) / SCAN_TILE;
+    int grid = (int)std::min<int64_t>(std::max<int64_t>(tiles, 1), (int64_t)c->num_sms * 2);
+    k_scan<Tin><<<grid, SCAN_THREADS, 0, s>>>(in, out, n_dev, n_fixed, total_dev, c->scan_status,
+                                              c->counters + CTR_SCAN);
+}
+
+void scan_i64(betty_ctx* c, const int64_t* in, int64_t* out, const int64_t* n_dev, int64_t n_fixed, int64_t n_cap,
+              int64_t* total_dev, cudaStream_t s) {
+    scan_impl<int64_t>(c, in, out, n_dev, n_fixed, n_cap, total_dev, s);
+}
+void scan_i32(betty_ctx* c, const int32_t* in, int64_t* out, const int64_t* n_dev, int64_t n_fixed, int64_t n_cap,
+              int64_t* total_dev, cudaStream_t s) {
+    scan_impl<int32_t>(c, in, out, n_dev, n_fixed, n_cap, total_dev, s);
+}
+
+// ---------------------------------------------------------------- memset
+__global__ void k_memset(uint32_t* p, uint32_t v, const int64_t* n_dev, int64_t elem_words, int64_t n_fixed) {
+    const int64_t n = (n_dev ? *n_dev : n_fixed) * elem_words;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        p[i] = v;
+}
+void memset_dev(void* p, int value, const int64_t* n_dev, int64_t elem_bytes, int64_t n_cap, cudaStream_t s) {
+    // elem_bytes must be a multiple of 4; value is replicated per byte
+    const uint32_t v = (uint32_t)(value & 0xff) * 0x01010101u;
+    const int64_t words = n_cap * (elem_bytes / 4);
+    int grid = (int)std::min<int64_t>((words + 255) / 256 + 1, 148 * 8);
+    k_memset<<<grid, 256, 0, s>>>((uint32_t*)p, v, n_dev, elem_bytes / 4, n_cap);
+}
+
+// --------------------------------------------------------- segmented sort
+constexpr int SEG_WARP_MAX = 512;
+constexpr int SEG_CTA_MAX = 32768;
+
+__device__ __forceinline__ int32_t warp_bitonic32(int32_t x) {
+    const int lane = lane_id();
+#pragma unroll
+    for (int k = 2; k <= 32; k <<= 1) {
+#pragma unroll
+        for (int j = k >> 1; j > 0; j >>= 1) {
+            const int32_t y = __shfl_xor_sync(0xffffffffu, x, j);
+            const bool up = ((lane & k) == 0);
+            const bool lower = ((lane & j) == 0);
+            // lower element keeps min when ascending
+            x = (lower == up) ? min(x, y) : max(x, y);
+        }
+    }
+    return x;
+}
+
+__device__ void smem_bitonic(int32_t* s, int P, int tid, int nthreads, bool warp_only) {
+    for (int k = 2; k <= P; k <<= 1) {
+        for (int j = k >> 1; j > 0; j >>= 1) {
+            for (int i = tid; i < P; i += nthreads) {
+                const int ixj = i ^ j;
+                if (ixj > i) {
+                    const int32_t a = s[i], b = s[ixj];
+                    const bool up = ((i & k) == 0);
+                    if ((a > b) == up) { s[i] = b; s[ixj] = a; }
+                }
+            }
+            if (warp_only) __syncwarp(); else __syncthreads();
+        }
+    }
+}
+
+__global__ void __launch_bounds__(256) k_segsort_warp(const int64_t* __restrict__ ptr, int32_t* __restrict__ keys,
+                                                      const int64_t* nseg_dev, int64_t nseg_fixed, int64_t* big,
+                                                      int* big_cnt, int64_t big_cap, int* dev_err) {
+    __shared__ int32_t buf[8][SEG_WARP_MAX];
+    const int64_t nseg = nseg_dev ? *nseg_dev : nseg_fixed;
+    const int w = warp_id(), lane = lane_id();
+    const int64_t gw = blockIdx.x * 8ll + w, nw = gridDim.x * 8ll;
+    for (int64_t seg = gw; seg < nseg; seg += nw) {
+        const int64_t b = ptr[seg], len = ptr[seg + 1] - b;
+        if (len <= 1) continue;
+        if (len <= 32) {
+            int32_t x = lane < len ? keys[b + lane] : INT_MAX;
+            x = warp_bitonic32(x);
+            if (lane < len) keys[b + lane] = x;
+        } else if (len <= SEG_WARP_MAX) {
+            int P = 64;
+            while (P < len) P <<= 1;
+            for (int i = lane; i < P; i += 32) buf[w][i] = i < len ? keys[b + i] : INT_MAX;
+            __syncwarp();
+            smem_bitonic(buf[w], P, lane, 32, true);
+            for (int i = lane; i < len; i += 32) keys[b + i] = buf[w][i];
+            __syncwarp();
+        } else if (lane == 0) {
+            const int i = atomicAdd(big_cnt, 1);
+            if (i < big_cap) big[i] = seg; else atomicOr(dev_err, DEVERR_OVERFLOW);
+        }
+    }
+}
+
+__global__ void __launch_bounds__(1024) k_segsort_big(const int64_t* __restrict__ ptr, int32_t* __restrict__ keys,
+                                                      const int64_t* big, int* big_cnt, int* dev_err) {
+    extern __shared__ int32_t sbuf[];
+    const int n_big = *big_cnt;
+    for (int t = blockIdx.x; t < n_big; t += gridDim.x) {
+        const int64_t seg = big[t];
+        const int64_t b = ptr[seg], len = ptr[seg + 1] - b;
+        if (len > SEG_CTA_MAX) {
+            if (threadIdx.x == 0) atomicOr(dev_err, DEVERR_OVERFLOW);
+            continue;
+        }
+        int P = 1024;
+        while (P < len) P <<= 1;
+        for (int i = threadIdx.x; i < P; i += blockDim.x) sbuf[i] = i < len ? keys[b + i] : INT_MAX;
+        __syncthreads();
+        smem_bitonic(sbuf, P, threadIdx.x, blockDim.x, false);
+        for (int i = threadIdx.x; i < len; i += blockDim.x) keys[b + i] = sbuf[i];
+        __syncthreads();
+    }
+}
+
+__global__ void k_reset_int(int* p) { *p = 0; }
+
+void init_prims_attrs() {
+    cudaFuncSetAttribute(k_segsort_big, cudaFuncAttributeMaxDynamicSharedMemorySize, SEG_CTA_MAX * 4);
+}
+
+void segsort_i32(betty_ctx* c, const int64_t* ptr, int32_t* keys, const int64_t* nseg_dev, int64_t nseg_fixed,
+                 int64_t nseg_cap, cudaStream_t s) {
+    if (!nseg_dev) nseg_cap = nseg_fixed;
+    int grid = (int)std::min<int64_t>((nseg_cap + 7) / 8 + 1, (int64_t)c->num_sms * 8);
+    k_reset_int<<<1, 1, 0, s>>>(c->big_count);
+    k_segsort_warp<<<grid, 256, 0, s>>>(ptr, keys, nseg_dev, nseg_fixed, c->big_list, c->big_count, c->big_list_cap,
+                                        c->dev_err);
+    k_segsort_big<<<c->num_sms, 1024, SEG_CTA_MAX * 4, s>>>(ptr, keys, c->big_list, c->big_count, c->dev_err);
+}
+
+// ------------------------------------------------------------- transpose
+__global__ void k_hist(const int32_t* __restrict__ idx, const int64_t* n_edges_dev, int32_t* cnt) {
+    const int64_t n = *n_edges_dev;
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < n; e += (int64_t)gridDim.x * blockDim.x)
+        atomicAdd(&cnt[idx[e]], 1);
+}
+
+__global__ void k_scatter_t(const int64_t* __restrict__ indptr, const int32_t* __restrict__ idx,
+                            const int64_t* n_rows_dev, const int64_t* __restrict__ t_indptr, int32_t* cursor,
+                            int32_t* __restrict__ t_idx) {
+    const int64_t n = *n_rows_dev;
+    const int lane = lane_id();
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t r = gw; r < n; r += nw) {
+        const int64_t b = indptr[r], e = indptr[r + 1];
+        for (int64_t i = b + lane; i < e; i += 32) {
+            const int32_t col = idx[i];
+            const int32_t k = atomicAdd(&cursor[col], 1);
+            t_idx[t_indptr[col] + k] = (int32_t)r;
+        }
+    }
+}
+
+__global__ void k_dup_check(const int64_t* __restrict__ t_indptr, const int32_t* __restrict__ t_idx,
+                            const int64_t* n_cols_dev, int* dev_err) {
+    const int64_t n = *n_cols_dev;
+    for (int64_t col = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; col < n; col += (int64_t)gridDim.x * blockDim.x)
+        for (int64_t i = t_indptr[col] + 1; i < t_indptr[col + 1]; ++i)
+            if (t_idx[i] == t_idx[i - 1]) { atomicOr(dev_err, DEVERR_DUP_EDGE); break; }
+}
+
+void csr_transpose(betty_ctx* c, const int64_t* indptr, const int32_t* idx, const int64_t* n_rows_dev,
+                   const int64_t* n_cols_dev, const int64_t* n_edges_dev, int64_t rows_cap, int64_t cols_cap,
+                   int64_t edges_cap, int64_t* t_indptr, int32_t* t_idx, int32_t* cnt, bool dup_check,
+                   cudaStream_t s) {
+    const int g_e = (int)std::min<int64_t>((edges_cap + 255) / 256 + 1, (int64_t)c->num_sms * 8);
+    const int g_r = (int)std::min<int64_t>((rows_cap * 32 + 255) / 256 + 1, (int64_t)c->num_sms * 8);
+    memset_dev(cnt, 0, n_cols_dev, 4, cols_cap, s);
+    k_hist<<<g_e, 256, 0, s>>>(idx, n_edges_dev, cnt);
+    scan_i32(c, cnt, t_indptr, n_cols_dev, 0, cols_cap, nullptr, s);
+    memset_dev(cnt, 0, n_cols_dev, 4, cols_cap, s);
+    k_scatter_t<<<g_r, 256, 0, s>>>(indptr, idx, n_rows_dev, t_indptr, cnt, t_idx);
+    segsort_i32(c, t_indptr, t_idx, n_cols_dev, 0, cols_cap, s);
+    if (dup_check) {
+        const int g_c = (int)std::min<int64_t>((cols_cap + 255) / 256 + 1, (int64_t)c->num_sms * 8);
+        k_dup_check<<<g_c, 256, 0, s>>>(t_indptr, t_idx, n_cols_dev, c->dev_err);
+    }
+}
+
+}  // namespace betty

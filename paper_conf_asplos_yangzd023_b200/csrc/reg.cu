@@ -1,0 +1,227 @@
+// reg.cu -- a1: the redundancy-embedded graph (REG) as an integer SpGEMM.
+//
+// PAPER.md:771-945 (§4.3.2, Eq. 2-4, Alg. 1 lines 1-7): A is the binary
+// adjacency of the output block (a_ui = 1 iff sampled edge u -> i), C = A^T A,
+// c_ij = sum_u a_ui a_uj = number of input neighbours shared by outputs i and
+// j; only output nodes are kept and self loops removed.  With B = A^T
+// restricted to (outputs x sources), C = B B^T.
+//
+// GPU design (row-wise expansion, sort-based accumulation, bit-exact):
+//   1. CSC of B (counting sort + per-column sort; rejects repeated edges)
+//   2. ub_i = sum_{u in S_i} (d_u - 1): exact number of candidate products of row i
+//   3. exclusive scan of ub -> a temporary slot per product
+//   4. per row: expand the candidates j (from the columns of its sources,
+//      skipping j = i), sort them (warp bitonic for ub <= 256, CTA bitonic
+//      in shared memory up to 32768), run-length encode -> (j, c_ij) ascending
+//   5. scan of the per-row counts -> indptr, compaction into col / w
+// Every step is integer and order-independent, so the result is bit-exact.
+#include <climits>
+#include "common.cuh"
+#include "internal.h"
+#include "reg.h"
+
+namespace betty {
+
+constexpr int REG_WARP_MAX = 256;
+constexpr int REG_CTA_MAX = 32768;
+
+__global__ void k_reset_big(int* p) { *p = 0; }
+
+__global__ void k_reg_ub(const int64_t* __restrict__ indptr, const int32_t* __restrict__ idx,
+                         const int64_t* __restrict__ t_indptr, const int64_t* n_rows_dev, int64_t* __restrict__ ub,
+                         int64_t* big, int* big_cnt, int64_t big_cap, int* dev_err) {
+    const int64_t n = *n_rows_dev;
+    const int lane = lane_id();
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t i = gw; i < n; i += nw) {
+        int64_t s = 0;
+        for (int64_t e = indptr[i] + lane; e < indptr[i + 1]; e += 32) {
+            const int32_t u = idx[e];
+            s += t_indptr[u + 1] - t_indptr[u] - 1;
+        }
+        s = warp_sum(s);
+        if (lane == 0) {
+            ub[i] = s;
+            if (s > REG_WARP_MAX) {
+                if (s > REG_CTA_MAX) atomicOr(dev_err, DEVERR_OVERFLOW);
+                const int k = atomicAdd(big_cnt, 1);
+                if (k < big_cap) big[k] = i; else atomicOr(dev_err, DEVERR_OVERFLOW);
+            }
+        }
+    }
+}
+
+// expand the candidate list of row i into buf[0, ub) (ub known), cooperative over `nthr` threads
+__device__ __forceinline__ void reg_expand(const int64_t* __restrict__ indptr, const int32_t* __restrict__ idx,
+                                           const int64_t* __restrict__ t_indptr, const int32_t* __restrict__ t_idx,
+                                           int64_t i, int32_t* buf, int tid, int nthr) {
+    int64_t o = 0;
+    for (int64_t e = indptr[i]; e < indptr[i + 1]; ++e) {
+        const int32_t u = idx[e];
+        const int64_t b = t_indptr[u], d = t_indptr[u + 1] - b;
+        // column u lists i exactly once (no repeated edges): skip it, keep order irrelevant
+        for (int64_t t = tid; t < d; t += nthr) {
+            const int32_t j = t_idx[b + t];
+            if (j == (int32_t)i) continue;
+            // position: entries before the one equal to i keep t, after it t-1
+            // (i appears once; find its slot by comparing: t_idx is ascending per column)
+            buf[o + (j < (int32_t)i ? t : t - 1)] = j;
+        }
+        o += d - 1;
+    }
+}
+
+// run-length encode sorted buf[0, n) -> (col, w) at out offset; returns count (to all threads)
+__device__ __forceinline__ void reg_rle_store(const int32_t* buf, int n, int32_t* __restrict__ ocol,
+                                              int32_t* __restrict__ ow, int tid, int nthr, int* s_cnt) {
+    // sequential over 32-element chunks per warp would be simplest; use a block-wide two-pass
+    for (int base = 0; base < n; base += nthr) {
+        const int t = base + tid;
+        const bool head = t < n && (t == 0 || buf[t] != buf[t - 1]);
+        int run = 0;
+        if (head) {
+            int e = t + 1;
+            while (e < n && buf[e] == buf[t]) ++e;
+            run = e - t;
+        }
+        // rank of heads before t within the whole row: count heads in [0, t)
+        // (computed with an atomic counter in shared memory per chunk, ordered by ballot)
+        const unsigned bal = __ballot_sync(0xffffffffu, head);
+        const int wpos = __popc(bal & ((1u << lane_id()) - 1));
+        __shared__ int s_wcnt[32];
+        if (nthr > 32) {
+            if (lane_id() == 0) s_wcnt[warp_id()] = __popc(bal);
+            __syncthreads();
+            int before = 0;
+            for (int w = 0; w < warp_id(); ++w) before += s_wcnt[w];
+            if (head) { ocol[*s_cnt + before + wpos] = buf[t]; ow[*s_cnt + before + wpos] = run; }
+            __syncthreads();
+            if (tid == 0) { int tot = 0; for (int w = 0; w < nthr / 32; ++w) tot += s_wcnt[w]; *s_cnt += tot; }
+            __syncthreads();
+        } else {
+            if (head) { ocol[*s_cnt + wpos] = buf[t]; ow[*s_cnt + wpos] = run; }
+            __syncwarp();
+            if (tid == 0) *s_cnt += __popc(bal);
+            __syncwarp();
+        }
+    }
+}
+
+__device__ void bitonic_sort(int32_t* s, int P, int tid, int nthr, bool warp_only) {
+    for (int k = 2; k <= P; k <<= 1)
+        for (int j = k >> 1; j > 0; j >>= 1) {
+            for (int i = tid; i < P; i += nthr) {
+                const int ixj = i ^ j;
+                if (ixj > i) {
+                    const int32_t a = s[i], b = s[ixj];
+                    if ((a > b) == ((i & k) == 0)) { s[i] = b; s[ixj] = a; }
+                }
+            }
+            if (warp_only) __syncwarp(); else __syncthreads();
+        }
+}
+
+__global__ void __launch_bounds__(256) k_reg_rows_warp(const int64_t* __restrict__ indptr,
+                                                       const int32_t* __restrict__ idx,
+                                                       const int64_t* __restrict__ t_indptr,
+                                                       const int32_t* __restrict__ t_idx, const int64_t* n_rows_dev,
+                                                       const int64_t* __restrict__ ub, const int64_t* __restrict__ off,
+                                                       int32_t* __restrict__ tcol, int32_t* __restrict__ tw,
+                                                       int64_t* __restrict__ nnz) {
+    __shared__ int32_t buf[8][REG_WARP_MAX];
+    __shared__ int s_cnt[8];
+    const int64_t n = *n_rows_dev;
+    const int w = warp_id(), lane = lane_id();
+    const int64_t gw = blockIdx.x * 8ll + w, nw = gridDim.x * 8ll;
+    for (int64_t i = gw; i < n; i += nw) {
+        const int64_t u = ub[i];
+        if (u > REG_WARP_MAX) continue;                 // handled by the CTA kernel
+        if (u == 0) { if (lane == 0) nnz[i] = 0; continue; }
+        reg_expand(indptr, idx, t_indptr, t_idx, i, buf[w], lane, 32);
+        int P = 32;
+        while (P < u) P <<= 1;
+        for (int t = (int)u + lane; t < P; t += 32) buf[w][t] = INT_MAX;
+        __syncwarp();
+        bitonic_sort(buf[w], P, lane, 32, true);
+        if (lane == 0) s_cnt[w] = 0;
+        __syncwarp();
+        reg_rle_store(buf[w], (int)u, tcol + off[i], tw + off[i], lane, 32, &s_cnt[w]);
+        if (lane == 0) nnz[i] = s_cnt[w];
+        __syncwarp();
+    }
+}
+
+__global__ void __launch_bounds__(1024) k_reg_rows_cta(const int64_t* __restrict__ indptr,
+                                                       const int32_t* __restrict__ idx,
+                                                       const int64_t* __restrict__ t_indptr,
+                                                       const int32_t* __restrict__ t_idx,
+                                                       const int64_t* __restrict__ ub, const int64_t* __restrict__ off,
+                                                       const int64_t* big, const int* big_cnt,
+                                                       int32_t* __restrict__ tcol, int32_t* __restrict__ tw,
+                                                       int64_t* __restrict__ nnz) {
+    extern __shared__ int32_t sbuf[];
+    __shared__ int s_cnt;
+    const int nb = *big_cnt;
+    for (int t = blockIdx.x; t < nb; t += gridDim.x) {
+        const int64_t i = big[t];
+        const int64_t u = ub[i];
+        if (u > REG_CTA_MAX) { if (threadIdx.x == 0) nnz[i] = 0; continue; }
+        reg_expand(indptr, idx, t_indptr, t_idx, i, sbuf, threadIdx.x, blockDim.x);
+        int P = 1024;
+        while (P < u) P <<= 1;
+        for (int q = (int)u + threadIdx.x; q < P; q += blockDim.x) sbuf[q] = INT_MAX;
+        __syncthreads();
+        bitonic_sort(sbuf, P, threadIdx.x, blockDim.x, false);
+        if (threadIdx.x == 0) s_cnt = 0;
+        __syncthreads();
+        reg_rle_store(sbuf, (int)u, tcol + off[i], tw + off[i], threadIdx.x, blockDim.x, &s_cnt);
+        if (threadIdx.x == 0) nnz[i] = s_cnt;
+        __syncthreads();
+    }
+}
+
+__global__ void k_reg_compact(const int64_t* __restrict__ off, const int64_t* __restrict__ rp,
+                              const int64_t* n_rows_dev, const int32_t* __restrict__ tcol,
+                              const int32_t* __restrict__ tw, int32_t* __restrict__ col, int32_t* __restrict__ w,
+                              int64_t nnz_cap) {
+    const int64_t n = *n_rows_dev;
+    const int lane = lane_id();
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t i = gw; i < n; i += nw) {
+        const int64_t b = rp[i], len = rp[i + 1] - b, o = off[i];
+        for (int64_t t = lane; t < len; t += 32)
+            if (b + t < nnz_cap) { col[b + t] = tcol[o + t]; w[b + t] = tw[o + t]; }
+    }
+}
+
+void init_reg_attrs() {
+    cudaFuncSetAttribute(k_reg_rows_cta, cudaFuncAttributeMaxDynamicSharedMemorySize, REG_CTA_MAX * 4);
+}
+
+void reg_phase1(betty_ctx* c, const RegArgs& a, cudaStream_t s) {
+    csr_transpose(c, a.indptr, a.idx, a.n_rows_dev, a.n_cols_dev, a.n_edges_dev, a.rows_cap, a.cols_cap, a.edges_cap,
+                  a.t_indptr, a.t_idx, a.tcnt, true, s);
+    const int gw = (int)std::max<int64_t>(1, std::min<int64_t>((a.rows_cap * 32 + 255) / 256, (int64_t)c->num_sms * 16));
+    k_reset_big<<<1, 1, 0, s>>>(c->big_count);
+    k_reg_ub<<<gw, 256, 0, s>>>(a.indptr, a.idx, a.t_indptr, a.n_rows_dev, a.ub, c->big_list, c->big_count,
+                                c->big_list_cap, c->dev_err);
+    scan_i64(c, a.ub, a.off, a.n_rows_dev, 0, a.rows_cap, a.ub_total_dev, s);
+}
+
+void reg_phase2(betty_ctx* c, const RegArgs& a, cudaStream_t s) {
+    const int gw = (int)std::max<int64_t>(1, std::min<int64_t>((a.rows_cap * 32 + 255) / 256, (int64_t)c->num_sms * 16));
+    k_reg_rows_warp<<<gw, 256, 0, s>>>(a.indptr, a.idx, a.t_indptr, a.t_idx, a.n_rows_dev, a.ub, a.off, a.tcol, a.tw,
+                                       a.row_nnz);
+    k_reg_rows_cta<<<c->num_sms, 1024, REG_CTA_MAX * 4, s>>>(a.indptr, a.idx, a.t_indptr, a.t_idx, a.ub, a.off,
+                                                            c->big_list, c->big_count, a.tcol, a.tw, a.row_nnz);
+    scan_i64(c, a.row_nnz, a.out_indptr, a.n_rows_dev, 0, a.rows_cap, a.nnz_total_dev, s);
+}
+
+void reg_phase3(betty_ctx* c, const RegArgs& a, int32_t* col, int32_t* w, int64_t nnz_cap, cudaStream_t s) {
+    const int gw = (int)std::max<int64_t>(1, std::min<int64_t>((a.rows_cap * 32 + 255) / 256, (int64_t)c->num_sms * 16));
+    k_reg_compact<<<gw, 256, 0, s>>>(a.off, a.out_indptr, a.n_rows_dev, a.tcol, a.tw, col, w, nnz_cap);
+}
+
+}  // namespace betty

@@ -1,0 +1,35 @@
+// reg.h -- internal interface of the REG SpGEMM (reg.cu).
+#pragma once
+#include <stdint.h>
+#include <cuda_runtime.h>
+
+struct betty_ctx;
+namespace betty {
+
+struct RegArgs {
+    const int64_t* indptr;      // output block CSR (rows = outputs)
+    const int32_t* idx;         // full-batch src positions
+    const int64_t* n_rows_dev;  // device counts
+    const int64_t* n_cols_dev;
+    const int64_t* n_edges_dev;
+    int64_t rows_cap, cols_cap, edges_cap;
+    int64_t* t_indptr;          // [cols_cap+1]
+    int32_t* t_idx;             // [edges_cap]
+    int32_t* tcnt;              // [cols_cap]
+    int64_t* ub;                // [rows_cap]
+    int64_t* off;               // [rows_cap+1]
+    int64_t* ub_total_dev;
+    int32_t* tcol;              // [ub_cap]
+    int32_t* tw;                // [ub_cap]
+    int64_t* row_nnz;           // [rows_cap]
+    int64_t* out_indptr;        // [rows_cap+1]
+    int64_t* nnz_total_dev;
+};
+// phase 1: CSC + product counts (ub) + their scan (ub_total known after it)
+void reg_phase1(betty_ctx* c, const RegArgs& a, cudaStream_t s);
+// phase 2: expand / sort / RLE per row into tcol/tw (sized >= ub_total) + indptr scan
+void reg_phase2(betty_ctx* c, const RegArgs& a, cudaStream_t s);
+// phase 3: compaction into col/w (sized >= nnz_total)
+void reg_phase3(betty_ctx* c, const RegArgs& a, int32_t* col, int32_t* w, int64_t nnz_cap, cudaStream_t s);
+
+}  // namespace betty

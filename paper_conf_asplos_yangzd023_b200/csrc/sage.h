@@ -1,0 +1,78 @@
+// sage.h -- internal launchers of the SAGE forward/backward kernels.
+#pragma once
+#include <stdint.h>
+#include <cuda_runtime.h>
+
+struct betty_ctx;
+namespace betty {
+
+// ---- agg.cu
+void agg_mean_xa(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const int32_t* xrow, const int64_t* indptr,
+                 const int32_t* idx, const int64_t* cnt, int64_t rows_cap, int Fi, int Fp, void* XA, bool xa_bf16,
+                 int64_t ldxa, cudaStream_t s);
+void agg_mean_pf(betty_ctx* c, const float* Y, int64_t ldy, const int64_t* indptr, const int32_t* idx,
+                 const int64_t* cnt, int64_t rows_cap, int Fo, int Fop, bool relu, void* out, bool out_bf16,
+                 int64_t ldo, cudaStream_t s);
+void gather_ones(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const int32_t* xrow, const int64_t* cnt_rows,
+                 int64_t rows_cap, int Fi, void* out, bool out_bf16, int64_t ldo, cudaStream_t s);
+void csc_mean(betty_ctx* c, const float* dXA, int64_t ldd, const int64_t* indptr, const int64_t* t_indptr,
+              const int32_t* t_idx, const int64_t* cnt, int64_t src_cap, int Fi, int Fp, const void* H, bool h_bf16,
+              int64_t ldh, void* out, bool out_bf16, int64_t ldo, cudaStream_t s);
+void csc_pf(betty_ctx* c, const void* dS, bool ds_bf16, int64_t ldds, const int64_t* indptr, const int64_t* t_indptr,
+            const int32_t* t_idx, const int64_t* cnt, int64_t src_cap, int Fo, int Fop, void* G, bool g_bf16,
+            int64_t ldg, cudaStream_t s);
+void agg_pool(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const int32_t* xrow, const float* Zp, int64_t ldz,
+              const int64_t* indptr, const int32_t* idx, const int64_t* cnt, int64_t rows_cap, int Fi, int Fp,
+              void* XA, bool xa_bf16, int64_t ldxa, int32_t* arg, int64_t ldarg, cudaStream_t s);
+void route_pool(betty_ctx* c, const float* dXA, int64_t ldd, const int32_t* arg, int64_t ldarg,
+                const int64_t* t_indptr, const int32_t* t_idx, const int64_t* cnt, int64_t src_cap, int Fi, int Fp,
+                const float* Zp, int64_t ldz, void* out, bool out_bf16, int64_t ldo, cudaStream_t s);
+
+// ---- gemm.cu (dense layers; SIMT fp32 FFMA path, operands fp32 or bf16)
+enum { EPI_STORE = 0, EPI_RELU_ONES = 1, EPI_MASK = 2, EPI_RES_MASK = 3 };
+struct GemmRow {                 // C[m, n] = sum_k A[m, k] B(k, n), m < *M_dev
+    const void* A; int64_t lda; bool a_bf16;
+    const void* B; int64_t ldb; bool b_bf16; bool transB;   // B(k,n) = transB ? B[n*ldb+k] : B[k*ldb+n]
+    const int64_t* M_dev; int64_t M_cap; int K; int N;
+    void* C; int64_t ldc; bool c_bf16;
+    int epi;
+    const void* mask; int64_t ldm; bool m_bf16;           // EPI_MASK / EPI_RES_MASK: C *= [mask > 0]
+    const float* res; int64_t ldr; const int64_t* nres_dev; // EPI_RES_MASK: C += res (rows < *nres_dev)
+};
+void gemm_row(betty_ctx* c, const GemmRow& g, cudaStream_t s);
+
+// P[i, j] = sum_{r < *M_dev} A[r, i] B[r, j], i < K1, j < N, split over S row groups into
+// partials[S][K1][N]; then grad[map(i,j)] += sum_s partials[s][i][j] (fixed order: deterministic).
+enum { MAP_AGG = 0, MAP_PF = 1, MAP_POOL = 2 };
+struct GradMap {
+    int mode;
+    int Fi, Fo, Fp, Fop;
+    int64_t off_ws, off_wn, off_b, off_wp, off_bp;
+};
+struct GemmRed {
+    const void* A; int64_t lda; bool a_bf16;
+    const void* B; int64_t ldb; bool b_bf16;
+    const int64_t* M_dev; int64_t M_cap; int K1; int N;
+    float* partials; int S;
+    float* grad; GradMap map;
+};
+void gemm_red(betty_ctx* c, const GemmRed& g, cudaStream_t s);
+int gemm_red_splits(int64_t M_cap, int K1, int N);
+
+// ---- misc.cu
+void loss_ce(betty_ctx* c, const float* logits, int64_t ldl, const int32_t* labels, const int32_t* gid,
+             const int64_t* cnt, int64_t rows_cap, int C, float scale, float* dS, int64_t ldds, void* dS_act,
+             bool act_bf16, int64_t ld_act, float* loss_accum, cudaStream_t s);
+void adam(betty_ctx* c, float* p, float* g, float* m, float* v, int64_t n, int t, float lr, float b1, float b2,
+          float eps, bool zero_grad, cudaStream_t s);
+// per-layer GEMM weight layouts from the flat parameter vector
+struct PrepLayer {
+    int kind;                    // 0 agg-first [Ws;0;Wn;0;b] ((2Fp+1) x Fo, ld ldb), 1 project-first, 2 pool
+    int Fi, Fo, Fp, Fop;
+    int64_t off_ws, off_wn, off_b, off_wp, off_bp;
+    void* B; int64_t ldb;        // main weight in GEMM layout
+    void* Bp; int64_t ldbp;      // pool: [Wp; bp] ((Fi+1) x Fi)
+};
+void prep_weights(betty_ctx* c, const float* params, const PrepLayer* layers, int L, bool bf16, cudaStream_t s);
+
+}  // namespace betty

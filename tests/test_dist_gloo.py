@@ -1,0 +1,68 @@
+"""Multi-rank host logic on CPU (gloo, world_size 2): LPT assignment of
+micro-batches to ranks + one all-reduce of the accumulated gradient gives the
+full-batch gradient (the oracle computes each rank's share)."""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+import oracle
+import synth
+from paper_conf_asplos_yangzd023_b200.dist import allreduce_grad, lpt_assign, micro_batch_costs
+from tests.helpers import tiny
+
+DIMS = [6, 10, 4]
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _worker(rank, world, port, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    g, sd, blocks, feats, labels = tiny(n=300, pairs=1000, fanouts=(3, 4), n_out=40, F=6, C=4, seed=9)
+    K = 7
+    part = synth.random_partition(len(sd), K, 5)
+    mine = lpt_assign(micro_batch_costs(part, K, blocks[-1].indptr), world)[rank]
+    params = synth.init_params(DIMS, "mean", seed=1).astype(np.float64)
+    grad, loss = oracle.step(DIMS, "mean", False, blocks, part, K, mine, params, feats, labels, 1.0 / len(sd))
+    t = torch.tensor(np.concatenate([grad, [loss]]))
+    allreduce_grad(t)
+    if rank == 0:
+        full, lfull, _ = oracle.sage(DIMS, "mean", False, blocks, params, feats, labels, 1.0 / len(sd))
+        q.put((t.numpy(), full, lfull, mine))
+    dist.destroy_process_group()
+
+
+def test_lpt_assign_properties():
+    costs = [5, 1, 9, 3, 3, 7, 2]
+    a = lpt_assign(costs, 3)
+    assert sorted(k for r in a for k in r) == list(range(7))
+    loads = [sum(costs[k] for k in r) for r in a]
+    assert max(loads) - min(loads) <= max(costs)
+    assert lpt_assign(costs, 3) == a                       # deterministic
+    assert lpt_assign(costs, 1) == [list(range(7))]
+
+
+def test_two_rank_allreduce_equals_full_batch():
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    ps = [ctx.Process(target=_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in ps:
+        p.start()
+    red, full, lfull, mine = q.get(timeout=120)
+    for p in ps:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    assert np.linalg.norm(red[:-1] - full) <= 1e-12 * np.linalg.norm(full)
+    assert abs(red[-1] - lfull) <= 1e-12 * abs(lfull)

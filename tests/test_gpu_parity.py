@@ -1,0 +1,265 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle on the
+same seeded inputs.  Integer results (REG, blocks) bit-exact; floating point
+within DESIGN.md §3 reading #18 (rtol 1e-5 fp32 / 2e-2 bf16-GEMM mode)."""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import synth
+from tests.helpers import assert_close, load_golden, tiny
+
+pytestmark = pytest.mark.gpu
+
+RTOL = {"fp32": 1e-5, "bf16": 2e-2}
+
+
+@pytest.fixture(scope="module")
+def B():
+    import paper_conf_asplos_yangzd023_b200 as B
+    assert torch.cuda.is_available()
+    return B
+
+
+@pytest.fixture(scope="module")
+def ctx(B):
+    return B.betty_ctx_create(0)
+
+
+def golden_full():
+    g = load_golden("g1.json")
+    rows = [{int(k): v for k, v in g["rows"][str(l)].items()} for l in (0, 1)]
+    return g, synth.blocks_from_rows(g["seeds"], rows)
+
+
+def reg_equal(B, ctx, blk_dev, blk_host):
+    ip, col, w = B.betty_reg_build(ctx, blk_dev)
+    rp, rc, rw = oracle.reg(blk_host.n_src, blk_host.indptr, blk_host.nbr_pos)
+    np.testing.assert_array_equal(ip.cpu().numpy(), rp)
+    np.testing.assert_array_equal(col.cpu().numpy(), rc)
+    np.testing.assert_array_equal(w.cpu().numpy(), rw)
+    return len(rc)
+
+
+def blocks_equal(gpu, ora):
+    assert len(gpu) == len(ora)
+    for l, (a, b) in enumerate(zip(gpu, ora)):
+        assert (a.n_dst, a.n_src, a.n_edges) == (b.n_dst, b.n_src, b.n_edges), l
+        for name, x, y in [("indptr", a.indptr, b.indptr), ("indices", a.indices, b.indices),
+                           ("src_pos", a.src_pos, b.src_pos), ("src_gid", a.src_gid, b.src_gid),
+                           ("t_indptr", a.t_indptr, b.t_indptr), ("t_indices", a.t_indices, b.t_indices)]:
+            np.testing.assert_array_equal(x.cpu().numpy(), y, err_msg=f"layer {l} {name}")
+
+
+# ------------------------------------------------------------------ REG (a1)
+def test_reg_golden(B, ctx):
+    g, full = golden_full()
+    dev = B.blocks_to_device(full)
+    ip, col, w = B.betty_reg_build(ctx, dev[1])
+    assert ip.tolist() == g["reg"]["indptr"] and col.tolist() == g["reg"]["col"] and w.tolist() == g["reg"]["w"]
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_reg_random_small(B, ctx, seed):
+    g, sd, blocks, feats, labels = tiny(n=500, pairs=3000, fanouts=(4, 7), n_out=120, seed=seed)
+    reg_equal(B, ctx, B.blocks_to_device(blocks)[-1], blocks[-1])
+
+
+def test_reg_rejects_duplicate_edges(B, ctx):
+    blk = B.Block(2, 3, torch.tensor([0, 2, 3], dtype=torch.int64, device="cuda"),
+                  torch.tensor([1, 1, 2], dtype=torch.int32, device="cuda"),
+                  torch.arange(3, dtype=torch.int32, device="cuda"))
+    with pytest.raises(B.BettyError, match="EINVAL"):
+        B.betty_reg_build(ctx, blk)
+
+
+def test_reg_hub_rows_use_cta_path(B, ctx):
+    """Star + K_mn shapes: rows with > 256 candidate products (CTA bitonic path)."""
+    n, m = 400, 3
+    indptr = np.arange(n + 1, dtype=np.int64) * m
+    idx = np.tile(np.arange(m, dtype=np.int32), n)
+    host = synth.Block(n, m, indptr, idx, np.arange(m, dtype=np.int32))
+    reg_equal(B, ctx, B.blocks_to_device([host])[0], host)
+
+
+# ----------------------------------------------------------- extraction (a2)
+def test_extract_golden(B, ctx):
+    g, full = golden_full()
+    dev = B.blocks_to_device(full)
+    part = torch.tensor(g["part"], dtype=torch.int32, device="cuda")
+    for k in range(g["K"]):
+        mb = B.betty_extract_blocks(ctx, dev, part, g["K"], k)
+        blocks_equal(mb, oracle.extract(full, np.array(g["part"]), g["K"], k))
+
+
+@pytest.mark.parametrize("seed,K,fan", [(1, 1, (3, 4)), (2, 3, (2, 3, 4)), (3, 7, (3, 5)), (4, 40, (2, 2, 3))])
+def test_extract_random(B, ctx, seed, K, fan):
+    g, sd, blocks, feats, labels = tiny(n=400, pairs=1500, fanouts=fan, n_out=40, seed=seed)
+    part = synth.random_partition(len(sd), K, seed)       # K=40 leaves parts empty
+    dev = B.blocks_to_device(blocks)
+    dpart = torch.as_tensor(part).cuda()
+    for k in range(K):
+        blocks_equal(B.betty_extract_blocks(ctx, dev, dpart, K, k), oracle.extract(blocks, part, K, k))
+
+
+def test_extract_bad_input(B, ctx):
+    g, sd, blocks, feats, labels = tiny(seed=5)
+    dev = B.blocks_to_device(blocks)
+    part = torch.zeros(len(sd), dtype=torch.int32, device="cuda")
+    with pytest.raises(B.BettyError, match="EINVAL"):
+        B.betty_extract_blocks(ctx, dev, part, 2, 2)
+    part[3] = 9
+    with pytest.raises(B.BettyError, match="EINVAL"):
+        B.betty_extract_blocks(ctx, dev, part, 2, 0)
+
+
+# ------------------------------------------------------- SAGE fwd/bwd (a3-a6)
+CASES = [
+    dict(name="mean2", aggr="mean", fanouts=(3, 4), dims=[20, 32, 5]),
+    dict(name="mean2-wide", aggr="mean", fanouts=(5, 8), dims=[100, 256, 47]),
+    dict(name="mean3", aggr="mean", fanouts=(3, 3, 4), dims=[24, 40, 40, 6]),
+    dict(name="mean2-pf0", aggr="mean", fanouts=(3, 4), dims=[70, 16, 4]),
+    dict(name="pool2", aggr="pool", fanouts=(3, 4), dims=[16, 24, 5]),
+    dict(name="pool3", aggr="pool", fanouts=(2, 3, 3), dims=[12, 16, 16, 3]),
+]
+
+
+def make_case(c, seed=1, n=600, pairs=2400, n_out=60):
+    F = c["dims"][0]
+    ld = (F + 7) // 8 * 8
+    g, sd, blocks, feats, _ = tiny(n=n, pairs=pairs, fanouts=c["fanouts"], n_out=n_out, F=F, C=c["dims"][-1],
+                                   seed=seed, ld=ld)
+    labels = (np.arange(n) * 5 % c["dims"][-1]).astype(np.int32)
+    params = synth.init_params(c["dims"], c["aggr"], seed=seed)
+    return sd, blocks, feats, labels, params
+
+
+def dev_feats(feats, mode):
+    t = torch.as_tensor(feats).cuda()
+    return t.to(torch.bfloat16).contiguous() if mode == "bf16" else t
+
+
+@pytest.mark.parametrize("mode", ["fp32", "bf16"])
+@pytest.mark.parametrize("c", CASES, ids=lambda c: c["name"])
+def test_sage_micro_batch(B, ctx, c, mode):
+    sd, blocks, feats, labels, params = make_case(c)
+    K = 3
+    part = synth.random_partition(len(sd), K, 7)
+    dev = B.blocks_to_device(blocks)
+    dpart = torch.as_tensor(part).cuda()
+    model = B.Model(c["dims"], c["aggr"], mode, mode)
+    assert B.betty_num_params(model) == len(params)
+    P = torch.as_tensor(params).cuda()
+    X = dev_feats(feats, mode)
+    Y = torch.as_tensor(labels).cuda()
+    scale = 1.0 / len(sd)
+    for k in range(K):
+        mb = B.betty_extract_blocks(ctx, dev, dpart, K, k)
+        if mb[-1].n_dst == 0:
+            continue
+        saved, logits = B.betty_sage_fwd(ctx, model, P, mb, X)
+        grad = torch.zeros_like(P)
+        loss = torch.zeros(1, device="cuda")
+        B.betty_sage_bwd(ctx, model, P, mb, saved, Y, scale, grad, loss)
+        torch.cuda.synchronize()
+        om = oracle.extract(blocks, part, K, k)
+        og, ol, olog = oracle.sage(c["dims"], c["aggr"], mode == "bf16", om, params, feats, labels, scale,
+                                   want_logits=True)
+        assert_close(logits.cpu().numpy(), olog, RTOL[mode], f"logits k={k}")
+        assert_close(grad.cpu().numpy(), og, RTOL[mode], f"grad k={k}")
+        assert loss.item() == pytest.approx(ol, rel=RTOL[mode])
+        saved.free()
+
+
+@pytest.mark.parametrize("mode", ["fp32", "bf16"])
+@pytest.mark.parametrize("group", [1, 2, 0])
+@pytest.mark.parametrize("graph", [False, True])
+@pytest.mark.parametrize("c", [CASES[1], CASES[2], CASES[4]], ids=lambda c: c["name"])
+def test_step_matches_oracle(B, ctx, c, mode, group, graph):
+    """betty_step (fused extraction + fwd + loss + bwd + accumulation over a
+    rank's micro-batches) vs oracle_step, for several launch groupings."""
+    sd, blocks, feats, labels, params = make_case(c, seed=2)
+    K = 5
+    part = synth.random_partition(len(sd), K, 11)
+    ks = [0, 2, 3, 4]
+    dev = B.blocks_to_device(blocks)
+    dpart = torch.as_tensor(part).cuda()
+    model = B.Model(c["dims"], c["aggr"], mode, mode)
+    P = torch.as_tensor(params).cuda()
+    X = dev_feats(feats, mode)
+    Y = torch.as_tensor(labels).cuda()
+    scale = 1.0 / len(sd)
+    plan = B.betty_plan_create(ctx, model, dev, dpart, K, ks, group=group, flags=B.PLAN_GRAPH if graph else 0)
+    og, ol = oracle.step(c["dims"], c["aggr"], mode == "bf16", blocks, part, K, ks, params, feats, labels, scale)
+    for rep in range(2):             # replay: graph / arenas reused across steps
+        grad = torch.zeros_like(P)
+        loss = torch.zeros(1, device="cuda")
+        B.betty_step(ctx, plan, P, X, Y, scale, grad, loss)
+        B.betty_sync_check(ctx)
+        assert_close(grad.cpu().numpy(), og, RTOL[mode], f"grad rep={rep}")
+        assert loss.item() == pytest.approx(ol, rel=RTOL[mode])
+    info = plan.info()
+    assert info["kernels_per_step"] > 0
+    plan.free()
+
+
+def test_sum_of_micro_batches_equals_full_batch_on_gpu(B, ctx):
+    """Betty's invariant on the GPU path itself: K=8 step == K=1 step (fp32)."""
+    c = CASES[1]
+    sd, blocks, feats, labels, params = make_case(c, seed=3)
+    dev = B.blocks_to_device(blocks)
+    model = B.Model(c["dims"], "mean", "fp32")
+    P = torch.as_tensor(params).cuda()
+    X = dev_feats(feats, "fp32")
+    Y = torch.as_tensor(labels).cuda()
+    res = []
+    for K in (1, 8):
+        part = torch.as_tensor(synth.random_partition(len(sd), K, 1)).cuda()
+        plan = B.betty_plan_create(ctx, model, dev, part, K, list(range(K)), group=3)
+        grad = torch.zeros_like(P)
+        loss = torch.zeros(1, device="cuda")
+        B.betty_step(ctx, plan, P, X, Y, 1.0 / len(sd), grad, loss)
+        torch.cuda.synchronize()
+        res.append((grad.cpu().numpy(), loss.item()))
+        plan.free()
+    assert_close(res[1][0], res[0][0], 1e-5, "sum_k g_k vs g_full")
+    assert res[1][1] == pytest.approx(res[0][1], rel=1e-5)
+
+
+def test_adam_matches_torch(B, ctx):
+    n = 10007
+    g = torch.randn(n, device="cuda")
+    p0 = torch.randn(n, device="cuda")
+    p, m, v = p0.clone(), torch.zeros(n, device="cuda"), torch.zeros(n, device="cuda")
+    ref = p0.clone().requires_grad_(True)
+    opt = torch.optim.Adam([ref], lr=1e-3)
+    for t in range(1, 4):
+        B.betty_adam(ctx, p, g, m, v, t)
+        ref.grad = g.clone()
+        opt.step()
+    torch.cuda.synchronize()
+    torch.testing.assert_close(p, ref.detach(), rtol=1e-5, atol=1e-6)
+
+
+# --------------------------------------------- Cora-shaped config (C1) end to end
+def test_c1_cora_config(B, ctx):
+    cfg = synth.CONFIGS["C1"]
+    ds = synth.make(cfg)
+    reg_equal(B, ctx, B.blocks_to_device(ds.blocks)[-1], ds.blocks[-1])
+    part = synth.random_partition(cfg.n_out, 2, 3)
+    dev = B.blocks_to_device(ds.blocks)
+    dpart = torch.as_tensor(part).cuda()
+    for mode in ("fp32", "bf16"):
+        model = B.Model(cfg.dims, "mean", mode, mode)
+        params = synth.init_params(cfg.dims, "mean")
+        plan = B.betty_plan_create(ctx, model, dev, dpart, 2, [0, 1], group=1)
+        grad = torch.zeros(len(params), device="cuda")
+        loss = torch.zeros(1, device="cuda")
+        B.betty_step(ctx, plan, torch.as_tensor(params).cuda(), dev_feats(ds.feats, mode),
+                     torch.as_tensor(ds.labels).cuda(), 1.0 / cfg.n_out, grad, loss)
+        torch.cuda.synchronize()
+        og, ol = oracle.step(cfg.dims, "mean", mode == "bf16", ds.blocks, part, 2, [0, 1], params, ds.feats,
+                             ds.labels, 1.0 / cfg.n_out)
+        assert_close(grad.cpu().numpy(), og, RTOL[mode], f"C1 grad {mode}")
+        assert loss.item() == pytest.approx(ol, rel=RTOL[mode])
+        plan.free()

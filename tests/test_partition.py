@@ -1,0 +1,37 @@
+"""Host REG partitioner (outside the hot path; stands in for METIS, Alg. 1
+line 8): validity, balance, and that it cuts far less REG weight -- i.e.
+creates less input redundancy -- than a random partition (§4.3.2)."""
+import numpy as np
+import pytest
+
+import oracle
+import synth
+import paper_conf_asplos_yangzd023_b200 as B
+from tests.helpers import tiny
+
+
+def cut_weight(rp, col, w, part):
+    rows = np.repeat(np.arange(len(rp) - 1), np.diff(rp))
+    return int(w[part[rows] != part[col]].sum())
+
+
+@pytest.mark.parametrize("K", [1, 2, 5, 16])
+def test_partition_valid_balanced(K):
+    g, sd, blocks, feats, labels = tiny(n=3000, pairs=12000, fanouts=(4, 6), n_out=400, n_comm=20, mu=0.1, seed=2)
+    rp, col, w = oracle.reg(blocks[-1].n_src, blocks[-1].indptr, blocks[-1].nbr_pos)
+    part = B.betty_reg_partition(rp, col, w, K)
+    assert part.shape == (400,) and part.min() >= 0 and part.max() < K
+    sizes = np.bincount(part, minlength=K)
+    assert sizes.max() - sizes.min() <= 1
+    assert np.array_equal(part, B.betty_reg_partition(rp, col, w, K))   # deterministic
+
+
+def test_partition_reduces_redundancy_vs_random():
+    g, sd, blocks, feats, labels = tiny(n=3000, pairs=12000, fanouts=(4, 6), n_out=400, n_comm=20, mu=0.1, seed=3)
+    rp, col, w = oracle.reg(blocks[-1].n_src, blocks[-1].indptr, blocks[-1].nbr_pos)
+    K = 8
+    ours = B.betty_reg_partition(rp, col, w, K)
+    rnd = synth.random_partition(400, K, 1)
+    assert cut_weight(rp, col, w, ours) < 0.8 * cut_weight(rp, col, w, rnd)
+    red = [sum(oracle.extract(blocks, p, K, k)[0].n_src for k in range(K)) for p in (ours, rnd)]
+    assert red[0] < red[1]
