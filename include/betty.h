@@ -195,6 +195,17 @@ BETTY_API betty_status betty_step(betty_ctx* ctx, betty_plan* plan, const float*
 BETTY_API betty_status betty_adam(betty_ctx* ctx, float* params, float* grad, float* m, float* v, int64_t n, int32_t t,
                         float lr, float b1, float b2, float eps, int32_t zero_grad, betty_stream stream);
 
+/* Inspection hook (tests): run the extraction of launch group g of the plan
+ * and describe its group-concatenated blocks: the block-diagonal union of the
+ * group's micro-batches (my_k order) with ids global within the group -- the
+ * output layer lists each micro-batch's outputs in turn; every layer's src
+ * list is [its dst list] ++ [new sources of micro-batch 0] ++ [of 1] ++ ...
+ * (dst ids stay a prefix of src ids), and the next layer's dst list is that
+ * src list.  Arrays point INTO the plan's arenas (valid until the next step);
+ * sizes are host values (synchronises). */
+BETTY_API betty_status betty_plan_group_blocks(betty_ctx* ctx, betty_plan* plan, int32_t g, betty_block* out,
+                                               betty_stream stream);
+
 /* Measurement hook: bracket every launch of one kernel site with CUDA events
  * on the step's stream in subsequent betty_step calls (graph replays
  * included; changing the site re-captures the graph).  Sites: 0 off,

@@ -230,6 +230,22 @@ class Plan:
                 "n_dst": list(i.n_dst[:n]), "max_group_edges": list(i.max_group_edges[:n]), "reg_nnz": i.reg_nnz,
                 "arena_bytes": i.arena_bytes, "kernels_per_step": i.kernels_per_step}
 
+    def group_blocks(self, g: int) -> List[Block]:
+        """Extraction of launch group g (group-concatenated), copied out (tests)."""
+        out = (L.betty_block * len(self._keep[0]))()
+        self.ctx.check(L.lib().betty_plan_group_blocks(self.ctx.h, self.h, g, out, _stream(None)),
+                       "betty_plan_group_blocks")
+        d = self.ctx.device
+        res = []
+        for o in out:
+            res.append(Block(o.n_dst, o.n_src, _copy_out(o.indptr, o.n_dst + 1, torch.int64, d),
+                             _copy_out(o.indices, o.n_edges, torch.int32, d),
+                             _copy_out(o.src_gid, o.n_src, torch.int32, d),
+                             _copy_out(o.src_pos, o.n_src, torch.int32, d),
+                             _copy_out(o.t_indptr, o.n_src + 1, torch.int64, d) if o.t_indptr else None,
+                             _copy_out(o.t_indices, o.n_edges, torch.int32, d) if o.t_indptr else None))
+        return res
+
     def probe(self, site: int):
         """Bracket the launches of one kernel site with CUDA events (see betty.h)."""
         self.ctx.check(L.lib().betty_plan_probe(self.h, site), "betty_plan_probe")

@@ -473,6 +473,7 @@ struct betty_plan {
     betty_block reg_block{};
     // graph
     cudaGraphExec_t gexec = nullptr;
+    cudaStream_t cap_stream = nullptr;
     const void* key[9] = {};
     betty_plan_info info{};
     Probe probe;
@@ -667,6 +668,7 @@ extern "C" void betty_plan_destroy(betty_ctx* c, betty_plan* p) {
     if (!c || !p) return;
     cudaDeviceSynchronize();
     if (p->gexec) cudaGraphExecDestroy(p->gexec);
+    if (p->cap_stream) cudaStreamDestroy(p->cap_stream);
     p->probe.destroy();
     sage_free(c, &p->sb, 0);
     if (p->arena) { p->arena->s = 0; p->arena->release(); delete p->arena; }
@@ -690,13 +692,17 @@ extern "C" betty_status betty_step(betty_ctx* c, betty_plan* p, const float* par
     int32_t scbits;
     memcpy(&scbits, &sc, 4);
     const void* key[9] = {params, feats, (const void*)(intptr_t)ld_feats, labels, grad_accum, loss_accum,
-                          (const void*)(intptr_t)scbits, s, (const void*)(intptr_t)p->probe.site};
+                          (const void*)(intptr_t)scbits, nullptr, (const void*)(intptr_t)p->probe.site};
     if (!p->gexec || memcmp(key, p->key, sizeof key) != 0) {
         if (p->gexec) { cudaGraphExecDestroy(p->gexec); p->gexec = nullptr; }
+        // capture on a private stream (the caller's may be the legacy default
+        // stream, which cannot be captured); the graph is launched on `s`
+        if (!p->cap_stream) CUDA_OK(c, cudaStreamCreateWithFlags(&p->cap_stream, cudaStreamNonBlocking));
+        CUDA_OK(c, cudaStreamSynchronize(s));
         cudaGraph_t g;
-        CUDA_OK(c, cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal));
-        step_body(c, p, params, feats, ld_feats, labels, loss_scale, grad_accum, loss_accum, s);
-        CUDA_OK(c, cudaStreamEndCapture(s, &g));
+        CUDA_OK(c, cudaStreamBeginCapture(p->cap_stream, cudaStreamCaptureModeThreadLocal));
+        step_body(c, p, params, feats, ld_feats, labels, loss_scale, grad_accum, loss_accum, p->cap_stream);
+        CUDA_OK(c, cudaStreamEndCapture(p->cap_stream, &g));
         cudaError_t e = cudaGraphInstantiate(&p->gexec, g, 0);
         cudaGraphDestroy(g);
         if (e != cudaSuccess) return fail(c, BETTY_ECUDA, "graph instantiate: %s", cudaGetErrorString(e));
@@ -712,6 +718,27 @@ extern "C" betty_status betty_adam(betty_ctx* c, float* params, float* grad, flo
     if (!params || !grad || !m || !v || n < 0 || t < 1) return fail(c, BETTY_EINVAL, "adam: bad argument");
     adam(c, params, grad, m, v, n, t, lr, b1, b2, eps, zero_grad != 0, (cudaStream_t)stream);
     return check_launch(c);
+}
+
+extern "C" betty_status betty_plan_group_blocks(betty_ctx* c, betty_plan* p, int32_t g, betty_block* out,
+                                                betty_stream stream) {
+    if (!c || !p || !out || g < 0 || g >= (int32_t)p->groups.size()) return BETTY_EINVAL;
+    cudaStream_t s = (cudaStream_t)stream;
+    ExtractArgs a{};
+    a.L = p->L; a.full = p->full.data(); a.part = p->part; a.K = p->K;
+    a.ks = p->d_ks + g * p->c; a.c = (int32_t)p->groups[g].size();
+    a.layers = p->X.layers.data(); a.sc = p->X.sc; a.csc_mask = p->csc_mask;
+    extract_group(c, a, s);
+    std::vector<int64_t> h(4 * p->L);
+    cudaMemcpyAsync(h.data(), p->X.cnt_all, sizeof(int64_t) * 4 * p->L, cudaMemcpyDeviceToHost, s);
+    betty_status st = sync_check(c, s);
+    if (st) return st;
+    for (int l = 0; l < p->L; ++l) {
+        const ExtractLayer& B = p->X.layers[l];
+        out[l] = betty_block{h[4 * l], h[4 * l + 1], h[4 * l + 2], B.indptr, B.indices, B.src_pos, B.src_gid,
+                             B.t_indptr, B.t_indices};
+    }
+    return BETTY_OK;
 }
 
 extern "C" betty_status betty_plan_probe(betty_plan* p, int32_t site) {

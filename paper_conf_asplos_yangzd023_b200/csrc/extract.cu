@@ -17,6 +17,12 @@
 // the bitmap words -- no sort, no hash, no atomics-order dependence -- and a
 // new source's local id is n_dst + (#set bits before it).  Only dst nodes
 // need an explicit position -> local id map.  All sizes stay on the device.
+//
+// Group layout (what the SAGE kernels see): rows = the dst rows of all c
+// micro-batches; src ids = [all dst rows (same order)] ++ [new sources of
+// micro-batch 0] ++ [new of 1] ++ ..., so that dst ids remain a prefix of the
+// src ids (the self term of SAGE needs it).  Per micro-batch this is exactly
+// its canonical block under a renumbering; for c = 1 it IS the canonical block.
 #include "common.cuh"
 #include "internal.h"
 #include "extract.h"
@@ -101,7 +107,8 @@ __global__ void k_mark_dst(const int32_t* __restrict__ dst_pos, const int32_t* _
         const int j = row_mb[r];
         const int32_t p = dst_pos[r];
         atomicOr(&dstbits[j * W + (p >> 5)], 1u << (p & 31));
-        map[j * map_stride + p] = (int32_t)(r - mb_dst_off[j]);
+        map[j * map_stride + p] = (int32_t)r;           // dst rows are the group's src prefix: id = row
+        (void)mb_dst_off;
     }
 }
 
@@ -141,24 +148,26 @@ __global__ void k_counts(const int64_t* __restrict__ mb_dst_off, const int64_t* 
     __syncthreads();
     for (int j0 = 0; j0 < c; j0 += blockDim.x) {
         const int j = j0 + threadIdx.x;
-        int64_t ns = 0;
-        if (j < c) ns = (mb_dst_off[j + 1] - mb_dst_off[j]) + (wordoff[(int64_t)(j + 1) * W] - wordoff[(int64_t)j * W]);
+        int64_t nn = 0;                                 // new sources of micro-batch j
+        if (j < c) nn = wordoff[(int64_t)(j + 1) * W] - wordoff[(int64_t)j * W];
         int64_t tot;
-        const int64_t ex = block_excl_scan(ns, s_warp, &tot);
-        if (j < c) mb_src_off[j] = s_base + ex;
+        const int64_t ex = block_excl_scan(nn, s_warp, &tot);
+        if (j < c) mb_src_off[j] = s_base + ex;         // offset of j's new sources after the dst prefix
         __syncthreads();
         if (threadIdx.x == 0) s_base += tot;
         __syncthreads();
     }
     if (threadIdx.x == 0) {
+        (void)mb_dst_off;
         mb_src_off[c] = s_base;
-        cnt[1] = s_base;
-        if (s_base > cap_src || cnt[2] > cap_e) atomicOr(dev_err, DEVERR_OVERFLOW);
-        if (next_cnt) next_cnt[0] = s_base;
+        const int64_t ns = cnt[0] + s_base;
+        cnt[1] = ns;
+        if (ns > cap_src || cnt[2] > cap_e) atomicOr(dev_err, DEVERR_OVERFLOW);
+        if (next_cnt) next_cnt[0] = ns;
     }
 }
 
-__global__ void k_emit_new(const uint32_t* __restrict__ newbits, int64_t W, int32_t c,
+__global__ void k_emit_new(const uint32_t* __restrict__ newbits, int64_t W, int32_t c, const int64_t* n_dst_tot,
                            const int64_t* __restrict__ wordoff, const int64_t* __restrict__ mb_dst_off,
                            const int64_t* __restrict__ mb_src_off, const int32_t* __restrict__ fsrc_gid,
                            int32_t* __restrict__ src_pos, int32_t* __restrict__ src_gid, int32_t* __restrict__ src_mb,
@@ -169,7 +178,8 @@ __global__ void k_emit_new(const uint32_t* __restrict__ newbits, int64_t W, int3
         if (!bits) continue;
         const int j = (int)(i / W);
         const int64_t w = i - (int64_t)j * W;
-        int64_t s = mb_src_off[j] + (mb_dst_off[j + 1] - mb_dst_off[j]) + (wordoff[i] - wordoff[(int64_t)j * W]);
+        int64_t s = n_dst_tot[0] + mb_src_off[j] + (wordoff[i] - wordoff[(int64_t)j * W]);
+        (void)mb_dst_off;
         while (bits) {
             const int b = __ffs(bits) - 1;
             bits &= bits - 1;
@@ -188,7 +198,8 @@ __global__ void k_emit_dst(const int32_t* __restrict__ dst_pos, const int32_t* _
     const int64_t n = cnt[0];
     for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < n; r += (int64_t)gridDim.x * blockDim.x) {
         const int j = row_mb[r];
-        const int64_t s = mb_src_off[j] + (r - mb_dst_off[j]);
+        const int64_t s = r;                            // dst prefix keeps the row order
+        (void)mb_dst_off; (void)mb_src_off;
         const int32_t p = dst_pos[r];
         if (s < cap_src) { src_pos[s] = p; src_gid[s] = fsrc_gid[p]; src_mb[s] = j; }
     }
@@ -213,17 +224,17 @@ __global__ void k_relabel(const int32_t* __restrict__ dst_pos, const int32_t* __
         const uint32_t* nb = newbits + j * W;
         const int64_t* wo = wordoff + j * W;
         const int64_t wo0 = wo[0];
-        const int64_t nd = mb_dst_off[j + 1] - mb_dst_off[j];
-        const int64_t so = mb_src_off[j];
+        const int64_t so = cnt[0] + mb_src_off[j];      // j's new sources follow the whole dst prefix
+        (void)mb_dst_off;
         for (int64_t i = fb + lane; i < fe; i += 32) {
             const int32_t p = fnbr[i];
             const int32_t w = p >> 5;
             const uint32_t bit = 1u << (p & 31);
-            int64_t local;
-            if (db[w] & bit) local = map[j * map_stride + p];
-            else local = nd + (wo[w] - wo0) + __popc(nb[w] & (bit - 1));
+            int64_t id;                                 // src id, global within the group
+            if (db[w] & bit) id = map[j * map_stride + p];
+            else id = so + (wo[w] - wo0) + __popc(nb[w] & (bit - 1));
             const int64_t o = ob + (i - fb);
-            if (o < cap_e) indices[o] = (int32_t)(so + local);
+            if (o < cap_e) indices[o] = (int32_t)id;
         }
     }
 }
@@ -284,7 +295,7 @@ void extract_group(betty_ctx* ctx, const ExtractArgs& a, cudaStream_t s) {
                                     l > 0 ? a.layers[l - 1].cnt : nullptr, ctx->dev_err);
         k_emit_dst<<<grid_for(ctx, cap_d, 256), 256, 0, s>>>(dst_pos, row_mb, B.cnt, dst_off, B.mb_src_off,
                                                              F.src_gid, B.src_pos, B.src_gid, B.src_mb, cap_s);
-        k_emit_new<<<grid_for(ctx, cW, 256), 256, 0, s>>>(a.sc.newbits, W, c, a.sc.wordoff, dst_off, B.mb_src_off,
+        k_emit_new<<<grid_for(ctx, cW, 256), 256, 0, s>>>(a.sc.newbits, W, c, B.cnt, a.sc.wordoff, dst_off, B.mb_src_off,
                                                           F.src_gid, B.src_pos, B.src_gid, B.src_mb, cap_s);
         k_relabel<<<grid_for(ctx, cap_d * 32, 256), 256, 0, s>>>(dst_pos, row_mb, B.cnt, F.indptr, F.nbr, B.indptr,
                                                                  a.sc.dstbits, a.sc.newbits, a.sc.wordoff, W, a.sc.map,

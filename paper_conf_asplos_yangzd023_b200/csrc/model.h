@@ -71,11 +71,11 @@ struct Probe {
             ev.push_back(a);
             ev.push_back(b);
         }
-        cudaEventRecord(ev[2 * used], s);
+        cudaEventRecordWithFlags(ev[2 * used], s, cudaEventRecordExternal);  // a real node when captured
     }
     void end(int here, cudaStream_t s) {
         if (site != here) return;
-        cudaEventRecord(ev[2 * used + 1], s);
+        cudaEventRecordWithFlags(ev[2 * used + 1], s, cudaEventRecordExternal);
         ++used;
     }
     void destroy() { for (auto e : ev) cudaEventDestroy(e); ev.clear(); used = 0; }

@@ -102,6 +102,69 @@ def test_extract_random(B, ctx, seed, K, fan):
         blocks_equal(B.betty_extract_blocks(ctx, dev, dpart, K, k), oracle.extract(blocks, part, K, k))
 
 
+def concat_oracle(blocks, part, K, ks):
+    """The layout of a launch group: the block-diagonal union
+    of the oracle's micro-batches ks with the dst rows of ALL of them first
+    (so dst ids stay a prefix of src ids), then each micro-batch's new
+    sources in micro-batch order; the output layer lists the micro-batches'
+    outputs in order; a layer's dst list is the src list of the layer above."""
+    mbs = [oracle.extract(blocks, part, K, k) for k in ks]
+    L = len(blocks)
+    D = [(j, t) for j, mb in enumerate(mbs) for t in range(mb[L - 1].n_dst)]
+    out = [None] * L
+    for l in range(L - 1, -1, -1):
+        gid = {jt: r for r, jt in enumerate(D)}
+        S = list(D)
+        for j, mb in enumerate(mbs):
+            for t in range(mb[l].n_dst, mb[l].n_src):
+                gid[(j, t)] = len(S)
+                S.append((j, t))
+        indptr, idx = [0], []
+        for (j, t) in D:
+            b = mbs[j][l]
+            idx += [gid[(j, int(u))] for u in b.indices[b.indptr[t]:b.indptr[t + 1]]]
+            indptr.append(len(idx))
+        cols = [[] for _ in S]
+        for r in range(len(D)):
+            for e in range(indptr[r], indptr[r + 1]):
+                cols[idx[e]].append(r)
+        t_indptr = np.cumsum([0] + [len(c) for c in cols]).astype(np.int64)
+        t_idx = np.array([r for c in cols for r in c], dtype=np.int32)
+        out[l] = oracle.MBlock(len(D), len(S), np.array(indptr, np.int64), np.array(idx, np.int32),
+                               np.array([mbs[j][l].src_pos[t] for j, t in S], np.int32),
+                               np.array([mbs[j][l].src_gid[t] for j, t in S], np.int32), t_indptr, t_idx)
+        D = S
+    return out
+
+
+@pytest.mark.parametrize("group", [1, 2, 3, 0])
+def test_group_extraction(B, ctx, group):
+    """The fused step's extraction of a launch group == the block-diagonal
+    union of the oracle's micro-batches (bit-exact)."""
+    g, sd, blocks, feats, labels = tiny(n=500, pairs=2000, fanouts=(3, 4, 5), n_out=50, seed=8)
+    K = 6
+    part = synth.random_partition(len(sd), K, 2)
+    ks = [5, 0, 2, 3, 4]
+    dev = B.blocks_to_device(blocks)
+    dpart = torch.as_tensor(part).cuda()
+    model = B.Model([8, 12, 12, 3], "mean", "fp32")
+    plan = B.betty_plan_create(ctx, model, dev, dpart, K, ks, group=group, flags=0)
+    c = len(ks) if group == 0 else group
+    groups = [ks[i:i + c] for i in range(0, len(ks), c)]
+    for gi, gk in enumerate(groups):
+        got = plan.group_blocks(gi)
+        want = concat_oracle(blocks, part, K, gk)
+        for l, (a, b) in enumerate(zip(got, want)):
+            assert (a.n_dst, a.n_src, a.n_edges) == (b.n_dst, b.n_src, b.n_edges), (gi, l)
+            for name in ("indptr", "indices", "src_pos", "src_gid"):
+                np.testing.assert_array_equal(getattr(a, name).cpu().numpy(), getattr(b, name),
+                                              err_msg=f"group {gi} layer {l} {name}")
+            if a.t_indptr is not None:
+                np.testing.assert_array_equal(a.t_indptr.cpu().numpy(), b.t_indptr, err_msg=f"g{gi} l{l} t_indptr")
+                np.testing.assert_array_equal(a.t_indices.cpu().numpy(), b.t_indices, err_msg=f"g{gi} l{l} t_idx")
+    plan.free()
+
+
 def test_extract_bad_input(B, ctx):
     g, sd, blocks, feats, labels = tiny(seed=5)
     dev = B.blocks_to_device(blocks)
