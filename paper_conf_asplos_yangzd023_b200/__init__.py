@@ -296,6 +296,21 @@ def betty_adam(ctx: Context, params: torch.Tensor, grad: torch.Tensor, m: torch.
                                  int(zero_grad), _stream(stream)), "betty_adam")
 
 
+def betty_test_gemm(ctx: Context, kind: int, A: torch.Tensor, B: torch.Tensor, K: int, N: int, use_tc: bool = True,
+                    M: Optional[int] = None, stream=None) -> torch.Tensor:
+    """Test hook of the dense kernels.  kind 0: A[M,K] @ B[N,K]^T; kind 1: A[M,K]^T @ B[M,N]."""
+    M = A.shape[0] if M is None else M
+    if kind == 0:
+        C = torch.zeros((M, N), dtype=torch.float32, device=A.device)
+        ldc = N
+    else:
+        C = torch.zeros((K, N), dtype=torch.float32, device=A.device)
+        ldc = N
+    ctx.check(L.lib().betty_test_gemm(ctx.h, kind, _p(A), A.stride(0), _p(B), B.stride(0), M, A.shape[0], K, N,
+                                      _p(C), ldc, int(use_tc), _stream(stream)), "betty_test_gemm")
+    return C
+
+
 def betty_sync_check(ctx: Context, stream=None):
     ctx.check(L.lib().betty_sync_check(ctx.h, _stream(stream)), "betty_sync_check")
 

@@ -93,6 +93,8 @@ extern "C" betty_status betty_ctx_create(int device, betty_alloc_fn alloc, betty
     if (cudaMalloc(&c->big_list, sizeof(int64_t) * c->big_list_cap) != cudaSuccess) { delete c; return BETTY_ENOMEM; }
     cudaMemset(c->counters, 0, 64 * 4 + 512 * 8);
     init_kernel_attrs();
+    const char* no_tc = getenv("BETTY_NO_TC");
+    c->use_tc = !(no_tc && no_tc[0] == '1') && tc_available();
     cudaMemset(c->dev_err, 0, 16);
     cudaMemset(c->big_count, 0, 16);
     cudaDeviceSynchronize();
@@ -739,6 +741,44 @@ extern "C" betty_status betty_plan_group_blocks(betty_ctx* c, betty_plan* p, int
                              B.t_indptr, B.t_indices};
     }
     return BETTY_OK;
+}
+
+// ------------------------------------------------- GEMM test hooks (bf16)
+extern "C" betty_status betty_test_gemm(betty_ctx* c, int32_t kind, const void* A, int64_t lda, const void* B,
+                                        int64_t ldb, int64_t M, int64_t M_cap, int32_t K, int32_t N, float* C,
+                                        int64_t ldc, int32_t use_tc, betty_stream stream) {
+    if (!c || !A || !B || !C || M < 0 || M_cap < M || K < 1 || N < 1) return BETTY_EINVAL;
+    cudaStream_t s = (cudaStream_t)stream;
+    int64_t* Md = (int64_t*)ctx_alloc(c, 8, s);
+    cudaMemcpyAsync(Md, &M, 8, cudaMemcpyHostToDevice, s);
+    const bool saved = c->use_tc;
+    c->use_tc = use_tc && tc_available();
+    betty_status st = BETTY_OK;
+    if (kind == 0) {            // C[M x N] = A[M x K] . B, B given as [N x K] (K-major)
+        GemmRow g{};
+        g.A = A; g.lda = lda; g.a_bf16 = true;
+        g.B = B; g.ldb = ldb; g.b_bf16 = true; g.transB = true;
+        g.M_dev = Md; g.M_cap = std::max<int64_t>(M_cap, 1); g.K = K; g.N = N;
+        g.C = C; g.ldc = ldc; g.c_bf16 = false; g.epi = EPI_STORE;
+        gemm_row(c, g, s);
+    } else {                    // C[K x N] = A[M x K]^T . B[M x N]  (C zero-initialised by the caller: it ADDS)
+        int64_t S = gemm_red_splits(M_cap, K, N);
+        float* part = (float*)ctx_alloc(c, sizeof(float) * S * K * N, s);
+        GemmRed r{};
+        r.A = A; r.lda = lda; r.a_bf16 = true;
+        r.B = B; r.ldb = ldb; r.b_bf16 = true;
+        r.M_dev = Md; r.M_cap = std::max<int64_t>(M_cap, 1); r.K1 = K; r.N = N;
+        r.partials = part; r.S = (int)S; r.grad = C;
+        r.map = GradMap{MAP_AGG, K, N, K, N, 0, 0, 0, 0, 0};   // identity: rows < K -> off_ws + i*N + j
+        r.map.Fp = 1 << 29;                                     // no neighbour / bias rows
+        gemm_red(c, r, s);
+        ctx_free(c, part, s);
+        (void)ldc;
+    }
+    c->use_tc = saved;
+    ctx_free(c, Md, s);
+    st = sync_check(c, s);
+    return st;
 }
 
 extern "C" betty_status betty_plan_probe(betty_plan* p, int32_t site) {

@@ -123,6 +123,11 @@ static void launch_row(betty_ctx* c, const GemmRow& g, cudaStream_t s) {
 }
 
 void gemm_row(betty_ctx* c, const GemmRow& g, cudaStream_t s) {
+    if (c->use_tc && g.a_bf16 && g.b_bf16) {
+        const void* Bk = g.transB ? g.B : g.Bt;
+        const int64_t ldbk = g.transB ? g.ldb : g.ldbt;
+        if (Bk && gemm_row_tc(c, g, Bk, ldbk, s)) return;
+    }
     if (g.a_bf16) {
         if (g.b_bf16) launch_row<__nv_bfloat16, __nv_bfloat16>(c, g, s);
         else launch_row<__nv_bfloat16, float>(c, g, s);
@@ -241,13 +246,22 @@ __global__ void k_red_final(const float* __restrict__ partials, int S, int K1, i
 }
 
 int gemm_red_splits(int64_t M_cap, int K1, int N) {
+    // the same split count serves the SIMT path (tiles of 64 x 64) and the tensor-core path
+    // (M tiles of 128 features, one CTA per SM): enough CTAs for either, never more than row chunks
     const int tiles = ((K1 + XB - 1) / XB) * ((N + XB - 1) / XB);
+    const int mtiles = (K1 + 127) / 128;
     const int64_t chunks = std::max<int64_t>(1, (M_cap + XCHUNK - 1) / XCHUNK);
-    const int want = std::max(1, (148 * 4) / tiles);
+    const int want = std::max(std::max(1, (148 * 4) / tiles), std::max(1, 148 / mtiles));
     return (int)std::max<int64_t>(1, std::min<int64_t>(chunks, want));
 }
 
 void gemm_red(betty_ctx* c, const GemmRed& g, cudaStream_t s) {
+    if (c->use_tc && g.a_bf16 && g.b_bf16 && gemm_red_tc(c, g, s)) {
+        const int64_t n = (int64_t)g.K1 * g.N;
+        const int gf = (int)std::max<int64_t>(1, std::min<int64_t>((n + 255) / 256, (int64_t)c->num_sms * 4));
+        k_red_final<<<gf, 256, 0, s>>>(g.partials, g.S, g.K1, g.N, g.grad, g.map);
+        return;
+    }
     const int tiles = ((g.K1 + XB - 1) / XB) * ((g.N + XB - 1) / XB);
     const int grid = tiles * g.S;
     if (g.a_bf16) {

@@ -9,6 +9,7 @@
 struct betty_ctx {
     int device = 0;
     int num_sms = 148;
+    bool use_tc = true;                          // tcgen05 GEMMs in BF16 mode (env BETTY_NO_TC=1 disables)
     betty_alloc_fn alloc = nullptr;
     betty_free_fn dealloc = nullptr;
     void* user = nullptr;

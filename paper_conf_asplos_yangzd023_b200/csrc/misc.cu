@@ -147,6 +147,7 @@ __global__ void k_prep(const float* __restrict__ params, PrepArgs a) {
                 else if (i == 2 * P.Fp) v = params[P.off_b + j];
             }
             st_act(B + t, v);
+            if (P.Bt && j < P.ldbt_rows) st_act((T*)P.Bt + (int64_t)j * P.ldbt + i, v);   // K-major copy
         }
         if (P.kind == 2) {
             T* Bp = (T*)P.Bp;
@@ -156,6 +157,7 @@ __global__ void k_prep(const float* __restrict__ params, PrepArgs a) {
                 float v = 0.f;
                 if (j < P.Fi) v = (i < P.Fi) ? params[P.off_wp + (int64_t)i * P.Fi + j] : params[P.off_bp + j];
                 st_act(Bp + t, v);
+                if (P.Bpt && j < P.Fi) st_act((T*)P.Bpt + (int64_t)j * P.ldbpt + i, v);
             }
         }
     }

@@ -52,6 +52,8 @@ struct LayerBufs {
     void* H = nullptr;    // input of layer l (l >= 1), written by layer l-1
     void* dS = nullptr;   // dS of layer l as GEMM operand (l < L-1)
     void* B = nullptr;    void* Bp = nullptr;
+    void* Bt = nullptr;   void* Bpt = nullptr;   // K-major weight copies (BF16 tensor-core path)
+    int64_t ldbt = 0, ldbpt = 0;
     int S_main = 1, S_pool = 1;   // split counts of the dW reductions
 };
 
@@ -71,12 +73,19 @@ struct Probe {
             ev.push_back(a);
             ev.push_back(b);
         }
-        cudaEventRecordWithFlags(ev[2 * used], s, cudaEventRecordExternal);  // a real node when captured
+        rec(ev[2 * used], s);
     }
     void end(int here, cudaStream_t s) {
         if (site != here) return;
-        cudaEventRecordWithFlags(ev[2 * used + 1], s, cudaEventRecordExternal);
+        rec(ev[2 * used + 1], s);
         ++used;
+    }
+    static void rec(cudaEvent_t e, cudaStream_t s) {
+        cudaStreamCaptureStatus st = cudaStreamCaptureStatusNone;
+        cudaStreamIsCapturing(s, &st);
+        // inside a capture the record must be an external event node to be timeable
+        if (st == cudaStreamCaptureStatusActive) cudaEventRecordWithFlags(e, s, cudaEventRecordExternal);
+        else cudaEventRecord(e, s);
     }
     void destroy() { for (auto e : ev) cudaEventDestroy(e); ev.clear(); used = 0; }
 };

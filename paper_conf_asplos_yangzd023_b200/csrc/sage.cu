@@ -111,6 +111,15 @@ bool sage_alloc(betty_ctx* c, const ModelCfg& m, const std::vector<int64_t>& cap
             B.S_pool = gemm_red_splits(ns, L.Fi + 1, L.Fi);
             part_max = std::max<int64_t>(part_max, (int64_t)B.S_pool * (L.Fi + 1) * L.Fi);
         }
+        if (m.bf16) {                // K-major (transposed) weights for the tcgen05 forward GEMMs
+            const int64_t krows = L.kind == KIND_PF ? (L.Fi + 1) : (2 * L.Fp + 1);
+            B.ldbt = r8(krows);
+            B.Bt = A(L.ld_B * B.ldbt * ea);
+            if (L.kind == KIND_POOL) {
+                B.ldbpt = r8(L.Fi + 1);
+                B.Bpt = A((int64_t)L.ld_Bp * B.ldbpt * ea);
+            }
+        }
         if (l >= 1) B.H = A(ns * m.layers[l - 1].ld_out * ea);
         if (!L.last) B.dS = A(nd * L.ld_ds * ea);
         if (L.last) {
@@ -140,6 +149,8 @@ void sage_prep(betty_ctx* c, const ModelCfg& m, SageBufs& b, const float* params
         p.off_ws = L.off_ws; p.off_wn = L.off_wn; p.off_b = L.off_b; p.off_wp = L.off_wp; p.off_bp = L.off_bp;
         p.B = b.l[l].B; p.ldb = L.ld_B;
         p.Bp = b.l[l].Bp; p.ldbp = L.ld_Bp;
+        p.Bt = b.l[l].Bt; p.ldbt = b.l[l].ldbt; p.ldbt_rows = L.ld_B;
+        p.Bpt = b.l[l].Bpt; p.ldbpt = b.l[l].ldbpt;
     }
     prep_weights(c, params, P.data(), m.L, m.bf16, s);
 }
@@ -184,6 +195,7 @@ void sage_forward(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView*
             g.A = Ao; g.lda = ldao; g.a_bf16 = m.bf16;
             g.B = B.B; g.ldb = L.ld_B; g.b_bf16 = m.bf16; g.transB = false;
             g.M_dev = V.cnt + 1; g.M_cap = V.cap_src; g.K = L.Fi + 1; g.N = 2 * L.Fop;
+            g.Bt = B.Bt; g.ldbt = B.ldbt;
             g.C = B.Y; g.ldc = L.ld_y; g.c_bf16 = false; g.epi = EPI_STORE;
             PB(l == 0 ? PROBE_GEMM_FWD_L0 : PROBE_GEMM_FWD_L1);
             gemm_row(c, g, s);
@@ -199,6 +211,7 @@ void sage_forward(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView*
             g.A = Ao; g.lda = ldao; g.a_bf16 = m.bf16;
             g.B = B.Bp; g.ldb = L.ld_Bp; g.b_bf16 = m.bf16;
             g.M_dev = V.cnt + 1; g.M_cap = V.cap_src; g.K = L.Fi + 1; g.N = L.Fi;
+            g.Bt = B.Bpt; g.ldbt = B.ldbpt;
             g.C = B.Zp; g.ldc = L.ld_zp; g.c_bf16 = false; g.epi = EPI_STORE;
             gemm_row(c, g, s);
             PB(l == 0 ? PROBE_AGG_L0 : PROBE_AGG_L1);
@@ -215,6 +228,7 @@ void sage_forward(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView*
         g.A = B.XA; g.lda = L.ld_xa; g.a_bf16 = m.bf16;
         g.B = B.B; g.ldb = L.ld_B; g.b_bf16 = m.bf16;
         g.M_dev = V.cnt + 0; g.M_cap = V.cap_dst; g.K = 2 * L.Fp + 1; g.N = L.Fo;
+        g.Bt = B.Bt; g.ldbt = B.ldbt;
         g.C = out; g.ldc = L.ld_out; g.c_bf16 = out_bf; g.epi = epi;
         PB(l == 0 ? PROBE_GEMM_FWD_L0 : PROBE_GEMM_FWD_L1);
         gemm_row(c, g, s);

@@ -38,8 +38,12 @@ struct GemmRow {                 // C[m, n] = sum_k A[m, k] B(k, n), m < *M_dev
     int epi;
     const void* mask; int64_t ldm; bool m_bf16;           // EPI_MASK / EPI_RES_MASK: C *= [mask > 0]
     const float* res; int64_t ldr; const int64_t* nres_dev; // EPI_RES_MASK: C += res (rows < *nres_dev)
+    const void* Bt; int64_t ldbt;                          // K-major copy of B (N x K) for the tensor-core path
 };
 void gemm_row(betty_ctx* c, const GemmRow& g, cudaStream_t s);
+// gemm_tc.cu: tcgen05 paths (false = shape not supported, caller falls back to SIMT)
+bool tc_available();
+bool gemm_row_tc(betty_ctx* c, const GemmRow& g, const void* Bk, int64_t ldbk, cudaStream_t s);
 
 // P[i, j] = sum_{r < *M_dev} A[r, i] B[r, j], i < K1, j < N, split over S row groups into
 // partials[S][K1][N]; then grad[map(i,j)] += sum_s partials[s][i][j] (fixed order: deterministic).
@@ -58,6 +62,7 @@ struct GemmRed {
 };
 void gemm_red(betty_ctx* c, const GemmRed& g, cudaStream_t s);
 int gemm_red_splits(int64_t M_cap, int K1, int N);
+bool gemm_red_tc(betty_ctx* c, const GemmRed& g, cudaStream_t s);
 
 // ---- misc.cu
 void loss_ce(betty_ctx* c, const float* logits, int64_t ldl, const int32_t* labels, const int32_t* gid,
@@ -72,6 +77,9 @@ struct PrepLayer {
     int64_t off_ws, off_wn, off_b, off_wp, off_bp;
     void* B; int64_t ldb;        // main weight in GEMM layout
     void* Bp; int64_t ldbp;      // pool: [Wp; bp] ((Fi+1) x Fi)
+    void* Bt; int64_t ldbt;      // K-major (transposed) copies for the tensor-core path (may be null)
+    int64_t ldbt_rows;           // rows of Bt (= columns of B that are written)
+    void* Bpt; int64_t ldbpt;
 };
 void prep_weights(betty_ctx* c, const float* params, const PrepLayer* layers, int L, bool bf16, cudaStream_t s);
 
