@@ -23,53 +23,65 @@ template <typename T> __device__ __forceinline__ const T* row_ptr(const T* X, in
 }
 
 // ------------------------------------------------ mean, aggregate-first fwd
-template <typename Tin, typename Tout>
+// LPR lanes own one dst row (RPW = 32/LPR rows per warp in flight); each lane
+// covers 16-byte vectors of the feature row.  The neighbour X-row of edge e is
+// emap ? emap[erow[e]] : erow[e] (layer 0 passes the edge -> global-id array
+// written by the extraction, so no dependent id lookup stays on the critical
+// path); the self row of dst v is srow ? srow[v] : v.
+template <typename Tin, typename Tout, int LPR>
 __global__ void __launch_bounds__(256) k_agg_mean_xa(const Tin* __restrict__ X, int64_t ldx,
-                                                     const int32_t* __restrict__ xrow,
-                                                     const int64_t* __restrict__ indptr,
-                                                     const int32_t* __restrict__ idx, const int64_t* cnt, int Fi,
+                                                     const int32_t* __restrict__ srow,
+                                                     const int32_t* __restrict__ erow,
+                                                     const int32_t* __restrict__ emap,
+                                                     const int64_t* __restrict__ indptr, const int64_t* cnt, int Fi,
                                                      int Fp, Tout* __restrict__ XA, int64_t ldxa) {
     using VI = Vec<Tin>;
     constexpr int VW = VI::N;
+    constexpr int RPW = 32 / LPR;
     const int64_t nd = cnt[0];
     const int NV = (Fi + VW - 1) / VW;
-    const int lane = lane_id();
+    const int lane = lane_id(), sub = lane % LPR, grp = lane / LPR;
+    const unsigned gmask = LPR == 32 ? 0xffffffffu : (((1u << LPR) - 1u) << (grp * LPR));
     const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    for (int64_t v = gw; v < nd; v += nw) {
-        const int64_t b = indptr[v], e = indptr[v + 1];
+    for (int64_t v0 = gw * RPW; v0 < nd; v0 += nw * RPW) {
+        const int64_t v = v0 + grp;
+        const bool rowok = v < nd;
+        int64_t b = 0, e = 0;
+        if (rowok) { b = indptr[v]; e = indptr[v + 1]; }
         const float inv = e > b ? 1.0f / (float)(e - b) : 0.0f;
         Tout* out = XA + v * ldxa;
-        for (int vb = 0; vb < NV; vb += 32) {
-            const int vi = vb + lane;
-            const bool act = vi < NV;
+        for (int vb = 0; vb < NV; vb += LPR) {
+            const int vi = vb + sub;
+            const bool act = rowok && vi < NV;
             float acc[VW];
 #pragma unroll
             for (int t = 0; t < VW; ++t) acc[t] = 0.f;
-            for (int64_t e0 = b; e0 < e; e0 += 32) {
-                const int n = (int)mn64(32, e - e0);
-                const int32_t my = lane < n ? idx[e0 + lane] : 0;
+            for (int64_t e0 = b; e0 < e; e0 += LPR) {
+                const int n = (int)mn64(LPR, e - e0);
+                int32_t my = 0;
+                if (sub < n) { my = erow[e0 + sub]; if (emap) my = emap[my]; }
                 int j = 0;
                 for (; j + 4 <= n; j += 4) {
-                    VI x0, x1, x2, x3;
-                    const int32_t u0 = __shfl_sync(0xffffffffu, my, j);
-                    const int32_t u1 = __shfl_sync(0xffffffffu, my, j + 1);
-                    const int32_t u2 = __shfl_sync(0xffffffffu, my, j + 2);
-                    const int32_t u3 = __shfl_sync(0xffffffffu, my, j + 3);
+                    const int32_t u0 = __shfl_sync(gmask, my, j, LPR);
+                    const int32_t u1 = __shfl_sync(gmask, my, j + 1, LPR);
+                    const int32_t u2 = __shfl_sync(gmask, my, j + 2, LPR);
+                    const int32_t u3 = __shfl_sync(gmask, my, j + 3, LPR);
                     if (act) {
-                        x0.load(row_ptr(X, ldx, xrow, u0) + vi * VW);
-                        x1.load(row_ptr(X, ldx, xrow, u1) + vi * VW);
-                        x2.load(row_ptr(X, ldx, xrow, u2) + vi * VW);
-                        x3.load(row_ptr(X, ldx, xrow, u3) + vi * VW);
+                        VI x0, x1, x2, x3;
+                        x0.load(X + (int64_t)u0 * ldx + vi * VW);
+                        x1.load(X + (int64_t)u1 * ldx + vi * VW);
+                        x2.load(X + (int64_t)u2 * ldx + vi * VW);
+                        x3.load(X + (int64_t)u3 * ldx + vi * VW);
 #pragma unroll
                         for (int t = 0; t < VW; ++t) acc[t] += (x0.v[t] + x1.v[t]) + (x2.v[t] + x3.v[t]);
                     }
                 }
                 for (; j < n; ++j) {
-                    const int32_t u = __shfl_sync(0xffffffffu, my, j);
+                    const int32_t u = __shfl_sync(gmask, my, j, LPR);
                     if (act) {
                         VI x;
-                        x.load(row_ptr(X, ldx, xrow, u) + vi * VW);
+                        x.load(X + (int64_t)u * ldx + vi * VW);
 #pragma unroll
                         for (int t = 0; t < VW; ++t) acc[t] += x.v[t];
                     }
@@ -77,20 +89,31 @@ __global__ void __launch_bounds__(256) k_agg_mean_xa(const Tin* __restrict__ X, 
             }
             if (act) {
                 VI self;
-                self.load(row_ptr(X, ldx, xrow, v) + vi * VW);
+                self.load(X + (int64_t)(srow ? srow[v] : (int32_t)v) * ldx + vi * VW);
+                if constexpr (sizeof(Tin) == sizeof(Tout)) {
+                    Vec<Tout> so, ao;
 #pragma unroll
-                for (int t = 0; t < VW; ++t) {
-                    const int col = vi * VW + t;
-                    if (col < Fi) {
-                        st_act(out + col, self.v[t]);
-                        st_act(out + Fp + col, acc[t] * inv);
+                    for (int t = 0; t < VW; ++t) {
+                        const bool in = vi * VW + t < Fi;
+                        so.v[t] = in ? self.v[t] : 0.f;
+                        ao.v[t] = in ? acc[t] * inv : 0.f;
+                    }
+                    so.store(out + vi * VW);
+                    ao.store(out + Fp + vi * VW);
+                } else {
+#pragma unroll
+                    for (int t = 0; t < VW; ++t) {
+                        const int col = vi * VW + t;
+                        if (col < Fi) { st_act(out + col, self.v[t]); st_act(out + Fp + col, acc[t] * inv); }
                     }
                 }
             }
         }
-        // pad columns of both halves, the ones column (bias), trailing pad
-        for (int col = Fi + lane; col < Fp; col += 32) { st_act(out + col, 0.f); st_act(out + Fp + col, 0.f); }
-        for (int col = 2 * Fp + lane; col < ldxa; col += 32) st_act(out + col, col == 2 * Fp ? 1.f : 0.f);
+        if (rowok) {
+            // pad columns of both halves, the ones column (bias), trailing pad
+            for (int col = NV * VW + sub; col < Fp; col += LPR) { st_act(out + col, 0.f); st_act(out + Fp + col, 0.f); }
+            for (int col = 2 * Fp + sub; col < ldxa; col += LPR) st_act(out + col, col == 2 * Fp ? 1.f : 0.f);
+        }
     }
 }
 
@@ -305,6 +328,119 @@ __global__ void __launch_bounds__(256) k_route_pool(const float* __restrict__ dX
     }
 }
 
+// ------------------------------------ vectorised narrow-row gathers (LPR lanes / row)
+// mean, project-first fwd: S[v] = Y[v, Fop:] + (1/D_v) sum_u Y[u, :Fo] ; out = logits or ReLU -> H (+ ones)
+template <typename Tout, int LPR>
+__global__ void __launch_bounds__(256) k_agg_pf_v(const float* __restrict__ Y, int64_t ldy,
+                                                  const int64_t* __restrict__ indptr,
+                                                  const int32_t* __restrict__ idx, const int64_t* cnt, int Fo, int Fop,
+                                                  int relu, Tout* __restrict__ out, int64_t ldo) {
+    constexpr int RPW = 32 / LPR;
+    const int64_t nd = cnt[0];
+    const int NV = (Fo + 3) / 4;
+    const int lane = lane_id(), sub = lane % LPR, grp = lane / LPR;
+    const unsigned gmask = LPR == 32 ? 0xffffffffu : (((1u << LPR) - 1u) << (grp * LPR));
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t v0 = gw * RPW; v0 < nd; v0 += nw * RPW) {
+        const int64_t v = v0 + grp;
+        const bool rowok = v < nd;
+        int64_t b = 0, e = 0;
+        if (rowok) { b = indptr[v]; e = indptr[v + 1]; }
+        const float inv = e > b ? 1.0f / (float)(e - b) : 0.0f;
+        for (int vb = 0; vb < NV; vb += LPR) {
+            const int vi = vb + sub;
+            const bool act = rowok && vi < NV;
+            float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+            for (int64_t e0 = b; e0 < e; e0 += LPR) {
+                const int n = (int)mn64(LPR, e - e0);
+                const int32_t my = sub < n ? idx[e0 + sub] : 0;
+                for (int j = 0; j < n; ++j) {
+                    const int32_t u = __shfl_sync(gmask, my, j, LPR);
+                    if (act) {
+                        const float4 y = *(const float4*)(Y + (int64_t)u * ldy + vi * 4);
+                        acc.x += y.x; acc.y += y.y; acc.z += y.z; acc.w += y.w;
+                    }
+                }
+            }
+            if (act) {
+                const float4 sf = *(const float4*)(Y + v * ldy + Fop + vi * 4);
+                float r[4] = {sf.x + acc.x * inv, sf.y + acc.y * inv, sf.z + acc.z * inv, sf.w + acc.w * inv};
+#pragma unroll
+                for (int t = 0; t < 4; ++t) {
+                    const int col = vi * 4 + t;
+                    if (col < Fo) st_act(out + v * ldo + col, relu ? fmaxf(r[t], 0.f) : r[t]);
+                }
+            }
+        }
+        if (rowok && relu)
+            for (int col = Fo + sub; col < ldo; col += LPR) st_act(out + v * ldo + col, col == Fo ? 1.f : 0.f);
+    }
+}
+
+// mean, project-first bwd: G[u] = [ sum_{v in CSC(u)} dS[v]/D_v | 0 | [u < nd] dS[u] | 0 ]
+template <typename Tin, typename Tout, int LPR>
+__global__ void __launch_bounds__(256) k_csc_pf_v(const Tin* __restrict__ dS, int64_t ldds,
+                                                  const int64_t* __restrict__ indptr,
+                                                  const int64_t* __restrict__ t_indptr,
+                                                  const int32_t* __restrict__ t_idx, const int64_t* cnt, int Fo,
+                                                  int Fop, Tout* __restrict__ G, int64_t ldg) {
+    using VI = Vec<Tin>;
+    constexpr int VW = VI::N;
+    constexpr int RPW = 32 / LPR;
+    const int64_t nd = cnt[0], ns = cnt[1];
+    const int NV = (Fop + VW - 1) / VW;
+    const int lane = lane_id(), sub = lane % LPR, grp = lane / LPR;
+    const unsigned gmask = LPR == 32 ? 0xffffffffu : (((1u << LPR) - 1u) << (grp * LPR));
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t u0 = gw * RPW; u0 < ns; u0 += nw * RPW) {
+        const int64_t u = u0 + grp;
+        const bool rowok = u < ns;
+        int64_t b = 0, e = 0;
+        if (rowok) { b = t_indptr[u]; e = t_indptr[u + 1]; }
+        for (int vb = 0; vb < NV; vb += LPR) {
+            const int vi = vb + sub;
+            const bool act = rowok && vi < NV;
+            float acc[VW];
+#pragma unroll
+            for (int t = 0; t < VW; ++t) acc[t] = 0.f;
+            for (int64_t e0 = b; e0 < e; e0 += LPR) {
+                const int n = (int)mn64(LPR, e - e0);
+                int32_t my = 0;
+                float myinv = 0.f;
+                if (sub < n) {
+                    my = t_idx[e0 + sub];
+                    myinv = 1.0f / (float)(indptr[my + 1] - indptr[my]);
+                }
+                for (int j = 0; j < n; ++j) {
+                    const int32_t v = __shfl_sync(gmask, my, j, LPR);
+                    const float iv = __shfl_sync(gmask, myinv, j, LPR);
+                    if (act) {
+                        VI x;
+                        x.load_cg(dS + (int64_t)v * ldds + vi * VW);
+#pragma unroll
+                        for (int t = 0; t < VW; ++t) acc[t] += x.v[t] * iv;
+                    }
+                }
+            }
+            if (act) {
+                VI self;
+                if (u < nd) self.load_cg(dS + u * ldds + vi * VW);
+#pragma unroll
+                for (int t = 0; t < VW; ++t) {
+                    const int col = vi * VW + t;
+                    const bool in = col < Fo;
+                    st_act(G + u * ldg + col, in ? acc[t] : 0.f);
+                    st_act(G + u * ldg + Fop + col, (in && u < nd) ? self.v[t] : 0.f);
+                }
+            }
+        }
+    }
+}
+
+static inline int pick_lpr(int nv) { return nv <= 4 ? 4 : (nv <= 8 ? 8 : (nv <= 16 ? 16 : 32)); }
+
 // ----------------------------------------------------------- launchers
 static inline int warps_grid(betty_ctx* c, int64_t rows_cap) {
     return (int)std::max<int64_t>(1, std::min<int64_t>((rows_cap * 32 + 255) / 256, (int64_t)c->num_sms * 16));
@@ -314,20 +450,30 @@ static inline int warps_grid(betty_ctx* c, int64_t rows_cap) {
     if (bf) { using T = __nv_bfloat16; __VA_ARGS__; }          \
     else { using T = float; __VA_ARGS__; }
 
-void agg_mean_xa(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const int32_t* xrow, const int64_t* indptr,
-                 const int32_t* idx, const int64_t* cnt, int64_t rows_cap, int Fi, int Fp, void* XA, bool xa_bf16,
-                 int64_t ldxa, cudaStream_t s) {
-    DISPATCH_ACT(x_bf16, TI, DISPATCH_ACT(xa_bf16, TO,
-        k_agg_mean_xa<TI, TO><<<warps_grid(c, rows_cap), 256, 0, s>>>((const TI*)X, ldx, xrow, indptr, idx, cnt, Fi,
-                                                                      Fp, (TO*)XA, ldxa)));
+void agg_mean_xa(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const int32_t* srow, const int32_t* erow,
+                 const int32_t* emap, const int64_t* indptr, const int64_t* cnt, int64_t rows_cap, int Fi, int Fp,
+                 void* XA, bool xa_bf16, int64_t ldxa, cudaStream_t s) {
+    const int vw = x_bf16 ? 8 : 4;
+    const int nv = (Fi + vw - 1) / vw;
+    const int lpr = nv <= 8 ? 8 : (nv <= 16 ? 16 : 32);
+    const int64_t warps = (rows_cap + (32 / lpr) - 1) / (32 / lpr);
+    const int grid = warps_grid(c, warps);
+#define AGG_L(LPR) DISPATCH_ACT(x_bf16, TI, DISPATCH_ACT(xa_bf16, TO, \
+        k_agg_mean_xa<TI, TO, LPR><<<grid, 256, 0, s>>>((const TI*)X, ldx, srow, erow, emap, indptr, cnt, Fi, Fp, \
+                                                       (TO*)XA, ldxa)))
+    if (lpr == 8) { AGG_L(8); } else if (lpr == 16) { AGG_L(16); } else { AGG_L(32); }
+#undef AGG_L
 }
 
 void agg_mean_pf(betty_ctx* c, const float* Y, int64_t ldy, const int64_t* indptr, const int32_t* idx,
                  const int64_t* cnt, int64_t rows_cap, int Fo, int Fop, bool relu, void* out, bool out_bf16,
                  int64_t ldo, cudaStream_t s) {
-    DISPATCH_ACT(out_bf16, TO,
-        k_agg_mean_pf<TO><<<warps_grid(c, rows_cap), 256, 0, s>>>(Y, ldy, indptr, idx, cnt, Fo, Fop, relu ? 1 : 0,
-                                                                  (TO*)out, ldo));
+    const int lpr = pick_lpr((Fo + 3) / 4);
+    const int grid = warps_grid(c, (rows_cap + (32 / lpr) - 1) / (32 / lpr));
+#define PF_L(LPR) DISPATCH_ACT(out_bf16, TO, \
+        k_agg_pf_v<TO, LPR><<<grid, 256, 0, s>>>(Y, ldy, indptr, idx, cnt, Fo, Fop, relu ? 1 : 0, (TO*)out, ldo))
+    if (lpr == 4) { PF_L(4); } else if (lpr == 8) { PF_L(8); } else if (lpr == 16) { PF_L(16); } else { PF_L(32); }
+#undef PF_L
 }
 
 void gather_ones(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const int32_t* xrow, const int64_t* cnt_rows,
@@ -348,9 +494,13 @@ void csc_mean(betty_ctx* c, const float* dXA, int64_t ldd, const int64_t* indptr
 void csc_pf(betty_ctx* c, const void* dS, bool ds_bf16, int64_t ldds, const int64_t* indptr, const int64_t* t_indptr,
             const int32_t* t_idx, const int64_t* cnt, int64_t src_cap, int Fo, int Fop, void* G, bool g_bf16,
             int64_t ldg, cudaStream_t s) {
-    DISPATCH_ACT(ds_bf16, TI, DISPATCH_ACT(g_bf16, TO,
-        k_csc_pf<TI, TO><<<warps_grid(c, src_cap), 256, 0, s>>>((const TI*)dS, ldds, indptr, t_indptr, t_idx, cnt, Fo,
-                                                                Fop, (TO*)G, ldg)));
+    const int lpr = pick_lpr((Fop + (ds_bf16 ? 7 : 3)) / (ds_bf16 ? 8 : 4));
+    const int grid = warps_grid(c, (src_cap + (32 / lpr) - 1) / (32 / lpr));
+#define CSC_L(LPR) DISPATCH_ACT(ds_bf16, TI, DISPATCH_ACT(g_bf16, TO, \
+        k_csc_pf_v<TI, TO, LPR><<<grid, 256, 0, s>>>((const TI*)dS, ldds, indptr, t_indptr, t_idx, cnt, Fo, Fop, \
+                                                    (TO*)G, ldg)))
+    if (lpr == 4) { CSC_L(4); } else if (lpr == 8) { CSC_L(8); } else if (lpr == 16) { CSC_L(16); } else { CSC_L(32); }
+#undef CSC_L
 }
 
 void agg_pool(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const int32_t* xrow, const float* Zp, int64_t ldz,

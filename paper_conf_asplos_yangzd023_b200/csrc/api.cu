@@ -589,6 +589,11 @@ extern "C" betty_status betty_plan_create(betty_ctx* c, const betty_model* model
         betty_plan_destroy(c, p);
         return fail(c, BETTY_ENOMEM, "plan: arena allocation failed");
     }
+    if (m.layers[0].kind == KIND_AGG) p->X.layers[0].egid = A.get<int32_t>(ce[0]);   // layer-0 gather by gid
+    if (!A.ok) {
+        betty_plan_destroy(c, p);
+        return fail(c, BETTY_ENOMEM, "plan: arena allocation failed");
+    }
     std::vector<int32_t> hk((size_t)p->groups.size() * p->c, 0);
     for (size_t g = 0; g < p->groups.size(); ++g)
         for (size_t t = 0; t < p->groups[g].size(); ++t) hk[g * p->c + t] = p->groups[g][t];
@@ -597,7 +602,7 @@ extern "C" betty_status betty_plan_create(betty_ctx* c, const betty_model* model
     for (int l = 0; l < L; ++l) {
         const ExtractLayer& B = p->X.layers[l];
         p->views[l] = BlockView{B.indptr, B.indices, B.t_indptr, B.t_indices, B.src_gid, B.cnt, B.cap_dst, B.cap_src,
-                                B.cap_e};
+                                B.cap_e, B.egid};
     }
     // scan scratch for the largest scan of a step (never grows inside a capture)
     {

@@ -112,20 +112,22 @@ __global__ void k_mark_dst(const int32_t* __restrict__ dst_pos, const int32_t* _
     }
 }
 
+// LPR lanes per dst row (LPR ~ the layer's mean degree): short sampled rows keep the lanes busy
+template <int LPR>
 __global__ void k_mark_new(const int32_t* __restrict__ dst_pos, const int32_t* __restrict__ row_mb,
                            const int64_t* cnt, const int64_t* __restrict__ findptr, const int32_t* __restrict__ fnbr,
                            const uint32_t* __restrict__ dstbits, uint32_t* newbits, int64_t W) {
     const int64_t n = cnt[0];
-    const int lane = lane_id();
-    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const int sub = lane_id() % LPR;
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / LPR;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) / LPR;
     for (int64_t r = gw; r < n; r += nw) {
         const int j = row_mb[r];
         const int32_t q = dst_pos[r];
         const int64_t b = findptr[q], e = findptr[q + 1];
         const uint32_t* db = dstbits + j * W;
         uint32_t* nb = newbits + j * W;
-        for (int64_t i = b + lane; i < e; i += 32) {
+        for (int64_t i = b + sub; i < e; i += LPR) {
             const int32_t p = fnbr[i];
             const uint32_t bit = 1u << (p & 31);
             if (!(db[p >> 5] & bit)) atomicOr(&nb[p >> 5], bit);
@@ -205,16 +207,18 @@ __global__ void k_emit_dst(const int32_t* __restrict__ dst_pos, const int32_t* _
     }
 }
 
+template <int LPR>
 __global__ void k_relabel(const int32_t* __restrict__ dst_pos, const int32_t* __restrict__ row_mb, const int64_t* cnt,
                           const int64_t* __restrict__ findptr, const int32_t* __restrict__ fnbr,
                           const int64_t* __restrict__ indptr, const uint32_t* __restrict__ dstbits,
                           const uint32_t* __restrict__ newbits, const int64_t* __restrict__ wordoff, int64_t W,
                           const int32_t* __restrict__ map, int64_t map_stride, const int64_t* __restrict__ mb_dst_off,
-                          const int64_t* __restrict__ mb_src_off, int32_t* __restrict__ indices, int64_t cap_e) {
+                          const int64_t* __restrict__ mb_src_off, int32_t* __restrict__ indices, int64_t cap_e,
+                          const int32_t* __restrict__ fsrc_gid, int32_t* __restrict__ egid) {
     const int64_t n = cnt[0];
-    const int lane = lane_id();
-    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const int lane = lane_id() % LPR;
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / LPR;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) / LPR;
     for (int64_t r = gw; r < n; r += nw) {
         const int j = row_mb[r];
         const int32_t q = dst_pos[r];
@@ -226,7 +230,7 @@ __global__ void k_relabel(const int32_t* __restrict__ dst_pos, const int32_t* __
         const int64_t wo0 = wo[0];
         const int64_t so = cnt[0] + mb_src_off[j];      // j's new sources follow the whole dst prefix
         (void)mb_dst_off;
-        for (int64_t i = fb + lane; i < fe; i += 32) {
+        for (int64_t i = fb + lane; i < fe; i += LPR) {
             const int32_t p = fnbr[i];
             const int32_t w = p >> 5;
             const uint32_t bit = 1u << (p & 31);
@@ -234,7 +238,10 @@ __global__ void k_relabel(const int32_t* __restrict__ dst_pos, const int32_t* __
             if (db[w] & bit) id = map[j * map_stride + p];
             else id = so + (wo[w] - wo0) + __popc(nb[w] & (bit - 1));
             const int64_t o = ob + (i - fb);
-            if (o < cap_e) indices[o] = (int32_t)id;
+            if (o < cap_e) {
+                indices[o] = (int32_t)id;
+                if (egid) egid[o] = fsrc_gid[p];
+            }
         }
     }
 }
@@ -286,8 +293,15 @@ void extract_group(betty_ctx* ctx, const ExtractArgs& a, cudaStream_t s) {
         // dedupe: dst bitmap + position map, then new-source bitmap
         k_mark_dst<<<grid_for(ctx, cap_d, 256), 256, 0, s>>>(dst_pos, row_mb, dst_off, B.cnt, a.sc.dstbits, W,
                                                              a.sc.map, a.sc.map_stride);
-        k_mark_new<<<grid_for(ctx, cap_d * 32, 256), 256, 0, s>>>(dst_pos, row_mb, B.cnt, F.indptr, F.nbr,
-                                                                  a.sc.dstbits, a.sc.newbits, W);
+        const int64_t avg = F.n_dst > 0 ? (F.n_edges + F.n_dst - 1) / F.n_dst : 1;
+        const int lpr = avg <= 4 ? 4 : (avg <= 8 ? 8 : (avg <= 16 ? 16 : 32));
+        const int g_rows = grid_for(ctx, cap_d * lpr, 256);
+#define LPR_DISPATCH(KERNEL, ...)                                                           \
+        if (lpr == 4) KERNEL<4><<<g_rows, 256, 0, s>>>(__VA_ARGS__);                        \
+        else if (lpr == 8) KERNEL<8><<<g_rows, 256, 0, s>>>(__VA_ARGS__);                   \
+        else if (lpr == 16) KERNEL<16><<<g_rows, 256, 0, s>>>(__VA_ARGS__);                 \
+        else KERNEL<32><<<g_rows, 256, 0, s>>>(__VA_ARGS__);
+        LPR_DISPATCH(k_mark_new, dst_pos, row_mb, B.cnt, F.indptr, F.nbr, a.sc.dstbits, a.sc.newbits, W)
         // ascending order of new sources = popcount scan over the bitmap words
         k_popc<<<grid_for(ctx, cW, 256), 256, 0, s>>>(a.sc.newbits, cW, a.sc.wordcnt);
         scan_i32(ctx, a.sc.wordcnt, a.sc.wordoff, nullptr, cW, 0, nullptr, s);
@@ -297,10 +311,10 @@ void extract_group(betty_ctx* ctx, const ExtractArgs& a, cudaStream_t s) {
                                                              F.src_gid, B.src_pos, B.src_gid, B.src_mb, cap_s);
         k_emit_new<<<grid_for(ctx, cW, 256), 256, 0, s>>>(a.sc.newbits, W, c, B.cnt, a.sc.wordoff, dst_off, B.mb_src_off,
                                                           F.src_gid, B.src_pos, B.src_gid, B.src_mb, cap_s);
-        k_relabel<<<grid_for(ctx, cap_d * 32, 256), 256, 0, s>>>(dst_pos, row_mb, B.cnt, F.indptr, F.nbr, B.indptr,
-                                                                 a.sc.dstbits, a.sc.newbits, a.sc.wordoff, W, a.sc.map,
-                                                                 a.sc.map_stride, dst_off, B.mb_src_off, B.indices,
-                                                                 cap_e);
+        LPR_DISPATCH(k_relabel, dst_pos, row_mb, B.cnt, F.indptr, F.nbr, B.indptr, a.sc.dstbits, a.sc.newbits,
+                     a.sc.wordoff, W, a.sc.map, a.sc.map_stride, dst_off, B.mb_src_off, B.indices, cap_e, F.src_gid,
+                     B.egid)
+#undef LPR_DISPATCH
         k_clear_bits<<<grid_for(ctx, cW, 256), 256, 0, s>>>(a.sc.dstbits, a.sc.newbits, cW);
         if (B.t_indptr && (a.csc_mask >> l & 1))
             csr_transpose(ctx, B.indptr, B.indices, B.cnt + 0, B.cnt + 1, B.cnt + 2, cap_d, cap_s, cap_e,

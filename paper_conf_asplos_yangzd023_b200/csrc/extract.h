@@ -21,6 +21,7 @@ struct ExtractLayer {           // group-concatenated micro-batch layer l (devic
     int32_t* src_mb;            // [cap_src] slot j of each src row
     int64_t* t_indptr;          // [cap_src+1] (null: no CSC)
     int32_t* t_indices;         // [cap_e]
+    int32_t* egid;              // [cap_e] or null: global id of each edge's source (feeds the layer-0 gather)
     int64_t* cnt;               // device [4]: n_dst, n_src, n_edges, spare
     int64_t* mb_src_off;        // [c+1]
     int64_t cap_dst, cap_src, cap_e;

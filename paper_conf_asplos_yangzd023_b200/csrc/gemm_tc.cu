@@ -103,6 +103,13 @@ __device__ __forceinline__ void tmem_free_warp(uint32_t taddr, uint32_t ncols) {
 __device__ __forceinline__ bool elect_lane0() { return (threadIdx.x & 31) == 0; }
 
 // --------------------------------------------------------------- row GEMM
+// B (the weights, <= 256 x K) stays resident in shared memory for the whole
+// persistent CTA; only A tiles stream through the TMA ring.  Eight epilogue
+// warps: warp w drains TMEM lanes 32*(w%4).. (tile rows) for one half of the
+// columns; each thread owns one output row and writes 16-byte vectors, with
+// the next chunk's TMEM load (and mask load) issued before the current chunk
+// is processed.
+constexpr int ROW_THREADS = 64 + 256;
 struct RowArgs {
     const int64_t* M_dev;
     int K, N, BN, nk, stages;
@@ -111,24 +118,87 @@ struct RowArgs {
     const void* mask; int64_t ldm; int m_bf16;
     const float* res; int64_t ldr; const int64_t* nres_dev;
     uint32_t tmem_cols;
+    int half_cols;           // columns per epilogue half (multiple of 32)
 };
 
-__device__ __forceinline__ float ld_any(const void* p, int64_t i, int bf) {
-    return bf ? __bfloat162float(((const __nv_bfloat16*)p)[i]) : ((const float*)p)[i];
+__device__ __forceinline__ uint32_t pack_bf16x2(float a, float b) {
+    __nv_bfloat162 h = __floats2bfloat162_rn(a, b);
+    return *(uint32_t*)&h;
 }
 
-__global__ void __launch_bounds__(THREADS, 1) k_tc_row(const __grid_constant__ CUtensorMap tmA,
-                                                       const __grid_constant__ CUtensorMap tmB, RowArgs p) {
+// one 32-column chunk of one row: epilogue math + vector stores
+__device__ __forceinline__ void row_chunk_out(const RowArgs& p, float* v, int64_t m, int c0, const uint4* mk,
+                                              int64_t nres) {
+    const int nval = min(32, p.N - c0);            // valid output columns in this chunk
+    if (nval <= 0) return;
+#pragma unroll
+    for (int j = 0; j < 32; ++j) {
+        float x = v[j];
+        if (p.epi == EPI_RELU_ONES) x = fmaxf(x, 0.f);
+        if (p.epi == EPI_RES_MASK && m < nres && j < nval) x += p.res[m * p.ldr + c0 + j];
+        if (p.epi == EPI_MASK || p.epi == EPI_RES_MASK) {
+            float mv;
+            if (p.m_bf16) {
+                const __nv_bfloat16* hb = (const __nv_bfloat16*)&mk[j / 8];
+                mv = __bfloat162float(hb[j % 8]);
+            } else {
+                mv = ((const float*)&mk[j / 4])[j % 4];
+            }
+            if (!(mv > 0.f)) x = 0.f;
+        }
+        v[j] = x;
+    }
+    if (p.c_bf16) {
+        __nv_bfloat16* cp = (__nv_bfloat16*)p.C + m * p.ldc + c0;
+        if (nval == 32 && (p.ldc & 7) == 0) {
+#pragma unroll
+            for (int q = 0; q < 4; ++q)
+                ((uint4*)cp)[q] = make_uint4(pack_bf16x2(v[8 * q], v[8 * q + 1]), pack_bf16x2(v[8 * q + 2], v[8 * q + 3]),
+                                             pack_bf16x2(v[8 * q + 4], v[8 * q + 5]),
+                                             pack_bf16x2(v[8 * q + 6], v[8 * q + 7]));
+        } else {
+#pragma unroll
+            for (int j = 0; j < 32; ++j)
+                if (j < nval) cp[j] = __float2bfloat16_rn(v[j]);
+        }
+    } else {
+        float* cp = (float*)p.C + m * p.ldc + c0;
+        if (nval == 32 && (p.ldc & 3) == 0) {
+#pragma unroll
+            for (int q = 0; q < 8; ++q) ((float4*)cp)[q] = make_float4(v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
+        } else {
+#pragma unroll
+            for (int j = 0; j < 32; ++j)
+                if (j < nval) cp[j] = v[j];
+        }
+    }
+}
+
+__device__ __forceinline__ void load_mask_chunk(const RowArgs& p, int64_t m, int c0, bool ok, uint4* mk) {
+    const int nv = p.m_bf16 ? 4 : 8;                // 16-byte vectors per 32 columns
+    if (!ok) return;
+    const char* base = (const char*)p.mask + (m * p.ldm + c0) * (p.m_bf16 ? 2 : 4);
+    const int64_t rowbytes = (int64_t)(p.N - c0) * (p.m_bf16 ? 2 : 4);
+#pragma unroll
+    for (int q = 0; q < 8; ++q)
+        if (q < nv && q * 16 < rowbytes) mk[q] = __ldg((const uint4*)(base + q * 16));
+}
+
+__global__ void __launch_bounds__(ROW_THREADS, 1) k_tc_row(const __grid_constant__ CUtensorMap tmA,
+                                                           const __grid_constant__ CUtensorMap tmB, RowArgs p) {
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
     const int S = p.stages;
-    const uint32_t a_bytes = BM * BK * 2, b_bytes = (uint32_t)p.BN * BK * 2;
-    const uint32_t stage_bytes = a_bytes + b_bytes;
-    uint64_t* full = (uint64_t*)(smem + S * stage_bytes);
+    const uint32_t a_bytes = BM * BK * 2;
+    const uint32_t bblk = (uint32_t)p.BN * BK * 2;          // one K-block of the resident B
+    uint8_t* bres = smem;                                    // nk * bblk
+    uint8_t* aring = smem + p.nk * bblk;                     // S * a_bytes
+    uint64_t* full = (uint64_t*)(aring + S * a_bytes);
     uint64_t* empty = full + S;
     uint64_t* tfull = empty + S;      // [2]
     uint64_t* tempty = tfull + 2;     // [2]
-    uint32_t* tslot = (uint32_t*)(tempty + 2);
+    uint64_t* bfull = tempty + 2;     // [1]
+    uint32_t* tslot = (uint32_t*)(bfull + 1);
 
     const int warp = threadIdx.x >> 5;
     const int64_t M = *p.M_dev;
@@ -136,7 +206,8 @@ __global__ void __launch_bounds__(THREADS, 1) k_tc_row(const __grid_constant__ C
 
     if (threadIdx.x == 0) {
         for (int s = 0; s < S; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
-        for (int a = 0; a < 2; ++a) { mbar_init(&tfull[a], 1); mbar_init(&tempty[a], 128); }
+        for (int a = 0; a < 2; ++a) { mbar_init(&tfull[a], 1); mbar_init(&tempty[a], 256); }
+        mbar_init(bfull, 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
         asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmA) : "memory");
         asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmB) : "memory");
@@ -148,16 +219,16 @@ __global__ void __launch_bounds__(THREADS, 1) k_tc_row(const __grid_constant__ C
     const uint32_t tmem = *tslot;
 
     if (warp == 0) {
-        if (elect_lane0()) {
+        if (elect_lane0() && blockIdx.x < tiles) {
+            mbar_expect_tx(bfull, p.nk * bblk);
+            for (int kb = 0; kb < p.nk; ++kb) tma_2d(bres + kb * bblk, &tmB, kb * BK, 0, bfull);
             int s = 0;
             uint32_t ph = 0;
             for (int64_t t = blockIdx.x; t < tiles; t += gridDim.x) {
                 for (int kb = 0; kb < p.nk; ++kb) {
                     mbar_wait(&empty[s], ph ^ 1);
-                    uint8_t* sa = smem + s * stage_bytes;
-                    mbar_expect_tx(&full[s], stage_bytes);
-                    tma_2d(sa, &tmA, kb * BK, (int)(t * BM), &full[s]);
-                    tma_2d(sa + a_bytes, &tmB, kb * BK, 0, &full[s]);
+                    mbar_expect_tx(&full[s], a_bytes);
+                    tma_2d(aring + s * a_bytes, &tmA, kb * BK, (int)(t * BM), &full[s]);
                     if (++s == S) { s = 0; ph ^= 1; }
                 }
             }
@@ -167,6 +238,7 @@ __global__ void __launch_bounds__(THREADS, 1) k_tc_row(const __grid_constant__ C
         int s = 0;
         uint32_t ph = 0;
         int it = 0;
+        if (blockIdx.x < tiles) mbar_wait(bfull, 0);
         for (int64_t t = blockIdx.x; t < tiles; t += gridDim.x, ++it) {
             const int acc = it & 1;
             const uint32_t aph = (it >> 1) & 1;
@@ -177,7 +249,7 @@ __global__ void __launch_bounds__(THREADS, 1) k_tc_row(const __grid_constant__ C
                 mbar_wait(&full[s], ph);
                 fence_after();
                 if (elect_lane0()) {
-                    const uint32_t a0 = su32(smem + s * stage_bytes), b0 = a0 + a_bytes;
+                    const uint32_t a0 = su32(aring + s * a_bytes), b0 = su32(bres + kb * bblk);
 #pragma unroll
                     for (int k = 0; k < BK / UK; ++k) {
                         const uint64_t ad = sdesc(a0 + k * UK * 2, 0, 1024);
@@ -192,66 +264,65 @@ __global__ void __launch_bounds__(THREADS, 1) k_tc_row(const __grid_constant__ C
             }
         }
     } else {
-        // epilogue: warp w reads TMEM lanes 32*(w%4) .. +31 = tile rows
-        const int q = warp & 3;
-        const int r_in = q * 32 + (threadIdx.x & 31);
-        int it = 0;
+        const int ew = warp - 2;                 // 0..7
+        const int q = warp & 3;                  // TMEM lane quadrant (hardware: warp id % 4)
+        const int h = ew >> 2;                   // column half
+        const int lane = threadIdx.x & 31;
+        const int cbeg = h * p.half_cols;
+        const int cend = min(p.BN, cbeg + p.half_cols);
+        const bool has_mask = p.epi == EPI_MASK || p.epi == EPI_RES_MASK;
         const int64_t nres = (p.epi == EPI_RES_MASK) ? *p.nres_dev : 0;
+        int it = 0;
         for (int64_t t = blockIdx.x; t < tiles; t += gridDim.x, ++it) {
             const int acc = it & 1;
             const uint32_t aph = (it >> 1) & 1;
+            const int64_t m = t * BM + q * 32 + lane;
+            const bool ok = m < M;
+            uint4 mk[8], mk_next[8];
+            if (has_mask && cbeg < cend) load_mask_chunk(p, m, cbeg, ok, mk);
             mbar_wait(&tfull[acc], aph);
             fence_after();
-            const int64_t m = t * BM + r_in;
-            const bool ok = m < M;
-            for (int c0 = 0; c0 < p.BN; c0 += 32) {
-                float v[32];
-                tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + acc * p.BN + c0, v);
-                if (!ok) continue;
+            const uint32_t tbase = tmem + ((uint32_t)(q * 32) << 16) + acc * p.BN;
+            float v[32];
+            if (cbeg < cend) tmem_ld32(tbase + cbeg, v);
+            for (int c0 = cbeg; c0 < cend; c0 += 32) {
+                const bool more = c0 + 32 < cend;
+                float nx[32];
+                if (more) {
+                    // next chunk's TMEM load in flight while this chunk is stored
+                    uint32_t r[32];
+                    asm volatile("tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,"
+                                 "%13,%14,%15,%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+                                 : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
+                                   "=r"(r[7]), "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]),
+                                   "=r"(r[13]), "=r"(r[14]), "=r"(r[15]), "=r"(r[16]), "=r"(r[17]), "=r"(r[18]),
+                                   "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]), "=r"(r[24]),
+                                   "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]),
+                                   "=r"(r[31])
+                                 : "r"(tbase + c0 + 32));
 #pragma unroll
-                for (int j = 0; j < 32; ++j) {
-                    const int n = c0 + j;
-                    if (n >= p.N) break;
-                    float x = v[j];
-                    if (p.epi == EPI_RELU_ONES) x = fmaxf(x, 0.f);
-                    if (p.epi == EPI_RES_MASK && m < nres) x += p.res[m * p.ldr + n];
-                    if (p.epi == EPI_MASK || p.epi == EPI_RES_MASK)
-                        if (!(ld_any(p.mask, m * p.ldm + n, p.m_bf16) > 0.f)) x = 0.f;
-                    v[j] = x;
+                    for (int j = 0; j < 32; ++j) nx[j] = __uint_as_float(r[j]);
+                    if (has_mask) load_mask_chunk(p, m, c0 + 32, ok, mk_next);
                 }
-                if (p.c_bf16) {
-                    __nv_bfloat16* crow = (__nv_bfloat16*)p.C + m * p.ldc;
-                    if (c0 + 32 <= p.N && ((p.ldc & 7) == 0)) {
+                if (ok) row_chunk_out(p, v, m, c0, mk, nres);
+                if (more) {
+                    asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
 #pragma unroll
-                        for (int j = 0; j < 32; j += 8) {
-                            uint4 u;
-                            __nv_bfloat162* h = (__nv_bfloat162*)&u;
+                    for (int j = 0; j < 32; ++j) v[j] = nx[j];
 #pragma unroll
-                            for (int i = 0; i < 4; ++i) h[i] = __floats2bfloat162_rn(v[j + 2 * i], v[j + 2 * i + 1]);
-                            *(uint4*)(crow + c0 + j) = u;
-                        }
-                    } else {
-                        for (int j = 0; j < 32 && c0 + j < p.N; ++j) crow[c0 + j] = __float2bfloat16_rn(v[j]);
-                    }
-                } else {
-                    float* crow = (float*)p.C + m * p.ldc;
-                    if (c0 + 32 <= p.N && ((p.ldc & 3) == 0)) {
-#pragma unroll
-                        for (int j = 0; j < 32; j += 4) *(float4*)(crow + c0 + j) = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
-                    } else {
-                        for (int j = 0; j < 32 && c0 + j < p.N; ++j) crow[c0 + j] = v[j];
-                    }
+                    for (int q2 = 0; q2 < 8; ++q2) mk[q2] = mk_next[q2];
                 }
             }
-            if (ok && p.ldc > p.N) {   // trailing columns: the ones column after ReLU, zeros otherwise
+            fence_before();
+            mbar_arrive(&tempty[acc]);
+            // trailing columns [N, ldc): the ones column after a ReLU layer, zeros elsewhere
+            if (h == 1 && ok && p.ldc > p.N) {
                 for (int col = p.N; col < p.ldc; ++col) {
                     const float x = (p.epi == EPI_RELU_ONES && col == p.N) ? 1.f : 0.f;
                     if (p.c_bf16) ((__nv_bfloat16*)p.C)[m * p.ldc + col] = __float2bfloat16_rn(x);
                     else ((float*)p.C)[m * p.ldc + col] = x;
                 }
             }
-            fence_before();
-            mbar_arrive(&tempty[acc]);
         }
     }
     __syncthreads();
@@ -419,18 +490,24 @@ bool tc_available() { return tc::encode_fn() != nullptr; }
 bool gemm_row_tc(betty_ctx* c, const GemmRow& g, const void* Bk, int64_t ldbk, cudaStream_t s) {
     using namespace tc;
     if (!g.a_bf16 || !g.b_bf16 || g.N > 256 || g.N < 1 || (g.lda & 7) || (ldbk & 7)) return false;
+    if ((g.epi == EPI_MASK || g.epi == EPI_RES_MASK) && (g.ldm & 7)) return false;
     const int BN = (g.N + 15) / 16 * 16;
+    const int nk = (g.K + BK - 1) / BK;
+    const size_t b_bytes = (size_t)nk * BN * BK * 2;
+    const size_t a_bytes = BM * BK * 2;
+    const size_t budget = 220 * 1024;
+    if (b_bytes + 2 * a_bytes + 2048 > budget) return false;       // B must fit resident
     CUtensorMap ma, mb;
     if (!make_map(&ma, g.A, g.K, g.M_cap, g.lda, BM) || !make_map(&mb, Bk, g.K, g.N, ldbk, BN)) return false;
     RowArgs p{};
-    p.M_dev = g.M_dev; p.K = g.K; p.N = g.N; p.BN = BN; p.nk = (g.K + BK - 1) / BK;
-    const int stage_bytes = BM * BK * 2 + BN * BK * 2;
-    p.stages = std::max(2, std::min(6, (200 * 1024) / stage_bytes));
+    p.M_dev = g.M_dev; p.K = g.K; p.N = g.N; p.BN = BN; p.nk = nk;
+    p.stages = (int)std::max<size_t>(2, std::min<size_t>(8, (budget - b_bytes - 2048) / a_bytes));
     p.C = g.C; p.ldc = g.ldc; p.c_bf16 = g.c_bf16; p.epi = g.epi;
     p.mask = g.mask; p.ldm = g.ldm; p.m_bf16 = g.m_bf16; p.res = g.res; p.ldr = g.ldr; p.nres_dev = g.nres_dev;
     p.tmem_cols = tmem_cols_for(2 * BN);
+    p.half_cols = ((BN + 63) / 64) * 32;
     if (p.tmem_cols > 512) return false;
-    const size_t smem = (size_t)p.stages * stage_bytes + 1024 + 256;
+    const size_t smem = b_bytes + (size_t)p.stages * a_bytes + 1024 + 256;
     static bool attr = false;
     if (!attr) {
         cudaFuncSetAttribute(k_tc_row, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
@@ -438,7 +515,7 @@ bool gemm_row_tc(betty_ctx* c, const GemmRow& g, const void* Bk, int64_t ldbk, c
     }
     const int64_t tiles = (g.M_cap + BM - 1) / BM;
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(tiles, c->num_sms));
-    k_tc_row<<<grid, THREADS, smem, s>>>(ma, mb, p);
+    k_tc_row<<<grid, ROW_THREADS, smem, s>>>(ma, mb, p);
     return true;
 }
 

@@ -44,6 +44,7 @@ struct BlockView {              // one layer of a (group-concatenated) micro-bat
     const int32_t* src_gid;
     const int64_t* cnt;         // device [3]: n_dst, n_src, n_edges
     int64_t cap_dst, cap_src, cap_e;
+    const int32_t* egid = nullptr;   // optional [n_edges]: global id of each edge's source (layer 0)
 };
 
 struct LayerBufs {

@@ -220,7 +220,11 @@ void sage_forward(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView*
             PE(l == 0 ? PROBE_AGG_L0 : PROBE_AGG_L1);
         } else {
             PB(l == 0 ? PROBE_AGG_L0 : PROBE_AGG_L1);
-            agg_mean_xa(c, X, xbf, ldx, xrow, V.indptr, V.indices, V.cnt, V.cap_dst, L.Fi, L.Fp, B.XA, m.bf16,
+            // layer 0 reads feature rows by global id: straight from the extraction's edge -> gid
+            // array when present, else through src_gid
+            const int32_t* erow = (l == 0 && V.egid) ? V.egid : V.indices;
+            const int32_t* emap = (l == 0 && !V.egid) ? V.src_gid : nullptr;
+            agg_mean_xa(c, X, xbf, ldx, xrow, erow, emap, V.indptr, V.cnt, V.cap_dst, L.Fi, L.Fp, B.XA, m.bf16,
                         L.ld_xa, s);
             PE(l == 0 ? PROBE_AGG_L0 : PROBE_AGG_L1);
         }

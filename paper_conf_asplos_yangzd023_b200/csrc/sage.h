@@ -7,9 +7,10 @@ struct betty_ctx;
 namespace betty {
 
 // ---- agg.cu
-void agg_mean_xa(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const int32_t* xrow, const int64_t* indptr,
-                 const int32_t* idx, const int64_t* cnt, int64_t rows_cap, int Fi, int Fp, void* XA, bool xa_bf16,
-                 int64_t ldxa, cudaStream_t s);
+// XA[v] = [X[srow v] | mean_e X[row(e)] | 1], row(e) = emap ? emap[erow[e]] : erow[e]
+void agg_mean_xa(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const int32_t* srow, const int32_t* erow,
+                 const int32_t* emap, const int64_t* indptr, const int64_t* cnt, int64_t rows_cap, int Fi, int Fp,
+                 void* XA, bool xa_bf16, int64_t ldxa, cudaStream_t s);
 void agg_mean_pf(betty_ctx* c, const float* Y, int64_t ldy, const int64_t* indptr, const int32_t* idx,
                  const int64_t* cnt, int64_t rows_cap, int Fo, int Fop, bool relu, void* out, bool out_bf16,
                  int64_t ldo, cudaStream_t s);
