@@ -301,8 +301,12 @@ def betty_test_gemm(ctx: Context, kind: int, A: torch.Tensor, B: torch.Tensor, K
     """Test hook of the dense kernels.  kind 0: A[M,K] @ B[N,K]^T; kind 1: A[M,K]^T @ B[M,N]."""
     M = A.shape[0] if M is None else M
     if kind == 0:
-        C = torch.zeros((M, N), dtype=torch.float32, device=A.device)
-        ldc = N
+        # rows up to A.shape[0] (the capacity) may be written; row stride padded to 16 bytes
+        ldc = (N + 3) // 4 * 4
+        Cfull = torch.zeros((A.shape[0], ldc), dtype=torch.float32, device=A.device)
+        ctx.check(L.lib().betty_test_gemm(ctx.h, kind, _p(A), A.stride(0), _p(B), B.stride(0), M, A.shape[0], K, N,
+                                          _p(Cfull), ldc, int(use_tc), _stream(stream)), "betty_test_gemm")
+        return Cfull[:M, :N]
     else:
         C = torch.zeros((K, N), dtype=torch.float32, device=A.device)
         ldc = N

@@ -15,6 +15,7 @@
 #include "common.cuh"
 #include "internal.h"
 #include "sage.h"
+#include "extract.h"
 
 namespace betty {
 
@@ -24,29 +25,39 @@ template <typename T> __device__ __forceinline__ const T* row_ptr(const T* X, in
 
 // ------------------------------------------------ mean, aggregate-first fwd
 // LPR lanes own one dst row (RPW = 32/LPR rows per warp in flight); each lane
-// covers 16-byte vectors of the feature row.  The neighbour X-row of edge e is
-// emap ? emap[erow[e]] : erow[e] (layer 0 passes the edge -> global-id array
-// written by the extraction, so no dependent id lookup stays on the critical
-// path); the self row of dst v is srow ? srow[v] : v.
+// covers 16-byte vectors of the feature row and keeps AGG_BATCH neighbour
+// rows in flight.  The neighbour X-row of edge e is emap ? emap[erow[e]] : erow[e]
+// (layer 0 passes the edge -> global-id array written by the extraction, so no
+// dependent id lookup stays on the critical path); the self row of dst v is
+// srow ? srow[v] : v.  With an order table (extract.h) the rows are visited
+// micro-batch by micro-batch, so the source rows one micro-batch shares stay
+// in L2 between their uses; the grid is exactly the resident CTAs so all warps
+// sweep the order together.
+constexpr int AGG_BATCH = 4;     // neighbour rows in flight per lane (x 16 B)
 template <typename Tin, typename Tout, int LPR>
-__global__ void __launch_bounds__(256) k_agg_mean_xa(const Tin* __restrict__ X, int64_t ldx,
+__global__ void __launch_bounds__(256, 4) k_agg_mean_xa(const Tin* __restrict__ X, int64_t ldx,
                                                      const int32_t* __restrict__ srow,
                                                      const int32_t* __restrict__ erow,
                                                      const int32_t* __restrict__ emap,
-                                                     const int64_t* __restrict__ indptr, const int64_t* cnt, int Fi,
-                                                     int Fp, Tout* __restrict__ XA, int64_t ldxa) {
+                                                     const int64_t* __restrict__ indptr, const int64_t* cnt,
+                                                     const int64_t* __restrict__ otab, int Fi, int Fp,
+                                                     Tout* __restrict__ XA, int64_t ldxa) {
     using VI = Vec<Tin>;
     constexpr int VW = VI::N;
     constexpr int RPW = 32 / LPR;
+    __shared__ int64_t s_vs[ORDER_SMEM + 1], s_rs[ORDER_SMEM];
     const int64_t nd = cnt[0];
+    const int nseg = order_load(otab, s_vs, s_rs);
     const int NV = (Fi + VW - 1) / VW;
     const int lane = lane_id(), sub = lane % LPR, grp = lane / LPR;
     const unsigned gmask = LPR == 32 ? 0xffffffffu : (((1u << LPR) - 1u) << (grp * LPR));
     const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    int seg = 0;
     for (int64_t v0 = gw * RPW; v0 < nd; v0 += nw * RPW) {
-        const int64_t v = v0 + grp;
-        const bool rowok = v < nd;
+        const int64_t vv = v0 + grp;
+        const bool rowok = vv < nd;
+        const int64_t v = rowok ? order_map(vv, nseg, s_vs, s_rs, seg) : vv;
         int64_t b = 0, e = 0;
         if (rowok) { b = indptr[v]; e = indptr[v + 1]; }
         const float inv = e > b ? 1.0f / (float)(e - b) : 0.0f;
@@ -61,30 +72,15 @@ __global__ void __launch_bounds__(256) k_agg_mean_xa(const Tin* __restrict__ X, 
                 const int n = (int)mn64(LPR, e - e0);
                 int32_t my = 0;
                 if (sub < n) { my = erow[e0 + sub]; if (emap) my = emap[my]; }
-                int j = 0;
-                for (; j + 4 <= n; j += 4) {
-                    const int32_t u0 = __shfl_sync(gmask, my, j, LPR);
-                    const int32_t u1 = __shfl_sync(gmask, my, j + 1, LPR);
-                    const int32_t u2 = __shfl_sync(gmask, my, j + 2, LPR);
-                    const int32_t u3 = __shfl_sync(gmask, my, j + 3, LPR);
-                    if (act) {
-                        VI x0, x1, x2, x3;
-                        x0.load(X + (int64_t)u0 * ldx + vi * VW);
-                        x1.load(X + (int64_t)u1 * ldx + vi * VW);
-                        x2.load(X + (int64_t)u2 * ldx + vi * VW);
-                        x3.load(X + (int64_t)u3 * ldx + vi * VW);
+                for (int j = 0; j < n; j += AGG_BATCH) {
+                    typename VI::Raw x[AGG_BATCH];
 #pragma unroll
-                        for (int t = 0; t < VW; ++t) acc[t] += (x0.v[t] + x1.v[t]) + (x2.v[t] + x3.v[t]);
+                    for (int t = 0; t < AGG_BATCH; ++t) {
+                        const int32_t u = __shfl_sync(gmask, my, (j + t) & (LPR - 1), LPR);
+                        x[t] = (act && j + t < n) ? VI::ld_raw(X + (int64_t)u * ldx + vi * VW) : VI::zero_raw();
                     }
-                }
-                for (; j < n; ++j) {
-                    const int32_t u = __shfl_sync(gmask, my, j, LPR);
-                    if (act) {
-                        VI x;
-                        x.load(X + (int64_t)u * ldx + vi * VW);
 #pragma unroll
-                        for (int t = 0; t < VW; ++t) acc[t] += x.v[t];
-                    }
+                    for (int t = 0; t < AGG_BATCH; ++t) VI::add_raw(acc, x[t]);
                 }
             }
             if (act) {
@@ -427,12 +423,17 @@ __global__ void __launch_bounds__(256) k_csc_pf_v(const Tin* __restrict__ dS, in
             if (act) {
                 VI self;
                 if (u < nd) self.load_cg(dS + u * ldds + vi * VW);
+                float ga[VW], gs[VW];
 #pragma unroll
                 for (int t = 0; t < VW; ++t) {
-                    const int col = vi * VW + t;
-                    const bool in = col < Fo;
-                    st_act(G + u * ldg + col, in ? acc[t] : 0.f);
-                    st_act(G + u * ldg + Fop + col, (in && u < nd) ? self.v[t] : 0.f);
+                    const bool in = vi * VW + t < Fo;
+                    ga[t] = in ? acc[t] : 0.f;
+                    gs[t] = (in && u < nd) ? self.v[t] : 0.f;
+                }
+#pragma unroll
+                for (int t = 0; t < VW; t += 4) {        // vector stores (Fop, ldg multiples of 8)
+                    st_act4(G + u * ldg + vi * VW + t, ga + t);
+                    st_act4(G + u * ldg + Fop + vi * VW + t, gs + t);
                 }
             }
         }
@@ -450,17 +451,24 @@ static inline int warps_grid(betty_ctx* c, int64_t rows_cap) {
     if (bf) { using T = __nv_bfloat16; __VA_ARGS__; }          \
     else { using T = float; __VA_ARGS__; }
 
+// grid = the CTAs that are resident at once (persistent sweep), at most the work
+template <typename K> static int resident_grid(betty_ctx* c, K kernel, int threads, int64_t want_ctas) {
+    int per_sm = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, threads, 0) != cudaSuccess || per_sm < 1)
+        per_sm = 1;
+    return (int)std::max<int64_t>(1, std::min<int64_t>(want_ctas, (int64_t)per_sm * c->num_sms));
+}
+
 void agg_mean_xa(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const int32_t* srow, const int32_t* erow,
-                 const int32_t* emap, const int64_t* indptr, const int64_t* cnt, int64_t rows_cap, int Fi, int Fp,
-                 void* XA, bool xa_bf16, int64_t ldxa, cudaStream_t s) {
+                 const int32_t* emap, const int64_t* indptr, const int64_t* cnt, const int64_t* otab, int64_t rows_cap,
+                 int Fi, int Fp, void* XA, bool xa_bf16, int64_t ldxa, cudaStream_t s) {
     const int vw = x_bf16 ? 8 : 4;
     const int nv = (Fi + vw - 1) / vw;
     const int lpr = nv <= 8 ? 8 : (nv <= 16 ? 16 : 32);
     const int64_t warps = (rows_cap + (32 / lpr) - 1) / (32 / lpr);
-    const int grid = warps_grid(c, warps);
 #define AGG_L(LPR) DISPATCH_ACT(x_bf16, TI, DISPATCH_ACT(xa_bf16, TO, \
-        k_agg_mean_xa<TI, TO, LPR><<<grid, 256, 0, s>>>((const TI*)X, ldx, srow, erow, emap, indptr, cnt, Fi, Fp, \
-                                                       (TO*)XA, ldxa)))
+        k_agg_mean_xa<TI, TO, LPR><<<resident_grid(c, k_agg_mean_xa<TI, TO, LPR>, 256, (warps + 7) / 8), 256, 0, s>>>( \
+            (const TI*)X, ldx, srow, erow, emap, indptr, cnt, otab, Fi, Fp, (TO*)XA, ldxa)))
     if (lpr == 8) { AGG_L(8); } else if (lpr == 16) { AGG_L(16); } else { AGG_L(32); }
 #undef AGG_L
 }

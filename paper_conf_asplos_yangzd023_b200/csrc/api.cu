@@ -166,6 +166,7 @@ static bool alloc_extract(Arena& A, int L, const ExtractFull* full, int64_t n_ou
         }
         B.cnt = X->cnt_all + 4 * l;
         B.mb_src_off = A.get<int64_t>(c + 1);
+        if (l + 1 < L) B.order_tab = A.get<int64_t>(2 * (ORDER_TAB_MAX + 1) + 1);
         max_src = std::max(max_src, std::max(full[l].n_src, B.cap_src));
         max_dst = std::max(max_dst, B.cap_dst);
     }
@@ -602,7 +603,7 @@ extern "C" betty_status betty_plan_create(betty_ctx* c, const betty_model* model
     for (int l = 0; l < L; ++l) {
         const ExtractLayer& B = p->X.layers[l];
         p->views[l] = BlockView{B.indptr, B.indices, B.t_indptr, B.t_indices, B.src_gid, B.cnt, B.cap_dst, B.cap_src,
-                                B.cap_e, B.egid};
+                                B.cap_e, B.egid, B.order_tab};
     }
     // scan scratch for the largest scan of a step (never grows inside a capture)
     {

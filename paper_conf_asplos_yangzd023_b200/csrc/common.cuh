@@ -15,6 +15,12 @@ __device__ __forceinline__ float ld_act(const float* p) { return *p; }
 __device__ __forceinline__ float ld_act(const __nv_bfloat16* p) { return __bfloat162float(*p); }
 __device__ __forceinline__ void st_act(float* p, float v) { *p = v; }
 __device__ __forceinline__ void st_act(__nv_bfloat16* p, float v) { *p = __float2bfloat16_rn(v); }
+// 4 consecutive activations in one vector store (p aligned to 4 elements)
+__device__ __forceinline__ void st_act4(float* p, const float* v) { *(float4*)p = make_float4(v[0], v[1], v[2], v[3]); }
+__device__ __forceinline__ void st_act4(__nv_bfloat16* p, const float* v) {
+    __nv_bfloat162 a = __floats2bfloat162_rn(v[0], v[1]), b = __floats2bfloat162_rn(v[2], v[3]);
+    *(uint2*)p = make_uint2(*(uint32_t*)&a, *(uint32_t*)&b);
+}
 
 // 16-byte vector of activations: 4 fp32 or 8 bf16
 template <typename T> struct Vec;
@@ -32,6 +38,11 @@ template <> struct Vec<float> {
     __device__ __forceinline__ void store(float* p) const {
         *reinterpret_cast<float4*>(p) = make_float4(v[0], v[1], v[2], v[3]);
     }
+    // raw 16-byte loads kept packed while in flight (registers), unpacked when summed
+    typedef float4 Raw;
+    __device__ __forceinline__ static Raw ld_raw(const float* p) { return __ldg(reinterpret_cast<const float4*>(p)); }
+    __device__ __forceinline__ static Raw zero_raw() { return make_float4(0.f, 0.f, 0.f, 0.f); }
+    __device__ __forceinline__ static void add_raw(float* acc, Raw t) { acc[0] += t.x; acc[1] += t.y; acc[2] += t.z; acc[3] += t.w; }
 };
 template <> struct Vec<__nv_bfloat16> {
     static constexpr int N = 8;
@@ -50,6 +61,14 @@ template <> struct Vec<__nv_bfloat16> {
         for (int i = 0; i < 4; ++i) h[i] = __floats2bfloat162_rn(v[2 * i], v[2 * i + 1]);
         *reinterpret_cast<uint4*>(p) = t;
     }
+    typedef uint4 Raw;
+    __device__ __forceinline__ static Raw ld_raw(const __nv_bfloat16* p) { return __ldg(reinterpret_cast<const uint4*>(p)); }
+    __device__ __forceinline__ static Raw zero_raw() { return make_uint4(0u, 0u, 0u, 0u); }
+    __device__ __forceinline__ static void add_raw(float* acc, Raw t) {
+        const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&t);
+#pragma unroll
+        for (int i = 0; i < 4; ++i) { float2 f = __bfloat1622float2(h[i]); acc[2 * i] += f.x; acc[2 * i + 1] += f.y; }
+    }
 };
 
 __host__ __device__ __forceinline__ int64_t mn64(int64_t a, int64_t b) { return a < b ? a : b; }
@@ -57,6 +76,23 @@ __host__ __device__ __forceinline__ int64_t mn64(int64_t a, int64_t b) { return 
 // ------------------------------------------------------------ warp / block
 __device__ __forceinline__ int lane_id() { return threadIdx.x & 31; }
 __device__ __forceinline__ int warp_id() { return threadIdx.x >> 5; }
+
+// ascending bitonic sort of one int32 per lane across the warp
+__device__ __forceinline__ int32_t warp_bitonic32(int32_t x) {
+    const int lane = lane_id();
+#pragma unroll
+    for (int k = 2; k <= 32; k <<= 1) {
+#pragma unroll
+        for (int j = k >> 1; j > 0; j >>= 1) {
+            const int32_t y = __shfl_xor_sync(0xffffffffu, x, j);
+            const bool up = ((lane & k) == 0);
+            const bool lower = ((lane & j) == 0);
+            // lower element keeps min when ascending
+            x = (lower == up) ? min(x, y) : max(x, y);
+        }
+    }
+    return x;
+}
 
 template <typename T> __device__ __forceinline__ T warp_incl_scan(T v) {
 #pragma unroll

@@ -116,12 +116,17 @@ __global__ void k_mark_dst(const int32_t* __restrict__ dst_pos, const int32_t* _
 template <int LPR>
 __global__ void k_mark_new(const int32_t* __restrict__ dst_pos, const int32_t* __restrict__ row_mb,
                            const int64_t* cnt, const int64_t* __restrict__ findptr, const int32_t* __restrict__ fnbr,
-                           const uint32_t* __restrict__ dstbits, uint32_t* newbits, int64_t W) {
+                           const uint32_t* __restrict__ dstbits, uint32_t* newbits, int64_t W,
+                           const int64_t* __restrict__ otab) {
+    __shared__ int64_t s_vs[ORDER_SMEM + 1], s_rs[ORDER_SMEM];
+    const int nseg = order_load(otab, s_vs, s_rs);
+    int seg = 0;
     const int64_t n = cnt[0];
     const int sub = lane_id() % LPR;
     const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / LPR;
     const int64_t nw = ((int64_t)gridDim.x * blockDim.x) / LPR;
-    for (int64_t r = gw; r < n; r += nw) {
+    for (int64_t rv = gw; rv < n; rv += nw) {
+        const int64_t r = order_map(rv, nseg, s_vs, s_rs, seg);
         const int j = row_mb[r];
         const int32_t q = dst_pos[r];
         const int64_t b = findptr[q], e = findptr[q + 1];
@@ -214,12 +219,17 @@ __global__ void k_relabel(const int32_t* __restrict__ dst_pos, const int32_t* __
                           const uint32_t* __restrict__ newbits, const int64_t* __restrict__ wordoff, int64_t W,
                           const int32_t* __restrict__ map, int64_t map_stride, const int64_t* __restrict__ mb_dst_off,
                           const int64_t* __restrict__ mb_src_off, int32_t* __restrict__ indices, int64_t cap_e,
-                          const int32_t* __restrict__ fsrc_gid, int32_t* __restrict__ egid) {
+                          const int32_t* __restrict__ fsrc_gid, int32_t* __restrict__ egid,
+                          const int64_t* __restrict__ otab) {
+    __shared__ int64_t s_vs[ORDER_SMEM + 1], s_rs[ORDER_SMEM];
+    const int nseg = order_load(otab, s_vs, s_rs);
+    int seg = 0;
     const int64_t n = cnt[0];
     const int lane = lane_id() % LPR;
     const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / LPR;
     const int64_t nw = ((int64_t)gridDim.x * blockDim.x) / LPR;
-    for (int64_t r = gw; r < n; r += nw) {
+    for (int64_t rv = gw; rv < n; rv += nw) {
+        const int64_t r = order_map(rv, nseg, s_vs, s_rs, seg);
         const int j = row_mb[r];
         const int32_t q = dst_pos[r];
         const int64_t fb = findptr[q], fe = findptr[q + 1];
@@ -244,6 +254,44 @@ __global__ void k_relabel(const int32_t* __restrict__ dst_pos, const int32_t* __
             }
         }
     }
+}
+
+// single CTA: the micro-batch-major order table of layer l (extract.h); segment (j, p), j-major
+struct LayerPtrs { const int64_t* cnt[16]; const int64_t* off[16]; };
+__global__ void k_order_tab(int32_t c, int L, int l, const int64_t* __restrict__ top_off, LayerPtrs lp_,
+                            int64_t* tab) {
+    __shared__ int64_t s_warp[33];
+    const int P = L - l, nseg = c * P;
+    if (nseg > ORDER_TAB_MAX) {                         // too many segments: identity order
+        if (threadIdx.x == 0) tab[2 * (ORDER_TAB_MAX + 1)] = 0;
+        return;
+    }
+    int64_t* vs = tab;
+    int64_t* rs = tab + ORDER_TAB_MAX + 1;
+    __shared__ int64_t s_base;
+    if (threadIdx.x == 0) s_base = 0;
+    __syncthreads();
+    for (int i0 = 0; i0 < nseg; i0 += blockDim.x) {
+        const int i = i0 + threadIdx.x;
+        int64_t len = 0, start = 0;
+        if (i < nseg) {
+            const int j = i / P, p = i % P;
+            if (p == 0) { start = top_off[j]; len = top_off[j + 1] - top_off[j]; }
+            else {
+                const int lp = L - p;                   // new sources of layer lp
+                const int64_t* o = lp_.off[lp];
+                start = lp_.cnt[lp][0] + o[j];
+                len = o[j + 1] - o[j];
+            }
+        }
+        int64_t tot;
+        const int64_t ex = block_excl_scan(len, s_warp, &tot);
+        if (i < nseg) { vs[i] = s_base + ex; rs[i] = start; }
+        __syncthreads();
+        if (threadIdx.x == 0) s_base += tot;
+        __syncthreads();
+    }
+    if (threadIdx.x == 0) { vs[nseg] = s_base; tab[2 * (ORDER_TAB_MAX + 1)] = nseg; }
 }
 
 __global__ void k_clear_bits(uint32_t* a, uint32_t* b, int64_t n) {
@@ -287,6 +335,14 @@ void extract_group(betty_ctx* ctx, const ExtractArgs& a, cudaStream_t s) {
         const int64_t W = (F.n_src + 31) / 32;
         const int64_t cW = (int64_t)c * W;
         const int64_t cap_d = B.cap_dst, cap_e = B.cap_e, cap_s = B.cap_src;
+        // micro-batch-major visiting order of this layer's dst rows (needs only the layers above)
+        const int64_t* otab = nullptr;
+        if (l + 1 < a.L && B.order_tab) {
+            LayerPtrs lp{};
+            for (int q = 0; q < a.L; ++q) { lp.cnt[q] = a.layers[q].cnt; lp.off[q] = a.layers[q].mb_src_off; }
+            k_order_tab<<<1, 1024, 0, s>>>(c, a.L, l, a.sc.top_dst_off, lp, B.order_tab);
+            otab = B.order_tab;
+        }
         // rows: degree of each dst row in the full batch -> local indptr
         k_deg<<<grid_for(ctx, cap_d, 256), 256, 0, s>>>(dst_pos, F.indptr, B.cnt, a.sc.deg);
         scan_i64(ctx, a.sc.deg, B.indptr, B.cnt + 0, 0, cap_d, B.cnt + 2, s);
@@ -301,7 +357,7 @@ void extract_group(betty_ctx* ctx, const ExtractArgs& a, cudaStream_t s) {
         else if (lpr == 8) KERNEL<8><<<g_rows, 256, 0, s>>>(__VA_ARGS__);                   \
         else if (lpr == 16) KERNEL<16><<<g_rows, 256, 0, s>>>(__VA_ARGS__);                 \
         else KERNEL<32><<<g_rows, 256, 0, s>>>(__VA_ARGS__);
-        LPR_DISPATCH(k_mark_new, dst_pos, row_mb, B.cnt, F.indptr, F.nbr, a.sc.dstbits, a.sc.newbits, W)
+        LPR_DISPATCH(k_mark_new, dst_pos, row_mb, B.cnt, F.indptr, F.nbr, a.sc.dstbits, a.sc.newbits, W, otab)
         // ascending order of new sources = popcount scan over the bitmap words
         k_popc<<<grid_for(ctx, cW, 256), 256, 0, s>>>(a.sc.newbits, cW, a.sc.wordcnt);
         scan_i32(ctx, a.sc.wordcnt, a.sc.wordoff, nullptr, cW, 0, nullptr, s);
@@ -313,7 +369,7 @@ void extract_group(betty_ctx* ctx, const ExtractArgs& a, cudaStream_t s) {
                                                           F.src_gid, B.src_pos, B.src_gid, B.src_mb, cap_s);
         LPR_DISPATCH(k_relabel, dst_pos, row_mb, B.cnt, F.indptr, F.nbr, B.indptr, a.sc.dstbits, a.sc.newbits,
                      a.sc.wordoff, W, a.sc.map, a.sc.map_stride, dst_off, B.mb_src_off, B.indices, cap_e, F.src_gid,
-                     B.egid)
+                     B.egid, otab)
 #undef LPR_DISPATCH
         k_clear_bits<<<grid_for(ctx, cW, 256), 256, 0, s>>>(a.sc.dstbits, a.sc.newbits, cW);
         if (B.t_indptr && (a.csc_mask >> l & 1))

@@ -24,8 +24,49 @@ struct ExtractLayer {           // group-concatenated micro-batch layer l (devic
     int32_t* egid;              // [cap_e] or null: global id of each edge's source (feeds the layer-0 gather)
     int64_t* cnt;               // device [4]: n_dst, n_src, n_edges, spare
     int64_t* mb_src_off;        // [c+1]
+    int64_t* order_tab;         // [2*(ORDER_TAB_MAX+1)] or null: micro-batch-major dst row order (see below)
     int64_t cap_dst, cap_src, cap_e;
 };
+
+// Micro-batch-major processing order of the dst rows of a layer l < L-1.  The
+// group layout lists them as [top rows] ++ [new sources of layer L-1] ++ ... ++
+// [new sources of layer l+1], each phase grouped by micro-batch; kernels that
+// gather per dst row (the layer-0 aggregation) visit them micro-batch by
+// micro-batch so that one micro-batch's source rows stay L2-resident.  The
+// table holds the virtual starts vs[0..n_seg] (ascending, at [0]), the real
+// starts rs[0..n_seg) (at [ORDER_TAB_MAX+1]) and n_seg (at [2*(ORDER_TAB_MAX+1)]):
+// virtual row v in [vs[i], vs[i+1]) is real row rs[i] + (v - vs[i]).
+constexpr int ORDER_TAB_MAX = 1024;
+__host__ __device__ inline int order_tab_segs(int c, int L, int l) { return c * (L - l); }
+
+#ifdef __CUDACC__
+constexpr int ORDER_SMEM = 256;       // segments a kernel keeps in shared memory (more: identity order)
+// block-cooperative: copy the table into shared memory; returns n_seg (0 = identity order)
+__device__ __forceinline__ int order_load(const int64_t* otab, int64_t* s_vs, int64_t* s_rs) {
+    if (!otab) return 0;
+    int nseg = (int)otab[2 * (ORDER_TAB_MAX + 1)];
+    if (nseg > ORDER_SMEM) nseg = 0;
+    for (int i = threadIdx.x; i <= nseg; i += blockDim.x) {
+        s_vs[i] = otab[i];
+        if (i < nseg) s_rs[i] = otab[ORDER_TAB_MAX + 1 + i];
+    }
+    __syncthreads();
+    return nseg;
+}
+// virtual row -> real row; `seg` caches the last segment
+__device__ __forceinline__ int64_t order_map(int64_t vv, int nseg, const int64_t* s_vs, const int64_t* s_rs, int& seg) {
+    if (nseg == 0) return vv;
+    if (!(s_vs[seg] <= vv && vv < s_vs[seg + 1])) {
+        int lo = 0, hi = nseg;                          // s_vs[lo] <= vv < s_vs[hi]
+        while (hi - lo > 1) {
+            const int mid = (lo + hi) >> 1;
+            if (s_vs[mid] <= vv) lo = mid; else hi = mid;
+        }
+        seg = lo;
+    }
+    return s_rs[seg] + (vv - s_vs[seg]);
+}
+#endif
 
 struct ExtractScratch {
     uint32_t* dstbits;          // [c*Wmax]

@@ -122,11 +122,11 @@ static void launch_row(betty_ctx* c, const GemmRow& g, cudaStream_t s) {
     }
 }
 
-void gemm_row(betty_ctx* c, const GemmRow& g, cudaStream_t s) {
+bool gemm_row(betty_ctx* c, const GemmRow& g, cudaStream_t s) {
     if (c->use_tc && g.a_bf16 && g.b_bf16) {
         const void* Bk = g.transB ? g.B : g.Bt;
         const int64_t ldbk = g.transB ? g.ldb : g.ldbt;
-        if (Bk && gemm_row_tc(c, g, Bk, ldbk, s)) return;
+        if (Bk && gemm_row_tc(c, g, Bk, ldbk, s)) return g.epi == EPI_RELU_ONES && g.obits;
     }
     if (g.a_bf16) {
         if (g.b_bf16) launch_row<__nv_bfloat16, __nv_bfloat16>(c, g, s);
@@ -135,6 +135,7 @@ void gemm_row(betty_ctx* c, const GemmRow& g, cudaStream_t s) {
         if (g.b_bf16) launch_row<float, __nv_bfloat16>(c, g, s);
         else launch_row<float, float>(c, g, s);
     }
+    return false;
 }
 
 // ----------------------------------------------------------- reduction GEMM

@@ -106,86 +106,165 @@ __device__ __forceinline__ bool elect_lane0() { return (threadIdx.x & 31) == 0; 
 // B (the weights, <= 256 x K) stays resident in shared memory for the whole
 // persistent CTA; only A tiles stream through the TMA ring.  Eight epilogue
 // warps: warp w drains TMEM lanes 32*(w%4).. (tile rows) for one half of the
-// columns; each thread owns one output row and writes 16-byte vectors, with
-// the next chunk's TMEM load (and mask load) issued before the current chunk
-// is processed.
-constexpr int ROW_THREADS = 64 + 256;
+// columns, one output row per thread.  Each 32-column chunk goes TMEM ->
+// registers (epilogue math) -> a swizzled shared-memory staging slot -> TMA
+// bulk-tensor store, so the global writes are full-line, asynchronous and off
+// the epilogue's critical path.  The ReLU' mask of a backward layer comes as
+// one bit per element (written by the forward epilogue), 32 B per 256-wide row
+// instead of re-reading the bf16 activations.  The kernel is templated on the
+// epilogue so each 32-column chunk is straight-line code (~150 instructions).
+constexpr int EPI_WARPS = 8;
+constexpr int ESLOTS = 2;                       // staging slots per epilogue warp
+constexpr int ROW_THREADS = 64 + 32 * EPI_WARPS;
+constexpr int MAXCH = 4;                        // 32-column chunks per epilogue half (N <= 256)
 struct RowArgs {
     const int64_t* M_dev;
     int K, N, BN, nk, stages;
-    void* C; int64_t ldc; int c_bf16;
-    int epi;
-    const void* mask; int64_t ldm; int m_bf16;
+    void* C; int64_t ldc;
+    const void* mask; int64_t ldm; int m_bf16;  // EPI_MASK / EPI_RES_MASK from activations (MBITS = false)
+    const uint32_t* mbits; int64_t ldmb;        // ... or from ReLU bits (MBITS = true)
+    uint32_t* obits; int64_t ldob;              // EPI_RELU_ONES: ReLU bits out (words per row), or null
     const float* res; int64_t ldr; const int64_t* nres_dev;
     uint32_t tmem_cols;
-    int half_cols;           // columns per epilogue half (multiple of 32)
+    int acc_stride;          // TMEM columns between the two accumulators (>= BN, multiple of 32)
+    int half_cols;           // columns per epilogue half (multiple of 32, <= 32 * MAXCH)
+    uint32_t slot_bytes;     // one staging slot: 32 rows x 32 columns
 };
 
 __device__ __forceinline__ uint32_t pack_bf16x2(float a, float b) {
     __nv_bfloat162 h = __floats2bfloat162_rn(a, b);
     return *(uint32_t*)&h;
 }
+__device__ __forceinline__ void tma_store_2d(const CUtensorMap* tm, const void* src, int c0, int c1) {
+    asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%1, %2}], [%3];"
+                 ::"l"((uint64_t)tm), "r"(c0), "r"(c1), "r"(su32(src)) : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+template <int N> __device__ __forceinline__ void bulk_wait_read() {
+    asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory");
+}
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 
-// one 32-column chunk of one row: epilogue math + vector stores
-__device__ __forceinline__ void row_chunk_out(const RowArgs& p, float* v, int64_t m, int c0, const uint4* mk,
-                                              int64_t nres) {
-    const int nval = min(32, p.N - c0);            // valid output columns in this chunk
-    if (nval <= 0) return;
+__device__ __forceinline__ void tmem_ld32_nowait(uint32_t taddr, uint32_t* r) {
+    asm volatile("tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+                 "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+                 : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+                   "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]),
+                   "=r"(r[15]), "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]),
+                   "=r"(r[22]), "=r"(r[23]), "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]),
+                   "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
+                 : "r"(taddr));
+}
+// tcgen05.wait::ld that the compiler cannot move reads of r across
+__device__ __forceinline__ void tmem_wait_regs(uint32_t* r) {
+    asm volatile("tcgen05.wait::ld.sync.aligned;"
+                 : "+r"(r[0]), "+r"(r[1]), "+r"(r[2]), "+r"(r[3]), "+r"(r[4]), "+r"(r[5]), "+r"(r[6]), "+r"(r[7]),
+                   "+r"(r[8]), "+r"(r[9]), "+r"(r[10]), "+r"(r[11]), "+r"(r[12]), "+r"(r[13]), "+r"(r[14]),
+                   "+r"(r[15]), "+r"(r[16]), "+r"(r[17]), "+r"(r[18]), "+r"(r[19]), "+r"(r[20]), "+r"(r[21]),
+                   "+r"(r[22]), "+r"(r[23]), "+r"(r[24]), "+r"(r[25]), "+r"(r[26]), "+r"(r[27]), "+r"(r[28]),
+                   "+r"(r[29]), "+r"(r[30]), "+r"(r[31])
+                 :
+                 : "memory");
+}
+
+// [activation > 0] of a stored 32-column chunk (mask from activations, MBITS = false)
+__device__ __forceinline__ uint32_t mask_word_from_act(const RowArgs& p, int64_t m, int c0, bool ok) {
+    if (!ok) return 0u;
+    uint32_t w = 0;
+    const int nval = min(32, p.N - c0);
+    if (p.m_bf16) {
+        const uint4* src = (const uint4*)((const __nv_bfloat16*)p.mask + m * p.ldm + c0);
 #pragma unroll
-    for (int j = 0; j < 32; ++j) {
-        float x = v[j];
-        if (p.epi == EPI_RELU_ONES) x = fmaxf(x, 0.f);
-        if (p.epi == EPI_RES_MASK && m < nres && j < nval) x += p.res[m * p.ldr + c0 + j];
-        if (p.epi == EPI_MASK || p.epi == EPI_RES_MASK) {
-            float mv;
-            if (p.m_bf16) {
-                const __nv_bfloat16* hb = (const __nv_bfloat16*)&mk[j / 8];
-                mv = __bfloat162float(hb[j % 8]);
-            } else {
-                mv = ((const float*)&mk[j / 4])[j % 4];
+        for (int q = 0; q < 4; ++q) {
+            if (q * 8 >= nval) break;
+            const uint4 t = src[q];
+            const uint32_t u[4] = {t.x, t.y, t.z, t.w};
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+                const __nv_bfloat162 h = *(const __nv_bfloat162*)&u[k];
+                w |= (uint32_t)(__low2float(h) > 0.f) << (8 * q + 2 * k);
+                w |= (uint32_t)(__high2float(h) > 0.f) << (8 * q + 2 * k + 1);
             }
-            if (!(mv > 0.f)) x = 0.f;
-        }
-        v[j] = x;
-    }
-    if (p.c_bf16) {
-        __nv_bfloat16* cp = (__nv_bfloat16*)p.C + m * p.ldc + c0;
-        if (nval == 32 && (p.ldc & 7) == 0) {
-#pragma unroll
-            for (int q = 0; q < 4; ++q)
-                ((uint4*)cp)[q] = make_uint4(pack_bf16x2(v[8 * q], v[8 * q + 1]), pack_bf16x2(v[8 * q + 2], v[8 * q + 3]),
-                                             pack_bf16x2(v[8 * q + 4], v[8 * q + 5]),
-                                             pack_bf16x2(v[8 * q + 6], v[8 * q + 7]));
-        } else {
-#pragma unroll
-            for (int j = 0; j < 32; ++j)
-                if (j < nval) cp[j] = __float2bfloat16_rn(v[j]);
         }
     } else {
-        float* cp = (float*)p.C + m * p.ldc + c0;
-        if (nval == 32 && (p.ldc & 3) == 0) {
+        const float4* src = (const float4*)((const float*)p.mask + m * p.ldm + c0);
 #pragma unroll
-            for (int q = 0; q < 8; ++q) ((float4*)cp)[q] = make_float4(v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
-        } else {
-#pragma unroll
-            for (int j = 0; j < 32; ++j)
-                if (j < nval) cp[j] = v[j];
+        for (int q = 0; q < 8; ++q) {
+            if (q * 4 >= nval) break;
+            const float4 t = src[q];
+            w |= (uint32_t)(t.x > 0.f) << (4 * q) | (uint32_t)(t.y > 0.f) << (4 * q + 1) |
+                 (uint32_t)(t.z > 0.f) << (4 * q + 2) | (uint32_t)(t.w > 0.f) << (4 * q + 3);
         }
     }
+    if (nval < 32) w &= (1u << nval) - 1u;
+    return w;
 }
 
-__device__ __forceinline__ void load_mask_chunk(const RowArgs& p, int64_t m, int c0, bool ok, uint4* mk) {
-    const int nv = p.m_bf16 ? 4 : 8;                // 16-byte vectors per 32 columns
-    if (!ok) return;
-    const char* base = (const char*)p.mask + (m * p.ldm + c0) * (p.m_bf16 ? 2 : 4);
-    const int64_t rowbytes = (int64_t)(p.N - c0) * (p.m_bf16 ? 2 : 4);
+// one 32-column chunk: epilogue math on v (fp32 bits in r), staged for the TMA store.
+// Returns the ReLU bits (EPI_RELU_ONES).
+template <int EPI, bool CBF>
+__device__ __forceinline__ uint32_t chunk_epilogue(const RowArgs& p, const uint32_t* r, int64_t m, int c0, bool ok,
+                                                   uint32_t mword, int64_t nres, uint8_t* slot, int lane) {
+    float v[32];
 #pragma unroll
-    for (int q = 0; q < 8; ++q)
-        if (q < nv && q * 16 < rowbytes) mk[q] = __ldg((const uint4*)(base + q * 16));
+    for (int j = 0; j < 32; ++j) v[j] = __uint_as_float(r[j]);
+    if (EPI == EPI_RES_MASK && ok && m < nres) {
+        const float* rp = p.res + m * p.ldr + c0;
+        const int nval = min(32, p.N - c0);
+#pragma unroll
+        for (int q = 0; q < 8; ++q) {
+            if (q * 4 < nval) {
+                const float4 t = *(const float4*)(rp + 4 * q);
+                v[4 * q] += t.x; v[4 * q + 1] += t.y; v[4 * q + 2] += t.z; v[4 * q + 3] += t.w;
+            }
+        }
+    }
+    if (EPI == EPI_MASK || EPI == EPI_RES_MASK) {
+#pragma unroll
+        for (int j = 0; j < 32; ++j) v[j] = ((mword >> j) & 1u) ? v[j] : 0.f;
+    }
+    if (EPI == EPI_RELU_ONES) {
+#pragma unroll
+        for (int j = 0; j < 32; ++j) v[j] = fmaxf(v[j], 0.f);
+    }
+    if (!ok) {
+#pragma unroll
+        for (int j = 0; j < 32; ++j) v[j] = 0.f;
+    }
+    uint32_t bits = 0;
+    if (CBF) {
+        uint32_t w[16];
+#pragma unroll
+        for (int k = 0; k < 16; ++k) w[k] = pack_bf16x2(v[2 * k], v[2 * k + 1]);
+        if (EPI == EPI_RELU_ONES) {     // bit = [stored bf16 value > 0] (ReLU output: non-negative)
+#pragma unroll
+            for (int k = 0; k < 16; ++k)
+                bits |= (uint32_t)((w[k] & 0x7fffu) != 0u) << (2 * k) | (uint32_t)((w[k] & 0x7fff0000u) != 0u) << (2 * k + 1);
+        }
+        // 64 B rows, SWIZZLE_64B: 16-B chunk c of row r at c ^ ((r >> 1) & 3)
+        uint8_t* row = slot + lane * 64;
+#pragma unroll
+        for (int c = 0; c < 4; ++c)
+            *(uint4*)(row + ((c ^ ((lane >> 1) & 3)) << 4)) = make_uint4(w[4 * c], w[4 * c + 1], w[4 * c + 2], w[4 * c + 3]);
+    } else {
+        if (EPI == EPI_RELU_ONES) {
+#pragma unroll
+            for (int j = 0; j < 32; ++j) bits |= (uint32_t)(v[j] > 0.f) << j;
+        }
+        // 128 B rows, SWIZZLE_128B: 16-B chunk c of row r at c ^ (r & 7)
+        uint8_t* row = slot + lane * 128;
+#pragma unroll
+        for (int c = 0; c < 8; ++c)
+            *(float4*)(row + ((c ^ (lane & 7)) << 4)) = make_float4(v[4 * c], v[4 * c + 1], v[4 * c + 2], v[4 * c + 3]);
+    }
+    return bits;
 }
 
+template <int EPI, bool CBF, bool MBITS>
 __global__ void __launch_bounds__(ROW_THREADS, 1) k_tc_row(const __grid_constant__ CUtensorMap tmA,
-                                                           const __grid_constant__ CUtensorMap tmB, RowArgs p) {
+                                                           const __grid_constant__ CUtensorMap tmB,
+                                                           const __grid_constant__ CUtensorMap tmC, RowArgs p) {
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
     const int S = p.stages;
@@ -193,7 +272,8 @@ __global__ void __launch_bounds__(ROW_THREADS, 1) k_tc_row(const __grid_constant
     const uint32_t bblk = (uint32_t)p.BN * BK * 2;          // one K-block of the resident B
     uint8_t* bres = smem;                                    // nk * bblk
     uint8_t* aring = smem + p.nk * bblk;                     // S * a_bytes
-    uint64_t* full = (uint64_t*)(aring + S * a_bytes);
+    uint8_t* stage = aring + S * a_bytes;                    // EPI_WARPS * ESLOTS * slot_bytes
+    uint64_t* full = (uint64_t*)(stage + EPI_WARPS * ESLOTS * p.slot_bytes);
     uint64_t* empty = full + S;
     uint64_t* tfull = empty + S;      // [2]
     uint64_t* tempty = tfull + 2;     // [2]
@@ -206,11 +286,12 @@ __global__ void __launch_bounds__(ROW_THREADS, 1) k_tc_row(const __grid_constant
 
     if (threadIdx.x == 0) {
         for (int s = 0; s < S; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
-        for (int a = 0; a < 2; ++a) { mbar_init(&tfull[a], 1); mbar_init(&tempty[a], 256); }
+        for (int a = 0; a < 2; ++a) { mbar_init(&tfull[a], 1); mbar_init(&tempty[a], 32 * EPI_WARPS); }
         mbar_init(bfull, 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
         asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmA) : "memory");
         asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmB) : "memory");
+        asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmC) : "memory");
     }
     if (warp == 1) tmem_alloc_warp(tslot, p.tmem_cols);
     fence_before();
@@ -244,7 +325,7 @@ __global__ void __launch_bounds__(ROW_THREADS, 1) k_tc_row(const __grid_constant
             const uint32_t aph = (it >> 1) & 1;
             mbar_wait(&tempty[acc], aph ^ 1);
             fence_after();
-            const uint32_t d = tmem + acc * p.BN;
+            const uint32_t d = tmem + acc * p.acc_stride;
             for (int kb = 0; kb < p.nk; ++kb) {
                 mbar_wait(&full[s], ph);
                 fence_after();
@@ -264,66 +345,94 @@ __global__ void __launch_bounds__(ROW_THREADS, 1) k_tc_row(const __grid_constant
             }
         }
     } else {
+        constexpr bool HAS_MASK = EPI == EPI_MASK || EPI == EPI_RES_MASK;
         const int ew = warp - 2;                 // 0..7
         const int q = warp & 3;                  // TMEM lane quadrant (hardware: warp id % 4)
         const int h = ew >> 2;                   // column half
         const int lane = threadIdx.x & 31;
         const int cbeg = h * p.half_cols;
-        const int cend = min(p.BN, cbeg + p.half_cols);
-        const bool has_mask = p.epi == EPI_MASK || p.epi == EPI_RES_MASK;
-        const int64_t nres = (p.epi == EPI_RES_MASK) ? *p.nres_dev : 0;
+        const int cstore = min(min(p.BN, cbeg + p.half_cols), p.N);   // chunks at or past N are not stored
+        const int nch = cstore > cbeg ? (cstore - cbeg + 31) / 32 : 0;
+        const int64_t nres = EPI == EPI_RES_MASK ? *p.nres_dev : 0;
+        uint8_t* my_stage = stage + ew * ESLOTS * p.slot_bytes;
+        int slot = 0;
         int it = 0;
         for (int64_t t = blockIdx.x; t < tiles; t += gridDim.x, ++it) {
             const int acc = it & 1;
             const uint32_t aph = (it >> 1) & 1;
-            const int64_t m = t * BM + q * 32 + lane;
+            const int64_t row0 = t * BM + q * 32;
+            const int64_t m = row0 + lane;
             const bool ok = m < M;
-            uint4 mk[8], mk_next[8];
-            if (has_mask && cbeg < cend) load_mask_chunk(p, m, cbeg, ok, mk);
+            // mask words of this thread's chunks, loaded before the accumulator wait (latency hidden)
+            uint32_t mw[MAXCH];
+#pragma unroll
+            for (int ci = 0; ci < MAXCH; ++ci) mw[ci] = 0u;
+            if (HAS_MASK) {
+                if (MBITS) {
+                    if (ok) {
+                        const uint32_t* wb = p.mbits + m * p.ldmb + cbeg / 32;
+#pragma unroll
+                        for (int ci = 0; ci < MAXCH; ++ci) if (ci < nch) mw[ci] = wb[ci];
+                    }
+                } else {
+#pragma unroll
+                    for (int ci = 0; ci < MAXCH; ++ci) if (ci < nch) mw[ci] = mask_word_from_act(p, m, cbeg + 32 * ci, ok);
+                }
+            }
             mbar_wait(&tfull[acc], aph);
             fence_after();
-            const uint32_t tbase = tmem + ((uint32_t)(q * 32) << 16) + acc * p.BN;
-            float v[32];
-            if (cbeg < cend) tmem_ld32(tbase + cbeg, v);
-            for (int c0 = cbeg; c0 < cend; c0 += 32) {
-                const bool more = c0 + 32 < cend;
-                float nx[32];
-                if (more) {
-                    // next chunk's TMEM load in flight while this chunk is stored
-                    uint32_t r[32];
-                    asm volatile("tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,"
-                                 "%13,%14,%15,%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
-                                 : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
-                                   "=r"(r[7]), "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]),
-                                   "=r"(r[13]), "=r"(r[14]), "=r"(r[15]), "=r"(r[16]), "=r"(r[17]), "=r"(r[18]),
-                                   "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]), "=r"(r[24]),
-                                   "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]),
-                                   "=r"(r[31])
-                                 : "r"(tbase + c0 + 32));
+            const uint32_t tbase = tmem + ((uint32_t)(q * 32) << 16) + acc * p.acc_stride;
+            uint32_t ra[32], rb[32];
+            uint32_t obits[MAXCH];
+            if (nch > 0) { tmem_ld32_nowait(tbase + cbeg, ra); tmem_wait_regs(ra); }
 #pragma unroll
-                    for (int j = 0; j < 32; ++j) nx[j] = __uint_as_float(r[j]);
-                    if (has_mask) load_mask_chunk(p, m, c0 + 32, ok, mk_next);
-                }
-                if (ok) row_chunk_out(p, v, m, c0, mk, nres);
-                if (more) {
-                    asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
-#pragma unroll
-                    for (int j = 0; j < 32; ++j) v[j] = nx[j];
-#pragma unroll
-                    for (int q2 = 0; q2 < 8; ++q2) mk[q2] = mk_next[q2];
+            for (int ci = 0; ci < MAXCH; ++ci) {
+                obits[ci] = 0u;
+                if (ci < nch) {
+                    uint32_t* cur = (ci & 1) ? rb : ra;
+                    uint32_t* nxt = (ci & 1) ? ra : rb;
+                    const int c0 = cbeg + 32 * ci;
+                    if (ci + 1 < nch) tmem_ld32_nowait(tbase + c0 + 32, nxt);   // next chunk in flight
+                    uint8_t* sl = my_stage + slot * p.slot_bytes;
+                    if (lane == 0) bulk_wait_read<ESLOTS - 1>();    // the store that used this slot has read it
+                    __syncwarp();
+                    obits[ci] = chunk_epilogue<EPI, CBF>(p, cur, m, c0, ok, mw[ci], nres, sl, lane);
+                    fence_proxy_async();
+                    __syncwarp();
+                    if (lane == 0) {
+                        tma_store_2d(&tmC, sl, c0, (int)row0);
+                        bulk_commit();
+                    }
+                    if (++slot == ESLOTS) slot = 0;
+                    if (ci + 1 < nch) tmem_wait_regs(nxt);
                 }
             }
             fence_before();
             mbar_arrive(&tempty[acc]);
+            if (EPI == EPI_RELU_ONES && p.obits && ok && nch > 0) {
+                uint32_t* ob = p.obits + m * p.ldob + cbeg / 32;
+                if (nch == 4 && ((uintptr_t)ob & 15) == 0)
+                    *(uint4*)ob = make_uint4(obits[0], obits[1], obits[2], obits[3]);
+                else
+#pragma unroll
+                    for (int ci = 0; ci < MAXCH; ++ci) if (ci < nch) ob[ci] = obits[ci];
+            }
             // trailing columns [N, ldc): the ones column after a ReLU layer, zeros elsewhere
             if (h == 1 && ok && p.ldc > p.N) {
-                for (int col = p.N; col < p.ldc; ++col) {
-                    const float x = (p.epi == EPI_RELU_ONES && col == p.N) ? 1.f : 0.f;
-                    if (p.c_bf16) ((__nv_bfloat16*)p.C)[m * p.ldc + col] = __float2bfloat16_rn(x);
-                    else ((float*)p.C)[m * p.ldc + col] = x;
+                const int w = (int)(p.ldc - p.N);
+                if (CBF && w == 8 && ((m * p.ldc + p.N) & 7) == 0) {
+                    const uint32_t one = EPI == EPI_RELU_ONES ? 0x3F80u : 0u;
+                    *(uint4*)((__nv_bfloat16*)p.C + m * p.ldc + p.N) = make_uint4(one, 0u, 0u, 0u);
+                } else {
+                    for (int col = p.N; col < p.ldc; ++col) {
+                        const float x = (EPI == EPI_RELU_ONES && col == p.N) ? 1.f : 0.f;
+                        if (CBF) ((__nv_bfloat16*)p.C)[m * p.ldc + col] = __float2bfloat16_rn(x);
+                        else ((float*)p.C)[m * p.ldc + col] = x;
+                    }
                 }
             }
         }
+        if (lane == 0) bulk_wait_all();
     }
     __syncthreads();
     if (warp == 1) {
@@ -463,17 +572,24 @@ static EncodeFn encode_fn() {
     return fn;
 }
 
-// 2-D bf16 tensor [rows x cols] with row stride ld (elements); box {64 cols, box_rows}
-static bool make_map(CUtensorMap* m, const void* base, int64_t cols, int64_t rows, int64_t ld, int box_rows) {
+// 2-D tensor [rows x cols] with row stride ld (elements); box {box_cols, box_rows}
+static bool make_map_t(CUtensorMap* m, const void* base, bool f32, int64_t cols, int64_t rows, int64_t ld,
+                       int box_cols, int box_rows, CUtensorMapSwizzle sw) {
     EncodeFn f = encode_fn();
     if (!f) return false;
+    const int es = f32 ? 4 : 2;
+    if (((uintptr_t)base & 15) || (ld * es) % 16) return false;
     cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)rows};
-    cuuint64_t strides[1] = {(cuuint64_t)ld * 2};
-    cuuint32_t box[2] = {64, (cuuint32_t)box_rows};
-    cuuint32_t es[2] = {1, 1};
-    return f(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base), dims, strides, box, es,
-             CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+    cuuint64_t strides[1] = {(cuuint64_t)ld * es};
+    cuuint32_t box[2] = {(cuuint32_t)box_cols, (cuuint32_t)box_rows};
+    cuuint32_t estr[2] = {1, 1};
+    return f(m, f32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base),
+             dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, sw, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+// bf16 operand maps: box {64 cols (128 B), box_rows}, 128-byte swizzle
+static bool make_map(CUtensorMap* m, const void* base, int64_t cols, int64_t rows, int64_t ld, int box_rows) {
+    return make_map_t(m, base, false, cols, rows, ld, 64, box_rows, CU_TENSOR_MAP_SWIZZLE_128B);
 }
 
 static uint32_t tmem_cols_for(int n) {
@@ -490,32 +606,62 @@ bool tc_available() { return tc::encode_fn() != nullptr; }
 bool gemm_row_tc(betty_ctx* c, const GemmRow& g, const void* Bk, int64_t ldbk, cudaStream_t s) {
     using namespace tc;
     if (!g.a_bf16 || !g.b_bf16 || g.N > 256 || g.N < 1 || (g.lda & 7) || (ldbk & 7)) return false;
-    if ((g.epi == EPI_MASK || g.epi == EPI_RES_MASK) && (g.ldm & 7)) return false;
+    if ((g.epi == EPI_MASK || g.epi == EPI_RES_MASK) && !g.mbits && (g.ldm & 7)) return false;
     const int BN = (g.N + 15) / 16 * 16;
     const int nk = (g.K + BK - 1) / BK;
     const size_t b_bytes = (size_t)nk * BN * BK * 2;
     const size_t a_bytes = BM * BK * 2;
-    const size_t budget = 220 * 1024;
-    if (b_bytes + 2 * a_bytes + 2048 > budget) return false;       // B must fit resident
-    CUtensorMap ma, mb;
+    const uint32_t slot_bytes = 32 * 32 * (g.c_bf16 ? 2 : 4);
+    const size_t stage_bytes = (size_t)EPI_WARPS * ESLOTS * slot_bytes;
+    const size_t budget = 225 * 1024;
+    if (b_bytes + stage_bytes + 2 * a_bytes + 1024 + 256 > budget) return false;   // B must fit resident
+    CUtensorMap ma, mb, mc;
     if (!make_map(&ma, g.A, g.K, g.M_cap, g.lda, BM) || !make_map(&mb, Bk, g.K, g.N, ldbk, BN)) return false;
+    if (!make_map_t(&mc, g.C, !g.c_bf16, g.N, g.M_cap, g.ldc, 32, 32,
+                    g.c_bf16 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_128B))
+        return false;
     RowArgs p{};
     p.M_dev = g.M_dev; p.K = g.K; p.N = g.N; p.BN = BN; p.nk = nk;
-    p.stages = (int)std::max<size_t>(2, std::min<size_t>(8, (budget - b_bytes - 2048) / a_bytes));
-    p.C = g.C; p.ldc = g.ldc; p.c_bf16 = g.c_bf16; p.epi = g.epi;
+    p.stages = (int)std::max<size_t>(2, std::min<size_t>(8, (budget - 1024 - 256 - b_bytes - stage_bytes) / a_bytes));
+    p.C = g.C; p.ldc = g.ldc;
     p.mask = g.mask; p.ldm = g.ldm; p.m_bf16 = g.m_bf16; p.res = g.res; p.ldr = g.ldr; p.nres_dev = g.nres_dev;
-    p.tmem_cols = tmem_cols_for(2 * BN);
+    p.mbits = g.mbits; p.ldmb = g.ldmb;
+    p.obits = g.epi == EPI_RELU_ONES ? g.obits : nullptr; p.ldob = g.ldob;
+    p.acc_stride = (BN + 31) / 32 * 32;
+    p.tmem_cols = tmem_cols_for(2 * p.acc_stride);
     p.half_cols = ((BN + 63) / 64) * 32;
-    if (p.tmem_cols > 512) return false;
-    const size_t smem = b_bytes + (size_t)p.stages * a_bytes + 1024 + 256;
-    static bool attr = false;
-    if (!attr) {
-        cudaFuncSetAttribute(k_tc_row, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
-        attr = true;
-    }
+    p.slot_bytes = slot_bytes;
+    if (p.tmem_cols > 512 || p.half_cols > 32 * MAXCH) return false;
+    const size_t smem = b_bytes + (size_t)p.stages * a_bytes + stage_bytes + 1024 + 256;
     const int64_t tiles = (g.M_cap + BM - 1) / BM;
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(tiles, c->num_sms));
-    k_tc_row<<<grid, ROW_THREADS, smem, s>>>(ma, mb, p);
+    const bool usebits = g.mbits != nullptr;
+#define ROW_LAUNCH(E, CB, MB)                                                                      \
+    do {                                                                                           \
+        static bool attr = false;                                                                  \
+        if (!attr) {                                                                               \
+            cudaFuncSetAttribute(k_tc_row<E, CB, MB>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024); \
+            attr = true;                                                                           \
+        }                                                                                          \
+        k_tc_row<E, CB, MB><<<grid, ROW_THREADS, smem, s>>>(ma, mb, mc, p);                       \
+    } while (0)
+    switch (g.epi) {
+    case EPI_STORE:
+        if (g.c_bf16) ROW_LAUNCH(EPI_STORE, true, false); else ROW_LAUNCH(EPI_STORE, false, false);
+        break;
+    case EPI_RELU_ONES:
+        if (g.c_bf16) ROW_LAUNCH(EPI_RELU_ONES, true, false); else ROW_LAUNCH(EPI_RELU_ONES, false, false);
+        break;
+    case EPI_MASK:
+        if (g.c_bf16) { if (usebits) ROW_LAUNCH(EPI_MASK, true, true); else ROW_LAUNCH(EPI_MASK, true, false); }
+        else { if (usebits) ROW_LAUNCH(EPI_MASK, false, true); else ROW_LAUNCH(EPI_MASK, false, false); }
+        break;
+    default:
+        if (g.c_bf16) { if (usebits) ROW_LAUNCH(EPI_RES_MASK, true, true); else ROW_LAUNCH(EPI_RES_MASK, true, false); }
+        else { if (usebits) ROW_LAUNCH(EPI_RES_MASK, false, true); else ROW_LAUNCH(EPI_RES_MASK, false, false); }
+        break;
+    }
+#undef ROW_LAUNCH
     return true;
 }
 

@@ -45,12 +45,16 @@ struct BlockView {              // one layer of a (group-concatenated) micro-bat
     const int64_t* cnt;         // device [3]: n_dst, n_src, n_edges
     int64_t cap_dst, cap_src, cap_e;
     const int32_t* egid = nullptr;   // optional [n_edges]: global id of each edge's source (layer 0)
+    const int64_t* order_tab = nullptr;   // optional micro-batch-major dst row order (extract.h)
 };
 
 struct LayerBufs {
     void* XA = nullptr;   void* gat = nullptr;  float* Y = nullptr;   void* G = nullptr;
     float* dXA = nullptr; float* Zp = nullptr;  int32_t* arg = nullptr; void* dZp = nullptr;
     void* H = nullptr;    // input of layer l (l >= 1), written by layer l-1
+    uint32_t* Hbits = nullptr;   // [H > 0] as bits (ldhb words per row), written with H by a tensor-core epilogue
+    int64_t ldhb = 0;
+    bool hbits_ok = false;       // Hbits holds the current H (set by the forward)
     void* dS = nullptr;   // dS of layer l as GEMM operand (l < L-1)
     void* B = nullptr;    void* Bp = nullptr;
     void* Bt = nullptr;   void* Bpt = nullptr;   // K-major weight copies (BF16 tensor-core path)

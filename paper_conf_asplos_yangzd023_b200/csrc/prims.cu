@@ -49,25 +49,41 @@ __global__ void __launch_bounds__(SCAN_THREADS) k_scan(const Tin* __restrict__ i
         }
         int64_t agg;
         const int64_t ex = block_excl_scan(sum, s_warp, &agg);
-        if (threadIdx.x == 0) {
+        if (threadIdx.x < 32) {
+            // warp-parallel decoupled look-back: inspect the 32 predecessor tiles at
+            // once, add the aggregates after the nearest inclusive prefix, repeat
+            // further back only while no prefix is found
+            const int lane = threadIdx.x;
             int64_t prefix = 0;
             if (t == 0) {
-                st_release(&status[0], ST_PRE | (unsigned long long)agg);
+                if (lane == 0) st_release(&status[0], ST_PRE | (unsigned long long)agg);
             } else {
-                st_release(&status[t], ST_AGG | (unsigned long long)agg);
-                for (int64_t j = t - 1;;) {
-                    const unsigned long long s = ld_acquire(&status[j]);
-                    const unsigned long long f = s >> 62;
-                    if (f == 0) continue;                     // predecessor not published yet
-                    prefix += (int64_t)(s & ST_VAL);
-                    if (f == 2) break;
-                    --j;
+                if (lane == 0) st_release(&status[t], ST_AGG | (unsigned long long)agg);
+                int64_t hi = t - 1;                          // window [hi-31, hi]
+                for (;;) {
+                    const int64_t j = hi - lane;
+                    unsigned long long st = j >= 0 ? ld_acquire(&status[j]) : (ST_PRE | 0ull);
+                    // wait until every tile of the window has published something
+                    while (__any_sync(0xffffffffu, (st >> 62) == 0)) {
+                        if ((st >> 62) == 0) st = ld_acquire(&status[j]);
+                    }
+                    const unsigned pre = __ballot_sync(0xffffffffu, (st >> 62) == 2);
+                    // lanes up to and including the nearest PRE (lowest lane index with PRE) contribute
+                    const int stop = pre ? __ffs(pre) - 1 : 31;
+                    int64_t v = lane <= stop ? (int64_t)(st & ST_VAL) : 0;
+#pragma unroll
+                    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+                    prefix += v;
+                    if (pre) break;
+                    hi -= 32;
                 }
-                st_release(&status[t], ST_PRE | (unsigned long long)(prefix + agg));
+                if (lane == 0) st_release(&status[t], ST_PRE | (unsigned long long)(prefix + agg));
             }
-            s_prefix = prefix;
-            if (t == n_tiles - 1 && total_dev) *total_dev = prefix + agg;
-            if (t == 0) out[0] = 0;
+            if (lane == 0) {
+                s_prefix = prefix;
+                if (t == n_tiles - 1 && total_dev) *total_dev = prefix + agg;
+                if (t == 0) out[0] = 0;
+            }
         }
         __syncthreads();
         int64_t run = s_prefix + ex;
@@ -147,22 +163,6 @@ void memset_dev(void* p, int value, const int64_t* n_dev, int64_t elem_bytes, in
 constexpr int SEG_WARP_MAX = 512;
 constexpr int SEG_CTA_MAX = 32768;
 
-__device__ __forceinline__ int32_t warp_bitonic32(int32_t x) {
-    const int lane = lane_id();
-#pragma unroll
-    for (int k = 2; k <= 32; k <<= 1) {
-#pragma unroll
-        for (int j = k >> 1; j > 0; j >>= 1) {
-            const int32_t y = __shfl_xor_sync(0xffffffffu, x, j);
-            const bool up = ((lane & k) == 0);
-            const bool lower = ((lane & j) == 0);
-            // lower element keeps min when ascending
-            x = (lower == up) ? min(x, y) : max(x, y);
-        }
-    }
-    return x;
-}
-
 __device__ void smem_bitonic(int32_t* s, int P, int tid, int nthreads, bool warp_only) {
     for (int k = 2; k <= P; k <<= 1) {
         for (int j = k >> 1; j > 0; j >>= 1) {
@@ -186,24 +186,48 @@ __global__ void __launch_bounds__(256) k_segsort_warp(const int64_t* __restrict_
     const int64_t nseg = nseg_dev ? *nseg_dev : nseg_fixed;
     const int w = warp_id(), lane = lane_id();
     const int64_t gw = blockIdx.x * 8ll + w, nw = gridDim.x * 8ll;
-    for (int64_t seg = gw; seg < nseg; seg += nw) {
-        const int64_t b = ptr[seg], len = ptr[seg + 1] - b;
-        if (len <= 1) continue;
-        if (len <= 32) {
-            int32_t x = lane < len ? keys[b + lane] : INT_MAX;
-            x = warp_bitonic32(x);
-            if (lane < len) keys[b + lane] = x;
-        } else if (len <= SEG_WARP_MAX) {
-            int P = 64;
-            while (P < len) P <<= 1;
-            for (int i = lane; i < P; i += 32) buf[w][i] = i < len ? keys[b + i] : INT_MAX;
-            __syncwarp();
-            smem_bitonic(buf[w], P, lane, 32, true);
-            for (int i = lane; i < len; i += 32) keys[b + i] = buf[w][i];
-            __syncwarp();
-        } else if (lane == 0) {
-            const int i = atomicAdd(big_cnt, 1);
-            if (i < big_cap) big[i] = seg; else atomicOr(dev_err, DEVERR_OVERFLOW);
+    // a warp takes 32 consecutive segments: segments of <= SEG_THREAD_MAX keys are
+    // insertion-sorted by one lane each (most CSC columns of a sampled block hold
+    // 1-4 entries); longer ones are sorted warp-cooperatively one at a time
+    constexpr int SEG_THREAD_MAX = 8;
+    for (int64_t s0 = gw * 32; s0 < nseg; s0 += nw * 32) {
+        const int64_t my = s0 + lane;
+        int64_t mb = 0, ml = 0;
+        if (my < nseg) { mb = ptr[my]; ml = ptr[my + 1] - mb; }
+        if (ml > 1 && ml <= SEG_THREAD_MAX) {
+            int32_t k[SEG_THREAD_MAX];
+#pragma unroll
+            for (int i = 0; i < SEG_THREAD_MAX; ++i) k[i] = i < ml ? keys[mb + i] : INT_MAX;
+#pragma unroll
+            for (int i = 1; i < SEG_THREAD_MAX; ++i)
+#pragma unroll
+                for (int j = i; j > 0; --j)
+                    if (k[j] < k[j - 1]) { const int32_t t = k[j]; k[j] = k[j - 1]; k[j - 1] = t; }
+#pragma unroll
+            for (int i = 0; i < SEG_THREAD_MAX; ++i) if (i < ml) keys[mb + i] = k[i];
+        }
+        unsigned long_mask = __ballot_sync(0xffffffffu, ml > SEG_THREAD_MAX);
+        while (long_mask) {
+            const int src = __ffs(long_mask) - 1;
+            long_mask &= long_mask - 1;
+            const int64_t seg = s0 + src;
+            const int64_t b = __shfl_sync(0xffffffffu, mb, src), len = __shfl_sync(0xffffffffu, ml, src);
+            if (len <= 32) {
+                int32_t x = lane < len ? keys[b + lane] : INT_MAX;
+                x = warp_bitonic32(x);
+                if (lane < len) keys[b + lane] = x;
+            } else if (len <= SEG_WARP_MAX) {
+                int P = 64;
+                while (P < len) P <<= 1;
+                for (int i = lane; i < P; i += 32) buf[w][i] = i < len ? keys[b + i] : INT_MAX;
+                __syncwarp();
+                smem_bitonic(buf[w], P, lane, 32, true);
+                for (int i = lane; i < len; i += 32) keys[b + i] = buf[w][i];
+                __syncwarp();
+            } else if (lane == 0) {
+                const int i = atomicAdd(big_cnt, 1);
+                if (i < big_cap) big[i] = seg; else atomicOr(dev_err, DEVERR_OVERFLOW);
+            }
         }
     }
 }
@@ -238,7 +262,7 @@ void init_prims_attrs() {
 void segsort_i32(betty_ctx* c, const int64_t* ptr, int32_t* keys, const int64_t* nseg_dev, int64_t nseg_fixed,
                  int64_t nseg_cap, cudaStream_t s) {
     if (!nseg_dev) nseg_cap = nseg_fixed;
-    int grid = (int)std::min<int64_t>((nseg_cap + 7) / 8 + 1, (int64_t)c->num_sms * 8);
+    int grid = (int)std::min<int64_t>((nseg_cap + 255) / 256 + 1, (int64_t)c->num_sms * 8);
     k_reset_int<<<1, 1, 0, s>>>(c->big_count);
     k_segsort_warp<<<grid, 256, 0, s>>>(ptr, keys, nseg_dev, nseg_fixed, c->big_list, c->big_count, c->big_list_cap,
                                         c->dev_err);

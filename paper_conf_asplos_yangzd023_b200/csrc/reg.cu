@@ -52,23 +52,47 @@ __global__ void k_reg_ub(const int64_t* __restrict__ indptr, const int32_t* __re
     }
 }
 
-// expand the candidate list of row i into buf[0, ub) (ub known), cooperative over `nthr` threads
+// expand the candidate list of row i into buf[0, ub) (ub known), cooperative over `nthr` threads.
+// The row's edges are taken 32 at a time: one warp loads their columns' extents and
+// prefix-sums the lengths into shared memory (s_pre[0..n], s_cb[0..n)), then every
+// thread handles flattened candidate positions independently (no serial chain of
+// dependent loads per edge).  Column u lists i exactly once (no repeated edges) and
+// is ascending, so a candidate j at offset t of its column lands at t - [j > i].
 __device__ __forceinline__ void reg_expand(const int64_t* __restrict__ indptr, const int32_t* __restrict__ idx,
                                            const int64_t* __restrict__ t_indptr, const int32_t* __restrict__ t_idx,
-                                           int64_t i, int32_t* buf, int tid, int nthr) {
+                                           int64_t i, int32_t* buf, int tid, int nthr, int* s_pre, int64_t* s_cb) {
+    const int64_t rb = indptr[i], re = indptr[i + 1];
+    const int lane = tid & 31;
     int64_t o = 0;
-    for (int64_t e = indptr[i]; e < indptr[i + 1]; ++e) {
-        const int32_t u = idx[e];
-        const int64_t b = t_indptr[u], d = t_indptr[u + 1] - b;
-        // column u lists i exactly once (no repeated edges): skip it, keep order irrelevant
-        for (int64_t t = tid; t < d; t += nthr) {
-            const int32_t j = t_idx[b + t];
-            if (j == (int32_t)i) continue;
-            // position: entries before the one equal to i keep t, after it t-1
-            // (i appears once; find its slot by comparing: t_idx is ascending per column)
-            buf[o + (j < (int32_t)i ? t : t - 1)] = j;
+    for (int64_t e0 = rb; e0 < re; e0 += 32) {
+        const int n = (int)mn64(32, re - e0);
+        if (tid < 32) {
+            int d = 0;
+            int64_t cb = 0;
+            if (lane < n) {
+                const int32_t u = idx[e0 + lane];
+                cb = t_indptr[u];
+                d = (int)(t_indptr[u + 1] - cb);
+            }
+            const int incl = warp_incl_scan(d);
+            if (lane == 0) s_pre[0] = 0;
+            s_pre[lane + 1] = incl;
+            s_cb[lane] = cb;
         }
-        o += d - 1;
+        if (nthr > 32) __syncthreads(); else __syncwarp();
+        const int total = s_pre[n];
+        for (int f = tid; f < total; f += nthr) {
+            int lo = 0, hi = n;                          // s_pre[lo] <= f < s_pre[hi]
+            while (hi - lo > 1) {
+                const int mid = (lo + hi) >> 1;
+                if (s_pre[mid] <= f) lo = mid; else hi = mid;
+            }
+            const int t = f - s_pre[lo];
+            const int32_t j = t_idx[s_cb[lo] + t];
+            if (j != (int32_t)i) buf[o + (s_pre[lo] - lo) + t - (j > (int32_t)i ? 1 : 0)] = j;
+        }
+        o += total - n;
+        if (nthr > 32) __syncthreads(); else __syncwarp();
     }
 }
 
@@ -131,6 +155,8 @@ __global__ void __launch_bounds__(256) k_reg_rows_warp(const int64_t* __restrict
                                                        int64_t* __restrict__ nnz) {
     __shared__ int32_t buf[8][REG_WARP_MAX];
     __shared__ int s_cnt[8];
+    __shared__ int s_pre[8][33];
+    __shared__ int64_t s_cb[8][32];
     const int64_t n = *n_rows_dev;
     const int w = warp_id(), lane = lane_id();
     const int64_t gw = blockIdx.x * 8ll + w, nw = gridDim.x * 8ll;
@@ -138,7 +164,21 @@ __global__ void __launch_bounds__(256) k_reg_rows_warp(const int64_t* __restrict
         const int64_t u = ub[i];
         if (u > REG_WARP_MAX) continue;                 // handled by the CTA kernel
         if (u == 0) { if (lane == 0) nnz[i] = 0; continue; }
-        reg_expand(indptr, idx, t_indptr, t_idx, i, buf[w], lane, 32);
+        reg_expand(indptr, idx, t_indptr, t_idx, i, buf[w], lane, 32, s_pre[w], s_cb[w]);
+        if (u <= 32) {               // sort + run-length encode in registers
+            int32_t x = lane < u ? buf[w][lane] : INT_MAX;
+            x = warp_bitonic32(x);
+            const int32_t prev = __shfl_up_sync(0xffffffffu, x, 1);
+            const bool head = lane < u && (lane == 0 || x != prev);
+            const unsigned hm = __ballot_sync(0xffffffffu, head);
+            const unsigned above = hm & ~((2u << lane) - 1u);
+            const int nxt = above ? __ffs(above) - 1 : (int)u;
+            const int pos = __popc(hm & ((1u << lane) - 1u));
+            if (head) { tcol[off[i] + pos] = x; tw[off[i] + pos] = nxt - lane; }
+            if (lane == 0) nnz[i] = __popc(hm);
+            __syncwarp();
+            continue;
+        }
         int P = 32;
         while (P < u) P <<= 1;
         for (int t = (int)u + lane; t < P; t += 32) buf[w][t] = INT_MAX;
@@ -162,12 +202,14 @@ __global__ void __launch_bounds__(1024) k_reg_rows_cta(const int64_t* __restrict
                                                        int64_t* __restrict__ nnz) {
     extern __shared__ int32_t sbuf[];
     __shared__ int s_cnt;
+    __shared__ int s_pre[33];
+    __shared__ int64_t s_cb[32];
     const int nb = *big_cnt;
     for (int t = blockIdx.x; t < nb; t += gridDim.x) {
         const int64_t i = big[t];
         const int64_t u = ub[i];
         if (u > REG_CTA_MAX) { if (threadIdx.x == 0) nnz[i] = 0; continue; }
-        reg_expand(indptr, idx, t_indptr, t_idx, i, sbuf, threadIdx.x, blockDim.x);
+        reg_expand(indptr, idx, t_indptr, t_idx, i, sbuf, threadIdx.x, blockDim.x, s_pre, s_cb);
         int P = 1024;
         while (P < u) P <<= 1;
         for (int q = (int)u + threadIdx.x; q < P; q += blockDim.x) sbuf[q] = INT_MAX;

@@ -121,6 +121,10 @@ bool sage_alloc(betty_ctx* c, const ModelCfg& m, const std::vector<int64_t>& cap
             }
         }
         if (l >= 1) B.H = A(ns * m.layers[l - 1].ld_out * ea);
+        if (l >= 1 && m.bf16) {
+            B.ldhb = (m.dims[l] + 127) / 128 * 4;
+            B.Hbits = (uint32_t*)A(ns * B.ldhb * 4);
+        }
         if (!L.last) B.dS = A(nd * L.ld_ds * ea);
         if (L.last) {
             b->logits = (float*)A(nd * L.ld_out * 4);
@@ -203,6 +207,7 @@ void sage_forward(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView*
             PB(l == 0 ? PROBE_AGG_L0 : PROBE_AGG_L1);
             agg_mean_pf(c, B.Y, L.ld_y, V.indptr, V.indices, V.cnt, V.cap_dst, L.Fo, L.Fop, !L.last, out, out_bf,
                         L.ld_out, s);
+            if (!L.last) b.l[l + 1].hbits_ok = false;
             PE(l == 0 ? PROBE_AGG_L0 : PROBE_AGG_L1);
             continue;
         }
@@ -224,8 +229,8 @@ void sage_forward(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView*
             // array when present, else through src_gid
             const int32_t* erow = (l == 0 && V.egid) ? V.egid : V.indices;
             const int32_t* emap = (l == 0 && !V.egid) ? V.src_gid : nullptr;
-            agg_mean_xa(c, X, xbf, ldx, xrow, erow, emap, V.indptr, V.cnt, V.cap_dst, L.Fi, L.Fp, B.XA, m.bf16,
-                        L.ld_xa, s);
+            agg_mean_xa(c, X, xbf, ldx, xrow, erow, emap, V.indptr, V.cnt, V.order_tab, V.cap_dst, L.Fi, L.Fp, B.XA,
+                        m.bf16, L.ld_xa, s);
             PE(l == 0 ? PROBE_AGG_L0 : PROBE_AGG_L1);
         }
         GemmRow g{};
@@ -234,8 +239,10 @@ void sage_forward(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView*
         g.M_dev = V.cnt + 0; g.M_cap = V.cap_dst; g.K = 2 * L.Fp + 1; g.N = L.Fo;
         g.Bt = B.Bt; g.ldbt = B.ldbt;
         g.C = out; g.ldc = L.ld_out; g.c_bf16 = out_bf; g.epi = epi;
+        if (!L.last) { g.obits = b.l[l + 1].Hbits; g.ldob = b.l[l + 1].ldhb; }
         PB(l == 0 ? PROBE_GEMM_FWD_L0 : PROBE_GEMM_FWD_L1);
-        gemm_row(c, g, s);
+        const bool bits = gemm_row(c, g, s);
+        if (!L.last) b.l[l + 1].hbits_ok = bits;
         PE(l == 0 ? PROBE_GEMM_FWD_L0 : PROBE_GEMM_FWD_L1);
     }
 }
@@ -279,6 +286,7 @@ void sage_backward(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView
                 g.M_dev = V.cnt + 1; g.M_cap = V.cap_src; g.K = 2 * L.Fop; g.N = L.Fi;
                 g.C = dS_prev; g.ldc = ld_prev; g.c_bf16 = m.bf16; g.epi = EPI_MASK;
                 g.mask = Hmask; g.ldm = ldh; g.m_bf16 = m.bf16;
+                if (B.hbits_ok) { g.mbits = B.Hbits; g.ldmb = B.ldhb; }
                 gemm_row(c, g, s);
             }
             continue;
@@ -328,6 +336,7 @@ void sage_backward(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView
             g.M_dev = V.cnt + 1; g.M_cap = V.cap_src; g.K = L.Fi; g.N = L.Fi;
             g.C = dS_prev; g.ldc = ld_prev; g.c_bf16 = m.bf16; g.epi = EPI_RES_MASK;
             g.mask = Hmask; g.ldm = ldh; g.m_bf16 = m.bf16;
+            if (B.hbits_ok) { g.mbits = B.Hbits; g.ldmb = B.ldhb; }
             g.res = B.dXA; g.ldr = L.ld_dxa; g.nres_dev = V.cnt + 0;
             gemm_row(c, g, s);
         }

@@ -8,9 +8,10 @@ namespace betty {
 
 // ---- agg.cu
 // XA[v] = [X[srow v] | mean_e X[row(e)] | 1], row(e) = emap ? emap[erow[e]] : erow[e]
+// otab: optional micro-batch-major row order (extract.h), null = ascending rows
 void agg_mean_xa(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const int32_t* srow, const int32_t* erow,
-                 const int32_t* emap, const int64_t* indptr, const int64_t* cnt, int64_t rows_cap, int Fi, int Fp,
-                 void* XA, bool xa_bf16, int64_t ldxa, cudaStream_t s);
+                 const int32_t* emap, const int64_t* indptr, const int64_t* cnt, const int64_t* otab, int64_t rows_cap,
+                 int Fi, int Fp, void* XA, bool xa_bf16, int64_t ldxa, cudaStream_t s);
 void agg_mean_pf(betty_ctx* c, const float* Y, int64_t ldy, const int64_t* indptr, const int32_t* idx,
                  const int64_t* cnt, int64_t rows_cap, int Fo, int Fop, bool relu, void* out, bool out_bf16,
                  int64_t ldo, cudaStream_t s);
@@ -40,8 +41,11 @@ struct GemmRow {                 // C[m, n] = sum_k A[m, k] B(k, n), m < *M_dev
     const void* mask; int64_t ldm; bool m_bf16;           // EPI_MASK / EPI_RES_MASK: C *= [mask > 0]
     const float* res; int64_t ldr; const int64_t* nres_dev; // EPI_RES_MASK: C += res (rows < *nres_dev)
     const void* Bt; int64_t ldbt;                          // K-major copy of B (N x K) for the tensor-core path
+    const uint32_t* mbits; int64_t ldmb;   // EPI_MASK / EPI_RES_MASK: mask as ReLU bits (tensor-core path), or null
+    uint32_t* obits; int64_t ldob;         // EPI_RELU_ONES: also write the ReLU bits [C > 0] (tensor-core path)
 };
-void gemm_row(betty_ctx* c, const GemmRow& g, cudaStream_t s);
+// returns true iff the ReLU bits g.obits were written (EPI_RELU_ONES on the tensor-core path)
+bool gemm_row(betty_ctx* c, const GemmRow& g, cudaStream_t s);
 // gemm_tc.cu: tcgen05 paths (false = shape not supported, caller falls back to SIMT)
 bool tc_available();
 bool gemm_row_tc(betty_ctx* c, const GemmRow& g, const void* Bk, int64_t ldbk, cudaStream_t s);
