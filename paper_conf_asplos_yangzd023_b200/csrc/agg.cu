@@ -1,3 +1,4 @@
+#include <cstdlib>
 // agg.cu -- a3/a5: GraphSAGE aggregation forward and backward (HBM-bound
 // CSR segment reductions), Table 1, Eq. 1 PAPER.md:269.
 //
@@ -24,33 +25,78 @@ template <typename T> __device__ __forceinline__ const T* row_ptr(const T* X, in
 }
 
 // ------------------------------------------------ mean, aggregate-first fwd
-// LPR lanes own one dst row (RPW = 32/LPR rows per warp in flight); each lane
-// covers 16-byte vectors of the feature row and keeps AGG_BATCH neighbour
-// rows in flight.  The neighbour X-row of edge e is emap ? emap[erow[e]] : erow[e]
-// (layer 0 passes the edge -> global-id array written by the extraction, so no
-// dependent id lookup stays on the critical path); the self row of dst v is
-// srow ? srow[v] : v.  With an order table (extract.h) the rows are visited
-// micro-batch by micro-batch, so the source rows one micro-batch shares stay
-// in L2 between their uses; the grid is exactly the resident CTAs so all warps
-// sweep the order together.
-constexpr int AGG_BATCH = 4;     // neighbour rows in flight per lane (x 16 B)
+// LPR lanes own one dst row (RPW = 32/LPR rows per warp); lane `sub` covers
+// 16-byte vector `sub` (+ LPR, ...) of the feature row.  All neighbour vectors
+// of a batch of up to EB edges are issued at once as cp.async copies into the
+// warp's shared-memory slice (no registers held while in flight, one memory
+// round trip per row instead of one per 4 edges) and summed from shared memory
+// after cp.async.wait_group; each lane reads back only what it copied itself.
+// Feature rows are fetched with an L2 evict_last policy and XA is written with
+// streaming stores, so the output stream does not evict the rows that one
+// micro-batch re-reads.  The neighbour X-row of edge e is emap ? emap[erow[e]]
+// : erow[e] (layer 0 passes the edge -> global-id array written by the
+// extraction); the self row of dst v is srow ? srow[v] : v.  With an order
+// table (extract.h) the rows are visited micro-batch by micro-batch, and the
+// grid is exactly the resident CTAs so all warps sweep the order together.
+constexpr int AGG_EB = 12;       // edges per cp.async batch (layer-0 fanout 10 fits one batch)
+__device__ __forceinline__ uint64_t l2_evict_last_policy() {
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+    return pol;
+}
+__device__ __forceinline__ void cp_async16(void* sdst, const void* gsrc, uint64_t pol, bool hint) {
+    if (hint)
+        asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2;"
+                     ::"r"((uint32_t)__cvta_generic_to_shared(sdst)), "l"(gsrc), "l"(pol) : "memory");
+    else
+        asm volatile("cp.async.cg.shared.global [%0], [%1], 16;"
+                     ::"r"((uint32_t)__cvta_generic_to_shared(sdst)), "l"(gsrc) : "memory");
+}
+__device__ __forceinline__ void cp_async_wait_all() {
+    asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
+}
+template <typename T> __device__ __forceinline__ void st_cs4(T* p, const float* v);
+template <> __device__ __forceinline__ void st_cs4<float>(float* p, const float* v) {
+    __stcs((float4*)p, make_float4(v[0], v[1], v[2], v[3]));
+}
+template <typename Tout, int VW> __device__ __forceinline__ void st_vec_cs(Tout* p, const float* v) {
+    if constexpr (sizeof(Tout) == 2) {
+        uint32_t w[VW / 2];
+#pragma unroll
+        for (int i = 0; i < VW / 2; ++i) {
+            __nv_bfloat162 h = __floats2bfloat162_rn(v[2 * i], v[2 * i + 1]);
+            w[i] = *(uint32_t*)&h;
+        }
+        if constexpr (VW == 8) __stcs((uint4*)p, make_uint4(w[0], w[1], w[2], w[3]));
+        else __stcs((uint2*)p, make_uint2(w[0], w[1]));
+    } else {
+#pragma unroll
+        for (int i = 0; i < VW; i += 4) __stcs((float4*)(p + i), make_float4(v[i], v[i + 1], v[i + 2], v[i + 3]));
+    }
+}
+
 template <typename Tin, typename Tout, int LPR>
-__global__ void __launch_bounds__(256, 4) k_agg_mean_xa(const Tin* __restrict__ X, int64_t ldx,
+__global__ void __launch_bounds__(256) k_agg_mean_xa(const Tin* __restrict__ X, int64_t ldx,
                                                      const int32_t* __restrict__ srow,
                                                      const int32_t* __restrict__ erow,
                                                      const int32_t* __restrict__ emap,
                                                      const int64_t* __restrict__ indptr, const int64_t* cnt,
                                                      const int64_t* __restrict__ otab, int Fi, int Fp,
-                                                     Tout* __restrict__ XA, int64_t ldxa) {
+                                                     Tout* __restrict__ XA, int64_t ldxa, int hint) {
     using VI = Vec<Tin>;
     constexpr int VW = VI::N;
     constexpr int RPW = 32 / LPR;
+    static_assert(AGG_EB <= LPR || LPR == 8, "edge batch indices come from one lane each");
+    constexpr int EB = AGG_EB < LPR ? AGG_EB : LPR;
+    extern __shared__ uint4 agg_sbuf[];              // [warps][RPW][EB][LPR]
     __shared__ int64_t s_vs[ORDER_SMEM + 1], s_rs[ORDER_SMEM];
     const int64_t nd = cnt[0];
     const int nseg = order_load(otab, s_vs, s_rs);
     const int NV = (Fi + VW - 1) / VW;
     const int lane = lane_id(), sub = lane % LPR, grp = lane / LPR;
     const unsigned gmask = LPR == 32 ? 0xffffffffu : (((1u << LPR) - 1u) << (grp * LPR));
+    uint4* wb = agg_sbuf + ((int64_t)(threadIdx.x >> 5) * RPW + grp) * EB * LPR;
+    const uint64_t pol = l2_evict_last_policy();
     const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
     int seg = 0;
@@ -59,7 +105,7 @@ __global__ void __launch_bounds__(256, 4) k_agg_mean_xa(const Tin* __restrict__ 
         const bool rowok = vv < nd;
         const int64_t v = rowok ? order_map(vv, nseg, s_vs, s_rs, seg) : vv;
         int64_t b = 0, e = 0;
-        if (rowok) { b = indptr[v]; e = indptr[v + 1]; }
+        if (rowok) { b = __ldcs(indptr + v); e = __ldcs(indptr + v + 1); }
         const float inv = e > b ? 1.0f / (float)(e - b) : 0.0f;
         Tout* out = XA + v * ldxa;
         for (int vb = 0; vb < NV; vb += LPR) {
@@ -68,39 +114,38 @@ __global__ void __launch_bounds__(256, 4) k_agg_mean_xa(const Tin* __restrict__ 
             float acc[VW];
 #pragma unroll
             for (int t = 0; t < VW; ++t) acc[t] = 0.f;
-            for (int64_t e0 = b; e0 < e; e0 += LPR) {
-                const int n = (int)mn64(LPR, e - e0);
+            for (int64_t e0 = b; e0 < e; e0 += EB) {
+                const int n = (int)mn64(EB, e - e0);
                 int32_t my = 0;
-                if (sub < n) { my = erow[e0 + sub]; if (emap) my = emap[my]; }
-                for (int j = 0; j < n; j += AGG_BATCH) {
-                    typename VI::Raw x[AGG_BATCH];
-#pragma unroll
-                    for (int t = 0; t < AGG_BATCH; ++t) {
-                        const int32_t u = __shfl_sync(gmask, my, (j + t) & (LPR - 1), LPR);
-                        x[t] = (act && j + t < n) ? VI::ld_raw(X + (int64_t)u * ldx + vi * VW) : VI::zero_raw();
-                    }
-#pragma unroll
-                    for (int t = 0; t < AGG_BATCH; ++t) VI::add_raw(acc, x[t]);
+                if (sub < n) { my = __ldcs(erow + e0 + sub); if (emap) my = emap[my]; }
+                for (int t = 0; t < n; ++t) {
+                    const int32_t u = __shfl_sync(gmask, my, t, LPR);
+                    if (act) cp_async16(wb + t * LPR + sub, X + (int64_t)u * ldx + vi * VW, pol, hint != 0);
                 }
+                cp_async_wait_all();
+                if (act) {
+                    for (int t = 0; t < n; ++t) VI::add_raw(acc, *(const typename VI::Raw*)(wb + t * LPR + sub));
+                }
+                __syncwarp(gmask);
             }
             if (act) {
                 VI self;
                 self.load(X + (int64_t)(srow ? srow[v] : (int32_t)v) * ldx + vi * VW);
-                if constexpr (sizeof(Tin) == sizeof(Tout)) {
-                    Vec<Tout> so, ao;
+                float so[VW], ao[VW];
 #pragma unroll
-                    for (int t = 0; t < VW; ++t) {
-                        const bool in = vi * VW + t < Fi;
-                        so.v[t] = in ? self.v[t] : 0.f;
-                        ao.v[t] = in ? acc[t] * inv : 0.f;
-                    }
-                    so.store(out + vi * VW);
-                    ao.store(out + Fp + vi * VW);
+                for (int t = 0; t < VW; ++t) {
+                    const bool in = vi * VW + t < Fi;
+                    so[t] = in ? self.v[t] : 0.f;
+                    ao[t] = in ? acc[t] * inv : 0.f;
+                }
+                if constexpr (sizeof(Tin) == sizeof(Tout)) {
+                    st_vec_cs<Tout, VW>(out + vi * VW, so);
+                    st_vec_cs<Tout, VW>(out + Fp + vi * VW, ao);
                 } else {
 #pragma unroll
                     for (int t = 0; t < VW; ++t) {
                         const int col = vi * VW + t;
-                        if (col < Fi) { st_act(out + col, self.v[t]); st_act(out + Fp + col, acc[t] * inv); }
+                        if (col < Fi) { st_act(out + col, so[t]); st_act(out + Fp + col, ao[t]); }
                     }
                 }
             }
@@ -325,6 +370,13 @@ __global__ void __launch_bounds__(256) k_route_pool(const float* __restrict__ dX
 }
 
 // ------------------------------------ vectorised narrow-row gathers (LPR lanes / row)
+// LPR lanes own a row and each lane up to PF_VPL 16-byte vectors of it, so a
+// warp keeps 32/LPR rows (8 for the 48-wide layer of the products model) in
+// flight; the edge loop takes LPR edge ids at a time (one per lane) and issues
+// every neighbour vector of the batch before summing (predicated, unrolled).
+constexpr int PF_VPL = 4;
+static inline int pick_lpr_vpl(int nv) { return nv <= 4 * PF_VPL ? 4 : (nv <= 8 * PF_VPL ? 8 : (nv <= 16 * PF_VPL ? 16 : 32)); }
+
 // mean, project-first fwd: S[v] = Y[v, Fop:] + (1/D_v) sum_u Y[u, :Fo] ; out = logits or ReLU -> H (+ ones)
 template <typename Tout, int LPR>
 __global__ void __launch_bounds__(256) k_agg_pf_v(const float* __restrict__ Y, int64_t ldy,
@@ -344,28 +396,40 @@ __global__ void __launch_bounds__(256) k_agg_pf_v(const float* __restrict__ Y, i
         int64_t b = 0, e = 0;
         if (rowok) { b = indptr[v]; e = indptr[v + 1]; }
         const float inv = e > b ? 1.0f / (float)(e - b) : 0.0f;
-        for (int vb = 0; vb < NV; vb += LPR) {
-            const int vi = vb + sub;
-            const bool act = rowok && vi < NV;
-            float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+        for (int vb = 0; vb < NV; vb += LPR * PF_VPL) {
+            float4 acc[PF_VPL];
+#pragma unroll
+            for (int k = 0; k < PF_VPL; ++k) acc[k] = make_float4(0.f, 0.f, 0.f, 0.f);
             for (int64_t e0 = b; e0 < e; e0 += LPR) {
                 const int n = (int)mn64(LPR, e - e0);
                 const int32_t my = sub < n ? idx[e0 + sub] : 0;
-                for (int j = 0; j < n; ++j) {
+#pragma unroll
+                for (int j = 0; j < LPR; ++j) {
                     const int32_t u = __shfl_sync(gmask, my, j, LPR);
-                    if (act) {
-                        const float4 y = *(const float4*)(Y + (int64_t)u * ldy + vi * 4);
-                        acc.x += y.x; acc.y += y.y; acc.z += y.z; acc.w += y.w;
+                    if (j < n) {
+#pragma unroll
+                        for (int k = 0; k < PF_VPL; ++k) {
+                            const int vi = vb + sub + LPR * k;
+                            if (rowok && vi < NV) {
+                                const float4 y = *(const float4*)(Y + (int64_t)u * ldy + vi * 4);
+                                acc[k].x += y.x; acc[k].y += y.y; acc[k].z += y.z; acc[k].w += y.w;
+                            }
+                        }
                     }
                 }
             }
-            if (act) {
-                const float4 sf = *(const float4*)(Y + v * ldy + Fop + vi * 4);
-                float r[4] = {sf.x + acc.x * inv, sf.y + acc.y * inv, sf.z + acc.z * inv, sf.w + acc.w * inv};
 #pragma unroll
-                for (int t = 0; t < 4; ++t) {
-                    const int col = vi * 4 + t;
-                    if (col < Fo) st_act(out + v * ldo + col, relu ? fmaxf(r[t], 0.f) : r[t]);
+            for (int k = 0; k < PF_VPL; ++k) {
+                const int vi = vb + sub + LPR * k;
+                if (rowok && vi < NV) {
+                    const float4 sf = *(const float4*)(Y + v * ldy + Fop + vi * 4);
+                    float r[4] = {sf.x + acc[k].x * inv, sf.y + acc[k].y * inv, sf.z + acc[k].z * inv,
+                                  sf.w + acc[k].w * inv};
+#pragma unroll
+                    for (int t = 0; t < 4; ++t) {
+                        const int col = vi * 4 + t;
+                        if (col < Fo) st_act(out + v * ldo + col, relu ? fmaxf(r[t], 0.f) : r[t]);
+                    }
                 }
             }
         }
@@ -395,12 +459,12 @@ __global__ void __launch_bounds__(256) k_csc_pf_v(const Tin* __restrict__ dS, in
         const bool rowok = u < ns;
         int64_t b = 0, e = 0;
         if (rowok) { b = t_indptr[u]; e = t_indptr[u + 1]; }
-        for (int vb = 0; vb < NV; vb += LPR) {
-            const int vi = vb + sub;
-            const bool act = rowok && vi < NV;
-            float acc[VW];
+        for (int vb = 0; vb < NV; vb += LPR * PF_VPL) {
+            float acc[PF_VPL][VW];
 #pragma unroll
-            for (int t = 0; t < VW; ++t) acc[t] = 0.f;
+            for (int k = 0; k < PF_VPL; ++k)
+#pragma unroll
+                for (int t = 0; t < VW; ++t) acc[k][t] = 0.f;
             for (int64_t e0 = b; e0 < e; e0 += LPR) {
                 const int n = (int)mn64(LPR, e - e0);
                 int32_t my = 0;
@@ -409,31 +473,42 @@ __global__ void __launch_bounds__(256) k_csc_pf_v(const Tin* __restrict__ dS, in
                     my = t_idx[e0 + sub];
                     myinv = 1.0f / (float)(indptr[my + 1] - indptr[my]);
                 }
-                for (int j = 0; j < n; ++j) {
+#pragma unroll
+                for (int j = 0; j < LPR; ++j) {
                     const int32_t v = __shfl_sync(gmask, my, j, LPR);
                     const float iv = __shfl_sync(gmask, myinv, j, LPR);
-                    if (act) {
-                        VI x;
-                        x.load_cg(dS + (int64_t)v * ldds + vi * VW);
+                    if (j < n) {
 #pragma unroll
-                        for (int t = 0; t < VW; ++t) acc[t] += x.v[t] * iv;
+                        for (int k = 0; k < PF_VPL; ++k) {
+                            const int vi = vb + sub + LPR * k;
+                            if (rowok && vi < NV) {
+                                VI x;
+                                x.load_cg(dS + (int64_t)v * ldds + vi * VW);
+#pragma unroll
+                                for (int t = 0; t < VW; ++t) acc[k][t] += x.v[t] * iv;
+                            }
+                        }
                     }
                 }
             }
-            if (act) {
-                VI self;
-                if (u < nd) self.load_cg(dS + u * ldds + vi * VW);
-                float ga[VW], gs[VW];
 #pragma unroll
-                for (int t = 0; t < VW; ++t) {
-                    const bool in = vi * VW + t < Fo;
-                    ga[t] = in ? acc[t] : 0.f;
-                    gs[t] = (in && u < nd) ? self.v[t] : 0.f;
-                }
+            for (int k = 0; k < PF_VPL; ++k) {
+                const int vi = vb + sub + LPR * k;
+                if (rowok && vi < NV) {
+                    VI self;
+                    if (u < nd) self.load_cg(dS + u * ldds + vi * VW);
+                    float ga[VW], gs[VW];
 #pragma unroll
-                for (int t = 0; t < VW; t += 4) {        // vector stores (Fop, ldg multiples of 8)
-                    st_act4(G + u * ldg + vi * VW + t, ga + t);
-                    st_act4(G + u * ldg + Fop + vi * VW + t, gs + t);
+                    for (int t = 0; t < VW; ++t) {
+                        const bool in = vi * VW + t < Fo;
+                        ga[t] = in ? acc[k][t] : 0.f;
+                        gs[t] = (in && u < nd) ? self.v[t] : 0.f;
+                    }
+#pragma unroll
+                    for (int t = 0; t < VW; t += 4) {        // vector stores (Fop, ldg multiples of 8)
+                        st_act4(G + u * ldg + vi * VW + t, ga + t);
+                        st_act4(G + u * ldg + Fop + vi * VW + t, gs + t);
+                    }
                 }
             }
         }
@@ -466,9 +541,19 @@ void agg_mean_xa(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const in
     const int nv = (Fi + vw - 1) / vw;
     const int lpr = nv <= 8 ? 8 : (nv <= 16 ? 16 : 32);
     const int64_t warps = (rows_cap + (32 / lpr) - 1) / (32 / lpr);
-#define AGG_L(LPR) DISPATCH_ACT(x_bf16, TI, DISPATCH_ACT(xa_bf16, TO, \
-        k_agg_mean_xa<TI, TO, LPR><<<resident_grid(c, k_agg_mean_xa<TI, TO, LPR>, 256, (warps + 7) / 8), 256, 0, s>>>( \
-            (const TI*)X, ldx, srow, erow, emap, indptr, cnt, otab, Fi, Fp, (TO*)XA, ldxa)))
+    // experiment switches (default: L2 evict_last hint on feature rows, micro-batch-major order)
+    static const int hint = getenv("BETTY_AGG_NOHINT") ? 0 : 1;
+    static const bool no_order = getenv("BETTY_AGG_NOORDER") != nullptr;
+#define AGG_L(LPR) DISPATCH_ACT(x_bf16, TI, DISPATCH_ACT(xa_bf16, TO, {                                           \
+        const size_t sm = (size_t)8 * (32 / LPR) * (AGG_EB < LPR ? AGG_EB : LPR) * LPR * 16;                    \
+        static bool attr = false;                                                                              \
+        if (!attr) { cudaFuncSetAttribute(k_agg_mean_xa<TI, TO, LPR>, cudaFuncAttributeMaxDynamicSharedMemorySize, \
+                                          (int)sm); attr = true; }                                             \
+        int per_sm = 1;                                                                                        \
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_agg_mean_xa<TI, TO, LPR>, 256, sm);           \
+        const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((warps + 7) / 8, (int64_t)std::max(per_sm, 1) * c->num_sms)); \
+        k_agg_mean_xa<TI, TO, LPR><<<grid, 256, sm, s>>>((const TI*)X, ldx, srow, erow, emap, indptr, cnt,        \
+                                                        no_order ? nullptr : otab, Fi, Fp, (TO*)XA, ldxa, hint); }))
     if (lpr == 8) { AGG_L(8); } else if (lpr == 16) { AGG_L(16); } else { AGG_L(32); }
 #undef AGG_L
 }
@@ -476,7 +561,7 @@ void agg_mean_xa(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const in
 void agg_mean_pf(betty_ctx* c, const float* Y, int64_t ldy, const int64_t* indptr, const int32_t* idx,
                  const int64_t* cnt, int64_t rows_cap, int Fo, int Fop, bool relu, void* out, bool out_bf16,
                  int64_t ldo, cudaStream_t s) {
-    const int lpr = pick_lpr((Fo + 3) / 4);
+    const int lpr = pick_lpr_vpl((Fo + 3) / 4);
     const int grid = warps_grid(c, (rows_cap + (32 / lpr) - 1) / (32 / lpr));
 #define PF_L(LPR) DISPATCH_ACT(out_bf16, TO, \
         k_agg_pf_v<TO, LPR><<<grid, 256, 0, s>>>(Y, ldy, indptr, idx, cnt, Fo, Fop, relu ? 1 : 0, (TO*)out, ldo))
@@ -502,7 +587,7 @@ void csc_mean(betty_ctx* c, const float* dXA, int64_t ldd, const int64_t* indptr
 void csc_pf(betty_ctx* c, const void* dS, bool ds_bf16, int64_t ldds, const int64_t* indptr, const int64_t* t_indptr,
             const int32_t* t_idx, const int64_t* cnt, int64_t src_cap, int Fo, int Fop, void* G, bool g_bf16,
             int64_t ldg, cudaStream_t s) {
-    const int lpr = pick_lpr((Fop + (ds_bf16 ? 7 : 3)) / (ds_bf16 ? 8 : 4));
+    const int lpr = pick_lpr_vpl((Fop + (ds_bf16 ? 7 : 3)) / (ds_bf16 ? 8 : 4));
     const int grid = warps_grid(c, (src_cap + (32 / lpr) - 1) / (32 / lpr));
 #define CSC_L(LPR) DISPATCH_ACT(ds_bf16, TI, DISPATCH_ACT(g_bf16, TO, \
         k_csc_pf_v<TI, TO, LPR><<<grid, 256, 0, s>>>((const TI*)dS, ldds, indptr, t_indptr, t_idx, cnt, Fo, Fop, \

@@ -83,20 +83,20 @@ extern "C" betty_status betty_ctx_create(int device, betty_alloc_fn alloc, betty
     c->dealloc = dealloc;
     c->user = user;
     cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, device);
-    // counters [64 unsigned] + loss partials [512 double] ; device error flags ; big-segment list
-    if (cudaMalloc(&c->counters, 64 * 4 + 512 * 8) != cudaSuccess || cudaMalloc(&c->dev_err, 16) != cudaSuccess ||
-        cudaMalloc(&c->big_count, 16) != cudaSuccess) {
-        delete c;
-        return BETTY_ENOMEM;
+    // per lane: counters [64 unsigned] + loss partials [512 double], big-segment list; device error flags
+    bool ok = cudaMalloc(&c->dev_err, 16) == cudaSuccess;
+    for (auto& ln : c->lanes) {
+        ln.big_list_cap = 1 << 20;
+        ok = ok && cudaMalloc(&ln.counters, 64 * 4 + 512 * 8) == cudaSuccess &&
+             cudaMalloc(&ln.big_count, 16) == cudaSuccess &&
+             cudaMalloc(&ln.big_list, sizeof(int64_t) * ln.big_list_cap) == cudaSuccess;
+        if (ok) { cudaMemset(ln.counters, 0, 64 * 4 + 512 * 8); cudaMemset(ln.big_count, 0, 16); }
     }
-    c->big_list_cap = 1 << 20;
-    if (cudaMalloc(&c->big_list, sizeof(int64_t) * c->big_list_cap) != cudaSuccess) { delete c; return BETTY_ENOMEM; }
-    cudaMemset(c->counters, 0, 64 * 4 + 512 * 8);
+    if (!ok) { betty_ctx_destroy(c); return BETTY_ENOMEM; }
     init_kernel_attrs();
     const char* no_tc = getenv("BETTY_NO_TC");
     c->use_tc = !(no_tc && no_tc[0] == '1') && tc_available();
     cudaMemset(c->dev_err, 0, 16);
-    cudaMemset(c->big_count, 0, 16);
     cudaDeviceSynchronize();
     *out = c;
     return BETTY_OK;
@@ -105,11 +105,13 @@ extern "C" betty_status betty_ctx_create(int device, betty_alloc_fn alloc, betty
 extern "C" void betty_ctx_destroy(betty_ctx* c) {
     if (!c) return;
     cudaDeviceSynchronize();
-    if (c->scan_status) ctx_free(c, c->scan_status, 0);
-    cudaFree(c->counters);
+    for (auto& ln : c->lanes) {
+        if (ln.scan_status) ctx_free(c, ln.scan_status, 0);
+        cudaFree(ln.counters);
+        cudaFree(ln.big_count);
+        cudaFree(ln.big_list);
+    }
     cudaFree(c->dev_err);
-    cudaFree(c->big_count);
-    cudaFree(c->big_list);
     cudaDeviceSynchronize();
     delete c;
 }
@@ -474,6 +476,9 @@ struct betty_plan {
     RegBufs R;
     const betty_block* reg_src = nullptr;
     betty_block reg_block{};
+    // side stream: the REG rebuild overlaps the rest of the step (it shares no data with it)
+    cudaStream_t side = nullptr;
+    cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
     // graph
     cudaGraphExec_t gexec = nullptr;
     cudaStream_t cap_stream = nullptr;
@@ -486,6 +491,18 @@ static void step_body(betty_ctx* c, betty_plan* p, const float* params, const vo
                       const int32_t* labels, float scale, float* grad, float* loss, cudaStream_t s) {
     Probe* pr = p->sb.probe;
     if (pr) pr->used = 0;
+    if (p->with_reg) {          // fork: REG on the side stream with its own primitive scratch (lane 1)
+        cudaEventRecord(p->ev_fork, s);
+        cudaStreamWaitEvent(p->side, p->ev_fork, 0);
+        c->lane = 1;
+        if (pr) pr->begin(PROBE_REG, p->side);
+        reg_phase1(c, p->R.a, p->side);
+        reg_phase2(c, p->R.a, p->side);
+        reg_phase3(c, p->R.a, p->R.col, p->R.w, p->R.nnz_cap, p->side);
+        if (pr) pr->end(PROBE_REG, p->side);
+        c->lane = 0;
+        cudaEventRecord(p->ev_join, p->side);
+    }
     sage_prep(c, p->m, p->sb, params, s);
     for (size_t g = 0; g < p->groups.size(); ++g) {
         ExtractArgs a{};
@@ -499,13 +516,7 @@ static void step_body(betty_ctx* c, betty_plan* p, const float* params, const vo
         sage_loss(c, p->m, p->sb, p->views.data(), labels, scale, loss, s);
         sage_backward(c, p->m, p->sb, p->views.data(), feats, ld_feats, grad, s);
     }
-    if (p->with_reg) {
-        if (pr) pr->begin(PROBE_REG, s);
-        reg_phase1(c, p->R.a, s);
-        reg_phase2(c, p->R.a, s);
-        reg_phase3(c, p->R.a, p->R.col, p->R.w, p->R.nnz_cap, s);
-        if (pr) pr->end(PROBE_REG, s);
-    }
+    if (p->with_reg) cudaStreamWaitEvent(s, p->ev_join, 0);   // join
 }
 
 extern "C" betty_status betty_plan_create(betty_ctx* c, const betty_model* model, const betty_block* full, int32_t L,
@@ -617,30 +628,38 @@ extern "C" betty_status betty_plan_create(betty_ctx* c, const betty_model* model
     }
     // ---- REG inside the step (once here to size its buffers)
     if (flags & BETTY_PLAN_REG) {
+        if (cudaStreamCreateWithFlags(&p->side, cudaStreamNonBlocking) != cudaSuccess ||
+            cudaEventCreateWithFlags(&p->ev_fork, cudaEventDisableTiming) != cudaSuccess ||
+            cudaEventCreateWithFlags(&p->ev_join, cudaEventDisableTiming) != cudaSuccess) {
+            betty_plan_destroy(c, p);
+            return fail(c, BETTY_ECUDA, "plan: side stream");
+        }
+        c->lane = 1;            // size the side lane's scan scratch with the REG's own calls
         p->with_reg = true;
         const betty_block* ob = &full[L - 1];
-        if (!alloc_reg_phase1(A, ob, &p->R)) { betty_plan_destroy(c, p); return fail(c, BETTY_ENOMEM, "plan: REG alloc"); }
+        if (!alloc_reg_phase1(A, ob, &p->R)) { c->lane = 0; betty_plan_destroy(c, p); return fail(c, BETTY_ENOMEM, "plan: REG alloc"); }
         int64_t h[4] = {ob->n_dst, ob->n_src, ob->n_edges, 0};
         cudaMemcpyAsync(p->R.cnt, h, sizeof(h), cudaMemcpyHostToDevice, s);
         reg_phase1(c, p->R.a, s);
         int64_t ub = 0;
         cudaMemcpyAsync(&ub, p->R.a.ub_total_dev, sizeof(int64_t), cudaMemcpyDeviceToHost, s);
-        if ((st = sync_check(c, s))) { betty_plan_destroy(c, p); return st; }
+        if ((st = sync_check(c, s))) { c->lane = 0; betty_plan_destroy(c, p); return st; }
         p->R.ub_cap = ub;
         p->R.a.tcol = A.get<int32_t>(ub);
         p->R.a.tw = A.get<int32_t>(ub);
         p->R.a.out_indptr = A.get<int64_t>(ob->n_dst + 1);
         p->R.a.nnz_total_dev = A.get<int64_t>(1);
-        if (!A.ok) { betty_plan_destroy(c, p); return fail(c, BETTY_ENOMEM, "plan: REG alloc"); }
+        if (!A.ok) { c->lane = 0; betty_plan_destroy(c, p); return fail(c, BETTY_ENOMEM, "plan: REG alloc"); }
         reg_phase2(c, p->R.a, s);
         int64_t nnz = 0;
         cudaMemcpyAsync(&nnz, p->R.a.nnz_total_dev, sizeof(int64_t), cudaMemcpyDeviceToHost, s);
-        if ((st = sync_check(c, s))) { betty_plan_destroy(c, p); return st; }
+        if ((st = sync_check(c, s))) { c->lane = 0; betty_plan_destroy(c, p); return st; }
         p->R.nnz_cap = nnz;
         p->R.col = A.get<int32_t>(nnz);
         p->R.w = A.get<int32_t>(nnz);
-        if (!A.ok) { betty_plan_destroy(c, p); return fail(c, BETTY_ENOMEM, "plan: REG alloc"); }
+        if (!A.ok) { c->lane = 0; betty_plan_destroy(c, p); return fail(c, BETTY_ENOMEM, "plan: REG alloc"); }
         p->info.reg_nnz = nnz;
+        c->lane = 0;
     }
     // ---- launches per step: capture the body once into a throw-away graph
     {
@@ -677,6 +696,9 @@ extern "C" void betty_plan_destroy(betty_ctx* c, betty_plan* p) {
     cudaDeviceSynchronize();
     if (p->gexec) cudaGraphExecDestroy(p->gexec);
     if (p->cap_stream) cudaStreamDestroy(p->cap_stream);
+    if (p->side) cudaStreamDestroy(p->side);
+    if (p->ev_fork) cudaEventDestroy(p->ev_fork);
+    if (p->ev_join) cudaEventDestroy(p->ev_join);
     p->probe.destroy();
     sage_free(c, &p->sb, 0);
     if (p->arena) { p->arena->s = 0; p->arena->release(); delete p->arena; }

@@ -112,31 +112,169 @@ __global__ void k_mark_dst(const int32_t* __restrict__ dst_pos, const int32_t* _
     }
 }
 
-// LPR lanes per dst row (LPR ~ the layer's mean degree): short sampled rows keep the lanes busy
-template <int LPR>
-__global__ void k_mark_new(const int32_t* __restrict__ dst_pos, const int32_t* __restrict__ row_mb,
-                           const int64_t* cnt, const int64_t* __restrict__ findptr, const int32_t* __restrict__ fnbr,
-                           const uint32_t* __restrict__ dstbits, uint32_t* newbits, int64_t W,
-                           const int64_t* __restrict__ otab) {
+// Warp-flattened edge loops: a warp takes 32 consecutive (virtual) dst rows, lane
+// i loads row i's extent, a warp scan of the degrees gives each row's edge
+// offset, and the warp then walks the rows' edges as one flat range, UNR edges
+// per lane in flight (independent load chains), every lane busy whatever the
+// degree mix.  Row data live in a per-warp shared slice.
+constexpr int FLAT_UNR = 4;
+struct FlatRows {
+    int pre[33];        // exclusive edge offsets of the warp's rows (pre[32] = total)
+    int64_t fb[32];     // full-batch row start of each row
+    int64_t ob[32];     // output offset (relabel) of each row
+    int64_t base[32];   // id base of the row's micro-batch new sources (relabel)
+    int j[32];          // slot (micro-batch) of each row
+};
+__device__ __forceinline__ int flat_row(const FlatRows& F, int f) {
+    int lo = 0, hi = 32;                                 // F.pre[lo] <= f < F.pre[hi]
+#pragma unroll
+    for (int step = 0; step < 5; ++step) {
+        const int mid = (lo + hi) >> 1;
+        if (F.pre[mid] <= f) lo = mid; else hi = mid;
+    }
+    return lo;
+}
+
+__global__ void __launch_bounds__(256) k_mark_new(const int32_t* __restrict__ dst_pos, const int32_t* __restrict__ row_mb,
+                                                  const int64_t* cnt, const int64_t* __restrict__ findptr,
+                                                  const int32_t* __restrict__ fnbr, const uint32_t* __restrict__ dstbits,
+                                                  uint32_t* newbits, int64_t W, const int64_t* __restrict__ otab) {
     __shared__ int64_t s_vs[ORDER_SMEM + 1], s_rs[ORDER_SMEM];
+    __shared__ FlatRows s_rows[8];
     const int nseg = order_load(otab, s_vs, s_rs);
     int seg = 0;
     const int64_t n = cnt[0];
-    const int sub = lane_id() % LPR;
-    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / LPR;
-    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) / LPR;
-    for (int64_t rv = gw; rv < n; rv += nw) {
-        const int64_t r = order_map(rv, nseg, s_vs, s_rs, seg);
-        const int j = row_mb[r];
-        const int32_t q = dst_pos[r];
-        const int64_t b = findptr[q], e = findptr[q + 1];
-        const uint32_t* db = dstbits + j * W;
-        uint32_t* nb = newbits + j * W;
-        for (int64_t i = b + sub; i < e; i += LPR) {
-            const int32_t p = fnbr[i];
-            const uint32_t bit = 1u << (p & 31);
-            if (!(db[p >> 5] & bit)) atomicOr(&nb[p >> 5], bit);
+    const int lane = lane_id();
+    FlatRows& F = s_rows[warp_id()];
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t v0 = gw * 32; v0 < n; v0 += nw * 32) {
+        const int64_t vv = v0 + lane;
+        int d = 0;
+        if (vv < n) {
+            const int64_t r = order_map(vv, nseg, s_vs, s_rs, seg);
+            const int32_t q = dst_pos[r];
+            const int64_t b = findptr[q];
+            d = (int)(findptr[q + 1] - b);
+            F.fb[lane] = b;
+            F.j[lane] = row_mb[r];
         }
+        const int incl = warp_incl_scan(d);
+        F.pre[lane + 1] = incl;
+        if (lane == 0) F.pre[0] = 0;
+        __syncwarp();
+        const int total = F.pre[32];
+        for (int f0 = lane; f0 < total; f0 += 32 * FLAT_UNR) {
+            int32_t p[FLAT_UNR];
+            int jj[FLAT_UNR];
+#pragma unroll
+            for (int u = 0; u < FLAT_UNR; ++u) {
+                const int f = f0 + 32 * u;
+                p[u] = -1;
+                if (f < total) {
+                    const int k = flat_row(F, f);
+                    p[u] = fnbr[F.fb[k] + (f - F.pre[k])];
+                    jj[u] = F.j[k];
+                }
+            }
+            uint32_t dw[FLAT_UNR];
+#pragma unroll
+            for (int u = 0; u < FLAT_UNR; ++u)
+                if (p[u] >= 0) dw[u] = dstbits[(int64_t)jj[u] * W + (p[u] >> 5)];
+#pragma unroll
+            for (int u = 0; u < FLAT_UNR; ++u) {
+                if (p[u] >= 0) {
+                    const uint32_t bit = 1u << (p[u] & 31);
+                    if (!(dw[u] & bit)) atomicOr(&newbits[(int64_t)jj[u] * W + (p[u] >> 5)], bit);
+                }
+            }
+        }
+        __syncwarp();
+    }
+}
+
+__global__ void __launch_bounds__(256) k_relabel(const int32_t* __restrict__ dst_pos, const int32_t* __restrict__ row_mb,
+                                                 const int64_t* cnt, const int64_t* __restrict__ findptr,
+                                                 const int32_t* __restrict__ fnbr, const int64_t* __restrict__ indptr,
+                                                 const uint32_t* __restrict__ dstbits, const uint32_t* __restrict__ newbits,
+                                                 const int64_t* __restrict__ wordoff, int64_t W,
+                                                 const int32_t* __restrict__ map, int64_t map_stride,
+                                                 const int64_t* __restrict__ mb_src_off, int32_t* __restrict__ indices,
+                                                 int64_t cap_e, const int32_t* __restrict__ fsrc_gid,
+                                                 int32_t* __restrict__ egid, const int64_t* __restrict__ otab) {
+    __shared__ int64_t s_vs[ORDER_SMEM + 1], s_rs[ORDER_SMEM];
+    __shared__ FlatRows s_rows[8];
+    const int nseg = order_load(otab, s_vs, s_rs);
+    int seg = 0;
+    const int64_t n = cnt[0];
+    const int lane = lane_id();
+    FlatRows& F = s_rows[warp_id()];
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t v0 = gw * 32; v0 < n; v0 += nw * 32) {
+        const int64_t vv = v0 + lane;
+        int d = 0;
+        if (vv < n) {
+            const int64_t r = order_map(vv, nseg, s_vs, s_rs, seg);
+            const int32_t q = dst_pos[r];
+            const int64_t b = findptr[q];
+            d = (int)(findptr[q + 1] - b);
+            const int j = row_mb[r];
+            F.fb[lane] = b;
+            F.j[lane] = j;
+            F.ob[lane] = indptr[r];
+            // j's new sources follow the whole dst prefix: id = n_dst + off_j + (wordoff - wordoff_j0) + rank
+            F.base[lane] = n + mb_src_off[j] - wordoff[(int64_t)j * W];
+        }
+        const int incl = warp_incl_scan(d);
+        F.pre[lane + 1] = incl;
+        if (lane == 0) F.pre[0] = 0;
+        __syncwarp();
+        const int total = F.pre[32];
+        for (int f0 = lane; f0 < total; f0 += 32 * FLAT_UNR) {
+            int32_t p[FLAT_UNR];
+            int kk[FLAT_UNR];
+#pragma unroll
+            for (int u = 0; u < FLAT_UNR; ++u) {
+                const int f = f0 + 32 * u;
+                p[u] = -1;
+                if (f < total) {
+                    const int k = flat_row(F, f);
+                    kk[u] = k;
+                    p[u] = fnbr[F.fb[k] + (f - F.pre[k])];
+                }
+            }
+            uint32_t dw[FLAT_UNR], nwd[FLAT_UNR];
+            int64_t wo[FLAT_UNR];
+            int32_t gid[FLAT_UNR];
+#pragma unroll
+            for (int u = 0; u < FLAT_UNR; ++u) {
+                if (p[u] >= 0) {
+                    const int64_t wi = (int64_t)F.j[kk[u]] * W + (p[u] >> 5);
+                    dw[u] = dstbits[wi];
+                    nwd[u] = newbits[wi];
+                    wo[u] = wordoff[wi];
+                    if (egid) gid[u] = fsrc_gid[p[u]];
+                }
+            }
+#pragma unroll
+            for (int u = 0; u < FLAT_UNR; ++u) {
+                if (p[u] >= 0) {
+                    const int k = kk[u];
+                    const int f = f0 + 32 * u;
+                    const uint32_t bit = 1u << (p[u] & 31);
+                    int64_t id;                         // src id, global within the group
+                    if (dw[u] & bit) id = map[(int64_t)F.j[k] * map_stride + p[u]];
+                    else id = F.base[k] + wo[u] + __popc(nwd[u] & (bit - 1));
+                    const int64_t o = F.ob[k] + (f - F.pre[k]);
+                    if (o < cap_e) {
+                        indices[o] = (int32_t)id;
+                        if (egid) egid[o] = gid[u];
+                    }
+                }
+            }
+        }
+        __syncwarp();
     }
 }
 
@@ -212,51 +350,6 @@ __global__ void k_emit_dst(const int32_t* __restrict__ dst_pos, const int32_t* _
     }
 }
 
-template <int LPR>
-__global__ void k_relabel(const int32_t* __restrict__ dst_pos, const int32_t* __restrict__ row_mb, const int64_t* cnt,
-                          const int64_t* __restrict__ findptr, const int32_t* __restrict__ fnbr,
-                          const int64_t* __restrict__ indptr, const uint32_t* __restrict__ dstbits,
-                          const uint32_t* __restrict__ newbits, const int64_t* __restrict__ wordoff, int64_t W,
-                          const int32_t* __restrict__ map, int64_t map_stride, const int64_t* __restrict__ mb_dst_off,
-                          const int64_t* __restrict__ mb_src_off, int32_t* __restrict__ indices, int64_t cap_e,
-                          const int32_t* __restrict__ fsrc_gid, int32_t* __restrict__ egid,
-                          const int64_t* __restrict__ otab) {
-    __shared__ int64_t s_vs[ORDER_SMEM + 1], s_rs[ORDER_SMEM];
-    const int nseg = order_load(otab, s_vs, s_rs);
-    int seg = 0;
-    const int64_t n = cnt[0];
-    const int lane = lane_id() % LPR;
-    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / LPR;
-    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) / LPR;
-    for (int64_t rv = gw; rv < n; rv += nw) {
-        const int64_t r = order_map(rv, nseg, s_vs, s_rs, seg);
-        const int j = row_mb[r];
-        const int32_t q = dst_pos[r];
-        const int64_t fb = findptr[q], fe = findptr[q + 1];
-        const int64_t ob = indptr[r];
-        const uint32_t* db = dstbits + j * W;
-        const uint32_t* nb = newbits + j * W;
-        const int64_t* wo = wordoff + j * W;
-        const int64_t wo0 = wo[0];
-        const int64_t so = cnt[0] + mb_src_off[j];      // j's new sources follow the whole dst prefix
-        (void)mb_dst_off;
-        for (int64_t i = fb + lane; i < fe; i += LPR) {
-            const int32_t p = fnbr[i];
-            const int32_t w = p >> 5;
-            const uint32_t bit = 1u << (p & 31);
-            int64_t id;                                 // src id, global within the group
-            if (db[w] & bit) id = map[j * map_stride + p];
-            else id = so + (wo[w] - wo0) + __popc(nb[w] & (bit - 1));
-            const int64_t o = ob + (i - fb);
-            if (o < cap_e) {
-                indices[o] = (int32_t)id;
-                if (egid) egid[o] = fsrc_gid[p];
-            }
-        }
-    }
-}
-
-// single CTA: the micro-batch-major order table of layer l (extract.h); segment (j, p), j-major
 struct LayerPtrs { const int64_t* cnt[16]; const int64_t* off[16]; };
 __global__ void k_order_tab(int32_t c, int L, int l, const int64_t* __restrict__ top_off, LayerPtrs lp_,
                             int64_t* tab) {
@@ -349,15 +442,8 @@ void extract_group(betty_ctx* ctx, const ExtractArgs& a, cudaStream_t s) {
         // dedupe: dst bitmap + position map, then new-source bitmap
         k_mark_dst<<<grid_for(ctx, cap_d, 256), 256, 0, s>>>(dst_pos, row_mb, dst_off, B.cnt, a.sc.dstbits, W,
                                                              a.sc.map, a.sc.map_stride);
-        const int64_t avg = F.n_dst > 0 ? (F.n_edges + F.n_dst - 1) / F.n_dst : 1;
-        const int lpr = avg <= 4 ? 4 : (avg <= 8 ? 8 : (avg <= 16 ? 16 : 32));
-        const int g_rows = grid_for(ctx, cap_d * lpr, 256);
-#define LPR_DISPATCH(KERNEL, ...)                                                           \
-        if (lpr == 4) KERNEL<4><<<g_rows, 256, 0, s>>>(__VA_ARGS__);                        \
-        else if (lpr == 8) KERNEL<8><<<g_rows, 256, 0, s>>>(__VA_ARGS__);                   \
-        else if (lpr == 16) KERNEL<16><<<g_rows, 256, 0, s>>>(__VA_ARGS__);                 \
-        else KERNEL<32><<<g_rows, 256, 0, s>>>(__VA_ARGS__);
-        LPR_DISPATCH(k_mark_new, dst_pos, row_mb, B.cnt, F.indptr, F.nbr, a.sc.dstbits, a.sc.newbits, W, otab)
+        const int g_rows = grid_for(ctx, cap_d, 256);       // 32 rows per warp
+        k_mark_new<<<g_rows, 256, 0, s>>>(dst_pos, row_mb, B.cnt, F.indptr, F.nbr, a.sc.dstbits, a.sc.newbits, W, otab);
         // ascending order of new sources = popcount scan over the bitmap words
         k_popc<<<grid_for(ctx, cW, 256), 256, 0, s>>>(a.sc.newbits, cW, a.sc.wordcnt);
         scan_i32(ctx, a.sc.wordcnt, a.sc.wordoff, nullptr, cW, 0, nullptr, s);
@@ -367,10 +453,9 @@ void extract_group(betty_ctx* ctx, const ExtractArgs& a, cudaStream_t s) {
                                                              F.src_gid, B.src_pos, B.src_gid, B.src_mb, cap_s);
         k_emit_new<<<grid_for(ctx, cW, 256), 256, 0, s>>>(a.sc.newbits, W, c, B.cnt, a.sc.wordoff, dst_off, B.mb_src_off,
                                                           F.src_gid, B.src_pos, B.src_gid, B.src_mb, cap_s);
-        LPR_DISPATCH(k_relabel, dst_pos, row_mb, B.cnt, F.indptr, F.nbr, B.indptr, a.sc.dstbits, a.sc.newbits,
-                     a.sc.wordoff, W, a.sc.map, a.sc.map_stride, dst_off, B.mb_src_off, B.indices, cap_e, F.src_gid,
-                     B.egid, otab)
-#undef LPR_DISPATCH
+        k_relabel<<<g_rows, 256, 0, s>>>(dst_pos, row_mb, B.cnt, F.indptr, F.nbr, B.indptr, a.sc.dstbits, a.sc.newbits,
+                                         a.sc.wordoff, W, a.sc.map, a.sc.map_stride, B.mb_src_off, B.indices, cap_e,
+                                         F.src_gid, B.egid, otab);
         k_clear_bits<<<grid_for(ctx, cW, 256), 256, 0, s>>>(a.sc.dstbits, a.sc.newbits, cW);
         if (B.t_indptr && (a.csc_mask >> l & 1))
             csr_transpose(ctx, B.indptr, B.indices, B.cnt + 0, B.cnt + 1, B.cnt + 2, cap_d, cap_s, cap_e,

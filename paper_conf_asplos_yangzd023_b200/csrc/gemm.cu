@@ -252,7 +252,8 @@ int gemm_red_splits(int64_t M_cap, int K1, int N) {
     const int tiles = ((K1 + XB - 1) / XB) * ((N + XB - 1) / XB);
     const int mtiles = (K1 + 127) / 128;
     const int64_t chunks = std::max<int64_t>(1, (M_cap + XCHUNK - 1) / XCHUNK);
-    const int want = std::max(std::max(1, (148 * 4) / tiles), std::max(1, 148 / mtiles));
+    (void)mtiles;
+    const int want = std::max(148, (148 * 4) / tiles);
     return (int)std::max<int64_t>(1, std::min<int64_t>(chunks, want));
 }
 

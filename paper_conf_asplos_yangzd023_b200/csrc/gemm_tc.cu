@@ -445,6 +445,8 @@ __global__ void __launch_bounds__(ROW_THREADS, 1) k_tc_row(const __grid_constant
 struct RedArgs {
     const int64_t* M_dev;      // rows (the reduction dimension)
     int K1, N, BN, nbA, nbB, stages, S, mtiles;
+    int mt_cta;                // feature tiles per CTA: 1 (grid = mtiles x S) or mtiles (grid = S; A, B read once)
+    int acc_stride;            // TMEM columns per feature tile accumulator
     float* partials;           // [S][K1][N]
     uint32_t tmem_cols;
 };
@@ -455,7 +457,8 @@ __global__ void __launch_bounds__(THREADS, 1) k_tc_red(const __grid_constant__ C
     uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
     const int S = p.stages;
     const uint32_t box = BK * 128;                    // 64 rows x 128 B
-    const uint32_t a_bytes = p.nbA * box, b_bytes = p.nbB * box;
+    const int nbA_cta = p.nbA * p.mt_cta;             // A boxes per stage (64 features each)
+    const uint32_t a_bytes = nbA_cta * box, b_bytes = p.nbB * box;
     const uint32_t stage_bytes = a_bytes + b_bytes;
     uint64_t* full = (uint64_t*)(smem + S * stage_bytes);
     uint64_t* empty = full + S;
@@ -463,7 +466,9 @@ __global__ void __launch_bounds__(THREADS, 1) k_tc_red(const __grid_constant__ C
     uint32_t* tslot = (uint32_t*)(tfull + 1);
 
     const int warp = threadIdx.x >> 5;
-    const int mt = blockIdx.x % p.mtiles, split = blockIdx.x / p.mtiles;
+    const int nsplit = p.mt_cta == 1 ? p.mtiles : 1;
+    const int mt0 = p.mt_cta == 1 ? blockIdx.x % p.mtiles : 0;
+    const int split = blockIdx.x / nsplit;
     const int64_t M = *p.M_dev;
     const int64_t nkb = (M + BK - 1) / BK;
     const int64_t kb0 = nkb * split / p.S, kb1 = nkb * (split + 1) / p.S;
@@ -487,7 +492,7 @@ __global__ void __launch_bounds__(THREADS, 1) k_tc_red(const __grid_constant__ C
                 mbar_wait(&empty[s], ph ^ 1);
                 uint8_t* sa = smem + s * stage_bytes;
                 mbar_expect_tx(&full[s], stage_bytes);
-                for (int i = 0; i < p.nbA; ++i) tma_2d(sa + i * box, &tmA, mt * BM + i * 64, (int)(kb * BK), &full[s]);
+                for (int i = 0; i < nbA_cta; ++i) tma_2d(sa + i * box, &tmA, mt0 * BM + i * 64, (int)(kb * BK), &full[s]);
                 for (int i = 0; i < p.nbB; ++i) tma_2d(sa + a_bytes + i * box, &tmB, i * 64, (int)(kb * BK), &full[s]);
                 if (++s == S) { s = 0; ph ^= 1; }
             }
@@ -501,7 +506,7 @@ __global__ void __launch_bounds__(THREADS, 1) k_tc_red(const __grid_constant__ C
             uint8_t* sa = smem + s * stage_bytes;
             const int64_t valid = M - kb * BK;       // rows of this k-block inside [0, M)
             if (valid < BK) {                        // zero the tail rows of every box (generic proxy)
-                const int nboxes = p.nbA + p.nbB;
+                const int nboxes = nbA_cta + p.nbB;
                 for (int idx = threadIdx.x & 31; idx < nboxes * (BK - (int)valid) * 8; idx += 32) {
                     const int b = idx / ((BK - (int)valid) * 8);
                     const int rr = (idx / 8) % (BK - (int)valid) + (int)valid;
@@ -513,13 +518,16 @@ __global__ void __launch_bounds__(THREADS, 1) k_tc_red(const __grid_constant__ C
             }
             fence_after();
             if (elect_lane0()) {
-                const uint32_t a0 = su32(sa), b0 = a0 + a_bytes;
+                const uint32_t b0 = su32(sa) + a_bytes;
+                for (int mt = 0; mt < p.mt_cta; ++mt) {
+                    const uint32_t a0 = su32(sa) + mt * p.nbA * box;
 #pragma unroll
-                for (int k = 0; k < BK / UK; ++k) {
-                    // MN-major SW128: atoms of 64 (MN) x 8 (K) at SBO = 1024 along K, LBO = box along MN
-                    const uint64_t ad = sdesc(a0 + k * UK * 128, box, 1024);
-                    const uint64_t bd = sdesc(b0 + k * UK * 128, box, 1024);
-                    umma_f16(tmem, ad, bd, idesc, (kb != kb0 || k != 0));
+                    for (int k = 0; k < BK / UK; ++k) {
+                        // MN-major SW128: atoms of 64 (MN) x 8 (K) at SBO = 1024 along K, LBO = box along MN
+                        const uint64_t ad = sdesc(a0 + k * UK * 128, box, 1024);
+                        const uint64_t bd = sdesc(b0 + k * UK * 128, box, 1024);
+                        umma_f16(tmem + mt * p.acc_stride, ad, bd, idesc, (kb != kb0 || k != 0));
+                    }
                 }
                 umma_commit(&empty[s]);
                 if (kb == kb1 - 1) umma_commit(&tfull[0]);
@@ -530,21 +538,29 @@ __global__ void __launch_bounds__(THREADS, 1) k_tc_red(const __grid_constant__ C
     } else {
         const int q = warp & 3;
         const int r_in = q * 32 + (threadIdx.x & 31);
-        const int feat = mt * BM + r_in;
-        float* out = p.partials + ((int64_t)split * p.K1 + feat) * p.N;
         if (kb1 > kb0) {
             mbar_wait(&tfull[0], 0);
             fence_after();
         }
-        for (int c0 = 0; c0 < p.BN; c0 += 32) {
-            float v[32];
-            if (kb1 > kb0) tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + c0, v);
-            else {
+        for (int mt = 0; mt < p.mt_cta; ++mt) {
+            const int feat = (mt0 + mt) * BM + r_in;
+            float* out = p.partials + ((int64_t)split * p.K1 + feat) * p.N;
+            for (int c0 = 0; c0 < p.BN; c0 += 32) {
+                float v[32];
+                if (kb1 > kb0) tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + mt * p.acc_stride + c0, v);
+                else {
 #pragma unroll
-                for (int j = 0; j < 32; ++j) v[j] = 0.f;
+                    for (int j = 0; j < 32; ++j) v[j] = 0.f;
+                }
+                if (feat < p.K1) {
+                    if (c0 + 32 <= p.N && (p.N & 3) == 0) {
+#pragma unroll
+                        for (int j = 0; j < 32; j += 4) *(float4*)(out + c0 + j) = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
+                    } else {
+                        for (int j = 0; j < 32 && c0 + j < p.N; ++j) out[c0 + j] = v[j];
+                    }
+                }
             }
-            if (feat < p.K1)
-                for (int j = 0; j < 32 && c0 + j < p.N; ++j) out[c0 + j] = v[j];
         }
         fence_before();
     }
@@ -674,19 +690,24 @@ bool gemm_red_tc(betty_ctx* c, const GemmRed& g, cudaStream_t s) {
     RedArgs p{};
     p.M_dev = g.M_dev; p.K1 = g.K1; p.N = g.N; p.BN = BN;
     p.nbA = BM / 64; p.nbB = (BN + 63) / 64;
-    const int stage_bytes = (p.nbA + p.nbB) * BK * 128;
-    p.stages = std::max(2, std::min(8, (200 * 1024) / stage_bytes));
     p.mtiles = (g.K1 + BM - 1) / BM;
+    p.acc_stride = (BN + 31) / 32 * 32;
+    // all feature tiles in one CTA when their accumulators fit TMEM and a stage fits 3x in smem:
+    // A and B are then read exactly once
+    const int stage_all = (p.nbA * p.mtiles + p.nbB) * BK * 128;
+    p.mt_cta = (p.mtiles * p.acc_stride <= 512 && 3 * stage_all <= 200 * 1024) ? p.mtiles : 1;
+    const int stage_bytes = (p.nbA * p.mt_cta + p.nbB) * BK * 128;
+    p.stages = std::max(2, std::min(8, (200 * 1024) / stage_bytes));
     p.S = g.S;
     p.partials = g.partials;
-    p.tmem_cols = tmem_cols_for(BN);
+    p.tmem_cols = tmem_cols_for(p.mt_cta * p.acc_stride);
     const size_t smem = (size_t)p.stages * stage_bytes + 1024 + 256;
     static bool attr = false;
     if (!attr) {
         cudaFuncSetAttribute(k_tc_red, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
         attr = true;
     }
-    k_tc_red<<<p.mtiles * p.S, THREADS, smem, s>>>(ma, mb, p);
+    k_tc_red<<<(p.mt_cta == 1 ? p.mtiles : 1) * p.S, THREADS, smem, s>>>(ma, mb, p);
     return true;
 }
 

@@ -14,14 +14,20 @@ struct betty_ctx {
     betty_free_fn dealloc = nullptr;
     void* user = nullptr;
     std::string err;
-    // scratch shared by stream-ordered primitives (one stream per ctx)
-    unsigned long long* scan_status = nullptr;   // decoupled look-back tile status
-    int64_t scan_status_cap = 0;
-    unsigned* counters = nullptr;                // [64] device counters, kept zero between launches
+    // scratch of the stream-ordered primitives, one set per concurrent stream ("lane"):
+    // lane 0 = the caller's stream, lane 1 = a plan's side stream (REG inside the step)
+    struct Lane {
+        unsigned long long* scan_status = nullptr;   // decoupled look-back tile status
+        int64_t scan_status_cap = 0;
+        unsigned* counters = nullptr;                // [64] device counters, kept zero between launches
+        int64_t* big_list = nullptr;                 // work list for oversize segments
+        int64_t big_list_cap = 0;
+        int* big_count = nullptr;
+    };
+    Lane lanes[2];
+    int lane = 0;                                // the set launches issued now use
+    Lane& L() { return lanes[lane]; }
     int* dev_err = nullptr;                      // device-side error flags (see betty::DEVERR_*)
-    int64_t* big_list = nullptr;                 // work list for oversize segments
-    int64_t big_list_cap = 0;
-    int* big_count = nullptr;
 };
 
 namespace betty {

@@ -86,14 +86,14 @@ void loss_ce(betty_ctx* c, const float* logits, int64_t ldl, const int32_t* labe
              const int64_t* cnt, int64_t rows_cap, int C, float scale, float* dS, int64_t ldds, void* dS_act,
              bool act_bf16, int64_t ld_act, float* loss_accum, cudaStream_t s) {
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((rows_cap * 32 + 255) / 256, 512));
-    double* partials = (double*)(c->counters + 64);   // 512 doubles after the counters
+    double* partials = (double*)(c->L().counters + 64);   // 512 doubles after the counters
     if (act_bf16)
         k_loss<__nv_bfloat16><<<grid, 256, 0, s>>>(logits, ldl, labels, gid, cnt, C, scale, dS, ldds,
-                                                   (__nv_bfloat16*)dS_act, ld_act, partials, c->counters + CTR_LOSS,
+                                                   (__nv_bfloat16*)dS_act, ld_act, partials, c->L().counters + CTR_LOSS,
                                                    loss_accum);
     else
         k_loss<float><<<grid, 256, 0, s>>>(logits, ldl, labels, gid, cnt, C, scale, dS, ldds, (float*)dS_act, ld_act,
-                                           partials, c->counters + CTR_LOSS, loss_accum);
+                                           partials, c->L().counters + CTR_LOSS, loss_accum);
 }
 
 // ------------------------------------------------------------------ adam

@@ -115,13 +115,13 @@ __global__ void __launch_bounds__(SCAN_THREADS) k_scan(const Tin* __restrict__ i
 
 void ensure_scan_scratch(betty_ctx* c, int64_t n_cap, cudaStream_t s) {
     const int64_t tiles = (n_cap + SCAN_TILE - 1) / SCAN_TILE + 1;
-    if (tiles > c->scan_status_cap) {
+    if (tiles > c->L().scan_status_cap) {
         // growing is only legal outside graph capture; plan creation sizes it first
-        if (c->scan_status) ctx_free(c, c->scan_status, s);
+        if (c->L().scan_status) ctx_free(c, c->L().scan_status, s);
         const int64_t cap = tiles * 2 + 1024;
-        c->scan_status = (unsigned long long*)ctx_alloc(c, sizeof(unsigned long long) * cap, s);
-        cudaMemsetAsync(c->scan_status, 0, sizeof(unsigned long long) * cap, s);
-        c->scan_status_cap = cap;
+        c->L().scan_status = (unsigned long long*)ctx_alloc(c, sizeof(unsigned long long) * cap, s);
+        cudaMemsetAsync(c->L().scan_status, 0, sizeof(unsigned long long) * cap, s);
+        c->L().scan_status_cap = cap;
     }
 }
 
@@ -132,8 +132,8 @@ static void scan_impl(betty_ctx* c, const Tin* in, int64_t* out, const int64_t* 
     ensure_scan_scratch(c, n_cap, s);
     int64_t tiles = (n_cap + SCAN_TILE - 1) / SCAN_TILE;
     int grid = (int)std::min<int64_t>(std::max<int64_t>(tiles, 1), (int64_t)c->num_sms * 2);
-    k_scan<Tin><<<grid, SCAN_THREADS, 0, s>>>(in, out, n_dev, n_fixed, total_dev, c->scan_status,
-                                              c->counters + CTR_SCAN);
+    k_scan<Tin><<<grid, SCAN_THREADS, 0, s>>>(in, out, n_dev, n_fixed, total_dev, c->L().scan_status,
+                                              c->L().counters + CTR_SCAN);
 }
 
 void scan_i64(betty_ctx* c, const int64_t* in, int64_t* out, const int64_t* n_dev, int64_t n_fixed, int64_t n_cap,
@@ -263,10 +263,10 @@ void segsort_i32(betty_ctx* c, const int64_t* ptr, int32_t* keys, const int64_t*
                  int64_t nseg_cap, cudaStream_t s) {
     if (!nseg_dev) nseg_cap = nseg_fixed;
     int grid = (int)std::min<int64_t>((nseg_cap + 255) / 256 + 1, (int64_t)c->num_sms * 8);
-    k_reset_int<<<1, 1, 0, s>>>(c->big_count);
-    k_segsort_warp<<<grid, 256, 0, s>>>(ptr, keys, nseg_dev, nseg_fixed, c->big_list, c->big_count, c->big_list_cap,
+    k_reset_int<<<1, 1, 0, s>>>(c->L().big_count);
+    k_segsort_warp<<<grid, 256, 0, s>>>(ptr, keys, nseg_dev, nseg_fixed, c->L().big_list, c->L().big_count, c->L().big_list_cap,
                                         c->dev_err);
-    k_segsort_big<<<c->num_sms, 1024, SEG_CTA_MAX * 4, s>>>(ptr, keys, c->big_list, c->big_count, c->dev_err);
+    k_segsort_big<<<c->num_sms, 1024, SEG_CTA_MAX * 4, s>>>(ptr, keys, c->L().big_list, c->L().big_count, c->dev_err);
 }
 
 // ------------------------------------------------------------- transpose

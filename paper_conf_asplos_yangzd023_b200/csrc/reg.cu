@@ -246,9 +246,9 @@ void reg_phase1(betty_ctx* c, const RegArgs& a, cudaStream_t s) {
     csr_transpose(c, a.indptr, a.idx, a.n_rows_dev, a.n_cols_dev, a.n_edges_dev, a.rows_cap, a.cols_cap, a.edges_cap,
                   a.t_indptr, a.t_idx, a.tcnt, true, s);
     const int gw = (int)std::max<int64_t>(1, std::min<int64_t>((a.rows_cap * 32 + 255) / 256, (int64_t)c->num_sms * 16));
-    k_reset_big<<<1, 1, 0, s>>>(c->big_count);
-    k_reg_ub<<<gw, 256, 0, s>>>(a.indptr, a.idx, a.t_indptr, a.n_rows_dev, a.ub, c->big_list, c->big_count,
-                                c->big_list_cap, c->dev_err);
+    k_reset_big<<<1, 1, 0, s>>>(c->L().big_count);
+    k_reg_ub<<<gw, 256, 0, s>>>(a.indptr, a.idx, a.t_indptr, a.n_rows_dev, a.ub, c->L().big_list, c->L().big_count,
+                                c->L().big_list_cap, c->dev_err);
     scan_i64(c, a.ub, a.off, a.n_rows_dev, 0, a.rows_cap, a.ub_total_dev, s);
 }
 
@@ -257,7 +257,7 @@ void reg_phase2(betty_ctx* c, const RegArgs& a, cudaStream_t s) {
     k_reg_rows_warp<<<gw, 256, 0, s>>>(a.indptr, a.idx, a.t_indptr, a.t_idx, a.n_rows_dev, a.ub, a.off, a.tcol, a.tw,
                                        a.row_nnz);
     k_reg_rows_cta<<<c->num_sms, 1024, REG_CTA_MAX * 4, s>>>(a.indptr, a.idx, a.t_indptr, a.t_idx, a.ub, a.off,
-                                                            c->big_list, c->big_count, a.tcol, a.tw, a.row_nnz);
+                                                            c->L().big_list, c->L().big_count, a.tcol, a.tw, a.row_nnz);
     scan_i64(c, a.row_nnz, a.out_indptr, a.n_rows_dev, 0, a.rows_cap, a.nnz_total_dev, s);
 }
 
