@@ -1,3 +1,4 @@
+#include <cmath>
 #include <cstdlib>
 // agg.cu -- a3/a5: GraphSAGE aggregation forward and backward (HBM-bound
 // CSR segment reductions), Table 1, Eq. 1 PAPER.md:269.
@@ -39,6 +40,7 @@ template <typename T> __device__ __forceinline__ const T* row_ptr(const T* X, in
 // table (extract.h) the rows are visited micro-batch by micro-batch, and the
 // grid is exactly the resident CTAs so all warps sweep the order together.
 constexpr int AGG_EB = 12;       // edges per cp.async batch (layer-0 fanout 10 fits one batch)
+constexpr int AGG_CHUNK = 64;    // rows a warp claims at a time
 __device__ __forceinline__ uint64_t l2_evict_last_policy() {
     uint64_t pol;
     asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
@@ -82,7 +84,8 @@ __global__ void __launch_bounds__(256) k_agg_mean_xa(const Tin* __restrict__ X, 
                                                      const int32_t* __restrict__ emap,
                                                      const int64_t* __restrict__ indptr, const int64_t* cnt,
                                                      const int64_t* __restrict__ otab, int Fi, int Fp,
-                                                     Tout* __restrict__ XA, int64_t ldxa, int hint) {
+                                                     Tout* __restrict__ XA, int64_t ldxa, int hint, int vlo, int vhi,
+                                                     unsigned* ctr) {
     using VI = Vec<Tin>;
     constexpr int VW = VI::N;
     constexpr int RPW = 32 / LPR;
@@ -100,34 +103,67 @@ __global__ void __launch_bounds__(256) k_agg_mean_xa(const Tin* __restrict__ X, 
     const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
     int seg = 0;
-    for (int64_t v0 = gw * RPW; v0 < nd; v0 += nw * RPW) {
+    // row meta of the next iteration is loaded while the current gather is in flight:
+    // (v, b, e) and the first batch of edge ids (one per lane)
+    auto meta = [&](int64_t v0, int64_t& v, int64_t& b, int64_t& e, int32_t& my) {
         const int64_t vv = v0 + grp;
-        const bool rowok = vv < nd;
-        const int64_t v = rowok ? order_map(vv, nseg, s_vs, s_rs, seg) : vv;
-        int64_t b = 0, e = 0;
-        if (rowok) { b = __ldcs(indptr + v); e = __ldcs(indptr + v + 1); }
+        v = vv; b = 0; e = 0; my = 0;
+        if (vv < nd) {
+            v = order_map(vv, nseg, s_vs, s_rs, seg);
+            b = __ldcs(indptr + v);
+            e = __ldcs(indptr + v + 1);
+            if (sub < e - b && sub < EB) { my = __ldcs(erow + b + sub); if (emap) my = emap[my]; }
+        }
+    };
+    // dynamic schedule: a warp claims AGG_CHUNK consecutive (virtual) rows at a time, so
+    // the rows in flight chip-wide stay a narrow window of the micro-batch-major order
+    // (statically strided warps drift apart and spread the gathered working set)
+    __shared__ int64_t s_claim[8];
+    const int wib = threadIdx.x >> 5;
+    auto claim = [&]() -> int64_t {
+        if (lane == 0) s_claim[wib] = (int64_t)atomicAdd(ctr, 1u) * AGG_CHUNK;
+        __syncwarp();
+        const int64_t c0 = s_claim[wib];
+        __syncwarp();
+        return c0;
+    };
+    int64_t cbase = claim();
+    int64_t v0 = cbase;
+    int64_t v, b, e;
+    int32_t my;
+    meta(v0, v, b, e, my);
+    while (v0 < nd) {
+        const bool rowok = v0 + grp < nd;
         const float inv = e > b ? 1.0f / (float)(e - b) : 0.0f;
         Tout* out = XA + v * ldxa;
-        for (int vb = 0; vb < NV; vb += LPR) {
-            const int vi = vb + sub;
-            const bool act = rowok && vi < NV;
-            float acc[VW];
+        float acc[VW];
 #pragma unroll
-            for (int t = 0; t < VW; ++t) acc[t] = 0.f;
-            for (int64_t e0 = b; e0 < e; e0 += EB) {
-                const int n = (int)mn64(EB, e - e0);
-                int32_t my = 0;
-                if (sub < n) { my = __ldcs(erow + e0 + sub); if (emap) my = emap[my]; }
-                for (int t = 0; t < n; ++t) {
-                    const int32_t u = __shfl_sync(gmask, my, t, LPR);
-                    if (act) cp_async16(wb + t * LPR + sub, X + (int64_t)u * ldx + vi * VW, pol, hint != 0);
-                }
-                cp_async_wait_all();
-                if (act) {
-                    for (int t = 0; t < n; ++t) VI::add_raw(acc, *(const typename VI::Raw*)(wb + t * LPR + sub));
-                }
-                __syncwarp(gmask);
+        for (int t = 0; t < VW; ++t) acc[t] = 0.f;
+        const int vi = vlo + sub;
+        const bool act = rowok && vi < vhi;
+        bool pending = false;
+        if (vhi - vlo <= LPR && e - b <= EB) {
+            // fast path: the whole row in one batch, its ids already in `my`
+            const int n = (int)(e - b);
+            for (int t = 0; t < n; ++t) {
+                const int32_t u = __shfl_sync(gmask, my, t, LPR);
+                if (act) cp_async16(wb + t * LPR + sub, X + (int64_t)u * ldx + vi * VW, pol, hint != 0);
             }
+            asm volatile("cp.async.commit_group;" ::: "memory");
+            pending = true;
+        }
+        // next rows' meta overlaps the gather
+        int64_t vn0 = v0 + RPW;
+        if (vn0 >= cbase + AGG_CHUNK) { cbase = claim(); vn0 = cbase; }
+        int64_t vn, bn, en;
+        int32_t myn;
+        meta(vn0, vn, bn, en, myn);
+        if (pending) {
+            asm volatile("cp.async.wait_group 0;" ::: "memory");
+            const int n = (int)(e - b);
+            if (act)
+                for (int t = 0; t < n; ++t) VI::add_raw(acc, *(const typename VI::Raw*)(wb + t * LPR + sub));
+            __syncwarp(gmask);
             if (act) {
                 VI self;
                 self.load(X + (int64_t)(srow ? srow[v] : (int32_t)v) * ldx + vi * VW);
@@ -149,12 +185,45 @@ __global__ void __launch_bounds__(256) k_agg_mean_xa(const Tin* __restrict__ X, 
                     }
                 }
             }
+        } else {
+            // general path: rows longer than a batch or wider than the lane group
+            for (int vb = vlo; vb < vhi; vb += LPR) {
+                const int vj = vb + sub;
+                const bool actj = rowok && vj < vhi;
+                float accj[VW];
+#pragma unroll
+                for (int t = 0; t < VW; ++t) accj[t] = 0.f;
+                for (int64_t e0 = b; e0 < e; e0 += EB) {
+                    const int n = (int)mn64(EB, e - e0);
+                    int32_t mj = 0;
+                    if (sub < n) { mj = erow[e0 + sub]; if (emap) mj = emap[mj]; }
+                    for (int t = 0; t < n; ++t) {
+                        const int32_t u = __shfl_sync(gmask, mj, t, LPR);
+                        if (actj) cp_async16(wb + t * LPR + sub, X + (int64_t)u * ldx + vj * VW, pol, hint != 0);
+                    }
+                    cp_async_wait_all();
+                    if (actj)
+                        for (int t = 0; t < n; ++t) VI::add_raw(accj, *(const typename VI::Raw*)(wb + t * LPR + sub));
+                    __syncwarp(gmask);
+                }
+                if (actj) {
+                    VI self;
+                    self.load(X + (int64_t)(srow ? srow[v] : (int32_t)v) * ldx + vj * VW);
+#pragma unroll
+                    for (int t = 0; t < VW; ++t) {
+                        const int col = vj * VW + t;
+                        if (col < Fi) { st_act(out + col, self.v[t]); st_act(out + Fp + col, accj[t] * inv); }
+                    }
+                }
+            }
         }
-        if (rowok) {
-            // pad columns of both halves, the ones column (bias), trailing pad
+        if (rowok && vhi == NV) {
+            // (last column pass) pad columns of both halves, the ones column (bias), trailing pad
             for (int col = NV * VW + sub; col < Fp; col += LPR) { st_act(out + col, 0.f); st_act(out + Fp + col, 0.f); }
             for (int col = 2 * Fp + sub; col < ldxa; col += LPR) st_act(out + col, col == 2 * Fp ? 1.f : 0.f);
         }
+        v = vn; b = bn; e = en; my = myn;
+        v0 = vn0;
     }
 }
 
@@ -536,14 +605,23 @@ template <typename K> static int resident_grid(betty_ctx* c, K kernel, int threa
 
 void agg_mean_xa(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const int32_t* srow, const int32_t* erow,
                  const int32_t* emap, const int64_t* indptr, const int64_t* cnt, const int64_t* otab, int64_t rows_cap,
-                 int Fi, int Fp, void* XA, bool xa_bf16, int64_t ldxa, cudaStream_t s) {
+                 int64_t src_per_mb, int Fi, int Fp, void* XA, bool xa_bf16, int64_t ldxa, cudaStream_t s) {
     const int vw = x_bf16 ? 8 : 4;
     const int nv = (Fi + vw - 1) / vw;
-    const int lpr = nv <= 8 ? 8 : (nv <= 16 ? 16 : 32);
-    const int64_t warps = (rows_cap + (32 / lpr) - 1) / (32 / lpr);
-    // experiment switches (default: L2 evict_last hint on feature rows, micro-batch-major order)
+    // Column passes: one micro-batch's gathered rows must stay L2-resident between their
+    // uses; when (source rows of a micro-batch) x (row bytes) exceeds the budget, the
+    // feature columns are gathered in several passes over the rows, each pass touching
+    // only a slice of every row (the rows' metadata is re-read, the features are not).
+    static const double budget = getenv("BETTY_AGG_WS_MB") ? atof(getenv("BETTY_AGG_WS_MB")) * 1e6 : 1e12;
+    unsigned* ctr = c->L().counters + CTR_AGG;
     static const int hint = getenv("BETTY_AGG_NOHINT") ? 0 : 1;
     static const bool no_order = getenv("BETTY_AGG_NOORDER") != nullptr;
+    const double ws = (double)src_per_mb * (double)nv * 16.0;
+    int passes = (int)std::max(1.0, std::min((double)nv, std::ceil(ws / budget)));
+    const int pv = (nv + passes - 1) / passes;
+    passes = (nv + pv - 1) / pv;
+    const int lpr = pv <= 8 ? 8 : (pv <= 16 ? 16 : 32);
+    const int64_t warps = (rows_cap + (32 / lpr) - 1) / (32 / lpr);
 #define AGG_L(LPR) DISPATCH_ACT(x_bf16, TI, DISPATCH_ACT(xa_bf16, TO, {                                           \
         const size_t sm = (size_t)8 * (32 / LPR) * (AGG_EB < LPR ? AGG_EB : LPR) * LPR * 16;                    \
         static bool attr = false;                                                                              \
@@ -552,8 +630,10 @@ void agg_mean_xa(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const in
         int per_sm = 1;                                                                                        \
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_agg_mean_xa<TI, TO, LPR>, 256, sm);           \
         const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((warps + 7) / 8, (int64_t)std::max(per_sm, 1) * c->num_sms)); \
-        k_agg_mean_xa<TI, TO, LPR><<<grid, 256, sm, s>>>((const TI*)X, ldx, srow, erow, emap, indptr, cnt,        \
-                                                        no_order ? nullptr : otab, Fi, Fp, (TO*)XA, ldxa, hint); }))
+        for (int pz = 0; pz < passes; ++pz) {                                                                   \
+            cudaMemsetAsync(ctr, 0, sizeof(unsigned), s);                                                      \
+            k_agg_mean_xa<TI, TO, LPR><<<grid, 256, sm, s>>>((const TI*)X, ldx, srow, erow, emap, indptr, cnt,    \
+                no_order ? nullptr : otab, Fi, Fp, (TO*)XA, ldxa, hint, pz * pv, std::min(nv, (pz + 1) * pv), ctr); } }))
     if (lpr == 8) { AGG_L(8); } else if (lpr == 16) { AGG_L(16); } else { AGG_L(32); }
 #undef AGG_L
 }

@@ -602,6 +602,24 @@ extern "C" betty_status betty_plan_create(betty_ctx* c, const betty_model* model
         return fail(c, BETTY_ENOMEM, "plan: arena allocation failed");
     }
     if (m.layers[0].kind == KIND_AGG) p->X.layers[0].egid = A.get<int32_t>(ce[0]);   // layer-0 gather by gid
+    // full-batch CSC of the layers whose micro-batch CSC is built every step (filtered from it)
+    for (int l = 0; l < L; ++l) {
+        if (!(p->csc_mask >> l & 1)) continue;
+        const betty_block& fb = full[l];
+        int64_t* fti = A.get<int64_t>(fb.n_src + 1);
+        int32_t* ftn = A.get<int32_t>(fb.n_edges);
+        int64_t* hc = A.get<int64_t>(4);
+        int32_t* tc = A.get<int32_t>(fb.n_src);
+        if (!A.ok) break;
+        const int64_t h3[4] = {fb.n_dst, fb.n_src, fb.n_edges, 0};
+        cudaMemcpyAsync(hc, h3, sizeof(h3), cudaMemcpyHostToDevice, s);
+        ensure_scan_scratch(c, std::max(fb.n_src, fb.n_edges) + 1, s);
+        csr_transpose(c, fb.indptr, fb.indices, hc, hc + 1, hc + 2, std::max<int64_t>(fb.n_dst, 1),
+                      std::max<int64_t>(fb.n_src, 1), std::max<int64_t>(fb.n_edges, 1), fti, ftn, tc, false, s);
+        if ((st = sync_check(c, s))) { betty_plan_destroy(c, p); return st; }
+        p->full[l].t_indptr = fti;
+        p->full[l].t_nbr = ftn;
+    }
     if (!A.ok) {
         betty_plan_destroy(c, p);
         return fail(c, BETTY_ENOMEM, "plan: arena allocation failed");
@@ -614,7 +632,8 @@ extern "C" betty_status betty_plan_create(betty_ctx* c, const betty_model* model
     for (int l = 0; l < L; ++l) {
         const ExtractLayer& B = p->X.layers[l];
         p->views[l] = BlockView{B.indptr, B.indices, B.t_indptr, B.t_indices, B.src_gid, B.cnt, B.cap_dst, B.cap_src,
-                                B.cap_e, B.egid, B.order_tab};
+                                B.cap_e, B.egid, B.order_tab,
+                                n_my > 0 ? std::max<int64_t>(1, p->info.n_src[std::min(l, 15)] / n_my) : 1};
     }
     // scan scratch for the largest scan of a step (never grows inside a capture)
     {

@@ -138,7 +138,8 @@ __device__ __forceinline__ int flat_row(const FlatRows& F, int f) {
 __global__ void __launch_bounds__(256) k_mark_new(const int32_t* __restrict__ dst_pos, const int32_t* __restrict__ row_mb,
                                                   const int64_t* cnt, const int64_t* __restrict__ findptr,
                                                   const int32_t* __restrict__ fnbr, const uint32_t* __restrict__ dstbits,
-                                                  uint32_t* newbits, int64_t W, const int64_t* __restrict__ otab) {
+                                                  uint32_t* newbits, int64_t W, const int64_t* __restrict__ otab,
+                                                  unsigned* ctr) {
     __shared__ int64_t s_vs[ORDER_SMEM + 1], s_rs[ORDER_SMEM];
     __shared__ FlatRows s_rows[8];
     const int nseg = order_load(otab, s_vs, s_rs);
@@ -146,9 +147,15 @@ __global__ void __launch_bounds__(256) k_mark_new(const int32_t* __restrict__ ds
     const int64_t n = cnt[0];
     const int lane = lane_id();
     FlatRows& F = s_rows[warp_id()];
-    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    for (int64_t v0 = gw * 32; v0 < n; v0 += nw * 32) {
+    // dynamic schedule (32-row claims): the rows in flight stay a narrow window of the
+    // micro-batch-major order, so one micro-batch's bitmaps / map stay in L2
+    __shared__ int64_t s_claim[8];
+    for (;;) {
+        if (lane == 0) s_claim[warp_id()] = (int64_t)atomicAdd(ctr, 1u) * 32;
+        __syncwarp();
+        const int64_t v0 = s_claim[warp_id()];
+        __syncwarp();
+        if (v0 >= n) break;
         const int64_t vv = v0 + lane;
         int d = 0;
         if (vv < n) {
@@ -201,7 +208,8 @@ __global__ void __launch_bounds__(256) k_relabel(const int32_t* __restrict__ dst
                                                  const int32_t* __restrict__ map, int64_t map_stride,
                                                  const int64_t* __restrict__ mb_src_off, int32_t* __restrict__ indices,
                                                  int64_t cap_e, const int32_t* __restrict__ fsrc_gid,
-                                                 int32_t* __restrict__ egid, const int64_t* __restrict__ otab) {
+                                                 int32_t* __restrict__ egid, const int64_t* __restrict__ otab,
+                                                 unsigned* ctr) {
     __shared__ int64_t s_vs[ORDER_SMEM + 1], s_rs[ORDER_SMEM];
     __shared__ FlatRows s_rows[8];
     const int nseg = order_load(otab, s_vs, s_rs);
@@ -209,9 +217,15 @@ __global__ void __launch_bounds__(256) k_relabel(const int32_t* __restrict__ dst
     const int64_t n = cnt[0];
     const int lane = lane_id();
     FlatRows& F = s_rows[warp_id()];
-    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    for (int64_t v0 = gw * 32; v0 < n; v0 += nw * 32) {
+    // dynamic schedule (32-row claims): the rows in flight stay a narrow window of the
+    // micro-batch-major order, so one micro-batch's bitmaps / map stay in L2
+    __shared__ int64_t s_claim[8];
+    for (;;) {
+        if (lane == 0) s_claim[warp_id()] = (int64_t)atomicAdd(ctr, 1u) * 32;
+        __syncwarp();
+        const int64_t v0 = s_claim[warp_id()];
+        __syncwarp();
+        if (v0 >= n) break;
         const int64_t vv = v0 + lane;
         int d = 0;
         if (vv < n) {
@@ -350,6 +364,44 @@ __global__ void k_emit_dst(const int32_t* __restrict__ dst_pos, const int32_t* _
     }
 }
 
+// CSC of a micro-batch layer from the full-batch CSC (no atomics, no sort for the
+// top layer): local src u (full position p, slot j) keeps the full-batch column of p
+// restricted to j's dst rows, relabelled through the dst map.  Top-layer dst ids
+// ascend with the full position, so the columns come out ascending.
+__global__ void k_csc_count(const int32_t* __restrict__ src_pos, const int32_t* __restrict__ src_mb, const int64_t* cnt,
+                            const int64_t* __restrict__ ft_indptr, const int32_t* __restrict__ ft_nbr,
+                            const uint32_t* __restrict__ dstbits, int64_t W, int32_t* __restrict__ tcnt) {
+    const int64_t n = cnt[1];
+    for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < n; u += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t p = src_pos[u];
+        const uint32_t* db = dstbits + (int64_t)src_mb[u] * W;
+        int k = 0;
+        for (int64_t e = ft_indptr[p], ee = ft_indptr[p + 1]; e < ee; ++e) {
+            const int32_t q = ft_nbr[e];
+            k += (db[q >> 5] >> (q & 31)) & 1u;
+        }
+        tcnt[u] = k;
+    }
+}
+__global__ void k_csc_fill(const int32_t* __restrict__ src_pos, const int32_t* __restrict__ src_mb, const int64_t* cnt,
+                           const int64_t* __restrict__ ft_indptr, const int32_t* __restrict__ ft_nbr,
+                           const uint32_t* __restrict__ dstbits, int64_t W, const int32_t* __restrict__ map,
+                           int64_t map_stride, const int64_t* __restrict__ t_indptr, int32_t* __restrict__ t_idx) {
+    const int64_t n = cnt[1];
+    for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < n; u += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t p = src_pos[u];
+        const int j = src_mb[u];
+        const uint32_t* db = dstbits + (int64_t)j * W;
+        const int32_t* mp = map + (int64_t)j * map_stride;
+        int64_t o = t_indptr[u];
+        for (int64_t e = ft_indptr[p], ee = ft_indptr[p + 1]; e < ee; ++e) {
+            const int32_t q = ft_nbr[e];
+            if ((db[q >> 5] >> (q & 31)) & 1u) t_idx[o++] = mp[q];
+        }
+    }
+}
+
+// single CTA: the micro-batch-major order table of layer l (extract.h); segment (j, p), j-major
 struct LayerPtrs { const int64_t* cnt[16]; const int64_t* off[16]; };
 __global__ void k_order_tab(int32_t c, int L, int l, const int64_t* __restrict__ top_off, LayerPtrs lp_,
                             int64_t* tab) {
@@ -443,7 +495,10 @@ void extract_group(betty_ctx* ctx, const ExtractArgs& a, cudaStream_t s) {
         k_mark_dst<<<grid_for(ctx, cap_d, 256), 256, 0, s>>>(dst_pos, row_mb, dst_off, B.cnt, a.sc.dstbits, W,
                                                              a.sc.map, a.sc.map_stride);
         const int g_rows = grid_for(ctx, cap_d, 256);       // 32 rows per warp
-        k_mark_new<<<g_rows, 256, 0, s>>>(dst_pos, row_mb, B.cnt, F.indptr, F.nbr, a.sc.dstbits, a.sc.newbits, W, otab);
+        unsigned* ctr = ctx->L().counters + CTR_EXTRACT;
+        cudaMemsetAsync(ctr, 0, sizeof(unsigned), s);
+        k_mark_new<<<g_rows, 256, 0, s>>>(dst_pos, row_mb, B.cnt, F.indptr, F.nbr, a.sc.dstbits, a.sc.newbits, W, otab,
+                                          ctr);
         // ascending order of new sources = popcount scan over the bitmap words
         k_popc<<<grid_for(ctx, cW, 256), 256, 0, s>>>(a.sc.newbits, cW, a.sc.wordcnt);
         scan_i32(ctx, a.sc.wordcnt, a.sc.wordoff, nullptr, cW, 0, nullptr, s);
@@ -453,11 +508,23 @@ void extract_group(betty_ctx* ctx, const ExtractArgs& a, cudaStream_t s) {
                                                              F.src_gid, B.src_pos, B.src_gid, B.src_mb, cap_s);
         k_emit_new<<<grid_for(ctx, cW, 256), 256, 0, s>>>(a.sc.newbits, W, c, B.cnt, a.sc.wordoff, dst_off, B.mb_src_off,
                                                           F.src_gid, B.src_pos, B.src_gid, B.src_mb, cap_s);
+        cudaMemsetAsync(ctr + 1, 0, sizeof(unsigned), s);
         k_relabel<<<g_rows, 256, 0, s>>>(dst_pos, row_mb, B.cnt, F.indptr, F.nbr, B.indptr, a.sc.dstbits, a.sc.newbits,
                                          a.sc.wordoff, W, a.sc.map, a.sc.map_stride, B.mb_src_off, B.indices, cap_e,
-                                         F.src_gid, B.egid, otab);
+                                         F.src_gid, B.egid, otab, ctr + 1);
+        const bool want_csc = B.t_indptr && (a.csc_mask >> l & 1);
+        if (want_csc && F.t_indptr) {           // from the full-batch CSC (needs the dst bitmap + map)
+            k_csc_count<<<grid_for(ctx, cap_s, 256), 256, 0, s>>>(B.src_pos, B.src_mb, B.cnt, F.t_indptr, F.t_nbr,
+                                                                  a.sc.dstbits, W, a.sc.tcnt);
+            scan_i32(ctx, a.sc.tcnt, B.t_indptr, B.cnt + 1, 0, cap_s, nullptr, s);
+            k_csc_fill<<<grid_for(ctx, cap_s, 256), 256, 0, s>>>(B.src_pos, B.src_mb, B.cnt, F.t_indptr, F.t_nbr,
+                                                                 a.sc.dstbits, W, a.sc.map, a.sc.map_stride,
+                                                                 B.t_indptr, B.t_indices);
+            if (l + 1 < a.L)                    // below the top layer dst ids are not monotone in position
+                segsort_i32(ctx, B.t_indptr, B.t_indices, B.cnt + 1, 0, cap_s, s);
+        }
         k_clear_bits<<<grid_for(ctx, cW, 256), 256, 0, s>>>(a.sc.dstbits, a.sc.newbits, cW);
-        if (B.t_indptr && (a.csc_mask >> l & 1))
+        if (want_csc && !F.t_indptr)
             csr_transpose(ctx, B.indptr, B.indices, B.cnt + 0, B.cnt + 1, B.cnt + 2, cap_d, cap_s, cap_e,
                           B.t_indptr, B.t_indices, a.sc.tcnt, false, s);
         dst_pos = B.src_pos;

@@ -11,6 +11,8 @@ struct ExtractFull {            // full-batch block l (device arrays, host sizes
     const int64_t* indptr;
     const int32_t* nbr;         // full-batch src positions
     const int32_t* src_gid;
+    const int64_t* t_indptr = nullptr;   // optional full-batch CSC (built once per plan): [n_src+1]
+    const int32_t* t_nbr = nullptr;      // [n_edges] full dst rows, ascending per column
 };
 
 struct ExtractLayer {           // group-concatenated micro-batch layer l (device arrays)

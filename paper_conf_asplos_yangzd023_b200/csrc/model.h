@@ -46,6 +46,7 @@ struct BlockView {              // one layer of a (group-concatenated) micro-bat
     int64_t cap_dst, cap_src, cap_e;
     const int32_t* egid = nullptr;   // optional [n_edges]: global id of each edge's source (layer 0)
     const int64_t* order_tab = nullptr;   // optional micro-batch-major dst row order (extract.h)
+    int64_t src_per_mb = 0;               // mean source rows per micro-batch (sizes the gather working set)
 };
 
 struct LayerBufs {

@@ -146,6 +146,75 @@ __device__ void bitonic_sort(int32_t* s, int P, int tid, int nthr, bool warp_onl
         }
 }
 
+// ascending bitonic sort of 32*K keys held lane-major in registers (lane l holds keys
+// [K*l, K*l+K)); strides >= K exchange across lanes with shuffles, smaller ones in-lane
+template <int K> __device__ __forceinline__ void warp_bitonic_regs(int32_t (&x)[K]) {
+    const int lane = lane_id();
+#pragma unroll
+    for (int size = 2; size <= 32 * K; size <<= 1) {
+#pragma unroll
+        for (int stride = size / 2; stride > 0; stride >>= 1) {
+            if (stride >= K) {
+                const int ls = stride / K;
+                const bool lower = (lane & ls) == 0;
+#pragma unroll
+                for (int k = 0; k < K; ++k) {
+                    const bool up = ((lane * K + k) & size) == 0;
+                    const int32_t y = __shfl_xor_sync(0xffffffffu, x[k], ls);
+                    x[k] = (lower == up) ? min(x[k], y) : max(x[k], y);
+                }
+            } else {
+#pragma unroll
+                for (int k = 0; k < K; ++k) {
+                    const int q = k ^ stride;
+                    if (q > k) {
+                        const bool up = ((lane * K + k) & size) == 0;
+                        const int32_t a = x[k], b = x[q];
+                        if ((a > b) == up) { x[k] = b; x[q] = a; }
+                    }
+                }
+            }
+        }
+    }
+}
+
+// sort buf[0, u) (u <= 32*K) in registers and run-length encode -> (col, w) ascending;
+// returns the count.  buf (>= 32*K+1 ints) is reused for the head positions.
+template <int K>
+__device__ __forceinline__ int warp_sort_rle(int32_t* buf, int u, int32_t* __restrict__ ocol, int32_t* __restrict__ ow) {
+    const int lane = lane_id();
+    int32_t x[K];
+#pragma unroll
+    for (int k = 0; k < K; ++k) x[k] = lane * K + k < u ? buf[lane * K + k] : INT_MAX;
+    __syncwarp();
+    warp_bitonic_regs<K>(x);
+    const int32_t prev_lane_last = __shfl_up_sync(0xffffffffu, x[K - 1], 1);
+    bool head[K];
+    int nh = 0;
+#pragma unroll
+    for (int k = 0; k < K; ++k) {
+        const int i = lane * K + k;
+        const int32_t prev = k == 0 ? prev_lane_last : x[k - 1];
+        head[k] = i < u && (i == 0 || x[k] != prev);
+        nh += head[k];
+    }
+    const int incl = warp_incl_scan(nh);
+    const int total = __shfl_sync(0xffffffffu, incl, 31);
+    int r = incl - nh;
+    // head positions -> buf (the keys live in registers now); run length = next head - this head
+#pragma unroll
+    for (int k = 0; k < K; ++k)
+        if (head[k]) buf[r++] = lane * K + k;
+    if (lane == 0) buf[total] = u;
+    __syncwarp();
+    r = incl - nh;
+#pragma unroll
+    for (int k = 0; k < K; ++k)
+        if (head[k]) { ocol[r] = x[k]; ow[r] = buf[r + 1] - buf[r]; ++r; }
+    __syncwarp();
+    return total;
+}
+
 __global__ void __launch_bounds__(256) k_reg_rows_warp(const int64_t* __restrict__ indptr,
                                                        const int32_t* __restrict__ idx,
                                                        const int64_t* __restrict__ t_indptr,
@@ -153,8 +222,7 @@ __global__ void __launch_bounds__(256) k_reg_rows_warp(const int64_t* __restrict
                                                        const int64_t* __restrict__ ub, const int64_t* __restrict__ off,
                                                        int32_t* __restrict__ tcol, int32_t* __restrict__ tw,
                                                        int64_t* __restrict__ nnz) {
-    __shared__ int32_t buf[8][REG_WARP_MAX];
-    __shared__ int s_cnt[8];
+    __shared__ int32_t buf[8][REG_WARP_MAX + 1];
     __shared__ int s_pre[8][33];
     __shared__ int64_t s_cb[8][32];
     const int64_t n = *n_rows_dev;
@@ -179,16 +247,11 @@ __global__ void __launch_bounds__(256) k_reg_rows_warp(const int64_t* __restrict
             __syncwarp();
             continue;
         }
-        int P = 32;
-        while (P < u) P <<= 1;
-        for (int t = (int)u + lane; t < P; t += 32) buf[w][t] = INT_MAX;
-        __syncwarp();
-        bitonic_sort(buf[w], P, lane, 32, true);
-        if (lane == 0) s_cnt[w] = 0;
-        __syncwarp();
-        reg_rle_store(buf[w], (int)u, tcol + off[i], tw + off[i], lane, 32, &s_cnt[w]);
-        if (lane == 0) nnz[i] = s_cnt[w];
-        __syncwarp();
+        int cnt;
+        if (u <= 64) cnt = warp_sort_rle<2>(buf[w], (int)u, tcol + off[i], tw + off[i]);
+        else if (u <= 128) cnt = warp_sort_rle<4>(buf[w], (int)u, tcol + off[i], tw + off[i]);
+        else cnt = warp_sort_rle<8>(buf[w], (int)u, tcol + off[i], tw + off[i]);
+        if (lane == 0) nnz[i] = cnt;
     }
 }
 

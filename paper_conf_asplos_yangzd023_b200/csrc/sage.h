@@ -11,7 +11,7 @@ namespace betty {
 // otab: optional micro-batch-major row order (extract.h), null = ascending rows
 void agg_mean_xa(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const int32_t* srow, const int32_t* erow,
                  const int32_t* emap, const int64_t* indptr, const int64_t* cnt, const int64_t* otab, int64_t rows_cap,
-                 int Fi, int Fp, void* XA, bool xa_bf16, int64_t ldxa, cudaStream_t s);
+                 int64_t src_per_mb, int Fi, int Fp, void* XA, bool xa_bf16, int64_t ldxa, cudaStream_t s);
 void agg_mean_pf(betty_ctx* c, const float* Y, int64_t ldy, const int64_t* indptr, const int32_t* idx,
                  const int64_t* cnt, int64_t rows_cap, int Fo, int Fop, bool relu, void* out, bool out_bf16,
                  int64_t ldo, cudaStream_t s);

@@ -26,8 +26,11 @@ def main():
     p.add_argument("--mode", default="bf16")
     p.add_argument("--graph", action="store_true")
     p.add_argument("--steps", type=int, default=1)
+    p.add_argument("--scale", type=float, default=1.0)
     a = p.parse_args()
     cfg = synth.CONFIGS[a.config]
+    if a.scale != 1.0:
+        cfg = synth.scaled(cfg, a.scale)
     ds = synth.make(cfg)
     ctx = B.betty_ctx_create(0)
     dev = B.blocks_to_device(ds.blocks)
@@ -53,7 +56,9 @@ def main():
     torch.cuda.synchronize()
     torch.cuda.profiler.stop()
     B.betty_sync_check(ctx)
-    print("prof_step ok", plan.info()["kernels_per_step"], "kernels/step")
+    info = plan.info()
+    print("prof_step ok", info["kernels_per_step"], "kernels/step; edges", info["edges"], "n_src", info["n_src"],
+          "n_dst", info["n_dst"])
     plan.free()
 
 
