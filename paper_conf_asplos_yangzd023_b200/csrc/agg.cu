@@ -40,7 +40,6 @@ template <typename T> __device__ __forceinline__ const T* row_ptr(const T* X, in
 // table (extract.h) the rows are visited micro-batch by micro-batch, and the
 // grid is exactly the resident CTAs so all warps sweep the order together.
 constexpr int AGG_EB = 12;       // edges per cp.async batch (layer-0 fanout 10 fits one batch)
-constexpr int AGG_CHUNK = 64;    // rows a warp claims at a time
 __device__ __forceinline__ uint64_t l2_evict_last_policy() {
     uint64_t pol;
     asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
@@ -53,6 +52,24 @@ __device__ __forceinline__ void cp_async16(void* sdst, const void* gsrc, uint64_
     else
         asm volatile("cp.async.cg.shared.global [%0], [%1], 16;"
                      ::"r"((uint32_t)__cvta_generic_to_shared(sdst)), "l"(gsrc) : "memory");
+}
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init1(uint64_t* b) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(b)) : "memory");
+}
+__device__ __forceinline__ void mbar_expect(uint64_t* b, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(b)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait_parity(uint64_t* b, uint32_t ph) {
+    uint32_t ok = 0;
+    while (!ok)
+        asm volatile("{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}"
+                     : "=r"(ok) : "r"(smem_u32(b)), "r"(ph) : "memory");
+}
+// one whole feature row global -> shared through the bulk-copy (TMA) engine, completion on `bar`
+__device__ __forceinline__ void bulk_row(void* sdst, const void* gsrc, uint32_t bytes, uint64_t* bar, uint64_t pol) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;"
+                 ::"r"(smem_u32(sdst)), "l"(gsrc), "r"(bytes), "r"(smem_u32(bar)), "l"(pol) : "memory");
 }
 __device__ __forceinline__ void cp_async_wait_all() {
     asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
@@ -91,87 +108,111 @@ __global__ void __launch_bounds__(256) k_agg_mean_xa(const Tin* __restrict__ X, 
     constexpr int RPW = 32 / LPR;
     static_assert(AGG_EB <= LPR || LPR == 8, "edge batch indices come from one lane each");
     constexpr int EB = AGG_EB < LPR ? AGG_EB : LPR;
-    extern __shared__ uint4 agg_sbuf[];              // [warps][RPW][EB][LPR]
+    constexpr int SLOTS = EB + 1;                    // EB neighbour rows + the self row
+    constexpr int CROWS = 8 * RPW;                   // rows a CTA claims per iteration
+    extern __shared__ uint4 agg_sbuf[];              // [warps][RPW][SLOTS][LPR]
     __shared__ int64_t s_vs[ORDER_SMEM + 1], s_rs[ORDER_SMEM];
+    __shared__ int64_t s_cta[3];
+    __shared__ uint64_t s_bar[8][RPW];               // per row group: bulk-copy completion
     const int64_t nd = cnt[0];
     const int nseg = order_load(otab, s_vs, s_rs);
     const int NV = (Fi + VW - 1) / VW;
     const int lane = lane_id(), sub = lane % LPR, grp = lane / LPR;
+    const int wib = threadIdx.x >> 5;
     const unsigned gmask = LPR == 32 ? 0xffffffffu : (((1u << LPR) - 1u) << (grp * LPR));
-    uint4* wb = agg_sbuf + ((int64_t)(threadIdx.x >> 5) * RPW + grp) * EB * LPR;
+    uint4* wb = agg_sbuf + ((int64_t)wib * RPW + grp) * SLOTS * LPR;
     const uint64_t pol = l2_evict_last_policy();
-    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const bool use_hint = hint != 0;
     int seg = 0;
-    // row meta of the next iteration is loaded while the current gather is in flight:
-    // (v, b, e) and the first batch of edge ids (one per lane)
-    auto meta = [&](int64_t v0, int64_t& v, int64_t& b, int64_t& e, int32_t& my) {
+    // Row meta (real row, edge range, first EB edge ids, self row) of the next iteration is
+    // loaded while the current gather is in flight.
+    struct Meta { int64_t v, b, e; int32_t my, sr; };
+    auto meta = [&](int64_t v0, Meta& m) {
         const int64_t vv = v0 + grp;
-        v = vv; b = 0; e = 0; my = 0;
+        m.v = vv; m.b = 0; m.e = 0; m.my = 0; m.sr = 0;
         if (vv < nd) {
-            v = order_map(vv, nseg, s_vs, s_rs, seg);
-            b = __ldcs(indptr + v);
-            e = __ldcs(indptr + v + 1);
-            if (sub < e - b && sub < EB) { my = __ldcs(erow + b + sub); if (emap) my = emap[my]; }
+            m.v = order_map(vv, nseg, s_vs, s_rs, seg);
+            m.b = __ldcs(indptr + m.v);
+            m.e = __ldcs(indptr + m.v + 1);
+            m.sr = srow ? __ldcs(srow + m.v) : (int32_t)m.v;
+            if (sub < m.e - m.b && sub < EB) { m.my = __ldcs(erow + m.b + sub); if (emap) m.my = emap[m.my]; }
         }
     };
-    // dynamic schedule: a warp claims AGG_CHUNK consecutive (virtual) rows at a time, so
-    // the rows in flight chip-wide stay a narrow window of the micro-batch-major order
-    // (statically strided warps drift apart and spread the gathered working set)
-    __shared__ int64_t s_claim[8];
-    const int wib = threadIdx.x >> 5;
-    auto claim = [&]() -> int64_t {
-        if (lane == 0) s_claim[wib] = (int64_t)atomicAdd(ctr, 1u) * AGG_CHUNK;
-        __syncwarp();
-        const int64_t c0 = s_claim[wib];
-        __syncwarp();
-        return c0;
-    };
-    int64_t cbase = claim();
-    int64_t v0 = cbase;
-    int64_t v, b, e;
-    int32_t my;
-    meta(v0, v, b, e, my);
-    while (v0 < nd) {
+    // Dynamic schedule: the CTA claims CROWS consecutive (virtual) rows per iteration, two
+    // iterations ahead (the atomic's latency is off the critical path).  The rows in flight
+    // chip-wide stay a narrow window of the micro-batch-major order, so the source rows one
+    // micro-batch shares are re-read from L2; statically strided warps drift apart instead.
+    // whole-row bulk copies (TMA engine): one instruction per neighbour row instead of one
+    // 16-byte cp.async per lane; only when one pass covers the whole row
+    const bool bulk = vlo == 0 && vhi == NV;
+    const uint32_t row_bytes = (uint32_t)NV * 16u;
+    uint64_t* bar = &s_bar[wib][grp];
+    uint32_t bph = 0;
+    if (sub == 0) mbar_init1(bar);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    unsigned pend = 0;
+    if (threadIdx.x == 0) {
+        s_cta[0] = (int64_t)atomicAdd(ctr, 1u) * CROWS;
+        s_cta[1] = (int64_t)atomicAdd(ctr, 1u) * CROWS;
+        pend = atomicAdd(ctr, 1u);
+    }
+    __syncthreads();
+    int64_t base = s_cta[0];
+    Meta cur;
+    meta(base + wib * RPW, cur);
+    for (int it = 0; base < nd; ++it) {
+        const int64_t v0 = base + wib * RPW;
         const bool rowok = v0 + grp < nd;
-        const float inv = e > b ? 1.0f / (float)(e - b) : 0.0f;
-        Tout* out = XA + v * ldxa;
-        float acc[VW];
-#pragma unroll
-        for (int t = 0; t < VW; ++t) acc[t] = 0.f;
         const int vi = vlo + sub;
         const bool act = rowok && vi < vhi;
-        bool pending = false;
-        if (vhi - vlo <= LPR && e - b <= EB) {
-            // fast path: the whole row in one batch, its ids already in `my`
-            const int n = (int)(e - b);
-            for (int t = 0; t < n; ++t) {
-                const int32_t u = __shfl_sync(gmask, my, t, LPR);
-                if (act) cp_async16(wb + t * LPR + sub, X + (int64_t)u * ldx + vi * VW, pol, hint != 0);
+        const int n = (int)(cur.e - cur.b);
+        const bool fast = vhi - vlo <= LPR && n <= EB;
+        if (fast && bulk) {      // neighbours + self: one bulk row copy per lane, completion on the group's barrier
+            if (rowok) {
+                if (sub == 0) mbar_expect(bar, (uint32_t)(n + 1) * row_bytes);
+                __syncwarp(gmask);
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                if (sub < n) bulk_row(wb + sub * LPR, X + (int64_t)cur.my * ldx, row_bytes, bar, pol);
+                if (sub == 0) bulk_row(wb + EB * LPR, X + (int64_t)cur.sr * ldx, row_bytes, bar, pol);
             }
+        } else if (fast) {      // the whole row (neighbours + self) in one batch of async copies
+            for (int t = 0; t < n; ++t) {
+                const int32_t u = __shfl_sync(gmask, cur.my, t, LPR);
+                if (act) cp_async16(wb + t * LPR + sub, X + (int64_t)u * ldx + vi * VW, pol, use_hint);
+            }
+            if (act) cp_async16(wb + EB * LPR + sub, X + (int64_t)cur.sr * ldx + vi * VW, pol, use_hint);
             asm volatile("cp.async.commit_group;" ::: "memory");
-            pending = true;
         }
-        // next rows' meta overlaps the gather
-        int64_t vn0 = v0 + RPW;
-        if (vn0 >= cbase + AGG_CHUNK) { cbase = claim(); vn0 = cbase; }
-        int64_t vn, bn, en;
-        int32_t myn;
-        meta(vn0, vn, bn, en, myn);
-        if (pending) {
-            asm volatile("cp.async.wait_group 0;" ::: "memory");
-            const int n = (int)(e - b);
-            if (act)
-                for (int t = 0; t < n; ++t) VI::add_raw(acc, *(const typename VI::Raw*)(wb + t * LPR + sub));
-            __syncwarp(gmask);
+        if (threadIdx.x == 0) {
+            s_cta[(it + 2) % 3] = (int64_t)pend * CROWS;
+            pend = atomicAdd(ctr, 1u);
+        }
+        __syncthreads();
+        const int64_t nbase = s_cta[(it + 1) % 3];
+        Meta nxt;
+        meta(nbase + wib * RPW, nxt);
+        Tout* out = XA + cur.v * ldxa;
+        const float inv = n > 0 ? 1.0f / (float)n : 0.0f;
+        if (fast) {
+            if (bulk) {
+                if (rowok) { mbar_wait_parity(bar, bph); bph ^= 1u; }
+            } else {
+                asm volatile("cp.async.wait_group 0;" ::: "memory");
+            }
             if (act) {
-                VI self;
-                self.load(X + (int64_t)(srow ? srow[v] : (int32_t)v) * ldx + vi * VW);
+                float acc[VW];
+#pragma unroll
+                for (int t = 0; t < VW; ++t) acc[t] = 0.f;
+                for (int t = 0; t < n; ++t) VI::add_raw(acc, *(const typename VI::Raw*)(wb + t * LPR + sub));
                 float so[VW], ao[VW];
+                const typename VI::Raw sraw = *(const typename VI::Raw*)(wb + EB * LPR + sub);
+#pragma unroll
+                for (int t = 0; t < VW; ++t) so[t] = 0.f;
+                VI::add_raw(so, sraw);
 #pragma unroll
                 for (int t = 0; t < VW; ++t) {
                     const bool in = vi * VW + t < Fi;
-                    so[t] = in ? self.v[t] : 0.f;
+                    so[t] = in ? so[t] : 0.f;
                     ao[t] = in ? acc[t] * inv : 0.f;
                 }
                 if constexpr (sizeof(Tin) == sizeof(Tout)) {
@@ -185,6 +226,7 @@ __global__ void __launch_bounds__(256) k_agg_mean_xa(const Tin* __restrict__ X, 
                     }
                 }
             }
+            __syncwarp(gmask);
         } else {
             // general path: rows longer than a batch or wider than the lane group
             for (int vb = vlo; vb < vhi; vb += LPR) {
@@ -193,22 +235,22 @@ __global__ void __launch_bounds__(256) k_agg_mean_xa(const Tin* __restrict__ X, 
                 float accj[VW];
 #pragma unroll
                 for (int t = 0; t < VW; ++t) accj[t] = 0.f;
-                for (int64_t e0 = b; e0 < e; e0 += EB) {
-                    const int n = (int)mn64(EB, e - e0);
+                for (int64_t e0 = cur.b; e0 < cur.e; e0 += EB) {
+                    const int nb = (int)mn64(EB, cur.e - e0);
                     int32_t mj = 0;
-                    if (sub < n) { mj = erow[e0 + sub]; if (emap) mj = emap[mj]; }
-                    for (int t = 0; t < n; ++t) {
+                    if (sub < nb) { mj = erow[e0 + sub]; if (emap) mj = emap[mj]; }
+                    for (int t = 0; t < nb; ++t) {
                         const int32_t u = __shfl_sync(gmask, mj, t, LPR);
-                        if (actj) cp_async16(wb + t * LPR + sub, X + (int64_t)u * ldx + vj * VW, pol, hint != 0);
+                        if (actj) cp_async16(wb + t * LPR + sub, X + (int64_t)u * ldx + vj * VW, pol, use_hint);
                     }
                     cp_async_wait_all();
                     if (actj)
-                        for (int t = 0; t < n; ++t) VI::add_raw(accj, *(const typename VI::Raw*)(wb + t * LPR + sub));
+                        for (int t = 0; t < nb; ++t) VI::add_raw(accj, *(const typename VI::Raw*)(wb + t * LPR + sub));
                     __syncwarp(gmask);
                 }
                 if (actj) {
                     VI self;
-                    self.load(X + (int64_t)(srow ? srow[v] : (int32_t)v) * ldx + vj * VW);
+                    self.load(X + (int64_t)cur.sr * ldx + vj * VW);
 #pragma unroll
                     for (int t = 0; t < VW; ++t) {
                         const int col = vj * VW + t;
@@ -222,8 +264,8 @@ __global__ void __launch_bounds__(256) k_agg_mean_xa(const Tin* __restrict__ X, 
             for (int col = NV * VW + sub; col < Fp; col += LPR) { st_act(out + col, 0.f); st_act(out + Fp + col, 0.f); }
             for (int col = 2 * Fp + sub; col < ldxa; col += LPR) st_act(out + col, col == 2 * Fp ? 1.f : 0.f);
         }
-        v = vn; b = bn; e = en; my = myn;
-        v0 = vn0;
+        cur = nxt;
+        base = nbase;
     }
 }
 
@@ -623,7 +665,7 @@ void agg_mean_xa(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const in
     const int lpr = pv <= 8 ? 8 : (pv <= 16 ? 16 : 32);
     const int64_t warps = (rows_cap + (32 / lpr) - 1) / (32 / lpr);
 #define AGG_L(LPR) DISPATCH_ACT(x_bf16, TI, DISPATCH_ACT(xa_bf16, TO, {                                           \
-        const size_t sm = (size_t)8 * (32 / LPR) * (AGG_EB < LPR ? AGG_EB : LPR) * LPR * 16;                    \
+        const size_t sm = (size_t)8 * (32 / LPR) * ((AGG_EB < LPR ? AGG_EB : LPR) + 1) * LPR * 16;                    \
         static bool attr = false;                                                                              \
         if (!attr) { cudaFuncSetAttribute(k_agg_mean_xa<TI, TO, LPR>, cudaFuncAttributeMaxDynamicSharedMemorySize, \
                                           (int)sm); attr = true; }                                             \

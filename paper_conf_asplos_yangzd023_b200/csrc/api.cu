@@ -179,8 +179,8 @@ static bool alloc_extract(Arena& A, int L, const ExtractFull* full, int64_t n_ou
     ExtractScratch& sc = X->sc;
     sc.dstbits = A.get<uint32_t>(c * W);
     sc.newbits = A.get<uint32_t>(c * W);
-    sc.map = A.get<int32_t>(c * max_full);
-    sc.map_stride = max_full;
+    for (int l = 0; l < L; ++l) sc.nrank[l] = A.get<uint2>(c * ((full[l].n_src + 31) / 32));
+    sc.drank_top = A.get<uint2>(c * ((full[L - 1].n_src + 31) / 32));
     sc.wordcnt = A.get<int32_t>(c * W);
     sc.wordoff = A.get<int64_t>(c * W + 1);
     sc.deg = A.get<int64_t>(max_dst);

@@ -100,16 +100,55 @@ __global__ void k_deg(const int32_t* __restrict__ dst_pos, const int64_t* __rest
 }
 
 __global__ void k_mark_dst(const int32_t* __restrict__ dst_pos, const int32_t* __restrict__ row_mb,
-                           const int64_t* __restrict__ mb_dst_off, const int64_t* cnt, uint32_t* dstbits, int64_t W,
-                           int32_t* __restrict__ map, int64_t map_stride) {
+                           const int64_t* cnt, uint32_t* dstbits, int64_t W) {
     const int64_t n = cnt[0];
     for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < n; r += (int64_t)gridDim.x * blockDim.x) {
         const int j = row_mb[r];
         const int32_t p = dst_pos[r];
         atomicOr(&dstbits[j * W + (p >> 5)], 1u << (p & 31));
-        map[j * map_stride + p] = (int32_t)r;           // dst rows are the group's src prefix: id = row
-        (void)mb_dst_off;
     }
+}
+
+// {bits, slot-relative popcount prefix} per bitmap word (wordoff: global exclusive scan)
+__global__ void k_pack_rank(const uint32_t* __restrict__ bits, const int64_t* __restrict__ wordoff, int64_t W,
+                            int64_t n, uint2* __restrict__ out) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        out[i] = make_uint2(bits[i], (uint32_t)(wordoff[i] - wordoff[(i / W) * W]));
+}
+
+// Local ids without a map.  Slot j's src list at layer l is [dst rows of layer l] ++ [new
+// sources, ascending position]; its dst rows ARE its src list at layer l+1 (same positions),
+// and at the top layer its outputs in ascending position.  So for a source p of slot j:
+//   new at layer l           -> n_dst(l) + off_l(j) + rank of p in j's new bitmap of layer l
+//   else new at layer q > l  -> the same at layer q (first such q)
+//   else (an output)         -> top_off(j) + rank of p in j's output bitmap
+struct RankSet {
+    const uint2* nr[16];
+    int64_t W[16];
+    const int64_t* cnt[16];     // layer counts (cnt[0] = group dst total)
+    const int64_t* off[16];     // per-slot offsets of the new sources
+    const uint2* dr;            // top layer output bitmap ranks
+    int64_t Wt;
+    const int64_t* top_off;
+    int L;
+};
+__device__ __forceinline__ int64_t rank_in(uint2 r, int32_t p) {
+    return (int64_t)r.y + __popc(r.x & ((1u << (p & 31)) - 1u));
+}
+// nr_l: the caller's (already loaded) word of layer l's new-rank array for (j, p)
+__device__ __forceinline__ int64_t src_id(const RankSet& R, int l, int j, int32_t p, uint2 nr_l) {
+    const uint32_t bit = 1u << (p & 31);
+    if (nr_l.x & bit) return R.cnt[l][0] + R.off[l][j] + rank_in(nr_l, p);
+    for (int q = l + 1; q < R.L; ++q) {
+        const uint2 nr = R.nr[q][(int64_t)j * R.W[q] + (p >> 5)];
+        if (nr.x & bit) return R.cnt[q][0] + R.off[q][j] + rank_in(nr, p);
+    }
+    return R.top_off[j] + rank_in(R.dr[(int64_t)j * R.Wt + (p >> 5)], p);
+}
+// id of dst row q of slot j at layer l (= its src id at layer l + 1, or its output rank)
+__device__ __forceinline__ int64_t dst_id(const RankSet& R, int l, int j, int32_t q) {
+    if (l + 1 >= R.L) return R.top_off[j] + rank_in(R.dr[(int64_t)j * R.Wt + (q >> 5)], q);
+    return src_id(R, l + 1, j, q, R.nr[l + 1][(int64_t)j * R.W[l + 1] + (q >> 5)]);
 }
 
 // Warp-flattened edge loops: a warp takes 32 consecutive (virtual) dst rows, lane
@@ -122,7 +161,6 @@ struct FlatRows {
     int pre[33];        // exclusive edge offsets of the warp's rows (pre[32] = total)
     int64_t fb[32];     // full-batch row start of each row
     int64_t ob[32];     // output offset (relabel) of each row
-    int64_t base[32];   // id base of the row's micro-batch new sources (relabel)
     int j[32];          // slot (micro-batch) of each row
 };
 __device__ __forceinline__ int flat_row(const FlatRows& F, int f) {
@@ -203,10 +241,7 @@ __global__ void __launch_bounds__(256) k_mark_new(const int32_t* __restrict__ ds
 __global__ void __launch_bounds__(256) k_relabel(const int32_t* __restrict__ dst_pos, const int32_t* __restrict__ row_mb,
                                                  const int64_t* cnt, const int64_t* __restrict__ findptr,
                                                  const int32_t* __restrict__ fnbr, const int64_t* __restrict__ indptr,
-                                                 const uint32_t* __restrict__ dstbits, const uint32_t* __restrict__ newbits,
-                                                 const int64_t* __restrict__ wordoff, int64_t W,
-                                                 const int32_t* __restrict__ map, int64_t map_stride,
-                                                 const int64_t* __restrict__ mb_src_off, int32_t* __restrict__ indices,
+                                                 const RankSet R, int l, int32_t* __restrict__ indices,
                                                  int64_t cap_e, const int32_t* __restrict__ fsrc_gid,
                                                  int32_t* __restrict__ egid, const int64_t* __restrict__ otab,
                                                  unsigned* ctr) {
@@ -237,8 +272,6 @@ __global__ void __launch_bounds__(256) k_relabel(const int32_t* __restrict__ dst
             F.fb[lane] = b;
             F.j[lane] = j;
             F.ob[lane] = indptr[r];
-            // j's new sources follow the whole dst prefix: id = n_dst + off_j + (wordoff - wordoff_j0) + rank
-            F.base[lane] = n + mb_src_off[j] - wordoff[(int64_t)j * W];
         }
         const int incl = warp_incl_scan(d);
         F.pre[lane + 1] = incl;
@@ -258,31 +291,25 @@ __global__ void __launch_bounds__(256) k_relabel(const int32_t* __restrict__ dst
                     p[u] = fnbr[F.fb[k] + (f - F.pre[k])];
                 }
             }
-            uint32_t dw[FLAT_UNR], nwd[FLAT_UNR];
-            int64_t wo[FLAT_UNR];
-            int32_t gid[FLAT_UNR];
+            uint2 nr[FLAT_UNR];
+            int32_t id[FLAT_UNR], gid[FLAT_UNR];
 #pragma unroll
             for (int u = 0; u < FLAT_UNR; ++u) {
                 if (p[u] >= 0) {
-                    const int64_t wi = (int64_t)F.j[kk[u]] * W + (p[u] >> 5);
-                    dw[u] = dstbits[wi];
-                    nwd[u] = newbits[wi];
-                    wo[u] = wordoff[wi];
+                    nr[u] = R.nr[l][(int64_t)F.j[kk[u]] * R.W[l] + (p[u] >> 5)];
                     if (egid) gid[u] = fsrc_gid[p[u]];
                 }
             }
 #pragma unroll
+            for (int u = 0; u < FLAT_UNR; ++u)
+                if (p[u] >= 0) id[u] = (int32_t)src_id(R, l, F.j[kk[u]], p[u], nr[u]);
+#pragma unroll
             for (int u = 0; u < FLAT_UNR; ++u) {
                 if (p[u] >= 0) {
                     const int k = kk[u];
-                    const int f = f0 + 32 * u;
-                    const uint32_t bit = 1u << (p[u] & 31);
-                    int64_t id;                         // src id, global within the group
-                    if (dw[u] & bit) id = map[(int64_t)F.j[k] * map_stride + p[u]];
-                    else id = F.base[k] + wo[u] + __popc(nwd[u] & (bit - 1));
-                    const int64_t o = F.ob[k] + (f - F.pre[k]);
+                    const int64_t o = F.ob[k] + (f0 + 32 * u - F.pre[k]);
                     if (o < cap_e) {
-                        indices[o] = (int32_t)id;
+                        indices[o] = id[u];
                         if (egid) egid[o] = gid[u];
                     }
                 }
@@ -385,18 +412,17 @@ __global__ void k_csc_count(const int32_t* __restrict__ src_pos, const int32_t* 
 }
 __global__ void k_csc_fill(const int32_t* __restrict__ src_pos, const int32_t* __restrict__ src_mb, const int64_t* cnt,
                            const int64_t* __restrict__ ft_indptr, const int32_t* __restrict__ ft_nbr,
-                           const uint32_t* __restrict__ dstbits, int64_t W, const int32_t* __restrict__ map,
-                           int64_t map_stride, const int64_t* __restrict__ t_indptr, int32_t* __restrict__ t_idx) {
+                           const uint32_t* __restrict__ dstbits, int64_t W, const RankSet R, int l,
+                           const int64_t* __restrict__ t_indptr, int32_t* __restrict__ t_idx) {
     const int64_t n = cnt[1];
     for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < n; u += (int64_t)gridDim.x * blockDim.x) {
         const int32_t p = src_pos[u];
         const int j = src_mb[u];
         const uint32_t* db = dstbits + (int64_t)j * W;
-        const int32_t* mp = map + (int64_t)j * map_stride;
         int64_t o = t_indptr[u];
         for (int64_t e = ft_indptr[p], ee = ft_indptr[p + 1]; e < ee; ++e) {
             const int32_t q = ft_nbr[e];
-            if ((db[q >> 5] >> (q & 31)) & 1u) t_idx[o++] = mp[q];
+            if ((db[q >> 5] >> (q & 31)) & 1u) t_idx[o++] = (int32_t)dst_id(R, l, j, q);
         }
     }
 }
@@ -492,8 +518,7 @@ void extract_group(betty_ctx* ctx, const ExtractArgs& a, cudaStream_t s) {
         k_deg<<<grid_for(ctx, cap_d, 256), 256, 0, s>>>(dst_pos, F.indptr, B.cnt, a.sc.deg);
         scan_i64(ctx, a.sc.deg, B.indptr, B.cnt + 0, 0, cap_d, B.cnt + 2, s);
         // dedupe: dst bitmap + position map, then new-source bitmap
-        k_mark_dst<<<grid_for(ctx, cap_d, 256), 256, 0, s>>>(dst_pos, row_mb, dst_off, B.cnt, a.sc.dstbits, W,
-                                                             a.sc.map, a.sc.map_stride);
+        k_mark_dst<<<grid_for(ctx, cap_d, 256), 256, 0, s>>>(dst_pos, row_mb, B.cnt, a.sc.dstbits, W);
         const int g_rows = grid_for(ctx, cap_d, 256);       // 32 rows per warp
         unsigned* ctr = ctx->L().counters + CTR_EXTRACT;
         cudaMemsetAsync(ctr, 0, sizeof(unsigned), s);
@@ -508,9 +533,26 @@ void extract_group(betty_ctx* ctx, const ExtractArgs& a, cudaStream_t s) {
                                                              F.src_gid, B.src_pos, B.src_gid, B.src_mb, cap_s);
         k_emit_new<<<grid_for(ctx, cW, 256), 256, 0, s>>>(a.sc.newbits, W, c, B.cnt, a.sc.wordoff, dst_off, B.mb_src_off,
                                                           F.src_gid, B.src_pos, B.src_gid, B.src_mb, cap_s);
+        // rank structures of this layer (and of the outputs at the top layer)
+        k_pack_rank<<<grid_for(ctx, cW, 256), 256, 0, s>>>(a.sc.newbits, a.sc.wordoff, W, cW, a.sc.nrank[l]);
+        if (l == a.L - 1) {
+            k_popc<<<grid_for(ctx, cW, 256), 256, 0, s>>>(a.sc.dstbits, cW, a.sc.wordcnt);
+            scan_i32(ctx, a.sc.wordcnt, a.sc.wordoff, nullptr, cW, 0, nullptr, s);
+            k_pack_rank<<<grid_for(ctx, cW, 256), 256, 0, s>>>(a.sc.dstbits, a.sc.wordoff, W, cW, a.sc.drank_top);
+        }
+        RankSet R{};
+        R.L = a.L;
+        for (int q = 0; q < a.L; ++q) {
+            R.nr[q] = a.sc.nrank[q];
+            R.W[q] = (a.full[q].n_src + 31) / 32;
+            R.cnt[q] = a.layers[q].cnt;
+            R.off[q] = a.layers[q].mb_src_off;
+        }
+        R.dr = a.sc.drank_top;
+        R.Wt = (a.full[a.L - 1].n_src + 31) / 32;
+        R.top_off = a.sc.top_dst_off;
         cudaMemsetAsync(ctr + 1, 0, sizeof(unsigned), s);
-        k_relabel<<<g_rows, 256, 0, s>>>(dst_pos, row_mb, B.cnt, F.indptr, F.nbr, B.indptr, a.sc.dstbits, a.sc.newbits,
-                                         a.sc.wordoff, W, a.sc.map, a.sc.map_stride, B.mb_src_off, B.indices, cap_e,
+        k_relabel<<<g_rows, 256, 0, s>>>(dst_pos, row_mb, B.cnt, F.indptr, F.nbr, B.indptr, R, l, B.indices, cap_e,
                                          F.src_gid, B.egid, otab, ctr + 1);
         const bool want_csc = B.t_indptr && (a.csc_mask >> l & 1);
         if (want_csc && F.t_indptr) {           // from the full-batch CSC (needs the dst bitmap + map)
@@ -518,8 +560,7 @@ void extract_group(betty_ctx* ctx, const ExtractArgs& a, cudaStream_t s) {
                                                                   a.sc.dstbits, W, a.sc.tcnt);
             scan_i32(ctx, a.sc.tcnt, B.t_indptr, B.cnt + 1, 0, cap_s, nullptr, s);
             k_csc_fill<<<grid_for(ctx, cap_s, 256), 256, 0, s>>>(B.src_pos, B.src_mb, B.cnt, F.t_indptr, F.t_nbr,
-                                                                 a.sc.dstbits, W, a.sc.map, a.sc.map_stride,
-                                                                 B.t_indptr, B.t_indices);
+                                                                 a.sc.dstbits, W, R, l, B.t_indptr, B.t_indices);
             if (l + 1 < a.L)                    // below the top layer dst ids are not monotone in position
                 segsort_i32(ctx, B.t_indptr, B.t_indices, B.cnt + 1, 0, cap_s, s);
         }

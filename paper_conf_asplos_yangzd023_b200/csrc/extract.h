@@ -73,8 +73,12 @@ __device__ __forceinline__ int64_t order_map(int64_t vv, int nseg, const int64_t
 struct ExtractScratch {
     uint32_t* dstbits;          // [c*Wmax]
     uint32_t* newbits;          // [c*Wmax]
-    int32_t* map;               // [c*map_stride]
-    int64_t map_stride;
+    // rank structures kept for the whole extraction: per layer the new-source bitmap of
+    // every slot with, per 32-bit word, the slot-relative count of set bits before it
+    // ({bits, prefix}); for the top layer the same for the dst (output) bitmap.  A source's
+    // local id is then computed (no position -> id map): see src_id() in extract.cu
+    uint2* nrank[16];           // [c*W_l]
+    uint2* drank_top;           // [c*W_{L-1}]
     int32_t* wordcnt;           // [c*Wmax]
     int64_t* wordoff;           // [c*Wmax+1]
     int64_t* deg;               // [max cap_dst]
