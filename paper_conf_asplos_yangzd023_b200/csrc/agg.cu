@@ -126,6 +126,8 @@ __global__ void __launch_bounds__(256) k_agg_mean_xa(const Tin* __restrict__ X, 
     int seg = 0;
     // Row meta (real row, edge range, first EB edge ids, self row) of the next iteration is
     // loaded while the current gather is in flight.
+    // Row meta (row id, edge range, first EB edge ids, self row) of the next iteration is
+    // loaded while the current rows' gathers are in flight.
     struct Meta { int64_t v, b, e; int32_t my, sr; };
     auto meta = [&](int64_t v0, Meta& m) {
         const int64_t vv = v0 + grp;
@@ -190,7 +192,7 @@ __global__ void __launch_bounds__(256) k_agg_mean_xa(const Tin* __restrict__ X, 
         __syncthreads();
         const int64_t nbase = s_cta[(it + 1) % 3];
         Meta nxt;
-        meta(nbase + wib * RPW, nxt);
+        meta(nbase + wib * RPW, nxt);       // next rows' meta overlaps the gather
         Tout* out = XA + cur.v * ldxa;
         const float inv = n > 0 ? 1.0f / (float)n : 0.0f;
         if (fast) {
@@ -490,7 +492,7 @@ static inline int pick_lpr_vpl(int nv) { return nv <= 4 * PF_VPL ? 4 : (nv <= 8 
 
 // mean, project-first fwd: S[v] = Y[v, Fop:] + (1/D_v) sum_u Y[u, :Fo] ; out = logits or ReLU -> H (+ ones)
 template <typename Tout, int LPR>
-__global__ void __launch_bounds__(256) k_agg_pf_v(const float* __restrict__ Y, int64_t ldy,
+__global__ void __launch_bounds__(256) k_agg_pf_v(const float* __restrict__ Y, const float* __restrict__ Ys, int64_t ldy,
                                                   const int64_t* __restrict__ indptr,
                                                   const int32_t* __restrict__ idx, const int64_t* cnt, int Fo, int Fop,
                                                   int relu, Tout* __restrict__ out, int64_t ldo) {
@@ -533,7 +535,7 @@ __global__ void __launch_bounds__(256) k_agg_pf_v(const float* __restrict__ Y, i
             for (int k = 0; k < PF_VPL; ++k) {
                 const int vi = vb + sub + LPR * k;
                 if (rowok && vi < NV) {
-                    const float4 sf = *(const float4*)(Y + v * ldy + Fop + vi * 4);
+                    const float4 sf = *(const float4*)(Ys + v * ldy + vi * 4);
                     float r[4] = {sf.x + acc[k].x * inv, sf.y + acc[k].y * inv, sf.z + acc[k].z * inv,
                                   sf.w + acc[k].w * inv};
 #pragma unroll
@@ -549,7 +551,7 @@ __global__ void __launch_bounds__(256) k_agg_pf_v(const float* __restrict__ Y, i
     }
 }
 
-// mean, project-first bwd: G[u] = [ sum_{v in CSC(u)} dS[v]/D_v | 0 | [u < nd] dS[u] | 0 ]
+// mean, project-first bwd: G[u] = sum_{v in CSC(u)} dS[v]/D_v (the self half is dS itself)
 template <typename Tin, typename Tout, int LPR>
 __global__ void __launch_bounds__(256) k_csc_pf_v(const Tin* __restrict__ dS, int64_t ldds,
                                                   const int64_t* __restrict__ indptr,
@@ -606,20 +608,11 @@ __global__ void __launch_bounds__(256) k_csc_pf_v(const Tin* __restrict__ dS, in
             for (int k = 0; k < PF_VPL; ++k) {
                 const int vi = vb + sub + LPR * k;
                 if (rowok && vi < NV) {
-                    VI self;
-                    if (u < nd) self.load_cg(dS + u * ldds + vi * VW);
-                    float ga[VW], gs[VW];
+                    float ga[VW];
 #pragma unroll
-                    for (int t = 0; t < VW; ++t) {
-                        const bool in = vi * VW + t < Fo;
-                        ga[t] = in ? acc[k][t] : 0.f;
-                        gs[t] = (in && u < nd) ? self.v[t] : 0.f;
-                    }
+                    for (int t = 0; t < VW; ++t) ga[t] = vi * VW + t < Fo ? acc[k][t] : 0.f;
 #pragma unroll
-                    for (int t = 0; t < VW; t += 4) {        // vector stores (Fop, ldg multiples of 8)
-                        st_act4(G + u * ldg + vi * VW + t, ga + t);
-                        st_act4(G + u * ldg + Fop + vi * VW + t, gs + t);
-                    }
+                    for (int t = 0; t < VW; t += 4) st_act4(G + u * ldg + vi * VW + t, ga + t);   // ldg multiple of 8
                 }
             }
         }
@@ -680,13 +673,13 @@ void agg_mean_xa(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const in
 #undef AGG_L
 }
 
-void agg_mean_pf(betty_ctx* c, const float* Y, int64_t ldy, const int64_t* indptr, const int32_t* idx,
+void agg_mean_pf(betty_ctx* c, const float* Y, const float* Ys, int64_t ldy, const int64_t* indptr, const int32_t* idx,
                  const int64_t* cnt, int64_t rows_cap, int Fo, int Fop, bool relu, void* out, bool out_bf16,
                  int64_t ldo, cudaStream_t s) {
     const int lpr = pick_lpr_vpl((Fo + 3) / 4);
     const int grid = warps_grid(c, (rows_cap + (32 / lpr) - 1) / (32 / lpr));
 #define PF_L(LPR) DISPATCH_ACT(out_bf16, TO, \
-        k_agg_pf_v<TO, LPR><<<grid, 256, 0, s>>>(Y, ldy, indptr, idx, cnt, Fo, Fop, relu ? 1 : 0, (TO*)out, ldo))
+        k_agg_pf_v<TO, LPR><<<grid, 256, 0, s>>>(Y, Ys, ldy, indptr, idx, cnt, Fo, Fop, relu ? 1 : 0, (TO*)out, ldo))
     if (lpr == 4) { PF_L(4); } else if (lpr == 8) { PF_L(8); } else if (lpr == 16) { PF_L(16); } else { PF_L(32); }
 #undef PF_L
 }

@@ -64,10 +64,18 @@ template <> struct Vec<__nv_bfloat16> {
     typedef uint4 Raw;
     __device__ __forceinline__ static Raw ld_raw(const __nv_bfloat16* p) { return __ldg(reinterpret_cast<const uint4*>(p)); }
     __device__ __forceinline__ static Raw zero_raw() { return make_uint4(0u, 0u, 0u, 0u); }
+    // bf16x2 word -> (lo << 16, hi & 0xffff0000) is the exact fp32 pair; summed with one FADD2
     __device__ __forceinline__ static void add_raw(float* acc, Raw t) {
-        const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&t);
+        const uint32_t w[4] = {t.x, t.y, t.z, t.w};
 #pragma unroll
-        for (int i = 0; i < 4; ++i) { float2 f = __bfloat1622float2(h[i]); acc[2 * i] += f.x; acc[2 * i + 1] += f.y; }
+        for (int i = 0; i < 4; ++i) {
+            const unsigned long long x = (unsigned long long)(w[i] << 16) | ((unsigned long long)(w[i] & 0xffff0000u) << 32);
+            unsigned long long a = (unsigned long long)__float_as_uint(acc[2 * i]) |
+                                   ((unsigned long long)__float_as_uint(acc[2 * i + 1]) << 32);
+            asm("add.rn.f32x2 %0, %0, %1;" : "+l"(a) : "l"(x));
+            acc[2 * i] = __uint_as_float((uint32_t)a);
+            acc[2 * i + 1] = __uint_as_float((uint32_t)(a >> 32));
+        }
     }
 };
 

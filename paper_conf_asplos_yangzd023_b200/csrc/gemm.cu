@@ -216,6 +216,14 @@ __device__ __forceinline__ int64_t map_index(const GradMap& m, int i, int j) {
         if (i >= m.Fp && i < m.Fp + m.Fi) return m.off_wn + (int64_t)(i - m.Fp) * m.Fo + j;
         if (i == 2 * m.Fp) return m.off_b + j;
         return -1;
+    } else if (m.mode == MAP_PF_N) {    // neighbour half alone: cols [0,Fo) W_neigh (bias row: none)
+        if (j >= m.Fo || i >= m.Fi) return -1;
+        return m.off_wn + (int64_t)i * m.Fo + j;
+    } else if (m.mode == MAP_PF_S) {    // self half alone: cols [0,Fo) W_self; row Fi = bias
+        if (j >= m.Fo) return -1;
+        if (i < m.Fi) return m.off_ws + (int64_t)i * m.Fo + j;
+        if (i == m.Fi) return m.off_b + j;
+        return -1;
     } else if (m.mode == MAP_PF) {      // cols [0,Fo) W_neigh, [Fop,Fop+Fo) W_self; row Fi = bias (self half)
         const bool self = j >= m.Fop && j < m.Fop + m.Fo;
         const bool nb = j < m.Fo;
@@ -234,15 +242,30 @@ __device__ __forceinline__ int64_t map_index(const GradMap& m, int i, int j) {
     }
 }
 
-__global__ void k_red_final(const float* __restrict__ partials, int S, int K1, int N, float* grad, GradMap map) {
+// grad[map(t)] += sum_s partials[s][t], t < K1*N: a CTA takes 32 consecutive outputs, its 8 warps
+// sum the splits s = w, w+8, ... (coalesced 128-byte rows of partials), then the 8 warp sums are
+// added in a fixed order -- deterministic, and 8x the parallelism of one thread per output
+__global__ void __launch_bounds__(256) k_red_final(const float* __restrict__ partials, int S, int K1, int N,
+                                                   float* grad, GradMap map) {
+    __shared__ float s_part[8][33];
     const int64_t n = (int64_t)K1 * N;
-    for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < n; t += (int64_t)gridDim.x * blockDim.x) {
-        const int i = (int)(t / N), j = (int)(t % N);
-        const int64_t dst = map_index(map, i, j);
-        if (dst < 0) continue;
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    for (int64_t t0 = (int64_t)blockIdx.x * 32; t0 < n; t0 += (int64_t)gridDim.x * 32) {
+        const int64_t t = t0 + lane;
         float sum = 0.f;
-        for (int sp = 0; sp < S; ++sp) sum += partials[(int64_t)sp * n + t];
-        grad[dst] += sum;
+        if (t < n)
+            for (int sp = w; sp < S; sp += 8) sum += partials[(int64_t)sp * n + t];
+        s_part[w][lane] = sum;
+        __syncthreads();
+        if (w == 0 && t < n) {
+            float tot = 0.f;
+#pragma unroll
+            for (int q = 0; q < 8; ++q) tot += s_part[q][lane];
+            const int i = (int)(t / N), j = (int)(t % N);
+            const int64_t dst = map_index(map, i, j);
+            if (dst >= 0) grad[dst] += tot;
+        }
+        __syncthreads();
     }
 }
 
@@ -260,7 +283,7 @@ int gemm_red_splits(int64_t M_cap, int K1, int N) {
 void gemm_red(betty_ctx* c, const GemmRed& g, cudaStream_t s) {
     if (c->use_tc && g.a_bf16 && g.b_bf16 && gemm_red_tc(c, g, s)) {
         const int64_t n = (int64_t)g.K1 * g.N;
-        const int gf = (int)std::max<int64_t>(1, std::min<int64_t>((n + 255) / 256, (int64_t)c->num_sms * 4));
+        const int gf = (int)std::max<int64_t>(1, std::min<int64_t>((n + 31) / 32, (int64_t)c->num_sms * 8));
         k_red_final<<<gf, 256, 0, s>>>(g.partials, g.S, g.K1, g.N, g.grad, g.map);
         return;
     }
@@ -274,7 +297,7 @@ void gemm_red(betty_ctx* c, const GemmRed& g, cudaStream_t s) {
         else k_gemm_red<float, float><<<grid, 256, 0, s>>>(g);
     }
     const int64_t n = (int64_t)g.K1 * g.N;
-    const int gf = (int)std::max<int64_t>(1, std::min<int64_t>((n + 255) / 256, (int64_t)c->num_sms * 4));
+    const int gf = (int)std::max<int64_t>(1, std::min<int64_t>((n + 31) / 32, (int64_t)c->num_sms * 8));
     k_red_final<<<gf, 256, 0, s>>>(g.partials, g.S, g.K1, g.N, g.grad, g.map);
 }
 

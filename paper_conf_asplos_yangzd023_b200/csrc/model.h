@@ -51,6 +51,7 @@ struct BlockView {              // one layer of a (group-concatenated) micro-bat
 
 struct LayerBufs {
     void* XA = nullptr;   void* gat = nullptr;  float* Y = nullptr;   void* G = nullptr;
+    float* Ys = nullptr;  float* R = nullptr;   // PF: self half over the dst rows; dS W_s^T residual
     float* dXA = nullptr; float* Zp = nullptr;  int32_t* arg = nullptr; void* dZp = nullptr;
     void* H = nullptr;    // input of layer l (l >= 1), written by layer l-1
     uint32_t* Hbits = nullptr;   // [H > 0] as bits (ldhb words per row), written with H by a tensor-core epilogue
@@ -60,7 +61,7 @@ struct LayerBufs {
     void* B = nullptr;    void* Bp = nullptr;
     void* Bt = nullptr;   void* Bpt = nullptr;   // K-major weight copies (BF16 tensor-core path)
     int64_t ldbt = 0, ldbpt = 0;
-    int S_main = 1, S_pool = 1;   // split counts of the dW reductions
+    int S_main = 1, S_pool = 1, S_self = 1;   // split counts of the dW reductions
 };
 
 // CUDA-event brackets around the launches of one kernel site (bench roofline)

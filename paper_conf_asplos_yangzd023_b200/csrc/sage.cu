@@ -53,8 +53,8 @@ bool make_model_cfg(int L, int aggr, int gemm, int feat_dtype, const int32_t* di
         base = c.off_b + c.Fo;
         c.ld_xa = r8(2 * c.Fp + 1);
         c.ld_gat = r8(c.Fi + 1);
-        c.ld_y = 2 * c.Fop;
-        c.ld_g = 2 * c.Fop;
+        c.ld_y = c.Fop;          // PF: Y = [H|1] [W_n; 0] over all src rows (the neighbour half only)
+        c.ld_g = c.Fop;          // PF: G = P^T D+ dS over all src rows (the self half is dS itself)
         c.ld_dxa = 2 * c.Fp;
         c.ld_zp = c.Fp;
         c.ld_dzp = c.Fp;
@@ -98,10 +98,14 @@ bool sage_alloc(betty_ctx* c, const ModelCfg& m, const std::vector<int64_t>& cap
         }
         if (L.kind == KIND_PF) {
             B.Y = (float*)A(ns * L.ld_y * 4);
+            B.Ys = (float*)A(nd * L.ld_y * 4);              // [H_dst|1] [W_s; b] over the dst rows only
             B.G = A(ns * L.ld_g * ea);
             B.B = A((L.Fi + 1) * L.ld_B * ea);
-            B.S_main = gemm_red_splits(ns, L.Fi + 1, 2 * L.Fop);
-            part_max = std::max<int64_t>(part_max, (int64_t)B.S_main * (L.Fi + 1) * 2 * L.Fop);
+            if (l > 0) B.R = (float*)A(nd * m.layers[l - 1].ld_ds * 4);   // dS W_s^T (dst rows), residual of dX
+            B.S_main = gemm_red_splits(ns, L.Fi + 1, L.Fop);
+            B.S_self = gemm_red_splits(nd, L.Fi + 1, L.Fop);
+            part_max = std::max<int64_t>(part_max, (int64_t)B.S_main * (L.Fi + 1) * L.Fop);
+            part_max = std::max<int64_t>(part_max, (int64_t)B.S_self * (L.Fi + 1) * L.Fop);
         }
         if (L.kind == KIND_POOL) {
             B.Zp = (float*)A(ns * L.ld_zp * 4);
@@ -129,7 +133,7 @@ bool sage_alloc(betty_ctx* c, const ModelCfg& m, const std::vector<int64_t>& cap
         if (L.last) {
             b->logits = (float*)A(nd * L.ld_out * 4);
             b->dS_last = (float*)A(nd * L.Fop * 4);
-            if (L.kind != KIND_PF) b->dS_last_act = A(nd * L.ld_ds * ea);
+            b->dS_last_act = A(nd * L.ld_ds * ea);
         }
     }
     b->partials = (float*)A(part_max * 4);
@@ -195,18 +199,27 @@ void sage_forward(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView*
             ones_operand(m, b, l, &Ao, &ldao);
         }
         if (L.kind == KIND_PF) {
+            // Y = [H|1] [W_n; 0] over every src row; Ys = [H_dst|1] [W_s; b] over the dst rows only
+            // (the combined weight matrix holds [W_n | W_s; 0 | b]: column sub-views)
+            const int64_t esz = m.bf16 ? 2 : 4;
             GemmRow g{};
             g.A = Ao; g.lda = ldao; g.a_bf16 = m.bf16;
             g.B = B.B; g.ldb = L.ld_B; g.b_bf16 = m.bf16; g.transB = false;
-            g.M_dev = V.cnt + 1; g.M_cap = V.cap_src; g.K = L.Fi + 1; g.N = 2 * L.Fop;
+            g.M_dev = V.cnt + 1; g.M_cap = V.cap_src; g.K = L.Fi + 1; g.N = L.Fop;
             g.Bt = B.Bt; g.ldbt = B.ldbt;
             g.C = B.Y; g.ldc = L.ld_y; g.c_bf16 = false; g.epi = EPI_STORE;
             PB(l == 0 ? PROBE_GEMM_FWD_L0 : PROBE_GEMM_FWD_L1);
             gemm_row(c, g, s);
             PE(l == 0 ? PROBE_GEMM_FWD_L0 : PROBE_GEMM_FWD_L1);
+            GemmRow gs = g;
+            gs.B = (const char*)B.B + L.Fop * esz;
+            gs.Bt = B.Bt ? (const void*)((const char*)B.Bt + (int64_t)L.Fop * B.ldbt * esz) : nullptr;
+            gs.M_dev = V.cnt + 0; gs.M_cap = V.cap_dst;
+            gs.C = B.Ys;
+            gemm_row(c, gs, s);
             PB(l == 0 ? PROBE_AGG_L0 : PROBE_AGG_L1);
-            agg_mean_pf(c, B.Y, L.ld_y, V.indptr, V.indices, V.cnt, V.cap_dst, L.Fo, L.Fop, !L.last, out, out_bf,
-                        L.ld_out, s);
+            agg_mean_pf(c, B.Y, B.Ys, L.ld_y, V.indptr, V.indices, V.cnt, V.cap_dst, L.Fo, L.Fop, !L.last, out,
+                        out_bf, L.ld_out, s);
             if (!L.last) b.l[l + 1].hbits_ok = false;
             PE(l == 0 ? PROBE_AGG_L0 : PROBE_AGG_L1);
             continue;
@@ -252,7 +265,7 @@ void sage_loss(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView* v,
     const LayerCfg& L = m.layers[m.L - 1];
     const BlockView& V = v[m.L - 1];
     loss_ce(c, b.logits, L.ld_out, labels, V.src_gid, V.cnt, V.cap_dst, L.Fo, scale, b.dS_last, L.Fop,
-            L.kind != KIND_PF ? b.dS_last_act : nullptr, m.bf16, L.ld_ds, loss_accum, s);
+            b.dS_last_act, m.bf16, L.ld_ds, loss_accum, s);
 }
 
 void sage_backward(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView* v, const void* feats,
@@ -268,6 +281,9 @@ void sage_backward(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView
         void* dS_prev = l > 0 ? b.l[l - 1].dS : nullptr;
         const int64_t ld_prev = l > 0 ? m.layers[l - 1].ld_ds : 0;
         if (L.kind == KIND_PF) {
+            // G = P^T D+ dS (all src rows); dW_n += [H|1]^T G ; [dW_s; db] += [H_dst|1]^T dS (dst rows);
+            // dX = G W_n^T + [dst] dS W_s^T (the second term as the epilogue residual), masked by ReLU'
+            const int64_t esz = m.bf16 ? 2 : 4;
             const bool ds_f32 = L.last;
             csc_pf(c, ds_f32 ? (const void*)b.dS_last : B.dS, !ds_f32 && m.bf16, ds_f32 ? L.Fop : L.ld_ds, V.indptr,
                    V.t_indptr, V.t_indices, V.cnt, V.cap_src, L.Fo, L.Fop, B.G, m.bf16, L.ld_g, s);
@@ -276,16 +292,27 @@ void sage_backward(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView
             GemmRed r{};
             r.A = Ao; r.lda = ldao; r.a_bf16 = m.bf16;
             r.B = B.G; r.ldb = L.ld_g; r.b_bf16 = m.bf16;
-            r.M_dev = V.cnt + 1; r.M_cap = V.cap_src; r.K1 = L.Fi + 1; r.N = 2 * L.Fop;
-            r.partials = b.partials; r.S = B.S_main; r.grad = grad; r.map = grad_map(L, MAP_PF);
+            r.M_dev = V.cnt + 1; r.M_cap = V.cap_src; r.K1 = L.Fi + 1; r.N = L.Fo;
+            r.partials = b.partials; r.S = B.S_main; r.grad = grad; r.map = grad_map(L, MAP_PF_N);
             gemm_red(c, r, s);
+            GemmRed rs = r;
+            rs.B = dS_act; rs.ldb = L.ld_ds;
+            rs.M_dev = V.cnt + 0; rs.M_cap = V.cap_dst; rs.S = B.S_self; rs.map = grad_map(L, MAP_PF_S);
+            gemm_red(c, rs, s);
             if (l > 0) {
+                GemmRow gr{};                       // R = dS W_s^T over the dst rows
+                gr.A = dS_act; gr.lda = L.ld_ds; gr.a_bf16 = m.bf16;
+                gr.B = (const char*)B.B + L.Fop * esz; gr.ldb = L.ld_B; gr.b_bf16 = m.bf16; gr.transB = true;
+                gr.M_dev = V.cnt + 0; gr.M_cap = V.cap_dst; gr.K = L.Fo; gr.N = L.Fi;
+                gr.C = B.R; gr.ldc = ld_prev; gr.c_bf16 = false; gr.epi = EPI_STORE;
+                gemm_row(c, gr, s);
                 GemmRow g{};
                 g.A = B.G; g.lda = L.ld_g; g.a_bf16 = m.bf16;
                 g.B = B.B; g.ldb = L.ld_B; g.b_bf16 = m.bf16; g.transB = true;
-                g.M_dev = V.cnt + 1; g.M_cap = V.cap_src; g.K = 2 * L.Fop; g.N = L.Fi;
-                g.C = dS_prev; g.ldc = ld_prev; g.c_bf16 = m.bf16; g.epi = EPI_MASK;
+                g.M_dev = V.cnt + 1; g.M_cap = V.cap_src; g.K = L.Fo; g.N = L.Fi;
+                g.C = dS_prev; g.ldc = ld_prev; g.c_bf16 = m.bf16; g.epi = EPI_RES_MASK;
                 g.mask = Hmask; g.ldm = ldh; g.m_bf16 = m.bf16;
+                g.res = B.R; g.ldr = ld_prev; g.nres_dev = V.cnt + 0;
                 if (B.hbits_ok) { g.mbits = B.Hbits; g.ldmb = B.ldhb; }
                 gemm_row(c, g, s);
             }

@@ -12,7 +12,8 @@ namespace betty {
 void agg_mean_xa(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const int32_t* srow, const int32_t* erow,
                  const int32_t* emap, const int64_t* indptr, const int64_t* cnt, const int64_t* otab, int64_t rows_cap,
                  int64_t src_per_mb, int Fi, int Fp, void* XA, bool xa_bf16, int64_t ldxa, cudaStream_t s);
-void agg_mean_pf(betty_ctx* c, const float* Y, int64_t ldy, const int64_t* indptr, const int32_t* idx,
+// S[v] = Ys[v] + (1/D_v) sum_u Y[u]  (Y: neighbour half over src rows, Ys: self half over dst rows, same ld)
+void agg_mean_pf(betty_ctx* c, const float* Y, const float* Ys, int64_t ldy, const int64_t* indptr, const int32_t* idx,
                  const int64_t* cnt, int64_t rows_cap, int Fo, int Fop, bool relu, void* out, bool out_bf16,
                  int64_t ldo, cudaStream_t s);
 void gather_ones(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const int32_t* xrow, const int64_t* cnt_rows,
@@ -52,7 +53,7 @@ bool gemm_row_tc(betty_ctx* c, const GemmRow& g, const void* Bk, int64_t ldbk, c
 
 // P[i, j] = sum_{r < *M_dev} A[r, i] B[r, j], i < K1, j < N, split over S row groups into
 // partials[S][K1][N]; then grad[map(i,j)] += sum_s partials[s][i][j] (fixed order: deterministic).
-enum { MAP_AGG = 0, MAP_PF = 1, MAP_POOL = 2 };
+enum { MAP_AGG = 0, MAP_PF = 1, MAP_POOL = 2, MAP_PF_N = 3, MAP_PF_S = 4 };
 struct GradMap {
     int mode;
     int Fi, Fo, Fp, Fop;
