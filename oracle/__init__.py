@@ -56,6 +56,8 @@ def lib():
         L.oracle_step.restype = ctypes.c_int
         L.oracle_step.argtypes = [ctypes.c_int, P, ctypes.c_int, ctypes.c_int, P, P, i64, i32, P, i32, P, P, i64,
                                   P, dbl, P, ctypes.POINTER(dbl)]
+        L.oracle_mem_estimate.restype = ctypes.c_int
+        L.oracle_mem_estimate.argtypes = [ctypes.c_int, P, ctypes.c_int, P, P, P, P]
         L.oracle_bf16_round.restype = dbl
         L.oracle_bf16_round.argtypes = [dbl]
         L.oracle_free.restype = None
@@ -186,3 +188,37 @@ def step(dims: Sequence[int], aggr: str, bf16: bool, full: Sequence, part: np.nd
     if rc != 0:
         raise ValueError("oracle_step: invalid input")
     return grad, loss.value
+
+
+def mem_estimate(dims: Sequence[int], aggr: str, blocks: Sequence) -> np.ndarray:
+    """Table 3 memory estimate of one (micro-)batch:
+    int64 [9] = element counts of terms (1)..(8) and the peak.  See
+    oracle_mem_estimate in oracle.c."""
+    L = len(blocks)
+    d = np.ascontiguousarray(dims, dtype=np.int32)
+    nd = np.array([b.n_dst for b in blocks], dtype=np.int64)
+    ns = np.array([b.n_src for b in blocks], dtype=np.int64)
+    ne = np.array([int(b.indptr[-1]) for b in blocks], dtype=np.int64)
+    t = np.zeros(9, dtype=np.int64)
+    lib().oracle_mem_estimate(L, _p(d), 1 if aggr == "pool" else 0, _p(nd), _p(ns), _p(ne), _p(t))
+    return t
+
+
+def memory_aware_k(full: Sequence, dims: Sequence[int], aggr: str, capacity_elems: int, partition_fn,
+                   K0: int = 1, K_max: Optional[int] = None):
+    """Memory-aware batch re-partitioning: partition the
+    REG K ways (partition_fn(K) -> part, supplied by the caller: the partition
+    is an input both sides share), estimate every micro-batch without running
+    it; if the largest estimate exceeds the capacity try K+1.  Returns
+    (K, part, peak) or (-1, None, smallest peak seen) when no K <= K_max
+    (default n_out) fits."""
+    n_out = full[-1].n_dst
+    K_max = n_out if K_max is None else K_max
+    best = None
+    for K in range(max(1, K0), K_max + 1):
+        part = np.asarray(partition_fn(K), dtype=np.int32)
+        peak = max(int(mem_estimate(dims, aggr, extract(full, part, K, k))[8]) for k in range(K))
+        best = peak if best is None else min(best, peak)
+        if peak <= capacity_elems:
+            return K, part, peak
+    return -1, None, best

@@ -531,3 +531,48 @@ int oracle_step(int L, const int32_t* dims, int aggr, int bf16, const oblock* fu
     free(mb);
     return 0;
 }
+
+/* ------------------------------------------------------------------------ */
+/* Memory estimate of one micro-batch, "Partition memory estimation"
+ * (§4.4, notation Table 3).
+ * Element counts, written in the paper's order:
+ *   t[0] (1) N_P_GNN              parameters without the aggregator's (W_self,
+ *                                 W_neigh, b of every layer; reading M3)
+ *   t[1] (2) N_in x H_in          input features: n_src of layer 0 x dims[0]
+ *   t[2] (3) N_out                output labels: n_dst of layer L-1
+ *   t[3] (4) sum over blocks E x 3 "two node IDs ... and a weight" per edge
+ *
+ *   t[4] (5) sum_i N_i x h_i      every layer's output, n_dst,l x dims[l+1]
+ *                                 (reading M1)
+ *   t[5] (6) aggregator intermediates: the paper gives only LSTM's (Eq. 5);
+ *                                 mean: sum_l n_dst,l x dims[l] (h_N); pool:
+ *                                 sum_l (n_src,l + n_dst,l) x dims[l]
+ *                                 (fc_pool output + max) (reading M2)
+ *   t[6] (7) N_P_GNN + N_P_Agg    gradients
+ *   t[7] (8) 2 (N_P_GNN + N_P_Agg) Adam's momentum and variance
+ *   t[8] peak = (1)+(2)+(3)+(4)+(5)+(8) + max((6), (7)): "(6) can be freed
+ *        during the backward propagation where ... (7) starts to dominate ...
+ *        the peak memory consumption comes from the maximum of (6) and (7)
+ *        plus other tensors".
+ * Sizes per layer l: n_dst[l], n_src[l], n_edges[l].  Bytes = 4 x elements
+ * (reading M4).  Returns 0. */
+int oracle_mem_estimate(int L, const int32_t* dims, int aggr, const int64_t* n_dst, const int64_t* n_src,
+                        const int64_t* n_edges, int64_t* t) {
+    int64_t np_gnn = 0, np_agg = 0;
+    for (int l = 0; l < L; ++l) {
+        int64_t fi = dims[l], fo = dims[l + 1];
+        np_gnn += 2 * fi * fo + fo;                /* W_self, W_neigh, b */
+        if (aggr == 1) np_agg += fi * fi + fi;     /* W_pool, b_pool */
+    }
+    for (int q = 0; q < 9; ++q) t[q] = 0;
+    t[0] = np_gnn;
+    t[1] = n_src[0] * dims[0];
+    t[2] = n_dst[L - 1];
+    for (int l = 0; l < L; ++l) t[3] += n_edges[l] * 3;
+    for (int l = 0; l < L; ++l) t[4] += n_dst[l] * dims[l + 1];
+    for (int l = 0; l < L; ++l) t[5] += (aggr == 1 ? n_src[l] + n_dst[l] : n_dst[l]) * dims[l];
+    t[6] = np_gnn + np_agg;
+    t[7] = 2 * (np_gnn + np_agg);
+    t[8] = t[0] + t[1] + t[2] + t[3] + t[4] + t[7] + (t[5] > t[6] ? t[5] : t[6]);
+    return 0;
+}
