@@ -234,6 +234,39 @@ BETTY_API betty_status betty_plan_probe_read(betty_plan* plan, float* total_ms, 
 BETTY_API betty_status betty_reg_partition(const int64_t* indptr, const int32_t* col, const int32_t* w, int64_t n,
                                            int32_t K, int32_t* part);
 
+/* §4.4 memory-aware batch-level partitioning (Table 3).
+ *
+ * betty_mb_sizes: count-only extraction (a2 without emitting the blocks) of
+ * every micro-batch k in [0,K) of the partition part[n_out] (device): writes
+ * sizes[(k*L + l)*3 + {0,1,2}] = n_dst, n_src, n_edges of layer l (HOST
+ * array, K*L*3 int64).  Synchronises once per micro-batch; EINVAL on bad
+ * arguments or part values out of range.
+ *
+ * betty_mem_estimate (HOST arithmetic, no GPU): the paper's estimate of one
+ * micro-batch from its per-layer sizes[L*3] (as above).  terms[9] receives
+ * element counts of (1) N_P_GNN, (2) N_in x H_in, (3) N_out, (4) 3 x sum E,
+ * (5) sum_l n_dst,l x dims[l+1], (6) aggregator intermediates (mean
+ * sum n_dst,l x dims[l]; pool sum (n_src,l + n_dst,l) x dims[l]), (7)
+ * gradients N_P_GNN + N_P_Agg, (8) Adam states 2 (N_P_GNN + N_P_Agg), and
+ * terms[8] = peak = (1)+(2)+(3)+(4)+(5)+(8) + max((6),(7)) (
+ * readings M1-M4 in DESIGN.md §3).  Bytes = 4 x elements.
+ *
+ * betty_memory_aware_k: for K = K0, K0+1, ... <= K_max (<= 0: n_out),
+ * partition the REG (HOST arrays, as betty_reg_partition) K ways, size every
+ * micro-batch on the GPU and estimate it; stop at the first K whose largest
+ * estimate (bytes) is <= capacity_bytes.  Writes
+ * part[n_out] (HOST) and *K_out = K, *peak_bytes = that K's largest
+ * estimate; when no K fits, *K_out = -1, part untouched and *peak_bytes =
+ * the smallest largest-estimate seen.  Synchronises. */
+BETTY_API betty_status betty_mb_sizes(betty_ctx* ctx, const betty_block* full, int32_t L, const int32_t* part,
+                                      int64_t n_out, int32_t K, int64_t* sizes, betty_stream stream);
+BETTY_API betty_status betty_mem_estimate(const betty_model* model, const int64_t* sizes, int64_t* terms);
+BETTY_API betty_status betty_memory_aware_k(betty_ctx* ctx, const betty_model* model, const betty_block* full,
+                                            int32_t L, const int64_t* reg_indptr, const int32_t* reg_col,
+                                            const int32_t* reg_w, int64_t n_out, int64_t capacity_bytes,
+                                            int32_t K0, int32_t K_max, int32_t* part, int32_t* K_out,
+                                            int64_t* peak_bytes, betty_stream stream);
+
 /* Synchronise `stream` and report device-side errors of earlier
  * asynchronous calls (part[] out of range -> EINVAL, capacity exceeded ->
  * EOVERFLOW, CUDA faults -> ECUDA). */

@@ -332,3 +332,48 @@ def betty_reg_partition(indptr, col, w, K: int):
     if st != 0:
         raise BettyError(f"betty_reg_partition: {L.STATUS.get(st, st)}")
     return part[:n]
+
+
+# ------------------------------------------------- §4.4 memory-aware micro-batch count
+def betty_mb_sizes(ctx: Context, full: Sequence[Block], part: torch.Tensor, K: int, stream=None):
+    """Count-only extraction: int64 numpy [K, L, 3] = (n_dst, n_src, n_edges)
+    of every layer of every micro-batch of the K-way partition (cuda int32)."""
+    import numpy as np
+    nL = len(full)
+    out = np.zeros((K, nL, 3), dtype=np.int64)
+    ctx.check(L.lib().betty_mb_sizes(ctx.h, _blocks_struct(full), nL, _p(part), full[-1].n_dst, K,
+                                     out.ctypes.data, _stream(stream)), "betty_mb_sizes")
+    return out
+
+
+def betty_mem_estimate(model: Model, sizes):
+    """Table 3 estimate of one micro-batch from its
+    [L, 3] sizes: int64 numpy [9] = element counts of terms (1)..(8), peak."""
+    import numpy as np
+    sz = np.ascontiguousarray(sizes, dtype=np.int64).reshape(-1)
+    t = np.zeros(9, dtype=np.int64)
+    m = model.struct()
+    st = L.lib().betty_mem_estimate(ctypes.byref(m), sz.ctypes.data, t.ctypes.data)
+    if st != 0:
+        raise BettyError(f"betty_mem_estimate: {L.STATUS.get(st, st)}")
+    return t
+
+
+def betty_memory_aware_k(ctx: Context, model: Model, full: Sequence[Block], reg, capacity_bytes: int, K0: int = 1,
+                         K_max: int = 0, stream=None):
+    """Memory-aware re-partitioning: the first K >= K0
+    whose largest micro-batch estimate fits capacity_bytes.  reg = host
+    (indptr, col, w) numpy arrays.  Returns (K, part int32 numpy, peak_bytes);
+    K = -1 (part None) when no K <= K_max fits."""
+    import numpy as np
+    ip, col, w = (np.ascontiguousarray(reg[0], dtype=np.int64), np.ascontiguousarray(reg[1], dtype=np.int32),
+                  np.ascontiguousarray(reg[2], dtype=np.int32))
+    n_out = full[-1].n_dst
+    part = np.zeros(max(1, n_out), dtype=np.int32)
+    k_out, peak = ctypes.c_int32(0), ctypes.c_int64(0)
+    m = model.struct()
+    ctx.check(L.lib().betty_memory_aware_k(ctx.h, ctypes.byref(m), _blocks_struct(full), len(full), ip.ctypes.data,
+                                           col.ctypes.data, w.ctypes.data, n_out, int(capacity_bytes), K0, K_max,
+                                           part.ctypes.data, ctypes.byref(k_out), ctypes.byref(peak),
+                                           _stream(stream)), "betty_memory_aware_k")
+    return k_out.value, (part[:n_out] if k_out.value > 0 else None), peak.value

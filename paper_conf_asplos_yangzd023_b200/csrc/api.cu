@@ -519,6 +519,39 @@ static void step_body(betty_ctx* c, betty_plan* p, const float* params, const vo
     if (p->with_reg) cudaStreamWaitEvent(s, p->ev_join, 0);   // join
 }
 
+// Count-only extraction of micro-batches ks[0..n) of a K-way partition, each alone with
+// full-batch capacities (one synchronisation per micro-batch): sz[i][3l + {0,1,2}] =
+// n_dst, n_src, n_edges of layer l.  Sizes plans and the memory estimate (§4.4).
+static betty_status size_micro_batches(betty_ctx* c, const ExtractFull* F, const betty_block* full, int L,
+                                       const int32_t* part, int64_t n_out, int32_t K, const int32_t* ks, int32_t n,
+                                       std::vector<std::vector<int64_t>>* sz, cudaStream_t s) {
+    sz->assign(n, std::vector<int64_t>(3 * L, 0));
+    std::vector<int64_t> fd(L), fs(L), fe(L);
+    for (int l = 0; l < L; ++l) { fd[l] = full[l].n_dst; fs[l] = full[l].n_src; fe[l] = full[l].n_edges; }
+    Arena A{c, s};
+    ExtractSet X;
+    int32_t* d_k = A.get<int32_t>(std::max(1, n));
+    if (!d_k || !alloc_extract(A, L, F, n_out, 1, fd, fs, fe, 0, &X)) {
+        A.release();
+        return fail(c, BETTY_ENOMEM, "sizing allocation failed");
+    }
+    if (n) cudaMemcpyAsync(d_k, ks, sizeof(int32_t) * n, cudaMemcpyHostToDevice, s);
+    std::vector<int64_t> h(4 * L);
+    betty_status st = BETTY_OK;
+    for (int i = 0; i < n && !st; ++i) {
+        ExtractArgs a{};
+        a.L = L; a.full = F; a.part = part; a.K = K; a.ks = d_k + i; a.c = 1;
+        a.layers = X.layers.data(); a.sc = X.sc; a.csc_mask = 0;
+        extract_group(c, a, s);
+        cudaMemcpyAsync(h.data(), X.cnt_all, sizeof(int64_t) * 4 * L, cudaMemcpyDeviceToHost, s);
+        if ((st = sync_check(c, s))) break;
+        for (int l = 0; l < L; ++l)
+            for (int q = 0; q < 3; ++q) (*sz)[i][3 * l + q] = h[4 * l + q];
+    }
+    A.release();
+    return st;
+}
+
 extern "C" betty_status betty_plan_create(betty_ctx* c, const betty_model* model, const betty_block* full, int32_t L,
                                           const int32_t* part, int64_t n_out, int32_t K, const int32_t* my_k,
                                           int32_t n_my, int32_t group, int32_t flags, betty_plan** out,
@@ -547,30 +580,10 @@ extern "C" betty_status betty_plan_create(betty_ctx* c, const betty_model* model
     for (int l = 0; l < L; ++l) if (m.needs_csc(l)) p->csc_mask |= 1u << l;
 
     // ---- sizing pass: every micro-batch alone, full-batch capacities
-    std::vector<int64_t> fd(L), fs(L), fe(L);
-    for (int l = 0; l < L; ++l) { fd[l] = full[l].n_dst; fs[l] = full[l].n_src; fe[l] = full[l].n_edges; }
-    std::vector<std::vector<int64_t>> sz(n_my, std::vector<int64_t>(3 * L));
-    {
-        Arena A{c, s};
-        ExtractSet X;
-        int32_t* d_k = A.get<int32_t>(std::max(1, n_my));
-        if (!d_k || !alloc_extract(A, L, p->full.data(), n_out, 1, fd, fs, fe, 0, &X)) {
-            A.release(); delete p;
-            return fail(c, BETTY_ENOMEM, "plan: sizing allocation failed");
-        }
-        if (n_my) cudaMemcpyAsync(d_k, my_k, sizeof(int32_t) * n_my, cudaMemcpyHostToDevice, s);
-        std::vector<int64_t> h(4 * L);
-        for (int i = 0; i < n_my; ++i) {
-            ExtractArgs a{};
-            a.L = L; a.full = p->full.data(); a.part = part; a.K = K; a.ks = d_k + i; a.c = 1;
-            a.layers = X.layers.data(); a.sc = X.sc; a.csc_mask = 0;
-            extract_group(c, a, s);
-            cudaMemcpyAsync(h.data(), X.cnt_all, sizeof(int64_t) * 4 * L, cudaMemcpyDeviceToHost, s);
-            if ((st = sync_check(c, s))) { A.release(); delete p; return st; }
-            for (int l = 0; l < L; ++l)
-                for (int q = 0; q < 3; ++q) sz[i][3 * l + q] = h[4 * l + q];
-        }
-        A.release();
+    std::vector<std::vector<int64_t>> sz;
+    if ((st = size_micro_batches(c, p->full.data(), full, L, part, n_out, K, my_k, n_my, &sz, s))) {
+        delete p;
+        return st;
     }
     std::vector<int64_t> cd(L, 1), cs(L, 1), ce(L, 1);
     p->info.L = L;
@@ -852,4 +865,95 @@ extern "C" betty_status betty_plan_probe_read(betty_plan* p, float* total_ms, in
 extern "C" betty_status betty_sync_check(betty_ctx* c, betty_stream stream) {
     if (!c) return BETTY_EINVAL;
     return sync_check(c, (cudaStream_t)stream);
+}
+
+// ------------------------------------------------------------------ §4.4 memory-aware K
+extern "C" betty_status betty_mb_sizes(betty_ctx* c, const betty_block* full, int32_t L, const int32_t* part,
+                                       int64_t n_out, int32_t K, int64_t* sizes, betty_stream stream) {
+    if (!c) return BETTY_EINVAL;
+    betty_status st = check_full(c, full, L);
+    if (st) return st;
+    if (K < 1 || !sizes || full[L - 1].n_dst != n_out || (n_out > 0 && !part))
+        return fail(c, BETTY_EINVAL, "mb_sizes: bad K / sizes / n_out / part");
+    std::vector<ExtractFull> F = to_full(full, L);
+    std::vector<int32_t> ks(K);
+    for (int k = 0; k < K; ++k) ks[k] = k;
+    std::vector<std::vector<int64_t>> sz;
+    if ((st = size_micro_batches(c, F.data(), full, L, part, n_out, K, ks.data(), K, &sz, (cudaStream_t)stream)))
+        return st;
+    for (int k = 0; k < K; ++k)
+        for (int q = 0; q < 3 * L; ++q) sizes[(int64_t)k * 3 * L + q] = sz[k][q];
+    return BETTY_OK;
+}
+
+extern "C" betty_status betty_mem_estimate(const betty_model* model, const int64_t* sizes, int64_t* terms) {
+    if (!model || !model->dims || model->L < 1 || !sizes || !terms) return BETTY_EINVAL;
+    const int L = model->L;
+    const int32_t* d = model->dims;
+    const bool pool = model->aggr == BETTY_AGGR_POOL;
+    int64_t p_gnn = 0, p_agg = 0;                       // N_P_GNN, N_P_Agg (Table 3)
+    int64_t blocks = 0, hidden = 0, inter = 0;
+    for (int l = 0; l < L; ++l) {
+        const int64_t nd = sizes[3 * l], ns = sizes[3 * l + 1], ne = sizes[3 * l + 2];
+        p_gnn += (int64_t)d[l] * d[l + 1] * 2 + d[l + 1];
+        if (pool) p_agg += (int64_t)d[l] * (d[l] + 1);
+        blocks += 3 * ne;                               // (4): src id, dst id, weight per edge
+        hidden += nd * d[l + 1];                        // (5): layer outputs
+        inter += (pool ? nd + ns : nd) * d[l];          // (6): h_N (mean) / fc_pool out + max (pool)
+    }
+    terms[0] = p_gnn;                                   // (1)
+    terms[1] = sizes[1] * d[0];                         // (2) N_in x H_in (layer-0 sources)
+    terms[2] = sizes[3 * (L - 1)];                      // (3) N_out
+    terms[3] = blocks;
+    terms[4] = hidden;
+    terms[5] = inter;
+    terms[6] = p_gnn + p_agg;                           // (7) gradients
+    terms[7] = 2 * (p_gnn + p_agg);                     // (8) Adam m, v
+    terms[8] = terms[0] + terms[1] + terms[2] + terms[3] + terms[4] + terms[7] + std::max(terms[5], terms[6]);
+    return BETTY_OK;
+}
+
+extern "C" betty_status betty_memory_aware_k(betty_ctx* c, const betty_model* model, const betty_block* full,
+                                             int32_t L, const int64_t* reg_indptr, const int32_t* reg_col,
+                                             const int32_t* reg_w, int64_t n_out, int64_t capacity_bytes,
+                                             int32_t K0, int32_t K_max, int32_t* part, int32_t* K_out,
+                                             int64_t* peak_bytes, betty_stream stream) {
+    if (!c) return BETTY_EINVAL;
+    if (!model || !part || !K_out || !peak_bytes || model->L != L || (n_out > 0 && !reg_indptr))
+        return fail(c, BETTY_EINVAL, "memory_aware_k: bad arguments");
+    betty_status st = check_full(c, full, L);
+    if (st) return st;
+    if (full[L - 1].n_dst != n_out) return fail(c, BETTY_EINVAL, "memory_aware_k: n_out != output block n_dst");
+    cudaStream_t s = (cudaStream_t)stream;
+    if (K_max <= 0 || K_max > n_out) K_max = (int32_t)std::max<int64_t>(1, n_out);
+    *K_out = -1;
+    *peak_bytes = -1;
+    Arena A{c, s};
+    int32_t* d_part = A.get<int32_t>(std::max<int64_t>(1, n_out));
+    if (!d_part) { A.release(); return fail(c, BETTY_ENOMEM, "memory_aware_k: allocation failed"); }
+    std::vector<ExtractFull> F = to_full(full, L);
+    std::vector<int32_t> hp(std::max<int64_t>(1, n_out));
+    std::vector<int64_t> terms(9);
+    for (int32_t K = std::max(1, K0); K <= K_max; ++K) {
+        if ((st = betty_reg_partition(reg_indptr, reg_col, reg_w, n_out, K, hp.data()))) break;
+        if (n_out) cudaMemcpyAsync(d_part, hp.data(), sizeof(int32_t) * n_out, cudaMemcpyHostToDevice, s);
+        std::vector<int32_t> ks(K);
+        for (int k = 0; k < K; ++k) ks[k] = k;
+        std::vector<std::vector<int64_t>> sz;
+        if ((st = size_micro_batches(c, F.data(), full, L, d_part, n_out, K, ks.data(), K, &sz, s))) break;
+        int64_t peak = 0;
+        for (int k = 0; k < K; ++k) {
+            betty_mem_estimate(model, sz[k].data(), terms.data());
+            peak = std::max(peak, terms[8] * 4);        // 4-byte elements (reading M4)
+        }
+        if (*peak_bytes < 0 || peak < *peak_bytes) *peak_bytes = peak;
+        if (peak <= capacity_bytes) {
+            *K_out = K;
+            *peak_bytes = peak;
+            std::copy(hp.begin(), hp.begin() + n_out, part);
+            break;
+        }
+    }
+    A.release();
+    return st;
 }
