@@ -252,7 +252,8 @@ BETTY_API betty_status betty_reg_partition(const int64_t* indptr, const int32_t*
  * readings M1-M4 in DESIGN.md §3).  Bytes = 4 x elements.
  *
  * betty_memory_aware_k: for K = K0, K0+1, ... <= K_max (<= 0: n_out),
- * partition the REG (HOST arrays, as betty_reg_partition) K ways, size every
+ * partition the REG (HOST arrays) K ways with betty_reg_partition_ex(method,
+ * imbalance 0.03), size every
  * micro-batch on the GPU and estimate it; stop at the first K whose largest
  * estimate (bytes) is <= capacity_bytes.  Writes
  * part[n_out] (HOST) and *K_out = K, *peak_bytes = that K's largest
@@ -264,8 +265,20 @@ BETTY_API betty_status betty_mem_estimate(const betty_model* model, const int64_
 BETTY_API betty_status betty_memory_aware_k(betty_ctx* ctx, const betty_model* model, const betty_block* full,
                                             int32_t L, const int64_t* reg_indptr, const int32_t* reg_col,
                                             const int32_t* reg_w, int64_t n_out, int64_t capacity_bytes,
-                                            int32_t K0, int32_t K_max, int32_t* part, int32_t* K_out,
-                                            int64_t* peak_bytes, betty_stream stream);
+                                            int32_t K0, int32_t K_max, int32_t method, int32_t* part,
+                                            int32_t* K_out, int64_t* peak_bytes, betty_stream stream);
+
+/* HOST function, outside the hot path: K-way REG partition by `method`:
+ * BETTY_PART_GREEDY = betty_reg_partition (exactly balanced sizes);
+ * BETTY_PART_MULTILEVEL = the METIS scheme the paper uses (Alg. 1 line 8,
+ * PAPER.md:917-941): heavy-edge-matching coarsening, greedy-growing initial
+ * partition, greedy boundary refinement while uncoarsening; minimises the
+ * cut REG weight (the inputs duplicated across micro-batches) subject to
+ * every part holding <= ceil((1 + imbalance) n / K) outputs.  Host arrays
+ * (as betty_reg_partition); deterministic; EINVAL on bad arguments. */
+enum { BETTY_PART_GREEDY = 0, BETTY_PART_MULTILEVEL = 1 };
+BETTY_API betty_status betty_reg_partition_ex(const int64_t* indptr, const int32_t* col, const int32_t* w, int64_t n,
+                                              int32_t K, int32_t method, double imbalance, int32_t* part);
 
 /* Synchronise `stream` and report device-side errors of earlier
  * asynchronous calls (part[] out of range -> EINVAL, capacity exceeded ->

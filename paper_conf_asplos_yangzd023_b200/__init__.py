@@ -319,9 +319,26 @@ def betty_sync_check(ctx: Context, stream=None):
     ctx.check(L.lib().betty_sync_check(ctx.h, _stream(stream)), "betty_sync_check")
 
 
-def betty_reg_partition(indptr, col, w, K: int):
-    """Host K-way partition of a REG (numpy int64/int32 arrays) -> int32 part[n]."""
+PART_METHODS = {"greedy": 0, "multilevel": 1}
+
+
+def betty_reg_partition(indptr, col, w, K: int, method: str = "greedy", imbalance: float = 0.03):
+    """Host K-way partition of a REG (numpy int64/int32 arrays) -> int32 part[n].
+    method 'greedy' (exactly balanced) or 'multilevel' (METIS scheme, parts <=
+    (1 + imbalance) n / K)."""
     import numpy as np
+    if method != "greedy":
+        indptr = np.ascontiguousarray(indptr, dtype=np.int64)
+        col = np.ascontiguousarray(col, dtype=np.int32)
+        w = None if w is None else np.ascontiguousarray(w, dtype=np.int32)
+        n = len(indptr) - 1
+        part = np.empty(max(n, 1), dtype=np.int32)
+        st = L.lib().betty_reg_partition_ex(indptr.ctypes.data, col.ctypes.data,
+                                            None if w is None else w.ctypes.data, n, K, PART_METHODS[method],
+                                            float(imbalance), part.ctypes.data)
+        if st != 0:
+            raise BettyError(f"betty_reg_partition_ex: {L.STATUS.get(st, st)}")
+        return part[:n]
     indptr = np.ascontiguousarray(indptr, dtype=np.int64)
     col = np.ascontiguousarray(col, dtype=np.int32)
     w = None if w is None else np.ascontiguousarray(w, dtype=np.int32)
@@ -360,7 +377,7 @@ def betty_mem_estimate(model: Model, sizes):
 
 
 def betty_memory_aware_k(ctx: Context, model: Model, full: Sequence[Block], reg, capacity_bytes: int, K0: int = 1,
-                         K_max: int = 0, stream=None):
+                         K_max: int = 0, method: str = "multilevel", stream=None):
     """Memory-aware re-partitioning: the first K >= K0
     whose largest micro-batch estimate fits capacity_bytes.  reg = host
     (indptr, col, w) numpy arrays.  Returns (K, part int32 numpy, peak_bytes);
@@ -374,6 +391,6 @@ def betty_memory_aware_k(ctx: Context, model: Model, full: Sequence[Block], reg,
     m = model.struct()
     ctx.check(L.lib().betty_memory_aware_k(ctx.h, ctypes.byref(m), _blocks_struct(full), len(full), ip.ctypes.data,
                                            col.ctypes.data, w.ctypes.data, n_out, int(capacity_bytes), K0, K_max,
-                                           part.ctypes.data, ctypes.byref(k_out), ctypes.byref(peak),
+                                           PART_METHODS[method], part.ctypes.data, ctypes.byref(k_out), ctypes.byref(peak),
                                            _stream(stream)), "betty_memory_aware_k")
     return k_out.value, (part[:n_out] if k_out.value > 0 else None), peak.value

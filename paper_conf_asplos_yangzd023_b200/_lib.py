@@ -74,10 +74,11 @@ def lib() -> ctypes.CDLL:
         "betty_plan_group_blocks": (i32, [vp, vp, i32, pp(betty_block), vp]),
         "betty_test_gemm": (i32, [vp, i32, vp, i64, vp, i64, i64, i64, i32, i32, vp, i64, i32, vp]),
         "betty_plan_probe_read": (i32, [vp, pp(f32), pp(i32)]),
+        "betty_reg_partition_ex": (i32, [vp, vp, vp, i64, i32, i32, ctypes.c_double, vp]),
         "betty_mb_sizes": (i32, [vp, pp(betty_block), i32, vp, i64, i32, vp, vp]),
         "betty_mem_estimate": (i32, [pp(betty_model), vp, vp]),
         "betty_memory_aware_k": (i32, [vp, pp(betty_model), pp(betty_block), i32, vp, vp, vp, i64, i64, i32, i32,
-                                       vp, pp(i32), pp(i64), vp]),
+                                       i32, vp, pp(i32), pp(i64), vp]),
     }
     for name, (res, args) in sigs.items():
         fn = getattr(L, name)
@@ -92,4 +93,4 @@ EXPORTED = ["betty_version", "betty_ctx_create", "betty_ctx_destroy", "betty_las
             "betty_sage_bwd", "betty_saved_free", "betty_plan_create", "betty_plan_info_get", "betty_plan_destroy",
             "betty_step", "betty_adam", "betty_sync_check", "betty_reg_partition", "betty_plan_probe",
             "betty_plan_probe_read", "betty_plan_group_blocks", "betty_test_gemm", "betty_mb_sizes",
-            "betty_mem_estimate", "betty_memory_aware_k"]
+            "betty_mem_estimate", "betty_memory_aware_k", "betty_reg_partition_ex"]

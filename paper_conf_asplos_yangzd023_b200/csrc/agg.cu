@@ -271,6 +271,287 @@ __global__ void __launch_bounds__(256) k_agg_mean_xa(const Tin* __restrict__ X, 
     }
 }
 
+// ------------------------------------------------ mean, aggregate-first fwd: TMA gather4 pipeline
+// Warp-specialised persistent kernel, one CTA per SM: G4_PROD producer warps, each owning every
+// G4_PROD-th stage of a G4_STAGES ring, and G4_CONS consumer warps.
+//  * A producer claims G4_CLAIM virtual rows at a time (dynamic, micro-batch-major order) ONE
+//    CLAIM AHEAD: the claim's real row ids, indptr pairs and self-row ids are copied into a
+//    per-warp shared buffer with cp.async while the previous claim is being issued, so no
+//    global latency sits between a stage's rows and its gathers except the edge ids.
+//  * A stage is a run of <= G4_MAXR consecutive real rows (one order segment, so their edges are
+//    one contiguous CSR range) whose neighbour rows fit the stage's slots.  Slot s holds the
+//    source row of edge E0a + s (E0a = first edge rounded down to 4): every row's neighbours are
+//    consecutive slots, and 4 consecutive edges are one tile::gather4 TMA copy (four arbitrary
+//    rows per instruction, completion on the stage's mbarrier; row -1 reads as zeros).  Self
+//    rows are gathered the same way.
+//  * Consumers map (row, 16-byte vector) pairs onto threads, sum the row's slots from shared
+//    memory and stream XA out.  A row whose neighbours exceed the slots ("long" row, e.g.
+//    full-neighbourhood layers) is a stage of its own that the consumers reduce straight from
+//    global memory.
+constexpr int G4_STAGES = 8, G4_PROD = 4, G4_THREADS = 256, G4_MAXR = 16, G4_CLAIM = 64;
+constexpr int G4_CONS = G4_THREADS / 32 - G4_PROD;
+struct G4Hdr {
+    int64_t r0;                  // first real row
+    int64_t hb, he;              // long row: its edge range
+    int32_t n;                   // rows (-1: end of work)
+    int32_t lng;                 // 1: long row
+    int32_t off[G4_MAXR + 1];    // slot offset of each row's first edge (relative to E0a)
+};
+struct G4Claim {                 // one claim's rows (virtual offset j)
+    int64_t r[G4_CLAIM];         // real row
+    int64_t lo[G4_CLAIM], hi[G4_CLAIM];   // indptr[r], indptr[r + 1]
+    int32_t sid[G4_CLAIM];       // self row (srow[r] or r)
+};
+struct G4Args {
+    const int32_t* srow; const int32_t* erow; const int32_t* emap;
+    const int64_t* indptr; const int64_t* cnt; const int64_t* otab;
+    void* XA; int64_t ldxa; const void* X; int64_t ldx;
+    unsigned* ctr;
+    int Fi, Fp, NV;
+    uint32_t row_bytes, grp_bytes, slot_groups, stage_bytes;
+    int hint;
+};
+__device__ __forceinline__ void gather4(uint32_t sdst, const CUtensorMap* tm, int32_t r0, int32_t r1, int32_t r2,
+                                        int32_t r3, uint64_t* bar, uint64_t pol) {
+    asm volatile("cp.async.bulk.tensor.2d.shared::cluster.global.tile::gather4.mbarrier::complete_tx::bytes.L2::cache_hint"
+                 " [%0], [%1, {%2, %3, %4, %5, %6}], [%7], %8;"
+                 ::"r"(sdst), "l"((uint64_t)tm), "r"(0), "r"(r0), "r"(r1), "r"(r2), "r"(r3), "r"(smem_u32(bar)),
+                   "l"(pol) : "memory");
+}
+__device__ __forceinline__ void mbar_init(uint64_t* b, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(b)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* b) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(b)) : "memory");
+}
+__device__ __forceinline__ void cp_async8(void* sdst, const void* gsrc) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(sdst)), "l"(gsrc) : "memory");
+}
+__device__ __forceinline__ void cp_async4(void* sdst, const void* gsrc) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(sdst)), "l"(gsrc) : "memory");
+}
+// the row tail of XA: pad columns of both halves and [1, 0, ...] from column 2 Fp
+template <typename Tout> __device__ __forceinline__ void xa_tail(Tout* out, int c0, int Fp, int64_t ldxa) {
+    for (int col = c0; col < Fp; ++col) { st_act(out + col, 0.f); st_act(out + Fp + col, 0.f); }
+    Tout* t = out + 2 * Fp;
+    const int w = (int)(ldxa - 2 * Fp);
+    if (w * (int)sizeof(Tout) == 16 && ((uintptr_t)t & 15) == 0) {
+        const uint32_t one = sizeof(Tout) == 2 ? 0x3F80u : 0x3F800000u;
+        __stcs((uint4*)t, make_uint4(one, 0u, 0u, 0u));
+    } else {
+        for (int col = 0; col < w; ++col) st_act(t + col, col == 0 ? 1.f : 0.f);
+    }
+}
+
+template <typename Tin, typename Tout>
+__global__ void __launch_bounds__(G4_THREADS, 1) k_agg_mean_g4(const __grid_constant__ CUtensorMap tmX, G4Args a) {
+    using VI = Vec<Tin>;
+    constexpr int VW = VI::N;
+    extern __shared__ __align__(128) uint8_t g4_smem[];
+    __shared__ G4Hdr hdr[G4_STAGES];
+    __shared__ G4Claim clm[G4_PROD][2];
+    __shared__ uint64_t full[G4_STAGES], empty[G4_STAGES];
+    __shared__ int64_t s_vs[ORDER_SMEM + 1], s_rs[ORDER_SMEM];
+    const int64_t nd = a.cnt[0];
+    const int nseg = order_load(a.otab, s_vs, s_rs);
+    const int warp = threadIdx.x >> 5, lane = lane_id();
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < G4_STAGES; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], G4_CONS); }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    const uint32_t sbase = smem_u32(g4_smem);
+    const uint32_t self_off = a.slot_groups * a.grp_bytes;          // self rows after the edge slots
+    if (warp < G4_PROD) {
+        // ---------------------------------------------------------------- producer
+        uint64_t pol;
+        if (a.hint) pol = l2_evict_last_policy();
+        else asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(pol));
+        int seg = 0;
+        // claim G4_CLAIM virtual rows into buffer C (async); returns the claim's first virtual row
+        auto claim = [&](G4Claim& C, int64_t& vend) -> int64_t {
+            int64_t v = 0;
+            if (lane == 0) v = (int64_t)atomicAdd(a.ctr, 1u) * G4_CLAIM;
+            v = __shfl_sync(0xffffffffu, v, 0);
+            vend = v < nd ? mn64(v + G4_CLAIM, nd) : v;
+            for (int j = lane; j < G4_CLAIM; j += 32) {
+                if (v + j >= vend) break;
+                const int64_t r = nseg > 0 ? order_map(v + j, nseg, s_vs, s_rs, seg) : v + j;
+                C.r[j] = r;
+                cp_async8(&C.lo[j], a.indptr + r);
+                cp_async8(&C.hi[j], a.indptr + r + 1);
+                if (a.srow) cp_async4(&C.sid[j], a.srow + r); else C.sid[j] = (int32_t)r;
+            }
+            asm volatile("cp.async.commit_group;" ::: "memory");
+            return v;
+        };
+        int cb = 0;                                     // buffer of the current claim
+        int64_t ce, ne;
+        int64_t cv = claim(clm[warp][0], ce);
+        int64_t nv = claim(clm[warp][1], ne);
+        asm volatile("cp.async.wait_group 1;" ::: "memory");
+        __syncwarp();
+        int j0 = 0;                                     // next virtual row of the current claim
+        const int64_t cap = (int64_t)a.slot_groups * 4;
+        for (uint32_t i = 0;; ++i) {
+            const int s = (warp + G4_PROD * i) % G4_STAGES;
+            const uint32_t visit = i / (G4_STAGES / G4_PROD);
+            G4Hdr& H = hdr[s];
+            uint64_t* fb = &full[s];
+            if (cv + j0 >= ce) {                        // current claim used up: rotate
+                cv = nv; ce = ne; cb ^= 1; j0 = 0;
+                if (cv < nd) nv = claim(clm[warp][cb ^ 1], ne);
+                else asm volatile("cp.async.commit_group;" ::: "memory");
+                asm volatile("cp.async.wait_group 1;" ::: "memory");
+                __syncwarp();
+            }
+            mbar_wait_parity(&empty[s], (visit & 1u) ^ 1u);
+            if (cv >= nd) {                            // no more work: tell the consumers
+                if (lane == 0) { H.n = -1; mbar_arrive(fb); }
+                break;
+            }
+            const G4Claim& C = clm[warp][cb];
+            const int rem = (int)mn64(G4_MAXR, ce - cv - j0);
+            const int jj = j0 + lane;
+            const bool valid = lane < rem;
+            const int64_t r = valid ? C.r[jj] : 0, lo = valid ? C.lo[jj] : 0, hi = valid ? C.hi[jj] : 0;
+            const int32_t sidv = valid ? C.sid[jj] : -1;
+            const int64_t r0 = __shfl_sync(0xffffffffu, r, 0);
+            const int64_t E0 = __shfl_sync(0xffffffffu, lo, 0);
+            const int64_t E0a = E0 & ~(int64_t)3;
+            const bool fits = valid && r == r0 + lane && hi - E0a <= cap;
+            int n = __ffs(~__ballot_sync(0xffffffffu, fits)) - 1;
+            const int lng = n == 0;
+            if (lng) n = 1;
+            const int64_t Eend = __shfl_sync(0xffffffffu, hi, n - 1);
+            if (lane == 0) { H.r0 = r0; H.n = n; H.lng = lng; H.hb = E0; H.he = Eend; }
+            if (lane < n) H.off[lane] = (int32_t)(lo - E0a);
+            if (lane == n - 1) H.off[n] = (int32_t)(hi - E0a);
+            const int groups = lng ? 0 : (int)((Eend - E0a + 3) >> 2);
+            const int sgroups = (n + 3) >> 2;
+            // edge ids of this lane's groups (independent loads, all in flight together)
+            int32_t id[2][4];
+#pragma unroll
+            for (int gg = 0; gg < 2; ++gg)
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    const int64_t e = E0a + 4 * (lane + 32 * gg) + q;
+                    id[gg][q] = (lane + 32 * gg < groups && e >= E0 && e < Eend) ? __ldg(a.erow + e) : -1;
+                }
+            if (a.emap) {
+#pragma unroll
+                for (int gg = 0; gg < 2; ++gg)
+#pragma unroll
+                    for (int q = 0; q < 4; ++q) if (id[gg][q] >= 0) id[gg][q] = __ldg(a.emap + id[gg][q]);
+            }
+            __syncwarp();
+            if (lane == 0) mbar_expect(fb, (uint32_t)(groups + sgroups) * 4u * a.row_bytes);
+            const uint32_t sdat = sbase + (uint32_t)s * a.stage_bytes;
+#pragma unroll
+            for (int gg = 0; gg < 2; ++gg) {
+                const int g = lane + 32 * gg;
+                if (g < groups)
+                    gather4(sdat + (uint32_t)g * a.grp_bytes, &tmX, id[gg][0], id[gg][1], id[gg][2], id[gg][3], fb, pol);
+            }
+            int32_t sv[4];
+#pragma unroll
+            for (int q = 0; q < 4; ++q) sv[q] = __shfl_sync(0xffffffffu, sidv, (4 * lane + q) & 31);
+#pragma unroll
+            for (int q = 0; q < 4; ++q) if (4 * lane + q >= n) sv[q] = -1;
+            if (lane < sgroups)
+                gather4(sdat + self_off + (uint32_t)lane * a.grp_bytes, &tmX, sv[0], sv[1], sv[2], sv[3], fb, pol);
+            j0 += n;
+        }
+        asm volatile("cp.async.wait_all;" ::: "memory");
+    } else {
+        // ---------------------------------------------------------------- consumers
+        const int ct = threadIdx.x - G4_PROD * 32;
+        const int NC = G4_CONS * 32;
+        const int NV = a.NV;
+        float* red = (float*)(g4_smem + (size_t)G4_STAGES * a.stage_bytes);   // [G4_CONS][NV*VW] long-row partials
+        unsigned done = 0;                      // producers that ran out of work
+        for (uint32_t it = 0; done != (1u << G4_PROD) - 1u; ++it) {
+            const int s = it % G4_STAGES;
+            if (done >> (s % G4_PROD) & 1u) continue;
+            mbar_wait_parity(&full[s], (it / G4_STAGES) & 1u);
+            const G4Hdr& H = hdr[s];
+            const int n = H.n;
+            if (n < 0) { done |= 1u << (s % G4_PROD); continue; }
+            const uint8_t* sdat = g4_smem + (size_t)s * a.stage_bytes;
+            if (!H.lng) {
+                for (int u = ct; u < n * NV; u += NC) {
+                    const int i = u / NV, j = u - i * NV;
+                    const int b = H.off[i], e = H.off[i + 1];
+                    float acc[VW];
+#pragma unroll
+                    for (int t = 0; t < VW; ++t) acc[t] = 0.f;
+                    const uint8_t* p = sdat + (b >> 2) * a.grp_bytes + (b & 3) * a.row_bytes + j * 16;
+                    for (int sl = b; sl < e; ++sl) {
+                        VI::add_raw(acc, *(const typename VI::Raw*)p);
+                        p += ((sl & 3) == 3) ? a.grp_bytes - 3 * a.row_bytes : a.row_bytes;
+                    }
+                    float so[VW];
+#pragma unroll
+                    for (int t = 0; t < VW; ++t) so[t] = 0.f;
+                    VI::add_raw(so, *(const typename VI::Raw*)(sdat + self_off + (i >> 2) * a.grp_bytes +
+                                                               (i & 3) * a.row_bytes + j * 16));
+                    const float inv = e > b ? 1.0f / (float)(e - b) : 0.0f;
+#pragma unroll
+                    for (int t = 0; t < VW; ++t) {
+                        const bool in = j * VW + t < a.Fi;
+                        acc[t] = in ? acc[t] * inv : 0.f;
+                        so[t] = in ? so[t] : 0.f;
+                    }
+                    Tout* out = (Tout*)a.XA + (H.r0 + i) * a.ldxa;
+                    st_vec_cs<Tout, VW>(out + j * VW, so);
+                    st_vec_cs<Tout, VW>(out + a.Fp + j * VW, acc);
+                }
+                if (ct < n) xa_tail<Tout>((Tout*)a.XA + (H.r0 + ct) * a.ldxa, NV * VW, a.Fp, a.ldxa);
+            } else {
+                // long row: consumer warp w sums edges w, w + G4_CONS, ...; lanes over vectors
+                const int w = ct >> 5;
+                const int64_t hb = H.hb, he = H.he;
+                for (int j = lane; j < NV; j += 32) {
+                    float acc[VW];
+#pragma unroll
+                    for (int t = 0; t < VW; ++t) acc[t] = 0.f;
+                    for (int64_t e = hb + w; e < he; e += G4_CONS) {
+                        int32_t u = __ldg(a.erow + e);
+                        if (a.emap) u = __ldg(a.emap + u);
+                        VI::add_raw(acc, VI::ld_raw((const Tin*)a.X + (int64_t)u * a.ldx + j * VW));
+                    }
+#pragma unroll
+                    for (int t = 0; t < VW; ++t) red[(w * NV + j) * VW + t] = acc[t];
+                }
+                asm volatile("bar.sync 1, %0;" ::"r"(NC) : "memory");
+                for (int j = ct; j < NV; j += NC) {
+                    float acc[VW], so[VW];
+#pragma unroll
+                    for (int t = 0; t < VW; ++t) { acc[t] = 0.f; so[t] = 0.f; }
+                    for (int q = 0; q < G4_CONS; ++q)
+#pragma unroll
+                        for (int t = 0; t < VW; ++t) acc[t] += red[(q * NV + j) * VW + t];
+                    VI::add_raw(so, *(const typename VI::Raw*)(sdat + self_off + j * 16));
+                    const float inv = he > hb ? 1.0f / (float)(he - hb) : 0.0f;
+#pragma unroll
+                    for (int t = 0; t < VW; ++t) {
+                        const bool in = j * VW + t < a.Fi;
+                        acc[t] = in ? acc[t] * inv : 0.f;
+                        so[t] = in ? so[t] : 0.f;
+                    }
+                    Tout* out = (Tout*)a.XA + H.r0 * a.ldxa;
+                    st_vec_cs<Tout, VW>(out + j * VW, so);
+                    st_vec_cs<Tout, VW>(out + a.Fp + j * VW, acc);
+                }
+                if (ct == 0) xa_tail<Tout>((Tout*)a.XA + H.r0 * a.ldxa, NV * VW, a.Fp, a.ldxa);
+                asm volatile("bar.sync 1, %0;" ::"r"(NC) : "memory");
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&empty[s]);
+        }
+    }
+}
+
 // ------------------------------------------------ mean, project-first fwd
 // S[v,c] = Y[v, Fop + c] + (1/D_v) sum_u Y[u, c];  out = logits (fp32) or ReLU -> H (+ones col)
 template <typename Tout>
@@ -638,6 +919,38 @@ template <typename K> static int resident_grid(betty_ctx* c, K kernel, int threa
     return (int)std::max<int64_t>(1, std::min<int64_t>(want_ctas, (int64_t)per_sm * c->num_sms));
 }
 
+// the gather4 pipeline (k_agg_mean_g4); false if the table cannot be described by a tensor map
+static bool agg_mean_g4(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const int32_t* srow,
+                        const int32_t* erow, const int32_t* emap, const int64_t* indptr, const int64_t* cnt,
+                        const int64_t* otab, int Fi, int Fp, int nv, void* XA, bool xa_bf16, int64_t ldxa, int hint,
+                        unsigned* ctr, cudaStream_t s) {
+    const int vw = x_bf16 ? 8 : 4;
+    CUtensorMap tm;
+    if (!make_gather_map(&tm, X, !x_bf16, (int64_t)nv * vw, (int64_t)INT32_MAX, ldx, nv * vw)) return false;
+    G4Args a{};
+    a.srow = srow; a.erow = erow; a.emap = emap; a.indptr = indptr; a.cnt = cnt; a.otab = otab;
+    a.XA = XA; a.ldxa = ldxa; a.X = X; a.ldx = ldx; a.ctr = ctr; a.Fi = Fi; a.Fp = Fp; a.NV = nv; a.hint = hint;
+    a.row_bytes = (uint32_t)nv * 16u;
+    a.grp_bytes = (4u * a.row_bytes + 127u) / 128u * 128u;
+    const size_t red_bytes = (size_t)G4_CONS * nv * vw * 4;
+    const size_t budget = (size_t)196 * 1024 - red_bytes;            // dynamic smem for the stage ring
+    const int64_t groups = (int64_t)(budget / G4_STAGES) / a.grp_bytes - G4_MAXR / 4;
+    if (groups < 4) return false;
+    a.slot_groups = (uint32_t)std::min<int64_t>(groups, 64);     // a producer lane issues <= 2 groups
+    a.stage_bytes = (a.slot_groups + G4_MAXR / 4) * a.grp_bytes;
+    const size_t sm = (size_t)G4_STAGES * a.stage_bytes + red_bytes;
+    DISPATCH_ACT(x_bf16, TI, DISPATCH_ACT(xa_bf16, TO, {
+        static bool attr = false;
+        if (!attr) {
+            cudaFuncSetAttribute(k_agg_mean_g4<TI, TO>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+            attr = true;
+        }
+        cudaMemsetAsync(ctr, 0, sizeof(unsigned), s);
+        k_agg_mean_g4<TI, TO><<<c->num_sms, G4_THREADS, sm, s>>>(tm, a);
+    }))
+    return true;
+}
+
 void agg_mean_xa(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const int32_t* srow, const int32_t* erow,
                  const int32_t* emap, const int64_t* indptr, const int64_t* cnt, const int64_t* otab, int64_t rows_cap,
                  int64_t src_per_mb, int Fi, int Fp, void* XA, bool xa_bf16, int64_t ldxa, cudaStream_t s) {
@@ -655,6 +968,10 @@ void agg_mean_xa(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const in
     int passes = (int)std::max(1.0, std::min((double)nv, std::ceil(ws / budget)));
     const int pv = (nv + passes - 1) / passes;
     passes = (nv + pv - 1) / pv;
+    static const bool g4_off = getenv("BETTY_AGG_G4") && atoi(getenv("BETTY_AGG_G4")) == 0;
+    if (!g4_off && passes == 1 && nv * vw <= 256 && agg_mean_g4(c, X, x_bf16, ldx, srow, erow, emap, indptr, cnt, otab,
+                                                                Fi, Fp, nv, XA, xa_bf16, ldxa, hint, ctr, s))
+        return;
     const int lpr = pv <= 8 ? 8 : (pv <= 16 ? 16 : 32);
     const int64_t warps = (rows_cap + (32 / lpr) - 1) / (32 / lpr);
 #define AGG_L(LPR) DISPATCH_ACT(x_bf16, TI, DISPATCH_ACT(xa_bf16, TO, {                                           \

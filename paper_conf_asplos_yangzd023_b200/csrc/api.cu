@@ -916,8 +916,8 @@ extern "C" betty_status betty_mem_estimate(const betty_model* model, const int64
 extern "C" betty_status betty_memory_aware_k(betty_ctx* c, const betty_model* model, const betty_block* full,
                                              int32_t L, const int64_t* reg_indptr, const int32_t* reg_col,
                                              const int32_t* reg_w, int64_t n_out, int64_t capacity_bytes,
-                                             int32_t K0, int32_t K_max, int32_t* part, int32_t* K_out,
-                                             int64_t* peak_bytes, betty_stream stream) {
+                                             int32_t K0, int32_t K_max, int32_t method, int32_t* part,
+                                             int32_t* K_out, int64_t* peak_bytes, betty_stream stream) {
     if (!c) return BETTY_EINVAL;
     if (!model || !part || !K_out || !peak_bytes || model->L != L || (n_out > 0 && !reg_indptr))
         return fail(c, BETTY_EINVAL, "memory_aware_k: bad arguments");
@@ -935,7 +935,7 @@ extern "C" betty_status betty_memory_aware_k(betty_ctx* c, const betty_model* mo
     std::vector<int32_t> hp(std::max<int64_t>(1, n_out));
     std::vector<int64_t> terms(9);
     for (int32_t K = std::max(1, K0); K <= K_max; ++K) {
-        if ((st = betty_reg_partition(reg_indptr, reg_col, reg_w, n_out, K, hp.data()))) break;
+        if ((st = betty_reg_partition_ex(reg_indptr, reg_col, reg_w, n_out, K, method, 0.03, hp.data()))) break;
         if (n_out) cudaMemcpyAsync(d_part, hp.data(), sizeof(int32_t) * n_out, cudaMemcpyHostToDevice, s);
         std::vector<int32_t> ks(K);
         for (int k = 0; k < K; ++k) ks[k] = k;

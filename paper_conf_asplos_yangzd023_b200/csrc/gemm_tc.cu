@@ -129,6 +129,7 @@ struct RowArgs {
     int acc_stride;          // TMEM columns between the two accumulators (>= BN, multiple of 32)
     int half_cols;           // columns per epilogue half (multiple of 32, <= 32 * MAXCH)
     uint32_t slot_bytes;     // one staging slot: 32 rows x 32 columns
+    int bstream;             // 1: B is streamed with A through the ring (B too large to stay resident)
 };
 
 __device__ __forceinline__ uint32_t pack_bf16x2(float a, float b) {
@@ -269,10 +270,11 @@ __global__ void __launch_bounds__(ROW_THREADS, 1) k_tc_row(const __grid_constant
     uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
     const int S = p.stages;
     const uint32_t a_bytes = BM * BK * 2;
-    const uint32_t bblk = (uint32_t)p.BN * BK * 2;          // one K-block of the resident B
-    uint8_t* bres = smem;                                    // nk * bblk
-    uint8_t* aring = smem + p.nk * bblk;                     // S * a_bytes
-    uint8_t* stage = aring + S * a_bytes;                    // EPI_WARPS * ESLOTS * slot_bytes
+    const uint32_t bblk = (uint32_t)p.BN * BK * 2;          // one K-block of B
+    const uint32_t ring_bytes = a_bytes + (p.bstream ? bblk : 0u);   // one ring stage: A (+ B when streamed)
+    uint8_t* bres = smem;                                    // nk * bblk (resident B) or nothing
+    uint8_t* aring = smem + (p.bstream ? 0 : p.nk * bblk);   // S * ring_bytes
+    uint8_t* stage = aring + S * ring_bytes;                 // EPI_WARPS * ESLOTS * slot_bytes
     uint64_t* full = (uint64_t*)(stage + EPI_WARPS * ESLOTS * p.slot_bytes);
     uint64_t* empty = full + S;
     uint64_t* tfull = empty + S;      // [2]
@@ -301,15 +303,18 @@ __global__ void __launch_bounds__(ROW_THREADS, 1) k_tc_row(const __grid_constant
 
     if (warp == 0) {
         if (elect_lane0() && blockIdx.x < tiles) {
-            mbar_expect_tx(bfull, p.nk * bblk);
-            for (int kb = 0; kb < p.nk; ++kb) tma_2d(bres + kb * bblk, &tmB, kb * BK, 0, bfull);
+            if (!p.bstream) {
+                mbar_expect_tx(bfull, p.nk * bblk);
+                for (int kb = 0; kb < p.nk; ++kb) tma_2d(bres + kb * bblk, &tmB, kb * BK, 0, bfull);
+            }
             int s = 0;
             uint32_t ph = 0;
             for (int64_t t = blockIdx.x; t < tiles; t += gridDim.x) {
                 for (int kb = 0; kb < p.nk; ++kb) {
                     mbar_wait(&empty[s], ph ^ 1);
-                    mbar_expect_tx(&full[s], a_bytes);
-                    tma_2d(aring + s * a_bytes, &tmA, kb * BK, (int)(t * BM), &full[s]);
+                    mbar_expect_tx(&full[s], ring_bytes);
+                    tma_2d(aring + s * ring_bytes, &tmA, kb * BK, (int)(t * BM), &full[s]);
+                    if (p.bstream) tma_2d(aring + s * ring_bytes + a_bytes, &tmB, kb * BK, 0, &full[s]);
                     if (++s == S) { s = 0; ph ^= 1; }
                 }
             }
@@ -319,7 +324,7 @@ __global__ void __launch_bounds__(ROW_THREADS, 1) k_tc_row(const __grid_constant
         int s = 0;
         uint32_t ph = 0;
         int it = 0;
-        if (blockIdx.x < tiles) mbar_wait(bfull, 0);
+        if (blockIdx.x < tiles && !p.bstream) mbar_wait(bfull, 0);
         for (int64_t t = blockIdx.x; t < tiles; t += gridDim.x, ++it) {
             const int acc = it & 1;
             const uint32_t aph = (it >> 1) & 1;
@@ -330,7 +335,8 @@ __global__ void __launch_bounds__(ROW_THREADS, 1) k_tc_row(const __grid_constant
                 mbar_wait(&full[s], ph);
                 fence_after();
                 if (elect_lane0()) {
-                    const uint32_t a0 = su32(aring + s * a_bytes), b0 = su32(bres + kb * bblk);
+                    const uint32_t a0 = su32(aring + s * ring_bytes);
+                    const uint32_t b0 = p.bstream ? a0 + a_bytes : su32(bres + kb * bblk);
 #pragma unroll
                     for (int k = 0; k < BK / UK; ++k) {
                         const uint64_t ad = sdesc(a0 + k * UK * 2, 0, 1024);
@@ -590,7 +596,8 @@ static EncodeFn encode_fn() {
 
 // 2-D tensor [rows x cols] with row stride ld (elements); box {box_cols, box_rows}
 static bool make_map_t(CUtensorMap* m, const void* base, bool f32, int64_t cols, int64_t rows, int64_t ld,
-                       int box_cols, int box_rows, CUtensorMapSwizzle sw) {
+                       int box_cols, int box_rows, CUtensorMapSwizzle sw,
+                       CUtensorMapL2promotion promo = CU_TENSOR_MAP_L2_PROMOTION_L2_256B) {
     EncodeFn f = encode_fn();
     if (!f) return false;
     const int es = f32 ? 4 : 2;
@@ -600,7 +607,7 @@ static bool make_map_t(CUtensorMap* m, const void* base, bool f32, int64_t cols,
     cuuint32_t box[2] = {(cuuint32_t)box_cols, (cuuint32_t)box_rows};
     cuuint32_t estr[2] = {1, 1};
     return f(m, f32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base),
-             dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, sw, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+             dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, sw, promo,
              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 // bf16 operand maps: box {64 cols (128 B), box_rows}, 128-byte swizzle
@@ -618,6 +625,15 @@ static uint32_t tmem_cols_for(int n) {
 
 bool tc_available() { return tc::encode_fn() != nullptr; }
 
+// Row-gather map for tile::gather4 (agg.cu): a [rows x cols] table with row stride ld, box
+// {box_cols, 1}; columns >= cols and out-of-range rows (e.g. -1) read as zeros.
+bool make_gather_map(CUtensorMap* m, const void* base, bool f32, int64_t cols, int64_t rows, int64_t ld,
+                     int box_cols) {
+    // no L2 promotion: a gathered row is fetched at sector granularity, not as 256-byte blocks
+    return tc::make_map_t(m, base, f32, cols, rows, ld, box_cols, 1, CU_TENSOR_MAP_SWIZZLE_NONE,
+                          CU_TENSOR_MAP_L2_PROMOTION_NONE);
+}
+
 // C = A B on the tensor cores; B given K-major as Bk[N x K] (ld ldbk).  Returns false if the shape is unsupported.
 bool gemm_row_tc(betty_ctx* c, const GemmRow& g, const void* Bk, int64_t ldbk, cudaStream_t s) {
     using namespace tc;
@@ -630,7 +646,12 @@ bool gemm_row_tc(betty_ctx* c, const GemmRow& g, const void* Bk, int64_t ldbk, c
     const uint32_t slot_bytes = 32 * 32 * (g.c_bf16 ? 2 : 4);
     const size_t stage_bytes = (size_t)EPI_WARPS * ESLOTS * slot_bytes;
     const size_t budget = 225 * 1024;
-    if (b_bytes + stage_bytes + 2 * a_bytes + 1024 + 256 > budget) return false;   // B must fit resident
+    const size_t bblk = (size_t)BN * BK * 2;
+    // B resident when it fits next to a 2-stage A ring, else streamed with A
+    const bool bstream = b_bytes + stage_bytes + 2 * a_bytes + 1024 + 256 > budget;
+    const size_t ring = a_bytes + (bstream ? bblk : 0);
+    const size_t fixed = (bstream ? 0 : b_bytes) + stage_bytes + 1024 + 256;
+    if (fixed + 2 * ring > budget) return false;
     CUtensorMap ma, mb, mc;
     if (!make_map(&ma, g.A, g.K, g.M_cap, g.lda, BM) || !make_map(&mb, Bk, g.K, g.N, ldbk, BN)) return false;
     if (!make_map_t(&mc, g.C, !g.c_bf16, g.N, g.M_cap, g.ldc, 32, 32,
@@ -638,7 +659,8 @@ bool gemm_row_tc(betty_ctx* c, const GemmRow& g, const void* Bk, int64_t ldbk, c
         return false;
     RowArgs p{};
     p.M_dev = g.M_dev; p.K = g.K; p.N = g.N; p.BN = BN; p.nk = nk;
-    p.stages = (int)std::max<size_t>(2, std::min<size_t>(8, (budget - 1024 - 256 - b_bytes - stage_bytes) / a_bytes));
+    p.stages = (int)std::max<size_t>(2, std::min<size_t>(8, (budget - fixed) / ring));
+    p.bstream = bstream ? 1 : 0;
     p.C = g.C; p.ldc = g.ldc;
     p.mask = g.mask; p.ldm = g.ldm; p.m_bf16 = g.m_bf16; p.res = g.res; p.ldr = g.ldr; p.nres_dev = g.nres_dev;
     p.mbits = g.mbits; p.ldmb = g.ldmb;
@@ -648,7 +670,7 @@ bool gemm_row_tc(betty_ctx* c, const GemmRow& g, const void* Bk, int64_t ldbk, c
     p.half_cols = ((BN + 63) / 64) * 32;
     p.slot_bytes = slot_bytes;
     if (p.tmem_cols > 512 || p.half_cols > 32 * MAXCH) return false;
-    const size_t smem = b_bytes + (size_t)p.stages * a_bytes + stage_bytes + 1024 + 256;
+    const size_t smem = fixed + (size_t)p.stages * ring;
     const int64_t tiles = (g.M_cap + BM - 1) / BM;
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(tiles, c->num_sms));
     const bool usebits = g.mbits != nullptr;

@@ -1,6 +1,7 @@
 // sage.h -- internal launchers of the SAGE forward/backward kernels.
 #pragma once
 #include <stdint.h>
+#include <cuda.h>
 #include <cuda_runtime.h>
 
 struct betty_ctx;
@@ -49,6 +50,8 @@ struct GemmRow {                 // C[m, n] = sum_k A[m, k] B(k, n), m < *M_dev
 bool gemm_row(betty_ctx* c, const GemmRow& g, cudaStream_t s);
 // gemm_tc.cu: tcgen05 paths (false = shape not supported, caller falls back to SIMT)
 bool tc_available();
+bool make_gather_map(CUtensorMap* m, const void* base, bool f32, int64_t cols, int64_t rows, int64_t ld,
+                     int box_cols);
 bool gemm_row_tc(betty_ctx* c, const GemmRow& g, const void* Bk, int64_t ldbk, cudaStream_t s);
 
 // P[i, j] = sum_{r < *M_dev} A[r, i] B[r, j], i < K1, j < N, split over S row groups into

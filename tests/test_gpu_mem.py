@@ -54,7 +54,7 @@ def test_memory_aware_k(B, ctx, aggr, dims):
     fan = (3, 5) if len(dims) == 3 else (3, 4, 5)
     g, sd, blocks, feats, labels = tiny(n=1500, pairs=6000, fanouts=fan, n_out=90, n_comm=9, seed=12)
     reg = oracle.reg(blocks[-1].n_src, blocks[-1].indptr, blocks[-1].nbr_pos)
-    fn = lambda K: B.betty_reg_partition(*reg, K)
+    fn = lambda K: B.betty_reg_partition(*reg, K, method="multilevel")
     dev = B.blocks_to_device(blocks)
     model = B.Model(dims, aggr)
     full_peak = int(oracle.mem_estimate(dims, aggr, blocks)[8])

@@ -35,3 +35,39 @@ def test_partition_reduces_redundancy_vs_random():
     assert cut_weight(rp, col, w, ours) < 0.8 * cut_weight(rp, col, w, rnd)
     red = [sum(oracle.extract(blocks, p, K, k)[0].n_src for k in range(K)) for p in (ours, rnd)]
     assert red[0] < red[1]
+
+
+@pytest.mark.parametrize("K", [1, 2, 7, 32])
+def test_multilevel_valid_bounded(K):
+    g, sd, blocks, feats, labels = tiny(n=3000, pairs=12000, fanouts=(4, 6), n_out=400, n_comm=20, mu=0.1, seed=2)
+    rp, col, w = oracle.reg(blocks[-1].n_src, blocks[-1].indptr, blocks[-1].nbr_pos)
+    part = B.betty_reg_partition(rp, col, w, K, method="multilevel", imbalance=0.03)
+    assert part.shape == (400,) and part.min() >= 0 and part.max() < K
+    assert np.bincount(part, minlength=K).max() <= int(np.ceil(1.03 * 400 / K))
+    assert np.array_equal(part, B.betty_reg_partition(rp, col, w, K, method="multilevel"))
+
+
+@pytest.mark.parametrize("K", [4, 16, 64])
+def test_multilevel_beats_greedy(K):
+    """The METIS scheme (Alg. 1 line 8) cuts less REG weight than greedy growing, and so
+    duplicates fewer inputs across micro-batches (Eq. 4)."""
+    g, sd, blocks, feats, labels = tiny(n=30000, pairs=150000, fanouts=(5, 10), n_out=4000, n_comm=200, mu=0.1,
+                                        seed=2)
+    rp, col, w = oracle.reg(blocks[-1].n_src, blocks[-1].indptr, blocks[-1].nbr_pos)
+    ml = B.betty_reg_partition(rp, col, w, K, method="multilevel")
+    gr = B.betty_reg_partition(rp, col, w, K)
+    assert cut_weight(rp, col, w, ml) < cut_weight(rp, col, w, gr)
+    red = [sum(oracle.extract(blocks, p, K, k)[0].n_src for k in range(K)) for p in (ml, gr)]
+    assert red[0] < red[1]
+
+
+def test_multilevel_edge_cases():
+    rp = np.zeros(1, np.int64)
+    assert len(B.betty_reg_partition(rp, np.zeros(0, np.int32), np.zeros(0, np.int32), 3, method="multilevel")) == 0
+    # no REG edges at all (every output reads distinct inputs): still a valid bounded partition
+    rp = np.zeros(101, np.int64)
+    part = B.betty_reg_partition(rp, np.zeros(0, np.int32), np.zeros(0, np.int32), 4, method="multilevel")
+    assert np.bincount(part, minlength=4).max() <= 26
+    with pytest.raises(Exception):
+        B.betty_reg_partition(np.array([0, 1], np.int64), np.array([5], np.int32), np.array([1], np.int32), 2,
+                              method="multilevel")

@@ -27,6 +27,7 @@ def main():
     p.add_argument("--graph", action="store_true")
     p.add_argument("--steps", type=int, default=1)
     p.add_argument("--scale", type=float, default=1.0)
+    p.add_argument("--group", type=int, default=0)
     a = p.parse_args()
     cfg = synth.CONFIGS[a.config]
     if a.scale != 1.0:
@@ -35,7 +36,7 @@ def main():
     ctx = B.betty_ctx_create(0)
     dev = B.blocks_to_device(ds.blocks)
     ip, col, w = B.betty_reg_build(ctx, dev[-1])
-    part = B.betty_reg_partition(ip.cpu().numpy(), col.cpu().numpy(), w.cpu().numpy(), a.K)
+    part = B.betty_reg_partition(ip.cpu().numpy(), col.cpu().numpy(), w.cpu().numpy(), a.K, method="multilevel")
     dpart = torch.as_tensor(part).cuda()
     feats = torch.as_tensor(ds.feats).cuda()
     if a.mode == "bf16":
@@ -46,7 +47,7 @@ def main():
     grad = torch.zeros_like(params)
     loss = torch.zeros(1, device="cuda")
     flags = B.PLAN_REG | (B.PLAN_GRAPH if a.graph else 0)
-    plan = B.betty_plan_create(ctx, model, dev, dpart, a.K, list(range(a.K)), group=0, flags=flags)
+    plan = B.betty_plan_create(ctx, model, dev, dpart, a.K, list(range(a.K)), group=a.group, flags=flags)
     B.betty_step(ctx, plan, params, feats, labels, 1.0 / cfg.n_out, grad, loss)
     B.betty_sync_check(ctx)
     torch.cuda.synchronize()
