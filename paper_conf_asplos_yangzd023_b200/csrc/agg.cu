@@ -271,6 +271,152 @@ __global__ void __launch_bounds__(256) k_agg_mean_xa(const Tin* __restrict__ X, 
     }
 }
 
+// ------------------------------------------------ pool, vectorised (one warp per row, float4 column groups)
+// Same semantics as k_agg_pool / k_route_pool (reading #14: max of ReLU(Zp) over the row, empty
+// row -> 0, ties -> first in row order; the gradient goes to that argmax), but every lane owns
+// T 4-column groups and a batch of 4 edges' rows is in flight at once.
+template <typename Tin, typename Tout, int T>
+__global__ void __launch_bounds__(256) k_agg_pool_v(const Tin* __restrict__ X, int64_t ldx,
+                                                    const int32_t* __restrict__ xrow, const float* __restrict__ Zp,
+                                                    int64_t ldz, const int64_t* __restrict__ indptr,
+                                                    const int32_t* __restrict__ idx, const int64_t* cnt, int Fi, int Fp,
+                                                    Tout* __restrict__ XA, int64_t ldxa, int32_t* __restrict__ arg,
+                                                    int64_t ldarg) {
+    const int64_t nd = cnt[0];
+    const int lane = lane_id();
+    const int NG = (Fi + 3) / 4;
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t v = gw; v < nd; v += nw) {
+        const int64_t b = indptr[v], e = indptr[v + 1];
+        float best[T][4];
+        int32_t am[T][4];
+#pragma unroll
+        for (int t = 0; t < T; ++t)
+#pragma unroll
+            for (int q = 0; q < 4; ++q) { best[t][q] = 0.f; am[t][q] = -1; }
+        for (int64_t e0 = b; e0 < e; e0 += 32) {
+            const int n = (int)mn64(32, e - e0);
+            const int32_t my = lane < n ? idx[e0 + lane] : 0;
+            for (int j0 = 0; j0 < n; j0 += 4) {
+                int32_t u[4];
+                float4 z[4][T];
+#pragma unroll
+                for (int k = 0; k < 4; ++k) u[k] = __shfl_sync(0xffffffffu, my, (j0 + k) & 31);
+#pragma unroll
+                for (int k = 0; k < 4; ++k)
+#pragma unroll
+                    for (int t = 0; t < T; ++t) {
+                        const int g = lane + 32 * t;
+                        z[k][t] = (j0 + k < n && g < NG) ? __ldg((const float4*)(Zp + (int64_t)u[k] * ldz) + g)
+                                                         : make_float4(0.f, 0.f, 0.f, 0.f);
+                    }
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                    if (j0 + k >= n) break;
+#pragma unroll
+                    for (int t = 0; t < T; ++t) {
+                        const float zz[4] = {fmaxf(z[k][t].x, 0.f), fmaxf(z[k][t].y, 0.f), fmaxf(z[k][t].z, 0.f),
+                                             fmaxf(z[k][t].w, 0.f)};
+#pragma unroll
+                        for (int q = 0; q < 4; ++q)
+                            if (am[t][q] < 0 || zz[q] > best[t][q]) { best[t][q] = zz[q]; am[t][q] = u[k]; }
+                    }
+                }
+            }
+        }
+        const Tin* xv = row_ptr(X, ldx, xrow, v);
+        Tout* o = XA + v * ldxa;
+#pragma unroll
+        for (int t = 0; t < T; ++t) {
+            const int g = lane + 32 * t;
+            if (g >= NG) continue;
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+                const int col = 4 * g + q;
+                if (col < Fi) {
+                    st_act(o + col, ld_act(xv + col));
+                    st_act(o + Fp + col, best[t][q]);
+                    arg[v * ldarg + col] = am[t][q];
+                }
+            }
+        }
+        for (int col = Fi + lane; col < Fp; col += 32) { st_act(o + col, 0.f); st_act(o + Fp + col, 0.f); }
+        for (int col = 2 * Fp + lane; col < ldxa; col += 32) st_act(o + col, col == 2 * Fp ? 1.f : 0.f);
+    }
+}
+template <typename Tout, int T>
+__global__ void __launch_bounds__(256) k_route_pool_v(const float* __restrict__ dXA, int64_t ldd,
+                                                      const int32_t* __restrict__ arg, int64_t ldarg,
+                                                      const int64_t* __restrict__ t_indptr,
+                                                      const int32_t* __restrict__ t_idx, const int64_t* cnt, int Fi,
+                                                      int Fp, const float* __restrict__ Zp, int64_t ldz,
+                                                      Tout* __restrict__ out, int64_t ldo) {
+    const int64_t ns = cnt[1];
+    const int lane = lane_id();
+    const int NG = (Fi + 3) / 4;
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t u = gw; u < ns; u += nw) {
+        const int64_t b = t_indptr[u], e = t_indptr[u + 1];
+        float acc[T][4];
+#pragma unroll
+        for (int t = 0; t < T; ++t)
+#pragma unroll
+            for (int q = 0; q < 4; ++q) acc[t][q] = 0.f;
+        for (int64_t e0 = b; e0 < e; e0 += 32) {
+            const int n = (int)mn64(32, e - e0);
+            const int32_t my = lane < n ? t_idx[e0 + lane] : 0;
+            for (int j0 = 0; j0 < n; j0 += 4) {
+                int32_t v[4];
+                int4 a[4][T];
+#pragma unroll
+                for (int k = 0; k < 4; ++k) v[k] = __shfl_sync(0xffffffffu, my, (j0 + k) & 31);
+#pragma unroll
+                for (int k = 0; k < 4; ++k)
+#pragma unroll
+                    for (int t = 0; t < T; ++t) {
+                        const int g = lane + 32 * t;
+                        a[k][t] = (j0 + k < n && g < NG) ? __ldg((const int4*)(arg + (int64_t)v[k] * ldarg) + g)
+                                                         : make_int4(-1, -1, -1, -1);
+                    }
+                float4 d[4][T];
+#pragma unroll
+                for (int k = 0; k < 4; ++k)
+#pragma unroll
+                    for (int t = 0; t < T; ++t) {
+                        const int g = lane + 32 * t;
+                        const bool hit = a[k][t].x == (int32_t)u || a[k][t].y == (int32_t)u || a[k][t].z == (int32_t)u ||
+                                         a[k][t].w == (int32_t)u;
+                        d[k][t] = hit ? __ldg((const float4*)(dXA + (int64_t)v[k] * ldd + Fp) + g)
+                                      : make_float4(0.f, 0.f, 0.f, 0.f);
+                    }
+#pragma unroll
+                for (int k = 0; k < 4; ++k)
+#pragma unroll
+                    for (int t = 0; t < T; ++t) {
+                        if (a[k][t].x == (int32_t)u) acc[t][0] += d[k][t].x;
+                        if (a[k][t].y == (int32_t)u) acc[t][1] += d[k][t].y;
+                        if (a[k][t].z == (int32_t)u) acc[t][2] += d[k][t].z;
+                        if (a[k][t].w == (int32_t)u) acc[t][3] += d[k][t].w;
+                    }
+            }
+        }
+        const float* zu = Zp + u * ldz;
+#pragma unroll
+        for (int t = 0; t < T; ++t) {
+            const int g = lane + 32 * t;
+            if (g >= NG) continue;
+            const float4 z = __ldg((const float4*)zu + g);
+            const float r[4] = {z.x > 0.f ? acc[t][0] : 0.f, z.y > 0.f ? acc[t][1] : 0.f, z.z > 0.f ? acc[t][2] : 0.f,
+                                z.w > 0.f ? acc[t][3] : 0.f};
+#pragma unroll
+            for (int q = 0; q < 4; ++q) if (4 * g + q < Fi) st_act(out + u * ldo + 4 * g + q, r[q]);
+        }
+        for (int col = Fi + lane; col < ldo; col += 32) st_act(out + u * ldo + col, 0.f);
+    }
+}
+
 // ------------------------------------------------ mean, aggregate-first fwd: TMA gather4 pipeline
 // Warp-specialised persistent kernel, one CTA per SM: G4_PROD producer warps, each owning every
 // G4_PROD-th stage of a G4_STAGES ring, and G4_CONS consumer warps.
@@ -288,8 +434,10 @@ __global__ void __launch_bounds__(256) k_agg_mean_xa(const Tin* __restrict__ X, 
 //    memory and stream XA out.  A row whose neighbours exceed the slots ("long" row, e.g.
 //    full-neighbourhood layers) is a stage of its own that the consumers reduce straight from
 //    global memory.
-constexpr int G4_STAGES = 8, G4_PROD = 4, G4_THREADS = 256, G4_MAXR = 16, G4_CLAIM = 64;
-constexpr int G4_CONS = G4_THREADS / 32 - G4_PROD;
+constexpr int G4_STAGES = 8, G4_PROD = 4, G4_CPP = 3, G4_MAXR = 16, G4_CLAIM = 64;
+constexpr int G4_CONS = G4_PROD * G4_CPP;             // consumer warps: G4_CPP per producer
+constexpr int G4_THREADS = 32 * (G4_PROD + G4_CONS);
+static_assert(G4_STAGES % G4_PROD == 0, "stages are dealt round-robin to the producers");
 struct G4Hdr {
     int64_t r0;                  // first real row
     int64_t hb, he;              // long row: its edge range
@@ -356,7 +504,7 @@ __global__ void __launch_bounds__(G4_THREADS, 1) k_agg_mean_g4(const __grid_cons
     const int nseg = order_load(a.otab, s_vs, s_rs);
     const int warp = threadIdx.x >> 5, lane = lane_id();
     if (threadIdx.x == 0) {
-        for (int s = 0; s < G4_STAGES; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], G4_CONS); }
+        for (int s = 0; s < G4_STAGES; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], G4_CPP); }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
@@ -465,31 +613,37 @@ __global__ void __launch_bounds__(G4_THREADS, 1) k_agg_mean_g4(const __grid_cons
         asm volatile("cp.async.wait_all;" ::: "memory");
     } else {
         // ---------------------------------------------------------------- consumers
-        const int ct = threadIdx.x - G4_PROD * 32;
-        const int NC = G4_CONS * 32;
+        // consumer warps w*G4_CPP .. w*G4_CPP + G4_CPP-1 drain the stages of producer w
+        const int w = (warp - G4_PROD) / G4_CPP, cw = (warp - G4_PROD) % G4_CPP;
+        const int ct = cw * 32 + lane, NCT = G4_CPP * 32;
         const int NV = a.NV;
-        float* red = (float*)(g4_smem + (size_t)G4_STAGES * a.stage_bytes);   // [G4_CONS][NV*VW] long-row partials
-        unsigned done = 0;                      // producers that ran out of work
-        for (uint32_t it = 0; done != (1u << G4_PROD) - 1u; ++it) {
-            const int s = it % G4_STAGES;
-            if (done >> (s % G4_PROD) & 1u) continue;
-            mbar_wait_parity(&full[s], (it / G4_STAGES) & 1u);
+        for (uint32_t i = 0;; ++i) {
+            const int s = (w + G4_PROD * i) % G4_STAGES;
+            mbar_wait_parity(&full[s], (i / (G4_STAGES / G4_PROD)) & 1u);
             const G4Hdr& H = hdr[s];
             const int n = H.n;
-            if (n < 0) { done |= 1u << (s % G4_PROD); continue; }
+            if (n < 0) break;
             const uint8_t* sdat = g4_smem + (size_t)s * a.stage_bytes;
             if (!H.lng) {
-                for (int u = ct; u < n * NV; u += NC) {
+                for (int u = ct; u < n * NV; u += NCT) {
                     const int i = u / NV, j = u - i * NV;
                     const int b = H.off[i], e = H.off[i + 1];
                     float acc[VW];
 #pragma unroll
                     for (int t = 0; t < VW; ++t) acc[t] = 0.f;
-                    const uint8_t* p = sdat + (b >> 2) * a.grp_bytes + (b & 3) * a.row_bytes + j * 16;
-                    for (int sl = b; sl < e; ++sl) {
-                        VI::add_raw(acc, *(const typename VI::Raw*)p);
-                        p += ((sl & 3) == 3) ? a.grp_bytes - 3 * a.row_bytes : a.row_bytes;
+                    const uint8_t* base = sdat + j * 16;
+                    int sl = b;
+                    for (; sl + 4 <= e; sl += 4) {          // 4 independent shared loads in flight
+                        typename VI::Raw r[4];
+#pragma unroll
+                        for (int q = 0; q < 4; ++q)
+                            r[q] = *(const typename VI::Raw*)(base + ((sl + q) >> 2) * a.grp_bytes +
+                                                               ((sl + q) & 3) * a.row_bytes);
+#pragma unroll
+                        for (int q = 0; q < 4; ++q) VI::add_raw(acc, r[q]);
                     }
+                    for (; sl < e; ++sl)
+                        VI::add_raw(acc, *(const typename VI::Raw*)(base + (sl >> 2) * a.grp_bytes + (sl & 3) * a.row_bytes));
                     float so[VW];
 #pragma unroll
                     for (int t = 0; t < VW; ++t) so[t] = 0.f;
@@ -506,31 +660,34 @@ __global__ void __launch_bounds__(G4_THREADS, 1) k_agg_mean_g4(const __grid_cons
                     st_vec_cs<Tout, VW>(out + j * VW, so);
                     st_vec_cs<Tout, VW>(out + a.Fp + j * VW, acc);
                 }
-                if (ct < n) xa_tail<Tout>((Tout*)a.XA + (H.r0 + ct) * a.ldxa, NV * VW, a.Fp, a.ldxa);
+                for (int i = ct; i < n; i += NCT) xa_tail<Tout>((Tout*)a.XA + (H.r0 + i) * a.ldxa, NV * VW, a.Fp, a.ldxa);
             } else {
-                // long row: consumer warp w sums edges w, w + G4_CONS, ...; lanes over vectors
-                const int w = ct >> 5;
+                // long row (first consumer warp of the pair): lanes over vectors, 4 edges in flight,
+                // straight from global memory
                 const int64_t hb = H.hb, he = H.he;
-                for (int j = lane; j < NV; j += 32) {
+                for (int j = lane; cw == 0 && j < NV; j += 32) {
                     float acc[VW];
 #pragma unroll
                     for (int t = 0; t < VW; ++t) acc[t] = 0.f;
-                    for (int64_t e = hb + w; e < he; e += G4_CONS) {
+                    int64_t e = hb;
+                    for (; e + 4 <= he; e += 4) {
+                        int32_t u[4];
+                        typename VI::Raw r[4];
+#pragma unroll
+                        for (int q = 0; q < 4; ++q) { u[q] = __ldg(a.erow + e + q); if (a.emap) u[q] = __ldg(a.emap + u[q]); }
+#pragma unroll
+                        for (int q = 0; q < 4; ++q) r[q] = VI::ld_raw((const Tin*)a.X + (int64_t)u[q] * a.ldx + j * VW);
+#pragma unroll
+                        for (int q = 0; q < 4; ++q) VI::add_raw(acc, r[q]);
+                    }
+                    for (; e < he; ++e) {
                         int32_t u = __ldg(a.erow + e);
                         if (a.emap) u = __ldg(a.emap + u);
                         VI::add_raw(acc, VI::ld_raw((const Tin*)a.X + (int64_t)u * a.ldx + j * VW));
                     }
+                    float so[VW];
 #pragma unroll
-                    for (int t = 0; t < VW; ++t) red[(w * NV + j) * VW + t] = acc[t];
-                }
-                asm volatile("bar.sync 1, %0;" ::"r"(NC) : "memory");
-                for (int j = ct; j < NV; j += NC) {
-                    float acc[VW], so[VW];
-#pragma unroll
-                    for (int t = 0; t < VW; ++t) { acc[t] = 0.f; so[t] = 0.f; }
-                    for (int q = 0; q < G4_CONS; ++q)
-#pragma unroll
-                        for (int t = 0; t < VW; ++t) acc[t] += red[(q * NV + j) * VW + t];
+                    for (int t = 0; t < VW; ++t) so[t] = 0.f;
                     VI::add_raw(so, *(const typename VI::Raw*)(sdat + self_off + j * 16));
                     const float inv = he > hb ? 1.0f / (float)(he - hb) : 0.0f;
 #pragma unroll
@@ -544,7 +701,6 @@ __global__ void __launch_bounds__(G4_THREADS, 1) k_agg_mean_g4(const __grid_cons
                     st_vec_cs<Tout, VW>(out + a.Fp + j * VW, acc);
                 }
                 if (ct == 0) xa_tail<Tout>((Tout*)a.XA + H.r0 * a.ldxa, NV * VW, a.Fp, a.ldxa);
-                asm volatile("bar.sync 1, %0;" ::"r"(NC) : "memory");
             }
             __syncwarp();
             if (lane == 0) mbar_arrive(&empty[s]);
@@ -932,7 +1088,7 @@ static bool agg_mean_g4(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, c
     a.XA = XA; a.ldxa = ldxa; a.X = X; a.ldx = ldx; a.ctr = ctr; a.Fi = Fi; a.Fp = Fp; a.NV = nv; a.hint = hint;
     a.row_bytes = (uint32_t)nv * 16u;
     a.grp_bytes = (4u * a.row_bytes + 127u) / 128u * 128u;
-    const size_t red_bytes = (size_t)G4_CONS * nv * vw * 4;
+    const size_t red_bytes = 0;
     const size_t budget = (size_t)196 * 1024 - red_bytes;            // dynamic smem for the stage ring
     const int64_t groups = (int64_t)(budget / G4_STAGES) / a.grp_bytes - G4_MAXR / 4;
     if (groups < 4) return false;
@@ -1031,6 +1187,17 @@ void csc_pf(betty_ctx* c, const void* dS, bool ds_bf16, int64_t ldds, const int6
 void agg_pool(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const int32_t* xrow, const float* Zp, int64_t ldz,
               const int64_t* indptr, const int32_t* idx, const int64_t* cnt, int64_t rows_cap, int Fi, int Fp,
               void* XA, bool xa_bf16, int64_t ldxa, int32_t* arg, int64_t ldarg, cudaStream_t s) {
+    const int ng = (Fi + 3) / 4;
+    const bool vec = (ldz % 4) == 0 && (ldarg % 4) == 0 && ng <= 64 && ((uintptr_t)Zp & 15) == 0 &&
+                     ((uintptr_t)arg & 15) == 0;
+    if (vec) {
+        DISPATCH_ACT(x_bf16, TI, DISPATCH_ACT(xa_bf16, TO, {
+            if (ng <= 32) k_agg_pool_v<TI, TO, 1><<<warps_grid(c, rows_cap), 256, 0, s>>>((const TI*)X, ldx, xrow, Zp,
+                ldz, indptr, idx, cnt, Fi, Fp, (TO*)XA, ldxa, arg, ldarg);
+            else k_agg_pool_v<TI, TO, 2><<<warps_grid(c, rows_cap), 256, 0, s>>>((const TI*)X, ldx, xrow, Zp, ldz,
+                indptr, idx, cnt, Fi, Fp, (TO*)XA, ldxa, arg, ldarg); }))
+        return;
+    }
     DISPATCH_ACT(x_bf16, TI, DISPATCH_ACT(xa_bf16, TO,
         k_agg_pool<TI, TO><<<warps_grid(c, rows_cap), 256, 0, s>>>((const TI*)X, ldx, xrow, Zp, ldz, indptr, idx, cnt,
                                                                    Fi, Fp, (TO*)XA, ldxa, arg, ldarg)));
@@ -1039,6 +1206,17 @@ void agg_pool(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const int32
 void route_pool(betty_ctx* c, const float* dXA, int64_t ldd, const int32_t* arg, int64_t ldarg,
                 const int64_t* t_indptr, const int32_t* t_idx, const int64_t* cnt, int64_t src_cap, int Fi, int Fp,
                 const float* Zp, int64_t ldz, void* out, bool out_bf16, int64_t ldo, cudaStream_t s) {
+    const int ng = (Fi + 3) / 4;
+    const bool vec = (ldz % 4) == 0 && (ldarg % 4) == 0 && (ldd % 4) == 0 && (Fp % 4) == 0 && ng <= 64 &&
+                     ((uintptr_t)Zp & 15) == 0 && ((uintptr_t)arg & 15) == 0 && ((uintptr_t)dXA & 15) == 0;
+    if (vec) {
+        DISPATCH_ACT(out_bf16, TO, {
+            if (ng <= 32) k_route_pool_v<TO, 1><<<warps_grid(c, src_cap), 256, 0, s>>>(dXA, ldd, arg, ldarg, t_indptr,
+                t_idx, cnt, Fi, Fp, Zp, ldz, (TO*)out, ldo);
+            else k_route_pool_v<TO, 2><<<warps_grid(c, src_cap), 256, 0, s>>>(dXA, ldd, arg, ldarg, t_indptr, t_idx,
+                cnt, Fi, Fp, Zp, ldz, (TO*)out, ldo); })
+        return;
+    }
     DISPATCH_ACT(out_bf16, TO,
         k_route_pool<TO><<<warps_grid(c, src_cap), 256, 0, s>>>(dXA, ldd, arg, ldarg, t_indptr, t_idx, cnt, Fi, Fp, Zp,
                                                                 ldz, (TO*)out, ldo));

@@ -9,6 +9,7 @@
 //             parameter layout mapping.
 // The tcgen05 tensor-core path (gemm_tc.cu) replaces these in BF16 mode for
 // the large shapes; these stay the FP32-mode path and the small-shape path.
+#include <algorithm>
 #include "common.cuh"
 #include "internal.h"
 #include "sage.h"
@@ -126,7 +127,21 @@ bool gemm_row(betty_ctx* c, const GemmRow& g, cudaStream_t s) {
     if (c->use_tc && g.a_bf16 && g.b_bf16) {
         const void* Bk = g.transB ? g.B : g.Bt;
         const int64_t ldbk = g.transB ? g.ldb : g.ldbt;
-        if (Bk && gemm_row_tc(c, g, Bk, ldbk, s)) return g.epi == EPI_RELU_ONES && g.obits;
+        if (Bk && g.N <= 256 && gemm_row_tc(c, g, Bk, ldbk, s)) return g.epi == EPI_RELU_ONES && g.obits;
+        // wider plain products (the pool layers' dXA, N = 2 Fp): 256-column blocks, left to right (each
+        // block writes only its own columns; the last one the trailing columns)
+        if (Bk && g.N > 256 && g.epi == EPI_STORE && (ldbk & 7) == 0) {
+            const size_t cs = g.c_bf16 ? 2 : 4;
+            bool ok = true;
+            for (int n0 = 0; n0 < g.N && ok; n0 += 256) {
+                GemmRow h = g;
+                h.N = std::min(256, g.N - n0);
+                h.C = (char*)g.C + (size_t)n0 * cs;
+                h.cend = n0 + 256 >= g.N ? g.ldc - n0 : h.N;
+                ok = gemm_row_tc(c, h, (const char*)Bk + (size_t)n0 * ldbk * 2, ldbk, s);
+            }
+            if (ok) return false;
+        }
     }
     if (g.a_bf16) {
         if (g.b_bf16) launch_row<__nv_bfloat16, __nv_bfloat16>(c, g, s);

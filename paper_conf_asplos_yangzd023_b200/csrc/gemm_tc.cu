@@ -130,6 +130,7 @@ struct RowArgs {
     int half_cols;           // columns per epilogue half (multiple of 32, <= 32 * MAXCH)
     uint32_t slot_bytes;     // one staging slot: 32 rows x 32 columns
     int bstream;             // 1: B is streamed with A through the ring (B too large to stay resident)
+    int64_t cend;            // trailing columns [N, cend) of a row are written (ones column / zeros)
 };
 
 __device__ __forceinline__ uint32_t pack_bf16x2(float a, float b) {
@@ -424,13 +425,13 @@ __global__ void __launch_bounds__(ROW_THREADS, 1) k_tc_row(const __grid_constant
                     for (int ci = 0; ci < MAXCH; ++ci) if (ci < nch) ob[ci] = obits[ci];
             }
             // trailing columns [N, ldc): the ones column after a ReLU layer, zeros elsewhere
-            if (h == 1 && ok && p.ldc > p.N) {
-                const int w = (int)(p.ldc - p.N);
+            if (h == 1 && ok && p.cend > p.N) {
+                const int w = (int)(p.cend - p.N);
                 if (CBF && w == 8 && ((m * p.ldc + p.N) & 7) == 0) {
                     const uint32_t one = EPI == EPI_RELU_ONES ? 0x3F80u : 0u;
                     *(uint4*)((__nv_bfloat16*)p.C + m * p.ldc + p.N) = make_uint4(one, 0u, 0u, 0u);
                 } else {
-                    for (int col = p.N; col < p.ldc; ++col) {
+                    for (int col = p.N; col < p.cend; ++col) {
                         const float x = (EPI == EPI_RELU_ONES && col == p.N) ? 1.f : 0.f;
                         if (CBF) ((__nv_bfloat16*)p.C)[m * p.ldc + col] = __float2bfloat16_rn(x);
                         else ((float*)p.C)[m * p.ldc + col] = x;
@@ -661,7 +662,7 @@ bool gemm_row_tc(betty_ctx* c, const GemmRow& g, const void* Bk, int64_t ldbk, c
     p.M_dev = g.M_dev; p.K = g.K; p.N = g.N; p.BN = BN; p.nk = nk;
     p.stages = (int)std::max<size_t>(2, std::min<size_t>(8, (budget - fixed) / ring));
     p.bstream = bstream ? 1 : 0;
-    p.C = g.C; p.ldc = g.ldc;
+    p.C = g.C; p.ldc = g.ldc; p.cend = g.cend > 0 ? g.cend : g.ldc;
     p.mask = g.mask; p.ldm = g.ldm; p.m_bf16 = g.m_bf16; p.res = g.res; p.ldr = g.ldr; p.nres_dev = g.nres_dev;
     p.mbits = g.mbits; p.ldmb = g.ldmb;
     p.obits = g.epi == EPI_RELU_ONES ? g.obits : nullptr; p.ldob = g.ldob;

@@ -58,7 +58,7 @@ bool make_model_cfg(int L, int aggr, int gemm, int feat_dtype, const int32_t* di
         c.ld_dxa = 2 * c.Fp;
         c.ld_zp = c.Fp;
         c.ld_dzp = c.Fp;
-        c.ld_arg = c.Fi;
+        c.ld_arg = c.Fp;                 // 16-byte aligned rows (vectorised pool kernels)
         c.ld_out = c.last ? c.Fop : r8(c.Fo + 1);
         c.ld_ds = c.Fop;
         c.ld_B = c.kind == KIND_PF ? 2 * c.Fop : c.Fop;

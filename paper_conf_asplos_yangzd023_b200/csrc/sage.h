@@ -45,6 +45,7 @@ struct GemmRow {                 // C[m, n] = sum_k A[m, k] B(k, n), m < *M_dev
     const void* Bt; int64_t ldbt;                          // K-major copy of B (N x K) for the tensor-core path
     const uint32_t* mbits; int64_t ldmb;   // EPI_MASK / EPI_RES_MASK: mask as ReLU bits (tensor-core path), or null
     uint32_t* obits; int64_t ldob;         // EPI_RELU_ONES: also write the ReLU bits [C > 0] (tensor-core path)
+    int64_t cend = 0;                      // tensor-core path: trailing columns [N, cend) written (0: ldc)
 };
 // returns true iff the ReLU bits g.obits were written (EPI_RELU_ONES on the tensor-core path)
 bool gemm_row(betty_ctx* c, const GemmRow& g, cudaStream_t s);

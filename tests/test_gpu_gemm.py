@@ -19,7 +19,8 @@ def ctx(B):
 
 
 SHAPES = [(1, 16, 16), (127, 64, 48), (128, 100, 47), (300, 209, 256), (5000, 257, 96), (4099, 513, 208),
-          (700, 40, 256), (2000, 513, 256), (1000, 257, 256)]   # the last three stream B (too big to stay resident)
+          (700, 40, 256), (2000, 513, 256), (1000, 257, 256),   # these three stream B (too big to stay resident)
+          (777, 200, 513)]                                       # 256-column blocks (the pool layers' dXA)
 
 
 def rel(a, b):

@@ -184,10 +184,14 @@ CASES = [
     dict(name="mean2-pf0", aggr="mean", fanouts=(3, 4), dims=[70, 16, 4]),
     dict(name="pool2", aggr="pool", fanouts=(3, 4), dims=[16, 24, 5]),
     dict(name="pool3", aggr="pool", fanouts=(2, 3, 3), dims=[12, 16, 16, 3]),
+    # full neighbourhoods on dense graphs: rows longer than the gather pipeline's stage ("long rows")
+    dict(name="mean2-full-hub", aggr="mean", fanouts=(-1, -1), dims=[8, 16, 3], n=400, pairs=30000),
+    dict(name="mean2-full-wide", aggr="mean", fanouts=(-1, -1), dims=[100, 128, 5], n=400, pairs=8000),
 ]
 
 
 def make_case(c, seed=1, n=600, pairs=2400, n_out=60):
+    n, pairs = c.get("n", n), c.get("pairs", pairs)
     F = c["dims"][0]
     ld = (F + 7) // 8 * 8
     g, sd, blocks, feats, _ = tiny(n=n, pairs=pairs, fanouts=c["fanouts"], n_out=n_out, F=F, C=c["dims"][-1],
@@ -237,7 +241,7 @@ def test_sage_micro_batch(B, ctx, c, mode):
 @pytest.mark.parametrize("mode", ["fp32", "bf16"])
 @pytest.mark.parametrize("group", [1, 2, 0])
 @pytest.mark.parametrize("graph", [False, True])
-@pytest.mark.parametrize("c", [CASES[1], CASES[2], CASES[4]], ids=lambda c: c["name"])
+@pytest.mark.parametrize("c", [CASES[1], CASES[2], CASES[4], CASES[7]], ids=lambda c: c["name"])
 def test_step_matches_oracle(B, ctx, c, mode, group, graph):
     """betty_step (fused extraction + fwd + loss + bwd + accumulation over a
     rank's micro-batches) vs oracle_step, for several launch groupings."""
