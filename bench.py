@@ -241,6 +241,18 @@ def alg_bytes(site: str, info: dict, cfg, mode: str, n_groups: int):
     return b / max(n_groups, 1)
 
 
+METRIC = "aggregated edges/s (SAGE, products-shape); epoch time = ms_per_step"
+
+
+def workload_config(args, cfg, ws):
+    """The `config` object both arms print (same workload, same K and partition)."""
+    return {"workload": f"{args.config}: {cfg.name}-shaped DC-SBM ({cfg.n} nodes, {cfg.n}x{cfg.F} feats), "
+                        f"{cfg.L}-layer SAGE-{cfg.aggr} {cfg.dims}, fanout {tuple(cfg.fanouts)}, {cfg.n_out} outputs",
+            "K": args.K, "partition": args.partition, "group": args.group or "all",
+            "step": ("REG + " if not args.no_reg else "") + "extract + fwd + loss + bwd + allreduce + adam",
+            "graph": not args.no_graph, "parallelism": f"dp{ws} over micro-batches"}
+
+
 # ------------------------------------------------------------ reference arm
 def run_reference(args, ws, rank):
     """The CPU oracle, as it stands, on a bounded sample of the same workload
@@ -265,10 +277,10 @@ def run_reference(args, ws, rank):
             times.append(time.perf_counter() - t0)
     t = float(np.mean(times))
     val = edges / t
-    line = {"impl": "reference", "metric": "aggregated edges/s (SAGE, products-shape)", "value": val,
+    line = {"impl": "reference", "metric": METRIC, "value": val,
             "unit": "edges/s", "higher_is_better": True, "n_gpus": args.gpus, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": t * 1e3, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": f"{args.config} {cfg.name}-shaped, bounded sample", "sample": sample_desc},
+            "config": dict(workload_config(args, cfg, ws), sample=sample_desc),
             "cpu_baseline": {"value": val, "unit": "edges/s", "cores": 1, "kind": "oracle", "sample": sample_desc},
             "e2e": {"value": val, "unit": "edges/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
@@ -456,20 +468,14 @@ def main():
 
     if rank == 0:
         line = {
-            "metric": "aggregated edges/s (SAGE, products-shape); epoch time = ms_per_step",
+            "metric": METRIC,
             "value": value, "unit": "edges/s", "n_gpus": ws, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": ms_step, "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
             "dtype": "bf16-gemm/fp32-accum" if args.mode == "bf16" else "fp32",
             "data": "synthetic",
-            "config": {"workload": f"{args.config}: {cfg.name}-shaped DC-SBM ({cfg.n} nodes, "
-                                   f"{len(ds.feats)}x{cfg.F} feats), {cfg.L}-layer SAGE-{cfg.aggr} "
-                                   f"{cfg.dims}, fanout {tuple(cfg.fanouts)}, {cfg.n_out} outputs",
-                       "K": args.K, "partition": args.partition, "group": args.group or "all",
-                       "micro_batches_per_rank": len(my_k), "step": ("REG + " if not args.no_reg else "") +
-                       "extract + fwd + loss + bwd + allreduce + adam", "graph": not args.no_graph,
-                       "parallelism": f"dp{ws} over micro-batches",
-                       "l2": "inputs > L2 (feature table %.2f GB + blocks)" % (feats.numel() * feats.element_size()
-                                                                           / 1e9)},
+            "config": dict(workload_config(args, cfg, ws), micro_batches_per_rank=len(my_k),
+                           l2="inputs > L2 (feature table %.2f GB + blocks)" % (feats.numel() * feats.element_size()
+                                                                              / 1e9)),
             "edges_per_step": edges_all,
             "full_batch_edges": int(sum(b.n_edges for b in ds.blocks)),
             "plan": {k: info[k] for k in ("n_groups", "edges", "n_src", "n_dst", "reg_nnz", "arena_bytes",

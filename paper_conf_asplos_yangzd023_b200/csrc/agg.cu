@@ -146,7 +146,7 @@ __global__ void __launch_bounds__(256) k_agg_mean_xa(const Tin* __restrict__ X, 
     // micro-batch shares are re-read from L2; statically strided warps drift apart instead.
     // whole-row bulk copies (TMA engine): one instruction per neighbour row instead of one
     // 16-byte cp.async per lane; only when one pass covers the whole row
-    const bool bulk = vlo == 0 && vhi == NV;
+    const bool bulk = vlo == 0 && vhi == NV && hint < 2;     // hint 2: per-lane cp.async instead
     const uint32_t row_bytes = (uint32_t)NV * 16u;
     uint64_t* bar = &s_bar[wib][grp];
     uint32_t bph = 0;
@@ -1118,7 +1118,7 @@ void agg_mean_xa(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const in
     // only a slice of every row (the rows' metadata is re-read, the features are not).
     static const double budget = getenv("BETTY_AGG_WS_MB") ? atof(getenv("BETTY_AGG_WS_MB")) * 1e6 : 1e12;
     unsigned* ctr = c->L().counters + CTR_AGG;
-    static const int hint = getenv("BETTY_AGG_NOHINT") ? 0 : 1;
+    static const int hint = getenv("BETTY_AGG_NOHINT") ? 0 : (getenv("BETTY_AGG_NOBULK") ? 2 : 1);
     static const bool no_order = getenv("BETTY_AGG_NOORDER") != nullptr;
     const double ws = (double)src_per_mb * (double)nv * 16.0;
     int passes = (int)std::max(1.0, std::min((double)nv, std::ceil(ws / budget)));
