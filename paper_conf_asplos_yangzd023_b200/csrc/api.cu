@@ -83,14 +83,14 @@ extern "C" betty_status betty_ctx_create(int device, betty_alloc_fn alloc, betty
     c->dealloc = dealloc;
     c->user = user;
     cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, device);
-    // per lane: counters [64 unsigned] + loss partials [512 double], big-segment list; device error flags
+    // per lane: counters [64 unsigned] + loss partials [2048 double], big-segment list; device error flags
     bool ok = cudaMalloc(&c->dev_err, 16) == cudaSuccess;
     for (auto& ln : c->lanes) {
         ln.big_list_cap = 1 << 20;
-        ok = ok && cudaMalloc(&ln.counters, 64 * 4 + 512 * 8) == cudaSuccess &&
+        ok = ok && cudaMalloc(&ln.counters, 64 * 4 + 2048 * 8) == cudaSuccess &&
              cudaMalloc(&ln.big_count, 16) == cudaSuccess &&
              cudaMalloc(&ln.big_list, sizeof(int64_t) * ln.big_list_cap) == cudaSuccess;
-        if (ok) { cudaMemset(ln.counters, 0, 64 * 4 + 512 * 8); cudaMemset(ln.big_count, 0, 16); }
+        if (ok) { cudaMemset(ln.counters, 0, 64 * 4 + 2048 * 8); cudaMemset(ln.big_count, 0, 16); }
     }
     if (!ok) { betty_ctx_destroy(c); return BETTY_ENOMEM; }
     init_kernel_attrs();

@@ -109,6 +109,92 @@ __global__ void k_mark_dst(const int32_t* __restrict__ dst_pos, const int32_t* _
     }
 }
 
+// Rank words {bits, slot-relative popcount prefix} of c slots x W bitmap words, in two fully
+// parallel passes (no look-back chain): chunk popcount sums, then each chunk adds the sums of
+// the slot's earlier chunks and scans its own words.  slot_total[j] (optional) = set bits of j.
+constexpr int RANK_THREADS = 256, RANK_ITEMS = 16, RANK_CHUNK = RANK_THREADS * RANK_ITEMS;
+__global__ void __launch_bounds__(RANK_THREADS) k_rank_sums(const uint32_t* __restrict__ bits,
+                                                             const uint32_t* __restrict__ mask, int64_t W,
+                                                             int64_t* __restrict__ csum) {
+    __shared__ int64_t s_warp[RANK_THREADS / 32 + 1];
+    const int j = blockIdx.y;
+    const int64_t c0 = (int64_t)blockIdx.x * RANK_CHUNK;
+    const uint32_t* b = bits + (int64_t)j * W;
+    const uint32_t* m = mask ? mask + (int64_t)j * W : nullptr;
+    int64_t cnt = 0;
+#pragma unroll
+    for (int i = 0; i < RANK_ITEMS; ++i) {              // coalesced: word c0 + i * RANK_THREADS + t
+        const int64_t w = c0 + i * RANK_THREADS + threadIdx.x;
+        if (w < W) cnt += __popc(b[w] & (m ? ~m[w] : ~0u));
+    }
+    int64_t tot;
+    block_excl_scan(cnt, s_warp, &tot);
+    if (threadIdx.x == 0) csum[(int64_t)j * gridDim.x + blockIdx.x] = tot;
+}
+// padded shared index: thread t's 16 consecutive words fall in distinct banks
+__device__ __forceinline__ int rpad(int w) { return w + (w >> 4); }
+__global__ void __launch_bounds__(RANK_THREADS) k_rank_write(const uint32_t* __restrict__ bits,
+                                                              const uint32_t* __restrict__ mask, int64_t W,
+                                                              const int64_t* __restrict__ csum, uint2* __restrict__ out,
+                                                              int64_t* __restrict__ slot_total) {
+    __shared__ int64_t s_warp[RANK_THREADS / 32 + 1];
+    __shared__ int64_t s_base;
+    __shared__ uint32_t s_bits[RANK_CHUNK + RANK_CHUNK / 16], s_pre[RANK_CHUNK + RANK_CHUNK / 16];
+    const int j = blockIdx.y;
+    const int nch = gridDim.x;
+    if (threadIdx.x < 32) {                             // sums of the slot's earlier chunks (and all of them)
+        int64_t pre = 0, all = 0;
+        for (int q = threadIdx.x; q < nch; q += 32) {
+            const int64_t v = csum[(int64_t)j * nch + q];
+            all += v;
+            if (q < (int)blockIdx.x) pre += v;
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            pre += __shfl_xor_sync(0xffffffffu, pre, o);
+            all += __shfl_xor_sync(0xffffffffu, all, o);
+        }
+        if (threadIdx.x == 0) {
+            s_base = pre;
+            if (slot_total && blockIdx.x == 0) slot_total[j] = all;
+        }
+    }
+    const int64_t c0 = (int64_t)blockIdx.x * RANK_CHUNK;
+    const uint32_t* b = bits + (int64_t)j * W;
+    const uint32_t* m = mask ? mask + (int64_t)j * W : nullptr;
+#pragma unroll
+    for (int i = 0; i < RANK_ITEMS; ++i) {              // coalesced load -> shared
+        const int wl = i * RANK_THREADS + threadIdx.x;
+        const int64_t w = c0 + wl;
+        s_bits[rpad(wl)] = w < W ? b[w] & (m ? ~m[w] : ~0u) : 0u;
+    }
+    __syncthreads();
+    uint32_t v[RANK_ITEMS];
+    int64_t cnt = 0;
+#pragma unroll
+    for (int i = 0; i < RANK_ITEMS; ++i) { v[i] = s_bits[rpad(threadIdx.x * RANK_ITEMS + i)]; cnt += __popc(v[i]); }
+    int64_t tot;
+    const int64_t ex = block_excl_scan(cnt, s_warp, &tot);    // (syncs: s_base visible)
+    uint32_t run = (uint32_t)(s_base + ex);
+#pragma unroll
+    for (int i = 0; i < RANK_ITEMS; ++i) { s_pre[rpad(threadIdx.x * RANK_ITEMS + i)] = run; run += __popc(v[i]); }
+    __syncthreads();
+    uint2* o = out + (int64_t)j * W;
+#pragma unroll
+    for (int i = 0; i < RANK_ITEMS; ++i) {              // coalesced store
+        const int wl = i * RANK_THREADS + threadIdx.x;
+        const int64_t w = c0 + wl;
+        if (w < W) o[w] = make_uint2(s_bits[rpad(wl)], s_pre[rpad(wl)]);
+    }
+}
+// bits & ~mask (mask optional)
+static void slot_rank(const uint32_t* bits, const uint32_t* mask, int32_t c, int64_t W, int64_t* csum, uint2* out,
+                      int64_t* slot_total, cudaStream_t s) {
+    const dim3 g((unsigned)std::max<int64_t>(1, (W + RANK_CHUNK - 1) / RANK_CHUNK), (unsigned)c);
+    k_rank_sums<<<g, RANK_THREADS, 0, s>>>(bits, mask, W, csum);
+    k_rank_write<<<g, RANK_THREADS, 0, s>>>(bits, mask, W, csum, out, slot_total);
+}
+
 // {bits, slot-relative popcount prefix} per bitmap word (wordoff: global exclusive scan)
 __global__ void k_pack_rank(const uint32_t* __restrict__ bits, const int64_t* __restrict__ wordoff, int64_t W,
                             int64_t n, uint2* __restrict__ out) {
@@ -222,10 +308,12 @@ __global__ void __launch_bounds__(256) k_mark_new(const int32_t* __restrict__ ds
                     jj[u] = F.j[k];
                 }
             }
+            // (measured: reading the new word too, to skip already-marked sources, is slower -- the
+            // random L2 reads cost more than the fire-and-forget atomics they save)
             uint32_t dw[FLAT_UNR];
 #pragma unroll
             for (int u = 0; u < FLAT_UNR; ++u)
-                if (p[u] >= 0) dw[u] = dstbits[(int64_t)jj[u] * W + (p[u] >> 5)];
+                dw[u] = (p[u] >= 0 && dstbits) ? dstbits[(int64_t)jj[u] * W + (p[u] >> 5)] : 0u;
 #pragma unroll
             for (int u = 0; u < FLAT_UNR; ++u) {
                 if (p[u] >= 0) {
@@ -319,13 +407,94 @@ __global__ void __launch_bounds__(256) k_relabel(const int32_t* __restrict__ dst
     }
 }
 
+// CSC of a micro-batch layer filtered from the full-batch CSC, warp-flattened: a warp takes 32
+// sources, loads their full-batch columns' extents at once, then walks all their entries as one
+// flat range (FLAT_UNR per lane in flight): keep an entry iff its dst is in the source's
+// micro-batch.  Count pass: kept entries per source.  Fill pass: kept entries in column order
+// (prefix of the keep flags within each source's run of lanes + a per-source running count).
+template <bool FILL>
+__global__ void __launch_bounds__(256) k_csc_flat(const int32_t* __restrict__ src_pos,
+                                                  const int32_t* __restrict__ src_mb, const int64_t* cnt,
+                                                  const int64_t* __restrict__ ft_indptr,
+                                                  const int32_t* __restrict__ ft_nbr,
+                                                  const uint32_t* __restrict__ dstbits, int64_t W, const RankSet R,
+                                                  int l, const int64_t* __restrict__ t_indptr,
+                                                  int32_t* __restrict__ t_idx, int32_t* __restrict__ tcnt) {
+    __shared__ FlatRows s_rows[8];
+    __shared__ int s_run[8][32];
+    const int64_t n = cnt[1];
+    const int lane = lane_id();
+    FlatRows& F = s_rows[warp_id()];
+    int* run = s_run[warp_id()];
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t u0 = gw * 32; u0 < n; u0 += nw * 32) {
+        const int64_t u = u0 + lane;
+        int d = 0;
+        if (u < n) {
+            const int32_t p = src_pos[u];
+            const int64_t b = ft_indptr[p];
+            d = (int)(ft_indptr[p + 1] - b);
+            F.fb[lane] = b;
+            F.j[lane] = src_mb[u];
+            if (FILL) F.ob[lane] = t_indptr[u];
+        }
+        run[lane] = 0;
+        const int incl = warp_incl_scan(d);
+        F.pre[lane + 1] = incl;
+        if (lane == 0) F.pre[0] = 0;
+        __syncwarp();
+        const int total = F.pre[32];
+        for (int fb = 0; fb < total; fb += 32 * FLAT_UNR) {      // warp-uniform: collectives inside
+            const int f0 = fb + lane;
+            int32_t q[FLAT_UNR];
+            int kk[FLAT_UNR];
+            uint32_t w[FLAT_UNR];
+#pragma unroll
+            for (int t = 0; t < FLAT_UNR; ++t) {
+                const int f = f0 + 32 * t;
+                q[t] = -1;
+                kk[t] = 32;
+                if (f < total) {
+                    const int k = flat_row(F, f);
+                    kk[t] = k;
+                    q[t] = ft_nbr[F.fb[k] + (f - F.pre[k])];
+                }
+            }
+#pragma unroll
+            for (int t = 0; t < FLAT_UNR; ++t)
+                w[t] = q[t] >= 0 ? dstbits[(int64_t)F.j[kk[t]] * W + (q[t] >> 5)] : 0u;
+#pragma unroll
+            for (int t = 0; t < FLAT_UNR; ++t) {
+                const bool keep = q[t] >= 0 && ((w[t] >> (q[t] & 31)) & 1u);
+                const unsigned km = __ballot_sync(0xffffffffu, keep);
+                const unsigned same = __match_any_sync(0xffffffffu, kk[t]);
+                const int before = __popc(km & same & ((1u << lane) - 1u));
+                if (FILL) {
+                    if (keep) {
+                        const int k = kk[t];
+                        t_idx[F.ob[k] + run[k] + before] = (int32_t)dst_id(R, l, F.j[k], q[t]);
+                    }
+                }
+                // the highest lane of each row's run adds the row's kept entries of this step
+                const int hi = 31 - __clz(same);
+                __syncwarp();
+                if (lane == hi && kk[t] < 32) run[kk[t]] += __popc(km & same);
+                __syncwarp();
+            }
+        }
+        if (!FILL && u < n) tcnt[u] = run[lane];
+        __syncwarp();
+    }
+}
+
 __global__ void k_popc(const uint32_t* __restrict__ newbits, int64_t n, int32_t* __restrict__ wc) {
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
         wc[i] = __popc(newbits[i]);
 }
 
 // single CTA: per micro-batch src counts and offsets; checks capacities
-__global__ void k_counts(const int64_t* __restrict__ mb_dst_off, const int64_t* __restrict__ wordoff, int64_t W,
+__global__ void k_counts(const int64_t* __restrict__ mb_dst_off, const int64_t* __restrict__ slot_total,
                          int32_t c, int64_t* __restrict__ mb_src_off, int64_t* cnt, int64_t cap_src, int64_t cap_e,
                          int64_t* next_cnt, int* dev_err) {
     __shared__ int64_t s_warp[33];
@@ -335,7 +504,7 @@ __global__ void k_counts(const int64_t* __restrict__ mb_dst_off, const int64_t* 
     for (int j0 = 0; j0 < c; j0 += blockDim.x) {
         const int j = j0 + threadIdx.x;
         int64_t nn = 0;                                 // new sources of micro-batch j
-        if (j < c) nn = wordoff[(int64_t)(j + 1) * W] - wordoff[(int64_t)j * W];
+        if (j < c) nn = slot_total[j];
         int64_t tot;
         const int64_t ex = block_excl_scan(nn, s_warp, &tot);
         if (j < c) mb_src_off[j] = s_base + ex;         // offset of j's new sources after the dst prefix
@@ -353,18 +522,19 @@ __global__ void k_counts(const int64_t* __restrict__ mb_dst_off, const int64_t* 
     }
 }
 
-__global__ void k_emit_new(const uint32_t* __restrict__ newbits, int64_t W, int32_t c, const int64_t* n_dst_tot,
-                           const int64_t* __restrict__ wordoff, const int64_t* __restrict__ mb_dst_off,
+__global__ void k_emit_new(const uint2* __restrict__ nrank, int64_t W, int32_t c, const int64_t* n_dst_tot,
+                           const int64_t* __restrict__ mb_dst_off,
                            const int64_t* __restrict__ mb_src_off, const int32_t* __restrict__ fsrc_gid,
                            int32_t* __restrict__ src_pos, int32_t* __restrict__ src_gid, int32_t* __restrict__ src_mb,
                            int64_t cap_src) {
     const int64_t n = (int64_t)c * W;
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-        uint32_t bits = newbits[i];
+        const uint2 r = nrank[i];
+        uint32_t bits = r.x;
         if (!bits) continue;
         const int j = (int)(i / W);
         const int64_t w = i - (int64_t)j * W;
-        int64_t s = n_dst_tot[0] + mb_src_off[j] + (wordoff[i] - wordoff[(int64_t)j * W]);
+        int64_t s = n_dst_tot[0] + mb_src_off[j] + r.y;
         (void)mb_dst_off;
         while (bits) {
             const int b = __ffs(bits) - 1;
@@ -515,31 +685,29 @@ void extract_group(betty_ctx* ctx, const ExtractArgs& a, cudaStream_t s) {
             otab = B.order_tab;
         }
         // rows: degree of each dst row in the full batch -> local indptr
-        k_deg<<<grid_for(ctx, cap_d, 256), 256, 0, s>>>(dst_pos, F.indptr, B.cnt, a.sc.deg);
-        scan_i64(ctx, a.sc.deg, B.indptr, B.cnt + 0, 0, cap_d, B.cnt + 2, s);
+        scan_deg(ctx, dst_pos, F.indptr, B.indptr, B.cnt + 0, cap_d, B.cnt + 2, s);
         // dedupe: dst bitmap + position map, then new-source bitmap
         k_mark_dst<<<grid_for(ctx, cap_d, 256), 256, 0, s>>>(dst_pos, row_mb, B.cnt, a.sc.dstbits, W);
         const int g_rows = grid_for(ctx, cap_d, 256);       // 32 rows per warp
         unsigned* ctr = ctx->L().counters + CTR_EXTRACT;
         cudaMemsetAsync(ctr, 0, sizeof(unsigned), s);
-        k_mark_new<<<g_rows, 256, 0, s>>>(dst_pos, row_mb, B.cnt, F.indptr, F.nbr, a.sc.dstbits, a.sc.newbits, W, otab,
-                                          ctr);
+        // mark_nocheck: mark every neighbour (no dst lookup per edge); the dst rows are masked out of
+        // the bitmap words by the rank pass instead
+        static const bool mark_nocheck = getenv("BETTY_MARK_NOCHECK") && atoi(getenv("BETTY_MARK_NOCHECK"));
+        k_mark_new<<<g_rows, 256, 0, s>>>(dst_pos, row_mb, B.cnt, F.indptr, F.nbr, mark_nocheck ? nullptr : a.sc.dstbits,
+                                          a.sc.newbits, W, otab, ctr);
         // ascending order of new sources = popcount scan over the bitmap words
-        k_popc<<<grid_for(ctx, cW, 256), 256, 0, s>>>(a.sc.newbits, cW, a.sc.wordcnt);
-        scan_i32(ctx, a.sc.wordcnt, a.sc.wordoff, nullptr, cW, 0, nullptr, s);
-        k_counts<<<1, 1024, 0, s>>>(dst_off, a.sc.wordoff, W, c, B.mb_src_off, B.cnt, cap_s, cap_e,
+        int64_t* csum = a.sc.wordoff;                   // chunk sums, then slot totals at the end
+        int64_t* slot_tot = a.sc.wordoff + (int64_t)c * ((W + RANK_CHUNK - 1) / RANK_CHUNK + 1);
+        slot_rank(a.sc.newbits, mark_nocheck ? a.sc.dstbits : nullptr, c, W, csum, a.sc.nrank[l], slot_tot, s);
+        k_counts<<<1, 1024, 0, s>>>(dst_off, slot_tot, c, B.mb_src_off, B.cnt, cap_s, cap_e,
                                     l > 0 ? a.layers[l - 1].cnt : nullptr, ctx->dev_err);
         k_emit_dst<<<grid_for(ctx, cap_d, 256), 256, 0, s>>>(dst_pos, row_mb, B.cnt, dst_off, B.mb_src_off,
                                                              F.src_gid, B.src_pos, B.src_gid, B.src_mb, cap_s);
-        k_emit_new<<<grid_for(ctx, cW, 256), 256, 0, s>>>(a.sc.newbits, W, c, B.cnt, a.sc.wordoff, dst_off, B.mb_src_off,
+        k_emit_new<<<grid_for(ctx, cW, 256), 256, 0, s>>>(a.sc.nrank[l], W, c, B.cnt, dst_off, B.mb_src_off,
                                                           F.src_gid, B.src_pos, B.src_gid, B.src_mb, cap_s);
         // rank structures of this layer (and of the outputs at the top layer)
-        k_pack_rank<<<grid_for(ctx, cW, 256), 256, 0, s>>>(a.sc.newbits, a.sc.wordoff, W, cW, a.sc.nrank[l]);
-        if (l == a.L - 1) {
-            k_popc<<<grid_for(ctx, cW, 256), 256, 0, s>>>(a.sc.dstbits, cW, a.sc.wordcnt);
-            scan_i32(ctx, a.sc.wordcnt, a.sc.wordoff, nullptr, cW, 0, nullptr, s);
-            k_pack_rank<<<grid_for(ctx, cW, 256), 256, 0, s>>>(a.sc.dstbits, a.sc.wordoff, W, cW, a.sc.drank_top);
-        }
+        if (l == a.L - 1) slot_rank(a.sc.dstbits, nullptr, c, W, csum, a.sc.drank_top, nullptr, s);
         RankSet R{};
         R.L = a.L;
         for (int q = 0; q < a.L; ++q) {
@@ -556,11 +724,12 @@ void extract_group(betty_ctx* ctx, const ExtractArgs& a, cudaStream_t s) {
                                          F.src_gid, B.egid, otab, ctr + 1);
         const bool want_csc = B.t_indptr && (a.csc_mask >> l & 1);
         if (want_csc && F.t_indptr) {           // from the full-batch CSC (needs the dst bitmap + map)
-            k_csc_count<<<grid_for(ctx, cap_s, 256), 256, 0, s>>>(B.src_pos, B.src_mb, B.cnt, F.t_indptr, F.t_nbr,
-                                                                  a.sc.dstbits, W, a.sc.tcnt);
+            const int g_src = grid_for(ctx, (cap_s + 31) / 32 * 32, 256);
+            k_csc_flat<false><<<g_src, 256, 0, s>>>(B.src_pos, B.src_mb, B.cnt, F.t_indptr, F.t_nbr, a.sc.dstbits, W,
+                                                    R, l, nullptr, nullptr, a.sc.tcnt);
             scan_i32(ctx, a.sc.tcnt, B.t_indptr, B.cnt + 1, 0, cap_s, nullptr, s);
-            k_csc_fill<<<grid_for(ctx, cap_s, 256), 256, 0, s>>>(B.src_pos, B.src_mb, B.cnt, F.t_indptr, F.t_nbr,
-                                                                 a.sc.dstbits, W, R, l, B.t_indptr, B.t_indices);
+            k_csc_flat<true><<<g_src, 256, 0, s>>>(B.src_pos, B.src_mb, B.cnt, F.t_indptr, F.t_nbr, a.sc.dstbits, W,
+                                                   R, l, B.t_indptr, B.t_indices, nullptr);
             if (l + 1 < a.L)                    // below the top layer dst ids are not monotone in position
                 segsort_i32(ctx, B.t_indptr, B.t_indices, B.cnt + 1, 0, cap_s, s);
         }

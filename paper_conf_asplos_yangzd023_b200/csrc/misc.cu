@@ -29,6 +29,7 @@ __global__ void __launch_bounds__(256) k_loss(const float* __restrict__ logits, 
     const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
     double wl = 0.0;
     for (int64_t v = gw; v < nd; v += nw) {
+        const int32_t y = labels[gid[v]];               // independent of the logits: issued first
         float x[LOSS_MAXT];
         float mx = -INFINITY;
 #pragma unroll
@@ -46,7 +47,6 @@ __global__ void __launch_bounds__(256) k_loss(const float* __restrict__ logits, 
         }
         se = warp_sum(se);
         const float lse = mx + logf(se);
-        const int32_t y = labels[gid[v]];
         float xy = 0.f;
 #pragma unroll
         for (int t = 0; t < LOSS_MAXT; ++t) {
@@ -73,20 +73,30 @@ __global__ void __launch_bounds__(256) k_loss(const float* __restrict__ logits, 
         s_last = (atomicAdd(&ctr[0], 1u) == gridDim.x - 1);
     }
     __syncthreads();
-    if (s_last && threadIdx.x == 0) {
+    if (s_last) {                       // fixed-order reduction of the partials by the last CTA
         __threadfence();
-        double tot = 0.0;
-        for (unsigned i = 0; i < gridDim.x; ++i) tot += ((volatile double*)partials)[i];
-        loss_accum[0] += (float)tot;
-        ctr[0] = 0;
+        double t = 0.0;
+        for (unsigned i = threadIdx.x; i < gridDim.x; i += blockDim.x) t += ((volatile double*)partials)[i];
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) t += __shfl_xor_sync(0xffffffffu, t, o);
+        __syncthreads();
+        if (lane == 0) s_w[warp_id()] = t;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            double tot = 0.0;
+            for (int i = 0; i < (int)(blockDim.x >> 5); ++i) tot += s_w[i];
+            loss_accum[0] += (float)tot;
+            ctr[0] = 0;
+        }
     }
 }
 
 void loss_ce(betty_ctx* c, const float* logits, int64_t ldl, const int32_t* labels, const int32_t* gid,
              const int64_t* cnt, int64_t rows_cap, int C, float scale, float* dS, int64_t ldds, void* dS_act,
              bool act_bf16, int64_t ld_act, float* loss_accum, cudaStream_t s) {
-    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((rows_cap * 32 + 255) / 256, 512));
-    double* partials = (double*)(c->L().counters + 64);   // 512 doubles after the counters
+    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((rows_cap * 32 + 255) / 256,
+                                                                 std::min(2048, c->num_sms * 8)));
+    double* partials = (double*)(c->L().counters + 64);   // 2048 doubles after the counters
     if (act_bf16)
         k_loss<__nv_bfloat16><<<grid, 256, 0, s>>>(logits, ldl, labels, gid, cnt, C, scale, dS, ldds,
                                                    (__nv_bfloat16*)dS_act, ld_act, partials, c->L().counters + CTR_LOSS,

@@ -24,8 +24,25 @@ __device__ __forceinline__ void st_release(unsigned long long* p, unsigned long 
     asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
-template <typename Tin>
-__global__ void __launch_bounds__(SCAN_THREADS) k_scan(const Tin* __restrict__ in, int64_t* __restrict__ out,
+// element loaders of the scan: plain values, popcounts of bitmap words, degrees of gathered rows
+template <typename Tin> struct LdPlain {
+    const Tin* in;
+    __device__ __forceinline__ int64_t operator()(int64_t i) const { return (int64_t)in[i]; }
+};
+struct LdPopc {
+    const uint32_t* bits;
+    __device__ __forceinline__ int64_t operator()(int64_t i) const { return __popc(bits[i]); }
+};
+struct LdDeg {
+    const int32_t* rows; const int64_t* indptr;
+    __device__ __forceinline__ int64_t operator()(int64_t i) const {
+        const int32_t p = rows[i];
+        return indptr[p + 1] - indptr[p];
+    }
+};
+
+template <typename Ld>
+__global__ void __launch_bounds__(SCAN_THREADS) k_scan(const Ld in, int64_t* __restrict__ out,
                                                        const int64_t* n_dev, int64_t n_fixed, int64_t* total_dev,
                                                        unsigned long long* status, unsigned* ctr) {
     __shared__ int64_t s_warp[SCAN_THREADS / 32 + 1];
@@ -44,7 +61,7 @@ __global__ void __launch_bounds__(SCAN_THREADS) k_scan(const Tin* __restrict__ i
 #pragma unroll
         for (int i = 0; i < SCAN_ITEMS; ++i) {
             const int64_t idx = base + i;
-            v[i] = idx < n ? (int64_t)in[idx] : 0;
+            v[i] = idx < n ? in(idx) : 0;
             sum += v[i];
         }
         int64_t agg;
@@ -125,24 +142,31 @@ void ensure_scan_scratch(betty_ctx* c, int64_t n_cap, cudaStream_t s) {
     }
 }
 
-template <typename Tin>
-static void scan_impl(betty_ctx* c, const Tin* in, int64_t* out, const int64_t* n_dev, int64_t n_fixed, int64_t n_cap,
+template <typename Ld>
+static void scan_impl(betty_ctx* c, const Ld in, int64_t* out, const int64_t* n_dev, int64_t n_fixed, int64_t n_cap,
                       int64_t* total_dev, cudaStream_t s) {
     if (!n_dev) n_cap = n_fixed;
     ensure_scan_scratch(c, n_cap, s);
     int64_t tiles = (n_cap + SCAN_TILE - 1) / SCAN_TILE;
     int grid = (int)std::min<int64_t>(std::max<int64_t>(tiles, 1), (int64_t)c->num_sms * 2);
-    k_scan<Tin><<<grid, SCAN_THREADS, 0, s>>>(in, out, n_dev, n_fixed, total_dev, c->L().scan_status,
-                                              c->L().counters + CTR_SCAN);
+    k_scan<Ld><<<grid, SCAN_THREADS, 0, s>>>(in, out, n_dev, n_fixed, total_dev, c->L().scan_status,
+                                             c->L().counters + CTR_SCAN);
 }
 
 void scan_i64(betty_ctx* c, const int64_t* in, int64_t* out, const int64_t* n_dev, int64_t n_fixed, int64_t n_cap,
               int64_t* total_dev, cudaStream_t s) {
-    scan_impl<int64_t>(c, in, out, n_dev, n_fixed, n_cap, total_dev, s);
+    scan_impl(c, LdPlain<int64_t>{in}, out, n_dev, n_fixed, n_cap, total_dev, s);
 }
 void scan_i32(betty_ctx* c, const int32_t* in, int64_t* out, const int64_t* n_dev, int64_t n_fixed, int64_t n_cap,
               int64_t* total_dev, cudaStream_t s) {
-    scan_impl<int32_t>(c, in, out, n_dev, n_fixed, n_cap, total_dev, s);
+    scan_impl(c, LdPlain<int32_t>{in}, out, n_dev, n_fixed, n_cap, total_dev, s);
+}
+void scan_popc(betty_ctx* c, const uint32_t* bits, int64_t* out, int64_t n, cudaStream_t s) {
+    scan_impl(c, LdPopc{bits}, out, nullptr, n, 0, nullptr, s);
+}
+void scan_deg(betty_ctx* c, const int32_t* rows, const int64_t* indptr, int64_t* out, const int64_t* n_dev,
+              int64_t n_cap, int64_t* total_dev, cudaStream_t s) {
+    scan_impl(c, LdDeg{rows, indptr}, out, n_dev, 0, n_cap, total_dev, s);
 }
 
 // ---------------------------------------------------------------- memset
