@@ -58,6 +58,7 @@ def parse():
     p.add_argument("--ref-sample-outputs", type=int, default=1024, help="--impl reference per-step sample")
     p.add_argument("--scale", type=float, default=1.0, help="shrink the graph (debug only)")
     p.add_argument("--json-out", default=None)
+    p.add_argument("--feat-align", type=int, default=256, help="feature-table row alignment in bytes (0: 16)")
     return p.parse_args()
 
 
@@ -339,6 +340,7 @@ def main():
     feats = torch.as_tensor(ds.feats).to(device)
     if args.mode == "bf16":
         feats = feats.to(torch.bfloat16).contiguous()       # bf16 feature table (reading #17)
+    feats = pad_rows(feats, args.feat_align)
     labels = torch.as_tensor(ds.labels).to(device)
     model = B.Model(cfg.dims, cfg.aggr, args.mode, args.mode)
     params = torch.as_tensor(synth_params(cfg)).to(device)
@@ -498,6 +500,22 @@ def main():
     plan.free()
     if ws > 1:
         dist.destroy_process_group()
+
+
+def pad_rows(t, align: int):
+    """Feature table with rows padded to a multiple of `align` bytes (zeros): random row gathers of
+    256-byte-aligned rows run closer to the HBM ceiling than 208-byte rows straddling bursts
+    (tools/micro/gather_ceiling.cu).  The pad columns are never read."""
+    import torch
+    if align <= 0:
+        return t
+    per = max(1, align // t.element_size())
+    ld = (t.shape[1] + per - 1) // per * per
+    if ld == t.shape[1]:
+        return t
+    out = torch.zeros((t.shape[0], ld), dtype=t.dtype, device=t.device)
+    out[:, :t.shape[1]] = t
+    return out
 
 
 def synth_params(cfg):

@@ -1,0 +1,156 @@
+"""Parity at BASELINE.json's full size, in the launch configuration bench.py
+times: C3 (products-shaped, 2.45 M nodes, 2-layer SAGE-mean, fanout (10, 25),
+196,615 outputs), K = 32 micro-batches of the multilevel REG partition, all in
+one launch group, bf16 GEMM mode, CUDA-graph replay.
+
+* REG (a1): the whole output block's REG, bit-exact against the oracle.
+* Extraction (a2): every micro-batch of the bench's launch group, bit-exact
+  against the oracle's micro-batch blocks mapped into the group layout
+  (DESIGN.md §3 row G) -- CSR, src_pos / src_gid and the top layer's CSC.
+* Numerics (a3-a6): a sampled micro-batch (16 outputs) through the fused step
+  on the full-size graph and feature table against the float64 oracle, and
+  Betty's invariant at full size on the GPU itself (the K = 32 step's
+  gradient equals the K = 1 step's).
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import synth
+from tests.helpers import assert_close
+
+pytestmark = pytest.mark.gpu
+
+K = 32
+
+
+@pytest.fixture(scope="module")
+def B():
+    import paper_conf_asplos_yangzd023_b200 as B
+    assert torch.cuda.is_available()
+    return B
+
+
+@pytest.fixture(scope="module")
+def ctx(B):
+    return B.betty_ctx_create(0)
+
+
+@pytest.fixture(scope="module")
+def c3(B, ctx):
+    cfg = synth.CONFIGS["C3"]
+    ds = synth.make(cfg)
+    dev = B.blocks_to_device(ds.blocks)
+    ip, col, w = B.betty_reg_build(ctx, dev[-1])
+    reg = (ip.cpu().numpy(), col.cpu().numpy(), w.cpu().numpy())
+    part = B.betty_reg_partition(*reg, K, method="multilevel")
+    return cfg, ds, dev, reg, part
+
+
+def test_reg_full_size(c3):
+    cfg, ds, dev, reg, part = c3
+    rp, rc, rw = oracle.reg(ds.blocks[-1].n_src, ds.blocks[-1].indptr, ds.blocks[-1].nbr_pos)
+    np.testing.assert_array_equal(reg[0], rp)
+    np.testing.assert_array_equal(reg[1], rc)
+    np.testing.assert_array_equal(reg[2], rw)
+
+
+def _segments(indptr, rows):
+    """Concatenated CSR segments of `rows` (vectorised gather index)."""
+    b, e = indptr[rows], indptr[rows + 1]
+    lens = e - b
+    if lens.sum() == 0:
+        return np.zeros(0, np.int64), lens
+    starts = np.repeat(b - np.concatenate([[0], np.cumsum(lens)[:-1]]), lens)
+    return starts + np.arange(lens.sum()), lens
+
+
+def test_extraction_full_size(B, ctx, c3):
+    """The bench's launch group (all 32 micro-batches) == the oracle's micro-batches, bit-exact."""
+    cfg, ds, dev, reg, part = c3
+    model = B.Model(cfg.dims, cfg.aggr, "bf16", "bf16")
+    plan = B.betty_plan_create(ctx, model, dev, torch.as_tensor(part).cuda(), K, list(range(K)), group=0,
+                               flags=B.PLAN_GRAPH)
+    got = [{k: (v.cpu().numpy() if isinstance(v, torch.Tensor) else v) for k, v in vars(b).items()}
+           for b in plan.group_blocks(0)]
+    mbs = [oracle.extract(ds.blocks, part, K, k) for k in range(K)]
+    L = cfg.L
+    # group ids of every micro-batch's local ids, layer by layer from the top (DESIGN.md §3 row G)
+    n_out = [mb[L - 1].n_dst for mb in mbs]
+    out_off = np.concatenate([[0], np.cumsum(n_out)])
+    dst_map = [out_off[j] + np.arange(n_out[j]) for j in range(K)]      # group dst row of each local dst row
+    for l in range(L - 1, -1, -1):
+        g = got[l]
+        n_dst_g = sum(len(m) for m in dst_map)
+        new = [mbs[j][l].n_src - mbs[j][l].n_dst for j in range(K)]
+        new_off = n_dst_g + np.concatenate([[0], np.cumsum(new)])
+        src_map = [np.concatenate([dst_map[j], new_off[j] + np.arange(new[j])]).astype(np.int64) for j in range(K)]
+        assert g["n_dst"] == n_dst_g and g["n_src"] == new_off[-1], l
+        assert len(g["indices"]) == sum(mb[l].n_edges for mb in mbs), l
+        for j in range(K):
+            m = mbs[j][l]
+            rows = dst_map[j]
+            gi, glen = _segments(g["indptr"], rows)
+            np.testing.assert_array_equal(glen, np.diff(m.indptr), err_msg=f"layer {l} mb {j} degrees")
+            np.testing.assert_array_equal(g["indices"][gi], src_map[j][m.indices], err_msg=f"layer {l} mb {j} idx")
+            np.testing.assert_array_equal(g["src_pos"][src_map[j]], m.src_pos, err_msg=f"layer {l} mb {j} src_pos")
+            np.testing.assert_array_equal(g["src_gid"][src_map[j]], m.src_gid, err_msg=f"layer {l} mb {j} src_gid")
+            if g.get("t_indptr") is not None and l == L - 1:
+                ci, clen = _segments(g["t_indptr"], src_map[j])
+                np.testing.assert_array_equal(clen, np.diff(m.t_indptr), err_msg=f"mb {j} CSC degrees")
+                np.testing.assert_array_equal(g["t_indices"][ci], dst_map[j][m.t_indices], err_msg=f"mb {j} CSC")
+        dst_map = src_map
+    plan.free()
+
+
+def test_sampled_micro_batch_full_size(B, ctx, c3):
+    """16 outputs of micro-batch 0 as their own micro-batch, through the fused step on the full-size
+    graph and feature table, against the float64 oracle (bf16 tolerance 2e-2, fp32 1e-5)."""
+    cfg, ds, dev, reg, part = c3
+    idx = np.nonzero(part == 0)[0][:16]
+    p2 = np.ones(cfg.n_out, np.int32)
+    p2[idx] = 0
+    params = synth.init_params(cfg.dims, cfg.aggr, seed=cfg.seeds["init"])
+    og, ol = oracle.step(cfg.dims, cfg.aggr, True, ds.blocks, p2, 2, [0], params, ds.feats, ds.labels,
+                         1.0 / cfg.n_out)
+    model = B.Model(cfg.dims, cfg.aggr, "bf16", "bf16")
+    plan = B.betty_plan_create(ctx, model, dev, torch.as_tensor(p2).cuda(), 2, [0], group=0,
+                               flags=B.PLAN_GRAPH | B.PLAN_REG)
+    P = torch.as_tensor(params).cuda()
+    X = torch.as_tensor(ds.feats).cuda().to(torch.bfloat16).contiguous()
+    Y = torch.as_tensor(ds.labels).cuda()
+    for rep in range(2):
+        grad = torch.zeros_like(P)
+        loss = torch.zeros(1, device="cuda")
+        B.betty_step(ctx, plan, P, X, Y, 1.0 / cfg.n_out, grad, loss)
+        B.betty_sync_check(ctx)
+        assert_close(grad.cpu().numpy(), og, 2e-2, f"grad rep {rep}")
+        assert loss.item() == pytest.approx(ol, rel=2e-2)
+    plan.free()
+
+
+@pytest.mark.parametrize("mode,rtol", [("bf16", 2e-2), ("fp32", 1e-5)])
+def test_invariant_full_size(B, ctx, c3, mode, rtol):
+    """Betty's defining invariant at full size on the GPU: the gradient and loss of the K = 32 step
+    (bench configuration) equal the full-batch (K = 1) step's."""
+    cfg, ds, dev, reg, part = c3
+    params = synth.init_params(cfg.dims, cfg.aggr, seed=cfg.seeds["init"])
+    P = torch.as_tensor(params).cuda()
+    X = torch.as_tensor(ds.feats).cuda()
+    if mode == "bf16":
+        X = X.to(torch.bfloat16).contiguous()
+    Y = torch.as_tensor(ds.labels).cuda()
+    model = B.Model(cfg.dims, cfg.aggr, mode, mode)
+    res = []
+    for k, p in ((K, part), (1, np.zeros(cfg.n_out, np.int32))):
+        plan = B.betty_plan_create(ctx, model, dev, torch.as_tensor(p).cuda(), k, list(range(k)), group=0,
+                                   flags=B.PLAN_GRAPH)
+        grad = torch.zeros_like(P)
+        loss = torch.zeros(1, device="cuda")
+        B.betty_step(ctx, plan, P, X, Y, 1.0 / cfg.n_out, grad, loss)
+        B.betty_sync_check(ctx)
+        res.append((grad.cpu().numpy().astype(np.float64), loss.item()))
+        plan.free()
+    assert_close(res[0][0], res[1][0], rtol, "sum of micro-batch gradients vs full batch")
+    assert res[0][1] == pytest.approx(res[1][1], rel=rtol)

@@ -28,6 +28,7 @@ def main():
     p.add_argument("--steps", type=int, default=1)
     p.add_argument("--scale", type=float, default=1.0)
     p.add_argument("--group", type=int, default=0)
+    p.add_argument("--feat-align", type=int, default=256)
     a = p.parse_args()
     cfg = synth.CONFIGS[a.config]
     if a.scale != 1.0:
@@ -41,6 +42,9 @@ def main():
     feats = torch.as_tensor(ds.feats).cuda()
     if a.mode == "bf16":
         feats = feats.to(torch.bfloat16).contiguous()
+    sys.path.insert(0, ROOT)
+    from bench import pad_rows
+    feats = pad_rows(feats, a.feat_align)
     labels = torch.as_tensor(ds.labels).cuda()
     model = B.Model(cfg.dims, cfg.aggr, a.mode, a.mode)
     params = torch.as_tensor(synth.init_params(cfg.dims, cfg.aggr, seed=cfg.seeds["init"])).cuda()
