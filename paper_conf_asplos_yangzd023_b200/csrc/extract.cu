@@ -388,9 +388,34 @@ __global__ void __launch_bounds__(256) k_relabel(const int32_t* __restrict__ dst
                     if (egid) gid[u] = fsrc_gid[p[u]];
                 }
             }
+            // src_id level by level for all FLAT_UNR edges at once: each level's rank-word loads are
+            // issued together (independent chains), not one edge's whole chain after another
+            bool done[FLAT_UNR];
+#pragma unroll
+            for (int u = 0; u < FLAT_UNR; ++u) {
+                done[u] = p[u] < 0;
+                if (!done[u] && (nr[u].x >> (p[u] & 31) & 1u)) {
+                    id[u] = (int32_t)(R.cnt[l][0] + R.off[l][F.j[kk[u]]] + rank_in(nr[u], p[u]));
+                    done[u] = true;
+                }
+            }
+            for (int q = l + 1; q < R.L; ++q) {
+#pragma unroll
+                for (int u = 0; u < FLAT_UNR; ++u)
+                    if (!done[u]) nr[u] = R.nr[q][(int64_t)F.j[kk[u]] * R.W[q] + (p[u] >> 5)];
+#pragma unroll
+                for (int u = 0; u < FLAT_UNR; ++u)
+                    if (!done[u] && (nr[u].x >> (p[u] & 31) & 1u)) {
+                        id[u] = (int32_t)(R.cnt[q][0] + R.off[q][F.j[kk[u]]] + rank_in(nr[u], p[u]));
+                        done[u] = true;
+                    }
+            }
 #pragma unroll
             for (int u = 0; u < FLAT_UNR; ++u)
-                if (p[u] >= 0) id[u] = (int32_t)src_id(R, l, F.j[kk[u]], p[u], nr[u]);
+                if (!done[u]) nr[u] = R.dr[(int64_t)F.j[kk[u]] * R.Wt + (p[u] >> 5)];
+#pragma unroll
+            for (int u = 0; u < FLAT_UNR; ++u)
+                if (!done[u]) id[u] = (int32_t)(R.top_off[F.j[kk[u]]] + rank_in(nr[u], p[u]));
 #pragma unroll
             for (int u = 0; u < FLAT_UNR; ++u) {
                 if (p[u] >= 0) {
