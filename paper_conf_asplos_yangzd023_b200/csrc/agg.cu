@@ -1,3 +1,4 @@
+#include <cstdio>
 #include <cmath>
 #include <cstdlib>
 // agg.cu -- a3/a5: GraphSAGE aggregation forward and backward (HBM-bound
@@ -275,12 +276,12 @@ __global__ void __launch_bounds__(256) k_agg_mean_xa(const Tin* __restrict__ X, 
 // Same semantics as k_agg_pool / k_route_pool (reading #14: max of ReLU(Zp) over the row, empty
 // row -> 0, ties -> first in row order; the gradient goes to that argmax), but every lane owns
 // T 4-column groups and a batch of 4 edges' rows is in flight at once.
-template <typename Tin, typename Tout, int T>
+template <typename Tin, typename Tout, int T, bool POS8>
 __global__ void __launch_bounds__(256) k_agg_pool_v(const Tin* __restrict__ X, int64_t ldx,
                                                     const int32_t* __restrict__ xrow, const float* __restrict__ Zp,
                                                     int64_t ldz, const int64_t* __restrict__ indptr,
                                                     const int32_t* __restrict__ idx, const int64_t* cnt, int Fi, int Fp,
-                                                    Tout* __restrict__ XA, int64_t ldxa, int32_t* __restrict__ arg,
+                                                    Tout* __restrict__ XA, int64_t ldxa, void* __restrict__ argv,
                                                     int64_t ldarg) {
     const int64_t nd = cnt[0];
     const int lane = lane_id();
@@ -314,13 +315,14 @@ __global__ void __launch_bounds__(256) k_agg_pool_v(const Tin* __restrict__ X, i
 #pragma unroll
                 for (int k = 0; k < 4; ++k) {
                     if (j0 + k >= n) break;
+                    const int32_t who = POS8 ? (int32_t)(e0 - b) + j0 + k : u[k];   // position in the row / id
 #pragma unroll
                     for (int t = 0; t < T; ++t) {
                         const float zz[4] = {fmaxf(z[k][t].x, 0.f), fmaxf(z[k][t].y, 0.f), fmaxf(z[k][t].z, 0.f),
                                              fmaxf(z[k][t].w, 0.f)};
 #pragma unroll
                         for (int q = 0; q < 4; ++q)
-                            if (am[t][q] < 0 || zz[q] > best[t][q]) { best[t][q] = zz[q]; am[t][q] = u[k]; }
+                            if (am[t][q] < 0 || zz[q] > best[t][q]) { best[t][q] = zz[q]; am[t][q] = who; }
                     }
                 }
             }
@@ -337,17 +339,25 @@ __global__ void __launch_bounds__(256) k_agg_pool_v(const Tin* __restrict__ X, i
                 if (col < Fi) {
                     st_act(o + col, ld_act(xv + col));
                     st_act(o + Fp + col, best[t][q]);
-                    arg[v * ldarg + col] = am[t][q];
+                    if (!POS8) ((int32_t*)argv)[v * ldarg + col] = am[t][q];
                 }
+            }
+            if (POS8) {               // 4 byte positions per group (255: empty row)
+                uint32_t w = 0;
+#pragma unroll
+                for (int q = 0; q < 4; ++q) w |= (uint32_t)(am[t][q] < 0 ? 255 : am[t][q]) << (8 * q);
+                *(uint32_t*)((uint8_t*)argv + v * ldarg + 4 * g) = w;
             }
         }
         for (int col = Fi + lane; col < Fp; col += 32) { st_act(o + col, 0.f); st_act(o + Fp + col, 0.f); }
         for (int col = 2 * Fp + lane; col < ldxa; col += 32) st_act(o + col, col == 2 * Fp ? 1.f : 0.f);
     }
 }
-template <typename Tout, int T>
+template <typename Tout, int T, bool POS8>
 __global__ void __launch_bounds__(256) k_route_pool_v(const float* __restrict__ dXA, int64_t ldd,
-                                                      const int32_t* __restrict__ arg, int64_t ldarg,
+                                                      const void* __restrict__ argv, int64_t ldarg,
+                                                      const int64_t* __restrict__ indptr,
+                                                      const int32_t* __restrict__ idx,
                                                       const int64_t* __restrict__ t_indptr,
                                                       const int32_t* __restrict__ t_idx, const int64_t* cnt, int Fi,
                                                       int Fp, const float* __restrict__ Zp, int64_t ldz,
@@ -370,15 +380,42 @@ __global__ void __launch_bounds__(256) k_route_pool_v(const float* __restrict__ 
             for (int j0 = 0; j0 < n; j0 += 4) {
                 int32_t v[4];
                 int4 a[4][T];
+                int32_t key[4];                 // what an argmax entry must equal: u, or u's position in v's row
 #pragma unroll
                 for (int k = 0; k < 4; ++k) v[k] = __shfl_sync(0xffffffffu, my, (j0 + k) & 31);
+                if (POS8) {
+                    int64_t rb[4], re[4];
+#pragma unroll
+                    for (int k = 0; k < 4; ++k) {
+                        rb[k] = j0 + k < n ? __ldg(indptr + v[k]) : 0;
+                        re[k] = j0 + k < n ? __ldg(indptr + v[k] + 1) : 0;
+                    }
+#pragma unroll
+                    for (int k = 0; k < 4; ++k) {
+                        key[k] = -2;
+                        for (int64_t e = rb[k]; e < re[k]; ++e)
+                            if (__ldg(idx + e) == (int32_t)u) { key[k] = (int32_t)(e - rb[k]); break; }
+                    }
+                } else {
+#pragma unroll
+                    for (int k = 0; k < 4; ++k) key[k] = (int32_t)u;
+                }
 #pragma unroll
                 for (int k = 0; k < 4; ++k)
 #pragma unroll
                     for (int t = 0; t < T; ++t) {
                         const int g = lane + 32 * t;
-                        a[k][t] = (j0 + k < n && g < NG) ? __ldg((const int4*)(arg + (int64_t)v[k] * ldarg) + g)
-                                                         : make_int4(-1, -1, -1, -1);
+                        if (j0 + k < n && g < NG) {
+                            if (POS8) {
+                                const uint32_t w = __ldg((const uint32_t*)((const uint8_t*)argv + (int64_t)v[k] * ldarg) + g);
+                                a[k][t] = make_int4((int)(w & 255u), (int)(w >> 8 & 255u), (int)(w >> 16 & 255u),
+                                                    (int)(w >> 24));
+                            } else {
+                                a[k][t] = __ldg((const int4*)((const int32_t*)argv + (int64_t)v[k] * ldarg) + g);
+                            }
+                        } else {
+                            a[k][t] = make_int4(-1, -1, -1, -1);
+                        }
                     }
                 float4 d[4][T];
 #pragma unroll
@@ -386,8 +423,8 @@ __global__ void __launch_bounds__(256) k_route_pool_v(const float* __restrict__ 
 #pragma unroll
                     for (int t = 0; t < T; ++t) {
                         const int g = lane + 32 * t;
-                        const bool hit = a[k][t].x == (int32_t)u || a[k][t].y == (int32_t)u || a[k][t].z == (int32_t)u ||
-                                         a[k][t].w == (int32_t)u;
+                        const bool hit = a[k][t].x == key[k] || a[k][t].y == key[k] || a[k][t].z == key[k] ||
+                                         a[k][t].w == key[k];
                         d[k][t] = hit ? __ldg((const float4*)(dXA + (int64_t)v[k] * ldd + Fp) + g)
                                       : make_float4(0.f, 0.f, 0.f, 0.f);
                     }
@@ -395,10 +432,10 @@ __global__ void __launch_bounds__(256) k_route_pool_v(const float* __restrict__ 
                 for (int k = 0; k < 4; ++k)
 #pragma unroll
                     for (int t = 0; t < T; ++t) {
-                        if (a[k][t].x == (int32_t)u) acc[t][0] += d[k][t].x;
-                        if (a[k][t].y == (int32_t)u) acc[t][1] += d[k][t].y;
-                        if (a[k][t].z == (int32_t)u) acc[t][2] += d[k][t].z;
-                        if (a[k][t].w == (int32_t)u) acc[t][3] += d[k][t].w;
+                        if (a[k][t].x == key[k]) acc[t][0] += d[k][t].x;
+                        if (a[k][t].y == key[k]) acc[t][1] += d[k][t].y;
+                        if (a[k][t].z == key[k]) acc[t][2] += d[k][t].z;
+                        if (a[k][t].w == key[k]) acc[t][3] += d[k][t].w;
                     }
             }
         }
@@ -1186,40 +1223,47 @@ void csc_pf(betty_ctx* c, const void* dS, bool ds_bf16, int64_t ldds, const int6
 
 void agg_pool(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const int32_t* xrow, const float* Zp, int64_t ldz,
               const int64_t* indptr, const int32_t* idx, const int64_t* cnt, int64_t rows_cap, int Fi, int Fp,
-              void* XA, bool xa_bf16, int64_t ldxa, int32_t* arg, int64_t ldarg, cudaStream_t s) {
+              void* XA, bool xa_bf16, int64_t ldxa, void* arg, int64_t ldarg, bool pos8, cudaStream_t s) {
     const int ng = (Fi + 3) / 4;
-    const bool vec = (ldz % 4) == 0 && (ldarg % 4) == 0 && ng <= 64 && ((uintptr_t)Zp & 15) == 0 &&
-                     ((uintptr_t)arg & 15) == 0;
+    const bool vec = (ldz % 4) == 0 && ng <= 64 && ((uintptr_t)Zp & 15) == 0 && ((uintptr_t)arg & 15) == 0 &&
+                     (pos8 ? (ldarg % 4) == 0 : (ldarg % 4) == 0);
     if (vec) {
+        const int g = warps_grid(c, rows_cap);
+#define POOL_V(T, P) k_agg_pool_v<TI, TO, T, P><<<g, 256, 0, s>>>((const TI*)X, ldx, xrow, Zp, ldz, indptr, idx, cnt, \
+                                                                   Fi, Fp, (TO*)XA, ldxa, arg, ldarg)
         DISPATCH_ACT(x_bf16, TI, DISPATCH_ACT(xa_bf16, TO, {
-            if (ng <= 32) k_agg_pool_v<TI, TO, 1><<<warps_grid(c, rows_cap), 256, 0, s>>>((const TI*)X, ldx, xrow, Zp,
-                ldz, indptr, idx, cnt, Fi, Fp, (TO*)XA, ldxa, arg, ldarg);
-            else k_agg_pool_v<TI, TO, 2><<<warps_grid(c, rows_cap), 256, 0, s>>>((const TI*)X, ldx, xrow, Zp, ldz,
-                indptr, idx, cnt, Fi, Fp, (TO*)XA, ldxa, arg, ldarg); }))
+            if (ng <= 32) { if (pos8) POOL_V(1, true); else POOL_V(1, false); }
+            else { if (pos8) POOL_V(2, true); else POOL_V(2, false); } }))
+#undef POOL_V
         return;
     }
+    if (pos8) { fprintf(stderr, "betty: pool byte positions need the vectorised kernel\n"); return; }
     DISPATCH_ACT(x_bf16, TI, DISPATCH_ACT(xa_bf16, TO,
         k_agg_pool<TI, TO><<<warps_grid(c, rows_cap), 256, 0, s>>>((const TI*)X, ldx, xrow, Zp, ldz, indptr, idx, cnt,
-                                                                   Fi, Fp, (TO*)XA, ldxa, arg, ldarg)));
+                                                                   Fi, Fp, (TO*)XA, ldxa, (int32_t*)arg, ldarg)));
 }
 
-void route_pool(betty_ctx* c, const float* dXA, int64_t ldd, const int32_t* arg, int64_t ldarg,
-                const int64_t* t_indptr, const int32_t* t_idx, const int64_t* cnt, int64_t src_cap, int Fi, int Fp,
-                const float* Zp, int64_t ldz, void* out, bool out_bf16, int64_t ldo, cudaStream_t s) {
+void route_pool(betty_ctx* c, const float* dXA, int64_t ldd, const void* arg, int64_t ldarg, bool pos8,
+                const int64_t* indptr, const int32_t* idx, const int64_t* t_indptr, const int32_t* t_idx,
+                const int64_t* cnt, int64_t src_cap, int Fi, int Fp, const float* Zp, int64_t ldz, void* out,
+                bool out_bf16, int64_t ldo, cudaStream_t s) {
     const int ng = (Fi + 3) / 4;
     const bool vec = (ldz % 4) == 0 && (ldarg % 4) == 0 && (ldd % 4) == 0 && (Fp % 4) == 0 && ng <= 64 &&
                      ((uintptr_t)Zp & 15) == 0 && ((uintptr_t)arg & 15) == 0 && ((uintptr_t)dXA & 15) == 0;
     if (vec) {
+        const int g = warps_grid(c, src_cap);
+#define ROUTE_V(T, P) k_route_pool_v<TO, T, P><<<g, 256, 0, s>>>(dXA, ldd, arg, ldarg, indptr, idx, t_indptr, t_idx, \
+                                                                 cnt, Fi, Fp, Zp, ldz, (TO*)out, ldo)
         DISPATCH_ACT(out_bf16, TO, {
-            if (ng <= 32) k_route_pool_v<TO, 1><<<warps_grid(c, src_cap), 256, 0, s>>>(dXA, ldd, arg, ldarg, t_indptr,
-                t_idx, cnt, Fi, Fp, Zp, ldz, (TO*)out, ldo);
-            else k_route_pool_v<TO, 2><<<warps_grid(c, src_cap), 256, 0, s>>>(dXA, ldd, arg, ldarg, t_indptr, t_idx,
-                cnt, Fi, Fp, Zp, ldz, (TO*)out, ldo); })
+            if (ng <= 32) { if (pos8) ROUTE_V(1, true); else ROUTE_V(1, false); }
+            else { if (pos8) ROUTE_V(2, true); else ROUTE_V(2, false); } })
+#undef ROUTE_V
         return;
     }
+    if (pos8) { fprintf(stderr, "betty: pool byte positions need the vectorised kernel\n"); return; }
     DISPATCH_ACT(out_bf16, TO,
-        k_route_pool<TO><<<warps_grid(c, src_cap), 256, 0, s>>>(dXA, ldd, arg, ldarg, t_indptr, t_idx, cnt, Fi, Fp, Zp,
-                                                                ldz, (TO*)out, ldo));
+        k_route_pool<TO><<<warps_grid(c, src_cap), 256, 0, s>>>(dXA, ldd, (const int32_t*)arg, ldarg, t_indptr, t_idx,
+                                                                cnt, Fi, Fp, Zp, ldz, (TO*)out, ldo));
 }
 
 }  // namespace betty

@@ -552,6 +552,13 @@ static betty_status size_micro_batches(betty_ctx* c, const ExtractFull* F, const
     return st;
 }
 
+__global__ void k_max_deg(const int64_t* __restrict__ indptr, int64_t n, int* out) {
+    int mx = 0;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        { const int64_t d = indptr[i + 1] - indptr[i]; mx = max(mx, d > 1000000 ? 1000000 : (int)d); }
+    atomicMax(out, mx);
+}
+
 extern "C" betty_status betty_plan_create(betty_ctx* c, const betty_model* model, const betty_block* full, int32_t L,
                                           const int32_t* part, int64_t n_out, int32_t K, const int32_t* my_k,
                                           int32_t n_my, int32_t group, int32_t flags, betty_plan** out,
@@ -569,6 +576,27 @@ extern "C" betty_status betty_plan_create(betty_ctx* c, const betty_model* model
         return fail(c, BETTY_EINVAL, "plan: bad K / my_k / n_out / part");
     for (int i = 0; i < n_my; ++i)
         if (my_k[i] < 0 || my_k[i] >= K) return fail(c, BETTY_EINVAL, "plan: my_k[%d] out of range", i);
+    // pool layers can keep the argmax as a byte position when every row of the block has <= 254 edges
+    // (micro-batch rows are full-batch rows; one reduction per pool layer, here at plan time).  Off by
+    // default (BETTY_POOL_POS8=1): on C4 it reads 23 % fewer bytes but the routing kernel's search of
+    // u's position in each row costs more latency than it saves (105 vs 63 ms per step, measured).
+    const bool pos8_on = getenv("BETTY_POOL_POS8") && atoi(getenv("BETTY_POOL_POS8"));
+    if (m.aggr == BETTY_AGGR_POOL && pos8_on) {
+        int* d_mx = nullptr;
+        if (cudaMalloc(&d_mx, sizeof(int) * L) != cudaSuccess) return fail(c, BETTY_ENOMEM, "plan: max degree");
+        cudaMemsetAsync(d_mx, 0, sizeof(int) * L, s);
+        for (int l = 0; l < L; ++l)
+            if (full[l].n_dst > 0)
+                k_max_deg<<<(int)std::min<int64_t>((full[l].n_dst + 255) / 256, 4096), 256, 0, s>>>(
+                    full[l].indptr, full[l].n_dst, d_mx + l);
+        std::vector<int> mx(L, 0);
+        cudaMemcpyAsync(mx.data(), d_mx, sizeof(int) * L, cudaMemcpyDeviceToHost, s);
+        st = sync_check(c, s);
+        cudaFree(d_mx);
+        if (st) return st;
+        m.pos8.assign(L, 0);
+        for (int l = 0; l < L; ++l) m.pos8[l] = mx[l] <= 254;
+    }
     betty_plan* p = new (std::nothrow) betty_plan();
     if (!p) return BETTY_ENOMEM;
     p->m = m; p->L = L; p->K = K; p->flags = flags; p->n_out = n_out; p->part = part;

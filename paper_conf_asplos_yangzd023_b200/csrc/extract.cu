@@ -243,6 +243,7 @@ __device__ __forceinline__ int64_t dst_id(const RankSet& R, int l, int j, int32_
 // per lane in flight (independent load chains), every lane busy whatever the
 // degree mix.  Row data live in a per-warp shared slice.
 constexpr int FLAT_UNR = 4;
+constexpr int RL_UNR = 4;          // relabel chains per lane (8: 128 registers, measured slower)
 struct FlatRows {
     int pre[33];        // exclusive edge offsets of the warp's rows (pre[32] = total)
     int64_t fb[32];     // full-batch row start of each row
@@ -366,11 +367,11 @@ __global__ void __launch_bounds__(256) k_relabel(const int32_t* __restrict__ dst
         if (lane == 0) F.pre[0] = 0;
         __syncwarp();
         const int total = F.pre[32];
-        for (int f0 = lane; f0 < total; f0 += 32 * FLAT_UNR) {
-            int32_t p[FLAT_UNR];
-            int kk[FLAT_UNR];
+        for (int f0 = lane; f0 < total; f0 += 32 * RL_UNR) {
+            int32_t p[RL_UNR];
+            int kk[RL_UNR];
 #pragma unroll
-            for (int u = 0; u < FLAT_UNR; ++u) {
+            for (int u = 0; u < RL_UNR; ++u) {
                 const int f = f0 + 32 * u;
                 p[u] = -1;
                 if (f < total) {
@@ -379,20 +380,20 @@ __global__ void __launch_bounds__(256) k_relabel(const int32_t* __restrict__ dst
                     p[u] = fnbr[F.fb[k] + (f - F.pre[k])];
                 }
             }
-            uint2 nr[FLAT_UNR];
-            int32_t id[FLAT_UNR], gid[FLAT_UNR];
+            uint2 nr[RL_UNR];
+            int32_t id[RL_UNR], gid[RL_UNR];
 #pragma unroll
-            for (int u = 0; u < FLAT_UNR; ++u) {
+            for (int u = 0; u < RL_UNR; ++u) {
                 if (p[u] >= 0) {
                     nr[u] = R.nr[l][(int64_t)F.j[kk[u]] * R.W[l] + (p[u] >> 5)];
                     if (egid) gid[u] = fsrc_gid[p[u]];
                 }
             }
-            // src_id level by level for all FLAT_UNR edges at once: each level's rank-word loads are
+            // src_id level by level for all RL_UNR edges at once: each level's rank-word loads are
             // issued together (independent chains), not one edge's whole chain after another
-            bool done[FLAT_UNR];
+            bool done[RL_UNR];
 #pragma unroll
-            for (int u = 0; u < FLAT_UNR; ++u) {
+            for (int u = 0; u < RL_UNR; ++u) {
                 done[u] = p[u] < 0;
                 if (!done[u] && (nr[u].x >> (p[u] & 31) & 1u)) {
                     id[u] = (int32_t)(R.cnt[l][0] + R.off[l][F.j[kk[u]]] + rank_in(nr[u], p[u]));
@@ -401,23 +402,23 @@ __global__ void __launch_bounds__(256) k_relabel(const int32_t* __restrict__ dst
             }
             for (int q = l + 1; q < R.L; ++q) {
 #pragma unroll
-                for (int u = 0; u < FLAT_UNR; ++u)
+                for (int u = 0; u < RL_UNR; ++u)
                     if (!done[u]) nr[u] = R.nr[q][(int64_t)F.j[kk[u]] * R.W[q] + (p[u] >> 5)];
 #pragma unroll
-                for (int u = 0; u < FLAT_UNR; ++u)
+                for (int u = 0; u < RL_UNR; ++u)
                     if (!done[u] && (nr[u].x >> (p[u] & 31) & 1u)) {
                         id[u] = (int32_t)(R.cnt[q][0] + R.off[q][F.j[kk[u]]] + rank_in(nr[u], p[u]));
                         done[u] = true;
                     }
             }
 #pragma unroll
-            for (int u = 0; u < FLAT_UNR; ++u)
+            for (int u = 0; u < RL_UNR; ++u)
                 if (!done[u]) nr[u] = R.dr[(int64_t)F.j[kk[u]] * R.Wt + (p[u] >> 5)];
 #pragma unroll
-            for (int u = 0; u < FLAT_UNR; ++u)
+            for (int u = 0; u < RL_UNR; ++u)
                 if (!done[u]) id[u] = (int32_t)(R.top_off[F.j[kk[u]]] + rank_in(nr[u], p[u]));
 #pragma unroll
-            for (int u = 0; u < FLAT_UNR; ++u) {
+            for (int u = 0; u < RL_UNR; ++u) {
                 if (p[u] >= 0) {
                     const int k = kk[u];
                     const int64_t o = F.ob[k] + (f0 + 32 * u - F.pre[k]);

@@ -28,6 +28,10 @@ struct ModelCfg {
     std::vector<int> dims;
     std::vector<LayerCfg> layers;
     int64_t n_params = 0;
+    // pool layers: the argmax is stored as the byte position of the winning edge in its row (plans
+    // whose pool blocks have rows of <= 254 edges), else as the source id (int32)
+    std::vector<char> pos8;
+    bool arg8(int l) const { return l < (int)pos8.size() && pos8[l]; }
     // does the backward of layer l need the CSC of block l?
     bool needs_csc(int l) const { return !(layers[l].kind == KIND_AGG && l == 0); }
     // layer l reads a gathered [X | 1] copy of the features (layer 0 of PF / POOL)

@@ -109,7 +109,7 @@ bool sage_alloc(betty_ctx* c, const ModelCfg& m, const std::vector<int64_t>& cap
         }
         if (L.kind == KIND_POOL) {
             B.Zp = (float*)A(ns * L.ld_zp * 4);
-            B.arg = (int32_t*)A(nd * L.ld_arg * 4);
+            B.arg = (int32_t*)A(nd * (m.arg8(l) ? (L.Fi + 15) / 16 * 16 : L.ld_arg * 4));
             B.dZp = A(ns * L.ld_dzp * ea);
             B.Bp = A((L.Fi + 1) * L.ld_Bp * ea);
             B.S_pool = gemm_red_splits(ns, L.Fi + 1, L.Fi);
@@ -234,7 +234,7 @@ void sage_forward(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView*
             gemm_row(c, g, s);
             PB(l == 0 ? PROBE_AGG_L0 : PROBE_AGG_L1);
             agg_pool(c, X, xbf, ldx, xrow, B.Zp, L.ld_zp, V.indptr, V.indices, V.cnt, V.cap_dst, L.Fi, L.Fp, B.XA,
-                     m.bf16, L.ld_xa, B.arg, L.ld_arg, s);
+                     m.bf16, L.ld_xa, B.arg, m.arg8(l) ? (L.Fi + 15) / 16 * 16 : L.ld_arg, m.arg8(l), s);
             PE(l == 0 ? PROBE_AGG_L0 : PROBE_AGG_L1);
         } else {
             PB(l == 0 ? PROBE_AGG_L0 : PROBE_AGG_L1);
@@ -344,8 +344,9 @@ void sage_backward(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView
             continue;
         }
         // POOL: route to the argmax, then W_pool
-        route_pool(c, B.dXA, L.ld_dxa, B.arg, L.ld_arg, V.t_indptr, V.t_indices, V.cnt, V.cap_src, L.Fi, L.Fp, B.Zp,
-                   L.ld_zp, B.dZp, m.bf16, L.ld_dzp, s);
+        route_pool(c, B.dXA, L.ld_dxa, B.arg, m.arg8(l) ? (L.Fi + 15) / 16 * 16 : L.ld_arg, m.arg8(l), V.indptr,
+                   V.indices, V.t_indptr, V.t_indices, V.cnt, V.cap_src, L.Fi, L.Fp, B.Zp, L.ld_zp, B.dZp, m.bf16,
+                   L.ld_dzp, s);
         const void* Ao; int64_t ldao;
         ones_operand(m, b, l, &Ao, &ldao);
         {

@@ -25,12 +25,15 @@ void csc_mean(betty_ctx* c, const float* dXA, int64_t ldd, const int64_t* indptr
 void csc_pf(betty_ctx* c, const void* dS, bool ds_bf16, int64_t ldds, const int64_t* indptr, const int64_t* t_indptr,
             const int32_t* t_idx, const int64_t* cnt, int64_t src_cap, int Fo, int Fop, void* G, bool g_bf16,
             int64_t ldg, cudaStream_t s);
+// pool: XA = [x_v | max_u ReLU(Zp[u]) | 1]; argmax per (v, column) as the source id (int32) or, with
+// pos8, the byte position of the winning edge in v's row (rows of <= 254 edges)
 void agg_pool(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const int32_t* xrow, const float* Zp, int64_t ldz,
               const int64_t* indptr, const int32_t* idx, const int64_t* cnt, int64_t rows_cap, int Fi, int Fp,
-              void* XA, bool xa_bf16, int64_t ldxa, int32_t* arg, int64_t ldarg, cudaStream_t s);
-void route_pool(betty_ctx* c, const float* dXA, int64_t ldd, const int32_t* arg, int64_t ldarg,
-                const int64_t* t_indptr, const int32_t* t_idx, const int64_t* cnt, int64_t src_cap, int Fi, int Fp,
-                const float* Zp, int64_t ldz, void* out, bool out_bf16, int64_t ldo, cudaStream_t s);
+              void* XA, bool xa_bf16, int64_t ldxa, void* arg, int64_t ldarg, bool pos8, cudaStream_t s);
+void route_pool(betty_ctx* c, const float* dXA, int64_t ldd, const void* arg, int64_t ldarg, bool pos8,
+                const int64_t* indptr, const int32_t* idx, const int64_t* t_indptr, const int32_t* t_idx,
+                const int64_t* cnt, int64_t src_cap, int Fi, int Fp, const float* Zp, int64_t ldz, void* out,
+                bool out_bf16, int64_t ldo, cudaStream_t s);
 
 // ---- gemm.cu (dense layers; SIMT fp32 FFMA path, operands fp32 or bf16)
 enum { EPI_STORE = 0, EPI_RELU_ONES = 1, EPI_MASK = 2, EPI_RES_MASK = 3 };

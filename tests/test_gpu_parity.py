@@ -330,3 +330,26 @@ def test_c1_cora_config(B, ctx):
         assert_close(grad.cpu().numpy(), og, RTOL[mode], f"C1 grad {mode}")
         assert loss.item() == pytest.approx(ol, rel=RTOL[mode])
         plan.free()
+
+
+@pytest.mark.parametrize("mode", ["fp32", "bf16"])
+def test_pool_byte_positions(B, ctx, mode, monkeypatch):
+    """The optional byte-position argmax of the pool layers (BETTY_POOL_POS8=1, plan path)
+    routes the gradient exactly like the source-id argmax."""
+    monkeypatch.setenv("BETTY_POOL_POS8", "1")
+    c = CASES[5]
+    sd, blocks, feats, labels, params = make_case(c, seed=3)
+    K = 3
+    part = synth.random_partition(len(sd), K, 5)
+    dev = B.blocks_to_device(blocks)
+    model = B.Model(c["dims"], c["aggr"], mode, mode)
+    P = torch.as_tensor(params).cuda()
+    plan = B.betty_plan_create(ctx, model, dev, torch.as_tensor(part).cuda(), K, [0, 1, 2], group=0, flags=0)
+    grad = torch.zeros_like(P)
+    loss = torch.zeros(1, device="cuda")
+    B.betty_step(ctx, plan, P, dev_feats(feats, mode), torch.as_tensor(labels).cuda(), 1.0 / len(sd), grad, loss)
+    B.betty_sync_check(ctx)
+    og, ol = oracle.step(c["dims"], c["aggr"], mode == "bf16", blocks, part, K, [0, 1, 2], params, feats, labels,
+                         1.0 / len(sd))
+    assert_close(grad.cpu().numpy(), og, RTOL[mode], "grad")
+    plan.free()
