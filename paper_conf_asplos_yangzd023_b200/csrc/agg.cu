@@ -1058,7 +1058,7 @@ __global__ void __launch_bounds__(256) k_csc_pf_v(const Tin* __restrict__ dS, in
                 float myinv = 0.f;
                 if (sub < n) {
                     my = t_idx[e0 + sub];
-                    myinv = 1.0f / (float)(indptr[my + 1] - indptr[my]);
+                    myinv = indptr ? 1.0f / (float)(indptr[my + 1] - indptr[my]) : 1.0f;
                 }
 #pragma unroll
                 for (int j = 0; j < LPR; ++j) {

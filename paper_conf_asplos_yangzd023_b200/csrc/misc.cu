@@ -20,7 +20,8 @@ __global__ void __launch_bounds__(256) k_loss(const float* __restrict__ logits, 
                                               const int32_t* __restrict__ labels, const int32_t* __restrict__ gid,
                                               const int64_t* cnt, int C, float scale, float* __restrict__ dS,
                                               int64_t ldds, TA* __restrict__ dS_act, int64_t ld_act,
-                                              double* partials, unsigned* ctr, float* loss_accum) {
+                                              const int64_t* __restrict__ indptr, double* partials, unsigned* ctr,
+                                              float* loss_accum) {
     __shared__ double s_w[8];
     __shared__ int s_last;
     const int64_t nd = cnt[0];
@@ -30,6 +31,9 @@ __global__ void __launch_bounds__(256) k_loss(const float* __restrict__ logits, 
     double wl = 0.0;
     for (int64_t v = gw; v < nd; v += nw) {
         const int32_t y = labels[gid[v]];               // independent of the logits: issued first
+        // indptr (project-first top layer): the fp32 dS is stored pre-scaled by 1/D_v for P^T D+ dS
+        float inv = 1.f;
+        if (indptr) { const int64_t dg = indptr[v + 1] - indptr[v]; inv = dg > 0 ? 1.f / (float)dg : 0.f; }
         float x[LOSS_MAXT];
         float mx = -INFINITY;
 #pragma unroll
@@ -54,7 +58,7 @@ __global__ void __launch_bounds__(256) k_loss(const float* __restrict__ logits, 
             if (c == y) xy = x[t];
             if (c < C) {
                 const float d = scale * (expf(x[t] - lse) - (c == y ? 1.f : 0.f));
-                dS[v * ldds + c] = d;
+                dS[v * ldds + c] = d * inv;
                 if (dS_act) st_act(dS_act + v * ld_act + c, d);
             }
         }
@@ -93,17 +97,17 @@ __global__ void __launch_bounds__(256) k_loss(const float* __restrict__ logits, 
 
 void loss_ce(betty_ctx* c, const float* logits, int64_t ldl, const int32_t* labels, const int32_t* gid,
              const int64_t* cnt, int64_t rows_cap, int C, float scale, float* dS, int64_t ldds, void* dS_act,
-             bool act_bf16, int64_t ld_act, float* loss_accum, cudaStream_t s) {
+             bool act_bf16, int64_t ld_act, const int64_t* prescale_indptr, float* loss_accum, cudaStream_t s) {
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((rows_cap * 32 + 255) / 256,
                                                                  std::min(2048, c->num_sms * 8)));
     double* partials = (double*)(c->L().counters + 64);   // 2048 doubles after the counters
     if (act_bf16)
         k_loss<__nv_bfloat16><<<grid, 256, 0, s>>>(logits, ldl, labels, gid, cnt, C, scale, dS, ldds,
-                                                   (__nv_bfloat16*)dS_act, ld_act, partials, c->L().counters + CTR_LOSS,
-                                                   loss_accum);
+                                                   (__nv_bfloat16*)dS_act, ld_act, prescale_indptr, partials,
+                                                   c->L().counters + CTR_LOSS, loss_accum);
     else
         k_loss<float><<<grid, 256, 0, s>>>(logits, ldl, labels, gid, cnt, C, scale, dS, ldds, (float*)dS_act, ld_act,
-                                           partials, c->L().counters + CTR_LOSS, loss_accum);
+                                           prescale_indptr, partials, c->L().counters + CTR_LOSS, loss_accum);
 }
 
 // ------------------------------------------------------------------ adam

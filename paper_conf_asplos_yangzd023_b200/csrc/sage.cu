@@ -264,8 +264,9 @@ void sage_loss(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView* v,
                float* loss_accum, cudaStream_t s) {
     const LayerCfg& L = m.layers[m.L - 1];
     const BlockView& V = v[m.L - 1];
+    // the fp32 dS of a project-first top layer is read only by P^T D+ dS: stored pre-scaled by 1/D_v
     loss_ce(c, b.logits, L.ld_out, labels, V.src_gid, V.cnt, V.cap_dst, L.Fo, scale, b.dS_last, L.Fop,
-            b.dS_last_act, m.bf16, L.ld_ds, loss_accum, s);
+            b.dS_last_act, m.bf16, L.ld_ds, L.kind == KIND_PF ? V.indptr : nullptr, loss_accum, s);
 }
 
 void sage_backward(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView* v, const void* feats,
@@ -285,7 +286,8 @@ void sage_backward(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView
             // dX = G W_n^T + [dst] dS W_s^T (the second term as the epilogue residual), masked by ReLU'
             const int64_t esz = m.bf16 ? 2 : 4;
             const bool ds_f32 = L.last;
-            csc_pf(c, ds_f32 ? (const void*)b.dS_last : B.dS, !ds_f32 && m.bf16, ds_f32 ? L.Fop : L.ld_ds, V.indptr,
+            csc_pf(c, ds_f32 ? (const void*)b.dS_last : B.dS, !ds_f32 && m.bf16, ds_f32 ? L.Fop : L.ld_ds,
+                   ds_f32 ? nullptr : V.indptr,
                    V.t_indptr, V.t_indices, V.cnt, V.cap_src, L.Fo, L.Fop, B.G, m.bf16, L.ld_g, s);
             const void* Ao; int64_t ldao;
             ones_operand(m, b, l, &Ao, &ldao);

@@ -22,6 +22,7 @@ void gather_ones(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const in
 void csc_mean(betty_ctx* c, const float* dXA, int64_t ldd, const int64_t* indptr, const int64_t* t_indptr,
               const int32_t* t_idx, const int64_t* cnt, int64_t src_cap, int Fi, int Fp, const void* H, bool h_bf16,
               int64_t ldh, void* out, bool out_bf16, int64_t ldo, cudaStream_t s);
+// G = P^T D+ dS via the CSC; indptr == null: dS is already scaled by 1/D_v (the loss kernel does it)
 void csc_pf(betty_ctx* c, const void* dS, bool ds_bf16, int64_t ldds, const int64_t* indptr, const int64_t* t_indptr,
             const int32_t* t_idx, const int64_t* cnt, int64_t src_cap, int Fo, int Fop, void* G, bool g_bf16,
             int64_t ldg, cudaStream_t s);
@@ -80,7 +81,7 @@ bool gemm_red_tc(betty_ctx* c, const GemmRed& g, cudaStream_t s);
 // ---- misc.cu
 void loss_ce(betty_ctx* c, const float* logits, int64_t ldl, const int32_t* labels, const int32_t* gid,
              const int64_t* cnt, int64_t rows_cap, int C, float scale, float* dS, int64_t ldds, void* dS_act,
-             bool act_bf16, int64_t ld_act, float* loss_accum, cudaStream_t s);
+             bool act_bf16, int64_t ld_act, const int64_t* prescale_indptr, float* loss_accum, cudaStream_t s);
 void adam(betty_ctx* c, float* p, float* g, float* m, float* v, int64_t n, int t, float lr, float b1, float b2,
           float eps, bool zero_grad, cudaStream_t s);
 // per-layer GEMM weight layouts from the flat parameter vector
