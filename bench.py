@@ -59,6 +59,9 @@ def parse():
     p.add_argument("--scale", type=float, default=1.0, help="shrink the graph (debug only)")
     p.add_argument("--json-out", default=None)
     p.add_argument("--feat-align", type=int, default=256, help="feature-table row alignment in bytes (0: 16)")
+    p.add_argument("--feat-layout", default="gid", choices=["gid", "owner"],
+                   help="feature-table row order: gid (as generated) or owner (rows grouped by the micro-batch "
+                        "that reads them most, experimental)")
     return p.parse_args()
 
 
@@ -153,8 +156,8 @@ def build_inputs(args, rank, ws, device):
         cfg = synth.scaled(cfg, args.scale)
     t0 = time.time()
     if rank == 0:
-        ds = synth.make(cfg)
-        arrays = [ds.feats, ds.labels, ds.seeds]
+        ds = synth.make(cfg, with_features=None)      # None: C5's table is generated in chunks on the device
+        arrays = [ds.graph.comm, ds.labels, ds.seeds]
         for b in ds.blocks:
             arrays += [b.indptr, b.nbr_pos, b.src_gid]
     else:
@@ -176,8 +179,48 @@ def build_inputs(args, rank, ws, device):
             for l in range(cfg.L):
                 ip, nb, sg = arrays[3 + 3 * l: 6 + 3 * l]
                 blocks.append(synth.Block(len(ip) - 1, len(sg), ip, nb, sg))
-            ds = synth.Dataset(cfg, None, arrays[0], arrays[1], arrays[2], blocks)
+            feats = synth.features(arrays[0], cfg.F, cfg.ld, cfg.feat_kind, seed=cfg.seeds["feat"]) \
+                if cfg.n * cfg.ld * 4 <= synth.HOST_FEATURE_LIMIT else None
+            ds = synth.Dataset(cfg, synth.Graph(None, None, arrays[0]), feats, arrays[1], arrays[2], blocks)
     return cfg, ds, time.time() - t0
+
+
+def device_features(cfg, ds, bf16: bool, align: int, device, chunk_rows: int = 1 << 22):
+    """The feature table in HBM (bf16 or fp32), rows padded to `align` bytes.  Tables too large for the
+    host (C5: 111 M x 128 fp32 = 57 GB) are generated in chunks of rows (synth.features_rows) and
+    converted on the device; the others are copied from the host array."""
+    import torch
+    import synth
+    dt = torch.bfloat16 if bf16 else torch.float32
+    esz = 2 if bf16 else 4
+    per = max(1, align // esz) if align > 0 else 1
+    ld = (cfg.ld + per - 1) // per * per
+    out = torch.zeros((cfg.n, ld), dtype=dt, device=device)
+    if ds.feats is not None:
+        out[:, :cfg.ld] = torch.as_tensor(ds.feats).to(device).to(dt)
+        return out
+    for r0 in range(0, cfg.n, chunk_rows):
+        n = min(chunk_rows, cfg.n - r0)
+        h = synth.features_rows(ds.graph.comm, cfg.F, cfg.ld, row0=r0, n=n, kind=cfg.feat_kind, seed=cfg.seeds["feat"])
+        out[r0:r0 + n, :cfg.ld] = torch.from_numpy(h).to(device).to(dt)
+    return out
+
+
+def oracle_inputs(cfg, ds, part):
+    """Full-batch blocks and a feature array for the oracle's micro-batch 0 of `part`: the host table
+    itself, or (C5) only the rows micro-batch 0 reads, with layer-0 ids remapped onto them."""
+    import synth
+    import oracle
+    if ds.feats is not None:
+        return ds.blocks, ds.feats
+    mb = oracle.extract(ds.blocks, part, 2, 0)
+    gids = np.unique(mb[0].src_gid)
+    feats = synth.features_rows(ds.graph.comm, cfg.F, cfg.ld, ids=gids, kind=cfg.feat_kind, seed=cfg.seeds["feat"])
+    b0 = ds.blocks[0]
+    j = np.minimum(np.searchsorted(gids, b0.src_gid), len(gids) - 1)
+    remap = np.where(gids[j] == b0.src_gid, j, 0).astype(np.int32)
+    blocks = [synth.Block(b0.n_dst, b0.n_src, b0.indptr, b0.nbr_pos, remap)] + list(ds.blocks[1:])
+    return blocks, feats
 
 
 def memory_aware(args, B, ctx, cfg, dev_blocks, rank, ws, device):
@@ -265,14 +308,15 @@ def run_reference(args, ws, rank):
     cfg = synth.CONFIGS[args.config]
     if args.scale != 1.0:
         cfg = synth.scaled(cfg, args.scale)
-    ds = synth.make(cfg)
+    ds = synth.make(cfg, with_features=None)
     args.K = args.K or 8
     part, sample_desc, edges = reference_sample(args, cfg, ds, args.ref_sample_outputs)
+    oblocks, ofeats = oracle_inputs(cfg, ds, part)
     params = synth.init_params(cfg.dims, cfg.aggr, seed=cfg.seeds["init"])
     times = []
     for it in range(args.warmup + args.steps):
         t0 = time.perf_counter()
-        oracle.step(cfg.dims, cfg.aggr, args.mode == "bf16", ds.blocks, part, 2, [0], params, ds.feats, ds.labels,
+        oracle.step(cfg.dims, cfg.aggr, args.mode == "bf16", oblocks, part, 2, [0], params, ofeats, ds.labels,
                     1.0 / cfg.n_out)
         if it >= args.warmup:
             times.append(time.perf_counter() - t0)
@@ -307,9 +351,12 @@ def reference_sample(args, cfg, ds, n_outputs):
 def main():
     args = parse()
     if args.K is None:
-        args.K = {"C1": 2, "C2": 8, "C3": 32, "C4": 0}.get(args.config, 32)
+        args.K = {"C1": 2, "C2": 8, "C3": 32, "C4": 0, "C5": 32}.get(args.config, 32)
     if args.group is None:
         args.group = 1 if args.config == "C4" else 0
+    if args.config == "C5":      # 3 hops over a 111 M-node graph: ~20 s of oracle per 1k outputs
+        args.cpu_sample_outputs = min(args.cpu_sample_outputs, 1024)
+        args.ref_sample_outputs = min(args.ref_sample_outputs, 256)
     if args.config == "C4":      # a 5-hop closure reaches most of the graph: keep the oracle samples bounded
         args.cpu_sample_outputs = min(args.cpu_sample_outputs, 2)
         args.ref_sample_outputs = min(args.ref_sample_outputs, 1)
@@ -337,10 +384,26 @@ def main():
     costs = micro_batch_costs(part, args.K, ds.blocks[-1].indptr)
     my_k = lpt_assign(costs, ws)[rank]
 
-    feats = torch.as_tensor(ds.feats).to(device)
-    if args.mode == "bf16":
-        feats = feats.to(torch.bfloat16).contiguous()       # bf16 feature table (reading #17)
-    feats = pad_rows(feats, args.feat_align)
+    feats = device_features(cfg, ds, args.mode == "bf16", args.feat_align, device)   # bf16: reading #17
+    host_gid0 = ds.blocks[0].src_gid
+    if args.feat_layout == "owner":
+        t_l = time.time()
+        perm = owner_layout(ds.blocks, part, args.K)
+        n_all = feats.shape[0]
+        full_perm = np.empty(n_all, np.int64)
+        miss = perm < 0
+        full_perm[:len(perm)] = perm
+        extra = np.nonzero(np.concatenate([miss, np.ones(n_all - len(perm), bool)]))[0]
+        full_perm[extra] = len(perm) - miss.sum() + np.arange(len(extra))
+        dperm = torch.as_tensor(full_perm).to(device)
+        fp = torch.empty_like(feats)
+        fp[dperm] = feats
+        feats = fp
+        b0 = dev_blocks[0]
+        b0.src_gid.copy_(dperm[b0.src_gid.long()].to(torch.int32))
+        del dperm, fp
+        host_gid0 = b0.src_gid.cpu().numpy()
+        print(f"feature layout: owner ({time.time() - t_l:.1f} s)", file=sys.stderr)
     labels = torch.as_tensor(ds.labels).to(device)
     model = B.Model(cfg.dims, cfg.aggr, args.mode, args.mode)
     params = torch.as_tensor(synth_params(cfg)).to(device)
@@ -350,7 +413,7 @@ def main():
     loss = torch.zeros(1, device=device)
     flags = (0 if args.no_graph else B.PLAN_GRAPH) | (0 if args.no_reg else B.PLAN_REG)
     t0 = time.time()
-    plan = B.betty_plan_create(ctx, model, dev_blocks, dpart, args.K, my_k, group=args.group, flags=flags)
+    plan, args.group = create_plan(B, ctx, model, dev_blocks, dpart, args.K, my_k, args.group, flags)
     t_plan = time.time() - t0
     info = plan.info()
     scale = 1.0 / cfg.n_out
@@ -399,9 +462,9 @@ def main():
 
     # ------------------------------------- e2e: host buffers through the ABI
     host = []
-    for b in ds.blocks:
+    for l, b in enumerate(ds.blocks):
         host += [torch.from_numpy(b.indptr).pin_memory(), torch.from_numpy(b.nbr_pos).pin_memory(),
-                 torch.from_numpy(b.src_gid).pin_memory()]
+                 torch.from_numpy(host_gid0 if l == 0 else b.src_gid).pin_memory()]
     host.append(torch.from_numpy(part).pin_memory())
     devs = []
     for db in dev_blocks:
@@ -460,9 +523,10 @@ def main():
     if rank == 0 and ws == 1:
         import oracle
         rpart, desc, redges = reference_sample(args, cfg, ds, args.cpu_sample_outputs)
+        oblocks, ofeats = oracle_inputs(cfg, ds, rpart)
         pr = synth_params(cfg).astype(np.float64)
         tc = time.perf_counter()
-        oracle.step(cfg.dims, cfg.aggr, args.mode == "bf16", ds.blocks, rpart, 2, [0], pr, ds.feats, ds.labels,
+        oracle.step(cfg.dims, cfg.aggr, args.mode == "bf16", oblocks, rpart, 2, [0], pr, ofeats, ds.labels,
                     scale)
         dt = time.perf_counter() - tc
         cpu = {"value": redges / dt, "unit": "edges/s", "cores": 1, "kind": "oracle", "sample": desc,
@@ -502,20 +566,78 @@ def main():
         dist.destroy_process_group()
 
 
-def pad_rows(t, align: int):
-    """Feature table with rows padded to a multiple of `align` bytes (zeros): random row gathers of
-    256-byte-aligned rows run closer to the HBM ceiling than 208-byte rows straddling bursts
-    (tools/micro/gather_ceiling.cu).  The pad columns are never read."""
+def create_plan(B, ctx, model, dev_blocks, dpart, K, my_k, group, flags):
+    """The plan with the requested launch group (0 = all of the rank's micro-batches).  When its arenas
+    do not fit in HBM (C5: ~10^9 micro-batch edges), a one-micro-batch plan measures the arena of the
+    largest micro-batch and the group becomes what fits in 85 % of the free HBM (halved further on
+    failure).  Returns (plan, group actually used; 0 = all)."""
     import torch
-    if align <= 0:
-        return t
-    per = max(1, align // t.element_size())
-    ld = (t.shape[1] + per - 1) // per * per
-    if ld == t.shape[1]:
-        return t
-    out = torch.zeros((t.shape[0], ld), dtype=t.dtype, device=t.device)
-    out[:, :t.shape[1]] = t
-    return out
+
+    def oom(e):
+        return "ENOMEM" in str(e) or "out of memory" in str(e)
+
+    def attempt(g):
+        try:
+            return B.betty_plan_create(ctx, model, dev_blocks, dpart, K, my_k, group=g, flags=flags)
+        except B.BettyError as e:
+            if not oom(e):
+                raise
+            torch.cuda.synchronize()
+            torch.cuda.empty_cache()
+            return None
+
+    n = max(1, len(my_k))
+    g = group if group > 0 else n
+    plan = attempt(g)
+    if plan is not None:
+        return plan, (0 if group == 0 else g)
+    one = attempt(1)
+    if one is None:
+        raise SystemExit("plan: one micro-batch does not fit in HBM")
+    a1 = one.info()["arena_bytes"]
+    one.free()
+    torch.cuda.synchronize()
+    torch.cuda.empty_cache()
+    free = torch.cuda.mem_get_info()[0]
+    g = max(1, min(g // 2, int(0.85 * free / max(a1, 1))))
+    while True:
+        print(f"plan: arenas of the full group do not fit; largest micro-batch {a1 / 2**30:.2f} GB, "
+              f"free {free / 2**30:.1f} GB -> launch group {g}", file=sys.stderr)
+        plan = attempt(g)
+        if plan is not None:
+            return plan, g
+        if g == 1:
+            raise SystemExit("plan: no launch group fits in HBM")
+        g = max(1, g // 2)
+
+
+def owner_layout(blocks, part, K):
+    """Row order of the feature table grouped by owner micro-batch (majority vote of the micro-batches
+    whose layer-0 sources contain the node, propagated down the full-batch blocks).  Returns perm with
+    perm[gid] = new row.  Host preprocessing, outside the step (like the partition)."""
+    def votes(n_items, idx, who):
+        key = idx.astype(np.int64) * (K + 1) + who.astype(np.int64)
+        u, c = np.unique(key, return_counts=True)
+        item, own = u // (K + 1), u % (K + 1)
+        o = np.lexsort((own, -c, item))
+        item, own = item[o], own[o]
+        first = np.ones(len(item), bool)
+        first[1:] = item[1:] != item[:-1]
+        out = np.full(n_items, K, np.int64)
+        out[item[first]] = own[first]
+        return out
+    own_dst = np.asarray(part, dtype=np.int64)
+    for b in reversed(blocks):
+        deg = np.diff(b.indptr)
+        idx = np.concatenate([b.nbr_pos.astype(np.int64), np.arange(b.n_dst)])
+        who = np.concatenate([np.repeat(own_dst, deg), own_dst])
+        own_dst = votes(b.n_src, idx, who)
+    b0 = blocks[0]
+    n = int(max(b0.src_gid.max() + 1, 1))
+    order = np.lexsort((b0.src_gid, own_dst))
+    perm = np.full(n, -1, np.int64)
+    perm[b0.src_gid[order]] = np.arange(b0.n_src)
+    return perm
 
 
 def synth_params(cfg):

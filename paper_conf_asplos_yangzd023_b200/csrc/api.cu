@@ -18,7 +18,12 @@ void* ctx_alloc(betty_ctx* c, size_t bytes, cudaStream_t s) {
     if (bytes == 0) bytes = 16;
     if (c->alloc) return c->alloc(bytes, (betty_stream)s, c->user);
     void* p = nullptr;
-    if (cudaMallocAsync(&p, bytes, s) != cudaSuccess) return nullptr;
+    if (cudaMallocAsync(&p, bytes, s) != cudaSuccess) {
+        // reported through the return value (BETTY_ENOMEM); consume the error so the next call's
+        // launch checks do not see it as a failure of their own
+        cudaGetLastError();
+        return nullptr;
+    }
     return p;
 }
 void ctx_free(betty_ctx* c, void* p, cudaStream_t s) {

@@ -49,6 +49,8 @@ def lib():
         L.synth_graph.argtypes = [i64, i64, i32, dbl, dbl, u64, ctypes.POINTER(P), ctypes.POINTER(P), P]
         L.synth_features.restype = None
         L.synth_features.argtypes = [i64, i32, i64, P, i32, dbl, dbl, u64, P]
+        L.synth_features_ids.restype = None
+        L.synth_features_ids.argtypes = [P, i64, i64, i32, i64, P, i32, dbl, dbl, u64, P]
         L.synth_seeds.restype = None
         L.synth_seeds.argtypes = [i64, i64, u64, P]
         L.synth_sample.restype = ctypes.c_int
@@ -116,6 +118,20 @@ def features(comm: np.ndarray, F: int, ld: int, kind: int = 0, signal: float = 0
     out = np.empty((n, ld), dtype=np.float32)
     lib().synth_features(n, F, ld, _ptr(np.ascontiguousarray(comm, dtype=np.int32)), kind, signal, p, seed,
                          _ptr(out))
+    return out
+
+
+def features_rows(comm: np.ndarray, F: int, ld: int, ids: Optional[np.ndarray] = None, row0: int = 0, n: int = 0,
+                  kind: int = 0, signal: float = 0.5, p: float = 0.0126, seed: int = 5) -> np.ndarray:
+    """Rows of `features(comm, ...)` for the nodes `ids` (or the range [row0, row0+n)) only: tables
+    too large for host memory (C5) are generated in chunks, and a sample's rows on their own."""
+    comm = np.ascontiguousarray(comm, dtype=np.int32)
+    if ids is not None:
+        ids = np.ascontiguousarray(ids, dtype=np.int32)
+        n = len(ids)
+    out = np.empty((n, ld), dtype=np.float32)
+    lib().synth_features_ids(None if ids is None else _ptr(ids), row0, n, F, ld, _ptr(comm), kind, signal, p, seed,
+                             _ptr(out))
     return out
 
 
@@ -224,7 +240,14 @@ CONFIGS = {
     # configs[3]: products-shaped, 5-layer SAGE-pool fanout 10 per layer
     "C4": Config("products-deep-pool", 2449029, 61859140, 100, 47, 256, 5, "pool", (10, 10, 10, 10, 10),
                  196615, (8,), 4000, 0.1, oversample=1.096),
+    # configs[4]: ogbn-papers100M-shaped, 3-layer SAGE-mean, fanout (5, 10, 15) (SURVEY.md §8(d) proposal),
+    # 1.2 M outputs, K 16..64; the 57 GB fp32 feature table is generated in chunks (features_rows)
+    "C5": Config("papers100M", 111059956, 800000000, 128, 172, 256, 3, "mean", (5, 10, 15), 1207179, (16, 32, 64),
+                 20000, 0.1),
 }
+
+# feature tables above this many bytes (fp32) are never materialised on the host
+HOST_FEATURE_LIMIT = 8 << 30
 
 
 def scaled(cfg: Config, frac: float, name: Optional[str] = None) -> Config:
@@ -239,17 +262,19 @@ def scaled(cfg: Config, frac: float, name: Optional[str] = None) -> Config:
 class Dataset:
     cfg: Config
     graph: Graph
-    feats: np.ndarray         # float32 [N, ld]
+    feats: Optional[np.ndarray]   # float32 [N, ld]; None when generated in chunks (features_rows)
     labels: np.ndarray        # int32 [N]
     seeds: np.ndarray         # int32 [n_out] ascending
     blocks: List[Block]       # block 0 (input) ... L-1 (output)
 
 
-def make(cfg: Config, with_features: bool = True) -> Dataset:
+def make(cfg: Config, with_features: Optional[bool] = True) -> Dataset:
     s = cfg.seeds
     g = graph(cfg.n, int(cfg.pairs * cfg.oversample), cfg.n_comm, cfg.mu, cfg.beta, s["graph"])
     sd = seeds(g.n, cfg.n_out, s["train"])
     blocks = sample(g, sd, cfg.fanouts, s["sample"])
+    if with_features is None:
+        with_features = cfg.n * cfg.ld * 4 <= HOST_FEATURE_LIMIT
     feats = features(g.comm, cfg.F, cfg.ld, cfg.feat_kind, seed=s["feat"]) if with_features else None
     labels = (g.comm % cfg.C).astype(np.int32)
     return Dataset(cfg, g, feats, labels, sd, blocks)

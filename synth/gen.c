@@ -194,24 +194,38 @@ static inline double gauss(uint64_t seed, uint64_t a, uint64_t b) {
 
 /* kind 0: N(0,1) + signal * community centroid (centroid ~ N(0,1) per (c,f));
  * kind 1: sparse 0/1 bag of words, Bernoulli(p) with community-specific words
- *         4x more likely (Cora-shaped).  Padding columns [F, ld) are zero. */
+ *         4x more likely (Cora-shaped).  Padding columns [F, ld) are zero.
+ * Row i is a pure function of (seed, node id, its community), so any subset of
+ * rows can be generated on its own (synth_features_ids). */
+static void feature_row(int64_t node, int32_t c, int32_t F, int64_t ld, int32_t kind, double signal, double p,
+                        uint64_t seed, float* row) {
+    for (int32_t f = 0; f < F; ++f) {
+        if (kind == 0) {
+            double v = gauss(seed, (uint64_t)node + 1000, (uint64_t)f) +
+                       signal * gauss(seed ^ 0xC0FFEEULL, (uint64_t)c, (uint64_t)f);
+            row[f] = (float)v;
+        } else {
+            double pf = ((f * 7 + c) % 16 == 0) ? 4.0 * p : 0.8 * p;
+            row[f] = u01(key3(seed, (uint64_t)node + 7, (uint64_t)f)) < pf ? 1.0f : 0.0f;
+        }
+    }
+    for (int64_t f = F; f < ld; ++f) row[f] = 0.0f;
+}
+
 void synth_features(int64_t N, int32_t F, int64_t ld, const int32_t* comm, int32_t kind,
                     double signal, double p, uint64_t seed, float* out) {
     #pragma omp parallel for schedule(static)
-    for (int64_t i = 0; i < N; ++i) {
-        float* row = out + i * ld;
-        int32_t c = comm[i];
-        for (int32_t f = 0; f < F; ++f) {
-            if (kind == 0) {
-                double v = gauss(seed, (uint64_t)i + 1000, (uint64_t)f) +
-                           signal * gauss(seed ^ 0xC0FFEEULL, (uint64_t)c, (uint64_t)f);
-                row[f] = (float)v;
-            } else {
-                double pf = ((f * 7 + c) % 16 == 0) ? 4.0 * p : 0.8 * p;
-                row[f] = u01(key3(seed, (uint64_t)i + 7, (uint64_t)f)) < pf ? 1.0f : 0.0f;
-            }
-        }
-        for (int64_t f = F; f < ld; ++f) row[f] = 0.0f;
+    for (int64_t i = 0; i < N; ++i) feature_row(i, comm[i], F, ld, kind, signal, p, seed, out + i * ld);
+}
+
+/* rows of the nodes ids[0..n) (ids == NULL: nodes row0 .. row0+n-1); comm is
+ * indexed by node id.  Row j of out is node ids[j]'s row of synth_features. */
+void synth_features_ids(const int32_t* ids, int64_t row0, int64_t n, int32_t F, int64_t ld, const int32_t* comm,
+                        int32_t kind, double signal, double p, uint64_t seed, float* out) {
+    #pragma omp parallel for schedule(static)
+    for (int64_t j = 0; j < n; ++j) {
+        const int64_t node = ids ? (int64_t)ids[j] : row0 + j;
+        feature_row(node, comm[node], F, ld, kind, signal, p, seed, out + j * ld);
     }
 }
 
