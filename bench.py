@@ -185,27 +185,6 @@ def build_inputs(args, rank, ws, device):
     return cfg, ds, time.time() - t0
 
 
-def device_features(cfg, ds, bf16: bool, align: int, device, chunk_rows: int = 1 << 22):
-    """The feature table in HBM (bf16 or fp32), rows padded to `align` bytes.  Tables too large for the
-    host (C5: 111 M x 128 fp32 = 57 GB) are generated in chunks of rows (synth.features_rows) and
-    converted on the device; the others are copied from the host array."""
-    import torch
-    import synth
-    dt = torch.bfloat16 if bf16 else torch.float32
-    esz = 2 if bf16 else 4
-    per = max(1, align // esz) if align > 0 else 1
-    ld = (cfg.ld + per - 1) // per * per
-    out = torch.zeros((cfg.n, ld), dtype=dt, device=device)
-    if ds.feats is not None:
-        out[:, :cfg.ld] = torch.as_tensor(ds.feats).to(device).to(dt)
-        return out
-    for r0 in range(0, cfg.n, chunk_rows):
-        n = min(chunk_rows, cfg.n - r0)
-        h = synth.features_rows(ds.graph.comm, cfg.F, cfg.ld, row0=r0, n=n, kind=cfg.feat_kind, seed=cfg.seeds["feat"])
-        out[r0:r0 + n, :cfg.ld] = torch.from_numpy(h).to(device).to(dt)
-    return out
-
-
 def oracle_inputs(cfg, ds, part):
     """Full-batch blocks and a feature array for the oracle's micro-batch 0 of `part`: the host table
     itself, or (C5) only the rows micro-batch 0 reads, with layer-0 ids remapped onto them."""
@@ -384,7 +363,8 @@ def main():
     costs = micro_batch_costs(part, args.K, ds.blocks[-1].indptr)
     my_k = lpt_assign(costs, ws)[rank]
 
-    feats = device_features(cfg, ds, args.mode == "bf16", args.feat_align, device)   # bf16: reading #17
+    import synth
+    feats = synth.features_device(cfg, ds, args.mode == "bf16", args.feat_align, device)   # bf16: reading #17
     host_gid0 = ds.blocks[0].src_gid
     if args.feat_layout == "owner":
         t_l = time.time()

@@ -280,6 +280,27 @@ def make(cfg: Config, with_features: Optional[bool] = True) -> Dataset:
     return Dataset(cfg, g, feats, labels, sd, blocks)
 
 
+def features_device(cfg: Config, ds: "Dataset", bf16: bool, align: int, device, chunk_rows: int = 1 << 22):
+    """The feature table as a torch tensor in HBM (bf16 or fp32), rows padded with zeros to a multiple
+    of `align` bytes (0: cfg.ld).  Tables too large for host memory (C5: 111 M x 128 fp32 = 57 GB)
+    are generated in chunks of rows (features_rows) and converted on the device; the others are
+    copied from ds.feats."""
+    import torch
+    dt = torch.bfloat16 if bf16 else torch.float32
+    esz = 2 if bf16 else 4
+    per = max(1, align // esz) if align > 0 else 1
+    ld = (cfg.ld + per - 1) // per * per
+    out = torch.zeros((cfg.n, ld), dtype=dt, device=device)
+    if ds.feats is not None:
+        out[:, :cfg.ld] = torch.as_tensor(ds.feats).to(device).to(dt)
+        return out
+    for r0 in range(0, cfg.n, chunk_rows):
+        n = min(chunk_rows, cfg.n - r0)
+        h = features_rows(ds.graph.comm, cfg.F, cfg.ld, row0=r0, n=n, kind=cfg.feat_kind, seed=cfg.seeds["feat"])
+        out[r0:r0 + n, :cfg.ld] = torch.from_numpy(h).to(device).to(dt)
+    return out
+
+
 def init_params(dims: Sequence[int], aggr: str, seed: int = 4) -> np.ndarray:
     """Xavier-uniform weights, zero... small uniform biases; flat fp32 in the
     layout of include/betty.h (per layer: [W_pool, b_pool] (pool only),
