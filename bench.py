@@ -346,12 +346,20 @@ def main():
     import torch
     import torch.distributed as dist
     import paper_conf_asplos_yangzd023_b200 as B
-    from paper_conf_asplos_yangzd023_b200.dist import allreduce_grad, lpt_assign, micro_batch_costs
+    from paper_conf_asplos_yangzd023_b200.dist import allreduce_grad, lpt_assign, micro_batch_costs, reg_rows
 
+    # BETTY_BENCH_ONE_GPU=1 (testing the multi-rank path on a one-GPU box): every rank on cuda:0 and
+    # gloo for the collectives -- timings of such a run are not bench values
+    one_gpu = os.environ.get("BETTY_BENCH_ONE_GPU", "0") == "1"
+    if one_gpu:
+        local = 0
     torch.cuda.set_device(local)
     device = torch.device("cuda", local)
     if ws > 1:
-        dist.init_process_group("nccl", device_id=device)
+        if one_gpu:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=device)
     cfg, ds, t_gen = build_inputs(args, rank, ws, device)
     ctx = B.betty_ctx_create(local)
     dev_blocks = B.blocks_to_device(ds.blocks, local)
@@ -395,6 +403,8 @@ def main():
     t0 = time.time()
     plan, args.group = create_plan(B, ctx, model, dev_blocks, dpart, args.K, my_k, args.group, flags)
     t_plan = time.time() - t0
+    if ws > 1 and not args.no_reg:
+        plan.set_reg_rows(*reg_rows(cfg.n_out, rank, ws))      # REG rows sharded across ranks
     info = plan.info()
     scale = 1.0 / cfg.n_out
     stream = torch.cuda.current_stream()
@@ -536,6 +546,8 @@ def main():
             "setup_s": {"generate": t_gen, "plan": t_plan},
             "memory_aware": mem_aware,
         }
+        if one_gpu and ws > 1:
+            line["note"] = "BETTY_BENCH_ONE_GPU: all ranks share cuda:0 over gloo (path test, not a bench value)"
         s = json.dumps(line)
         print(s, flush=True)
         if args.json_out:

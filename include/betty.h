@@ -118,6 +118,12 @@ BETTY_API int64_t betty_num_params(const betty_model* model);
  * reading #2): a repeat returns EINVAL.  Allocates reg's arrays; synchronizes
  * the stream once to learn nnz.  Result is bit-exact (integer). */
 BETTY_API betty_status betty_reg_build(betty_ctx* ctx, const betty_block* out_layer, betty_csr* reg, betty_stream stream);
+/* The REG rows [row0, row1) only (0 <= row0 <= row1 <= n_out), e.g. one rank's share when the
+ * rows are sharded across ranks: reg->n = row1 - row0, reg->indptr rebased to
+ * the slice, columns are GLOBAL output ids.  Row i of the slice equals row row0 + i of
+ * betty_reg_build's result, bit-exact.  Bad ranges return EINVAL. */
+BETTY_API betty_status betty_reg_build_rows(betty_ctx* ctx, const betty_block* out_layer, int64_t row0, int64_t row1,
+                                            betty_csr* reg, betty_stream stream);
 BETTY_API void betty_csr_free(betty_ctx* ctx, betty_csr* reg);
 
 /* a2 -- micro-batch extraction (batch-level partition, PAPER.md:535-547;
@@ -178,6 +184,13 @@ BETTY_API betty_status betty_plan_create(betty_ctx* ctx, const betty_model* mode
                                const int32_t* part, int64_t n_out, int32_t K, const int32_t* my_k, int32_t n_my,
                                int32_t group, int32_t flags, betty_plan** out, betty_stream stream);
 BETTY_API betty_status betty_plan_info_get(const betty_plan* plan, betty_plan_info* info);
+/* Restrict the in-step REG rebuild (BETTY_PLAN_REG) of this plan to output rows [row0, row1):
+ * with R ranks, rank r takes rows [r n_out / R, (r+1) n_out / R) so the REG work is sharded
+ * instead of repeated on every rank.  Synchronises `stream`, re-sizes the REG buffers (one
+ * sizing pass) and drops a captured graph (re-captured by the next betty_step).  EINVAL for a
+ * plan created without BETTY_PLAN_REG or a bad range. */
+BETTY_API betty_status betty_plan_set_reg_rows(betty_ctx* ctx, betty_plan* plan, int64_t row0, int64_t row1,
+                                               betty_stream stream);
 BETTY_API void betty_plan_destroy(betty_ctx* ctx, betty_plan* plan);
 
 /* One training step on this rank: for every micro-batch of the plan,

@@ -138,6 +138,20 @@ def betty_reg_build(ctx: Context, out_block: Block, stream=None):
         L.lib().betty_csr_free(ctx.h, ctypes.byref(csr))
 
 
+def betty_reg_build_rows(ctx: Context, out_block: Block, row0: int, row1: int, stream=None):
+    """a1 for output rows [row0, row1) only (one rank's share): (indptr rebased, col global, w)."""
+    ob = out_block.struct()
+    csr = L.betty_csr()
+    ctx.check(L.lib().betty_reg_build_rows(ctx.h, ctypes.byref(ob), row0, row1, ctypes.byref(csr), _stream(stream)),
+              "betty_reg_build_rows")
+    try:
+        return (_copy_out(csr.indptr, csr.n + 1, torch.int64, ctx.device),
+                _copy_out(csr.col, csr.nnz, torch.int32, ctx.device),
+                _copy_out(csr.w, csr.nnz, torch.int32, ctx.device))
+    finally:
+        L.lib().betty_csr_free(ctx.h, ctypes.byref(csr))
+
+
 def betty_extract_blocks(ctx: Context, full: Sequence[Block], part: torch.Tensor, K: int, k: int,
                          stream=None) -> List[Block]:
     """a2: micro-batch k of the K-way partition `part` (int32 cuda [n_out])."""
@@ -245,6 +259,11 @@ class Plan:
                              _copy_out(o.t_indptr, o.n_src + 1, torch.int64, d) if o.t_indptr else None,
                              _copy_out(o.t_indices, o.n_edges, torch.int32, d) if o.t_indptr else None))
         return res
+
+    def set_reg_rows(self, row0: int, row1: int, stream=None):
+        """Shard the in-step REG rebuild: this plan computes output rows [row0, row1) only."""
+        self.ctx.check(L.lib().betty_plan_set_reg_rows(self.ctx.h, self.h, row0, row1, _stream(stream)),
+                       "betty_plan_set_reg_rows")
 
     def probe(self, site: int):
         """Bracket the launches of one kernel site with CUDA events (see betty.h)."""

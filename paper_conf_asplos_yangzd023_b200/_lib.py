@@ -56,6 +56,7 @@ def lib() -> ctypes.CDLL:
         "betty_last_error": (ctypes.c_char_p, [vp]),
         "betty_num_params": (i64, [pp(betty_model)]),
         "betty_reg_build": (i32, [vp, pp(betty_block), pp(betty_csr), vp]),
+        "betty_reg_build_rows": (i32, [vp, pp(betty_block), i64, i64, pp(betty_csr), vp]),
         "betty_csr_free": (None, [vp, pp(betty_csr)]),
         "betty_extract_blocks": (i32, [vp, pp(betty_block), i32, vp, i64, i32, i32, pp(betty_block), vp]),
         "betty_block_free": (None, [vp, pp(betty_block), i32]),
@@ -66,6 +67,7 @@ def lib() -> ctypes.CDLL:
                                     pp(vp), vp]),
         "betty_plan_info_get": (i32, [vp, pp(betty_plan_info)]),
         "betty_plan_destroy": (None, [vp, vp]),
+        "betty_plan_set_reg_rows": (i32, [vp, vp, i64, i64, vp]),
         "betty_step": (i32, [vp, vp, vp, vp, i64, vp, f32, vp, vp, vp]),
         "betty_adam": (i32, [vp, vp, vp, vp, vp, i64, i32, f32, f32, f32, f32, i32, vp]),
         "betty_sync_check": (i32, [vp, vp]),
@@ -93,4 +95,5 @@ EXPORTED = ["betty_version", "betty_ctx_create", "betty_ctx_destroy", "betty_las
             "betty_sage_bwd", "betty_saved_free", "betty_plan_create", "betty_plan_info_get", "betty_plan_destroy",
             "betty_step", "betty_adam", "betty_sync_check", "betty_reg_partition", "betty_plan_probe",
             "betty_plan_probe_read", "betty_plan_group_blocks", "betty_test_gemm", "betty_mb_sizes",
-            "betty_mem_estimate", "betty_memory_aware_k", "betty_reg_partition_ex"]
+            "betty_mem_estimate", "betty_memory_aware_k", "betty_reg_partition_ex", "betty_reg_build_rows",
+            "betty_plan_set_reg_rows"]

@@ -299,13 +299,21 @@ struct RegBufs {
     int64_t ub_cap = 0, nnz_cap = 0;
 };
 
-static bool alloc_reg_phase1(Arena& A, const betty_block* ob, RegBufs* R) {
-    const int64_t n = ob->n_dst, ns = ob->n_src, E = ob->n_edges;
-    R->cnt = A.get<int64_t>(4);
+// REG rows [r0, r1) of the output block ob (the CSC always covers the whole block); uploads the
+// device counts {rows of the slice, n_src, n_edges, -, n_dst} on stream s.
+static bool alloc_reg_phase1(Arena& A, const betty_block* ob, int64_t r0, int64_t r1, RegBufs* R, cudaStream_t s) {
+    const int64_t n = r1 - r0, ns = ob->n_src, E = ob->n_edges;
+    R->cnt = A.get<int64_t>(5);
     RegArgs& a = R->a;
-    a.indptr = ob->indptr; a.idx = ob->indices;
-    a.n_rows_dev = R->cnt; a.n_cols_dev = R->cnt + 1; a.n_edges_dev = R->cnt + 2;
+    a.indptr = ob->indptr + r0; a.idx = ob->indices;
+    a.full_indptr = ob->indptr; a.full_rows_cap = std::max<int64_t>(ob->n_dst, 1); a.row0 = r0;
+    a.n_rows_dev = R->cnt; a.n_cols_dev = R->cnt + 1; a.n_edges_dev = R->cnt + 2; a.n_full_rows_dev = R->cnt + 4;
     a.rows_cap = std::max<int64_t>(n, 1); a.cols_cap = std::max<int64_t>(ns, 1); a.edges_cap = std::max<int64_t>(E, 1);
+    if (R->cnt) {
+        const int64_t h[5] = {n, ns, E, 0, ob->n_dst};
+        cudaMemcpyAsync(R->cnt, h, sizeof(h), cudaMemcpyHostToDevice, s);
+        cudaStreamSynchronize(s);       // h is a host stack array
+    }
     a.t_indptr = A.get<int64_t>(ns + 1);
     a.t_idx = A.get<int32_t>(E);
     a.tcnt = A.get<int32_t>(ns);
@@ -318,16 +326,22 @@ static bool alloc_reg_phase1(Arena& A, const betty_block* ob, RegBufs* R) {
 
 extern "C" betty_status betty_reg_build(betty_ctx* c, const betty_block* ob, betty_csr* reg, betty_stream stream) {
     if (!c) return BETTY_EINVAL;
+    if (!ob) return fail(c, BETTY_EINVAL, "reg: null argument");
+    return betty_reg_build_rows(c, ob, 0, ob->n_dst, reg, stream);
+}
+
+extern "C" betty_status betty_reg_build_rows(betty_ctx* c, const betty_block* ob, int64_t row0, int64_t row1,
+                                             betty_csr* reg, betty_stream stream) {
+    if (!c) return BETTY_EINVAL;
     cudaStream_t s = (cudaStream_t)stream;
     if (!ob || !reg || !ob->indptr || (ob->n_edges > 0 && !ob->indices) || ob->n_dst < 0)
         return fail(c, BETTY_EINVAL, "reg: null argument");
+    if (row0 < 0 || row1 < row0 || row1 > ob->n_dst) return fail(c, BETTY_EINVAL, "reg: bad row range");
     if (ob->n_src >= INT32_MAX || ob->n_dst >= INT32_MAX) return fail(c, BETTY_EOVERFLOW, "reg: sizes exceed int32");
     memset(reg, 0, sizeof(*reg));
     Arena A{c, s};
     RegBufs R;
-    if (!alloc_reg_phase1(A, ob, &R)) { A.release(); return fail(c, BETTY_ENOMEM, "reg: allocation failed"); }
-    int64_t h[4] = {ob->n_dst, ob->n_src, ob->n_edges, 0};
-    cudaMemcpyAsync(R.cnt, h, sizeof(h), cudaMemcpyHostToDevice, s);
+    if (!alloc_reg_phase1(A, ob, row0, row1, &R, s)) { A.release(); return fail(c, BETTY_ENOMEM, "reg: allocation failed"); }
     reg_phase1(c, R.a, s);
     int64_t ub_total = 0;
     cudaMemcpyAsync(&ub_total, R.a.ub_total_dev, sizeof(int64_t), cudaMemcpyDeviceToHost, s);
@@ -335,7 +349,7 @@ extern "C" betty_status betty_reg_build(betty_ctx* c, const betty_block* ob, bet
     if (st) { A.release(); return st; }
     R.a.tcol = A.get<int32_t>(ub_total);
     R.a.tw = A.get<int32_t>(ub_total);
-    reg->indptr = (int64_t*)ctx_alloc(c, sizeof(int64_t) * (ob->n_dst + 1), s);
+    reg->indptr = (int64_t*)ctx_alloc(c, sizeof(int64_t) * (row1 - row0 + 1), s);
     R.a.out_indptr = reg->indptr;
     int64_t* nnz_dev = A.get<int64_t>(1);
     R.a.nnz_total_dev = nnz_dev;
@@ -351,7 +365,7 @@ extern "C" betty_status betty_reg_build(betty_ctx* c, const betty_block* ob, bet
     reg->w = (int32_t*)ctx_alloc(c, sizeof(int32_t) * std::max<int64_t>(nnz, 1), s);
     if (!reg->col || !reg->w) { A.release(); betty_csr_free(c, reg); return fail(c, BETTY_ENOMEM, "reg: allocation failed"); }
     reg_phase3(c, R.a, reg->col, reg->w, nnz, s);
-    reg->n = ob->n_dst;
+    reg->n = row1 - row0;
     reg->nnz = nnz;
     A.release();
     return sync_check(c, s);
@@ -564,6 +578,52 @@ __global__ void k_max_deg(const int64_t* __restrict__ indptr, int64_t n, int* ou
     atomicMax(out, mx);
 }
 
+// Size and allocate the in-step REG of output rows [r0, r1) (phases 1-2 run once here, synchronising).
+static betty_status plan_reg_setup(betty_ctx* c, betty_plan* p, const betty_block* ob, int64_t r0, int64_t r1,
+                                   cudaStream_t s) {
+    Arena& A = *p->arena;
+    c->lane = 1;            // size the side lane's scan scratch with the REG's own calls
+    RegBufs R;
+    if (!alloc_reg_phase1(A, ob, r0, r1, &R, s)) { c->lane = 0; return fail(c, BETTY_ENOMEM, "plan: REG alloc"); }
+    reg_phase1(c, R.a, s);
+    int64_t ub = 0;
+    cudaMemcpyAsync(&ub, R.a.ub_total_dev, sizeof(int64_t), cudaMemcpyDeviceToHost, s);
+    betty_status st = sync_check(c, s);
+    if (st) { c->lane = 0; return st; }
+    R.ub_cap = ub;
+    R.a.tcol = A.get<int32_t>(ub);
+    R.a.tw = A.get<int32_t>(ub);
+    R.a.out_indptr = A.get<int64_t>(r1 - r0 + 1);
+    R.a.nnz_total_dev = A.get<int64_t>(1);
+    if (!A.ok) { c->lane = 0; return fail(c, BETTY_ENOMEM, "plan: REG alloc"); }
+    reg_phase2(c, R.a, s);
+    int64_t nnz = 0;
+    cudaMemcpyAsync(&nnz, R.a.nnz_total_dev, sizeof(int64_t), cudaMemcpyDeviceToHost, s);
+    if ((st = sync_check(c, s))) { c->lane = 0; return st; }
+    R.nnz_cap = nnz;
+    R.col = A.get<int32_t>(nnz);
+    R.w = A.get<int32_t>(nnz);
+    c->lane = 0;
+    if (!A.ok) return fail(c, BETTY_ENOMEM, "plan: REG alloc");
+    p->R = R;
+    p->with_reg = true;
+    p->info.reg_nnz = nnz;
+    p->info.arena_bytes = A.bytes + p->sb.bytes;
+    return BETTY_OK;
+}
+
+extern "C" betty_status betty_plan_set_reg_rows(betty_ctx* c, betty_plan* p, int64_t row0, int64_t row1,
+                                                betty_stream stream) {
+    if (!c) return BETTY_EINVAL;
+    if (!p || !p->side) return fail(c, BETTY_EINVAL, "plan_set_reg_rows: plan without BETTY_PLAN_REG");
+    const betty_block* ob = &p->reg_block;
+    if (row0 < 0 || row1 < row0 || row1 > ob->n_dst) return fail(c, BETTY_EINVAL, "plan_set_reg_rows: bad row range");
+    cudaStream_t s = (cudaStream_t)stream;
+    if (cudaStreamSynchronize(s) != cudaSuccess) return fail(c, BETTY_ECUDA, "plan_set_reg_rows: stream");
+    if (p->gexec) { cudaGraphExecDestroy(p->gexec); p->gexec = nullptr; }     // buffers change: re-capture
+    return plan_reg_setup(c, p, ob, row0, row1, s);
+}
+
 extern "C" betty_status betty_plan_create(betty_ctx* c, const betty_model* model, const betty_block* full, int32_t L,
                                           const int32_t* part, int64_t n_out, int32_t K, const int32_t* my_k,
                                           int32_t n_my, int32_t group, int32_t flags, betty_plan** out,
@@ -691,7 +751,7 @@ extern "C" betty_status betty_plan_create(betty_ctx* c, const betty_model* model
         mx = std::max(mx, (int64_t)p->c * ((n_out + 1023) / 1024 + 1));
         ensure_scan_scratch(c, mx, s);
     }
-    // ---- REG inside the step (once here to size its buffers)
+    // ---- REG inside the step (once here to size its buffers): all rows until betty_plan_set_reg_rows
     if (flags & BETTY_PLAN_REG) {
         if (cudaStreamCreateWithFlags(&p->side, cudaStreamNonBlocking) != cudaSuccess ||
             cudaEventCreateWithFlags(&p->ev_fork, cudaEventDisableTiming) != cudaSuccess ||
@@ -699,32 +759,8 @@ extern "C" betty_status betty_plan_create(betty_ctx* c, const betty_model* model
             betty_plan_destroy(c, p);
             return fail(c, BETTY_ECUDA, "plan: side stream");
         }
-        c->lane = 1;            // size the side lane's scan scratch with the REG's own calls
-        p->with_reg = true;
-        const betty_block* ob = &full[L - 1];
-        if (!alloc_reg_phase1(A, ob, &p->R)) { c->lane = 0; betty_plan_destroy(c, p); return fail(c, BETTY_ENOMEM, "plan: REG alloc"); }
-        int64_t h[4] = {ob->n_dst, ob->n_src, ob->n_edges, 0};
-        cudaMemcpyAsync(p->R.cnt, h, sizeof(h), cudaMemcpyHostToDevice, s);
-        reg_phase1(c, p->R.a, s);
-        int64_t ub = 0;
-        cudaMemcpyAsync(&ub, p->R.a.ub_total_dev, sizeof(int64_t), cudaMemcpyDeviceToHost, s);
-        if ((st = sync_check(c, s))) { c->lane = 0; betty_plan_destroy(c, p); return st; }
-        p->R.ub_cap = ub;
-        p->R.a.tcol = A.get<int32_t>(ub);
-        p->R.a.tw = A.get<int32_t>(ub);
-        p->R.a.out_indptr = A.get<int64_t>(ob->n_dst + 1);
-        p->R.a.nnz_total_dev = A.get<int64_t>(1);
-        if (!A.ok) { c->lane = 0; betty_plan_destroy(c, p); return fail(c, BETTY_ENOMEM, "plan: REG alloc"); }
-        reg_phase2(c, p->R.a, s);
-        int64_t nnz = 0;
-        cudaMemcpyAsync(&nnz, p->R.a.nnz_total_dev, sizeof(int64_t), cudaMemcpyDeviceToHost, s);
-        if ((st = sync_check(c, s))) { c->lane = 0; betty_plan_destroy(c, p); return st; }
-        p->R.nnz_cap = nnz;
-        p->R.col = A.get<int32_t>(nnz);
-        p->R.w = A.get<int32_t>(nnz);
-        if (!A.ok) { c->lane = 0; betty_plan_destroy(c, p); return fail(c, BETTY_ENOMEM, "plan: REG alloc"); }
-        p->info.reg_nnz = nnz;
-        c->lane = 0;
+        p->reg_block = full[L - 1];
+        if ((st = plan_reg_setup(c, p, &p->reg_block, 0, full[L - 1].n_dst, s))) { betty_plan_destroy(c, p); return st; }
     }
     // ---- launches per step: capture the body once into a throw-away graph
     {

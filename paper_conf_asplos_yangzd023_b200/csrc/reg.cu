@@ -60,8 +60,10 @@ __global__ void k_reg_ub(const int64_t* __restrict__ indptr, const int32_t* __re
 // is ascending, so a candidate j at offset t of its column lands at t - [j > i].
 __device__ __forceinline__ void reg_expand(const int64_t* __restrict__ indptr, const int32_t* __restrict__ idx,
                                            const int64_t* __restrict__ t_indptr, const int32_t* __restrict__ t_idx,
-                                           int64_t i, int32_t* buf, int tid, int nthr, int* s_pre, int64_t* s_cb) {
+                                           int64_t i, int64_t row0, int32_t* buf, int tid, int nthr, int* s_pre,
+                                           int64_t* s_cb) {
     const int64_t rb = indptr[i], re = indptr[i + 1];
+    const int32_t gi = (int32_t)(row0 + i);             // the row's global id: its own column entry
     const int lane = tid & 31;
     int64_t o = 0;
     for (int64_t e0 = rb; e0 < re; e0 += 32) {
@@ -89,7 +91,7 @@ __device__ __forceinline__ void reg_expand(const int64_t* __restrict__ indptr, c
             }
             const int t = f - s_pre[lo];
             const int32_t j = t_idx[s_cb[lo] + t];
-            if (j != (int32_t)i) buf[o + (s_pre[lo] - lo) + t - (j > (int32_t)i ? 1 : 0)] = j;
+            if (j != gi) buf[o + (s_pre[lo] - lo) + t - (j > gi ? 1 : 0)] = j;
         }
         o += total - n;
         if (nthr > 32) __syncthreads(); else __syncwarp();
@@ -219,6 +221,7 @@ __global__ void __launch_bounds__(256) k_reg_rows_warp(const int64_t* __restrict
                                                        const int32_t* __restrict__ idx,
                                                        const int64_t* __restrict__ t_indptr,
                                                        const int32_t* __restrict__ t_idx, const int64_t* n_rows_dev,
+                                                       int64_t row0,
                                                        const int64_t* __restrict__ ub, const int64_t* __restrict__ off,
                                                        int32_t* __restrict__ tcol, int32_t* __restrict__ tw,
                                                        int64_t* __restrict__ nnz) {
@@ -232,7 +235,7 @@ __global__ void __launch_bounds__(256) k_reg_rows_warp(const int64_t* __restrict
         const int64_t u = ub[i];
         if (u > REG_WARP_MAX) continue;                 // handled by the CTA kernel
         if (u == 0) { if (lane == 0) nnz[i] = 0; continue; }
-        reg_expand(indptr, idx, t_indptr, t_idx, i, buf[w], lane, 32, s_pre[w], s_cb[w]);
+        reg_expand(indptr, idx, t_indptr, t_idx, i, row0, buf[w], lane, 32, s_pre[w], s_cb[w]);
         if (u <= 32) {               // sort + run-length encode in registers
             int32_t x = lane < u ? buf[w][lane] : INT_MAX;
             x = warp_bitonic32(x);
@@ -258,7 +261,7 @@ __global__ void __launch_bounds__(256) k_reg_rows_warp(const int64_t* __restrict
 __global__ void __launch_bounds__(1024) k_reg_rows_cta(const int64_t* __restrict__ indptr,
                                                        const int32_t* __restrict__ idx,
                                                        const int64_t* __restrict__ t_indptr,
-                                                       const int32_t* __restrict__ t_idx,
+                                                       const int32_t* __restrict__ t_idx, int64_t row0,
                                                        const int64_t* __restrict__ ub, const int64_t* __restrict__ off,
                                                        const int64_t* big, const int* big_cnt,
                                                        int32_t* __restrict__ tcol, int32_t* __restrict__ tw,
@@ -272,7 +275,7 @@ __global__ void __launch_bounds__(1024) k_reg_rows_cta(const int64_t* __restrict
         const int64_t i = big[t];
         const int64_t u = ub[i];
         if (u > REG_CTA_MAX) { if (threadIdx.x == 0) nnz[i] = 0; continue; }
-        reg_expand(indptr, idx, t_indptr, t_idx, i, sbuf, threadIdx.x, blockDim.x, s_pre, s_cb);
+        reg_expand(indptr, idx, t_indptr, t_idx, i, row0, sbuf, threadIdx.x, blockDim.x, s_pre, s_cb);
         int P = 1024;
         while (P < u) P <<= 1;
         for (int q = (int)u + threadIdx.x; q < P; q += blockDim.x) sbuf[q] = INT_MAX;
@@ -306,8 +309,8 @@ void init_reg_attrs() {
 }
 
 void reg_phase1(betty_ctx* c, const RegArgs& a, cudaStream_t s) {
-    csr_transpose(c, a.indptr, a.idx, a.n_rows_dev, a.n_cols_dev, a.n_edges_dev, a.rows_cap, a.cols_cap, a.edges_cap,
-                  a.t_indptr, a.t_idx, a.tcnt, true, s);
+    csr_transpose(c, a.full_indptr, a.idx, a.n_full_rows_dev, a.n_cols_dev, a.n_edges_dev, a.full_rows_cap, a.cols_cap,
+                  a.edges_cap, a.t_indptr, a.t_idx, a.tcnt, true, s);
     const int gw = (int)std::max<int64_t>(1, std::min<int64_t>((a.rows_cap * 32 + 255) / 256, (int64_t)c->num_sms * 16));
     k_reset_big<<<1, 1, 0, s>>>(c->L().big_count);
     k_reg_ub<<<gw, 256, 0, s>>>(a.indptr, a.idx, a.t_indptr, a.n_rows_dev, a.ub, c->L().big_list, c->L().big_count,
@@ -317,9 +320,9 @@ void reg_phase1(betty_ctx* c, const RegArgs& a, cudaStream_t s) {
 
 void reg_phase2(betty_ctx* c, const RegArgs& a, cudaStream_t s) {
     const int gw = (int)std::max<int64_t>(1, std::min<int64_t>((a.rows_cap * 32 + 255) / 256, (int64_t)c->num_sms * 16));
-    k_reg_rows_warp<<<gw, 256, 0, s>>>(a.indptr, a.idx, a.t_indptr, a.t_idx, a.n_rows_dev, a.ub, a.off, a.tcol, a.tw,
-                                       a.row_nnz);
-    k_reg_rows_cta<<<c->num_sms, 1024, REG_CTA_MAX * 4, s>>>(a.indptr, a.idx, a.t_indptr, a.t_idx, a.ub, a.off,
+    k_reg_rows_warp<<<gw, 256, 0, s>>>(a.indptr, a.idx, a.t_indptr, a.t_idx, a.n_rows_dev, a.row0, a.ub, a.off, a.tcol,
+                                       a.tw, a.row_nnz);
+    k_reg_rows_cta<<<c->num_sms, 1024, REG_CTA_MAX * 4, s>>>(a.indptr, a.idx, a.t_indptr, a.t_idx, a.row0, a.ub, a.off,
                                                             c->L().big_list, c->L().big_count, a.tcol, a.tw, a.row_nnz);
     scan_i64(c, a.row_nnz, a.out_indptr, a.n_rows_dev, 0, a.rows_cap, a.nnz_total_dev, s);
 }

@@ -7,12 +7,19 @@ struct betty_ctx;
 namespace betty {
 
 struct RegArgs {
-    const int64_t* indptr;      // output block CSR (rows = outputs)
+    // The REG rows [row0, row0 + n_rows) of the output block: `indptr` points at the block's
+    // indptr + row0 (offsets stay absolute into idx); the CSC is built from the whole block
+    // (full_indptr, n_full_rows), since a row's candidates are every output sharing a source.
+    const int64_t* indptr;      // output block CSR rows of the slice (rows = outputs)
     const int32_t* idx;         // full-batch src positions
-    const int64_t* n_rows_dev;  // device counts
+    const int64_t* n_rows_dev;  // device counts: rows of the slice
     const int64_t* n_cols_dev;
-    const int64_t* n_edges_dev;
+    const int64_t* n_edges_dev; // edges of the whole block
     int64_t rows_cap, cols_cap, edges_cap;
+    const int64_t* full_indptr; // the whole output block
+    const int64_t* n_full_rows_dev;
+    int64_t full_rows_cap;
+    int64_t row0;               // global id of the slice's first row (diagonal exclusion)
     int64_t* t_indptr;          // [cols_cap+1]
     int32_t* t_idx;             // [edges_cap]
     int32_t* tcnt;              // [cols_cap]

@@ -37,6 +37,12 @@ def lpt_assign(costs: Sequence[float], world: int) -> List[List[int]]:
     return [sorted(x) for x in out]
 
 
+def reg_rows(n_out: int, rank: int, world: int):
+    """This rank's share [row0, row1) of the REG rows: the in-step REG rebuild is sharded by output
+    rows instead of repeated on every rank (contiguous, sizes differ by at most one)."""
+    return n_out * rank // world, n_out * (rank + 1) // world
+
+
 def allreduce_grad(grad, group=None):
     """The one exchange step of a training step: sum of the ranks' gradients."""
     import torch.distributed as dist

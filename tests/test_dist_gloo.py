@@ -12,7 +12,7 @@ import torch.multiprocessing as mp
 
 import oracle
 import synth
-from paper_conf_asplos_yangzd023_b200.dist import allreduce_grad, lpt_assign, micro_batch_costs
+from paper_conf_asplos_yangzd023_b200.dist import allreduce_grad, lpt_assign, micro_batch_costs, reg_rows
 from tests.helpers import tiny
 
 DIMS = [6, 10, 4]
@@ -37,8 +37,19 @@ def _worker(rank, world, port, q):
     grad, loss = oracle.step(DIMS, "mean", False, blocks, part, K, mine, params, feats, labels, 1.0 / len(sd))
     t = torch.tensor(np.concatenate([grad, [loss]]))
     allreduce_grad(t)
+    # row-sharded REG: each rank's share of the rows, gathered, is the whole REG
+    rp, rc, rw = oracle.reg(blocks[-1].n_src, blocks[-1].indptr, blocks[-1].nbr_pos)
+    r0, r1 = reg_rows(len(sd), rank, world)
+    shares = [None] * world
+    dist.all_gather_object(shares, (r0, r1, rp[r0:r1 + 1] - rp[r0], rc[rp[r0]:rp[r1]], rw[rp[r0]:rp[r1]]))
     if rank == 0:
         full, lfull, _ = oracle.sage(DIMS, "mean", False, blocks, params, feats, labels, 1.0 / len(sd))
+        assert [s_[0] for s_ in shares] == [0, shares[0][1]] and shares[-1][1] == len(sd)
+        ip = np.concatenate([[0]] + [s_[2][1:] + off for s_, off in
+                                     zip(shares, np.cumsum([0] + [s_[2][-1] for s_ in shares[:-1]]))])
+        np.testing.assert_array_equal(ip, rp)
+        np.testing.assert_array_equal(np.concatenate([s_[3] for s_ in shares]), rc)
+        np.testing.assert_array_equal(np.concatenate([s_[4] for s_ in shares]), rw)
         q.put((t.numpy(), full, lfull, mine))
     dist.destroy_process_group()
 
@@ -51,6 +62,15 @@ def test_lpt_assign_properties():
     assert max(loads) - min(loads) <= max(costs)
     assert lpt_assign(costs, 3) == a                       # deterministic
     assert lpt_assign(costs, 1) == [list(range(7))]
+
+
+def test_reg_rows_cover_every_row_once():
+    for n in (0, 1, 7, 120, 196615):
+        for world in (1, 2, 3, 8):
+            shares = [reg_rows(n, r, world) for r in range(world)]
+            assert shares[0][0] == 0 and shares[-1][1] == n
+            assert all(a[1] == b[0] for a, b in zip(shares, shares[1:]))
+            assert max(b - a for a, b in shares) - min(b - a for a, b in shares) <= 1
 
 
 def test_two_rank_allreduce_equals_full_batch():

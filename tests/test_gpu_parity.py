@@ -65,6 +65,58 @@ def test_reg_random_small(B, ctx, seed):
     reg_equal(B, ctx, B.blocks_to_device(blocks)[-1], blocks[-1])
 
 
+@pytest.mark.parametrize("world", [1, 2, 3, 8])
+def test_reg_row_shards(B, ctx, world):
+    """Row-sharded REG (one share per rank): every rank's rows [r n / R, (r+1) n / R)
+    equal the oracle's REG rows, bit-exact, with global column ids; an empty share and a bad range."""
+    g, sd, blocks, feats, labels = tiny(n=500, pairs=3000, fanouts=(4, 7), n_out=120, seed=7)
+    dev = B.blocks_to_device(blocks)[-1]
+    rp, rc, rw = oracle.reg(blocks[-1].n_src, blocks[-1].indptr, blocks[-1].nbr_pos)
+    n = blocks[-1].n_dst
+    for r in range(world):
+        r0, r1 = r * n // world, (r + 1) * n // world
+        ip, col, w = B.betty_reg_build_rows(ctx, dev, r0, r1)
+        np.testing.assert_array_equal(ip.cpu().numpy(), rp[r0:r1 + 1] - rp[r0])
+        np.testing.assert_array_equal(col.cpu().numpy(), rc[rp[r0]:rp[r1]])
+        np.testing.assert_array_equal(w.cpu().numpy(), rw[rp[r0]:rp[r1]])
+    ip, col, w = B.betty_reg_build_rows(ctx, dev, 5, 5)           # empty share
+    assert ip.tolist() == [0] and col.numel() == 0
+    with pytest.raises(B.BettyError):
+        B.betty_reg_build_rows(ctx, dev, 10, n + 1)
+
+
+def test_plan_reg_rows(B, ctx):
+    """A plan's in-step REG restricted to one rank's rows: sized to that share's nnz, and the step
+    (graph replay included) still produces the oracle's gradient."""
+    g, sd, blocks, feats, labels = tiny(n=400, pairs=2000, fanouts=(3, 5), n_out=60, F=8, C=4, seed=3)
+    dims = [8, 16, 4]
+    dev = B.blocks_to_device(blocks)
+    K = 3
+    part = synth.random_partition(len(sd), K, 1)
+    params = synth.init_params(dims, "mean", seed=2)
+    og, ol = oracle.step(dims, "mean", False, blocks, part, K, list(range(K)), params, feats, labels, 1.0 / len(sd))
+    rp, rc, rw = oracle.reg(blocks[-1].n_src, blocks[-1].indptr, blocks[-1].nbr_pos)
+    model = B.Model(dims, "mean", "fp32", "fp32")
+    plan = B.betty_plan_create(ctx, model, dev, torch.as_tensor(part).cuda(), K, list(range(K)), group=0,
+                               flags=B.PLAN_GRAPH | B.PLAN_REG)
+    assert plan.info()["reg_nnz"] == len(rc)
+    P = torch.as_tensor(params).cuda()
+    X = torch.as_tensor(feats).cuda()
+    Y = torch.as_tensor(labels).cuda()
+    for r0, r1 in ((0, 60), (20, 40), (59, 60)):
+        plan.set_reg_rows(r0, r1)
+        assert plan.info()["reg_nnz"] == rp[r1] - rp[r0]
+        for rep in range(2):
+            grad = torch.zeros_like(P)
+            loss = torch.zeros(1, device="cuda")
+            B.betty_step(ctx, plan, P, X, Y, 1.0 / len(sd), grad, loss)
+            B.betty_sync_check(ctx)
+            assert_close(grad.cpu().numpy(), og, 1e-5, f"rows {r0}:{r1} rep {rep}")
+    with pytest.raises(B.BettyError):
+        plan.set_reg_rows(0, 61)
+    plan.free()
+
+
 def test_reg_rejects_duplicate_edges(B, ctx):
     blk = B.Block(2, 3, torch.tensor([0, 2, 3], dtype=torch.int64, device="cuda"),
                   torch.tensor([1, 1, 2], dtype=torch.int32, device="cuda"),

@@ -33,18 +33,13 @@ def main():
     cfg = synth.CONFIGS[a.config]
     if a.scale != 1.0:
         cfg = synth.scaled(cfg, a.scale)
-    ds = synth.make(cfg)
+    ds = synth.make(cfg, with_features=None)
     ctx = B.betty_ctx_create(0)
     dev = B.blocks_to_device(ds.blocks)
     ip, col, w = B.betty_reg_build(ctx, dev[-1])
     part = B.betty_reg_partition(ip.cpu().numpy(), col.cpu().numpy(), w.cpu().numpy(), a.K, method="multilevel")
     dpart = torch.as_tensor(part).cuda()
-    feats = torch.as_tensor(ds.feats).cuda()
-    if a.mode == "bf16":
-        feats = feats.to(torch.bfloat16).contiguous()
-    sys.path.insert(0, ROOT)
-    from bench import pad_rows
-    feats = pad_rows(feats, a.feat_align)
+    feats = synth.features_device(cfg, ds, a.mode == "bf16", a.feat_align, "cuda")
     labels = torch.as_tensor(ds.labels).cuda()
     model = B.Model(cfg.dims, cfg.aggr, a.mode, a.mode)
     params = torch.as_tensor(synth.init_params(cfg.dims, cfg.aggr, seed=cfg.seeds["init"])).cuda()
