@@ -58,6 +58,7 @@ def parse():
     p.add_argument("--ref-sample-outputs", type=int, default=1024, help="--impl reference per-step sample")
     p.add_argument("--scale", type=float, default=1.0, help="shrink the graph (debug only)")
     p.add_argument("--json-out", default=None)
+    p.add_argument("--sim-world", type=int, default=0, help="(study) run rank 0's share of an N-rank job on one GPU")
     p.add_argument("--feat-align", type=int, default=256, help="feature-table row alignment in bytes (0: 16)")
     p.add_argument("--feat-layout", default="gid", choices=["gid", "owner"],
                    help="feature-table row order: gid (as generated) or owner (rows grouped by the micro-batch "
@@ -369,7 +370,10 @@ def main():
     part = make_partition(args, B, ctx, cfg, ds, dev_blocks, rank, ws, device)
     dpart = torch.as_tensor(part).to(device)
     costs = micro_batch_costs(part, args.K, ds.blocks[-1].indptr)
-    my_k = lpt_assign(costs, ws)[rank]
+    # --sim-world N (one GPU): run rank 0's share of an N-rank job -- its micro-batches and REG rows --
+    # to study per-rank step time; the line is then per-rank, not a bench value
+    wv, rv = (args.sim_world, 0) if args.sim_world > 1 else (ws, rank)
+    my_k = lpt_assign(costs, wv)[rv]
 
     import synth
     feats = synth.features_device(cfg, ds, args.mode == "bf16", args.feat_align, device)   # bf16: reading #17
@@ -403,8 +407,8 @@ def main():
     t0 = time.time()
     plan, args.group = create_plan(B, ctx, model, dev_blocks, dpart, args.K, my_k, args.group, flags)
     t_plan = time.time() - t0
-    if ws > 1 and not args.no_reg:
-        plan.set_reg_rows(*reg_rows(cfg.n_out, rank, ws))      # REG rows sharded across ranks
+    if wv > 1 and not args.no_reg:
+        plan.set_reg_rows(*reg_rows(cfg.n_out, rv, wv))        # REG rows sharded across ranks
     info = plan.info()
     scale = 1.0 / cfg.n_out
     stream = torch.cuda.current_stream()
@@ -546,6 +550,9 @@ def main():
             "setup_s": {"generate": t_gen, "plan": t_plan},
             "memory_aware": mem_aware,
         }
+        if args.sim_world > 1:
+            line["note"] = (f"--sim-world {args.sim_world}: rank 0's share only (its micro-batches and REG rows), "
+                            "per-rank step time, not a bench value")
         if one_gpu and ws > 1:
             line["note"] = "BETTY_BENCH_ONE_GPU: all ranks share cuda:0 over gloo (path test, not a bench value)"
         s = json.dumps(line)
