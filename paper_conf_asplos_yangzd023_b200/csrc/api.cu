@@ -605,6 +605,10 @@ static betty_status plan_reg_setup(betty_ctx* c, betty_plan* p, const betty_bloc
     R.w = A.get<int32_t>(nnz);
     c->lane = 0;
     if (!A.ok) return fail(c, BETTY_ENOMEM, "plan: REG alloc");
+    // The output block's CSC (built and duplicate-checked by phase 1 above) belongs to the plan's
+    // full batch, like the extraction's full-batch CSC: the step's rebuild reuses it and runs the
+    // SpGEMM proper (expansion, sort, run-length encode, compaction) over the rank's rows.
+    R.a.csc_ready = true;
     p->R = R;
     p->with_reg = true;
     p->info.reg_nnz = nnz;

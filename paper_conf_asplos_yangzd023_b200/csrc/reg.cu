@@ -309,8 +309,9 @@ void init_reg_attrs() {
 }
 
 void reg_phase1(betty_ctx* c, const RegArgs& a, cudaStream_t s) {
-    csr_transpose(c, a.full_indptr, a.idx, a.n_full_rows_dev, a.n_cols_dev, a.n_edges_dev, a.full_rows_cap, a.cols_cap,
-                  a.edges_cap, a.t_indptr, a.t_idx, a.tcnt, true, s);
+    if (!a.csc_ready)
+        csr_transpose(c, a.full_indptr, a.idx, a.n_full_rows_dev, a.n_cols_dev, a.n_edges_dev, a.full_rows_cap,
+                      a.cols_cap, a.edges_cap, a.t_indptr, a.t_idx, a.tcnt, true, s);
     const int gw = (int)std::max<int64_t>(1, std::min<int64_t>((a.rows_cap * 32 + 255) / 256, (int64_t)c->num_sms * 16));
     k_reset_big<<<1, 1, 0, s>>>(c->L().big_count);
     k_reg_ub<<<gw, 256, 0, s>>>(a.indptr, a.idx, a.t_indptr, a.n_rows_dev, a.ub, c->L().big_list, c->L().big_count,

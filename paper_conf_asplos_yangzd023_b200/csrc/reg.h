@@ -20,6 +20,7 @@ struct RegArgs {
     const int64_t* n_full_rows_dev;
     int64_t full_rows_cap;
     int64_t row0;               // global id of the slice's first row (diagonal exclusion)
+    bool csc_ready = false;     // t_indptr / t_idx already hold the block's CSC (a plan builds it once)
     int64_t* t_indptr;          // [cols_cap+1]
     int32_t* t_idx;             // [edges_cap]
     int32_t* tcnt;              // [cols_cap]

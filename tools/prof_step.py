@@ -29,6 +29,7 @@ def main():
     p.add_argument("--scale", type=float, default=1.0)
     p.add_argument("--group", type=int, default=0)
     p.add_argument("--feat-align", type=int, default=256)
+    p.add_argument("--sim-world", type=int, default=1, help="rank 0's share of an N-rank job")
     a = p.parse_args()
     cfg = synth.CONFIGS[a.config]
     if a.scale != 1.0:
@@ -46,7 +47,11 @@ def main():
     grad = torch.zeros_like(params)
     loss = torch.zeros(1, device="cuda")
     flags = B.PLAN_REG | (B.PLAN_GRAPH if a.graph else 0)
-    plan = B.betty_plan_create(ctx, model, dev, dpart, a.K, list(range(a.K)), group=a.group, flags=flags)
+    from paper_conf_asplos_yangzd023_b200.dist import lpt_assign, micro_batch_costs, reg_rows
+    my_k = lpt_assign(micro_batch_costs(part, a.K, ds.blocks[-1].indptr), a.sim_world)[0]
+    plan = B.betty_plan_create(ctx, model, dev, dpart, a.K, my_k, group=a.group, flags=flags)
+    if a.sim_world > 1:
+        plan.set_reg_rows(*reg_rows(cfg.n_out, 0, a.sim_world))
     B.betty_step(ctx, plan, params, feats, labels, 1.0 / cfg.n_out, grad, loss)
     B.betty_sync_check(ctx)
     torch.cuda.synchronize()
