@@ -60,7 +60,9 @@ def parse():
     p.add_argument("--json-out", default=None)
     p.add_argument("--sim-world", type=int, default=0, help="(study) run rank 0's share of an N-rank job on one GPU")
     p.add_argument("--feat-align", type=int, default=256, help="feature-table row alignment in bytes (0: 16)")
-    p.add_argument("--feat-layout", default="gid", choices=["gid", "owner"],
+    p.add_argument("--input-order", default="random", choices=["random", "community"],
+                   help="(study) node ids as generated (communities scattered) or community-contiguous")
+    p.add_argument("--feat-layout", default="gid", choices=["gid", "owner", "l2"],
                    help="feature-table row order: gid (as generated) or owner (rows grouped by the micro-batch "
                         "that reads them most, experimental)")
     return p.parse_args()
@@ -157,7 +159,8 @@ def build_inputs(args, rank, ws, device):
         cfg = synth.scaled(cfg, args.scale)
     t0 = time.time()
     if rank == 0:
-        ds = synth.make(cfg, with_features=None)      # None: C5's table is generated in chunks on the device
+        ds = synth.make(cfg, with_features=None,      # None: C5's table is generated in chunks on the device
+                        community_order=args.input_order == "community")
         arrays = [ds.graph.comm, ds.labels, ds.seeds]
         for b in ds.blocks:
             arrays += [b.indptr, b.nbr_pos, b.src_gid]
@@ -378,6 +381,10 @@ def main():
     import synth
     feats = synth.features_device(cfg, ds, args.mode == "bf16", args.feat_align, device)   # bf16: reading #17
     host_gid0 = ds.blocks[0].src_gid
+    if args.feat_layout == "l2":       # (study only) every layer-0 row read hits 64 Ki rows = 16 MB: L2-resident
+        b0 = dev_blocks[0]
+        b0.src_gid.copy_(torch.remainder(b0.src_gid, 65536))
+        host_gid0 = b0.src_gid.cpu().numpy()
     if args.feat_layout == "owner":
         t_l = time.time()
         perm = owner_layout(ds.blocks, part, args.K)

@@ -46,8 +46,11 @@ __device__ __forceinline__ uint64_t l2_evict_last_policy() {
     asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
     return pol;
 }
-__device__ __forceinline__ void cp_async16(void* sdst, const void* gsrc, uint64_t pol, bool hint) {
-    if (hint)
+__device__ __forceinline__ void cp_async16(void* sdst, const void* gsrc, uint64_t pol, int hint) {
+    if (hint == 3)          // L1-allocating: rows re-read by the same SM hit L1
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 16;"
+                     ::"r"((uint32_t)__cvta_generic_to_shared(sdst)), "l"(gsrc) : "memory");
+    else if (hint)
         asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2;"
                      ::"r"((uint32_t)__cvta_generic_to_shared(sdst)), "l"(gsrc), "l"(pol) : "memory");
     else
@@ -123,7 +126,7 @@ __global__ void __launch_bounds__(256) k_agg_mean_xa(const Tin* __restrict__ X, 
     const unsigned gmask = LPR == 32 ? 0xffffffffu : (((1u << LPR) - 1u) << (grp * LPR));
     uint4* wb = agg_sbuf + ((int64_t)wib * RPW + grp) * SLOTS * LPR;
     const uint64_t pol = l2_evict_last_policy();
-    const bool use_hint = hint != 0;
+    const int use_hint = hint == 3 ? 3 : (hint != 0 ? 1 : 0);
     int seg = 0;
     // Row meta (real row, edge range, first EB edge ids, self row) of the next iteration is
     // loaded while the current gather is in flight.
@@ -840,6 +843,178 @@ __global__ void __launch_bounds__(256) k_csc_mean(const float* __restrict__ dXA,
     }
 }
 
+// Vectorised form of k_csc_mean for wide layers (C2 / C5 hidden layers, Fi = 256): one warp per
+// source u, lane owns float4 column groups lane + 32 k (k < VPL, so a warp reads a whole 1 KB
+// half-row per edge, coalesced); the CSC entries and 1/D_v of 32 edges are loaded at once and
+// broadcast by shuffles, and CM_UNR edges' rows are in flight per lane before they are added.
+// The additions run in CSC order per column exactly like k_csc_mean (bit-identical results).
+constexpr int CM_UNR = 4;
+template <typename Tm, typename Tout, int VPL>
+__global__ void __launch_bounds__(256) k_csc_mean_v(const float* __restrict__ dXA, int64_t ldd,
+                                                    const int64_t* __restrict__ indptr,
+                                                    const int64_t* __restrict__ t_indptr,
+                                                    const int32_t* __restrict__ t_idx, const int64_t* cnt, int Fi,
+                                                    int Fp, const Tm* __restrict__ H, int64_t ldh,
+                                                    const uint32_t* __restrict__ hbits, int64_t ldhb,
+                                                    Tout* __restrict__ out, int64_t ldo) {
+    const int64_t nd = cnt[0], ns = cnt[1];
+    const int lane = lane_id();
+    const int NG = Fi / 4;                                  // float4 groups of a row
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t u = gw; u < ns; u += nw) {
+        const int64_t b = t_indptr[u], e = t_indptr[u + 1];
+        float acc[VPL][4];
+#pragma unroll
+        for (int k = 0; k < VPL; ++k)
+#pragma unroll
+            for (int t = 0; t < 4; ++t) acc[k][t] = 0.f;
+        for (int64_t e0 = b; e0 < e; e0 += 32) {
+            const int n = (int)mn64(32, e - e0);
+            int32_t my = 0;
+            float myinv = 0.f;
+            if (lane < n) {
+                my = t_idx[e0 + lane];
+                myinv = 1.0f / (float)(indptr[my + 1] - indptr[my]);
+            }
+            for (int j0 = 0; j0 < n; j0 += CM_UNR) {
+                float4 x[CM_UNR][VPL];
+                float iv[CM_UNR];
+#pragma unroll
+                for (int q = 0; q < CM_UNR; ++q) {
+                    const int32_t v = __shfl_sync(0xffffffffu, my, (j0 + q) & 31);
+                    iv[q] = __shfl_sync(0xffffffffu, myinv, (j0 + q) & 31);
+#pragma unroll
+                    for (int k = 0; k < VPL; ++k) {
+                        const int g = lane + 32 * k;
+                        x[q][k] = (j0 + q < n && g < NG)
+                                      ? *reinterpret_cast<const float4*>(dXA + (int64_t)v * ldd + Fp + 4 * g)
+                                      : make_float4(0.f, 0.f, 0.f, 0.f);
+                    }
+                }
+#pragma unroll
+                for (int q = 0; q < CM_UNR; ++q) {
+                    if (j0 + q < n) {
+#pragma unroll
+                        for (int k = 0; k < VPL; ++k) {
+                            acc[k][0] += x[q][k].x * iv[q];
+                            acc[k][1] += x[q][k].y * iv[q];
+                            acc[k][2] += x[q][k].z * iv[q];
+                            acc[k][3] += x[q][k].w * iv[q];
+                        }
+                    }
+                }
+            }
+        }
+#pragma unroll
+        for (int k = 0; k < VPL; ++k) {
+            const int g = lane + 32 * k;
+            if (g < NG) {
+                const int c = 4 * g;
+                float4 sf = u < nd ? *reinterpret_cast<const float4*>(dXA + u * ldd + c) : make_float4(0.f, 0.f, 0.f, 0.f);
+                float gv[4] = {acc[k][0] + sf.x, acc[k][1] + sf.y, acc[k][2] + sf.z, acc[k][3] + sf.w};
+                if (hbits) {            // ReLU' from the forward's bits (32 B per 256-wide row, not 512 B of H)
+                    const uint32_t w = hbits[u * ldhb + (c >> 5)] >> (c & 31);
+#pragma unroll
+                    for (int t = 0; t < 4; ++t)
+                        if (!(w >> t & 1u)) gv[t] = 0.f;
+                } else {
+#pragma unroll
+                    for (int t = 0; t < 4; ++t)
+                        if (!(ld_act(H + u * ldh + c + t) > 0.f)) gv[t] = 0.f;
+                }
+                st_act4(out + u * ldo + c, gv);
+            }
+        }
+        for (int col = Fi + lane; col < ldo; col += 32) st_act(out + u * ldo + col, 0.f);
+    }
+}
+
+// Lane-group form (sources of low CSC degree, e.g. C5's layer 1 with 1.2 entries per source): LPR
+// lanes per source own VPL float4 groups each (LPR * VPL = Fi / 4), so a warp works on 32 / LPR
+// sources at once; per source the CSC entries / 1/D_v of LPR edges are loaded together and the
+// rows of two edges are in flight before they are added (same per-column CSC order: bit-identical).
+template <typename Tm, typename Tout, int LPR, int VPL>
+__global__ void __launch_bounds__(256) k_csc_mean_g(const float* __restrict__ dXA, int64_t ldd,
+                                                    const int64_t* __restrict__ indptr,
+                                                    const int64_t* __restrict__ t_indptr,
+                                                    const int32_t* __restrict__ t_idx, const int64_t* cnt, int Fi,
+                                                    int Fp, const Tm* __restrict__ H, int64_t ldh,
+                                                    const uint32_t* __restrict__ hbits, int64_t ldhb,
+                                                    Tout* __restrict__ out, int64_t ldo) {
+    constexpr int RPW = 32 / LPR;
+    const int64_t nd = cnt[0], ns = cnt[1];
+    const int lane = lane_id(), sub = lane % LPR, grp = lane / LPR;
+    const unsigned gmask = LPR == 32 ? 0xffffffffu : (((1u << LPR) - 1u) << (grp * LPR));
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t u0 = gw * RPW; u0 < ns; u0 += nw * RPW) {
+        const int64_t u = u0 + grp;
+        if (u >= ns) continue;                              // whole lane group idle
+        const int64_t b = t_indptr[u], e = t_indptr[u + 1];
+        float acc[VPL][4];
+#pragma unroll
+        for (int k = 0; k < VPL; ++k)
+#pragma unroll
+            for (int t = 0; t < 4; ++t) acc[k][t] = 0.f;
+        for (int64_t e0 = b; e0 < e; e0 += LPR) {
+            const int n = (int)mn64(LPR, e - e0);
+            int32_t my = 0;
+            float myinv = 0.f;
+            if (sub < n) {
+                my = t_idx[e0 + sub];
+                myinv = 1.0f / (float)(indptr[my + 1] - indptr[my]);
+            }
+#pragma unroll
+            for (int j0 = 0; j0 < LPR; j0 += 2) {
+                if (j0 >= n) break;
+                float4 x[2][VPL];
+                float iv[2];
+#pragma unroll
+                for (int q = 0; q < 2; ++q) {
+                    const int32_t v = __shfl_sync(gmask, my, j0 + q, LPR);
+                    iv[q] = __shfl_sync(gmask, myinv, j0 + q, LPR);
+#pragma unroll
+                    for (int k = 0; k < VPL; ++k)
+                        x[q][k] = j0 + q < n
+                                      ? *reinterpret_cast<const float4*>(dXA + (int64_t)v * ldd + Fp + 4 * (sub * VPL + k))
+                                      : make_float4(0.f, 0.f, 0.f, 0.f);
+                }
+#pragma unroll
+                for (int q = 0; q < 2; ++q) {
+                    if (j0 + q < n) {
+#pragma unroll
+                        for (int k = 0; k < VPL; ++k) {
+                            acc[k][0] += x[q][k].x * iv[q];
+                            acc[k][1] += x[q][k].y * iv[q];
+                            acc[k][2] += x[q][k].z * iv[q];
+                            acc[k][3] += x[q][k].w * iv[q];
+                        }
+                    }
+                }
+            }
+        }
+#pragma unroll
+        for (int k = 0; k < VPL; ++k) {
+            const int c = 4 * (sub * VPL + k);
+            float4 sf = u < nd ? *reinterpret_cast<const float4*>(dXA + u * ldd + c) : make_float4(0.f, 0.f, 0.f, 0.f);
+            float gv[4] = {acc[k][0] + sf.x, acc[k][1] + sf.y, acc[k][2] + sf.z, acc[k][3] + sf.w};
+            if (hbits) {                // ReLU' from the forward's bits
+                const uint32_t w = hbits[u * ldhb + (c >> 5)] >> (c & 31);
+#pragma unroll
+                for (int t = 0; t < 4; ++t)
+                    if (!(w >> t & 1u)) gv[t] = 0.f;
+            } else {
+#pragma unroll
+                for (int t = 0; t < 4; ++t)
+                    if (!(ld_act(H + u * ldh + c + t) > 0.f)) gv[t] = 0.f;
+            }
+            st_act4(out + u * ldo + c, gv);
+        }
+        for (int col = Fi + sub; col < ldo; col += LPR) st_act(out + u * ldo + col, 0.f);
+    }
+}
+
 // --------------------------------------- mean, project-first bwd (via CSC)
 // G[u] = [ sum_{v in CSC(u)} dS[v]/D_v (Fo) | 0 | [u < nd] dS[u] (Fo) | 0 ]
 template <typename Tin, typename Tout>
@@ -1155,7 +1330,8 @@ void agg_mean_xa(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const in
     // only a slice of every row (the rows' metadata is re-read, the features are not).
     static const double budget = getenv("BETTY_AGG_WS_MB") ? atof(getenv("BETTY_AGG_WS_MB")) * 1e6 : 1e12;
     unsigned* ctr = c->L().counters + CTR_AGG;
-    static const int hint = getenv("BETTY_AGG_NOHINT") ? 0 : (getenv("BETTY_AGG_NOBULK") ? 2 : 1);
+    static const int hint = getenv("BETTY_AGG_CA") ? 3 :
+                            (getenv("BETTY_AGG_NOHINT") ? 0 : (getenv("BETTY_AGG_NOBULK") ? 2 : 1));
     static const bool no_order = getenv("BETTY_AGG_NOORDER") != nullptr;
     const double ws = (double)src_per_mb * (double)nv * 16.0;
     int passes = (int)std::max(1.0, std::min((double)nv, std::ceil(ws / budget)));
@@ -1203,7 +1379,34 @@ void gather_ones(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const in
 
 void csc_mean(betty_ctx* c, const float* dXA, int64_t ldd, const int64_t* indptr, const int64_t* t_indptr,
               const int32_t* t_idx, const int64_t* cnt, int64_t src_cap, int Fi, int Fp, const void* H, bool h_bf16,
-              int64_t ldh, void* out, bool out_bf16, int64_t ldo, cudaStream_t s) {
+              int64_t ldh, const uint32_t* hbits, int64_t ldhb, void* out, bool out_bf16, int64_t ldo,
+              cudaStream_t s) {
+    static const bool scalar = getenv("BETTY_CSC_MEAN_SCALAR") != nullptr;     // A/B switches
+    static const bool warp_form = getenv("BETTY_CSC_MEAN_WARP") != nullptr;
+    const int vpl = (Fi / 4 + 31) / 32;
+    const int ng = Fi / 4;
+    if (!scalar && !warp_form && Fi % 4 == 0 && Fp % 4 == 0 && ldd % 4 == 0 && ldo % 4 == 0 && ng % 8 == 0 &&
+        (ng / 8) <= 32 && ((ng / 8) & (ng / 8 - 1)) == 0 && ((uintptr_t)dXA & 15) == 0 && ((uintptr_t)out & 15) == 0) {
+        const int lpr = ng / 8;                         // 8 float4 groups per lane
+        const int g = warps_grid(c, (src_cap + (32 / lpr) - 1) / (32 / lpr));
+#define CM_G(LP) DISPATCH_ACT(h_bf16, TM, DISPATCH_ACT(out_bf16, TO,                                             \
+        k_csc_mean_g<TM, TO, LP, 8><<<g, 256, 0, s>>>(dXA, ldd, indptr, t_indptr, t_idx, cnt, Fi, Fp, (const TM*)H, \
+                                                      ldh, hbits, ldhb, (TO*)out, ldo)))
+        if (lpr == 1) { CM_G(1); } else if (lpr == 2) { CM_G(2); } else if (lpr == 4) { CM_G(4); }
+        else if (lpr == 8) { CM_G(8); } else if (lpr == 16) { CM_G(16); } else { CM_G(32); }
+#undef CM_G
+        return;
+    }
+    if (!scalar && Fi % 4 == 0 && Fp % 4 == 0 && ldd % 4 == 0 && ldo % 4 == 0 && vpl <= 4 &&
+        ((uintptr_t)dXA & 15) == 0 && ((uintptr_t)out & 15) == 0) {
+        const int g = warps_grid(c, src_cap);
+#define CM_V(V) DISPATCH_ACT(h_bf16, TM, DISPATCH_ACT(out_bf16, TO,                                              \
+        k_csc_mean_v<TM, TO, V><<<g, 256, 0, s>>>(dXA, ldd, indptr, t_indptr, t_idx, cnt, Fi, Fp, (const TM*)H, ldh, \
+                                                  hbits, ldhb, (TO*)out, ldo)))
+        if (vpl <= 1) { CM_V(1); } else if (vpl == 2) { CM_V(2); } else { CM_V(4); }
+#undef CM_V
+        return;
+    }
     DISPATCH_ACT(h_bf16, TM, DISPATCH_ACT(out_bf16, TO,
         k_csc_mean<TM, TO><<<warps_grid(c, src_cap), 256, 0, s>>>(dXA, ldd, indptr, t_indptr, t_idx, cnt, Fi, Fp,
                                                                   (const TM*)H, ldh, (TO*)out, ldo)));

@@ -342,7 +342,7 @@ void sage_backward(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView
         }
         if (L.kind == KIND_AGG) {
             csc_mean(c, B.dXA, L.ld_dxa, V.indptr, V.t_indptr, V.t_indices, V.cnt, V.cap_src, L.Fi, L.Fp, Hmask,
-                     m.bf16, ldh, dS_prev, m.bf16, ld_prev, s);
+                     m.bf16, ldh, B.hbits_ok ? B.Hbits : nullptr, B.ldhb, dS_prev, m.bf16, ld_prev, s);
             continue;
         }
         // POOL: route to the argmax, then W_pool

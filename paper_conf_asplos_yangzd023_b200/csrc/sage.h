@@ -21,7 +21,8 @@ void gather_ones(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const in
                  int64_t rows_cap, int Fi, void* out, bool out_bf16, int64_t ldo, cudaStream_t s);
 void csc_mean(betty_ctx* c, const float* dXA, int64_t ldd, const int64_t* indptr, const int64_t* t_indptr,
               const int32_t* t_idx, const int64_t* cnt, int64_t src_cap, int Fi, int Fp, const void* H, bool h_bf16,
-              int64_t ldh, void* out, bool out_bf16, int64_t ldo, cudaStream_t s);
+              int64_t ldh, const uint32_t* hbits, int64_t ldhb, void* out, bool out_bf16, int64_t ldo,
+              cudaStream_t s);   // hbits (optional): [H > 0] as bits, ldhb words per row
 // G = P^T D+ dS via the CSC; indptr == null: dS is already scaled by 1/D_v (the loss kernel does it)
 void csc_pf(betty_ctx* c, const void* dS, bool ds_bf16, int64_t ldds, const int64_t* indptr, const int64_t* t_indptr,
             const int32_t* t_idx, const int64_t* cnt, int64_t src_cap, int Fo, int Fop, void* G, bool g_bf16,

@@ -268,9 +268,27 @@ class Dataset:
     blocks: List[Block]       # block 0 (input) ... L-1 (output)
 
 
-def make(cfg: Config, with_features: Optional[bool] = True) -> Dataset:
+def relabel_by_community(g: Graph) -> Graph:
+    """(Study input) the same graph with node ids renumbered so that every community is a contiguous id
+    range (stable within a community): an upper bound on what a locality-aware node order can do."""
+    order = np.argsort(g.comm, kind="stable")
+    inv = np.empty_like(order)
+    inv[order] = np.arange(len(order))
+    deg = np.diff(g.indptr)[order]
+    indptr = np.concatenate([[0], np.cumsum(deg)]).astype(np.int64)
+    starts = g.indptr[order]
+    idx = np.repeat(starts - indptr[:-1], deg) + np.arange(indptr[-1])
+    vals = inv[g.indices[idx]].astype(np.int64)
+    rows = np.repeat(np.arange(len(order), dtype=np.int64), deg)
+    vals = vals[np.lexsort((vals, rows))].astype(np.int32)
+    return Graph(indptr, vals, g.comm[order])
+
+
+def make(cfg: Config, with_features: Optional[bool] = True, community_order: bool = False) -> Dataset:
     s = cfg.seeds
     g = graph(cfg.n, int(cfg.pairs * cfg.oversample), cfg.n_comm, cfg.mu, cfg.beta, s["graph"])
+    if community_order:
+        g = relabel_by_community(g)
     sd = seeds(g.n, cfg.n_out, s["train"])
     blocks = sample(g, sd, cfg.fanouts, s["sample"])
     if with_features is None:
