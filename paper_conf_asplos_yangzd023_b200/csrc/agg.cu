@@ -393,11 +393,21 @@ __global__ void __launch_bounds__(256) k_route_pool_v(const float* __restrict__ 
                         rb[k] = j0 + k < n ? __ldg(indptr + v[k]) : 0;
                         re[k] = j0 + k < n ? __ldg(indptr + v[k] + 1) : 0;
                     }
+                    // u's position in each v's row, warp-cooperatively: 32 row entries per load, one
+                    // ballot (the 4 edges' loads are independent and issued together)
+                    int32_t xs[4];
+#pragma unroll
+                    for (int k = 0; k < 4; ++k)
+                        xs[k] = lane < re[k] - rb[k] ? __ldg(idx + rb[k] + lane) : -1;
 #pragma unroll
                     for (int k = 0; k < 4; ++k) {
-                        key[k] = -2;
-                        for (int64_t e = rb[k]; e < re[k]; ++e)
-                            if (__ldg(idx + e) == (int32_t)u) { key[k] = (int32_t)(e - rb[k]); break; }
+                        const unsigned m = __ballot_sync(0xffffffffu, xs[k] == (int32_t)u);
+                        key[k] = m ? __ffs(m) - 1 : -2;
+                        for (int64_t base = rb[k] + 32; !m && key[k] < 0 && base < re[k]; base += 32) {
+                            const int32_t x = base + lane < re[k] ? __ldg(idx + base + lane) : -1;
+                            const unsigned m2 = __ballot_sync(0xffffffffu, x == (int32_t)u);
+                            if (m2) key[k] = (int32_t)(base - rb[k]) + __ffs(m2) - 1;
+                        }
                     }
                 } else {
 #pragma unroll

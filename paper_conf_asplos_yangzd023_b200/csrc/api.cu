@@ -645,11 +645,12 @@ extern "C" betty_status betty_plan_create(betty_ctx* c, const betty_model* model
         return fail(c, BETTY_EINVAL, "plan: bad K / my_k / n_out / part");
     for (int i = 0; i < n_my; ++i)
         if (my_k[i] < 0 || my_k[i] >= K) return fail(c, BETTY_EINVAL, "plan: my_k[%d] out of range", i);
-    // pool layers can keep the argmax as a byte position when every row of the block has <= 254 edges
-    // (micro-batch rows are full-batch rows; one reduction per pool layer, here at plan time).  Off by
-    // default (BETTY_POOL_POS8=1): on C4 it reads 23 % fewer bytes but the routing kernel's search of
-    // u's position in each row costs more latency than it saves (105 vs 63 ms per step, measured).
-    const bool pos8_on = getenv("BETTY_POOL_POS8") && atoi(getenv("BETTY_POOL_POS8"));
+    // pool layers keep the argmax as a byte position when every row of the block has <= 254 edges
+    // (micro-batch rows are full-batch rows; one reduction per pool layer, here at plan time): a
+    // quarter of the int32 argmax bytes and memory.  The routing kernel finds u's position in each
+    // row with one warp-wide load + ballot (C4: 135.4 vs 137.7 ms per step for int32 positions;
+    // the first, serial search was 105 vs 63 ms).  BETTY_POOL_POS8=0 keeps int32 argmax ids.
+    const bool pos8_on = !(getenv("BETTY_POOL_POS8") && atoi(getenv("BETTY_POOL_POS8")) == 0);
     if (m.aggr == BETTY_AGGR_POOL && pos8_on) {
         int* d_mx = nullptr;
         if (cudaMalloc(&d_mx, sizeof(int) * L) != cudaSuccess) return fail(c, BETTY_ENOMEM, "plan: max degree");

@@ -239,6 +239,10 @@ CASES = [
     # full neighbourhoods on dense graphs: rows longer than the gather pipeline's stage ("long rows")
     dict(name="mean2-full-hub", aggr="mean", fanouts=(-1, -1), dims=[8, 16, 3], n=400, pairs=30000),
     dict(name="mean2-full-wide", aggr="mean", fanouts=(-1, -1), dims=[100, 128, 5], n=400, pairs=8000),
+    # aggregate-first hidden layer of width 64: the lane-group CSC backward (2 lanes per source)
+    dict(name="mean3-agg64", aggr="mean", fanouts=(3, 4, 5), dims=[32, 64, 64, 5]),
+    # pool rows longer than one warp-wide position search (byte-position argmax, rows of ~150 edges)
+    dict(name="pool2-full-hub", aggr="pool", fanouts=(-1, -1), dims=[8, 16, 3], n=400, pairs=30000),
 ]
 
 
@@ -293,7 +297,7 @@ def test_sage_micro_batch(B, ctx, c, mode):
 @pytest.mark.parametrize("mode", ["fp32", "bf16"])
 @pytest.mark.parametrize("group", [1, 2, 0])
 @pytest.mark.parametrize("graph", [False, True])
-@pytest.mark.parametrize("c", [CASES[1], CASES[2], CASES[4], CASES[7]], ids=lambda c: c["name"])
+@pytest.mark.parametrize("c", [CASES[1], CASES[2], CASES[4], CASES[7], CASES[8], CASES[9]], ids=lambda c: c["name"])
 def test_step_matches_oracle(B, ctx, c, mode, group, graph):
     """betty_step (fused extraction + fwd + loss + bwd + accumulation over a
     rank's micro-batches) vs oracle_step, for several launch groupings."""
@@ -384,11 +388,12 @@ def test_c1_cora_config(B, ctx):
         plan.free()
 
 
+@pytest.mark.parametrize("pos8", ["0", "1"])
 @pytest.mark.parametrize("mode", ["fp32", "bf16"])
-def test_pool_byte_positions(B, ctx, mode, monkeypatch):
-    """The optional byte-position argmax of the pool layers (BETTY_POOL_POS8=1, plan path)
-    routes the gradient exactly like the source-id argmax."""
-    monkeypatch.setenv("BETTY_POOL_POS8", "1")
+def test_pool_byte_positions(B, ctx, mode, pos8, monkeypatch):
+    """Both argmax encodings of the pool layers (plan path): byte positions in the row (default) and
+    int32 source ids (BETTY_POOL_POS8=0) route the gradient like the oracle."""
+    monkeypatch.setenv("BETTY_POOL_POS8", pos8)
     c = CASES[5]
     sd, blocks, feats, labels, params = make_case(c, seed=3)
     K = 3
