@@ -646,7 +646,7 @@ bool gemm_row_tc(betty_ctx* c, const GemmRow& g, const void* Bk, int64_t ldbk, c
     const size_t a_bytes = BM * BK * 2;
     const uint32_t slot_bytes = 32 * 32 * (g.c_bf16 ? 2 : 4);
     const size_t stage_bytes = (size_t)EPI_WARPS * ESLOTS * slot_bytes;
-    const size_t budget = 225 * 1024;
+    const size_t budget = 227 * 1024;           // the sm_100 opt-in maximum of dynamic shared memory per CTA
     const size_t bblk = (size_t)BN * BK * 2;
     // B resident when it fits next to a 2-stage A ring, else streamed with A
     const bool bstream = b_bytes + stage_bytes + 2 * a_bytes + 1024 + 256 > budget;
