@@ -758,7 +758,12 @@ extern "C" betty_status betty_plan_create(betty_ctx* c, const betty_model* model
     }
     // ---- REG inside the step (once here to size its buffers): all rows until betty_plan_set_reg_rows
     if (flags & BETTY_PLAN_REG) {
-        if (cudaStreamCreateWithFlags(&p->side, cudaStreamNonBlocking) != cudaSuccess ||
+        // the REG shares no data with the rest of the step: its side stream gets the LOWEST priority
+        // and the step's capture stream the highest, so the block scheduler fills the main path's
+        // SMs first and the REG runs in the gaps (tails, latency-bound phases)
+        int prio_lo = 0, prio_hi = 0;
+        cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
+        if (cudaStreamCreateWithPriority(&p->side, cudaStreamNonBlocking, prio_lo) != cudaSuccess ||
             cudaEventCreateWithFlags(&p->ev_fork, cudaEventDisableTiming) != cudaSuccess ||
             cudaEventCreateWithFlags(&p->ev_join, cudaEventDisableTiming) != cudaSuccess) {
             betty_plan_destroy(c, p);
@@ -833,13 +838,18 @@ extern "C" betty_status betty_step(betty_ctx* c, betty_plan* p, const float* par
         if (p->gexec) { cudaGraphExecDestroy(p->gexec); p->gexec = nullptr; }
         // capture on a private stream (the caller's may be the legacy default
         // stream, which cannot be captured); the graph is launched on `s`
-        if (!p->cap_stream) CUDA_OK(c, cudaStreamCreateWithFlags(&p->cap_stream, cudaStreamNonBlocking));
+        if (!p->cap_stream) {
+            int prio_lo = 0, prio_hi = 0;
+            cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
+            CUDA_OK(c, cudaStreamCreateWithPriority(&p->cap_stream, cudaStreamNonBlocking, prio_hi));
+        }
         CUDA_OK(c, cudaStreamSynchronize(s));
         cudaGraph_t g;
         CUDA_OK(c, cudaStreamBeginCapture(p->cap_stream, cudaStreamCaptureModeThreadLocal));
         step_body(c, p, params, feats, ld_feats, labels, loss_scale, grad_accum, loss_accum, p->cap_stream);
         CUDA_OK(c, cudaStreamEndCapture(p->cap_stream, &g));
-        cudaError_t e = cudaGraphInstantiate(&p->gexec, g, 0);
+        static const bool no_prio = getenv("BETTY_NO_NODE_PRIORITY") != nullptr;     // A/B switch
+        cudaError_t e = cudaGraphInstantiate(&p->gexec, g, no_prio ? 0 : cudaGraphInstantiateFlagUseNodePriority);
         cudaGraphDestroy(g);
         if (e != cudaSuccess) return fail(c, BETTY_ECUDA, "graph instantiate: %s", cudaGetErrorString(e));
         memcpy(p->key, key, sizeof key);
