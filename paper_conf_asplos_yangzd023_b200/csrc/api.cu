@@ -506,11 +506,20 @@ struct betty_plan {
     Probe probe;
 };
 
+// Where the REG rebuild forks onto its side stream: 0 at the start of the step (with the extraction),
+// 1 after the first group's extraction (with the aggregation / GEMMs), 2 (default) before its
+// backward.  Measured on C3: 5.10 / 5.25 / 5.04 ms per step -- the latency-bound extraction suffers
+// most from sharing the SMs (1.13 ms alone, 1.44 ms beside the REG), the backward least.
+static int reg_fork_point() {
+    static const int v = getenv("BETTY_REG_FORK") ? atoi(getenv("BETTY_REG_FORK")) : 2;
+    return v;
+}
+
 static void step_body(betty_ctx* c, betty_plan* p, const float* params, const void* feats, int64_t ld_feats,
                       const int32_t* labels, float scale, float* grad, float* loss, cudaStream_t s) {
     Probe* pr = p->sb.probe;
     if (pr) pr->used = 0;
-    if (p->with_reg) {          // fork: REG on the side stream with its own primitive scratch (lane 1)
+    auto fork_reg = [&]() {     // REG on the side stream with its own primitive scratch (lane 1)
         cudaEventRecord(p->ev_fork, s);
         cudaStreamWaitEvent(p->side, p->ev_fork, 0);
         c->lane = 1;
@@ -521,7 +530,9 @@ static void step_body(betty_ctx* c, betty_plan* p, const float* params, const vo
         if (pr) pr->end(PROBE_REG, p->side);
         c->lane = 0;
         cudaEventRecord(p->ev_join, p->side);
-    }
+    };
+    const int fp = p->groups.empty() ? 0 : reg_fork_point();
+    if (p->with_reg && fp == 0) fork_reg();
     sage_prep(c, p->m, p->sb, params, s);
     for (size_t g = 0; g < p->groups.size(); ++g) {
         ExtractArgs a{};
@@ -531,8 +542,10 @@ static void step_body(betty_ctx* c, betty_plan* p, const float* params, const vo
         if (pr) pr->begin(PROBE_EXTRACT, s);
         extract_group(c, a, s);
         if (pr) pr->end(PROBE_EXTRACT, s);
+        if (p->with_reg && fp == 1 && g == 0) fork_reg();
         sage_forward(c, p->m, p->sb, p->views.data(), feats, ld_feats, s);
         sage_loss(c, p->m, p->sb, p->views.data(), labels, scale, loss, s);
+        if (p->with_reg && fp == 2 && g == 0) fork_reg();
         sage_backward(c, p->m, p->sb, p->views.data(), feats, ld_feats, grad, s);
     }
     if (p->with_reg) cudaStreamWaitEvent(s, p->ev_join, 0);   // join
