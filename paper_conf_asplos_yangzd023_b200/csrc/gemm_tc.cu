@@ -364,6 +364,20 @@ __global__ void __launch_bounds__(ROW_THREADS, 1) k_tc_row(const __grid_constant
         uint8_t* my_stage = stage + ew * ESLOTS * p.slot_bytes;
         int slot = 0;
         int it = 0;
+        // ReLU' bit words of this thread's row, one tile ahead (short-K layers finish the MMA long
+        // before a load round trip, so loading them at the top of the tile left them exposed)
+        uint32_t mw_next[MAXCH];
+#pragma unroll
+        for (int ci = 0; ci < MAXCH; ++ci) mw_next[ci] = 0u;
+        auto load_bits = [&](int64_t tt, uint32_t (&dst)[MAXCH]) {
+            const int64_t mm = tt * BM + q * 32 + lane;
+            if (tt < tiles && mm < M) {
+                const uint32_t* wb = p.mbits + mm * p.ldmb + cbeg / 32;
+#pragma unroll
+                for (int ci = 0; ci < MAXCH; ++ci) if (ci < nch) dst[ci] = wb[ci];
+            }
+        };
+        if (HAS_MASK && MBITS) load_bits(blockIdx.x, mw_next);
         for (int64_t t = blockIdx.x; t < tiles; t += gridDim.x, ++it) {
             const int acc = it & 1;
             const uint32_t aph = (it >> 1) & 1;
@@ -376,11 +390,9 @@ __global__ void __launch_bounds__(ROW_THREADS, 1) k_tc_row(const __grid_constant
             for (int ci = 0; ci < MAXCH; ++ci) mw[ci] = 0u;
             if (HAS_MASK) {
                 if (MBITS) {
-                    if (ok) {
-                        const uint32_t* wb = p.mbits + m * p.ldmb + cbeg / 32;
 #pragma unroll
-                        for (int ci = 0; ci < MAXCH; ++ci) if (ci < nch) mw[ci] = wb[ci];
-                    }
+                    for (int ci = 0; ci < MAXCH; ++ci) { mw[ci] = ok ? mw_next[ci] : 0u; mw_next[ci] = 0u; }
+                    load_bits(t + gridDim.x, mw_next);
                 } else {
 #pragma unroll
                     for (int ci = 0; ci < MAXCH; ++ci) if (ci < nch) mw[ci] = mask_word_from_act(p, m, cbeg + 32 * ci, ok);
