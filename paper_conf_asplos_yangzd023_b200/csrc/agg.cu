@@ -1162,11 +1162,20 @@ __global__ void __launch_bounds__(256) k_agg_pf_v(const float* __restrict__ Y, c
     const unsigned gmask = LPR == 32 ? 0xffffffffu : (((1u << LPR) - 1u) << (grp * LPR));
     const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    int64_t nb = 0, ne = 0;                  // row extents one iteration ahead
+    {
+        const int64_t v = gw * RPW + grp;
+        if (v < nd) { nb = indptr[v]; ne = indptr[v + 1]; }
+    }
     for (int64_t v0 = gw * RPW; v0 < nd; v0 += nw * RPW) {
         const int64_t v = v0 + grp;
         const bool rowok = v < nd;
-        int64_t b = 0, e = 0;
-        if (rowok) { b = indptr[v]; e = indptr[v + 1]; }
+        const int64_t b = nb, e = ne;
+        {
+            const int64_t vn = v + nw * RPW;
+            nb = 0; ne = 0;
+            if (vn < nd) { nb = indptr[vn]; ne = indptr[vn + 1]; }
+        }
         const float inv = e > b ? 1.0f / (float)(e - b) : 0.0f;
         for (int vb = 0; vb < NV; vb += LPR * PF_VPL) {
             float4 acc[PF_VPL];
@@ -1226,11 +1235,22 @@ __global__ void __launch_bounds__(256) k_csc_pf_v(const Tin* __restrict__ dS, in
     const unsigned gmask = LPR == 32 ? 0xffffffffu : (((1u << LPR) - 1u) << (grp * LPR));
     const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    // the next row group's column extents are loaded one iteration ahead (the CSC columns are short:
+    // their extents are a dependent round trip in front of every other load)
+    int64_t nb = 0, ne = 0;
+    {
+        const int64_t u = gw * RPW + grp;
+        if (u < ns) { nb = t_indptr[u]; ne = t_indptr[u + 1]; }
+    }
     for (int64_t u0 = gw * RPW; u0 < ns; u0 += nw * RPW) {
         const int64_t u = u0 + grp;
         const bool rowok = u < ns;
-        int64_t b = 0, e = 0;
-        if (rowok) { b = t_indptr[u]; e = t_indptr[u + 1]; }
+        const int64_t b = nb, e = ne;
+        {
+            const int64_t un = u + nw * RPW;
+            nb = 0; ne = 0;
+            if (un < ns) { nb = t_indptr[un]; ne = t_indptr[un + 1]; }
+        }
         for (int vb = 0; vb < NV; vb += LPR * PF_VPL) {
             float acc[PF_VPL][VW];
 #pragma unroll
