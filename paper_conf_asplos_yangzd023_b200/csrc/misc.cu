@@ -13,9 +13,9 @@ namespace betty {
 // (reading #15: scale = 1 / n_out of the full batch).  One warp per row,
 // C <= 256.  The loss is reduced deterministically: per-CTA partials in a
 // fixed order, summed by the last CTA.
-constexpr int LOSS_MAXT = 8;
+constexpr int LOSS_MAXT_CAP = 8;               // C <= 256
 
-template <typename TA>
+template <typename TA, int LOSS_MAXT>        // LOSS_MAXT = ceil(C / 32) column groups per lane
 __global__ void __launch_bounds__(256) k_loss(const float* __restrict__ logits, int64_t ldl,
                                               const int32_t* __restrict__ labels, const int32_t* __restrict__ gid,
                                               const int64_t* cnt, int C, float scale, float* __restrict__ dS,
@@ -29,19 +29,36 @@ __global__ void __launch_bounds__(256) k_loss(const float* __restrict__ logits, 
     const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
     double wl = 0.0;
+    // the next row's label, degree and logits are loaded while this row is reduced (a row's
+    // arithmetic is a chain of shuffles; its loads would otherwise sit in front of it)
+    int32_t ny = 0;
+    int64_t ndg = 1;
+    float nx[LOSS_MAXT];
+    auto fetch = [&](int64_t vv) {
+        if (vv < nd) {
+            ny = labels[gid[vv]];
+            if (indptr) ndg = indptr[vv + 1] - indptr[vv];
+#pragma unroll
+            for (int t = 0; t < LOSS_MAXT; ++t) {
+                const int c = lane + 32 * t;
+                nx[t] = c < C ? logits[vv * ldl + c] : -INFINITY;
+            }
+        }
+    };
+    fetch(gw);
     for (int64_t v = gw; v < nd; v += nw) {
-        const int32_t y = labels[gid[v]];               // independent of the logits: issued first
+        const int32_t y = ny;
         // indptr (project-first top layer): the fp32 dS is stored pre-scaled by 1/D_v for P^T D+ dS
         float inv = 1.f;
-        if (indptr) { const int64_t dg = indptr[v + 1] - indptr[v]; inv = dg > 0 ? 1.f / (float)dg : 0.f; }
+        if (indptr) inv = ndg > 0 ? 1.f / (float)ndg : 0.f;
         float x[LOSS_MAXT];
         float mx = -INFINITY;
 #pragma unroll
         for (int t = 0; t < LOSS_MAXT; ++t) {
-            const int c = lane + 32 * t;
-            x[t] = c < C ? logits[v * ldl + c] : -INFINITY;
+            x[t] = nx[t];
             mx = fmaxf(mx, x[t]);
         }
+        fetch(v + nw);
         mx = warp_max(mx);
         float se = 0.f;
 #pragma unroll
@@ -101,13 +118,19 @@ void loss_ce(betty_ctx* c, const float* logits, int64_t ldl, const int32_t* labe
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((rows_cap * 32 + 255) / 256,
                                                                  std::min(2048, c->num_sms * 8)));
     double* partials = (double*)(c->L().counters + 64);   // 2048 doubles after the counters
-    if (act_bf16)
-        k_loss<__nv_bfloat16><<<grid, 256, 0, s>>>(logits, ldl, labels, gid, cnt, C, scale, dS, ldds,
-                                                   (__nv_bfloat16*)dS_act, ld_act, prescale_indptr, partials,
-                                                   c->L().counters + CTR_LOSS, loss_accum);
-    else
-        k_loss<float><<<grid, 256, 0, s>>>(logits, ldl, labels, gid, cnt, C, scale, dS, ldds, (float*)dS_act, ld_act,
-                                           prescale_indptr, partials, c->L().counters + CTR_LOSS, loss_accum);
+    const int T = (C + 31) / 32;               // instantiated for 1, 2, 4 and 8 column groups per lane
+#define LOSS_L(TT) do {                                                                                        \
+        if (act_bf16)                                                                                          \
+            k_loss<__nv_bfloat16, TT><<<grid, 256, 0, s>>>(logits, ldl, labels, gid, cnt, C, scale, dS, ldds,     \
+                                                         (__nv_bfloat16*)dS_act, ld_act, prescale_indptr, partials, \
+                                                         c->L().counters + CTR_LOSS, loss_accum);              \
+        else                                                                                                   \
+            k_loss<float, TT><<<grid, 256, 0, s>>>(logits, ldl, labels, gid, cnt, C, scale, dS, ldds,             \
+                                                 (float*)dS_act, ld_act, prescale_indptr, partials,            \
+                                                 c->L().counters + CTR_LOSS, loss_accum);                      \
+    } while (0)
+    if (T <= 1) LOSS_L(1); else if (T <= 2) LOSS_L(2); else if (T <= 4) LOSS_L(4); else LOSS_L(LOSS_MAXT_CAP);
+#undef LOSS_L
 }
 
 // ------------------------------------------------------------------ adam
