@@ -380,38 +380,32 @@ __global__ void __launch_bounds__(256) k_route_pool_v(const float* __restrict__ 
         for (int64_t e0 = b; e0 < e; e0 += 32) {
             const int n = (int)mn64(32, e - e0);
             const int32_t my = lane < n ? t_idx[e0 + lane] : 0;
+            // POS8: u's position in each edge's row v, one lane per edge for the whole 32-edge chunk:
+            // the row's entries are loaded 8 at a time (independent loads) and compared, so the
+            // search costs ~1 round trip per chunk instead of a dependent chain per 4 edges
+            int32_t mykey = (int32_t)u;
+            if (POS8) {
+                mykey = -2;
+                if (lane < n) {
+                    const int64_t rb = __ldg(indptr + my), re = __ldg(indptr + my + 1);
+                    for (int64_t base = rb; base < re && mykey < 0; base += 8) {
+                        int32_t w[8];
+#pragma unroll
+                        for (int i = 0; i < 8; ++i) w[i] = base + i < re ? __ldg(idx + base + i) : -1;
+#pragma unroll
+                        for (int i = 0; i < 8; ++i)
+                            if (mykey < 0 && w[i] == (int32_t)u) mykey = (int32_t)(base + i - rb);
+                    }
+                }
+            }
             for (int j0 = 0; j0 < n; j0 += 4) {
                 int32_t v[4];
                 int4 a[4][T];
                 int32_t key[4];                 // what an argmax entry must equal: u, or u's position in v's row
 #pragma unroll
-                for (int k = 0; k < 4; ++k) v[k] = __shfl_sync(0xffffffffu, my, (j0 + k) & 31);
-                if (POS8) {
-                    int64_t rb[4], re[4];
-#pragma unroll
-                    for (int k = 0; k < 4; ++k) {
-                        rb[k] = j0 + k < n ? __ldg(indptr + v[k]) : 0;
-                        re[k] = j0 + k < n ? __ldg(indptr + v[k] + 1) : 0;
-                    }
-                    // u's position in each v's row, warp-cooperatively: 32 row entries per load, one
-                    // ballot (the 4 edges' loads are independent and issued together)
-                    int32_t xs[4];
-#pragma unroll
-                    for (int k = 0; k < 4; ++k)
-                        xs[k] = lane < re[k] - rb[k] ? __ldg(idx + rb[k] + lane) : -1;
-#pragma unroll
-                    for (int k = 0; k < 4; ++k) {
-                        const unsigned m = __ballot_sync(0xffffffffu, xs[k] == (int32_t)u);
-                        key[k] = m ? __ffs(m) - 1 : -2;
-                        for (int64_t base = rb[k] + 32; !m && key[k] < 0 && base < re[k]; base += 32) {
-                            const int32_t x = base + lane < re[k] ? __ldg(idx + base + lane) : -1;
-                            const unsigned m2 = __ballot_sync(0xffffffffu, x == (int32_t)u);
-                            if (m2) key[k] = (int32_t)(base - rb[k]) + __ffs(m2) - 1;
-                        }
-                    }
-                } else {
-#pragma unroll
-                    for (int k = 0; k < 4; ++k) key[k] = (int32_t)u;
+                for (int k = 0; k < 4; ++k) {
+                    v[k] = __shfl_sync(0xffffffffu, my, (j0 + k) & 31);
+                    key[k] = __shfl_sync(0xffffffffu, mykey, (j0 + k) & 31);
                 }
 #pragma unroll
                 for (int k = 0; k < 4; ++k)
