@@ -512,7 +512,7 @@ def main():
     per_launch_ms, launches_per_step = probe_ms[dom]
     ab = alg_bytes(dom, info, cfg, args.mode, info["n_groups"]) if cfg.aggr == "mean" else None
     achieved = ab / (per_launch_ms * 1e-3) / 1e9 if ab else None
-    roof = None if ab is None else {"kernel": "k_agg_mean_xa (layer-0 mean aggregation)", "bound": "hbm", "achieved": achieved,
+    roof = None if ab is None else {"kernel": "k_agg_mean_g4 (layer-0 mean aggregation)", "bound": "hbm", "achieved": achieved,
             "peak": peaks["hbm_gbs"], "unit": "GB/s", "frac": achieved / peaks["hbm_gbs"],
             "traffic": load_traffic(dom, key), "alg_bytes_per_launch": ab, "avg_launch_ms": per_launch_ms,
             "launches_per_step": launches_per_step, "peak_source": peak_src,
