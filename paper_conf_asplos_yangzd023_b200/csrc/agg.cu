@@ -952,10 +952,20 @@ __global__ void __launch_bounds__(256) k_csc_mean_g(const float* __restrict__ dX
     const unsigned gmask = LPR == 32 ? 0xffffffffu : (((1u << LPR) - 1u) << (grp * LPR));
     const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    int64_t nb = 0, ne = 0;                             // column extents one iteration ahead
+    {
+        const int64_t u = gw * RPW + grp;
+        if (u < ns) { nb = t_indptr[u]; ne = t_indptr[u + 1]; }
+    }
     for (int64_t u0 = gw * RPW; u0 < ns; u0 += nw * RPW) {
         const int64_t u = u0 + grp;
+        const int64_t b = nb, e = ne;
+        {
+            const int64_t un = u + nw * RPW;
+            nb = 0; ne = 0;
+            if (un < ns) { nb = t_indptr[un]; ne = t_indptr[un + 1]; }
+        }
         if (u >= ns) continue;                              // whole lane group idle
-        const int64_t b = t_indptr[u], e = t_indptr[u + 1];
         float acc[VPL][4];
 #pragma unroll
         for (int k = 0; k < VPL; ++k)
