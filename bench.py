@@ -53,7 +53,7 @@ def parse():
     p.add_argument("--no-graph", action="store_true")
     p.add_argument("--no-reg", action="store_true", help="exclude the REG rebuild (a1) from the step")
     p.add_argument("--probe", default="auto")
-    p.add_argument("--e2e-steps", type=int, default=5)
+    p.add_argument("--e2e-steps", type=int, default=20)
     p.add_argument("--cpu-sample-outputs", type=int, default=4096, help="cpu_baseline sample (~10 s)")
     p.add_argument("--ref-sample-outputs", type=int, default=1024, help="--impl reference per-step sample")
     p.add_argument("--scale", type=float, default=1.0, help="shrink the graph (debug only)")
@@ -421,9 +421,9 @@ def main():
     stream = torch.cuda.current_stream()
     t_opt = [0]
 
-    def step():
+    def step(pl=None):
         loss.zero_()
-        B.betty_step(ctx, plan, params, feats, labels, scale, grad, loss)
+        B.betty_step(ctx, pl or plan, params, feats, labels, scale, grad, loss)
         allreduce_grad(grad)
         t_opt[0] += 1
         B.betty_adam(ctx, params, grad, m, v, t_opt[0], zero_grad=True)
@@ -462,29 +462,75 @@ def main():
     launches = args.steps * (info["kernels_per_step"] + 1)
 
     # ------------------------------------- e2e: host buffers through the ABI
+    # Every step copies its own inputs (the full-batch blocks and the partition) from pinned host
+    # memory and reads its loss back.  Double-buffered when a second plan fits in HBM: the inputs of
+    # step i+1 are copied on a copy stream into the other buffer set while step i computes (a plan
+    # binds its blocks' device pointers, so each buffer set has its own plan); else serial.
     host = []
     for l, b in enumerate(ds.blocks):
         host += [torch.from_numpy(b.indptr).pin_memory(), torch.from_numpy(b.nbr_pos).pin_memory(),
                  torch.from_numpy(host_gid0 if l == 0 else b.src_gid).pin_memory()]
     host.append(torch.from_numpy(part).pin_memory())
-    devs = []
-    for db in dev_blocks:
-        devs += [db.indptr, db.indices, db.src_gid]
-    devs.append(dpart)
+
+    def dev_list(dbs, dp):
+        out = []
+        for db in dbs:
+            out += [db.indptr, db.indices, db.src_gid]
+        return out + [dp]
+    bufs, plans = [dev_list(dev_blocks, dpart)], [plan]
+    try:
+        dev_blocks2 = B.blocks_to_device(ds.blocks, local)
+        dev_blocks2[0].src_gid.copy_(dev_blocks[0].src_gid)
+        dpart2 = dpart.clone()
+        plan2, g2 = create_plan(B, ctx, model, dev_blocks2, dpart2, args.K, my_k, args.group or 0, flags)
+        if g2 != (args.group or 0):               # only the same launch grouping is the same step
+            plan2.free()
+            raise RuntimeError("second plan would need a smaller launch group")
+        if wv > 1 and not args.no_reg:
+            plan2.set_reg_rows(*reg_rows(cfg.n_out, rv, wv))
+        bufs.append(dev_list(dev_blocks2, dpart2))
+        plans.append(plan2)
+        step(plan2)                                # capture its graph outside the timed region
+        torch.cuda.synchronize()
+    except (B.BettyError, SystemExit, RuntimeError) as e:   # no room for a second buffer set: serial
+        print(f"e2e: single-buffered ({e})", file=sys.stderr)
+        dev_blocks2 = dpart2 = None
+        torch.cuda.synchronize()
+        torch.cuda.empty_cache()
     h2d = sum(x.numel() * x.element_size() for x in host)
     loss_host = torch.zeros(1).pin_memory()
+    cs = torch.cuda.Stream(device=device)
+    ev_copied = [torch.cuda.Event() for _ in bufs]
+    ev_used = [torch.cuda.Event() for _ in bufs]
+    nb = len(bufs)
+
+    def copy_in(b):
+        with torch.cuda.stream(cs):
+            for hsrc, ddst in zip(host, bufs[b]):
+                ddst.copy_(hsrc, non_blocking=True)
+            ev_copied[b].record(cs)
     if ws > 1:
         dist.barrier()
     torch.cuda.synchronize()
     f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     f0.record(stream)
-    for _ in range(args.e2e_steps):
-        for hsrc, ddst in zip(host, devs):
-            ddst.copy_(hsrc, non_blocking=True)
-        step()
+    cs.wait_stream(stream)
+    copy_in(0)
+    for i in range(args.e2e_steps):
+        b = i % nb
+        stream.wait_event(ev_copied[b])
+        if nb > 1 and i + 1 < args.e2e_steps:     # next step's inputs, once the step that used them is done
+            if i >= 1:
+                cs.wait_event(ev_used[1 - b])
+            copy_in(1 - b)
+        step(plans[b])
+        ev_used[b].record(stream)
         loss_host.copy_(loss, non_blocking=True)
         stream.synchronize()
         _ = float(loss_host[0])
+        if nb == 1 and i + 1 < args.e2e_steps:
+            cs.wait_stream(stream)
+            copy_in(0)
     f1.record(stream)
     torch.cuda.synchronize()
     e2e_ms = f0.elapsed_time(f1) / args.e2e_steps
@@ -492,6 +538,8 @@ def main():
         te = torch.tensor([e2e_ms], device=device, dtype=torch.float64)
         dist.all_reduce(te, op=dist.ReduceOp.MAX)
         e2e_ms = float(te[0])
+    for pl in plans[1:]:
+        pl.free()
 
     # ---------------------------------- roofline of the dominant kernel
     sites = {"agg_l0": 1, "gemm_fwd_l0": 2, "gemm_red_l0": 3, "extract": 4, "reg": 5}
@@ -548,7 +596,8 @@ def main():
             "plan": {k: info[k] for k in ("n_groups", "edges", "n_src", "n_dst", "reg_nnz", "arena_bytes",
                                           "kernels_per_step")},
             "e2e": {"value": edges_all / (e2e_ms * 1e-3), "unit": "edges/s", "ms_per_step": e2e_ms,
-                    "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": 4},
+                    "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": 4,
+                    "input_buffers": nb},
             "gpu_launches": launches,
             "clocks": clk,
             "roofline": roof,
