@@ -1,5 +1,5 @@
 """The bench line contract (task statement / SURVEY.md §8(d)) on the committed measurement
-(profiles/r01h_bench_C3.jsonl, written by bench.py on a B200): every key the driver and the judge
+(profiles/r01i_bench_C3.jsonl, written by bench.py on a B200): every key the driver and the judge
 read is present with a sane value.  CPU only (reads the committed JSON)."""
 import json
 import os
@@ -13,7 +13,7 @@ def _line(name):
 
 
 def test_c3_bench_line_contract():
-    d = _line("r01h_bench_C3.jsonl")
+    d = _line("r01i_bench_C3.jsonl")
     for k in ("metric", "value", "unit", "n_gpus", "steps", "warmup", "ms_per_step", "higher_is_better", "scaling",
               "vs_baseline", "dtype", "data", "config", "e2e", "gpu_launches", "clocks", "roofline", "cpu_baseline"):
         assert k in d, k
@@ -25,6 +25,7 @@ def test_c3_bench_line_contract():
     assert abs(d["value"] - d["edges_per_step"] / (d["ms_per_step"] * 1e-3)) < 1e-6 * d["value"]
     e = d["e2e"]
     assert e["h2d_bytes_per_step"] > 0 and e["d2h_bytes_per_step"] > 0 and 0 < e["value"] < d["value"]
+    assert e["input_buffers"] in (1, 2)
     r = d["roofline"]
     assert r["bound"] == "hbm" and r["unit"] == "GB/s" and 0 < r["frac"] < 1
     assert abs(r["frac"] - r["achieved"] / r["peak"]) < 1e-9
@@ -36,6 +37,6 @@ def test_c3_bench_line_contract():
 
 
 def test_other_config_lines():
-    for name, cfg in (("r01h_bench_C4.jsonl", "C4"), ("r01h_bench_C5.jsonl", "C5")):
+    for name, cfg in (("r01h_bench_C4.jsonl", "C4"), ("r01i_bench_C5.jsonl", "C5")):
         d = _line(name)
         assert d["config"]["workload"].startswith(cfg) and d["value"] > 0 and d["ms_per_step"] > 0
