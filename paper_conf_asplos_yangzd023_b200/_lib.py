@@ -9,7 +9,8 @@ import ctypes
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libbetty.so")
+# BETTY_LIB_PATH: an alternative build of the same library (tuning sweeps only, tools/sweep_g4.sh)
+LIB_PATH = os.environ.get("BETTY_LIB_PATH") or os.path.join(_HERE, "libbetty.so")
 
 i32, i64, f32, vp = ctypes.c_int32, ctypes.c_int64, ctypes.c_float, ctypes.c_void_p
 P_i32 = ctypes.POINTER(ctypes.c_int32)

@@ -478,7 +478,17 @@ __global__ void __launch_bounds__(256) k_route_pool_v(const float* __restrict__ 
 //    memory and stream XA out.  A row whose neighbours exceed the slots ("long" row, e.g.
 //    full-neighbourhood layers) is a stage of its own that the consumers reduce straight from
 //    global memory.
-constexpr int G4_STAGES = 8, G4_PROD = 4, G4_CPP = 3, G4_MAXR = 16, G4_CLAIM = 64;
+#ifndef BETTY_G4_STAGES          // (overridable at build time for tuning sweeps: tools/sweep_g4.sh)
+#define BETTY_G4_STAGES 8
+#endif
+#ifndef BETTY_G4_PROD
+#define BETTY_G4_PROD 4
+#endif
+#ifndef BETTY_G4_CPP
+#define BETTY_G4_CPP 4
+#endif
+constexpr int G4_STAGES = BETTY_G4_STAGES, G4_PROD = BETTY_G4_PROD, G4_CPP = BETTY_G4_CPP, G4_MAXR = 16,
+              G4_CLAIM = 64;
 constexpr int G4_CONS = G4_PROD * G4_CPP;             // consumer warps: G4_CPP per producer
 constexpr int G4_THREADS = 32 * (G4_PROD + G4_CONS);
 static_assert(G4_STAGES % G4_PROD == 0, "stages are dealt round-robin to the producers");
