@@ -679,8 +679,11 @@ __global__ void __launch_bounds__(G4_THREADS, 1) k_agg_mean_g4(const __grid_cons
             if (n < 0) break;
             const uint8_t* sdat = g4_smem + (size_t)s * a.stage_bytes;
             if (!H.lng) {
-                for (int u = ct; u < n * NV; u += NCT) {
-                    const int i = u / NV, j = u - i * NV;
+                // (row i, vector j) pairs u = ct, ct + NCT, ...: i, j advance incrementally (no division)
+                int i = ct / NV, j = ct - (ct / NV) * NV;
+                const int di = NCT / NV, dj = NCT - di * NV;
+                for (int u = ct; u < n * NV; u += NCT, i += di, j += dj) {
+                    if (j >= NV) { j -= NV; ++i; }
                     const int b = H.off[i], e = H.off[i + 1];
                     float acc[VW];
 #pragma unroll
