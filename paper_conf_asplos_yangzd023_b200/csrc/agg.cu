@@ -487,8 +487,14 @@ __global__ void __launch_bounds__(256) k_route_pool_v(const float* __restrict__ 
 #ifndef BETTY_G4_CPP
 #define BETTY_G4_CPP 4
 #endif
-constexpr int G4_STAGES = BETTY_G4_STAGES, G4_PROD = BETTY_G4_PROD, G4_CPP = BETTY_G4_CPP, G4_MAXR = 16,
-              G4_CLAIM = 64;
+#ifndef BETTY_G4_MAXR
+#define BETTY_G4_MAXR 16
+#endif
+#ifndef BETTY_G4_CLAIM
+#define BETTY_G4_CLAIM 64
+#endif
+constexpr int G4_STAGES = BETTY_G4_STAGES, G4_PROD = BETTY_G4_PROD, G4_CPP = BETTY_G4_CPP, G4_MAXR = BETTY_G4_MAXR,
+              G4_CLAIM = BETTY_G4_CLAIM;
 constexpr int G4_CONS = G4_PROD * G4_CPP;             // consumer warps: G4_CPP per producer
 constexpr int G4_THREADS = 32 * (G4_PROD + G4_CONS);
 static_assert(G4_STAGES % G4_PROD == 0, "stages are dealt round-robin to the producers");
