@@ -242,8 +242,14 @@ __device__ __forceinline__ int64_t dst_id(const RankSet& R, int l, int j, int32_
 // offset, and the warp then walks the rows' edges as one flat range, UNR edges
 // per lane in flight (independent load chains), every lane busy whatever the
 // degree mix.  Row data live in a per-warp shared slice.
-constexpr int FLAT_UNR = 4;
-constexpr int RL_UNR = 4;          // relabel chains per lane (8: 128 registers, measured slower)
+#ifndef BETTY_FLAT_UNR             // (overridable at build time for tuning sweeps)
+#define BETTY_FLAT_UNR 4
+#endif
+#ifndef BETTY_RL_UNR
+#define BETTY_RL_UNR 4
+#endif
+constexpr int FLAT_UNR = BETTY_FLAT_UNR;
+constexpr int RL_UNR = BETTY_RL_UNR;   // relabel chains per lane (8: 128 registers, measured slower)
 struct FlatRows {
     int pre[33];        // exclusive edge offsets of the warp's rows (pre[32] = total)
     int64_t fb[32];     // full-batch row start of each row
