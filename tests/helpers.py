@@ -109,3 +109,20 @@ def assert_close(x, ref, rtol, name=""):
     assert np.all(np.isfinite(x)), f"{name}: non-finite values"
     assert re <= rtol, f"{name}: rel l2 err {re:.3e} > {rtol:.1e}"
     assert ma <= 10 * rtol * mx + 1e-300, f"{name}: max abs err {ma:.3e} > 10*rtol*max|ref| = {10 * rtol * mx:.3e}"
+
+
+def param_tensors(flat, dims, aggr):
+    """Flat gradient -> [(name, array)] per layer and tensor (W_pool, b_pool,
+    W_self, W_neigh, b), the flat layout of synth.init_params."""
+    out = []
+    for l, d in enumerate(split_params(np.asarray(flat, dtype=np.float64), dims, aggr)):
+        for name, a in d.items():
+            out.append((f"{name}{l}", a))
+    return out
+
+
+def assert_grad_close(x, ref, dims, aggr, rtol, name=""):
+    """Reading #18 applied PER PARAMETER TENSOR (not to the flat vector, where
+    a small tensor such as a bias could hide a large relative error)."""
+    for (tn, a), (_, b) in zip(param_tensors(x, dims, aggr), param_tensors(ref, dims, aggr)):
+        assert_close(a, b, rtol, f"{name} {tn}")

@@ -18,7 +18,7 @@ import torch
 
 import oracle
 import synth
-from tests.helpers import assert_close
+from tests.helpers import assert_close, assert_grad_close
 
 pytestmark = pytest.mark.gpu
 
@@ -77,7 +77,7 @@ def test_c5_scaled_step_vs_oracle(B, ctx, c5s, group):
     Y = torch.as_tensor(ds.labels).cuda()
     for rep in range(2):          # graph replay: the second step re-extracts into the same arenas
         g, l = _step(B, ctx, plan, cfg, P, X, Y)
-        assert_close(g, og, 2e-2, f"grad rep {rep}")
+        assert_grad_close(g, og, cfg.dims, cfg.aggr, 2e-2, f"grad rep {rep}")
         assert l == pytest.approx(ol, rel=2e-2)
     plan.free()
 
@@ -95,7 +95,66 @@ def test_c5_scaled_invariant(B, ctx, c5s):
                                    flags=B.PLAN_GRAPH)
         res.append(_step(B, ctx, plan, cfg, P, X, Y))
         plan.free()
-    assert_close(res[0][0], res[1][0], 1e-5, "sum of micro-batch gradients vs full batch")
+    assert_grad_close(res[0][0], res[1][0], cfg.dims, cfg.aggr, 1e-5, "sum of micro-batch gradients vs full batch")
+    assert res[0][1] == pytest.approx(res[1][1], rel=1e-5)
+
+
+# ----------------------------------------------- C5 at 1/50: the feature table exceeds L2
+@pytest.fixture(scope="module")
+def c5m(B, ctx):
+    """C5's shape at 1/50 (2.2 M nodes, 16 M pairs, 24 k outputs): the bf16 table (570 MB) and the
+    fp32 table (1.1 GB) are several times the 126 MB L2, so the layer-0 gathers stream from HBM as
+    in the full-size run."""
+    cfg = synth.scaled(synth.CONFIGS["C5"], 0.02)
+    ds = synth.make(cfg)
+    dev = B.blocks_to_device(ds.blocks)
+    ip, col, w = B.betty_reg_build(ctx, dev[-1])
+    part = B.betty_reg_partition(ip.cpu().numpy(), col.cpu().numpy(), w.cpu().numpy(), 8, method="multilevel")
+    return cfg, ds, dev, part
+
+
+@pytest.mark.parametrize("mode,rtol", [("bf16", 2e-2), ("fp32", 1e-5)])
+def test_c5_beyond_l2_sampled_micro_batch(B, ctx, c5m, mode, rtol):
+    """24 outputs of micro-batch 0 as their own micro-batch through the fused step, on the whole
+    > L2 feature table, against the float64 oracle (per tensor, reading #18)."""
+    cfg, ds, dev, part = c5m
+    assert ds.feats.nbytes > 4 * 126 * 2 ** 20
+    idx = np.nonzero(part == 0)[0][:24]
+    p2 = np.ones(cfg.n_out, np.int32)
+    p2[idx] = 0
+    params = synth.init_params(cfg.dims, cfg.aggr, seed=cfg.seeds["init"])
+    og, ol = oracle.step(cfg.dims, cfg.aggr, mode == "bf16", ds.blocks, p2, 2, [0], params, ds.feats, ds.labels,
+                         1.0 / cfg.n_out)
+    model = B.Model(cfg.dims, cfg.aggr, mode, mode)
+    plan = B.betty_plan_create(ctx, model, dev, torch.as_tensor(p2).cuda(), 2, [0], group=0,
+                               flags=B.PLAN_GRAPH | B.PLAN_REG)
+    X = torch.as_tensor(ds.feats).cuda()
+    if mode == "bf16":
+        X = X.to(torch.bfloat16).contiguous()
+    P = torch.as_tensor(params).cuda()
+    Y = torch.as_tensor(ds.labels).cuda()
+    g, l = _step(B, ctx, plan, cfg, P, X, Y)
+    assert_grad_close(g, og, cfg.dims, cfg.aggr, rtol, f"{mode} grad")
+    assert l == pytest.approx(ol, rel=rtol)
+    plan.free()
+
+
+def test_c5_beyond_l2_invariant(B, ctx, c5m):
+    """Betty's invariant on the > L2 table: the K = 8 step (launch groups of 3) equals the K = 1 step
+    (fp32, 1e-5 per tensor)."""
+    cfg, ds, dev, part = c5m
+    params = synth.init_params(cfg.dims, cfg.aggr, seed=cfg.seeds["init"])
+    P = torch.as_tensor(params).cuda()
+    X = torch.as_tensor(ds.feats).cuda()
+    Y = torch.as_tensor(ds.labels).cuda()
+    model = B.Model(cfg.dims, cfg.aggr, "fp32", "fp32")
+    res = []
+    for k, p, grp in ((8, part, 3), (1, np.zeros(cfg.n_out, np.int32), 0)):
+        plan = B.betty_plan_create(ctx, model, dev, torch.as_tensor(p).cuda(), k, list(range(k)), group=grp,
+                                   flags=B.PLAN_GRAPH)
+        res.append(_step(B, ctx, plan, cfg, P, X, Y))
+        plan.free()
+    assert_grad_close(res[0][0], res[1][0], cfg.dims, cfg.aggr, 1e-5, "K=8 vs K=1")
     assert res[0][1] == pytest.approx(res[1][1], rel=1e-5)
 
 
@@ -177,6 +236,6 @@ def test_c5_full_sampled_micro_batch(B, ctx, c5):
     P = torch.as_tensor(params).cuda()
     Y = torch.as_tensor(ds.labels).cuda()
     g, l = _step(B, ctx, plan, cfg, P, X, Y)
-    assert_close(g, og, 2e-2, "grad")
+    assert_grad_close(g, og, cfg.dims, cfg.aggr, 2e-2, "grad")
     assert l == pytest.approx(ol, rel=2e-2)
     plan.free()

@@ -7,7 +7,7 @@ import torch
 
 import oracle
 import synth
-from tests.helpers import assert_close, load_golden, tiny
+from tests.helpers import assert_close, assert_grad_close, load_golden, tiny
 
 pytestmark = pytest.mark.gpu
 
@@ -111,7 +111,7 @@ def test_plan_reg_rows(B, ctx):
             loss = torch.zeros(1, device="cuda")
             B.betty_step(ctx, plan, P, X, Y, 1.0 / len(sd), grad, loss)
             B.betty_sync_check(ctx)
-            assert_close(grad.cpu().numpy(), og, 1e-5, f"rows {r0}:{r1} rep {rep}")
+            assert_grad_close(grad.cpu().numpy(), og, dims, "mean", 1e-5, f"rows {r0}:{r1} rep {rep}")
     with pytest.raises(B.BettyError):
         plan.set_reg_rows(0, 61)
     plan.free()
@@ -289,7 +289,7 @@ def test_sage_micro_batch(B, ctx, c, mode):
         og, ol, olog = oracle.sage(c["dims"], c["aggr"], mode == "bf16", om, params, feats, labels, scale,
                                    want_logits=True)
         assert_close(logits.cpu().numpy(), olog, RTOL[mode], f"logits k={k}")
-        assert_close(grad.cpu().numpy(), og, RTOL[mode], f"grad k={k}")
+        assert_grad_close(grad.cpu().numpy(), og, c["dims"], c["aggr"], RTOL[mode], f"grad k={k}")
         assert loss.item() == pytest.approx(ol, rel=RTOL[mode])
         saved.free()
 
@@ -319,7 +319,7 @@ def test_step_matches_oracle(B, ctx, c, mode, group, graph):
         loss = torch.zeros(1, device="cuda")
         B.betty_step(ctx, plan, P, X, Y, scale, grad, loss)
         B.betty_sync_check(ctx)
-        assert_close(grad.cpu().numpy(), og, RTOL[mode], f"grad rep={rep}")
+        assert_grad_close(grad.cpu().numpy(), og, c["dims"], c["aggr"], RTOL[mode], f"grad rep={rep}")
         assert loss.item() == pytest.approx(ol, rel=RTOL[mode])
     info = plan.info()
     assert info["kernels_per_step"] > 0
@@ -345,7 +345,7 @@ def test_sum_of_micro_batches_equals_full_batch_on_gpu(B, ctx):
         torch.cuda.synchronize()
         res.append((grad.cpu().numpy(), loss.item()))
         plan.free()
-    assert_close(res[1][0], res[0][0], 1e-5, "sum_k g_k vs g_full")
+    assert_grad_close(res[1][0], res[0][0], c["dims"], "mean", 1e-5, "sum_k g_k vs g_full")
     assert res[1][1] == pytest.approx(res[0][1], rel=1e-5)
 
 
@@ -383,7 +383,7 @@ def test_c1_cora_config(B, ctx):
         torch.cuda.synchronize()
         og, ol = oracle.step(cfg.dims, "mean", mode == "bf16", ds.blocks, part, 2, [0, 1], params, ds.feats,
                              ds.labels, 1.0 / cfg.n_out)
-        assert_close(grad.cpu().numpy(), og, RTOL[mode], f"C1 grad {mode}")
+        assert_grad_close(grad.cpu().numpy(), og, cfg.dims, "mean", RTOL[mode], f"C1 grad {mode}")
         assert loss.item() == pytest.approx(ol, rel=RTOL[mode])
         plan.free()
 
@@ -408,5 +408,5 @@ def test_pool_byte_positions(B, ctx, mode, pos8, monkeypatch):
     B.betty_sync_check(ctx)
     og, ol = oracle.step(c["dims"], c["aggr"], mode == "bf16", blocks, part, K, [0, 1, 2], params, feats, labels,
                          1.0 / len(sd))
-    assert_close(grad.cpu().numpy(), og, RTOL[mode], "grad")
+    assert_grad_close(grad.cpu().numpy(), og, c["dims"], c["aggr"], RTOL[mode], "grad")
     plan.free()
