@@ -219,10 +219,12 @@ BETTY_API betty_status betty_adam(betty_ctx* ctx, float* params, float* grad, fl
 BETTY_API betty_status betty_plan_group_blocks(betty_ctx* ctx, betty_plan* plan, int32_t g, betty_block* out,
                                                betty_stream stream);
 
-/* Test hook for the dense kernels (bf16 operands, fp32 result; synchronises).
+/* Test hook for the dense kernels (fp32 result; synchronises).
  * kind 0: C[M x N] = A[M x K] . B^T with B given K-major as [N x K];
  * kind 1: C[K x N] += A[M x K]^T . B[M x N] (the dW reduction; C must be
- * [K x N] contiguous).  use_tc selects the tcgen05 path (else SIMT). */
+ * [K x N] contiguous).  kind | 2: fp32 operands (FP32 mode: 3xTF32 on
+ * tcgen05 when use_tc, else SIMT FFMA); otherwise bf16 operands.  use_tc
+ * selects the tcgen05 path (else SIMT). */
 BETTY_API betty_status betty_test_gemm(betty_ctx* ctx, int32_t kind, const void* A, int64_t lda, const void* B,
                                        int64_t ldb, int64_t M, int64_t M_cap, int32_t K, int32_t N, float* C,
                                        int64_t ldc, int32_t use_tc, betty_stream stream);

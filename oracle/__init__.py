@@ -56,6 +56,9 @@ def lib():
         L.oracle_step.restype = ctypes.c_int
         L.oracle_step.argtypes = [ctypes.c_int, P, ctypes.c_int, ctypes.c_int, P, P, i64, i32, P, i32, P, P, i64,
                                   P, dbl, P, ctypes.POINTER(dbl)]
+        L.oracle_sage_ties.restype = i64
+        L.oracle_sage_ties.argtypes = [ctypes.c_int, P, ctypes.c_int, ctypes.c_int, P, P, P, i64, P, dbl, P,
+                                       ctypes.POINTER(dbl), dbl, i64, P, P, P, P, P, P]
         L.oracle_mem_estimate.restype = ctypes.c_int
         L.oracle_mem_estimate.argtypes = [ctypes.c_int, P, ctypes.c_int, P, P, P, P]
         L.oracle_bf16_round.restype = dbl
@@ -66,6 +69,11 @@ def lib():
         L.oracle_block_free.argtypes = [P, ctypes.c_int]
         _lib = L
     return _lib
+
+
+def _aggr(aggr: str) -> int:
+    """aggregator code of oracle.c: 0 mean, 1 pool (Table 1)"""
+    return {"mean": 0, "pool": 1}[aggr]
 
 
 def _p(a: Optional[np.ndarray]):
@@ -163,10 +171,33 @@ def sage(dims: Sequence[int], aggr: str, bf16: bool, blocks: Sequence, params: n
     grad = np.zeros(len(params), dtype=np.float64)
     loss = ctypes.c_double(0.0)
     logits = np.zeros((blocks[-1].n_dst, dims[-1]), dtype=np.float64) if want_logits else None
-    lib().oracle_sage(L, _p(d), 1 if aggr == "pool" else 0, int(bf16), force_form, ctypes.addressof(arr),
+    lib().oracle_sage(L, _p(d), _aggr(aggr), int(bf16), force_form, ctypes.addressof(arr),
                       _p(params), _p(feats), feats.shape[1], _p(labels), loss_scale, _p(grad), ctypes.byref(loss),
                       _p(logits))
     return grad, loss.value, logits
+
+
+def sage_ties(dims: Sequence[int], aggr: str, bf16: bool, blocks: Sequence, params: np.ndarray, feats: np.ndarray,
+              labels: np.ndarray, loss_scale: float, tau: float, cap: int = 1 << 20):
+    """oracle_sage plus the hidden ReLU decisions finite precision may take either way (reading #24):
+    every (level, v, j) with |S| <= tau * M (M = sum of the magnitudes of S's terms), with S, M and
+    the gradient g the decision gates.  Returns (grad, loss, ties dict of arrays, found)."""
+    L = len(blocks)
+    arr, keep = _oblocks(blocks)
+    d = np.ascontiguousarray(dims, dtype=np.int32)
+    params = np.ascontiguousarray(params, dtype=np.float64)
+    feats = np.ascontiguousarray(feats, dtype=np.float32)
+    labels = np.ascontiguousarray(labels, dtype=np.int32)
+    grad = np.zeros(len(params), dtype=np.float64)
+    loss = ctypes.c_double(0.0)
+    t = {"level": np.zeros(cap, np.int32), "v": np.zeros(cap, np.int64), "j": np.zeros(cap, np.int32),
+         "S": np.zeros(cap), "M": np.zeros(cap), "g": np.zeros(cap)}
+    found = lib().oracle_sage_ties(L, _p(d), _aggr(aggr), int(bf16), ctypes.addressof(arr),
+                                   _p(params), _p(feats), feats.shape[1], _p(labels), loss_scale, _p(grad),
+                                   ctypes.byref(loss), tau, cap, _p(t["level"]), _p(t["v"]), _p(t["j"]), _p(t["S"]),
+                                   _p(t["M"]), _p(t["g"]))
+    n = min(found, cap)
+    return grad, loss.value, {k: a[:n] for k, a in t.items()}, found
 
 
 def step(dims: Sequence[int], aggr: str, bf16: bool, full: Sequence, part: np.ndarray, K: int,
@@ -182,7 +213,7 @@ def step(dims: Sequence[int], aggr: str, bf16: bool, full: Sequence, part: np.nd
     labels = np.ascontiguousarray(labels, dtype=np.int32)
     grad = np.zeros(len(params), dtype=np.float64)
     loss = ctypes.c_double(0.0)
-    rc = lib().oracle_step(L, _p(d), 1 if aggr == "pool" else 0, int(bf16), ctypes.addressof(arr), _p(part),
+    rc = lib().oracle_step(L, _p(d), _aggr(aggr), int(bf16), ctypes.addressof(arr), _p(part),
                            full[-1].n_dst, K, _p(ks), len(ks), _p(params), _p(feats), feats.shape[1], _p(labels),
                            loss_scale, _p(grad), ctypes.byref(loss))
     if rc != 0:
@@ -200,7 +231,7 @@ def mem_estimate(dims: Sequence[int], aggr: str, blocks: Sequence) -> np.ndarray
     ns = np.array([b.n_src for b in blocks], dtype=np.int64)
     ne = np.array([int(b.indptr[-1]) for b in blocks], dtype=np.int64)
     t = np.zeros(9, dtype=np.int64)
-    lib().oracle_mem_estimate(L, _p(d), 1 if aggr == "pool" else 0, _p(nd), _p(ns), _p(ne), _p(t))
+    lib().oracle_mem_estimate(L, _p(d), _aggr(aggr), _p(nd), _p(ns), _p(ne), _p(t))
     return t
 
 

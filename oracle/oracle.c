@@ -21,6 +21,11 @@
  *
  *   oracle_step     -- one batch: all K micro-batches, gradients summed
  *                      (Fig. 6)
+ *   oracle_sage_ties -- oracle_sage, also reporting every hidden ReLU decision
+ *                      that finite precision can take either way (reading
+ *                      #24): |S| <= tau * M with M = the sum of the magnitudes
+ *                      of the terms of S, and the gradient g that the decision
+ *                      gates in the backward (dS = g if S > 0 else 0)
  *
  * Readings of the paper where it is silent or garbled are listed in DESIGN.md
  * §3 and SURVEY.md §8(c); the numbers in comments (#n) refer to that table.
@@ -271,6 +276,34 @@ static void mm_acc(mat* out, const mat* A, int tA, const mat* B, int tB, int bf1
     free(a); free(b);
 }
 
+/* out[i][j] += sum_k |opA(i,k)| * |opB(k,j)| -- the magnitude of the terms of
+ * the same product (for the ReLU-decision report of oracle_sage_ties). */
+static void mm_acc_abs(mat* out, const mat* A, int tA, const mat* B, int tB, int bf16) {
+    int64_t M = tA ? A->c : A->r, K = tA ? A->r : A->c, N = tB ? B->r : B->c;
+    for (int64_t i = 0; i < M; ++i)
+        for (int64_t k = 0; k < K; ++k) {
+            double a = tA ? AT(*A, k, i) : AT(*A, i, k);
+            a = fabs(bf16 ? bf16_round(a) : a);
+            for (int64_t j = 0; j < N; ++j) {
+                double b = tB ? AT(*B, j, k) : AT(*B, k, j);
+                AT(*out, i, j) += a * fabs(bf16 ? bf16_round(b) : b);
+            }
+        }
+}
+
+/* ReLU-decision report (oracle_sage_ties): set while that call runs */
+typedef struct {
+    double tau;
+    int64_t cap, n, found;   /* stored entries (<= cap), decisions found */
+    int32_t* level;      /* the decision is the mask of H_level (level = l + 1 for layer l's output) */
+    int64_t* v;
+    int32_t* j;
+    double* S;           /* the pre-activation */
+    double* M;           /* sum of the magnitudes of its terms */
+    double* g;           /* the gradient the decision gates (dX of layer level, before the mask) */
+} tie_report;
+static tie_report* g_ties = NULL;
+
 /* parameter block of layer l: (pool: W_pool [Fi x Fi], b_pool [Fi]),
  * W_self [Fi x Fo], W_neigh [Fi x Fo], b [Fo] -- flat, row-major */
 typedef struct { int64_t wp, bp, ws, wn, b, end; } poff;
@@ -403,6 +436,38 @@ int oracle_sage(int L, const int32_t* dims, int aggr, int bf16, int force_form, 
             mm_acc(&S, &Aagg[l], 0, &Wn, 0, bf16);
             mat_free(&Wp); mat_free(&bp); mat_free(&onesS);
         }
+        if (g_ties && l < L - 1) {
+            /* M = the same sum over magnitudes: |X_d||W_s| + |A||W_n| (or D+ P |X||W_n|) + |b| */
+            mat Mg = mat_new(nd, fo);
+            mm_acc_abs(&Mg, &Xd, 0, &Ws, 0, bf16);
+            mm_acc_abs(&Mg, &ones, 0, &bb, 0, bf16);
+            if (!pool && projf[l]) {
+                mat Za = mat_new(ns, fo);
+                mm_acc_abs(&Za, &X, 0, &Wn, 0, bf16);
+                for (int64_t v = 0; v < nd; ++v) {
+                    int64_t deg = B->indptr[v + 1] - B->indptr[v];
+                    for (int64_t e = B->indptr[v]; e < B->indptr[v + 1]; ++e)
+                        for (int64_t f = 0; f < fo; ++f) AT(Mg, v, f) += AT(Za, B->indices[e], f) / (double)deg;
+                }
+                mat_free(&Za);
+            } else {
+                mat Aa = mat_new(nd, fi);
+                for (int64_t t = 0; t < nd * fi; ++t) Aa.a[t] = fabs(Aagg[l].a[t]);
+                mm_acc_abs(&Mg, &Aa, 0, &Wn, 0, bf16);
+                mat_free(&Aa);
+            }
+            for (int64_t v = 0; v < nd; ++v)
+                for (int64_t f = 0; f < fo; ++f) {
+                    if (!(fabs(AT(S, v, f)) <= g_ties->tau * AT(Mg, v, f))) continue;
+                    g_ties->found++;
+                    if (g_ties->n < g_ties->cap) {
+                        int64_t q = g_ties->n++;
+                        g_ties->level[q] = l + 1; g_ties->v[q] = v; g_ties->j[q] = (int32_t)f;
+                        g_ties->S[q] = AT(S, v, f); g_ties->M[q] = AT(Mg, v, f); g_ties->g[q] = 0.0;
+                    }
+                }
+            mat_free(&Mg);
+        }
         mat_free(&Ws); mat_free(&Wn); mat_free(&bb); mat_free(&ones);
         if (l < L - 1) {
             H[l + 1] = S;                                     /* ReLU; bf16: stored in bf16 */
@@ -501,6 +566,9 @@ int oracle_sage(int L, const int32_t* dims, int aggr, int bf16, int force_form, 
         mat_free(&Ws); mat_free(&Wn); mat_free(&gWs); mat_free(&gWn); mat_free(&gb); mat_free(&ones);
         mat_free(&dS);
         if (l > 0) {                                          /* dS_{l-1} = dX (.) [H_l > 0] */
+            if (g_ties)
+                for (int64_t q = 0; q < g_ties->n; ++q)
+                    if (g_ties->level[q] == l) g_ties->g[q] = AT(dX, g_ties->v[q], g_ties->j[q]);
             for (int64_t t = 0; t < ns * fi; ++t) if (!(X.a[t] > 0.0)) dX.a[t] = 0.0;
             dS = dX;
         } else {
@@ -512,6 +580,20 @@ int oracle_sage(int L, const int32_t* dims, int aggr, int bf16, int force_form, 
     for (int l = 0; l < L; ++l) { mat_free(&Aagg[l]); mat_free(&Zp[l]); free(arg[l]); }
     free(H); free(Aagg); free(Zp); free(arg); free(projf);
     return 0;
+}
+
+/* oracle_sage plus the report of the hidden ReLU decisions within tau of the
+ * boundary (reading #24): up to cap entries (level, v, j, S, M, g); returns
+ * the number of such decisions (if it exceeds cap only the first cap are stored). */
+int64_t oracle_sage_ties(int L, const int32_t* dims, int aggr, int bf16, const oblock* mb, const double* params,
+                         const float* feats, int64_t ld, const int32_t* labels, double loss_scale, double* grad,
+                         double* loss, double tau, int64_t cap, int32_t* level, int64_t* v, int32_t* j, double* S,
+                         double* M, double* g) {
+    tie_report r = {tau, cap, 0, 0, level, v, j, S, M, g};
+    g_ties = &r;
+    oracle_sage(L, dims, aggr, bf16, -1, mb, params, feats, ld, labels, loss_scale, grad, loss, NULL);
+    g_ties = NULL;
+    return r.found;
 }
 
 /* ------------------------------------------------------------------------ */

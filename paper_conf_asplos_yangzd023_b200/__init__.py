@@ -317,9 +317,12 @@ def betty_adam(ctx: Context, params: torch.Tensor, grad: torch.Tensor, m: torch.
 
 def betty_test_gemm(ctx: Context, kind: int, A: torch.Tensor, B: torch.Tensor, K: int, N: int, use_tc: bool = True,
                     M: Optional[int] = None, stream=None) -> torch.Tensor:
-    """Test hook of the dense kernels.  kind 0: A[M,K] @ B[N,K]^T; kind 1: A[M,K]^T @ B[M,N]."""
+    """Test hook of the dense kernels.  kind 0: A[M,K] @ B[N,K]^T; kind 1: A[M,K]^T @ B[M,N].  fp32
+    operands (A.dtype float32) select FP32 mode (3xTF32 on tcgen05 when use_tc, else SIMT)."""
     M = A.shape[0] if M is None else M
-    if kind == 0:
+    if A.dtype == torch.float32:
+        kind |= 2
+    if kind & 1 == 0:
         # rows up to A.shape[0] (the capacity) may be written; row stride padded to 16 bytes
         ldc = (N + 3) // 4 * 4
         Cfull = torch.zeros((A.shape[0], ldc), dtype=torch.float32, device=A.device)

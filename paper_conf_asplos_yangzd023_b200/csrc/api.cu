@@ -101,6 +101,8 @@ extern "C" betty_status betty_ctx_create(int device, betty_alloc_fn alloc, betty
     init_kernel_attrs();
     const char* no_tc = getenv("BETTY_NO_TC");
     c->use_tc = !(no_tc && no_tc[0] == '1') && tc_available();
+    const char* simt = getenv("BETTY_FP32_SIMT");
+    c->fp32_tc = !(simt && simt[0] == '1');
     cudaMemset(c->dev_err, 0, 16);
     cudaDeviceSynchronize();
     *out = c;
@@ -911,19 +913,29 @@ extern "C" betty_status betty_test_gemm(betty_ctx* c, int32_t kind, const void* 
     const bool saved = c->use_tc;
     c->use_tc = use_tc && tc_available();
     betty_status st = BETTY_OK;
-    if (kind == 0) {            // C[M x N] = A[M x K] . B, B given as [N x K] (K-major)
+    const bool f32 = (kind & 2) != 0;     // fp32 operands: 3xTF32 on the tensor cores (use_tc) or SIMT FFMA
+    const bool saved_f = c->fp32_tc;
+    c->fp32_tc = use_tc != 0;
+    if ((kind & 1) == 0) {      // C[M x N] = A[M x K] . B, B given as [N x K] (K-major)
         GemmRow g{};
-        g.A = A; g.lda = lda; g.a_bf16 = true;
-        g.B = B; g.ldb = ldb; g.b_bf16 = true; g.transB = true;
+        g.A = A; g.lda = lda; g.a_bf16 = !f32;
+        g.B = B; g.ldb = ldb; g.b_bf16 = !f32; g.transB = true;
         g.M_dev = Md; g.M_cap = std::max<int64_t>(M_cap, 1); g.K = K; g.N = N;
         g.C = C; g.ldc = ldc; g.c_bf16 = false; g.epi = EPI_STORE;
+        float* hl = nullptr;
+        if (f32 && use_tc) {
+            hl = (float*)ctx_alloc(c, sizeof(float) * 2 * N * ldb, s);
+            split_tf32_dev((const float*)B, hl, hl + N * ldb, (int64_t)N * ldb, s);
+            g.Bhi = hl; g.Blo = hl + N * ldb;
+        }
         gemm_row(c, g, s);
+        if (hl) ctx_free(c, hl, s);
     } else {                    // C[K x N] = A[M x K]^T . B[M x N]  (C zero-initialised by the caller: it ADDS)
         int64_t S = gemm_red_splits(M_cap, K, N);
         float* part = (float*)ctx_alloc(c, sizeof(float) * S * K * N, s);
         GemmRed r{};
-        r.A = A; r.lda = lda; r.a_bf16 = true;
-        r.B = B; r.ldb = ldb; r.b_bf16 = true;
+        r.A = A; r.lda = lda; r.a_bf16 = !f32;
+        r.B = B; r.ldb = ldb; r.b_bf16 = !f32;
         r.M_dev = Md; r.M_cap = std::max<int64_t>(M_cap, 1); r.K1 = K; r.N = N;
         r.partials = part; r.S = (int)S; r.grad = C;
         r.map = GradMap{MAP_AGG, K, N, K, N, 0, 0, 0, 0, 0};   // identity: rows < K -> off_ws + i*N + j
@@ -933,6 +945,7 @@ extern "C" betty_status betty_test_gemm(betty_ctx* c, int32_t kind, const void* 
         (void)ldc;
     }
     c->use_tc = saved;
+    c->fp32_tc = saved_f;
     ctx_free(c, Md, s);
     st = sync_check(c, s);
     return st;

@@ -124,10 +124,14 @@ static void launch_row(betty_ctx* c, const GemmRow& g, cudaStream_t s) {
 }
 
 bool gemm_row(betty_ctx* c, const GemmRow& g, cudaStream_t s) {
-    if (c->use_tc && g.a_bf16 && g.b_bf16) {
-        const void* Bk = g.transB ? g.B : g.Bt;
+    // tensor cores: bf16 operands, or FP32 mode as 3xTF32 when the weights come split (hi / lo)
+    const bool tf = !g.a_bf16 && !g.b_bf16 && !g.c_bf16 && (g.transB ? (g.Bhi && g.Blo) : (g.Bt && g.Btlo));
+    if (c->use_tc && ((g.a_bf16 && g.b_bf16) || tf)) {
+        const void* Bk = tf ? (g.transB ? g.Bhi : g.Bt) : (g.transB ? g.B : g.Bt);
+        const void* Bl = tf ? (g.transB ? g.Blo : g.Btlo) : nullptr;
         const int64_t ldbk = g.transB ? g.ldb : g.ldbt;
-        if (Bk && g.N <= 256 && gemm_row_tc(c, g, Bk, ldbk, s)) return g.epi == EPI_RELU_ONES && g.obits;
+        const size_t bs = tf ? 4 : 2;
+        if (Bk && g.N <= 256 && gemm_row_tc(c, g, Bk, Bl, ldbk, s)) return g.epi == EPI_RELU_ONES && g.obits;
         // wider plain products (the pool layers' dXA, N = 2 Fp): 256-column blocks, left to right (each
         // block writes only its own columns; the last one the trailing columns)
         if (Bk && g.N > 256 && g.epi == EPI_STORE && (ldbk & 7) == 0) {
@@ -138,7 +142,8 @@ bool gemm_row(betty_ctx* c, const GemmRow& g, cudaStream_t s) {
                 h.N = std::min(256, g.N - n0);
                 h.C = (char*)g.C + (size_t)n0 * cs;
                 h.cend = n0 + 256 >= g.N ? g.ldc - n0 : h.N;
-                ok = gemm_row_tc(c, h, (const char*)Bk + (size_t)n0 * ldbk * 2, ldbk, s);
+                ok = gemm_row_tc(c, h, (const char*)Bk + (size_t)n0 * ldbk * bs,
+                                 Bl ? (const char*)Bl + (size_t)n0 * ldbk * bs : nullptr, ldbk, s);
             }
             if (ok) return false;
         }
@@ -296,10 +301,13 @@ int gemm_red_splits(int64_t M_cap, int K1, int N) {
 }
 
 void gemm_red(betty_ctx* c, const GemmRed& g, cudaStream_t s) {
-    if (c->use_tc && g.a_bf16 && g.b_bf16 && gemm_red_tc(c, g, s)) {
+    // tensor cores: bf16 operands, or fp32 operands as 3xTF32 (FP32 mode, unless BETTY_FP32_SIMT=1)
+    const bool tf = !g.a_bf16 && !g.b_bf16 && c->fp32_tc;
+    int S_used = g.S;
+    if (c->use_tc && ((g.a_bf16 && g.b_bf16) || tf) && gemm_red_tc(c, g, &S_used, s)) {
         const int64_t n = (int64_t)g.K1 * g.N;
         const int gf = (int)std::max<int64_t>(1, std::min<int64_t>((n + 31) / 32, (int64_t)c->num_sms * 8));
-        k_red_final<<<gf, 256, 0, s>>>(g.partials, g.S, g.K1, g.N, g.grad, g.map);
+        k_red_final<<<gf, 256, 0, s>>>(g.partials, S_used, g.K1, g.N, g.grad, g.map);
         return;
     }
     const int tiles = ((g.K1 + XB - 1) / XB) * ((g.N + XB - 1) / XB);

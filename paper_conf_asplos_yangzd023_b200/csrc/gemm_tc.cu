@@ -63,19 +63,54 @@ __device__ __forceinline__ void umma_f16(uint32_t tmem_d, uint64_t ad, uint64_t 
                  "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}"
                  ::"r"(tmem_d), "l"(ad), "l"(bd), "r"(idesc), "r"(acc));
 }
-// shared-memory matrix descriptor, SWIZZLE_128B, sm_100 version 1
-__device__ __forceinline__ uint64_t sdesc(uint32_t saddr, uint32_t lbo, uint32_t sbo) {
+__device__ __forceinline__ void umma_tf32(uint32_t tmem_d, uint64_t ad, uint64_t bd, uint32_t idesc, uint32_t acc) {
+    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+                 "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n\t}"
+                 ::"r"(tmem_d), "l"(ad), "l"(bd), "r"(idesc), "r"(acc));
+}
+// shared-memory matrix descriptor, sm_100 version 1; layout type 2 = SWIZZLE_128B (16-byte swizzle
+// base, 8-row atoms), 1 = SWIZZLE_128B_BASE32B (32-byte base, 4-row atoms: the only layout an MN-major
+// tf32 operand may use; TMA's CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B writes it)
+__device__ __forceinline__ uint64_t sdesc(uint32_t saddr, uint32_t lbo, uint32_t sbo, uint32_t layout = 2) {
     uint64_t d = (uint64_t)((saddr >> 4) & 0x3FFF);
     d |= (uint64_t)((lbo >> 4) & 0x3FFF) << 16;
     d |= (uint64_t)((sbo >> 4) & 0x3FFF) << 32;
     d |= (uint64_t)1 << 46;
-    d |= (uint64_t)2 << 61;
+    d |= (uint64_t)layout << 61;
     return d;
 }
 // instruction descriptor: bf16 x bf16 -> f32, M x N, operand majors (0 = K, 1 = MN)
 __host__ __device__ constexpr uint32_t idesc_bf16(int M, int N, int a_mn, int b_mn) {
     return (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)a_mn << 15) | ((uint32_t)b_mn << 16) |
            ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
+}
+// tf32 x tf32 -> f32 (operands are fp32 words in shared memory; FP32 mode's 3xTF32 split)
+__host__ __device__ constexpr uint32_t idesc_tf32(int M, int N, int a_mn, int b_mn) {
+    return (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)a_mn << 15) | ((uint32_t)b_mn << 16) |
+           ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
+}
+// 3xTF32 split of a float4 in shared memory: hi = x rounded to the nearest tf32 (10 mantissa bits,
+// so the tensor core's own fp32 -> tf32 conversion is the identity on it), lo = x - hi (exact in fp32,
+// |lo| <= 2^-11 |x|) also rounded to the nearest tf32 (the dropped remainder is <= 2^-23 |x|).  With
+// the lo*lo term dropped (<= 2^-22 of the product), each product is exact to ~2^-22.  hi overwrites x.
+__device__ __forceinline__ float tf32_rn(float x) {
+    return __uint_as_float((__float_as_uint(x) + 0x1000u) & 0xFFFFE000u);
+}
+// x, lo: shared-memory addresses (explicit ld/st.shared: generic accesses were the converter's cost)
+__device__ __forceinline__ void split_tf32(uint32_t x, uint32_t lo) {
+    float4 v;
+    asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "r"(x));
+    float4 h, l;
+    h.x = tf32_rn(v.x); l.x = tf32_rn(v.x - h.x);
+    h.y = tf32_rn(v.y); l.y = tf32_rn(v.y - h.y);
+    h.z = tf32_rn(v.z); l.z = tf32_rn(v.z - h.z);
+    h.w = tf32_rn(v.w); l.w = tf32_rn(v.w - h.w);
+    asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};" ::"r"(x), "f"(h.x), "f"(h.y), "f"(h.z), "f"(h.w) : "memory");
+    asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};" ::"r"(lo), "f"(l.x), "f"(l.y), "f"(l.z), "f"(l.w) : "memory");
+}
+__device__ __forceinline__ void zero2_shared(uint32_t x, uint32_t lo) {
+    asm volatile("st.shared.v4.u32 [%0], {%1, %1, %1, %1};" ::"r"(x), "r"(0u) : "memory");
+    asm volatile("st.shared.v4.u32 [%0], {%1, %1, %1, %1};" ::"r"(lo), "r"(0u) : "memory");
 }
 __device__ __forceinline__ void tmem_ld32(uint32_t taddr, float* v) {
     uint32_t r[32];
@@ -114,8 +149,12 @@ __device__ __forceinline__ bool elect_lane0() { return (threadIdx.x & 31) == 0; 
 // instead of re-reading the bf16 activations.  The kernel is templated on the
 // epilogue so each 32-column chunk is straight-line code (~150 instructions).
 constexpr int EPI_WARPS = 8;
-constexpr int ESLOTS = 2;                       // staging slots per epilogue warp
+constexpr int ESLOTS = 2;                       // staging slots per epilogue warp (bf16 operands)
+constexpr int ESLOTS_TF = 1;                    // ... FP32 mode (the 3xTF32 ring needs the room)
 constexpr int ROW_THREADS = 64 + 32 * EPI_WARPS;
+constexpr int CONV_WARPS = 4;                   // FP32 mode: hi/lo split of each stage (k_tc_red)
+constexpr int ROW_CONV_WARPS = 2;               // ... of each A stage (k_tc_row; keeps the epilogue unspilled)
+constexpr int ROW_THREADS_TF = ROW_THREADS + 32 * ROW_CONV_WARPS;
 constexpr int MAXCH = 4;                        // 32-column chunks per epilogue half (N <= 256)
 struct RowArgs {
     const int64_t* M_dev;
@@ -126,7 +165,9 @@ struct RowArgs {
     uint32_t* obits; int64_t ldob;              // EPI_RELU_ONES: ReLU bits out (words per row), or null
     const float* res; int64_t ldr; const int64_t* nres_dev;
     uint32_t tmem_cols;
-    int acc_stride;          // TMEM columns between the two accumulators (>= BN, multiple of 32)
+    int acc_stride;          // TMEM columns of one accumulator (>= BN, multiple of 32)
+    int nbuf;                // accumulator buffers (2: the epilogue of tile i overlaps the MMAs of tile i+1)
+    int buf_stride;          // TMEM columns between buffers (TF: main + lo-term accumulators)
     int half_cols;           // columns per epilogue half (multiple of 32, <= 32 * MAXCH)
     uint32_t slot_bytes;     // one staging slot: 32 rows x 32 columns
     int bstream;             // 1: B is streamed with A through the ring (B too large to stay resident)
@@ -169,6 +210,17 @@ __device__ __forceinline__ void tmem_wait_regs(uint32_t* r) {
                  :
                  : "memory");
 }
+
+__device__ __forceinline__ void tmem_st32(uint32_t taddr, const uint32_t* r) {
+    asm volatile("tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,"
+                 "%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32};"
+                 ::"r"(taddr), "r"(r[0]), "r"(r[1]), "r"(r[2]), "r"(r[3]), "r"(r[4]), "r"(r[5]), "r"(r[6]), "r"(r[7]),
+                   "r"(r[8]), "r"(r[9]), "r"(r[10]), "r"(r[11]), "r"(r[12]), "r"(r[13]), "r"(r[14]), "r"(r[15]),
+                   "r"(r[16]), "r"(r[17]), "r"(r[18]), "r"(r[19]), "r"(r[20]), "r"(r[21]), "r"(r[22]), "r"(r[23]),
+                   "r"(r[24]), "r"(r[25]), "r"(r[26]), "r"(r[27]), "r"(r[28]), "r"(r[29]), "r"(r[30]), "r"(r[31])
+                 : "memory");
+}
+__device__ __forceinline__ void tmem_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
 
 // [activation > 0] of a stored 32-column chunk (mask from activations, MBITS = false)
 __device__ __forceinline__ uint32_t mask_word_from_act(const RowArgs& p, int64_t m, int c0, bool ok) {
@@ -263,25 +315,33 @@ __device__ __forceinline__ uint32_t chunk_epilogue(const RowArgs& p, const uint3
     return bits;
 }
 
-template <int EPI, bool CBF, bool MBITS>
-__global__ void __launch_bounds__(ROW_THREADS, 1) k_tc_row(const __grid_constant__ CUtensorMap tmA,
-                                                           const __grid_constant__ CUtensorMap tmB,
-                                                           const __grid_constant__ CUtensorMap tmC, RowArgs p) {
+// TF (FP32 mode, 3xTF32): A, B are fp32 words; one k-block is 32 of them (the same 128-byte swizzle
+// rows as 64 bf16).  Four converter warps split each landed A stage into hi (in place) and lo, B comes
+// pre-split (hi, lo) from the weight prep; per k-block the MMA warp issues lo*hi, hi*lo, hi*hi into
+// the same fp32 accumulator (the lo*lo term, ~2^-22 relative, is dropped).
+template <int EPI, bool CBF, bool MBITS, bool TF>
+__global__ void __launch_bounds__(TF ? ROW_THREADS_TF : ROW_THREADS, 1)
+k_tc_row(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+         const __grid_constant__ CUtensorMap tmC, const __grid_constant__ CUtensorMap tmBlo, RowArgs p) {
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+    constexpr int ES = TF ? ESLOTS_TF : ESLOTS;
+    constexpr int NSPLIT = TF ? 2 : 1;                       // hi (+ lo) copies of each operand block
     const int S = p.stages;
-    const uint32_t a_bytes = BM * BK * 2;
-    const uint32_t bblk = (uint32_t)p.BN * BK * 2;          // one K-block of B
-    const uint32_t ring_bytes = a_bytes + (p.bstream ? bblk : 0u);   // one ring stage: A (+ B when streamed)
-    uint8_t* bres = smem;                                    // nk * bblk (resident B) or nothing
-    uint8_t* aring = smem + (p.bstream ? 0 : p.nk * bblk);   // S * ring_bytes
-    uint8_t* stage = aring + S * ring_bytes;                 // EPI_WARPS * ESLOTS * slot_bytes
-    uint64_t* full = (uint64_t*)(stage + EPI_WARPS * ESLOTS * p.slot_bytes);
+    const uint32_t a_bytes = BM * 128;                       // one A k-block: 128 rows x 128 B
+    const uint32_t bblk = (uint32_t)p.BN * 128;              // one K-block of B
+    // one ring stage: A (+ A lo) (+ B (+ B lo) when streamed)
+    const uint32_t ring_bytes = NSPLIT * (a_bytes + (p.bstream ? bblk : 0u));
+    uint8_t* bres = smem;                                    // NSPLIT * nk * bblk (resident B) or nothing
+    uint8_t* aring = smem + (p.bstream ? 0 : NSPLIT * p.nk * bblk);   // S * ring_bytes
+    uint8_t* stage = aring + S * ring_bytes;                 // EPI_WARPS * ES * slot_bytes
+    uint64_t* full = (uint64_t*)(stage + EPI_WARPS * ES * p.slot_bytes);
     uint64_t* empty = full + S;
     uint64_t* tfull = empty + S;      // [2]
     uint64_t* tempty = tfull + 2;     // [2]
     uint64_t* bfull = tempty + 2;     // [1]
-    uint32_t* tslot = (uint32_t*)(bfull + 1);
+    uint64_t* conv = bfull + 1;       // [S] (TF) A stage split into hi / lo
+    uint32_t* tslot = (uint32_t*)(conv + (TF ? S : 0));
 
     const int warp = threadIdx.x >> 5;
     const int64_t M = *p.M_dev;
@@ -291,10 +351,12 @@ __global__ void __launch_bounds__(ROW_THREADS, 1) k_tc_row(const __grid_constant
         for (int s = 0; s < S; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
         for (int a = 0; a < 2; ++a) { mbar_init(&tfull[a], 1); mbar_init(&tempty[a], 32 * EPI_WARPS); }
         mbar_init(bfull, 1);
+        if (TF) for (int s = 0; s < S; ++s) mbar_init(&conv[s], ROW_CONV_WARPS);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
         asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmA) : "memory");
         asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmB) : "memory");
         asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmC) : "memory");
+        if (TF) asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmBlo) : "memory");
     }
     if (warp == 1) tmem_alloc_warp(tslot, p.tmem_cols);
     fence_before();
@@ -304,50 +366,97 @@ __global__ void __launch_bounds__(ROW_THREADS, 1) k_tc_row(const __grid_constant
 
     if (warp == 0) {
         if (elect_lane0() && blockIdx.x < tiles) {
+            constexpr int KE = TF ? 32 : BK;                 // elements per k-block
             if (!p.bstream) {
-                mbar_expect_tx(bfull, p.nk * bblk);
-                for (int kb = 0; kb < p.nk; ++kb) tma_2d(bres + kb * bblk, &tmB, kb * BK, 0, bfull);
+                mbar_expect_tx(bfull, NSPLIT * p.nk * bblk);
+                for (int kb = 0; kb < p.nk; ++kb) {
+                    tma_2d(bres + kb * bblk, &tmB, kb * KE, 0, bfull);
+                    if (TF) tma_2d(bres + (p.nk + kb) * bblk, &tmBlo, kb * KE, 0, bfull);
+                }
             }
+            // TF stage: [A | A lo | B | B lo]; TMA fills A, B, B lo (the converter writes A lo)
+            const uint32_t land = ring_bytes - (TF ? a_bytes : 0u);
             int s = 0;
             uint32_t ph = 0;
             for (int64_t t = blockIdx.x; t < tiles; t += gridDim.x) {
                 for (int kb = 0; kb < p.nk; ++kb) {
                     mbar_wait(&empty[s], ph ^ 1);
-                    mbar_expect_tx(&full[s], ring_bytes);
-                    tma_2d(aring + s * ring_bytes, &tmA, kb * BK, (int)(t * BM), &full[s]);
-                    if (p.bstream) tma_2d(aring + s * ring_bytes + a_bytes, &tmB, kb * BK, 0, &full[s]);
+                    mbar_expect_tx(&full[s], land);
+                    uint8_t* st = aring + s * ring_bytes;
+                    tma_2d(st, &tmA, kb * KE, (int)(t * BM), &full[s]);
+                    if (p.bstream) {
+                        tma_2d(st + NSPLIT * a_bytes, &tmB, kb * KE, 0, &full[s]);
+                        if (TF) tma_2d(st + NSPLIT * a_bytes + bblk, &tmBlo, kb * KE, 0, &full[s]);
+                    }
                     if (++s == S) { s = 0; ph ^= 1; }
                 }
             }
         }
     } else if (warp == 1) {
-        const uint32_t idesc = idesc_bf16(BM, p.BN, 0, 0);
+        const uint32_t idesc = TF ? idesc_tf32(BM, p.BN, 0, 0) : idesc_bf16(BM, p.BN, 0, 0);
         int s = 0;
         uint32_t ph = 0;
         int it = 0;
         if (blockIdx.x < tiles && !p.bstream) mbar_wait(bfull, 0);
         for (int64_t t = blockIdx.x; t < tiles; t += gridDim.x, ++it) {
-            const int acc = it & 1;
-            const uint32_t aph = (it >> 1) & 1;
+            const int acc = it % p.nbuf;
+            const uint32_t aph = (it / p.nbuf) & 1;
             mbar_wait(&tempty[acc], aph ^ 1);
             fence_after();
-            const uint32_t d = tmem + acc * p.acc_stride;
+            const uint32_t d = tmem + acc * p.buf_stride;
             for (int kb = 0; kb < p.nk; ++kb) {
-                mbar_wait(&full[s], ph);
+                mbar_wait(TF ? &conv[s] : &full[s], ph);
                 fence_after();
                 if (elect_lane0()) {
                     const uint32_t a0 = su32(aring + s * ring_bytes);
-                    const uint32_t b0 = p.bstream ? a0 + a_bytes : su32(bres + kb * bblk);
+                    const uint32_t b0 = p.bstream ? a0 + NSPLIT * a_bytes : su32(bres + kb * bblk);
+                    if (TF) {
+                        // 4 MMAs of K = 8 fp32 words (32 B) per 128-byte k-block, per product term.  The
+                        // small terms go to their own accumulator (d + acc_stride): the tensor core's
+                        // fp32 accumulation rounds toward zero (~2e-8 relative per accumulation into a
+                        // growing sum), so the main sum gets only the K/8 hi*hi accumulations
+                        const uint32_t alo = a0 + a_bytes;
+                        const uint32_t blo = p.bstream ? b0 + bblk : su32(bres + (p.nk + kb) * bblk);
+                        const uint32_t dl = d + p.acc_stride;
 #pragma unroll
-                    for (int k = 0; k < BK / UK; ++k) {
-                        const uint64_t ad = sdesc(a0 + k * UK * 2, 0, 1024);
-                        const uint64_t bd = sdesc(b0 + k * UK * 2, 0, 1024);
-                        umma_f16(d, ad, bd, idesc, (kb | k) != 0);
+                        for (int k = 0; k < 4; ++k)
+                            umma_tf32(dl, sdesc(alo + k * 32, 0, 1024), sdesc(b0 + k * 32, 0, 1024), idesc, (kb | k) != 0);
+#pragma unroll
+                        for (int k = 0; k < 4; ++k)
+                            umma_tf32(dl, sdesc(a0 + k * 32, 0, 1024), sdesc(blo + k * 32, 0, 1024), idesc, 1);
+#pragma unroll
+                        for (int k = 0; k < 4; ++k)
+                            umma_tf32(d, sdesc(a0 + k * 32, 0, 1024), sdesc(b0 + k * 32, 0, 1024), idesc, (kb | k) != 0);
+                    } else {
+#pragma unroll
+                        for (int k = 0; k < BK / UK; ++k) {
+                            const uint64_t ad = sdesc(a0 + k * UK * 2, 0, 1024);
+                            const uint64_t bd = sdesc(b0 + k * UK * 2, 0, 1024);
+                            umma_f16(d, ad, bd, idesc, (kb | k) != 0);
+                        }
                     }
                     umma_commit(&empty[s]);
                     if (kb == p.nk - 1) umma_commit(&tfull[acc]);
                 }
                 __syncwarp();
+                if (++s == S) { s = 0; ph ^= 1; }
+            }
+        }
+    } else if (TF && warp >= 2 + EPI_WARPS) {
+        // converter warps: split each landed A k-block (128 rows x 32 fp32) into hi (in place) and lo
+        const int tid = (warp - 2 - EPI_WARPS) * 32 + (threadIdx.x & 31);
+        int s = 0;
+        uint32_t ph = 0;
+        for (int64_t t = blockIdx.x; t < tiles; t += gridDim.x) {
+            for (int kb = 0; kb < p.nk; ++kb) {
+                mbar_wait(&full[s], ph);
+                const uint32_t a = su32(aring + s * ring_bytes);
+#pragma unroll 4
+                for (int i = tid; i < (int)(a_bytes / 16); i += 32 * ROW_CONV_WARPS)
+                    split_tf32(a + 16 * i, a + a_bytes + 16 * i);
+                fence_proxy_async();             // generic-proxy writes -> visible to the tensor core
+                __syncwarp();
+                if ((threadIdx.x & 31) == 0) mbar_arrive(&conv[s]);
                 if (++s == S) { s = 0; ph ^= 1; }
             }
         }
@@ -361,7 +470,7 @@ __global__ void __launch_bounds__(ROW_THREADS, 1) k_tc_row(const __grid_constant
         const int cstore = min(min(p.BN, cbeg + p.half_cols), p.N);   // chunks at or past N are not stored
         const int nch = cstore > cbeg ? (cstore - cbeg + 31) / 32 : 0;
         const int64_t nres = EPI == EPI_RES_MASK ? *p.nres_dev : 0;
-        uint8_t* my_stage = stage + ew * ESLOTS * p.slot_bytes;
+        uint8_t* my_stage = stage + ew * ES * p.slot_bytes;
         int slot = 0;
         int it = 0;
         // ReLU' bit words of this thread's row, one tile ahead (short-K layers finish the MMA long
@@ -379,8 +488,8 @@ __global__ void __launch_bounds__(ROW_THREADS, 1) k_tc_row(const __grid_constant
         };
         if (HAS_MASK && MBITS) load_bits(blockIdx.x, mw_next);
         for (int64_t t = blockIdx.x; t < tiles; t += gridDim.x, ++it) {
-            const int acc = it & 1;
-            const uint32_t aph = (it >> 1) & 1;
+            const int acc = it % p.nbuf;
+            const uint32_t aph = (it / p.nbuf) & 1;
             const int64_t row0 = t * BM + q * 32;
             const int64_t m = row0 + lane;
             const bool ok = m < M;
@@ -400,9 +509,36 @@ __global__ void __launch_bounds__(ROW_THREADS, 1) k_tc_row(const __grid_constant
             }
             mbar_wait(&tfull[acc], aph);
             fence_after();
-            const uint32_t tbase = tmem + ((uint32_t)(q * 32) << 16) + acc * p.acc_stride;
+            const uint32_t tbase = tmem + ((uint32_t)(q * 32) << 16) + acc * p.buf_stride;
             uint32_t ra[32], rb[32];
             uint32_t obits[MAXCH];
+            if constexpr (TF) {
+                // main + lo-term accumulators, summed with round-to-nearest fp32 adds
+#pragma unroll
+                for (int ci = 0; ci < MAXCH; ++ci) {
+                    obits[ci] = 0u;
+                    if (ci < nch) {
+                        const int c0 = cbeg + 32 * ci;
+                        tmem_ld32_nowait(tbase + c0, ra);
+                        tmem_ld32_nowait(tbase + p.acc_stride + c0, rb);
+                        tmem_wait_regs(ra);
+                        tmem_wait_regs(rb);
+#pragma unroll
+                        for (int j = 0; j < 32; ++j) ra[j] = __float_as_uint(__uint_as_float(ra[j]) + __uint_as_float(rb[j]));
+                        uint8_t* sl = my_stage + slot * p.slot_bytes;
+                        if (lane == 0) bulk_wait_read<ES - 1>();
+                        __syncwarp();
+                        obits[ci] = chunk_epilogue<EPI, CBF>(p, ra, m, c0, ok, mw[ci], nres, sl, lane);
+                        fence_proxy_async();
+                        __syncwarp();
+                        if (lane == 0) {
+                            tma_store_2d(&tmC, sl, c0, (int)row0);
+                            bulk_commit();
+                        }
+                        if (++slot == ES) slot = 0;
+                    }
+                }
+            } else {
             if (nch > 0) { tmem_ld32_nowait(tbase + cbeg, ra); tmem_wait_regs(ra); }
 #pragma unroll
             for (int ci = 0; ci < MAXCH; ++ci) {
@@ -413,7 +549,7 @@ __global__ void __launch_bounds__(ROW_THREADS, 1) k_tc_row(const __grid_constant
                     const int c0 = cbeg + 32 * ci;
                     if (ci + 1 < nch) tmem_ld32_nowait(tbase + c0 + 32, nxt);   // next chunk in flight
                     uint8_t* sl = my_stage + slot * p.slot_bytes;
-                    if (lane == 0) bulk_wait_read<ESLOTS - 1>();    // the store that used this slot has read it
+                    if (lane == 0) bulk_wait_read<ES - 1>();        // the store that used this slot has read it
                     __syncwarp();
                     obits[ci] = chunk_epilogue<EPI, CBF>(p, cur, m, c0, ok, mw[ci], nres, sl, lane);
                     fence_proxy_async();
@@ -422,9 +558,10 @@ __global__ void __launch_bounds__(ROW_THREADS, 1) k_tc_row(const __grid_constant
                         tma_store_2d(&tmC, sl, c0, (int)row0);
                         bulk_commit();
                     }
-                    if (++slot == ESLOTS) slot = 0;
+                    if (++slot == ES) slot = 0;
                     if (ci + 1 < nch) tmem_wait_regs(nxt);
                 }
+            }
             }
             fence_before();
             mbar_arrive(&tempty[acc]);
@@ -468,33 +605,52 @@ struct RedArgs {
     int acc_stride;            // TMEM columns per feature tile accumulator
     float* partials;           // [S][K1][N]
     uint32_t tmem_cols;
+    uint32_t sbo;              // TF: byte stride between 4-row K atoms (512)
 };
 
-__global__ void __launch_bounds__(THREADS, 1) k_tc_red(const __grid_constant__ CUtensorMap tmA,
-                                                       const __grid_constant__ CUtensorMap tmB, RedArgs p) {
+// TF (FP32 mode, 3xTF32): fp32 operands, k-blocks of 16 nodes (boxes of 32 features x 16 nodes, the
+// same 128-byte swizzle rows), four converter warps split both operands of each landed stage into hi
+// (in place) and lo (a second copy of the stage) and zero the rows past M; three MMA terms per step.
+// The tensor core's fp32 accumulation rounds toward zero (measured: ~2e-8 relative shrink per MMA
+// accumulation into a growing sum), so a CTA's long reduction over nodes is NOT left in one
+// accumulator: every RED_SB k-blocks (64 nodes, 24 accumulations) the epilogue warps add the TMEM
+// accumulator into a TMEM running total with round-to-nearest fp32 adds (one feature tile per CTA,
+// TMEM = accumulator + total).
+constexpr int RED_THREADS_TF = THREADS + 32 * CONV_WARPS;
+constexpr int RED_SB = 4;
+template <bool TF>
+__global__ void __launch_bounds__(TF ? RED_THREADS_TF : THREADS, 1)
+k_tc_red(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB, RedArgs p) {
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+    constexpr int KN = TF ? 16 : BK;                  // nodes (reduction rows) per k-block
     const int S = p.stages;
-    const uint32_t box = BK * 128;                    // 64 rows x 128 B
-    const int nbA_cta = p.nbA * p.mt_cta;             // A boxes per stage (64 features each)
+    const uint32_t box = KN * 128;                    // KN rows x 128 B (64 bf16 / 32 fp32 features)
+    const int nbA_cta = p.nbA * p.mt_cta;             // A boxes per stage
     const uint32_t a_bytes = nbA_cta * box, b_bytes = p.nbB * box;
-    const uint32_t stage_bytes = a_bytes + b_bytes;
+    const uint32_t raw_bytes = a_bytes + b_bytes;
+    const uint32_t stage_bytes = raw_bytes * (TF ? 2 : 1);   // TF: + the lo copy
     uint64_t* full = (uint64_t*)(smem + S * stage_bytes);
     uint64_t* empty = full + S;
     uint64_t* tfull = empty + S;
-    uint32_t* tslot = (uint32_t*)(tfull + 1);
+    uint64_t* tempty_r = tfull + 1;                   // [1] (TF) accumulator drained into the total
+    uint64_t* conv = tempty_r + 1;                    // [S] (TF)
+    uint32_t* tslot = (uint32_t*)(conv + (TF ? S : 0));
 
     const int warp = threadIdx.x >> 5;
     const int nsplit = p.mt_cta == 1 ? p.mtiles : 1;
     const int mt0 = p.mt_cta == 1 ? blockIdx.x % p.mtiles : 0;
     const int split = blockIdx.x / nsplit;
     const int64_t M = *p.M_dev;
-    const int64_t nkb = (M + BK - 1) / BK;
+    const int64_t nkb = (M + KN - 1) / KN;
     const int64_t kb0 = nkb * split / p.S, kb1 = nkb * (split + 1) / p.S;
+    const int fbox = TF ? 32 : 64;                    // features per box
 
     if (threadIdx.x == 0) {
         for (int s = 0; s < S; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
         mbar_init(&tfull[0], 1);
+        mbar_init(&tempty_r[0], 128);
+        if (TF) for (int s = 0; s < S; ++s) mbar_init(&conv[s], CONV_WARPS);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     if (warp == 1) tmem_alloc_warp(tslot, p.tmem_cols);
@@ -510,54 +666,135 @@ __global__ void __launch_bounds__(THREADS, 1) k_tc_red(const __grid_constant__ C
             for (int64_t kb = kb0; kb < kb1; ++kb) {
                 mbar_wait(&empty[s], ph ^ 1);
                 uint8_t* sa = smem + s * stage_bytes;
-                mbar_expect_tx(&full[s], stage_bytes);
-                for (int i = 0; i < nbA_cta; ++i) tma_2d(sa + i * box, &tmA, mt0 * BM + i * 64, (int)(kb * BK), &full[s]);
-                for (int i = 0; i < p.nbB; ++i) tma_2d(sa + a_bytes + i * box, &tmB, i * 64, (int)(kb * BK), &full[s]);
+                mbar_expect_tx(&full[s], raw_bytes);
+                for (int i = 0; i < nbA_cta; ++i) tma_2d(sa + i * box, &tmA, mt0 * BM + i * fbox, (int)(kb * KN), &full[s]);
+                for (int i = 0; i < p.nbB; ++i) tma_2d(sa + a_bytes + i * box, &tmB, i * fbox, (int)(kb * KN), &full[s]);
                 if (++s == S) { s = 0; ph ^= 1; }
             }
         }
     } else if (warp == 1) {
-        const uint32_t idesc = idesc_bf16(BM, p.BN, 1, 1);
+        const uint32_t idesc = TF ? idesc_tf32(BM, p.BN, 1, 1) : idesc_bf16(BM, p.BN, 1, 1);
         int s = 0;
         uint32_t ph = 0;
         for (int64_t kb = kb0; kb < kb1; ++kb) {
-            mbar_wait(&full[s], ph);
             uint8_t* sa = smem + s * stage_bytes;
-            const int64_t valid = M - kb * BK;       // rows of this k-block inside [0, M)
-            if (valid < BK) {                        // zero the tail rows of every box (generic proxy)
-                const int nboxes = nbA_cta + p.nbB;
-                for (int idx = threadIdx.x & 31; idx < nboxes * (BK - (int)valid) * 8; idx += 32) {
-                    const int b = idx / ((BK - (int)valid) * 8);
-                    const int rr = (idx / 8) % (BK - (int)valid) + (int)valid;
-                    const int ch = idx & 7;
-                    *(uint4*)(sa + b * box + rr * 128 + ch * 16) = make_uint4(0, 0, 0, 0);
+            const int64_t sb = (kb - kb0) / RED_SB;          // TF: super-block index
+            const bool sb_first = TF && (kb - kb0) % RED_SB == 0;
+            const bool sb_last = TF && ((kb - kb0) % RED_SB == RED_SB - 1 || kb == kb1 - 1);
+            if (sb_first && sb > 0) {                        // the epilogue has drained the accumulator
+                mbar_wait(&tempty_r[0], (uint32_t)((sb - 1) & 1));
+                fence_after();
+            }
+            if (TF) {
+                mbar_wait(&conv[s], ph);
+            } else {
+                mbar_wait(&full[s], ph);
+                const int64_t valid = M - kb * BK;       // rows of this k-block inside [0, M)
+                if (valid < BK) {                        // zero the tail rows of every box (generic proxy)
+                    const int nboxes = nbA_cta + p.nbB;
+                    for (int idx = threadIdx.x & 31; idx < nboxes * (BK - (int)valid) * 8; idx += 32) {
+                        const int b = idx / ((BK - (int)valid) * 8);
+                        const int rr = (idx / 8) % (BK - (int)valid) + (int)valid;
+                        const int ch = idx & 7;
+                        *(uint4*)(sa + b * box + rr * 128 + ch * 16) = make_uint4(0, 0, 0, 0);
+                    }
+                    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                    __syncwarp();
                 }
-                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-                __syncwarp();
             }
             fence_after();
             if (elect_lane0()) {
                 const uint32_t b0 = su32(sa) + a_bytes;
-                for (int mt = 0; mt < p.mt_cta; ++mt) {
-                    const uint32_t a0 = su32(sa) + mt * p.nbA * box;
+                if (TF) {
+                    // MN-major tf32, SWIZZLE_128B_BASE32B: atoms of 32 (MN) x 4 (K) rows of 128 B (SBO = 512
+                    // between the two atoms one K = 8 MMA spans), LBO = box between 32-feature columns
+                    for (int mt = 0; mt < p.mt_cta; ++mt) {
+                        const uint32_t a0 = su32(sa) + mt * p.nbA * box;
 #pragma unroll
-                    for (int k = 0; k < BK / UK; ++k) {
-                        // MN-major SW128: atoms of 64 (MN) x 8 (K) at SBO = 1024 along K, LBO = box along MN
-                        const uint64_t ad = sdesc(a0 + k * UK * 128, box, 1024);
-                        const uint64_t bd = sdesc(b0 + k * UK * 128, box, 1024);
-                        umma_f16(tmem + mt * p.acc_stride, ad, bd, idesc, (kb != kb0 || k != 0));
+                        for (int k = 0; k < KN / 8; ++k) {
+                            const uint64_t ah = sdesc(a0 + k * 1024, box, p.sbo, 1), al = sdesc(a0 + raw_bytes + k * 1024, box, p.sbo, 1);
+                            const uint64_t bh = sdesc(b0 + k * 1024, box, p.sbo, 1), bl = sdesc(b0 + raw_bytes + k * 1024, box, p.sbo, 1);
+                            const uint32_t d = tmem + mt * p.acc_stride;
+                            umma_tf32(d, al, bh, idesc, (!sb_first || k != 0));
+                            umma_tf32(d, ah, bl, idesc, 1);
+                            umma_tf32(d, ah, bh, idesc, 1);
+                        }
+                    }
+                } else {
+                    for (int mt = 0; mt < p.mt_cta; ++mt) {
+                        const uint32_t a0 = su32(sa) + mt * p.nbA * box;
+#pragma unroll
+                        for (int k = 0; k < BK / UK; ++k) {
+                            // MN-major SW128: atoms of 64 (MN) x 8 (K) at SBO = 1024 along K, LBO = box along MN
+                            const uint64_t ad = sdesc(a0 + k * UK * 128, box, 1024);
+                            const uint64_t bd = sdesc(b0 + k * UK * 128, box, 1024);
+                            umma_f16(tmem + mt * p.acc_stride, ad, bd, idesc, (kb != kb0 || k != 0));
+                        }
                     }
                 }
                 umma_commit(&empty[s]);
-                if (kb == kb1 - 1) umma_commit(&tfull[0]);
+                if (TF ? sb_last : kb == kb1 - 1) umma_commit(&tfull[0]);
             }
             __syncwarp();
+            if (++s == S) { s = 0; ph ^= 1; }
+        }
+    } else if (TF && warp >= 2 + 4) {
+        // converter warps: hi in place, lo into the second half of the stage, rows >= M zeroed
+        const int tid = (warp - 6) * 32 + (threadIdx.x & 31);
+        int s = 0;
+        uint32_t ph = 0;
+        for (int64_t kb = kb0; kb < kb1; ++kb) {
+            mbar_wait(&full[s], ph);
+            const uint32_t sa = su32(smem + s * stage_bytes);
+            const int64_t valid = M - kb * KN;
+            const int n16 = (int)(raw_bytes / 16);
+            if (valid >= KN) {
+#pragma unroll 4
+                for (int i = tid; i < n16; i += 32 * CONV_WARPS) split_tf32(sa + 16 * i, sa + raw_bytes + 16 * i);
+            } else {                                     // the last k-block: rows >= M are zeroed
+                for (int i = tid; i < n16; i += 32 * CONV_WARPS) {
+                    const int row = (i >> 3) & (KN - 1); // 8 float4 per 128-byte row, KN rows per box
+                    if (row < (int)valid) split_tf32(sa + 16 * i, sa + raw_bytes + 16 * i);
+                    else zero2_shared(sa + 16 * i, sa + raw_bytes + 16 * i);
+                }
+            }
+            fence_proxy_async();
+            __syncwarp();
+            if ((threadIdx.x & 31) == 0) mbar_arrive(&conv[s]);
             if (++s == S) { s = 0; ph ^= 1; }
         }
     } else {
         const int q = warp & 3;
         const int r_in = q * 32 + (threadIdx.x & 31);
-        if (kb1 > kb0) {
+        if (TF) {
+            // drain each super-block's accumulator (columns [0, acc_stride)) into the running total
+            // (columns [acc_stride, 2 acc_stride)) with round-to-nearest fp32 adds; the total ends
+            // in the accumulator columns' place for the write-out below
+            const uint32_t lane_base = tmem + ((uint32_t)(q * 32) << 16);
+            const int64_t nsb = (kb1 - kb0 + RED_SB - 1) / RED_SB;
+            for (int64_t sb = 0; sb < nsb; ++sb) {
+                mbar_wait(&tfull[0], (uint32_t)(sb & 1));
+                fence_after();
+                for (int c0 = 0; c0 < p.BN; c0 += 32) {
+                    uint32_t a[32], t[32];
+                    tmem_ld32_nowait(lane_base + c0, a);
+                    if (sb > 0) tmem_ld32_nowait(lane_base + p.acc_stride + c0, t);
+                    tmem_wait_regs(a);
+                    if (sb > 0) {
+                        tmem_wait_regs(t);
+#pragma unroll
+                        for (int j = 0; j < 32; ++j) t[j] = __float_as_uint(__uint_as_float(t[j]) + __uint_as_float(a[j]));
+                    } else {
+#pragma unroll
+                        for (int j = 0; j < 32; ++j) t[j] = a[j];
+                    }
+                    tmem_st32(lane_base + p.acc_stride + c0, t);
+                }
+                tmem_wait_st();
+                fence_before();
+                mbar_arrive(&tempty_r[0]);
+            }
+        } else if (kb1 > kb0) {
             mbar_wait(&tfull[0], 0);
             fence_after();
         }
@@ -566,7 +803,7 @@ __global__ void __launch_bounds__(THREADS, 1) k_tc_red(const __grid_constant__ C
             float* out = p.partials + ((int64_t)split * p.K1 + feat) * p.N;
             for (int c0 = 0; c0 < p.BN; c0 += 32) {
                 float v[32];
-                if (kb1 > kb0) tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + mt * p.acc_stride + c0, v);
+                if (kb1 > kb0) tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + (TF ? p.acc_stride : mt * p.acc_stride) + c0, v);
                 else {
 #pragma unroll
                     for (int j = 0; j < 32; ++j) v[j] = 0.f;
@@ -648,25 +885,35 @@ bool make_gather_map(CUtensorMap* m, const void* base, bool f32, int64_t cols, i
 }
 
 // C = A B on the tensor cores; B given K-major as Bk[N x K] (ld ldbk).  Returns false if the shape is unsupported.
-bool gemm_row_tc(betty_ctx* c, const GemmRow& g, const void* Bk, int64_t ldbk, cudaStream_t s) {
+bool gemm_row_tc(betty_ctx* c, const GemmRow& g, const void* Bk, const void* Bk_lo, int64_t ldbk, cudaStream_t s) {
     using namespace tc;
-    if (!g.a_bf16 || !g.b_bf16 || g.N > 256 || g.N < 1 || (g.lda & 7) || (ldbk & 7)) return false;
-    if ((g.epi == EPI_MASK || g.epi == EPI_RES_MASK) && !g.mbits && (g.ldm & 7)) return false;
+    // TF: FP32 mode (fp32 A, B hi / lo, fp32 C) as 3xTF32; else bf16 operands
+    const bool TF = !g.a_bf16;
+    if (TF && (g.b_bf16 || g.c_bf16 || !Bk_lo || (g.lda & 3) || (ldbk & 3))) return false;
+    if (!TF && (!g.a_bf16 || !g.b_bf16 || (g.lda & 7) || (ldbk & 7))) return false;
+    if (g.N > 256 || g.N < 1) return false;
+    if ((g.epi == EPI_MASK || g.epi == EPI_RES_MASK) && !g.mbits && (g.ldm & (g.m_bf16 ? 7 : 3))) return false;
+    const int KE = TF ? 32 : BK;                // elements per 128-byte k-block
+    const int NS = TF ? 2 : 1;                  // hi (+ lo) copies
     const int BN = (g.N + 15) / 16 * 16;
-    const int nk = (g.K + BK - 1) / BK;
-    const size_t b_bytes = (size_t)nk * BN * BK * 2;
-    const size_t a_bytes = BM * BK * 2;
+    const int nk = (g.K + KE - 1) / KE;
+    const size_t bblk = (size_t)BN * 128;
+    const size_t b_bytes = (size_t)nk * bblk * NS;
+    const size_t a_bytes = (size_t)BM * 128 * NS;
     const uint32_t slot_bytes = 32 * 32 * (g.c_bf16 ? 2 : 4);
-    const size_t stage_bytes = (size_t)EPI_WARPS * ESLOTS * slot_bytes;
+    const size_t stage_bytes = (size_t)EPI_WARPS * (TF ? ESLOTS_TF : ESLOTS) * slot_bytes;
     const size_t budget = 227 * 1024;           // the sm_100 opt-in maximum of dynamic shared memory per CTA
-    const size_t bblk = (size_t)BN * BK * 2;
     // B resident when it fits next to a 2-stage A ring, else streamed with A
     const bool bstream = b_bytes + stage_bytes + 2 * a_bytes + 1024 + 256 > budget;
-    const size_t ring = a_bytes + (bstream ? bblk : 0);
+    const size_t ring = a_bytes + (bstream ? bblk * NS : 0);
     const size_t fixed = (bstream ? 0 : b_bytes) + stage_bytes + 1024 + 256;
     if (fixed + 2 * ring > budget) return false;
-    CUtensorMap ma, mb, mc;
-    if (!make_map(&ma, g.A, g.K, g.M_cap, g.lda, BM) || !make_map(&mb, Bk, g.K, g.N, ldbk, BN)) return false;
+    CUtensorMap ma, mb, mc, mbl;
+    if (!make_map_t(&ma, g.A, TF, g.K, g.M_cap, g.lda, KE, BM, CU_TENSOR_MAP_SWIZZLE_128B) ||
+        !make_map_t(&mb, Bk, TF, g.K, g.N, ldbk, KE, BN, CU_TENSOR_MAP_SWIZZLE_128B))
+        return false;
+    if (TF && !make_map_t(&mbl, Bk_lo, true, g.K, g.N, ldbk, KE, BN, CU_TENSOR_MAP_SWIZZLE_128B)) return false;
+    if (!TF) mbl = mb;
     if (!make_map_t(&mc, g.C, !g.c_bf16, g.N, g.M_cap, g.ldc, 32, 32,
                     g.c_bf16 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_128B))
         return false;
@@ -679,7 +926,9 @@ bool gemm_row_tc(betty_ctx* c, const GemmRow& g, const void* Bk, int64_t ldbk, c
     p.mbits = g.mbits; p.ldmb = g.ldmb;
     p.obits = g.epi == EPI_RELU_ONES ? g.obits : nullptr; p.ldob = g.ldob;
     p.acc_stride = (BN + 31) / 32 * 32;
-    p.tmem_cols = tmem_cols_for(2 * p.acc_stride);
+    p.buf_stride = (TF ? 2 : 1) * p.acc_stride;
+    p.nbuf = 2 * p.buf_stride <= 512 ? 2 : 1;
+    p.tmem_cols = tmem_cols_for(p.nbuf * p.buf_stride);
     p.half_cols = ((BN + 63) / 64) * 32;
     p.slot_bytes = slot_bytes;
     if (p.tmem_cols > 512 || p.half_cols > 32 * MAXCH) return false;
@@ -687,62 +936,98 @@ bool gemm_row_tc(betty_ctx* c, const GemmRow& g, const void* Bk, int64_t ldbk, c
     const int64_t tiles = (g.M_cap + BM - 1) / BM;
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(tiles, c->num_sms));
     const bool usebits = g.mbits != nullptr;
-#define ROW_LAUNCH(E, CB, MB)                                                                      \
+#define ROW_LAUNCH(E, CB, MB, T)                                                                   \
     do {                                                                                           \
         static bool attr = false;                                                                  \
         if (!attr) {                                                                               \
-            cudaFuncSetAttribute(k_tc_row<E, CB, MB>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024); \
+            cudaFuncSetAttribute(k_tc_row<E, CB, MB, T>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024); \
             attr = true;                                                                           \
         }                                                                                          \
-        k_tc_row<E, CB, MB><<<grid, ROW_THREADS, smem, s>>>(ma, mb, mc, p);                       \
+        k_tc_row<E, CB, MB, T><<<grid, T ? ROW_THREADS_TF : ROW_THREADS, smem, s>>>(ma, mb, mc, mbl, p); \
     } while (0)
+    if (TF) {
+        switch (g.epi) {
+        case EPI_STORE: ROW_LAUNCH(EPI_STORE, false, false, true); break;
+        case EPI_RELU_ONES: ROW_LAUNCH(EPI_RELU_ONES, false, false, true); break;
+        case EPI_MASK:
+            if (usebits) ROW_LAUNCH(EPI_MASK, false, true, true); else ROW_LAUNCH(EPI_MASK, false, false, true);
+            break;
+        default:
+            if (usebits) ROW_LAUNCH(EPI_RES_MASK, false, true, true); else ROW_LAUNCH(EPI_RES_MASK, false, false, true);
+            break;
+        }
+        return true;
+    }
     switch (g.epi) {
     case EPI_STORE:
-        if (g.c_bf16) ROW_LAUNCH(EPI_STORE, true, false); else ROW_LAUNCH(EPI_STORE, false, false);
+        if (g.c_bf16) ROW_LAUNCH(EPI_STORE, true, false, false); else ROW_LAUNCH(EPI_STORE, false, false, false);
         break;
     case EPI_RELU_ONES:
-        if (g.c_bf16) ROW_LAUNCH(EPI_RELU_ONES, true, false); else ROW_LAUNCH(EPI_RELU_ONES, false, false);
+        if (g.c_bf16) ROW_LAUNCH(EPI_RELU_ONES, true, false, false); else ROW_LAUNCH(EPI_RELU_ONES, false, false, false);
         break;
     case EPI_MASK:
-        if (g.c_bf16) { if (usebits) ROW_LAUNCH(EPI_MASK, true, true); else ROW_LAUNCH(EPI_MASK, true, false); }
-        else { if (usebits) ROW_LAUNCH(EPI_MASK, false, true); else ROW_LAUNCH(EPI_MASK, false, false); }
+        if (g.c_bf16) { if (usebits) ROW_LAUNCH(EPI_MASK, true, true, false); else ROW_LAUNCH(EPI_MASK, true, false, false); }
+        else { if (usebits) ROW_LAUNCH(EPI_MASK, false, true, false); else ROW_LAUNCH(EPI_MASK, false, false, false); }
         break;
     default:
-        if (g.c_bf16) { if (usebits) ROW_LAUNCH(EPI_RES_MASK, true, true); else ROW_LAUNCH(EPI_RES_MASK, true, false); }
-        else { if (usebits) ROW_LAUNCH(EPI_RES_MASK, false, true); else ROW_LAUNCH(EPI_RES_MASK, false, false); }
+        if (g.c_bf16) { if (usebits) ROW_LAUNCH(EPI_RES_MASK, true, true, false); else ROW_LAUNCH(EPI_RES_MASK, true, false, false); }
+        else { if (usebits) ROW_LAUNCH(EPI_RES_MASK, false, true, false); else ROW_LAUNCH(EPI_RES_MASK, false, false, false); }
         break;
     }
 #undef ROW_LAUNCH
     return true;
 }
 
-bool gemm_red_tc(betty_ctx* c, const GemmRed& g, cudaStream_t s) {
+bool gemm_red_tc(betty_ctx* c, const GemmRed& g, int* S_used, cudaStream_t s) {
     using namespace tc;
-    if (!g.a_bf16 || !g.b_bf16 || g.N > 256 || (g.lda & 7) || (g.ldb & 7)) return false;
+    const bool TF = !g.a_bf16;
+    if (TF && (g.b_bf16 || (g.lda & 3) || (g.ldb & 3))) return false;
+    if (!TF && (!g.a_bf16 || !g.b_bf16 || (g.lda & 7) || (g.ldb & 7))) return false;
+    if (g.N > 256) return false;
+    const int KN = TF ? 16 : BK, fbox = TF ? 32 : 64;
     const int BN = (g.N + 15) / 16 * 16;
     CUtensorMap ma, mb;
-    if (!make_map(&ma, g.A, g.K1, g.M_cap, g.lda, BK) || !make_map(&mb, g.B, g.N, g.M_cap, g.ldb, BK)) return false;
+    const CUtensorMapSwizzle sw = TF ? CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B : CU_TENSOR_MAP_SWIZZLE_128B;
+    if (!make_map_t(&ma, g.A, TF, g.K1, g.M_cap, g.lda, fbox, KN, sw) ||
+        !make_map_t(&mb, g.B, TF, g.N, g.M_cap, g.ldb, fbox, KN, sw))
+        return false;
     RedArgs p{};
     p.M_dev = g.M_dev; p.K1 = g.K1; p.N = g.N; p.BN = BN;
-    p.nbA = BM / 64; p.nbB = (BN + 63) / 64;
+    p.nbA = BM / fbox; p.nbB = (BN + fbox - 1) / fbox;
     p.mtiles = (g.K1 + BM - 1) / BM;
     p.acc_stride = (BN + 31) / 32 * 32;
     // all feature tiles in one CTA when their accumulators fit TMEM and a stage fits 3x in smem:
     // A and B are then read exactly once
-    const int stage_all = (p.nbA * p.mtiles + p.nbB) * BK * 128;
-    p.mt_cta = (p.mtiles * p.acc_stride <= 512 && 3 * stage_all <= 200 * 1024) ? p.mtiles : 1;
-    const int stage_bytes = (p.nbA * p.mt_cta + p.nbB) * BK * 128;
+    const int mult = TF ? 2 : 1;
+    const int stage_all = (p.nbA * p.mtiles + p.nbB) * KN * 128 * mult;
+    // TF: one feature tile per CTA (TMEM holds its accumulator and the running total)
+    p.mt_cta = (!TF && p.mtiles * p.acc_stride <= 512 && 3 * stage_all <= 200 * 1024) ? p.mtiles : 1;
+    const int stage_bytes = (p.nbA * p.mt_cta + p.nbB) * KN * 128 * mult;
     p.stages = std::max(2, std::min(8, (200 * 1024) / stage_bytes));
-    p.S = g.S;
+    // one CTA per SM: TF runs one feature tile per CTA, so mtiles x S CTAs (fewer splits than planned)
+    p.S = TF ? std::max(1, std::min(g.S, c->num_sms / std::max(1, p.mtiles))) : g.S;
+    *S_used = p.S;
     p.partials = g.partials;
-    p.tmem_cols = tmem_cols_for(p.mt_cta * p.acc_stride);
+    p.tmem_cols = tmem_cols_for((TF ? 2 : p.mt_cta) * p.acc_stride);
+    static const uint32_t sbo_env = getenv("BETTY_TF_SBO") ? (uint32_t)atoi(getenv("BETTY_TF_SBO")) : 512u;
+    p.sbo = sbo_env;
     const size_t smem = (size_t)p.stages * stage_bytes + 1024 + 256;
-    static bool attr = false;
-    if (!attr) {
-        cudaFuncSetAttribute(k_tc_red, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
-        attr = true;
+    const int grid = (p.mt_cta == 1 ? p.mtiles : 1) * p.S;
+    if (TF) {
+        static bool attr = false;
+        if (!attr) {
+            cudaFuncSetAttribute(k_tc_red<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+            attr = true;
+        }
+        k_tc_red<true><<<grid, RED_THREADS_TF, smem, s>>>(ma, mb, p);
+    } else {
+        static bool attr = false;
+        if (!attr) {
+            cudaFuncSetAttribute(k_tc_red<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+            attr = true;
+        }
+        k_tc_red<false><<<grid, THREADS, smem, s>>>(ma, mb, p);
     }
-    k_tc_red<<<(p.mt_cta == 1 ? p.mtiles : 1) * p.S, THREADS, smem, s>>>(ma, mb, p);
     return true;
 }
 

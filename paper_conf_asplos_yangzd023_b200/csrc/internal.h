@@ -9,7 +9,8 @@
 struct betty_ctx {
     int device = 0;
     int num_sms = 148;
-    bool use_tc = true;                          // tcgen05 GEMMs in BF16 mode (env BETTY_NO_TC=1 disables)
+    bool use_tc = true;                          // tcgen05 GEMMs (env BETTY_NO_TC=1 disables)
+    bool fp32_tc = true;                         // FP32 mode as 3xTF32 on tcgen05 (env BETTY_FP32_SIMT=1: FFMA)
     betty_alloc_fn alloc = nullptr;
     betty_free_fn dealloc = nullptr;
     void* user = nullptr;

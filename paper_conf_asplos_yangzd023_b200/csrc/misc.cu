@@ -160,6 +160,11 @@ void adam(betty_ctx* c, float* p, float* g, float* m, float* v, int64_t n, int t
 constexpr int PREP_MAX_L = 16;
 struct PrepArgs { PrepLayer l[PREP_MAX_L]; int L; };
 
+// nearest tf32 (10 mantissa bits) of an fp32 value, as an fp32 word (the 3xTF32 split, gemm_tc.cu)
+__device__ __forceinline__ float tf32_rn(float x) {
+    return __uint_as_float((__float_as_uint(x) + 0x1000u) & 0xFFFFE000u);
+}
+
 template <typename T>
 __global__ void k_prep(const float* __restrict__ params, PrepArgs a) {
     for (int li = 0; li < a.L; ++li) {
@@ -184,7 +189,17 @@ __global__ void k_prep(const float* __restrict__ params, PrepArgs a) {
                 else if (i == 2 * P.Fp) v = params[P.off_b + j];
             }
             st_act(B + t, v);
-            if (P.Bt && j < P.ldbt_rows) st_act((T*)P.Bt + (int64_t)j * P.ldbt + i, v);   // K-major copy
+            // FP32 mode on the tensor cores (3xTF32): hi = v rounded to the nearest tf32, lo = tf32(v - hi)
+            const float hi = tf32_rn(v), lo = tf32_rn(v - hi);
+            if (P.Bhi) { ((float*)P.Bhi)[t] = hi; ((float*)P.Blo)[t] = lo; }
+            if (P.Bt && j < P.ldbt_rows) {                                               // K-major copy
+                if (P.Btlo) {
+                    ((float*)P.Bt)[(int64_t)j * P.ldbt + i] = hi;
+                    ((float*)P.Btlo)[(int64_t)j * P.ldbt + i] = lo;
+                } else {
+                    st_act((T*)P.Bt + (int64_t)j * P.ldbt + i, v);
+                }
+            }
         }
         if (P.kind == 2) {
             T* Bp = (T*)P.Bp;
@@ -194,10 +209,32 @@ __global__ void k_prep(const float* __restrict__ params, PrepArgs a) {
                 float v = 0.f;
                 if (j < P.Fi) v = (i < P.Fi) ? params[P.off_wp + (int64_t)i * P.Fi + j] : params[P.off_bp + j];
                 st_act(Bp + t, v);
-                if (P.Bpt && j < P.Fi) st_act((T*)P.Bpt + (int64_t)j * P.ldbpt + i, v);
+                const float hi = tf32_rn(v), lo = tf32_rn(v - hi);
+                if (P.Bphi) { ((float*)P.Bphi)[t] = hi; ((float*)P.Bplo)[t] = lo; }
+                if (P.Bpt && j < P.Fi) {
+                    if (P.Bptlo) {
+                        ((float*)P.Bpt)[(int64_t)j * P.ldbpt + i] = hi;
+                        ((float*)P.Bptlo)[(int64_t)j * P.ldbpt + i] = lo;
+                    } else {
+                        st_act((T*)P.Bpt + (int64_t)j * P.ldbpt + i, v);
+                    }
+                }
             }
         }
     }
+}
+
+__global__ void k_split_tf32(const float* __restrict__ x, float* hi, float* lo, int64_t n) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        const float v = x[i];
+        const float h = tf32_rn(v);
+        hi[i] = h;
+        lo[i] = tf32_rn(v - h);
+    }
+}
+
+void split_tf32_dev(const float* x, float* hi, float* lo, int64_t n, cudaStream_t s) {
+    k_split_tf32<<<(int)std::min<int64_t>(1024, (n + 255) / 256 + 1), 256, 0, s>>>(x, hi, lo, n);
 }
 
 void prep_weights(betty_ctx* c, const float* params, const PrepLayer* layers, int L, bool bf16, cudaStream_t s) {

@@ -63,7 +63,10 @@ struct LayerBufs {
     bool hbits_ok = false;       // Hbits holds the current H (set by the forward)
     void* dS = nullptr;   // dS of layer l as GEMM operand (l < L-1)
     void* B = nullptr;    void* Bp = nullptr;
-    void* Bt = nullptr;   void* Bpt = nullptr;   // K-major weight copies (BF16 tensor-core path)
+    void* Bt = nullptr;   void* Bpt = nullptr;   // K-major weight copies (tensor-core paths; FP32 mode: hi part)
+    // FP32 mode on the tensor cores (3xTF32): hi / lo parts of the weights (null: SIMT FFMA)
+    void* Bhi = nullptr;  void* Blo = nullptr;  void* Btlo = nullptr;
+    void* Bphi = nullptr; void* Bplo = nullptr; void* Bptlo = nullptr;
     int64_t ldbt = 0, ldbpt = 0;
     int S_main = 1, S_pool = 1, S_self = 1;   // split counts of the dW reductions
 };
@@ -103,6 +106,7 @@ struct Probe {
 
 struct SageBufs {
     Probe* probe = nullptr;
+    bool tf32 = false;            // FP32 mode products as 3xTF32 on tcgen05 (else SIMT FFMA)
     std::vector<LayerBufs> l;
     float* logits = nullptr;
     float* dS_last = nullptr;

@@ -80,6 +80,8 @@ static void* balloc(betty_ctx* c, SageBufs* b, int64_t bytes, cudaStream_t s) {
 bool sage_alloc(betty_ctx* c, const ModelCfg& m, const std::vector<int64_t>& cap_dst,
                 const std::vector<int64_t>& cap_src, SageBufs* b, cudaStream_t s) {
     const int64_t ea = m.bf16 ? 2 : 4;
+    const bool tf = !m.bf16 && c->use_tc && c->fp32_tc;     // FP32 mode as 3xTF32 on the tensor cores
+    b->tf32 = tf;
     b->l.assign(m.L, LayerBufs{});
     int64_t part_max = 1;
     bool ok = true;
@@ -93,6 +95,7 @@ bool sage_alloc(betty_ctx* c, const ModelCfg& m, const std::vector<int64_t>& cap
             B.XA = A(nd * L.ld_xa * ea);
             if (l > 0 || L.kind == KIND_POOL) B.dXA = (float*)A(nd * L.ld_dxa * 4);
             B.B = A((2 * L.Fp + 1) * L.ld_B * ea);
+            if (tf) { B.Bhi = A((2 * L.Fp + 1) * L.ld_B * 4); B.Blo = A((2 * L.Fp + 1) * L.ld_B * 4); }
             B.S_main = gemm_red_splits(nd, 2 * L.Fp + 1, L.Fo);
             part_max = std::max<int64_t>(part_max, (int64_t)B.S_main * (2 * L.Fp + 1) * L.Fo);
         }
@@ -101,6 +104,7 @@ bool sage_alloc(betty_ctx* c, const ModelCfg& m, const std::vector<int64_t>& cap
             B.Ys = (float*)A(nd * L.ld_y * 4);              // [H_dst|1] [W_s; b] over the dst rows only
             B.G = A(ns * L.ld_g * ea);
             B.B = A((L.Fi + 1) * L.ld_B * ea);
+            if (tf) { B.Bhi = A((L.Fi + 1) * L.ld_B * 4); B.Blo = A((L.Fi + 1) * L.ld_B * 4); }
             if (l > 0) B.R = (float*)A(nd * m.layers[l - 1].ld_ds * 4);   // dS W_s^T (dst rows), residual of dX
             B.S_main = gemm_red_splits(ns, L.Fi + 1, L.Fop);
             B.S_self = gemm_red_splits(nd, L.Fi + 1, L.Fop);
@@ -112,20 +116,23 @@ bool sage_alloc(betty_ctx* c, const ModelCfg& m, const std::vector<int64_t>& cap
             B.arg = (int32_t*)A(nd * (m.arg8(l) ? (L.Fi + 15) / 16 * 16 : L.ld_arg * 4));
             B.dZp = A(ns * L.ld_dzp * ea);
             B.Bp = A((L.Fi + 1) * L.ld_Bp * ea);
+            if (tf) { B.Bphi = A((L.Fi + 1) * L.ld_Bp * 4); B.Bplo = A((L.Fi + 1) * L.ld_Bp * 4); }
             B.S_pool = gemm_red_splits(ns, L.Fi + 1, L.Fi);
             part_max = std::max<int64_t>(part_max, (int64_t)B.S_pool * (L.Fi + 1) * L.Fi);
         }
-        if (m.bf16) {                // K-major (transposed) weights for the tcgen05 forward GEMMs
+        if (m.bf16 || tf) {          // K-major (transposed) weights for the tcgen05 forward GEMMs (TF: hi + lo)
             const int64_t krows = L.kind == KIND_PF ? (L.Fi + 1) : (2 * L.Fp + 1);
             B.ldbt = r8(krows);
             B.Bt = A(L.ld_B * B.ldbt * ea);
+            if (tf) B.Btlo = A(L.ld_B * B.ldbt * 4);
             if (L.kind == KIND_POOL) {
                 B.ldbpt = r8(L.Fi + 1);
                 B.Bpt = A((int64_t)L.ld_Bp * B.ldbpt * ea);
+                if (tf) B.Bptlo = A((int64_t)L.ld_Bp * B.ldbpt * 4);
             }
         }
         if (l >= 1) B.H = A(ns * m.layers[l - 1].ld_out * ea);
-        if (l >= 1 && m.bf16) {
+        if (l >= 1 && (m.bf16 || tf)) {
             B.ldhb = (m.dims[l] + 127) / 128 * 4;
             B.Hbits = (uint32_t*)A(ns * B.ldhb * 4);
         }
@@ -159,6 +166,8 @@ void sage_prep(betty_ctx* c, const ModelCfg& m, SageBufs& b, const float* params
         p.Bp = b.l[l].Bp; p.ldbp = L.ld_Bp;
         p.Bt = b.l[l].Bt; p.ldbt = b.l[l].ldbt; p.ldbt_rows = L.ld_B;
         p.Bpt = b.l[l].Bpt; p.ldbpt = b.l[l].ldbpt;
+        p.Bhi = b.l[l].Bhi; p.Blo = b.l[l].Blo; p.Btlo = b.l[l].Btlo;
+        p.Bphi = b.l[l].Bphi; p.Bplo = b.l[l].Bplo; p.Bptlo = b.l[l].Bptlo;
     }
     prep_weights(c, params, P.data(), m.L, m.bf16, s);
 }
@@ -167,6 +176,18 @@ void sage_prep(betty_ctx* c, const ModelCfg& m, SageBufs& b, const float* params
 static void ones_operand(const ModelCfg& m, SageBufs& b, int l, const void** A, int64_t* lda) {
     if (l == 0) { *A = b.l[0].gat; *lda = m.layers[0].ld_gat; }
     else { *A = b.l[l].H; *lda = m.layers[l - 1].ld_out; }
+}
+
+// FP32 mode (3xTF32): the hi / lo weight parts of a GemmRow whose B is the main weight (pool = false)
+// or the pool weight, viewed from column col0 of B (row col0 of its K-major copy)
+static void tf_weights(GemmRow& g, const LayerBufs& B, bool pool, int64_t col0) {
+    void* hi = pool ? B.Bphi : B.Bhi;
+    void* lo = pool ? B.Bplo : B.Blo;
+    void* tlo = pool ? B.Bptlo : B.Btlo;
+    const int64_t ldbt = pool ? B.ldbpt : B.ldbt;
+    g.Bhi = hi ? (const char*)hi + col0 * 4 : nullptr;
+    g.Blo = lo ? (const char*)lo + col0 * 4 : nullptr;
+    g.Btlo = tlo ? (const char*)tlo + col0 * ldbt * 4 : nullptr;
 }
 
 static GradMap grad_map(const LayerCfg& L, int mode) {
@@ -208,6 +229,7 @@ void sage_forward(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView*
             g.M_dev = V.cnt + 1; g.M_cap = V.cap_src; g.K = L.Fi + 1; g.N = L.Fop;
             g.Bt = B.Bt; g.ldbt = B.ldbt;
             g.C = B.Y; g.ldc = L.ld_y; g.c_bf16 = false; g.epi = EPI_STORE;
+            tf_weights(g, B, false, 0);
             PB(l == 0 ? PROBE_GEMM_FWD_L0 : PROBE_GEMM_FWD_L1);
             gemm_row(c, g, s);
             PE(l == 0 ? PROBE_GEMM_FWD_L0 : PROBE_GEMM_FWD_L1);
@@ -216,6 +238,7 @@ void sage_forward(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView*
             gs.Bt = B.Bt ? (const void*)((const char*)B.Bt + (int64_t)L.Fop * B.ldbt * esz) : nullptr;
             gs.M_dev = V.cnt + 0; gs.M_cap = V.cap_dst;
             gs.C = B.Ys;
+            tf_weights(gs, B, false, L.Fop);
             gemm_row(c, gs, s);
             PB(l == 0 ? PROBE_AGG_L0 : PROBE_AGG_L1);
             agg_mean_pf(c, B.Y, B.Ys, L.ld_y, V.indptr, V.indices, V.cnt, V.cap_dst, L.Fo, L.Fop, !L.last, out,
@@ -231,6 +254,7 @@ void sage_forward(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView*
             g.M_dev = V.cnt + 1; g.M_cap = V.cap_src; g.K = L.Fi + 1; g.N = L.Fi;
             g.Bt = B.Bpt; g.ldbt = B.ldbpt;
             g.C = B.Zp; g.ldc = L.ld_zp; g.c_bf16 = false; g.epi = EPI_STORE;
+            tf_weights(g, B, true, 0);
             gemm_row(c, g, s);
             PB(l == 0 ? PROBE_AGG_L0 : PROBE_AGG_L1);
             agg_pool(c, X, xbf, ldx, xrow, B.Zp, L.ld_zp, V.indptr, V.indices, V.cnt, V.cap_dst, L.Fi, L.Fp, B.XA,
@@ -252,6 +276,7 @@ void sage_forward(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView*
         g.M_dev = V.cnt + 0; g.M_cap = V.cap_dst; g.K = 2 * L.Fp + 1; g.N = L.Fo;
         g.Bt = B.Bt; g.ldbt = B.ldbt;
         g.C = out; g.ldc = L.ld_out; g.c_bf16 = out_bf; g.epi = epi;
+        tf_weights(g, B, false, 0);
         if (!L.last) { g.obits = b.l[l + 1].Hbits; g.ldob = b.l[l + 1].ldhb; }
         PB(l == 0 ? PROBE_GEMM_FWD_L0 : PROBE_GEMM_FWD_L1);
         const bool bits = gemm_row(c, g, s);
@@ -307,6 +332,7 @@ void sage_backward(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView
                 gr.B = (const char*)B.B + L.Fop * esz; gr.ldb = L.ld_B; gr.b_bf16 = m.bf16; gr.transB = true;
                 gr.M_dev = V.cnt + 0; gr.M_cap = V.cap_dst; gr.K = L.Fo; gr.N = L.Fi;
                 gr.C = B.R; gr.ldc = ld_prev; gr.c_bf16 = false; gr.epi = EPI_STORE;
+                tf_weights(gr, B, false, L.Fop);
                 gemm_row(c, gr, s);
                 GemmRow g{};
                 g.A = B.G; g.lda = L.ld_g; g.a_bf16 = m.bf16;
@@ -316,6 +342,7 @@ void sage_backward(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView
                 g.mask = Hmask; g.ldm = ldh; g.m_bf16 = m.bf16;
                 g.res = B.R; g.ldr = ld_prev; g.nres_dev = V.cnt + 0;
                 if (B.hbits_ok) { g.mbits = B.Hbits; g.ldmb = B.ldhb; }
+                tf_weights(g, B, false, 0);
                 gemm_row(c, g, s);
             }
             continue;
@@ -338,6 +365,7 @@ void sage_backward(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView
             g.B = B.B; g.ldb = L.ld_B; g.b_bf16 = m.bf16; g.transB = true;
             g.M_dev = V.cnt + 0; g.M_cap = V.cap_dst; g.K = L.Fo; g.N = 2 * L.Fp;
             g.C = B.dXA; g.ldc = L.ld_dxa; g.c_bf16 = false; g.epi = EPI_STORE;
+            tf_weights(g, B, false, 0);
             gemm_row(c, g, s);
         }
         if (L.kind == KIND_AGG) {
@@ -368,6 +396,7 @@ void sage_backward(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView
             g.mask = Hmask; g.ldm = ldh; g.m_bf16 = m.bf16;
             if (B.hbits_ok) { g.mbits = B.Hbits; g.ldmb = B.ldhb; }
             g.res = B.dXA; g.ldr = L.ld_dxa; g.nres_dev = V.cnt + 0;
+            tf_weights(g, B, true, 0);
             gemm_row(c, g, s);
         }
     }

@@ -48,6 +48,9 @@ struct GemmRow {                 // C[m, n] = sum_k A[m, k] B(k, n), m < *M_dev
     const void* mask; int64_t ldm; bool m_bf16;           // EPI_MASK / EPI_RES_MASK: C *= [mask > 0]
     const float* res; int64_t ldr; const int64_t* nres_dev; // EPI_RES_MASK: C += res (rows < *nres_dev)
     const void* Bt; int64_t ldbt;                          // K-major copy of B (N x K) for the tensor-core path
+    // FP32 mode on the tensor cores (3xTF32): B split into hi (tf32-exact) + lo, in B's layout (transB
+    // products) and K-major (Bt holds hi, Btlo lo); null: SIMT FFMA
+    const void* Bhi = nullptr; const void* Blo = nullptr; const void* Btlo = nullptr;
     const uint32_t* mbits; int64_t ldmb;   // EPI_MASK / EPI_RES_MASK: mask as ReLU bits (tensor-core path), or null
     uint32_t* obits; int64_t ldob;         // EPI_RELU_ONES: also write the ReLU bits [C > 0] (tensor-core path)
     int64_t cend = 0;                      // tensor-core path: trailing columns [N, cend) written (0: ldc)
@@ -58,7 +61,7 @@ bool gemm_row(betty_ctx* c, const GemmRow& g, cudaStream_t s);
 bool tc_available();
 bool make_gather_map(CUtensorMap* m, const void* base, bool f32, int64_t cols, int64_t rows, int64_t ld,
                      int box_cols);
-bool gemm_row_tc(betty_ctx* c, const GemmRow& g, const void* Bk, int64_t ldbk, cudaStream_t s);
+bool gemm_row_tc(betty_ctx* c, const GemmRow& g, const void* Bk, const void* Bk_lo, int64_t ldbk, cudaStream_t s);
 
 // P[i, j] = sum_{r < *M_dev} A[r, i] B[r, j], i < K1, j < N, split over S row groups into
 // partials[S][K1][N]; then grad[map(i,j)] += sum_s partials[s][i][j] (fixed order: deterministic).
@@ -77,7 +80,8 @@ struct GemmRed {
 };
 void gemm_red(betty_ctx* c, const GemmRed& g, cudaStream_t s);
 int gemm_red_splits(int64_t M_cap, int K1, int N);
-bool gemm_red_tc(betty_ctx* c, const GemmRed& g, cudaStream_t s);
+// S_used: the row splits (partials) the launch wrote (<= g.S)
+bool gemm_red_tc(betty_ctx* c, const GemmRed& g, int* S_used, cudaStream_t s);
 
 // ---- misc.cu
 void loss_ce(betty_ctx* c, const float* logits, int64_t ldl, const int32_t* labels, const int32_t* gid,
@@ -95,7 +99,11 @@ struct PrepLayer {
     void* Bt; int64_t ldbt;      // K-major (transposed) copies for the tensor-core path (may be null)
     int64_t ldbt_rows;           // rows of Bt (= columns of B that are written)
     void* Bpt; int64_t ldbpt;
+    // FP32 mode, 3xTF32 (null otherwise): Bt / Bpt then hold the hi parts
+    void* Bhi; void* Blo; void* Btlo; void* Bphi; void* Bplo; void* Bptlo;
 };
 void prep_weights(betty_ctx* c, const float* params, const PrepLayer* layers, int L, bool bf16, cudaStream_t s);
+// hi = x with the low 13 mantissa bits cleared, lo = x - hi (the 3xTF32 operand split), n elements
+void split_tf32_dev(const float* x, float* hi, float* lo, int64_t n, cudaStream_t s);
 
 }  // namespace betty

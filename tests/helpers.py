@@ -126,3 +126,56 @@ def assert_grad_close(x, ref, dims, aggr, rtol, name=""):
     a small tensor such as a bias could hide a large relative error)."""
     for (tn, a), (_, b) in zip(param_tensors(x, dims, aggr), param_tensors(ref, dims, aggr)):
         assert_close(a, b, rtol, f"{name} {tn}")
+
+
+def explain_relu_flips(gpu, ref, ties, mb, feats, dims, aggr, rtol, name=""):
+    """Reading #24: compare a gradient whose hidden ReLU decisions may legitimately differ.
+
+    Where |S| <= tau * M (oracle.sage_ties), fp32 evaluation can take the ReLU decision either way:
+    both gradients are correct.  A decision on H_1 (layer 0's output) at (v, j) gates dS_0[v, j] = g,
+    and flipping it changes only layer 0's gradient, by d * g * (x_v (x) e_j, A_v (x) e_j, e_j) for
+    (W_self, W_neigh, b) (d = +1 if the oracle's S <= 0, else -1; x_v the dst row's input, A_v its
+    aggregated neighbours, the same rank-1 form for either SAGEConv form of mean/sum).  Per output
+    column the flips are fitted by least squares and rounded to {0, 1}; the residual must then pass
+    the per-tensor bound of reading #18 and every flip must be one of the oracle's candidates.
+    Returns the number of flips explained."""
+    assert aggr in ("mean", "sum")
+    gpu = np.asarray(gpu, np.float64)
+    ref = np.asarray(ref, np.float64)
+    lev = ties["level"]
+    assert (lev == 1).all() or len(lev) == 0 or len(dims) == 2, "flip explanation covers decisions on H_1"
+    sel = lev == 1
+    tv, tj, tS, tg = ties["v"][sel], ties["j"][sel], ties["S"][sel], ties["g"][sel]
+    F, Fo = dims[0], dims[1]
+    b0 = mb[0]
+    X = feats[b0.src_gid, :F].astype(np.float64)
+    delta = gpu - ref
+    W = split_params(delta, dims, aggr)
+    dWs, dWn, db = W[0]["Ws"].copy(), W[0]["Wn"].copy(), W[0]["b"].copy()
+    flips = 0
+    for j in np.unique(tj):
+        idx = np.nonzero(tj == j)[0]
+        cols = []
+        for i in idx:
+            v = int(tv[i])
+            nb = (b0.indices if hasattr(b0, "indices") else b0.nbr_pos)[b0.indptr[v]:b0.indptr[v + 1]]
+            Av = X[nb].sum(0) if len(nb) else np.zeros(F)
+            if aggr == "mean" and len(nb):
+                Av = Av / len(nb)
+            d = 1.0 if tS[i] <= 0 else -1.0
+            cols.append(d * tg[i] * np.concatenate([X[v], Av, [1.0]]))
+        Amat = np.stack(cols, 1)
+        rhs = np.concatenate([dWs[:, j], dWn[:, j], [db[j]]])
+        c, *_ = np.linalg.lstsq(Amat, rhs, rcond=None)
+        c = np.clip(np.rint(c), 0, 1)
+        fix = Amat @ c
+        dWs[:, j] -= fix[:F]
+        dWn[:, j] -= fix[F:2 * F]
+        db[j] -= fix[2 * F]
+        flips += int(c.sum())
+    R = split_params(ref, dims, aggr)
+    for tn, d, r in (("Ws0", dWs, R[0]["Ws"]), ("Wn0", dWn, R[0]["Wn"]), ("b0", db, R[0]["b"])):
+        assert_close(r + d, r, rtol, f"{name} {tn} (after {flips} explained ReLU flips)")
+    for (tn, a), (_, b) in list(zip(param_tensors(gpu, dims, aggr), param_tensors(ref, dims, aggr)))[3:]:
+        assert_close(a, b, rtol, f"{name} {tn}")
+    return flips
