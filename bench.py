@@ -54,6 +54,9 @@ def parse():
     p.add_argument("--no-reg", action="store_true", help="exclude the REG rebuild (a1) from the step")
     p.add_argument("--probe", default="auto")
     p.add_argument("--e2e-steps", type=int, default=20)
+    p.add_argument("--no-fp32", action="store_true",
+                   help="skip the nested paper-precision (fp32, 3xTF32 GEMMs) measurement of a bf16 run")
+    p.add_argument("--cpu-threads", type=int, default=0, help="cpu_baseline / reference threads (0: all cores)")
     p.add_argument("--cpu-sample-outputs", type=int, default=4096, help="cpu_baseline sample (~10 s)")
     p.add_argument("--ref-sample-outputs", type=int, default=1024, help="--impl reference per-step sample")
     p.add_argument("--scale", type=float, default=1.0, help="shrink the graph (debug only)")
@@ -218,12 +221,13 @@ def memory_aware(args, B, ctx, cfg, dev_blocks, rank, ws, device):
         reg = (ip.cpu().numpy(), col.cpu().numpy(), w.cpu().numpy())
         model = B.Model(cfg.dims, cfg.aggr, args.mode, args.mode)
         K, part, peak = B.betty_memory_aware_k(ctx, model, dev_blocks, reg, int(args.capacity_gb * 2 ** 30))
-        if K < 0:
-            raise SystemExit(f"memory-aware K: no K fits {args.capacity_gb} GB (smallest peak {peak / 2**30:.2f} GB)")
         res = [{"K": K, "capacity_gb": args.capacity_gb, "peak_estimate_gb": peak / 2 ** 30,
                 "search_s": time.time() - t0}]
-    if ws > 1:
+    if ws > 1:                     # every rank learns the outcome (a failure marker included) before exiting
         dist.broadcast_object_list(res, src=0)
+    if res[0]["K"] < 0:
+        raise SystemExit(f"memory-aware K: no K fits {args.capacity_gb} GB "
+                         f"(smallest peak {res[0]['peak_estimate_gb']:.2f} GB)")
     args.K = res[0]["K"]
     return res[0]
 
@@ -251,7 +255,11 @@ def make_partition(args, B, ctx, cfg, ds, dev_blocks, rank, ws, device):
 
 def alg_bytes(site: str, info: dict, cfg, mode: str, n_groups: int):
     """Algorithmic (compulsory) bytes of ONE launch of a kernel site, from the
-    plan's per-layer totals.  Totals / n_groups = per launch."""
+    plan's per-layer totals.  Totals / n_groups = per launch.
+    agg_l0 is SURVEY.md §8(d)'s AGG-MEAN formula with the gather stream replaced by each
+    micro-batch's distinct source rows: 4E + 8(n_dst+1) + s F n_src + s F n_dst (index stream,
+    indptr, every needed feature row once, the aggregated rows written) -- the kernel's extra
+    self-row copy into XA and the ones column are not algorithmic."""
     s_feat = 2 if mode == "bf16" else 4
     s_act = 2 if mode == "bf16" else 4
     E, ns, nd = info["edges"], info["n_src"], info["n_dst"]
@@ -259,7 +267,7 @@ def alg_bytes(site: str, info: dict, cfg, mode: str, n_groups: int):
     Fp = (F + 7) // 8 * 8
     ld_xa = (2 * Fp + 1 + 7) // 8 * 8
     if site == "agg_l0":
-        b = 8 * (nd[0] + 1) + 4 * E[0] + 4 * ns[0] + s_feat * F * ns[0] + s_act * ld_xa * nd[0]
+        b = 4 * E[0] + 8 * (nd[0] + 1) + s_feat * F * ns[0] + s_act * F * nd[0]
     elif site == "gemm_fwd_l0":
         H = cfg.hidden
         b = s_act * ld_xa * nd[0] + s_act * (2 * Fp + 1) * H + s_act * ((H + 1 + 7) // 8 * 8) * nd[0]
@@ -268,7 +276,8 @@ def alg_bytes(site: str, info: dict, cfg, mode: str, n_groups: int):
     return b / max(n_groups, 1)
 
 
-METRIC = "aggregated edges/s (SAGE, products-shape); epoch time = ms_per_step"
+METRIC = ("aggregated edges/s (SAGE, products-shape; edges of every micro-batch, redundant ones included, "
+          "SURVEY §8(d)); epoch time = ms_per_step")
 
 
 def workload_config(args, cfg, ws):
@@ -282,50 +291,63 @@ def workload_config(args, cfg, ws):
 
 # ------------------------------------------------------------ reference arm
 def run_reference(args, ws, rank):
-    """The CPU oracle, as it stands, on a bounded sample of the same workload
-    (micro-batch 0 of the bench's partition, its first S outputs)."""
+    """The CPU oracle, as it stands, on a bounded sample of the same workload: per step, one sample per
+    host core in parallel (the first S outputs of micro-batch t of a range split, t = 0..cores-1)."""
     if rank != 0:
         return
     import synth
     import oracle
+    from concurrent.futures import ThreadPoolExecutor
     cfg = synth.CONFIGS[args.config]
     if args.scale != 1.0:
         cfg = synth.scaled(cfg, args.scale)
     ds = synth.make(cfg, with_features=None)
     args.K = args.K or 8
-    part, sample_desc, edges = reference_sample(args, cfg, ds, args.ref_sample_outputs)
-    oblocks, ofeats = oracle_inputs(cfg, ds, part)
+    nt = cpu_threads(args)
+    jobs = []
+    for t in range(nt):
+        part, sample_desc, edges = reference_sample(args, cfg, ds, args.ref_sample_outputs, mb=t % args.K)
+        oblocks, ofeats = oracle_inputs(cfg, ds, part)
+        jobs.append((part, oblocks, ofeats, edges))
     params = synth.init_params(cfg.dims, cfg.aggr, seed=cfg.seeds["init"])
-    times = []
-    for it in range(args.warmup + args.steps):
-        t0 = time.perf_counter()
+    edges = sum(j[3] for j in jobs)
+
+    def run(j):
+        part, oblocks, ofeats, _ = j
         oracle.step(cfg.dims, cfg.aggr, args.mode == "bf16", oblocks, part, 2, [0], params, ofeats, ds.labels,
                     1.0 / cfg.n_out)
-        if it >= args.warmup:
-            times.append(time.perf_counter() - t0)
+    times = []
+    with ThreadPoolExecutor(nt) as ex:
+        for it in range(args.warmup + args.steps):
+            t0 = time.perf_counter()
+            list(ex.map(run, jobs))
+            if it >= args.warmup:
+                times.append(time.perf_counter() - t0)
     t = float(np.mean(times))
     val = edges / t
+    desc = (f"{nt} samples in parallel per step, each {args.ref_sample_outputs} outputs of one micro-batch "
+            f"(K={args.K} range split) through {cfg.L} layers, extraction+fwd+bwd in float64; {edges} edges")
     line = {"impl": "reference", "metric": METRIC, "value": val,
             "unit": "edges/s", "higher_is_better": True, "n_gpus": args.gpus, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": t * 1e3, "dtype": "f64", "data": "synthetic",
-            "config": dict(workload_config(args, cfg, ws), sample=sample_desc),
-            "cpu_baseline": {"value": val, "unit": "edges/s", "cores": 1, "kind": "oracle", "sample": sample_desc},
+            "config": dict(workload_config(args, cfg, ws), sample=desc),
+            "cpu_baseline": {"value": val, "unit": "edges/s", "cores": nt, "kind": "oracle", "sample": desc},
             "e2e": {"value": val, "unit": "edges/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
 
-def reference_sample(args, cfg, ds, n_outputs):
-    """Outputs: the first S outputs (ascending) of micro-batch 0 of a range
+def reference_sample(args, cfg, ds, n_outputs, mb=0):
+    """Outputs: the first S outputs (ascending) of micro-batch mb of a range
     partition into K parts -> a 2-way partition {sample, rest}."""
     import synth
     import oracle
-    base = synth.range_partition(cfg.n_out, args.K)
-    idx = np.nonzero(base == 0)[0][:n_outputs]
+    base = synth.range_partition(cfg.n_out, max(args.K, 1))
+    idx = np.nonzero(base == mb)[0][:n_outputs]
     part = np.ones(cfg.n_out, dtype=np.int32)
     part[idx] = 0
     mb = oracle.extract(ds.blocks, part, 2, 0)
     edges = sum(b.n_edges for b in mb)
-    desc = (f"{len(idx)} outputs (first of micro-batch 0, K={args.K}); {edges} edges through "
+    desc = (f"{len(idx)} outputs (first of micro-batch {mb}, K={args.K}); {edges} edges through "
             f"{cfg.L} layers; extraction+fwd+bwd in float64, 1 thread")
     return part, desc, edges
 
@@ -434,20 +456,9 @@ def main():
 
     # ------------------------------------------------------ timed region
     clocks = ClockSampler(local)
-    if ws > 1:
-        dist.barrier()
-    torch.cuda.synchronize()
     clocks.start()
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    e0.record(stream)
-    for _ in range(args.steps):
-        step()
-    e1.record(stream)
-    torch.cuda.synchronize()
-    if ws > 1:
-        dist.barrier()
+    ms = timed_ms(step, args.steps, ws, stream)
     clk = clocks.stop()
-    ms = e0.elapsed_time(e1) / args.steps
     t = torch.tensor([ms, float(sum(info["edges"])), float(info["kernels_per_step"])], device=device,
                      dtype=torch.float64)
     if ws > 1:
@@ -460,12 +471,56 @@ def main():
         ms_step, edges_all = ms, float(t[1])
     value = edges_all / (ms_step * 1e-3)
     launches = args.steps * (info["kernels_per_step"] + 1)
+    full_edges = int(sum(b.n_edges for b in ds.blocks))
+    peaks, peak_src = measured_peaks()
+    tkey = lambda mode: f"{args.config}:K{args.K}:{mode}:n{ws}"     # noqa: E731 (profiles/traffic.json key)
+    roof = roofline(plan, step, info, cfg, args.mode, ms, peaks, peak_src, tkey(args.mode))
+
+    # ---------------------- paper precision (fp32) beside a bf16 headline
+    paper = None
+    if args.mode == "bf16" and not args.no_fp32:
+        feats32 = synth.features_device(cfg, ds, False, args.feat_align, device)
+        if args.feat_layout != "gid":
+            feats32 = None                       # (study layouts permute the bf16 table only)
+        if feats32 is not None:
+            model32 = B.Model(cfg.dims, cfg.aggr, "fp32", "fp32")
+            plan32, g32 = create_plan(B, ctx, model32, dev_blocks, dpart, args.K, my_k, args.group, flags)
+            if wv > 1 and not args.no_reg:
+                plan32.set_reg_rows(*reg_rows(cfg.n_out, rv, wv))
+
+            def step32():
+                loss.zero_()
+                B.betty_step(ctx, plan32, params, feats32, labels, scale, grad, loss)
+                allreduce_grad(grad)
+                t_opt[0] += 1
+                B.betty_adam(ctx, params, grad, m, v, t_opt[0], zero_grad=True)
+            for _ in range(args.warmup):
+                step32()
+            ms32 = timed_ms(step32, args.steps, ws, stream)
+            info32 = plan32.info()
+            t32 = torch.tensor([ms32], device=device, dtype=torch.float64)
+            if ws > 1:
+                dist.all_reduce(t32, op=dist.ReduceOp.MAX)
+            ms32 = float(t32[0])
+            paper = {"dtype": "fp32 (GEMMs as 3xTF32 on tcgen05: hi*hi + lo*hi + hi*lo, fp32 accumulation)",
+                     "value": edges_all / (ms32 * 1e-3), "unit": "edges/s", "ms_per_step": ms32,
+                     "full_batch_edges_per_s": full_edges / (ms32 * 1e-3), "group": g32 or "all",
+                     "arena_gb": info32["arena_bytes"] / 2 ** 30,
+                     "roofline": roofline(plan32, step32, info32, cfg, "fp32", ms32, peaks, peak_src,
+                                          tkey("fp32"))}
+            plan32.free()
+            del feats32
+            torch.cuda.synchronize()
+            torch.cuda.empty_cache()
 
     # ------------------------------------- e2e: host buffers through the ABI
     # Every step copies its own inputs (the full-batch blocks and the partition) from pinned host
-    # memory and reads its loss back.  Double-buffered when a second plan fits in HBM: the inputs of
-    # step i+1 are copied on a copy stream into the other buffer set while step i computes (a plan
-    # binds its blocks' device pointers, so each buffer set has its own plan); else serial.
+    # memory and reads its loss back.  The e2e plans are BETTY_PLAN_FRESH: each step derives everything
+    # from the copied buffers (the full-batch CSCs and the REG's CSC are rebuilt inside the step), so a
+    # step would consume a resampled batch of the same sizes.  Double-buffered when two plans fit in HBM
+    # (the inputs of step i+1 are copied on a copy stream into the other buffer set while step i
+    # computes; a plan binds its blocks' device pointers, so each buffer set has its own plan); else
+    # serial.
     host = []
     for l, b in enumerate(ds.blocks):
         host += [torch.from_numpy(b.indptr).pin_memory(), torch.from_numpy(b.nbr_pos).pin_memory(),
@@ -477,26 +532,30 @@ def main():
         for db in dbs:
             out += [db.indptr, db.indices, db.src_gid]
         return out + [dp]
-    bufs, plans = [dev_list(dev_blocks, dpart)], [plan]
-    try:
-        dev_blocks2 = B.blocks_to_device(ds.blocks, local)
-        dev_blocks2[0].src_gid.copy_(dev_blocks[0].src_gid)
-        dpart2 = dpart.clone()
-        plan2, g2 = create_plan(B, ctx, model, dev_blocks2, dpart2, args.K, my_k, args.group or 0, flags)
-        if g2 != (args.group or 0):               # only the same launch grouping is the same step
-            plan2.free()
-            raise RuntimeError("second plan would need a smaller launch group")
-        if wv > 1 and not args.no_reg:
-            plan2.set_reg_rows(*reg_rows(cfg.n_out, rv, wv))
-        bufs.append(dev_list(dev_blocks2, dpart2))
-        plans.append(plan2)
-        step(plan2)                                # capture its graph outside the timed region
-        torch.cuda.synchronize()
-    except (B.BettyError, SystemExit, RuntimeError) as e:   # no room for a second buffer set: serial
-        print(f"e2e: single-buffered ({e})", file=sys.stderr)
-        dev_blocks2 = dpart2 = None
-        torch.cuda.synchronize()
-        torch.cuda.empty_cache()
+    fresh = flags | B.PLAN_FRESH
+    plans, bufs = [], []
+    for _ in range(2):
+        try:
+            dbs = B.blocks_to_device(ds.blocks, local)
+            dbs[0].src_gid.copy_(dev_blocks[0].src_gid)
+            dp = dpart.clone()
+            pe, ge = create_plan(B, ctx, model, dbs, dp, args.K, my_k, args.group or 0, fresh)
+            if ge != (args.group or 0):            # only the same launch grouping is the same step
+                pe.free()
+                raise RuntimeError("e2e plan would need a smaller launch group")
+            if wv > 1 and not args.no_reg:
+                pe.set_reg_rows(*reg_rows(cfg.n_out, rv, wv))
+            plans.append(pe)
+            bufs.append(dev_list(dbs, dp))
+            step(pe)                               # capture its graph outside the timed region
+            torch.cuda.synchronize()
+        except (B.BettyError, SystemExit, RuntimeError) as e:
+            print(f"e2e: {len(plans)} buffer set(s) ({e})", file=sys.stderr)
+            torch.cuda.synchronize()
+            torch.cuda.empty_cache()
+            break
+    if not plans:                                  # no room for a FRESH plan: re-copy into the timed plan
+        plans, bufs = [plan], [dev_list(dev_blocks, dpart)]
     h2d = sum(x.numel() * x.element_size() for x in host)
     loss_host = torch.zeros(1).pin_memory()
     cs = torch.cuda.Stream(device=device)
@@ -509,6 +568,7 @@ def main():
             for hsrc, ddst in zip(host, bufs[b]):
                 ddst.copy_(hsrc, non_blocking=True)
             ev_copied[b].record(cs)
+    e2e_steps = max(1, args.e2e_steps)
     if ws > 1:
         dist.barrier()
     torch.cuda.synchronize()
@@ -516,10 +576,10 @@ def main():
     f0.record(stream)
     cs.wait_stream(stream)
     copy_in(0)
-    for i in range(args.e2e_steps):
+    for i in range(e2e_steps):
         b = i % nb
         stream.wait_event(ev_copied[b])
-        if nb > 1 and i + 1 < args.e2e_steps:     # next step's inputs, once the step that used them is done
+        if nb > 1 and i + 1 < e2e_steps:          # next step's inputs, once the step that used them is done
             if i >= 1:
                 cs.wait_event(ev_used[1 - b])
             copy_in(1 - b)
@@ -528,58 +588,25 @@ def main():
         loss_host.copy_(loss, non_blocking=True)
         stream.synchronize()
         _ = float(loss_host[0])
-        if nb == 1 and i + 1 < args.e2e_steps:
+        if nb == 1 and i + 1 < e2e_steps:
             cs.wait_stream(stream)
             copy_in(0)
     f1.record(stream)
     torch.cuda.synchronize()
-    e2e_ms = f0.elapsed_time(f1) / args.e2e_steps
+    e2e_ms = f0.elapsed_time(f1) / e2e_steps
     if ws > 1:
         te = torch.tensor([e2e_ms], device=device, dtype=torch.float64)
         dist.all_reduce(te, op=dist.ReduceOp.MAX)
         e2e_ms = float(te[0])
-    for pl in plans[1:]:
-        pl.free()
-
-    # ---------------------------------- roofline of the dominant kernel
-    sites = {"agg_l0": 1, "gemm_fwd_l0": 2, "gemm_red_l0": 3, "extract": 4, "reg": 5}
-    probe_ms = {}
-    for name, sid in sites.items():
-        plan.probe(sid)
-        tot, n = 0.0, 0
-        for _ in range(3):
-            step()
-            ms_k, nl = plan.probe_read()
-            tot += ms_k
-            n += nl
-        probe_ms[name] = (tot / max(n, 1), n / 3)
-    plan.probe(0)
-    peaks, peak_src = measured_peaks()
-    key = f"{args.config}:K{args.K}:{args.mode}:n{ws}"
-    dom = "agg_l0"
-    per_launch_ms, launches_per_step = probe_ms[dom]
-    ab = alg_bytes(dom, info, cfg, args.mode, info["n_groups"]) if cfg.aggr == "mean" else None
-    achieved = ab / (per_launch_ms * 1e-3) / 1e9 if ab else None
-    roof = None if ab is None else {"kernel": "k_agg_mean_g4 (layer-0 mean aggregation)", "bound": "hbm", "achieved": achieved,
-            "peak": peaks["hbm_gbs"], "unit": "GB/s", "frac": achieved / peaks["hbm_gbs"],
-            "traffic": load_traffic(dom, key), "alg_bytes_per_launch": ab, "avg_launch_ms": per_launch_ms,
-            "launches_per_step": launches_per_step, "peak_source": peak_src,
-            "share_of_step": per_launch_ms * launches_per_step / ms,
-            "other_sites_ms_per_step": {k: v[0] * v[1] for k, v in probe_ms.items()}}
+    for pl in plans:
+        if pl is not plan:
+            pl.free()
+    B.betty_sync_check(ctx)                        # FRESH steps validate the copied inputs on the device
 
     # ------------------------------------------------------- cpu baseline
     cpu = None
-    if rank == 0 and ws == 1:
-        import oracle
-        rpart, desc, redges = reference_sample(args, cfg, ds, args.cpu_sample_outputs)
-        oblocks, ofeats = oracle_inputs(cfg, ds, rpart)
-        pr = synth_params(cfg).astype(np.float64)
-        tc = time.perf_counter()
-        oracle.step(cfg.dims, cfg.aggr, args.mode == "bf16", oblocks, rpart, 2, [0], pr, ofeats, ds.labels,
-                    scale)
-        dt = time.perf_counter() - tc
-        cpu = {"value": redges / dt, "unit": "edges/s", "cores": 1, "kind": "oracle", "sample": desc,
-               "seconds": dt}
+    if rank == 0 and ws == 1 and args.cpu_sample_outputs > 0:
+        cpu = cpu_baseline(args, cfg, ds, scale)
 
     if rank == 0:
         line = {
@@ -592,12 +619,17 @@ def main():
                            l2="inputs > L2 (feature table %.2f GB + blocks)" % (feats.numel() * feats.element_size()
                                                                               / 1e9)),
             "edges_per_step": edges_all,
-            "full_batch_edges": int(sum(b.n_edges for b in ds.blocks)),
+            "full_batch_edges": full_edges,
+            "full_batch_edges_per_s": full_edges / (ms_step * 1e-3),
             "plan": {k: info[k] for k in ("n_groups", "edges", "n_src", "n_dst", "reg_nnz", "arena_bytes",
                                           "kernels_per_step")},
+            "memory": {"group": args.group or "all", "plan_arena_gb": info["arena_bytes"] / 2 ** 30,
+                       "feature_table_gb": feats.numel() * feats.element_size() / 2 ** 30,
+                       "peak_allocated_gb": torch.cuda.max_memory_allocated(device) / 2 ** 30},
+            "paper_precision": paper,
             "e2e": {"value": edges_all / (e2e_ms * 1e-3), "unit": "edges/s", "ms_per_step": e2e_ms,
                     "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": 4,
-                    "input_buffers": nb},
+                    "input_buffers": nb, "fresh_inputs": plans[0] is not plan},
             "gpu_launches": launches,
             "clocks": clk,
             "roofline": roof,
@@ -619,6 +651,90 @@ def main():
     plan.free()
     if ws > 1:
         dist.destroy_process_group()
+
+
+def timed_ms(step, steps, ws, stream):
+    """K steps between a barrier + synchronize on both sides, timed with CUDA events on the launching
+    stream; ms per step of THIS rank (the caller takes the max over ranks)."""
+    import torch
+    import torch.distributed as dist
+    if ws > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for _ in range(steps):
+        step()
+    e1.record(stream)
+    torch.cuda.synchronize()
+    if ws > 1:
+        dist.barrier()
+    return e0.elapsed_time(e1) / steps
+
+
+SITES = {"agg_l0": 1, "gemm_fwd_l0": 2, "gemm_red_l0": 3, "extract": 4, "reg": 5}
+
+
+def roofline(plan, step, info, cfg, mode, ms, peaks, peak_src, key):
+    """Roofline of the dominant kernel (the layer-0 mean aggregation): its launches bracketed by CUDA
+    events on the step's stream (betty_plan_probe) over 3 steps; the other sites alongside."""
+    probe_ms = {}
+    for name, sid in SITES.items():
+        plan.probe(sid)
+        tot, n = 0.0, 0
+        for _ in range(3):
+            step()
+            ms_k, nl = plan.probe_read()
+            tot += ms_k
+            n += nl
+        probe_ms[name] = (tot / max(n, 1), n / 3)
+    plan.probe(0)
+    dom = "agg_l0"
+    per_launch_ms, launches_per_step = probe_ms[dom]
+    ab = alg_bytes(dom, info, cfg, mode, info["n_groups"]) if cfg.aggr == "mean" else None
+    if ab is None:
+        return None
+    achieved = ab / (per_launch_ms * 1e-3) / 1e9
+    return {"kernel": "k_agg_mean_g4 (layer-0 mean aggregation)", "bound": "hbm", "achieved": achieved,
+            "peak": peaks["hbm_gbs"], "unit": "GB/s", "frac": achieved / peaks["hbm_gbs"],
+            "traffic": load_traffic(dom, key), "alg_bytes_per_launch": ab,
+            "alg_bytes_formula": "4E + 8(n_dst+1) + s*F*n_src + s*F*n_dst (SURVEY §8(d), distinct sources)",
+            "avg_launch_ms": per_launch_ms, "launches_per_step": launches_per_step, "peak_source": peak_src,
+            "share_of_step": per_launch_ms * launches_per_step / ms,
+            "other_sites_ms_per_step": {k: v[0] * v[1] for k, v in probe_ms.items()}}
+
+
+def cpu_threads(args):
+    n = args.cpu_threads or len(os.sched_getaffinity(0))
+    return max(1, n)
+
+
+def cpu_baseline(args, cfg, ds, scale):
+    """The float64 oracle as it stands on the host cores: one bounded sample per thread (the first S
+    outputs of micro-batch t of a range split of the outputs), threads in parallel (ctypes releases the
+    GIL for the C call); value = the samples' edges / wall time."""
+    import oracle
+    from concurrent.futures import ThreadPoolExecutor
+    nt = cpu_threads(args)
+    jobs = []
+    for t in range(nt):
+        rpart, desc, redges = reference_sample(args, cfg, ds, args.cpu_sample_outputs, mb=t % max(args.K, 1))
+        oblocks, ofeats = oracle_inputs(cfg, ds, rpart)
+        jobs.append((rpart, oblocks, ofeats, redges))
+    pr = synth_params(cfg).astype(np.float64)
+
+    def run(j):
+        rpart, oblocks, ofeats, _ = j
+        oracle.step(cfg.dims, cfg.aggr, args.mode == "bf16", oblocks, rpart, 2, [0], pr, ofeats, ds.labels, scale)
+    tc = time.perf_counter()
+    with ThreadPoolExecutor(nt) as ex:
+        list(ex.map(run, jobs))
+    dt = time.perf_counter() - tc
+    edges = sum(j[3] for j in jobs)
+    return {"value": edges / dt, "unit": "edges/s", "cores": nt, "kind": "oracle",
+            "sample": f"{nt} samples in parallel, each {args.cpu_sample_outputs} outputs of one micro-batch "
+                      f"(K={args.K} range split) through {cfg.L} layers, extraction+fwd+bwd in float64; "
+                      f"{edges} edges", "seconds": dt}
 
 
 def create_plan(B, ctx, model, dev_blocks, dpart, K, my_k, group, flags):

@@ -166,9 +166,16 @@ BETTY_API void betty_saved_free(betty_ctx* ctx, betty_saved* saved);
  * this rank's).  A group is the block-diagonal union of its micro-batches:
  * per-micro-batch dedupe / relabel / numerics are unchanged; memory grows
  * with the group.  flags: BETTY_PLAN_GRAPH captures the step as a CUDA graph
- * on first use; BETTY_PLAN_REG rebuilds the REG (a1) inside every step. */
+ * on first use; BETTY_PLAN_REG rebuilds the REG (a1) inside every step;
+ * BETTY_PLAN_FRESH makes every step derive everything it needs from the
+ * current contents of the bound full-batch buffers (indptr / indices /
+ * src_gid and part): the full-batch CSCs the extraction filters and the
+ * REG's CSC are rebuilt in the step (duplicate edges flagged) instead of
+ * once at plan creation -- the mode for a batch re-copied or resampled into
+ * the same buffers every step (sizes must stay within the plan's, checked on
+ * the device: BETTY_EOVERFLOW at the next synchronising call). */
 typedef struct betty_plan betty_plan;
-enum { BETTY_PLAN_GRAPH = 1, BETTY_PLAN_REG = 2 };
+enum { BETTY_PLAN_GRAPH = 1, BETTY_PLAN_REG = 2, BETTY_PLAN_FRESH = 4 };
 typedef struct {
     int32_t n_groups;            /* launch groups per step */
     int32_t L;

@@ -20,7 +20,7 @@ from ._lib import LIB_PATH  # noqa: F401
 
 AGGR = {"mean": 0, "pool": 1}
 GEMM = {"fp32": 0, "bf16": 1}
-PLAN_GRAPH, PLAN_REG = 1, 2
+PLAN_GRAPH, PLAN_REG, PLAN_FRESH = 1, 2, 4
 
 
 class BettyError(RuntimeError):

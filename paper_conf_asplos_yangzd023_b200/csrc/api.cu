@@ -118,6 +118,7 @@ extern "C" void betty_ctx_destroy(betty_ctx* c) {
         cudaFree(ln.big_count);
         cudaFree(ln.big_list);
     }
+    for (void* p : c->retired) ctx_free(c, p, 0);
     cudaFree(c->dev_err);
     cudaDeviceSynchronize();
     delete c;
@@ -323,6 +324,10 @@ static bool alloc_reg_phase1(Arena& A, const betty_block* ob, int64_t r0, int64_
     a.off = A.get<int64_t>(n + 1);
     a.ub_total_dev = R->cnt + 3;
     a.row_nnz = A.get<int64_t>(n);
+    // hub-row scratch: a bitmap over the output ids and its popcount prefix per CTA of k_reg_rows_cta
+    a.hub_words = (ob->n_dst + 31) / 32 + 1;
+    a.hub_bits = A.get<uint32_t>(a.hub_words * A.c->num_sms);
+    a.hub_pre = A.get<int32_t>(a.hub_words * A.c->num_sms);
     return A.ok;
 }
 
@@ -488,8 +493,13 @@ struct betty_plan {
     std::vector<std::vector<int32_t>> groups;
     int32_t* d_ks = nullptr;
     Arena* arena = nullptr;
+    Arena* reg_arena = nullptr;   // the in-step REG's buffers (re-sized by betty_plan_set_reg_rows)
     ExtractSet X;
     uint32_t csc_mask = 0;
+    // BETTY_PLAN_FRESH: per layer in csc_mask, the device counts and scratch of the in-step rebuild of
+    // the full-batch CSC
+    std::vector<int64_t*> fcsc_cnt;
+    std::vector<int32_t*> fcsc_tmp;
     SageBufs sb;
     std::vector<BlockView> views;
     // REG inside the step
@@ -533,6 +543,16 @@ static void step_body(betty_ctx* c, betty_plan* p, const float* params, const vo
         c->lane = 0;
         cudaEventRecord(p->ev_join, p->side);
     };
+    if (p->flags & BETTY_PLAN_FRESH) {        // full-batch CSCs from the current block buffers
+        for (int l = 0; l < p->L; ++l) {
+            if (!(p->csc_mask >> l & 1)) continue;
+            const ExtractFull& fb = p->full[l];
+            csr_transpose(c, fb.indptr, fb.nbr, p->fcsc_cnt[l], p->fcsc_cnt[l] + 1, p->fcsc_cnt[l] + 2,
+                          std::max<int64_t>(fb.n_dst, 1), std::max<int64_t>(fb.n_src, 1),
+                          std::max<int64_t>(fb.n_edges, 1), (int64_t*)fb.t_indptr, (int32_t*)fb.t_nbr,
+                          p->fcsc_tmp[l], l == p->L - 1, s);
+        }
+    }
     const int fp = p->groups.empty() ? 0 : reg_fork_point();
     if (p->with_reg && fp == 0) fork_reg();
     sage_prep(c, p->m, p->sb, params, s);
@@ -596,7 +616,12 @@ __global__ void k_max_deg(const int64_t* __restrict__ indptr, int64_t n, int* ou
 // Size and allocate the in-step REG of output rows [r0, r1) (phases 1-2 run once here, synchronising).
 static betty_status plan_reg_setup(betty_ctx* c, betty_plan* p, const betty_block* ob, int64_t r0, int64_t r1,
                                    cudaStream_t s) {
-    Arena& A = *p->arena;
+    // the REG's buffers live in their own arena: a new row share releases the previous share's
+    // buffers first (set_reg_rows used to leak the all-rows REG scratch in the plan arena)
+    if (p->reg_arena) { p->reg_arena->s = s; p->reg_arena->release(); p->reg_arena->bytes = 0; p->reg_arena->ok = true; }
+    else p->reg_arena = new Arena{c, s};
+    p->with_reg = false;
+    Arena& A = *p->reg_arena;
     c->lane = 1;            // size the side lane's scan scratch with the REG's own calls
     RegBufs R;
     if (!alloc_reg_phase1(A, ob, r0, r1, &R, s)) { c->lane = 0; return fail(c, BETTY_ENOMEM, "plan: REG alloc"); }
@@ -623,11 +648,11 @@ static betty_status plan_reg_setup(betty_ctx* c, betty_plan* p, const betty_bloc
     // The output block's CSC (built and duplicate-checked by phase 1 above) belongs to the plan's
     // full batch, like the extraction's full-batch CSC: the step's rebuild reuses it and runs the
     // SpGEMM proper (expansion, sort, run-length encode, compaction) over the rank's rows.
-    R.a.csc_ready = true;
+    R.a.csc_ready = !(p->flags & BETTY_PLAN_FRESH);    // FRESH: the step rebuilds it from the block
     p->R = R;
     p->with_reg = true;
     p->info.reg_nnz = nnz;
-    p->info.arena_bytes = A.bytes + p->sb.bytes;
+    p->info.arena_bytes = p->arena->bytes + A.bytes + p->sb.bytes;
     return BETTY_OK;
 }
 
@@ -729,6 +754,8 @@ extern "C" betty_status betty_plan_create(betty_ctx* c, const betty_model* model
     }
     if (m.layers[0].kind == KIND_AGG) p->X.layers[0].egid = A.get<int32_t>(ce[0]);   // layer-0 gather by gid
     // full-batch CSC of the layers whose micro-batch CSC is built every step (filtered from it)
+    p->fcsc_cnt.assign(L, nullptr);
+    p->fcsc_tmp.assign(L, nullptr);
     for (int l = 0; l < L; ++l) {
         if (!(p->csc_mask >> l & 1)) continue;
         const betty_block& fb = full[l];
@@ -745,6 +772,8 @@ extern "C" betty_status betty_plan_create(betty_ctx* c, const betty_model* model
         if ((st = sync_check(c, s))) { betty_plan_destroy(c, p); return st; }
         p->full[l].t_indptr = fti;
         p->full[l].t_nbr = ftn;
+        p->fcsc_cnt[l] = hc;
+        p->fcsc_tmp[l] = tc;
     }
     if (!A.ok) {
         betty_plan_destroy(c, p);
@@ -805,7 +834,7 @@ extern "C" betty_status betty_plan_create(betty_ctx* c, const betty_model* model
         cudaGetLastError();
         cudaStreamDestroy(cs2);
     }
-    p->info.arena_bytes = A.bytes + p->sb.bytes;
+    p->info.arena_bytes = A.bytes + (p->reg_arena ? p->reg_arena->bytes : 0) + p->sb.bytes;
     if ((st = sync_check(c, s))) { betty_plan_destroy(c, p); return st; }
     *out = p;
     return BETTY_OK;
@@ -828,6 +857,7 @@ extern "C" void betty_plan_destroy(betty_ctx* c, betty_plan* p) {
     p->probe.destroy();
     sage_free(c, &p->sb, 0);
     if (p->arena) { p->arena->s = 0; p->arena->release(); delete p->arena; }
+    if (p->reg_arena) { p->reg_arena->s = 0; p->reg_arena->release(); delete p->reg_arena; }
     cudaDeviceSynchronize();
     delete p;
 }

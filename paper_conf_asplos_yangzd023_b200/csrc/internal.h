@@ -29,6 +29,7 @@ struct betty_ctx {
     int lane = 0;                                // the set launches issued now use
     Lane& L() { return lanes[lane]; }
     int* dev_err = nullptr;                      // device-side error flags (see betty::DEVERR_*)
+    std::vector<void*> retired;                  // outgrown scratch still referenced by captured graphs
 };
 
 namespace betty {

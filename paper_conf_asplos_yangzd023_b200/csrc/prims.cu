@@ -133,8 +133,11 @@ __global__ void __launch_bounds__(SCAN_THREADS) k_scan(const Ld in, int64_t* __r
 void ensure_scan_scratch(betty_ctx* c, int64_t n_cap, cudaStream_t s) {
     const int64_t tiles = (n_cap + SCAN_TILE - 1) / SCAN_TILE + 1;
     if (tiles > c->L().scan_status_cap) {
-        // growing is only legal outside graph capture; plan creation sizes it first
-        if (c->L().scan_status) ctx_free(c, c->L().scan_status, s);
+        // growing is only legal outside graph capture; plan creation sizes it first.  A plan's
+        // instantiated CUDA graph holds the old pointer by value, so the old buffer is retired (kept
+        // until the context is destroyed), never freed here (a later larger call must not turn an
+        // existing graph's scratch into freed memory)
+        if (c->L().scan_status) c->retired.push_back(c->L().scan_status);
         const int64_t cap = tiles * 2 + 1024;
         c->L().scan_status = (unsigned long long*)ctx_alloc(c, sizeof(unsigned long long) * cap, s);
         cudaMemsetAsync(c->L().scan_status, 0, sizeof(unsigned long long) * cap, s);

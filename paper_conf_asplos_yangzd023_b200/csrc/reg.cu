@@ -12,7 +12,12 @@
 //   3. exclusive scan of ub -> a temporary slot per product
 //   4. per row: expand the candidates j (from the columns of its sources,
 //      skipping j = i), sort them (warp bitonic for ub <= 256, CTA bitonic
-//      in shared memory up to 32768), run-length encode -> (j, c_ij) ascending
+//      in shared memory up to 32768), run-length encode -> (j, c_ij) ascending;
+//      hub rows (ub > 32768, no degree bound in Eq. 2-4) take a CTA each: the
+//      candidates (expanded in place in the row's global slot) set bits of a
+//      bitmap over the output ids, a popcount prefix over its words ranks
+//      every distinct j (ascending by construction), and c_ij is counted by
+//      integer atomics into its rank's slot -- no sort, exact
 //   5. scan of the per-row counts -> indptr, compaction into col / w
 // Every step is integer and order-independent, so the result is bit-exact.
 #include <climits>
@@ -43,8 +48,7 @@ __global__ void k_reg_ub(const int64_t* __restrict__ indptr, const int32_t* __re
         s = warp_sum(s);
         if (lane == 0) {
             ub[i] = s;
-            if (s > REG_WARP_MAX) {
-                if (s > REG_CTA_MAX) atomicOr(dev_err, DEVERR_OVERFLOW);
+            if (s > REG_WARP_MAX) {                     // CTA rows (hub rows included)
                 const int k = atomicAdd(big_cnt, 1);
                 if (k < big_cap) big[k] = i; else atomicOr(dev_err, DEVERR_OVERFLOW);
             }
@@ -258,6 +262,81 @@ __global__ void __launch_bounds__(256) k_reg_rows_warp(const int64_t* __restrict
     }
 }
 
+// exclusive scan of v over the CTA (blockDim.x a multiple of 32, <= 1024); returns the prefix,
+// *total gets the sum (to every thread)
+__device__ __forceinline__ int64_t cta_excl_scan(int64_t v, int64_t* total, int64_t* s_w) {
+    const int lane = lane_id(), w = warp_id(), nw = blockDim.x >> 5;
+    int64_t incl = v;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        const int64_t y = __shfl_up_sync(0xffffffffu, incl, d);
+        if (lane >= d) incl += y;
+    }
+    if (lane == 31) s_w[w] = incl;
+    __syncthreads();
+    if (w == 0) {
+        int64_t x = lane < nw ? s_w[lane] : 0, xi = x;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const int64_t y = __shfl_up_sync(0xffffffffu, xi, d);
+            if (lane >= d) xi += y;
+        }
+        if (lane < nw) s_w[lane] = xi - x;
+        if (lane == 31) s_w[32] = xi;
+    }
+    __syncthreads();
+    const int64_t r = s_w[w] + incl - v;
+    *total = s_w[32];
+    __syncthreads();
+    return r;
+}
+
+// One hub row (ub > REG_CTA_MAX) by the whole CTA: the candidates are expanded into the row's
+// global slot cand[0, u), marked in a bitmap over the output ids, ranked by a popcount prefix, and
+// counted into w[rank] by integer atomics; finally the distinct ids overwrite cand ascending.
+__device__ void reg_hub_row(const int64_t* __restrict__ indptr, const int32_t* __restrict__ idx,
+                            const int64_t* __restrict__ t_indptr, const int32_t* __restrict__ t_idx, int64_t i,
+                            int64_t row0, int64_t u, int32_t* cand, int32_t* wout, uint32_t* bits, int32_t* pre,
+                            int64_t W, int* s_pre, int64_t* s_cb, int64_t* s_w, int64_t* nnz_out) {
+    const int tid = threadIdx.x, nthr = blockDim.x;
+    reg_expand(indptr, idx, t_indptr, t_idx, i, row0, cand, tid, nthr, s_pre, s_cb);
+    for (int64_t q = tid; q < W; q += nthr) bits[q] = 0u;
+    for (int64_t q = tid; q < u; q += nthr) wout[q] = 0;
+    __syncthreads();
+    for (int64_t q = tid; q < u; q += nthr) {
+        const int32_t j = cand[q];
+        atomicOr(&bits[j >> 5], 1u << (j & 31));
+    }
+    __syncthreads();
+    int64_t run = 0;
+    for (int64_t base = 0; base < W; base += nthr) {
+        const int64_t q = base + tid;
+        const int64_t v = q < W ? __popc(bits[q]) : 0;
+        int64_t tot;
+        const int64_t ex = cta_excl_scan(v, &tot, s_w);
+        if (q < W) pre[q] = (int32_t)(run + ex);
+        run += tot;
+    }
+    __syncthreads();
+    for (int64_t q = tid; q < u; q += nthr) {
+        const int32_t j = cand[q];
+        const uint32_t m = bits[j >> 5] & ((1u << (j & 31)) - 1u);
+        atomicAdd(&wout[pre[j >> 5] + __popc(m)], 1);
+    }
+    __syncthreads();
+    for (int64_t q = tid; q < W; q += nthr) {
+        uint32_t m = bits[q];
+        int32_t r = pre[q];
+        while (m) {
+            const int b = __ffs(m) - 1;
+            cand[r++] = (int32_t)(q * 32 + b);
+            m &= m - 1u;
+        }
+    }
+    if (tid == 0) *nnz_out = run;
+    __syncthreads();
+}
+
 __global__ void __launch_bounds__(1024) k_reg_rows_cta(const int64_t* __restrict__ indptr,
                                                        const int32_t* __restrict__ idx,
                                                        const int64_t* __restrict__ t_indptr,
@@ -265,16 +344,24 @@ __global__ void __launch_bounds__(1024) k_reg_rows_cta(const int64_t* __restrict
                                                        const int64_t* __restrict__ ub, const int64_t* __restrict__ off,
                                                        const int64_t* big, const int* big_cnt,
                                                        int32_t* __restrict__ tcol, int32_t* __restrict__ tw,
-                                                       int64_t* __restrict__ nnz) {
+                                                       int64_t* __restrict__ nnz, uint32_t* hub_bits, int32_t* hub_pre,
+                                                       int64_t hub_words, int* dev_err) {
     extern __shared__ int32_t sbuf[];
     __shared__ int s_cnt;
     __shared__ int s_pre[33];
     __shared__ int64_t s_cb[32];
+    __shared__ int64_t s_w[33];
     const int nb = *big_cnt;
     for (int t = blockIdx.x; t < nb; t += gridDim.x) {
         const int64_t i = big[t];
         const int64_t u = ub[i];
-        if (u > REG_CTA_MAX) { if (threadIdx.x == 0) nnz[i] = 0; continue; }
+        if (u > REG_CTA_MAX) {
+            if (!hub_bits) { if (threadIdx.x == 0) { nnz[i] = 0; atomicOr(dev_err, DEVERR_OVERFLOW); } continue; }
+            reg_hub_row(indptr, idx, t_indptr, t_idx, i, row0, u, tcol + off[i], tw + off[i],
+                        hub_bits + blockIdx.x * hub_words, hub_pre + blockIdx.x * hub_words, hub_words, s_pre, s_cb,
+                        s_w, &nnz[i]);
+            continue;
+        }
         reg_expand(indptr, idx, t_indptr, t_idx, i, row0, sbuf, threadIdx.x, blockDim.x, s_pre, s_cb);
         int P = 1024;
         while (P < u) P <<= 1;
@@ -324,7 +411,8 @@ void reg_phase2(betty_ctx* c, const RegArgs& a, cudaStream_t s) {
     k_reg_rows_warp<<<gw, 256, 0, s>>>(a.indptr, a.idx, a.t_indptr, a.t_idx, a.n_rows_dev, a.row0, a.ub, a.off, a.tcol,
                                        a.tw, a.row_nnz);
     k_reg_rows_cta<<<c->num_sms, 1024, REG_CTA_MAX * 4, s>>>(a.indptr, a.idx, a.t_indptr, a.t_idx, a.row0, a.ub, a.off,
-                                                            c->L().big_list, c->L().big_count, a.tcol, a.tw, a.row_nnz);
+                                                            c->L().big_list, c->L().big_count, a.tcol, a.tw, a.row_nnz,
+                                                            a.hub_bits, a.hub_pre, a.hub_words, c->dev_err);
     scan_i64(c, a.row_nnz, a.out_indptr, a.n_rows_dev, 0, a.rows_cap, a.nnz_total_dev, s);
 }
 

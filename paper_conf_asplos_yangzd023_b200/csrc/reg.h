@@ -32,6 +32,11 @@ struct RegArgs {
     int64_t* row_nnz;           // [rows_cap]
     int64_t* out_indptr;        // [rows_cap+1]
     int64_t* nnz_total_dev;
+    // hub rows (more than REG_CTA_MAX candidate products): one CTA per row over a bitmap of the
+    // output ids, per-CTA scratch of hub_words words (bitmap + popcount prefix) x num_sms CTAs
+    uint32_t* hub_bits = nullptr;
+    int32_t* hub_pre = nullptr;
+    int64_t hub_words = 0;
 };
 // phase 1: CSC + product counts (ub) + their scan (ub_total known after it)
 void reg_phase1(betty_ctx* c, const RegArgs& a, cudaStream_t s);

@@ -18,7 +18,7 @@ import torch
 
 import oracle
 import synth
-from tests.helpers import assert_close, assert_grad_close
+from tests.helpers import assert_close, assert_grad_close, explain_relu_flips
 
 pytestmark = pytest.mark.gpu
 
@@ -132,14 +132,21 @@ def test_sampled_micro_batch_full_size(B, ctx, c3):
 
 @pytest.mark.parametrize("mode,rtol", [("fp32", 1e-5), ("bf16", 2e-2)])
 def test_whole_micro_batch_full_size(B, ctx, c3, mode, rtol):
-    """One WHOLE micro-batch of the bench's K = 32 REG partition (micro-batch 0: ~6 k outputs, ~1 M
+    """One WHOLE micro-batch of the bench's K = 32 REG partition (micro-batch 0: ~6 k outputs, ~0.9 M
     sampled edges over both layers) through the fused step (graph replay, in-step REG) on the
-    full-size graph and feature table, against oracle_step on the same micro-batch: per parameter
-    tensor within 1e-5 (fp32) / 2e-2 (bf16), loss likewise (reading #18)."""
+    full-size graph and feature table, against the oracle on the same micro-batch: per parameter
+    tensor within 1e-5 (fp32) / 2e-2 (bf16), loss likewise (reading #18).  In fp32 the ~20 M hidden
+    ReLU decisions include some that finite precision takes either way (|S| <= tau M); the layer-0
+    gradient is compared after explaining such flips (reading #24, tests/helpers.explain_relu_flips)."""
     cfg, ds, dev, reg, part = c3
     params = synth.init_params(cfg.dims, cfg.aggr, seed=cfg.seeds["init"])
-    og, ol = oracle.step(cfg.dims, cfg.aggr, mode == "bf16", ds.blocks, part, K, [0], params, ds.feats,
-                         ds.labels, 1.0 / cfg.n_out)
+    mb = oracle.extract(ds.blocks, part, K, 0)
+    if mode == "fp32":
+        og, ol, ties, found = oracle.sage_ties(cfg.dims, cfg.aggr, False, mb, params, ds.feats, ds.labels,
+                                               1.0 / cfg.n_out, tau=2.0 ** -17)
+        assert found == len(ties["v"])
+    else:
+        og, ol, _ = oracle.sage(cfg.dims, cfg.aggr, True, mb, params, ds.feats, ds.labels, 1.0 / cfg.n_out)
     model = B.Model(cfg.dims, cfg.aggr, mode, mode)
     plan = B.betty_plan_create(ctx, model, dev, torch.as_tensor(part).cuda(), K, [0], group=0,
                                flags=B.PLAN_GRAPH | B.PLAN_REG)
@@ -155,7 +162,12 @@ def test_whole_micro_batch_full_size(B, ctx, c3, mode, rtol):
         loss = torch.zeros(1, device="cuda")
         B.betty_step(ctx, plan, P, X, Y, 1.0 / cfg.n_out, grad, loss)
         B.betty_sync_check(ctx)
-        assert_grad_close(grad.cpu().numpy(), og, cfg.dims, cfg.aggr, rtol, f"{mode} grad rep {rep}")
+        g = grad.cpu().numpy()
+        if mode == "fp32":
+            flips = explain_relu_flips(g, og, ties, mb, ds.feats, cfg.dims, cfg.aggr, rtol, f"{mode} rep {rep}")
+            print(f"fp32 whole micro-batch: {found} ReLU decisions within tau, {flips} taken the other way")
+        else:
+            assert_grad_close(g, og, cfg.dims, cfg.aggr, rtol, f"{mode} grad rep {rep}")
         assert loss.item() == pytest.approx(ol, rel=rtol)
     plan.free()
 

@@ -117,6 +117,23 @@ def test_plan_reg_rows(B, ctx):
     plan.free()
 
 
+@pytest.mark.parametrize("n,m,d", [(2000, 150, 60), (600, 40, 30)])
+def test_reg_hub_rows(B, ctx, n, m, d):
+    """Hub rows: every output samples d of m shared sources, so each column has ~n d / m outputs and a
+    row has ~d (n d / m - 1) candidate products -- (2000, 150, 60): ~48 k > 32768, the bitmap-rank
+    path (no degree bound in Eq. 2-4); (600, 40, 30): ~13 k, the CTA sort path.
+    A mixed block (hub rows + short rows) as well.  Bit-exact against the oracle."""
+    rng = np.random.default_rng(n + m)
+    rows = [np.sort(rng.choice(m, size=d, replace=False)).astype(np.int32) for _ in range(n)]
+    # a few short rows on private sources (warp path) in the same block
+    rows += [np.array([m + k], np.int32) for k in range(50)]
+    indptr = np.concatenate([[0], np.cumsum([len(r) for r in rows])]).astype(np.int64)
+    idx = np.concatenate(rows).astype(np.int32)
+    host = synth.Block(len(rows), m + 50, indptr, idx, np.arange(m + 50, dtype=np.int32))
+    nnz = reg_equal(B, ctx, B.blocks_to_device([host])[0], host)
+    assert nnz > 0
+
+
 def test_reg_rejects_duplicate_edges(B, ctx):
     blk = B.Block(2, 3, torch.tensor([0, 2, 3], dtype=torch.int64, device="cuda"),
                   torch.tensor([1, 1, 2], dtype=torch.int32, device="cuda"),
