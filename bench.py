@@ -58,7 +58,7 @@ def parse():
                    help="skip the nested paper-precision (fp32, 3xTF32 GEMMs) measurement of a bf16 run")
     p.add_argument("--cpu-threads", type=int, default=0, help="cpu_baseline / reference threads (0: all cores)")
     p.add_argument("--cpu-sample-outputs", type=int, default=4096, help="cpu_baseline sample (~10 s)")
-    p.add_argument("--ref-sample-outputs", type=int, default=1024, help="--impl reference per-step sample")
+    p.add_argument("--ref-sample-outputs", type=int, default=512, help="--impl reference per-step sample (per core)")
     p.add_argument("--scale", type=float, default=1.0, help="shrink the graph (debug only)")
     p.add_argument("--json-out", default=None)
     p.add_argument("--sim-world", type=int, default=0, help="(study) run rank 0's share of an N-rank job on one GPU")

@@ -88,7 +88,9 @@ typedef struct {
     int32_t* w;
 } betty_csr;
 
-enum { BETTY_AGGR_MEAN = 0, BETTY_AGGR_POOL = 1 };
+/* aggregators of Table 1: mean h_N = (1/D_v) sum_u h_u; pool max_u ReLU(W_pool h_u +
+ * b_pool); sum h_N = sum_u h_u (mean without 1/D_v, the same SAGEConv form and project-first rule) */
+enum { BETTY_AGGR_MEAN = 0, BETTY_AGGR_POOL = 1, BETTY_AGGR_SUM = 2 };
 enum { BETTY_GEMM_FP32 = 0, BETTY_GEMM_BF16 = 1 };
 enum { BETTY_FEAT_FP32 = 0, BETTY_FEAT_BF16 = 1 };
 
@@ -97,7 +99,10 @@ enum { BETTY_FEAT_FP32 = 0, BETTY_FEAT_BF16 = 1 };
  * Parameters are one flat fp32 vector; per layer l (Fi = dims[l], Fo = dims[l+1]):
  *   pool only: W_pool [Fi x Fi], b_pool [Fi]
  *   W_self [Fi x Fo], W_neigh [Fi x Fo], b [Fo]          (row-major, x . W)
- * gemm: FP32 = fp32 SIMT everywhere (no TF32); BF16 = GEMM operands in bf16,
+ * gemm: FP32 = fp32 operands; the products run on tcgen05 as 3xTF32 (hi*hi +
+ * lo*hi + hi*lo of an RN tf32 split, fp32 accumulation with the small terms
+ * in their own accumulator and dW totals drained every 64 nodes: ~fp32
+ * accuracy, never plain TF32; env BETTY_FP32_SIMT=1 selects SIMT FFMA); BF16 = GEMM operands in bf16,
  * fp32 accumulation, aggregation / loss / gradients fp32, hidden activations
  * stored bf16 (reading #17).  feat_dtype says how `feats` is stored. */
 typedef struct {

@@ -73,7 +73,7 @@ def lib():
 
 def _aggr(aggr: str) -> int:
     """aggregator code of oracle.c: 0 mean, 1 pool (Table 1)"""
-    return {"mean": 0, "pool": 1}[aggr]
+    return {"mean": 0, "pool": 1, "sum": 2}[aggr]
 
 
 def _p(a: Optional[np.ndarray]):

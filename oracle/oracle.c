@@ -351,7 +351,7 @@ static mat param_mat(const double* params, int64_t off, int64_t r, int64_t c, in
  *
  * params: float64 in the flat layout (the caller widens fp32 parameters;
  * float64 lets the finite-difference pins perturb them exactly).
- * aggr: 0 mean, 1 pool.  force_form: -1 DGL rule, 0 aggregate-first,
+ * aggr: 0 mean, 1 pool, 2 sum.  force_form: -1 DGL rule, 0 aggregate-first,
  * 1 project-first (mean only; for the tests that pin the two forms equal).
  * logits_out: optional [n_dst(L-1) x dims[L]].  Returns 0.
  */
@@ -359,6 +359,9 @@ int oracle_sage(int L, const int32_t* dims, int aggr, int bf16, int force_form, 
                 const double* params, const float* feats, int64_t ld, const int32_t* labels, double loss_scale,
                 double* grad, double* loss, double* logits_out) {
     const int pool = (aggr == 1);
+    /* Table 1 "Sum": h_N = sum_u h_u, i.e. the mean without 1/D_v; the same
+     * SAGEConv form and project-first rule (reading #11) */
+    const int sum = (aggr == 2);
     mat* H = (mat*)calloc((size_t)L + 1, sizeof(mat));       /* H[l] = input of layer l, [n_src(l) x dims[l]] */
     mat* Aagg = (mat*)calloc((size_t)L, sizeof(mat));        /* aggregated neighbour features (or D+P(XWn)) */
     mat* Zp = (mat*)calloc((size_t)L, sizeof(mat));          /* pool pre-activation */
@@ -397,7 +400,7 @@ int oracle_sage(int L, const int32_t* dims, int aggr, int bf16, int force_form, 
                     int64_t deg = B->indptr[v + 1] - B->indptr[v];
                     for (int64_t e = B->indptr[v]; e < B->indptr[v + 1]; ++e)
                         for (int64_t f = 0; f < fi; ++f) AT(Aagg[l], v, f) += AT(X, B->indices[e], f);
-                    for (int64_t f = 0; f < fi && deg > 0; ++f) AT(Aagg[l], v, f) /= (double)deg;
+                    for (int64_t f = 0; f < fi && deg > 0 && !sum; ++f) AT(Aagg[l], v, f) /= (double)deg;
                 }
                 mm_acc(&S, &Aagg[l], 0, &Wn, 0, bf16);      /* + A W_n */
             } else {
@@ -408,7 +411,7 @@ int oracle_sage(int L, const int32_t* dims, int aggr, int bf16, int force_form, 
                     int64_t deg = B->indptr[v + 1] - B->indptr[v];
                     for (int64_t e = B->indptr[v]; e < B->indptr[v + 1]; ++e)
                         for (int64_t f = 0; f < fo; ++f) AT(Aagg[l], v, f) += AT(Z, B->indices[e], f);
-                    for (int64_t f = 0; f < fo && deg > 0; ++f) AT(Aagg[l], v, f) /= (double)deg;
+                    for (int64_t f = 0; f < fo && deg > 0 && !sum; ++f) AT(Aagg[l], v, f) /= (double)deg;
                 }
                 for (int64_t t = 0; t < nd * fo; ++t) S.a[t] += Aagg[l].a[t];
                 mat_free(&Z);
@@ -447,7 +450,8 @@ int oracle_sage(int L, const int32_t* dims, int aggr, int bf16, int force_form, 
                 for (int64_t v = 0; v < nd; ++v) {
                     int64_t deg = B->indptr[v + 1] - B->indptr[v];
                     for (int64_t e = B->indptr[v]; e < B->indptr[v + 1]; ++e)
-                        for (int64_t f = 0; f < fo; ++f) AT(Mg, v, f) += AT(Za, B->indices[e], f) / (double)deg;
+                        for (int64_t f = 0; f < fo; ++f)
+                            AT(Mg, v, f) += sum ? AT(Za, B->indices[e], f) : AT(Za, B->indices[e], f) / (double)deg;
                 }
                 mat_free(&Za);
             } else {
@@ -525,7 +529,8 @@ int oracle_sage(int L, const int32_t* dims, int aggr, int bf16, int force_form, 
                 for (int64_t v = 0; v < nd; ++v) {           /* dX += P^T D+ dA */
                     int64_t deg = B->indptr[v + 1] - B->indptr[v];
                     for (int64_t e = B->indptr[v]; e < B->indptr[v + 1]; ++e)
-                        for (int64_t f = 0; f < fi; ++f) AT(dX, B->indices[e], f) += AT(dA, v, f) / (double)deg;
+                        for (int64_t f = 0; f < fi; ++f)
+                            AT(dX, B->indices[e], f) += sum ? AT(dA, v, f) : AT(dA, v, f) / (double)deg;
                 }
                 mat_free(&dA);
             }
@@ -534,7 +539,8 @@ int oracle_sage(int L, const int32_t* dims, int aggr, int bf16, int force_form, 
             for (int64_t v = 0; v < nd; ++v) {
                 int64_t deg = B->indptr[v + 1] - B->indptr[v];
                 for (int64_t e = B->indptr[v]; e < B->indptr[v + 1]; ++e)
-                    for (int64_t f = 0; f < fo; ++f) AT(dZ, B->indices[e], f) += AT(dS, v, f) / (double)deg;
+                    for (int64_t f = 0; f < fo; ++f)
+                        AT(dZ, B->indices[e], f) += sum ? AT(dS, v, f) : AT(dS, v, f) / (double)deg;
             }
             mm_acc(&gWn, &X, 1, &dZ, 0, bf16);               /* dW_n += X^T dZ */
             if (l > 0) mm_acc(&dX, &dZ, 0, &Wn, 1, bf16);    /* dX += dZ W_n^T */

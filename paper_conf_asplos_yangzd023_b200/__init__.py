@@ -18,7 +18,7 @@ import torch
 from . import _lib as L
 from ._lib import LIB_PATH  # noqa: F401
 
-AGGR = {"mean": 0, "pool": 1}
+AGGR = {"mean": 0, "pool": 1, "sum": 2}
 GEMM = {"fp32": 0, "bf16": 1}
 PLAN_GRAPH, PLAN_REG, PLAN_FRESH = 1, 2, 4
 

@@ -106,7 +106,7 @@ __global__ void __launch_bounds__(256) k_agg_mean_xa(const Tin* __restrict__ X, 
                                                      const int64_t* __restrict__ indptr, const int64_t* cnt,
                                                      const int64_t* __restrict__ otab, int Fi, int Fp,
                                                      Tout* __restrict__ XA, int64_t ldxa, int hint, int vlo, int vhi,
-                                                     unsigned* ctr) {
+                                                     unsigned* ctr, int sum) {
     using VI = Vec<Tin>;
     constexpr int VW = VI::N;
     constexpr int RPW = 32 / LPR;
@@ -198,7 +198,7 @@ __global__ void __launch_bounds__(256) k_agg_mean_xa(const Tin* __restrict__ X, 
         Meta nxt;
         meta(nbase + wib * RPW, nxt);       // next rows' meta overlaps the gather
         Tout* out = XA + cur.v * ldxa;
-        const float inv = n > 0 ? 1.0f / (float)n : 0.0f;
+        const float inv = n > 0 ? (sum ? 1.0f : 1.0f / (float)n) : 0.0f;     // sum aggregator: no 1/D
         if (fast) {
             if (bulk) {
                 if (rowok) { mbar_wait_parity(bar, bph); bph ^= 1u; }
@@ -518,6 +518,7 @@ struct G4Args {
     int Fi, Fp, NV;
     uint32_t row_bytes, grp_bytes, slot_groups, stage_bytes;
     int hint;
+    int sum;                       // sum aggregator (Table 1 "Sum"): no 1/D
 };
 __device__ __forceinline__ void gather4(uint32_t sdst, const CUtensorMap* tm, int32_t r0, int32_t r1, int32_t r2,
                                         int32_t r3, uint64_t* bar, uint64_t pol) {
@@ -712,7 +713,7 @@ __global__ void __launch_bounds__(G4_THREADS, 1) k_agg_mean_g4(const __grid_cons
                     for (int t = 0; t < VW; ++t) so[t] = 0.f;
                     VI::add_raw(so, *(const typename VI::Raw*)(sdat + self_off + (i >> 2) * a.grp_bytes +
                                                                (i & 3) * a.row_bytes + j * 16));
-                    const float inv = e > b ? 1.0f / (float)(e - b) : 0.0f;
+                    const float inv = e > b ? (a.sum ? 1.0f : 1.0f / (float)(e - b)) : 0.0f;
 #pragma unroll
                     for (int t = 0; t < VW; ++t) {
                         const bool in = j * VW + t < a.Fi;
@@ -752,7 +753,7 @@ __global__ void __launch_bounds__(G4_THREADS, 1) k_agg_mean_g4(const __grid_cons
 #pragma unroll
                     for (int t = 0; t < VW; ++t) so[t] = 0.f;
                     VI::add_raw(so, *(const typename VI::Raw*)(sdat + self_off + j * 16));
-                    const float inv = he > hb ? 1.0f / (float)(he - hb) : 0.0f;
+                    const float inv = he > hb ? (a.sum ? 1.0f : 1.0f / (float)(he - hb)) : 0.0f;
 #pragma unroll
                     for (int t = 0; t < VW; ++t) {
                         const bool in = j * VW + t < a.Fi;
@@ -777,14 +778,14 @@ template <typename Tout>
 __global__ void __launch_bounds__(256) k_agg_mean_pf(const float* __restrict__ Y, int64_t ldy,
                                                      const int64_t* __restrict__ indptr,
                                                      const int32_t* __restrict__ idx, const int64_t* cnt, int Fo,
-                                                     int Fop, int relu, Tout* __restrict__ out, int64_t ldo) {
+                                                     int Fop, int relu, Tout* __restrict__ out, int64_t ldo, int sum) {
     const int64_t nd = cnt[0];
     const int lane = lane_id();
     const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
     for (int64_t v = gw; v < nd; v += nw) {
         const int64_t b = indptr[v], e = indptr[v + 1];
-        const float inv = e > b ? 1.0f / (float)(e - b) : 0.0f;
+        const float inv = e > b ? (sum ? 1.0f : 1.0f / (float)(e - b)) : 0.0f;
         for (int c0 = 0; c0 < Fo; c0 += 32) {
             const int c = c0 + lane;
             const bool act = c < Fo;
@@ -848,7 +849,7 @@ __global__ void __launch_bounds__(256) k_csc_mean(const float* __restrict__ dXA,
                 float myinv = 0.f;
                 if (lane < n) {
                     my = t_idx[e0 + lane];
-                    myinv = 1.0f / (float)(indptr[my + 1] - indptr[my]);
+                    myinv = indptr ? 1.0f / (float)(indptr[my + 1] - indptr[my]) : 1.0f;   // null: sum
                 }
                 for (int j = 0; j < n; ++j) {
                     const int32_t v = __shfl_sync(0xffffffffu, my, j);
@@ -898,7 +899,7 @@ __global__ void __launch_bounds__(256) k_csc_mean_v(const float* __restrict__ dX
             float myinv = 0.f;
             if (lane < n) {
                 my = t_idx[e0 + lane];
-                myinv = 1.0f / (float)(indptr[my + 1] - indptr[my]);
+                myinv = indptr ? 1.0f / (float)(indptr[my + 1] - indptr[my]) : 1.0f;       // null: sum
             }
             for (int j0 = 0; j0 < n; j0 += CM_UNR) {
                 float4 x[CM_UNR][VPL];
@@ -996,7 +997,7 @@ __global__ void __launch_bounds__(256) k_csc_mean_g(const float* __restrict__ dX
             float myinv = 0.f;
             if (sub < n) {
                 my = t_idx[e0 + sub];
-                myinv = 1.0f / (float)(indptr[my + 1] - indptr[my]);
+                myinv = indptr ? 1.0f / (float)(indptr[my + 1] - indptr[my]) : 1.0f;       // null: sum
             }
 #pragma unroll
             for (int j0 = 0; j0 < LPR; j0 += UNR) {
@@ -1072,7 +1073,7 @@ __global__ void __launch_bounds__(256) k_csc_pf(const Tin* __restrict__ dS, int6
                 float myinv = 0.f;
                 if (lane < n) {
                     my = t_idx[e0 + lane];
-                    myinv = 1.0f / (float)(indptr[my + 1] - indptr[my]);
+                    myinv = indptr ? 1.0f / (float)(indptr[my + 1] - indptr[my]) : 1.0f;   // null: sum
                 }
                 for (int j = 0; j < n; ++j) {
                     const int32_t v = __shfl_sync(0xffffffffu, my, j);
@@ -1177,7 +1178,7 @@ template <typename Tout, int LPR>
 __global__ void __launch_bounds__(256) k_agg_pf_v(const float* __restrict__ Y, const float* __restrict__ Ys, int64_t ldy,
                                                   const int64_t* __restrict__ indptr,
                                                   const int32_t* __restrict__ idx, const int64_t* cnt, int Fo, int Fop,
-                                                  int relu, Tout* __restrict__ out, int64_t ldo) {
+                                                  int relu, Tout* __restrict__ out, int64_t ldo, int sum) {
     constexpr int RPW = 32 / LPR;
     const int64_t nd = cnt[0];
     const int NV = (Fo + 3) / 4;
@@ -1199,7 +1200,7 @@ __global__ void __launch_bounds__(256) k_agg_pf_v(const float* __restrict__ Y, c
             nb = 0; ne = 0;
             if (vn < nd) { nb = indptr[vn]; ne = indptr[vn + 1]; }
         }
-        const float inv = e > b ? 1.0f / (float)(e - b) : 0.0f;
+        const float inv = e > b ? (sum ? 1.0f : 1.0f / (float)(e - b)) : 0.0f;
         for (int vb = 0; vb < NV; vb += LPR * PF_VPL) {
             float4 acc[PF_VPL];
 #pragma unroll
@@ -1344,13 +1345,14 @@ template <typename K> static int resident_grid(betty_ctx* c, K kernel, int threa
 static bool agg_mean_g4(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const int32_t* srow,
                         const int32_t* erow, const int32_t* emap, const int64_t* indptr, const int64_t* cnt,
                         const int64_t* otab, int Fi, int Fp, int nv, void* XA, bool xa_bf16, int64_t ldxa, int hint,
-                        unsigned* ctr, cudaStream_t s) {
+                        unsigned* ctr, bool sum, cudaStream_t s) {
     const int vw = x_bf16 ? 8 : 4;
     CUtensorMap tm;
     if (!make_gather_map(&tm, X, !x_bf16, (int64_t)nv * vw, (int64_t)INT32_MAX, ldx, nv * vw)) return false;
     G4Args a{};
     a.srow = srow; a.erow = erow; a.emap = emap; a.indptr = indptr; a.cnt = cnt; a.otab = otab;
     a.XA = XA; a.ldxa = ldxa; a.X = X; a.ldx = ldx; a.ctr = ctr; a.Fi = Fi; a.Fp = Fp; a.NV = nv; a.hint = hint;
+    a.sum = sum ? 1 : 0;
     a.row_bytes = (uint32_t)nv * 16u;
     a.grp_bytes = (4u * a.row_bytes + 127u) / 128u * 128u;
     const size_t red_bytes = 0;
@@ -1374,7 +1376,7 @@ static bool agg_mean_g4(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, c
 
 void agg_mean_xa(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const int32_t* srow, const int32_t* erow,
                  const int32_t* emap, const int64_t* indptr, const int64_t* cnt, const int64_t* otab, int64_t rows_cap,
-                 int64_t src_per_mb, int Fi, int Fp, void* XA, bool xa_bf16, int64_t ldxa, cudaStream_t s) {
+                 int64_t src_per_mb, int Fi, int Fp, void* XA, bool xa_bf16, int64_t ldxa, bool sum, cudaStream_t s) {
     const int vw = x_bf16 ? 8 : 4;
     const int nv = (Fi + vw - 1) / vw;
     // Column passes: one micro-batch's gathered rows must stay L2-resident between their
@@ -1392,7 +1394,7 @@ void agg_mean_xa(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const in
     passes = (nv + pv - 1) / pv;
     static const bool g4_off = getenv("BETTY_AGG_G4") && atoi(getenv("BETTY_AGG_G4")) == 0;
     if (!g4_off && passes == 1 && nv * vw <= 256 && agg_mean_g4(c, X, x_bf16, ldx, srow, erow, emap, indptr, cnt, otab,
-                                                                Fi, Fp, nv, XA, xa_bf16, ldxa, hint, ctr, s))
+                                                                Fi, Fp, nv, XA, xa_bf16, ldxa, hint, ctr, sum, s))
         return;
     const int lpr = pv <= 8 ? 8 : (pv <= 16 ? 16 : 32);
     const int64_t warps = (rows_cap + (32 / lpr) - 1) / (32 / lpr);
@@ -1407,18 +1409,20 @@ void agg_mean_xa(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const in
         for (int pz = 0; pz < passes; ++pz) {                                                                   \
             cudaMemsetAsync(ctr, 0, sizeof(unsigned), s);                                                      \
             k_agg_mean_xa<TI, TO, LPR><<<grid, 256, sm, s>>>((const TI*)X, ldx, srow, erow, emap, indptr, cnt,    \
-                no_order ? nullptr : otab, Fi, Fp, (TO*)XA, ldxa, hint, pz * pv, std::min(nv, (pz + 1) * pv), ctr); } }))
+                no_order ? nullptr : otab, Fi, Fp, (TO*)XA, ldxa, hint, pz * pv, std::min(nv, (pz + 1) * pv), ctr, \
+                sum ? 1 : 0); } }))
     if (lpr == 8) { AGG_L(8); } else if (lpr == 16) { AGG_L(16); } else { AGG_L(32); }
 #undef AGG_L
 }
 
 void agg_mean_pf(betty_ctx* c, const float* Y, const float* Ys, int64_t ldy, const int64_t* indptr, const int32_t* idx,
                  const int64_t* cnt, int64_t rows_cap, int Fo, int Fop, bool relu, void* out, bool out_bf16,
-                 int64_t ldo, cudaStream_t s) {
+                 int64_t ldo, bool sum, cudaStream_t s) {
     const int lpr = pick_lpr_vpl((Fo + 3) / 4);
     const int grid = warps_grid(c, (rows_cap + (32 / lpr) - 1) / (32 / lpr));
 #define PF_L(LPR) DISPATCH_ACT(out_bf16, TO, \
-        k_agg_pf_v<TO, LPR><<<grid, 256, 0, s>>>(Y, Ys, ldy, indptr, idx, cnt, Fo, Fop, relu ? 1 : 0, (TO*)out, ldo))
+        k_agg_pf_v<TO, LPR><<<grid, 256, 0, s>>>(Y, Ys, ldy, indptr, idx, cnt, Fo, Fop, relu ? 1 : 0, (TO*)out, ldo, \
+                                                 sum ? 1 : 0))
     if (lpr == 4) { PF_L(4); } else if (lpr == 8) { PF_L(8); } else if (lpr == 16) { PF_L(16); } else { PF_L(32); }
 #undef PF_L
 }

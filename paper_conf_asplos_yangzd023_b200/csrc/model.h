@@ -22,7 +22,8 @@ struct LayerCfg {
 
 struct ModelCfg {
     int L = 0;
-    int aggr = 0;
+    int aggr = 0;             // 0 mean, 1 pool, 2 sum (Table 1)
+    bool sum = false;         // the sum aggregator: mean's kernels without 1/D_v
     bool bf16 = false;        // GEMM operands / hidden activations in bf16
     bool feat_bf16 = false;
     std::vector<int> dims;

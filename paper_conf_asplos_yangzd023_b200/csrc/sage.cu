@@ -19,12 +19,13 @@ namespace betty {
 #define PE(site) do { if (b.probe) b.probe->end((site), s); } while (0)
 
 bool make_model_cfg(int L, int aggr, int gemm, int feat_dtype, const int32_t* dims, ModelCfg* out) {
-    if (L < 1 || L > 16 || !dims || (aggr != 0 && aggr != 1) || (gemm != 0 && gemm != 1) ||
+    if (L < 1 || L > 16 || !dims || aggr < 0 || aggr > 2 || (gemm != 0 && gemm != 1) ||
         (feat_dtype != 0 && feat_dtype != 1))
         return false;
     ModelCfg m;
     m.L = L;
     m.aggr = aggr;
+    m.sum = aggr == 2;
     m.bf16 = gemm == 1;
     m.feat_bf16 = feat_dtype == 1;
     m.dims.assign(dims, dims + L + 1);
@@ -242,7 +243,7 @@ void sage_forward(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView*
             gemm_row(c, gs, s);
             PB(l == 0 ? PROBE_AGG_L0 : PROBE_AGG_L1);
             agg_mean_pf(c, B.Y, B.Ys, L.ld_y, V.indptr, V.indices, V.cnt, V.cap_dst, L.Fo, L.Fop, !L.last, out,
-                        out_bf, L.ld_out, s);
+                        out_bf, L.ld_out, m.sum, s);
             if (!L.last) b.l[l + 1].hbits_ok = false;
             PE(l == 0 ? PROBE_AGG_L0 : PROBE_AGG_L1);
             continue;
@@ -267,7 +268,7 @@ void sage_forward(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView*
             const int32_t* erow = (l == 0 && V.egid) ? V.egid : V.indices;
             const int32_t* emap = (l == 0 && !V.egid) ? V.src_gid : nullptr;
             agg_mean_xa(c, X, xbf, ldx, xrow, erow, emap, V.indptr, V.cnt, V.order_tab, V.cap_dst,
-                        V.src_per_mb > 0 ? V.src_per_mb : V.cap_src, L.Fi, L.Fp, B.XA, m.bf16, L.ld_xa, s);
+                        V.src_per_mb > 0 ? V.src_per_mb : V.cap_src, L.Fi, L.Fp, B.XA, m.bf16, L.ld_xa, m.sum, s);
             PE(l == 0 ? PROBE_AGG_L0 : PROBE_AGG_L1);
         }
         GemmRow g{};
@@ -291,7 +292,7 @@ void sage_loss(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView* v,
     const BlockView& V = v[m.L - 1];
     // the fp32 dS of a project-first top layer is read only by P^T D+ dS: stored pre-scaled by 1/D_v
     loss_ce(c, b.logits, L.ld_out, labels, V.src_gid, V.cnt, V.cap_dst, L.Fo, scale, b.dS_last, L.Fop,
-            b.dS_last_act, m.bf16, L.ld_ds, L.kind == KIND_PF ? V.indptr : nullptr, loss_accum, s);
+            b.dS_last_act, m.bf16, L.ld_ds, (L.kind == KIND_PF && !m.sum) ? V.indptr : nullptr, loss_accum, s);
 }
 
 void sage_backward(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView* v, const void* feats,
@@ -312,7 +313,7 @@ void sage_backward(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView
             const int64_t esz = m.bf16 ? 2 : 4;
             const bool ds_f32 = L.last;
             csc_pf(c, ds_f32 ? (const void*)b.dS_last : B.dS, !ds_f32 && m.bf16, ds_f32 ? L.Fop : L.ld_ds,
-                   ds_f32 ? nullptr : V.indptr,
+                   (ds_f32 || m.sum) ? nullptr : V.indptr,      // null: no 1/D (pre-scaled, or sum)
                    V.t_indptr, V.t_indices, V.cnt, V.cap_src, L.Fo, L.Fop, B.G, m.bf16, L.ld_g, s);
             const void* Ao; int64_t ldao;
             ones_operand(m, b, l, &Ao, &ldao);
@@ -369,7 +370,7 @@ void sage_backward(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView
             gemm_row(c, g, s);
         }
         if (L.kind == KIND_AGG) {
-            csc_mean(c, B.dXA, L.ld_dxa, V.indptr, V.t_indptr, V.t_indices, V.cnt, V.cap_src, L.Fi, L.Fp, Hmask,
+            csc_mean(c, B.dXA, L.ld_dxa, m.sum ? nullptr : V.indptr, V.t_indptr, V.t_indices, V.cnt, V.cap_src, L.Fi, L.Fp, Hmask,
                      m.bf16, ldh, B.hbits_ok ? B.Hbits : nullptr, B.ldhb, dS_prev, m.bf16, ld_prev, s);
             continue;
         }

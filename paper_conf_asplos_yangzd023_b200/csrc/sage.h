@@ -12,11 +12,12 @@ namespace betty {
 // otab: optional micro-batch-major row order (extract.h), null = ascending rows
 void agg_mean_xa(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const int32_t* srow, const int32_t* erow,
                  const int32_t* emap, const int64_t* indptr, const int64_t* cnt, const int64_t* otab, int64_t rows_cap,
-                 int64_t src_per_mb, int Fi, int Fp, void* XA, bool xa_bf16, int64_t ldxa, cudaStream_t s);
+                 int64_t src_per_mb, int Fi, int Fp, void* XA, bool xa_bf16, int64_t ldxa, bool sum, cudaStream_t s);
 // S[v] = Ys[v] + (1/D_v) sum_u Y[u]  (Y: neighbour half over src rows, Ys: self half over dst rows, same ld)
+// sum: the sum aggregator (no 1/D_v); likewise agg_mean_xa's sum and a null indptr of the CSC kernels
 void agg_mean_pf(betty_ctx* c, const float* Y, const float* Ys, int64_t ldy, const int64_t* indptr, const int32_t* idx,
                  const int64_t* cnt, int64_t rows_cap, int Fo, int Fop, bool relu, void* out, bool out_bf16,
-                 int64_t ldo, cudaStream_t s);
+                 int64_t ldo, bool sum, cudaStream_t s);
 void gather_ones(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const int32_t* xrow, const int64_t* cnt_rows,
                  int64_t rows_cap, int Fi, void* out, bool out_bf16, int64_t ldo, cudaStream_t s);
 void csc_mean(betty_ctx* c, const float* dXA, int64_t ldd, const int64_t* indptr, const int64_t* t_indptr,

@@ -260,6 +260,10 @@ CASES = [
     dict(name="mean3-agg64", aggr="mean", fanouts=(3, 4, 5), dims=[32, 64, 64, 5]),
     # pool rows longer than one warp-wide position search (byte-position argmax, rows of ~150 edges)
     dict(name="pool2-full-hub", aggr="pool", fanouts=(-1, -1), dims=[8, 16, 3], n=400, pairs=30000),
+    # the sum aggregator (Table 1 "Sum"): aggregate-first, project-first, the 3-layer hidden CSC path
+    dict(name="sum2", aggr="sum", fanouts=(3, 4), dims=[20, 32, 5]),
+    dict(name="sum2-pf", aggr="sum", fanouts=(3, 4), dims=[70, 16, 4]),
+    dict(name="sum3-agg64", aggr="sum", fanouts=(3, 4, 5), dims=[32, 64, 64, 5]),
 ]
 
 
@@ -314,7 +318,8 @@ def test_sage_micro_batch(B, ctx, c, mode):
 @pytest.mark.parametrize("mode", ["fp32", "bf16"])
 @pytest.mark.parametrize("group", [1, 2, 0])
 @pytest.mark.parametrize("graph", [False, True])
-@pytest.mark.parametrize("c", [CASES[1], CASES[2], CASES[4], CASES[7], CASES[8], CASES[9]], ids=lambda c: c["name"])
+@pytest.mark.parametrize("c", [CASES[1], CASES[2], CASES[4], CASES[7], CASES[8], CASES[9], CASES[10], CASES[11],
+                               CASES[12]], ids=lambda c: c["name"])
 def test_step_matches_oracle(B, ctx, c, mode, group, graph):
     """betty_step (fused extraction + fwd + loss + bwd + accumulation over a
     rank's micro-batches) vs oracle_step, for several launch groupings."""

@@ -2,8 +2,8 @@
 pool aggregator's tie rule (reading #14).
 
 The reference here is an independent dense re-derivation in numpy float64: no
-oracle code, its own layer loop over dense P matrices, and torch's
-float32->bfloat16 conversion (a library routine) as the rounding.  It applies
+oracle code, its own layer loop over dense P matrices, and its own bfloat16
+rounding (integer carry on the float64 bits, pinned to torch's conversion).  It applies
 the bf16 casts at exactly the points reading #17 names:
   * the feature table (H_0) and every parameter tensor (W_s, W_n, b, W_p, b_p)
     are GEMM operands -> bf16;
@@ -31,9 +31,26 @@ def idx_of(b):
 
 
 def q(x):
-    """RNE to bfloat16 through torch (library rounding), back to float64."""
-    x = np.asarray(x, dtype=np.float64)
-    return torch.from_numpy(x.astype(np.float32)).to(torch.bfloat16).double().numpy().reshape(x.shape)
+    """RNE of float64 values to bfloat16's 8 significant bits, by integer arithmetic on the float64 bit
+    pattern (the carry trick: add 2^44 - 1 + lsb, clear the low 45 mantissa bits).  A single rounding
+    from float64: going through float32 first (torch's double -> bfloat16 conversion does) double-rounds
+    values with more than 24 significant bits, which the sum aggregator's exact sums produce.  The
+    helper is itself pinned to torch's float32 -> bfloat16 conversion below."""
+    x = np.ascontiguousarray(x, dtype=np.float64)
+    b = x.view(np.uint64)
+    lsb = (b >> np.uint64(45)) & np.uint64(1)
+    r = ((b + np.uint64((1 << 44) - 1) + lsb) >> np.uint64(45)) << np.uint64(45)
+    return np.where(np.isfinite(x) & (x != 0), r.view(np.float64), x)
+
+
+def test_q_equals_torch_bfloat16_on_float32_inputs():
+    rng = np.random.default_rng(5)
+    x = rng.standard_normal(20000).astype(np.float32)
+    base = torch.tensor(x[:3000]).to(torch.bfloat16).float().numpy()
+    ties = (base.view(np.uint32) | np.uint32(0x8000)).view(np.float32)       # exact bf16 ties
+    x = np.concatenate([x, ties, np.float32([0.0, -0.0, 1.0, -3.0, 65504.0])])
+    want = torch.tensor(x).to(torch.bfloat16).double().numpy()
+    np.testing.assert_array_equal(q(x.astype(np.float64)), want)
 
 
 def dense_step(blocks, dims, aggr, params, feats, labels, scale, bf16=True, tie="first"):
@@ -150,6 +167,8 @@ CASES = [
     dict(name="mean3-wide", aggr="mean", fanouts=(3, 3, 4), dims=[12, 20, 6, 5]),
     dict(name="pool2", aggr="pool", fanouts=(3, 4), dims=[5, 6, 3]),
     dict(name="pool3", aggr="pool", fanouts=(2, 3, 3), dims=[4, 5, 5, 3]),
+    dict(name="sum2-aggfirst", aggr="sum", fanouts=(3, 4), dims=[5, 7, 3]),
+    dict(name="sum2-projfirst", aggr="sum", fanouts=(3, 4), dims=[9, 4, 3]),
 ]
 
 

@@ -24,6 +24,8 @@ def dense_forward(blocks, dims, aggr, params, feats, src_gid0):
         if aggr == "mean":
             deg = P.sum(1, keepdims=True)
             A = np.divide(P @ X, deg, out=np.zeros((nd, X.shape[1])), where=deg > 0)
+        elif aggr == "sum":                      # Table 1 "Sum": no 1/D
+            A = P @ X
         else:
             Z = np.maximum(X @ W[l]["Wp"] + W[l]["bp"], 0.0)
             A = np.zeros((nd, X.shape[1]))
@@ -42,6 +44,8 @@ CASES = [
     dict(name="mean2-projfirst", aggr="mean", fanouts=(3, 4), dims=[9, 4, 3]),
     dict(name="pool2", aggr="pool", fanouts=(3, 4), dims=[5, 6, 3]),
     dict(name="pool3", aggr="pool", fanouts=(2, 3, 3), dims=[4, 5, 5, 3]),
+    dict(name="sum2", aggr="sum", fanouts=(3, 4), dims=[5, 7, 3]),
+    dict(name="sum3-projfirst", aggr="sum", fanouts=(2, 3, 4), dims=[6, 8, 4, 3]),
 ]
 
 
@@ -94,11 +98,11 @@ def test_mean_all_equal_rows_and_pool_identity_reduction():
     assert (lg[deg == 0] == 0).all()
 
 
-@pytest.mark.parametrize("c", [c for c in CASES if c["aggr"] == "mean"], ids=lambda c: c["name"])
+@pytest.mark.parametrize("c", [c for c in CASES if c["aggr"] != "pool"], ids=lambda c: c["name"])
 def test_two_sageconv_forms_agree(c):
     g, sd, blocks, feats, labels, params = make_case(c)
-    a = oracle.sage(c["dims"], "mean", False, blocks, params, feats, labels, 0.1, force_form=0, want_logits=True)
-    b = oracle.sage(c["dims"], "mean", False, blocks, params, feats, labels, 0.1, force_form=1, want_logits=True)
+    a = oracle.sage(c["dims"], c["aggr"], False, blocks, params, feats, labels, 0.1, force_form=0, want_logits=True)
+    b = oracle.sage(c["dims"], c["aggr"], False, blocks, params, feats, labels, 0.1, force_form=1, want_logits=True)
     np.testing.assert_allclose(a[2], b[2], rtol=1e-12, atol=1e-13)
     np.testing.assert_allclose(a[0], b[0], rtol=1e-10, atol=1e-13)
     assert a[1] == pytest.approx(b[1], rel=1e-13)
@@ -174,3 +178,17 @@ def test_bf16_mode_is_close_to_fp32_mode(c):
     e_log = np.linalg.norm(a[2] - b[2]) / np.linalg.norm(a[2])
     e_grad = np.linalg.norm(a[0] - b[0]) / np.linalg.norm(a[0])
     assert 0 < e_log < 3e-2 and 0 < e_grad < 5e-2, (e_log, e_grad)
+
+
+def test_sum_is_degree_times_mean():
+    """Table 1: the sum aggregator equals D_v times the mean (one layer, W_self = 0, b = 0, W_neigh = I:
+    the logits are the aggregated rows themselves)."""
+    c = dict(aggr="sum", fanouts=(4,), dims=[4, 4])
+    g, sd, blocks, feats, labels, params = make_case(c, n_out=12)
+    P = np.zeros(4 * 4 * 2 + 4)
+    P[16:32] = np.eye(4).ravel()                 # W_neigh = I, W_self = 0, b = 0
+    _, _, ls = oracle.sage([4, 4], "sum", False, blocks, P, feats, labels, 1.0, want_logits=True)
+    _, _, lm = oracle.sage([4, 4], "mean", False, blocks, P, feats, labels, 1.0, want_logits=True)
+    deg = np.diff(blocks[0].indptr).astype(np.float64)[:, None]
+    np.testing.assert_allclose(ls, deg * lm, rtol=1e-13, atol=1e-13)
+    assert (deg > 1).any()
