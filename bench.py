@@ -48,8 +48,10 @@ def parse():
     p.add_argument("--mode", default="bf16", choices=["fp32", "bf16"], help="GEMM operand precision")
     p.add_argument("--group", type=int, default=None,
                    help="micro-batches per launch group (0 = all of a rank's; default all, 1 for C4)")
-    p.add_argument("--partition", default="reg", choices=["reg", "reg-greedy", "range", "random"],
-                   help="reg = REG + multilevel (METIS scheme, Alg. 1); reg-greedy = REG + greedy growing")
+    p.add_argument("--partition", default="reg", choices=["reg", "reg-greedy", "range", "random", "metis-raw"],
+                   help="reg = REG + multilevel (METIS scheme, Alg. 1); reg-greedy = REG + greedy growing; "
+                        "range / random / metis-raw = the paper's redundancy-unaware baselines (PAPER.md:1222-1230; "
+                        "metis-raw: the multilevel partitioner on the raw graph induced on the outputs)")
     p.add_argument("--no-graph", action="store_true")
     p.add_argument("--no-reg", action="store_true", help="exclude the REG rebuild (a1) from the step")
     p.add_argument("--probe", default="auto")
@@ -240,6 +242,15 @@ def make_partition(args, B, ctx, cfg, ds, dev_blocks, rank, ws, device):
         part = synth.range_partition(cfg.n_out, args.K)
     elif args.partition == "random":
         part = synth.random_partition(cfg.n_out, args.K, cfg.seeds["part"])
+    elif args.partition == "metis-raw":
+        from paper_conf_asplos_yangzd023_b200.partition import raw_graph_partition
+        part = None
+        if rank == 0:
+            part = raw_graph_partition(ds.graph.indptr, ds.graph.indices, ds.seeds, args.K)
+        if ws > 1:
+            t = torch.as_tensor(part if rank == 0 else np.zeros(cfg.n_out, np.int32)).to(device)
+            dist.broadcast(t, src=0)
+            part = t.cpu().numpy()
     else:
         part = None
         if rank == 0:
