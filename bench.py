@@ -383,7 +383,7 @@ def main():
     import torch
     import torch.distributed as dist
     import paper_conf_asplos_yangzd023_b200 as B
-    from paper_conf_asplos_yangzd023_b200.dist import allreduce_grad, lpt_assign, micro_batch_costs, reg_rows
+    from paper_conf_asplos_yangzd023_b200.dist import allreduce_grad, lpt_assign, plan_costs, reg_rows
 
     # BETTY_BENCH_ONE_GPU=1 (testing the multi-rank path on a one-GPU box): every rank on cuda:0 and
     # gloo for the collectives -- timings of such a run are not bench values
@@ -405,7 +405,8 @@ def main():
         mem_aware = memory_aware(args, B, ctx, cfg, dev_blocks, rank, ws, device)
     part = make_partition(args, B, ctx, cfg, ds, dev_blocks, rank, ws, device)
     dpart = torch.as_tensor(part).to(device)
-    costs = micro_batch_costs(part, args.K, ds.blocks[-1].indptr)
+    # LPT cost per micro-batch from its per-layer sizes (GPU count-only extraction)
+    costs = plan_costs(B.betty_mb_sizes(ctx, dev_blocks, dpart, args.K), cfg.dims)
     # --sim-world N (one GPU): run rank 0's share of an N-rank job -- its micro-batches and REG rows --
     # to study per-rank step time; the line is then per-rank, not a bench value
     wv, rv = (args.sim_world, 0) if args.sim_world > 1 else (ws, rank)

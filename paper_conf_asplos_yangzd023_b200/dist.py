@@ -23,6 +23,18 @@ def micro_batch_costs(part: np.ndarray, K: int, out_indptr: np.ndarray) -> np.nd
     return np.bincount(np.asarray(part, dtype=np.int64), weights=deg + 1, minlength=K).astype(np.float64)
 
 
+def plan_costs(sizes: np.ndarray, dims: Sequence[int], gamma: float = 0.008) -> np.ndarray:
+    """Scheduling cost per micro-batch from its per-layer sizes (betty_mb_sizes: [K, L, 3] = n_dst,
+    n_src, n_edges of every layer, a GPU count-only extraction): SURVEY.md §8(e)'s
+    cost_k = sum_l (E_{k,l} F_l + gamma n_dst,k,l F_l F_{l+1}) -- the aggregation's gathered elements
+    plus the dense layer's flops converted to element-equivalents (gamma = 2 / ridge, ridge ~ 250 flop
+    per byte).  Host arithmetic, outside the hot path."""
+    sizes = np.asarray(sizes, dtype=np.float64)
+    F = np.asarray(dims, dtype=np.float64)
+    nd, E = sizes[:, :, 0], sizes[:, :, 2]
+    return (E * F[None, :-1] + gamma * nd * F[None, :-1] * F[None, 1:]).sum(1)
+
+
 def lpt_assign(costs: Sequence[float], world: int) -> List[List[int]]:
     """Longest-processing-time-first: micro-batches in decreasing cost go to
     the least loaded rank.  Deterministic (ties by index).  Returns, per rank,

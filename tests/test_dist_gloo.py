@@ -86,3 +86,13 @@ def test_two_rank_allreduce_equals_full_batch():
         assert p.exitcode == 0
     assert np.linalg.norm(red[:-1] - full) <= 1e-12 * np.linalg.norm(full)
     assert abs(red[-1] - lfull) <= 1e-12 * abs(lfull)
+
+
+def test_plan_costs_closed_form():
+    """cost_k = sum_l (E_{k,l} F_l + gamma n_dst,k,l F_l F_{l+1})."""
+    from paper_conf_asplos_yangzd023_b200.dist import plan_costs
+    sizes = np.array([[[10, 20, 100], [2, 10, 30]], [[5, 9, 40], [1, 5, 8]]])
+    dims = [24, 48, 5]
+    g = 0.5
+    want = [100 * 24 + g * 10 * 24 * 48 + 30 * 48 + g * 2 * 48 * 5, 40 * 24 + g * 5 * 24 * 48 + 8 * 48 + g * 1 * 48 * 5]
+    np.testing.assert_allclose(plan_costs(sizes, dims, gamma=g), want)
