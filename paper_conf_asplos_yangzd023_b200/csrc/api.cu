@@ -500,6 +500,7 @@ struct betty_plan {
     // the full-batch CSC
     std::vector<int64_t*> fcsc_cnt;
     std::vector<int32_t*> fcsc_tmp;
+    bool lean0 = false;           // the step extracts layer 0 lean (extract.h ExtractArgs::lean0)
     SageBufs sb;
     std::vector<BlockView> views;
     // REG inside the step
@@ -543,6 +544,8 @@ static void step_body(betty_ctx* c, betty_plan* p, const float* params, const vo
         c->lane = 0;
         cudaEventRecord(p->ev_join, p->side);
     };
+    if ((p->flags & BETTY_PLAN_FRESH) && p->lean0)      // full-batch edge -> gid of layer 0
+        full_egid(c, p->full[0].nbr, p->full[0].src_gid, p->full[0].n_edges, (int32_t*)p->full[0].egid, s);
     if (p->flags & BETTY_PLAN_FRESH) {        // full-batch CSCs from the current block buffers
         for (int l = 0; l < p->L; ++l) {
             if (!(p->csc_mask >> l & 1)) continue;
@@ -561,6 +564,7 @@ static void step_body(betty_ctx* c, betty_plan* p, const float* params, const vo
         a.L = p->L; a.full = p->full.data(); a.part = p->part; a.K = p->K;
         a.ks = p->d_ks + g * p->c; a.c = (int32_t)p->groups[g].size();
         a.layers = p->X.layers.data(); a.sc = p->X.sc; a.csc_mask = p->csc_mask;
+        a.lean0 = p->lean0;
         if (pr) pr->begin(PROBE_EXTRACT, s);
         extract_group(c, a, s);
         if (pr) pr->end(PROBE_EXTRACT, s);
@@ -774,6 +778,19 @@ extern "C" betty_status betty_plan_create(betty_ctx* c, const betty_model* model
         p->full[l].t_nbr = ftn;
         p->fcsc_cnt[l] = hc;
         p->fcsc_tmp[l] = tc;
+    }
+    // lean layer 0 (aggregate-first layer 0 without a CSC: its features are gathered by global id, no
+    // kernel reads its src list): the full batch's edge -> source gid array, once per plan
+    static const bool full_extract = getenv("BETTY_FULL_EXTRACT") && atoi(getenv("BETTY_FULL_EXTRACT"));
+    p->lean0 = !full_extract && L >= 2 && m.layers[0].kind == KIND_AGG && !(p->csc_mask & 1) && p->X.layers[0].egid;
+    if (p->lean0 && A.ok) {
+        int32_t* fe = A.get<int32_t>(full[0].n_edges);
+        if (fe) {
+            full_egid(c, full[0].indices, full[0].src_gid, full[0].n_edges, fe, s);
+            p->full[0].egid = fe;
+        } else {
+            p->lean0 = false;
+        }
     }
     if (!A.ok) {
         betty_plan_destroy(c, p);

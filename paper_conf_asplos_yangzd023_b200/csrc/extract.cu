@@ -667,6 +667,69 @@ __global__ void k_order_tab(int32_t c, int L, int l, const int64_t* __restrict__
     if (threadIdx.x == 0) { vs[nseg] = s_base; tab[2 * (ORDER_TAB_MAX + 1)] = nseg; }
 }
 
+// lean layer 0: each dst row's full-batch edge segment of source gids -> the group's egid (rows in
+// their group order; warp-flattened like the relabel, coalesced within a row); n_src := n_dst
+__global__ void __launch_bounds__(256) k_seg_egid(const int32_t* __restrict__ dst_pos, int64_t* cnt,
+                                                  const int64_t* __restrict__ findptr,
+                                                  const int32_t* __restrict__ fegid,
+                                                  const int64_t* __restrict__ indptr, int32_t* __restrict__ egid,
+                                                  int64_t cap_e, int* dev_err) {
+    __shared__ FlatRows s_rows[8];
+    const int64_t n = cnt[0];
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        cnt[1] = n;
+        if (cnt[2] > cap_e) atomicOr(dev_err, DEVERR_OVERFLOW);
+    }
+    const int lane = lane_id();
+    FlatRows& F = s_rows[warp_id()];
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t v0 = gw * 32; v0 < n; v0 += nw * 32) {
+        const int64_t r = v0 + lane;
+        int d = 0;
+        if (r < n) {
+            const int32_t q = dst_pos[r];
+            const int64_t b = findptr[q];
+            d = (int)(findptr[q + 1] - b);
+            F.fb[lane] = b;
+            F.ob[lane] = indptr[r];
+        }
+        const int incl = warp_incl_scan(d);
+        F.pre[lane + 1] = incl;
+        if (lane == 0) F.pre[0] = 0;
+        __syncwarp();
+        const int total = F.pre[32];
+        for (int f0 = lane; f0 < total; f0 += 32 * FLAT_UNR) {
+            int32_t g[FLAT_UNR];
+            int64_t o[FLAT_UNR];
+#pragma unroll
+            for (int u = 0; u < FLAT_UNR; ++u) {
+                const int f = f0 + 32 * u;
+                o[u] = -1;
+                if (f < total) {
+                    const int k = flat_row(F, f);
+                    g[u] = fegid[F.fb[k] + (f - F.pre[k])];
+                    o[u] = F.ob[k] + (f - F.pre[k]);
+                }
+            }
+#pragma unroll
+            for (int u = 0; u < FLAT_UNR; ++u) if (o[u] >= 0 && o[u] < cap_e) egid[o[u]] = g[u];
+        }
+        __syncwarp();
+    }
+}
+
+// full-batch edge -> source gid of a layer (once per plan; every step with BETTY_PLAN_FRESH)
+__global__ void k_full_egid(const int32_t* __restrict__ nbr, const int32_t* __restrict__ src_gid, int64_t E,
+                            int32_t* __restrict__ egid) {
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < E; e += (int64_t)gridDim.x * blockDim.x)
+        egid[e] = src_gid[nbr[e]];
+}
+void full_egid(betty_ctx* c, const int32_t* nbr, const int32_t* src_gid, int64_t E, int32_t* egid, cudaStream_t s) {
+    const int g = (int)std::max<int64_t>(1, std::min<int64_t>((E + 255) / 256, (int64_t)c->num_sms * 8));
+    k_full_egid<<<g, 256, 0, s>>>(nbr, src_gid, E, egid);
+}
+
 __global__ void k_clear_bits(uint32_t* a, uint32_t* b, int64_t n) {
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
         a[i] = 0u;
@@ -718,6 +781,14 @@ void extract_group(betty_ctx* ctx, const ExtractArgs& a, cudaStream_t s) {
         }
         // rows: degree of each dst row in the full batch -> local indptr
         scan_deg(ctx, dst_pos, F.indptr, B.indptr, B.cnt + 0, cap_d, B.cnt + 2, s);
+        if (l == 0 && a.lean0 && F.egid && B.egid) {
+            // lean layer 0: the dst prefix (self rows) and the edges' source gids, nothing else
+            k_emit_dst<<<grid_for(ctx, cap_d, 256), 256, 0, s>>>(dst_pos, row_mb, B.cnt, dst_off, B.mb_src_off,
+                                                                 F.src_gid, B.src_pos, B.src_gid, B.src_mb, cap_s);
+            k_seg_egid<<<grid_for(ctx, (cap_d + 31) / 32 * 32, 256), 256, 0, s>>>(dst_pos, B.cnt, F.indptr, F.egid,
+                                                                                  B.indptr, B.egid, cap_e, ctx->dev_err);
+            break;
+        }
         // dedupe: dst bitmap + position map, then new-source bitmap
         k_mark_dst<<<grid_for(ctx, cap_d, 256), 256, 0, s>>>(dst_pos, row_mb, B.cnt, a.sc.dstbits, W);
         const int g_rows = grid_for(ctx, cap_d, 256);       // 32 rows per warp

@@ -13,6 +13,7 @@ struct ExtractFull {            // full-batch block l (device arrays, host sizes
     const int32_t* src_gid;
     const int64_t* t_indptr = nullptr;   // optional full-batch CSC (built once per plan): [n_src+1]
     const int32_t* t_nbr = nullptr;      // [n_edges] full dst rows, ascending per column
+    const int32_t* egid = nullptr;       // optional [n_edges]: global id of each edge's source (src_gid[nbr])
 };
 
 struct ExtractLayer {           // group-concatenated micro-batch layer l (device arrays)
@@ -100,6 +101,12 @@ struct ExtractArgs {
     ExtractLayer* layers;       // [L]
     ExtractScratch sc;
     uint32_t csc_mask;          // bit l: build the CSC of layer l
+    // lean0: layer 0's sources are not materialised -- its rows (indptr, the dst prefix's src_pos /
+    // src_gid) and the per-edge source gids (egid, copied row segment by row segment from the
+    // full batch's full[0].egid) are all an aggregate-first layer 0 consumes: its features are
+    // gathered by global id from the resident table, no kernel reads the layer's src list, local
+    // indices or CSC.  The plan's step sets it; standalone / inspection extractions never do.
+    bool lean0 = false;
 };
 
 void extract_group(betty_ctx* ctx, const ExtractArgs& a, cudaStream_t s);

@@ -106,5 +106,7 @@ struct PrepLayer {
 void prep_weights(betty_ctx* c, const float* params, const PrepLayer* layers, int L, bool bf16, cudaStream_t s);
 // hi = x with the low 13 mantissa bits cleared, lo = x - hi (the 3xTF32 operand split), n elements
 void split_tf32_dev(const float* x, float* hi, float* lo, int64_t n, cudaStream_t s);
+// ---- extract.cu: egid[e] = src_gid[nbr[e]] over a full-batch layer's E edges
+void full_egid(betty_ctx* c, const int32_t* nbr, const int32_t* src_gid, int64_t E, int32_t* egid, cudaStream_t s);
 
 }  // namespace betty
