@@ -59,6 +59,10 @@ def parse():
     p.add_argument("--no-fp32", action="store_true",
                    help="skip the nested paper-precision (fp32, 3xTF32 GEMMs) measurement of a bf16 run")
     p.add_argument("--cpu-threads", type=int, default=0, help="cpu_baseline / reference threads (0: all cores)")
+    p.add_argument("--feat-shards", type=int, default=-1,
+                   help="layer-0 feature table sharded by rows over R buffers: with N > 1 ranks R = N means one "
+                        "shard per GPU, mapped by every rank through CUDA IPC (reads cross NVLink); at N = 1, R "
+                        "virtual shards on the one GPU.  -1 (default): N for C5 (BASELINE configs[4]), else 0")
     p.add_argument("--cpu-sample-outputs", type=int, default=4096, help="cpu_baseline sample (~10 s)")
     p.add_argument("--ref-sample-outputs", type=int, default=512, help="--impl reference per-step sample (per core)")
     p.add_argument("--scale", type=float, default=1.0, help="shrink the graph (debug only)")
@@ -413,7 +417,15 @@ def main():
     my_k = lpt_assign(costs, wv)[rv]
 
     import synth
-    feats = synth.features_device(cfg, ds, args.mode == "bf16", args.feat_align, device)   # bf16: reading #17
+    if args.feat_shards < 0:
+        args.feat_shards = ws if (args.config == "C5" and ws > 1) else 0
+    shard = None
+    if args.feat_shards > 0:       # rows sharded over R buffers (per GPU with IPC at N > 1)
+        shard = make_shards(args, B, ctx, cfg, ds, rank, ws, device)
+        feats = shard["stub"]
+        args.no_fp32 = True
+    else:
+        feats = synth.features_device(cfg, ds, args.mode == "bf16", args.feat_align, device)   # bf16: reading #17
     host_gid0 = ds.blocks[0].src_gid
     if args.feat_layout == "l2":       # (study only) every layer-0 row read hits 64 Ki rows = 16 MB: L2-resident
         b0 = dev_blocks[0]
@@ -447,6 +459,8 @@ def main():
     flags = (0 if args.no_graph else B.PLAN_GRAPH) | (0 if args.no_reg else B.PLAN_REG)
     t0 = time.time()
     plan, args.group = create_plan(B, ctx, model, dev_blocks, dpart, args.K, my_k, args.group, flags)
+    if shard:
+        plan.set_feature_shards(shard["bases"], shard["rps"])
     t_plan = time.time() - t0
     if wv > 1 and not args.no_reg:
         plan.set_reg_rows(*reg_rows(cfg.n_out, rv, wv))        # REG rows sharded across ranks
@@ -557,6 +571,8 @@ def main():
                 raise RuntimeError("e2e plan would need a smaller launch group")
             if wv > 1 and not args.no_reg:
                 pe.set_reg_rows(*reg_rows(cfg.n_out, rv, wv))
+            if shard:
+                pe.set_feature_shards(shard["bases"], shard["rps"])
             plans.append(pe)
             bufs.append(dev_list(dbs, dp))
             step(pe)                               # capture its graph outside the timed region
@@ -616,6 +632,7 @@ def main():
     B.betty_sync_check(ctx)                        # FRESH steps validate the copied inputs on the device
 
     # ------------------------------------------------------- cpu baseline
+    table_bytes = cfg.n * feats.shape[1] * feats.element_size() if shard else feats.numel() * feats.element_size()
     cpu = None
     if rank == 0 and ws == 1 and args.cpu_sample_outputs > 0:
         cpu = cpu_baseline(args, cfg, ds, scale)
@@ -628,17 +645,22 @@ def main():
             "dtype": "bf16-gemm/fp32-accum" if args.mode == "bf16" else "fp32",
             "data": "synthetic",
             "config": dict(workload_config(args, cfg, ws), micro_batches_per_rank=len(my_k),
-                           l2="inputs > L2 (feature table %.2f GB + blocks)" % (feats.numel() * feats.element_size()
-                                                                              / 1e9)),
+                           l2="inputs > L2 (feature table %.2f GB + blocks)" % (table_bytes / 1e9)),
             "edges_per_step": edges_all,
             "full_batch_edges": full_edges,
             "full_batch_edges_per_s": full_edges / (ms_step * 1e-3),
             "plan": {k: info[k] for k in ("n_groups", "edges", "n_src", "n_dst", "reg_nnz", "arena_bytes",
                                           "kernels_per_step")},
             "memory": {"group": args.group or "all", "plan_arena_gb": info["arena_bytes"] / 2 ** 30,
-                       "feature_table_gb": feats.numel() * feats.element_size() / 2 ** 30,
+                       "feature_table_gb": table_bytes / 2 ** 30,
                        "peak_allocated_gb": torch.cuda.max_memory_allocated(device) / 2 ** 30},
             "paper_precision": paper,
+            "feature_shards": None if not shard else {
+                "R": shard["R"], "rows_per_shard": shard["rps"], "mapping": shard["mapping"],
+                "remote_row_fraction": shard["remote_fraction"],
+                "layer0_gather_remote_GBps": (shard["remote_fraction"] * info["edges"][0] * shard["row_bytes"] /
+                                              (roof["avg_launch_ms"] * roof["launches_per_step"] * 1e-3) / 1e9)
+                if roof else None},
             "e2e": {"value": edges_all / (e2e_ms * 1e-3), "unit": "edges/s", "ms_per_step": e2e_ms,
                     "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": 4,
                     "input_buffers": nb, "fresh_inputs": plans[0] is not plan},
@@ -661,8 +683,61 @@ def main():
             with open(args.json_out, "w") as f:
                 f.write(s + "\n")
     plan.free()
+    if shard:
+        if ws > 1:
+            dist.barrier()                         # no rank still reads a peer's shard
+        for b in shard["buffers"]:
+            b.free()
     if ws > 1:
         dist.destroy_process_group()
+
+
+def make_shards(args, B, ctx, cfg, ds, rank, ws, device):
+    """The layer-0 feature table split by rows into R shards.  N > 1 with R == N: rank r owns rows
+    [r rps, (r+1) rps) in a cudaMalloc'd buffer and maps every other rank's buffer through CUDA IPC
+    (handles exchanged with one all_gather_object; no collective in the step: the layer-0 gathers
+    read remote rows over NVLink).  N = 1: R buffers on the one GPU (virtual shards)."""
+    import torch
+    import torch.distributed as dist
+    import synth
+    bf16 = args.mode == "bf16"
+    dt = torch.bfloat16 if bf16 else torch.float32
+    esz = 2 if bf16 else 4
+    per = max(1, args.feat_align // esz) if args.feat_align > 0 else 1
+    ld = (cfg.ld + per - 1) // per * per
+    R = args.feat_shards
+    rps = (cfg.n + R - 1) // R
+    own = []
+    if ws > 1:
+        if R != ws:
+            raise SystemExit("--feat-shards with N > 1 ranks must be N (one shard per GPU)")
+        mine = B.DevBuffer(ctx, rps * ld * esz)
+        synth.features_fill_rows(cfg, ds, mine.tensor(dt, (rps, ld)), rank * rps)
+        torch.cuda.synchronize()
+        handles = [None] * ws
+        dist.all_gather_object(handles, mine.ipc_handle())
+        bases = []
+        for r in range(ws):
+            if r == rank:
+                bases.append(mine.ptr)
+            else:
+                o = B.DevBuffer.open(ctx, handles[r], rps * ld * esz)
+                own.append(o)
+                bases.append(o.ptr)
+        own.append(mine)
+        mapping = f"one shard per GPU, peers mapped with CUDA IPC ({ws} GPUs)"
+    else:
+        bases = []
+        for r in range(R):
+            b = B.DevBuffer(ctx, rps * ld * esz)
+            synth.features_fill_rows(cfg, ds, b.tensor(dt, (rps, ld)), r * rps)
+            own.append(b)
+            bases.append(b.ptr)
+        mapping = f"{R} virtual shards on one GPU"
+    torch.cuda.synchronize()
+    return {"R": R, "rps": rps, "bases": bases, "buffers": own, "mapping": mapping, "row_bytes": cfg.F * esz,
+            "remote_fraction": (R - 1) / R if ws > 1 else 0.0,
+            "stub": torch.zeros((1, ld), dtype=dt, device=device)}
 
 
 def timed_ms(step, steps, ws, stream):

@@ -205,6 +205,27 @@ BETTY_API betty_status betty_plan_set_reg_rows(betty_ctx* ctx, betty_plan* plan,
                                                betty_stream stream);
 BETTY_API void betty_plan_destroy(betty_ctx* ctx, betty_plan* plan);
 
+/* Feature table sharded by rows across R device buffers (BASELINE.json configs[4]: "features sharded
+ * across 8 GPUs' HBM"): global row g lives in base[g / rows_per_shard] at local row
+ * g % rows_per_shard, with the row stride (ld_feats) and dtype betty_step is called with.  base[]
+ * (HOST array of R device pointers, 16-byte aligned) may hold other GPUs' buffers mapped with
+ * betty_ipc_open: the plan's layer-0 gathers then read remote rows over NVLink (owner-computes is
+ * not needed: the one gather per edge goes to the owning shard).  The feats argument of betty_step
+ * is then ignored for layer 0.  R = 0 returns to one contiguous table.  Supported for an
+ * aggregate-first layer 0 (mean / sum with F_in <= F_out), else BETTY_EUNSUPPORTED; EINVAL for
+ * R > 64 or bad pointers.  The caller owns the buffers (they must outlive the plan's steps). */
+BETTY_API betty_status betty_plan_set_feature_shards(betty_ctx* ctx, betty_plan* plan, int32_t R,
+                                                     const void* const* base, int64_t rows_per_shard);
+/* Device buffers other processes can map (CUDA IPC): betty_dev_alloc (cudaMalloc on the ctx's
+ * device), betty_ipc_handle (64 opaque bytes, host), betty_ipc_open (maps another process's buffer
+ * into this one; peer access enabled lazily), betty_ipc_close, betty_dev_free.  ECUDA on failure. */
+#define BETTY_IPC_HANDLE_BYTES 64
+BETTY_API betty_status betty_dev_alloc(betty_ctx* ctx, size_t bytes, void** out);
+BETTY_API betty_status betty_dev_free(betty_ctx* ctx, void* p);
+BETTY_API betty_status betty_ipc_handle(betty_ctx* ctx, void* dev_ptr, void* handle);
+BETTY_API betty_status betty_ipc_open(betty_ctx* ctx, const void* handle, void** dev_ptr);
+BETTY_API betty_status betty_ipc_close(betty_ctx* ctx, void* dev_ptr);
+
 /* One training step on this rank: for every micro-batch of the plan,
  * extraction (a2) -> forward (a3) -> loss (a4) -> backward (a5) with the
  * gradient ADDED into grad_accum (a6).  The caller then all-reduces

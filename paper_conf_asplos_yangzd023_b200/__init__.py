@@ -13,6 +13,7 @@ import ctypes
 from dataclasses import dataclass, field
 from typing import List, Optional, Sequence
 
+import numpy as np
 import torch
 
 from . import _lib as L
@@ -265,6 +266,13 @@ class Plan:
         self.ctx.check(L.lib().betty_plan_set_reg_rows(self.ctx.h, self.h, row0, row1, _stream(stream)),
                        "betty_plan_set_reg_rows")
 
+    def set_feature_shards(self, bases: Sequence[int], rows_per_shard: int):
+        """Layer-0 features sharded by rows: row g in bases[g // rows_per_shard] (device pointers, peer
+        mappings included); [] = one contiguous table (the feats argument of betty_step)."""
+        arr = (ctypes.c_void_p * max(1, len(bases)))(*[int(b) for b in bases])
+        self.ctx.check(L.lib().betty_plan_set_feature_shards(self.ctx.h, self.h, len(bases), arr, int(rows_per_shard)),
+                       "betty_plan_set_feature_shards")
+
     def probe(self, site: int):
         """Bracket the launches of one kernel site with CUDA events (see betty.h)."""
         self.ctx.check(L.lib().betty_plan_probe(self.h, site), "betty_plan_probe")
@@ -416,3 +424,46 @@ def betty_memory_aware_k(ctx: Context, model: Model, full: Sequence[Block], reg,
                                            PART_METHODS[method], part.ctypes.data, ctypes.byref(k_out), ctypes.byref(peak),
                                            _stream(stream)), "betty_memory_aware_k")
     return k_out.value, (part[:n_out] if k_out.value > 0 else None), peak.value
+
+
+# ------------------------------------------------------------------ CUDA IPC buffers (sharded features)
+class DevBuffer:
+    """A cudaMalloc'd device buffer other processes can map (betty_dev_alloc); .tensor(dtype, shape)
+    views it as a torch tensor (no copy)."""
+
+    def __init__(self, ctx: Context, nbytes: int, ptr: Optional[int] = None, owned: bool = True):
+        self.ctx, self.nbytes, self.owned = ctx, int(nbytes), owned
+        if ptr is None:
+            p = ctypes.c_void_p()
+            ctx.check(L.lib().betty_dev_alloc(ctx.h, self.nbytes, ctypes.byref(p)), "betty_dev_alloc")
+            ptr = p.value
+        self.ptr = int(ptr)
+
+    def tensor(self, dtype: torch.dtype, shape) -> torch.Tensor:
+        ts = {torch.float32: "<f4", torch.bfloat16: "<V2", torch.int32: "<i4"}[dtype]
+        n = int(np.prod(shape))
+        cai = _CAI(self.ptr, n, ts if dtype != torch.bfloat16 else "<i2")
+        t = torch.as_tensor(cai, device=f"cuda:{self.ctx.device}")
+        if dtype == torch.bfloat16:
+            t = t.view(torch.bfloat16)
+        return t.view(*shape)
+
+    def ipc_handle(self) -> bytes:
+        buf = ctypes.create_string_buffer(64)
+        self.ctx.check(L.lib().betty_ipc_handle(self.ctx.h, ctypes.c_void_p(self.ptr), buf), "betty_ipc_handle")
+        return buf.raw
+
+    @staticmethod
+    def open(ctx: Context, handle: bytes, nbytes: int) -> "DevBuffer":
+        p = ctypes.c_void_p()
+        ctx.check(L.lib().betty_ipc_open(ctx.h, ctypes.create_string_buffer(handle, 64), ctypes.byref(p)),
+                  "betty_ipc_open")
+        return DevBuffer(ctx, nbytes, p.value, owned=False)
+
+    def free(self):
+        if self.ptr:
+            if self.owned:
+                L.lib().betty_dev_free(self.ctx.h, ctypes.c_void_p(self.ptr))
+            else:
+                L.lib().betty_ipc_close(self.ctx.h, ctypes.c_void_p(self.ptr))
+            self.ptr = 0

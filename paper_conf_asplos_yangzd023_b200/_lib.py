@@ -69,6 +69,12 @@ def lib() -> ctypes.CDLL:
         "betty_plan_info_get": (i32, [vp, pp(betty_plan_info)]),
         "betty_plan_destroy": (None, [vp, vp]),
         "betty_plan_set_reg_rows": (i32, [vp, vp, i64, i64, vp]),
+        "betty_plan_set_feature_shards": (i32, [vp, vp, i32, vp, i64]),
+        "betty_dev_alloc": (i32, [vp, ctypes.c_size_t, pp(vp)]),
+        "betty_dev_free": (i32, [vp, vp]),
+        "betty_ipc_handle": (i32, [vp, vp, vp]),
+        "betty_ipc_open": (i32, [vp, vp, pp(vp)]),
+        "betty_ipc_close": (i32, [vp, vp]),
         "betty_step": (i32, [vp, vp, vp, vp, i64, vp, f32, vp, vp, vp]),
         "betty_adam": (i32, [vp, vp, vp, vp, vp, i64, i32, f32, f32, f32, f32, i32, vp]),
         "betty_sync_check": (i32, [vp, vp]),
@@ -97,4 +103,5 @@ EXPORTED = ["betty_version", "betty_ctx_create", "betty_ctx_destroy", "betty_las
             "betty_step", "betty_adam", "betty_sync_check", "betty_reg_partition", "betty_plan_probe",
             "betty_plan_probe_read", "betty_plan_group_blocks", "betty_test_gemm", "betty_mb_sizes",
             "betty_mem_estimate", "betty_memory_aware_k", "betty_reg_partition_ex", "betty_reg_build_rows",
-            "betty_plan_set_reg_rows"]
+            "betty_plan_set_reg_rows", "betty_plan_set_feature_shards", "betty_dev_alloc", "betty_dev_free",
+            "betty_ipc_handle", "betty_ipc_open", "betty_ipc_close"]

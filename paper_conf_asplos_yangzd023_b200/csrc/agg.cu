@@ -25,6 +25,13 @@ namespace betty {
 template <typename T> __device__ __forceinline__ const T* row_ptr(const T* X, int64_t ld, const int32_t* xrow, int64_t r) {
     return X + (int64_t)(xrow ? xrow[r] : (int32_t)r) * ld;
 }
+// feature row g of a (possibly sharded) table: base[g / rps] + (g % rps) * ld, or X + g * ld
+template <typename T> __device__ __forceinline__ const T* feat_row(const T* X, int64_t ld, const FeatShards& sh,
+                                                                   int32_t g) {
+    if (sh.R == 0) return X + (int64_t)g * ld;
+    const int s = (int)((int64_t)g / sh.rps);
+    return (const T*)sh.base[s] + ((int64_t)g - (int64_t)s * sh.rps) * ld;
+}
 
 // ------------------------------------------------ mean, aggregate-first fwd
 // LPR lanes own one dst row (RPW = 32/LPR rows per warp); lane `sub` covers
@@ -106,7 +113,7 @@ __global__ void __launch_bounds__(256) k_agg_mean_xa(const Tin* __restrict__ X, 
                                                      const int64_t* __restrict__ indptr, const int64_t* cnt,
                                                      const int64_t* __restrict__ otab, int Fi, int Fp,
                                                      Tout* __restrict__ XA, int64_t ldxa, int hint, int vlo, int vhi,
-                                                     unsigned* ctr, int sum) {
+                                                     unsigned* ctr, int sum, const __grid_constant__ FeatShards sh) {
     using VI = Vec<Tin>;
     constexpr int VW = VI::N;
     constexpr int RPW = 32 / LPR;
@@ -178,15 +185,15 @@ __global__ void __launch_bounds__(256) k_agg_mean_xa(const Tin* __restrict__ X, 
                 if (sub == 0) mbar_expect(bar, (uint32_t)(n + 1) * row_bytes);
                 __syncwarp(gmask);
                 asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-                if (sub < n) bulk_row(wb + sub * LPR, X + (int64_t)cur.my * ldx, row_bytes, bar, pol);
-                if (sub == 0) bulk_row(wb + EB * LPR, X + (int64_t)cur.sr * ldx, row_bytes, bar, pol);
+                if (sub < n) bulk_row(wb + sub * LPR, feat_row(X, ldx, sh, cur.my), row_bytes, bar, pol);
+                if (sub == 0) bulk_row(wb + EB * LPR, feat_row(X, ldx, sh, cur.sr), row_bytes, bar, pol);
             }
         } else if (fast) {      // the whole row (neighbours + self) in one batch of async copies
             for (int t = 0; t < n; ++t) {
                 const int32_t u = __shfl_sync(gmask, cur.my, t, LPR);
-                if (act) cp_async16(wb + t * LPR + sub, X + (int64_t)u * ldx + vi * VW, pol, use_hint);
+                if (act) cp_async16(wb + t * LPR + sub, feat_row(X, ldx, sh, u) + vi * VW, pol, use_hint);
             }
-            if (act) cp_async16(wb + EB * LPR + sub, X + (int64_t)cur.sr * ldx + vi * VW, pol, use_hint);
+            if (act) cp_async16(wb + EB * LPR + sub, feat_row(X, ldx, sh, cur.sr) + vi * VW, pol, use_hint);
             asm volatile("cp.async.commit_group;" ::: "memory");
         }
         if (threadIdx.x == 0) {
@@ -247,7 +254,7 @@ __global__ void __launch_bounds__(256) k_agg_mean_xa(const Tin* __restrict__ X, 
                     if (sub < nb) { mj = erow[e0 + sub]; if (emap) mj = emap[mj]; }
                     for (int t = 0; t < nb; ++t) {
                         const int32_t u = __shfl_sync(gmask, mj, t, LPR);
-                        if (actj) cp_async16(wb + t * LPR + sub, X + (int64_t)u * ldx + vj * VW, pol, use_hint);
+                        if (actj) cp_async16(wb + t * LPR + sub, feat_row(X, ldx, sh, u) + vj * VW, pol, use_hint);
                     }
                     cp_async_wait_all();
                     if (actj)
@@ -256,7 +263,7 @@ __global__ void __launch_bounds__(256) k_agg_mean_xa(const Tin* __restrict__ X, 
                 }
                 if (actj) {
                     VI self;
-                    self.load(X + (int64_t)cur.sr * ldx + vj * VW);
+                    self.load(feat_row(X, ldx, sh, cur.sr) + vj * VW);
 #pragma unroll
                     for (int t = 0; t < VW; ++t) {
                         const int col = vj * VW + t;
@@ -1376,8 +1383,11 @@ static bool agg_mean_g4(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, c
 
 void agg_mean_xa(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const int32_t* srow, const int32_t* erow,
                  const int32_t* emap, const int64_t* indptr, const int64_t* cnt, const int64_t* otab, int64_t rows_cap,
-                 int64_t src_per_mb, int Fi, int Fp, void* XA, bool xa_bf16, int64_t ldxa, bool sum, cudaStream_t s) {
+                 int64_t src_per_mb, int Fi, int Fp, void* XA, bool xa_bf16, int64_t ldxa, bool sum,
+                 const FeatShards* shards, cudaStream_t s) {
     const int vw = x_bf16 ? 8 : 4;
+    FeatShards sh;
+    if (shards) sh = *shards;
     const int nv = (Fi + vw - 1) / vw;
     // Column passes: one micro-batch's gathered rows must stay L2-resident between their
     // uses; when (source rows of a micro-batch) x (row bytes) exceeds the budget, the
@@ -1385,15 +1395,17 @@ void agg_mean_xa(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const in
     // only a slice of every row (the rows' metadata is re-read, the features are not).
     static const double budget = getenv("BETTY_AGG_WS_MB") ? atof(getenv("BETTY_AGG_WS_MB")) * 1e6 : 1e12;
     unsigned* ctr = c->L().counters + CTR_AGG;
-    static const int hint = getenv("BETTY_AGG_CA") ? 3 :
-                            (getenv("BETTY_AGG_NOHINT") ? 0 : (getenv("BETTY_AGG_NOBULK") ? 2 : 1));
+    static const int hint_env = getenv("BETTY_AGG_CA") ? 3 :
+                                (getenv("BETTY_AGG_NOHINT") ? 0 : (getenv("BETTY_AGG_NOBULK") ? 2 : 1));
+    // sharded tables: per-lane cp.async gathers (whole-row bulk copies are not used on peer memory)
+    const int hint = sh.R > 0 ? 2 : hint_env;
     static const bool no_order = getenv("BETTY_AGG_NOORDER") != nullptr;
     const double ws = (double)src_per_mb * (double)nv * 16.0;
     int passes = (int)std::max(1.0, std::min((double)nv, std::ceil(ws / budget)));
     const int pv = (nv + passes - 1) / passes;
     passes = (nv + pv - 1) / pv;
     static const bool g4_off = getenv("BETTY_AGG_G4") && atoi(getenv("BETTY_AGG_G4")) == 0;
-    if (!g4_off && passes == 1 && nv * vw <= 256 && agg_mean_g4(c, X, x_bf16, ldx, srow, erow, emap, indptr, cnt, otab,
+    if (!g4_off && sh.R == 0 && passes == 1 && nv * vw <= 256 && agg_mean_g4(c, X, x_bf16, ldx, srow, erow, emap, indptr, cnt, otab,
                                                                 Fi, Fp, nv, XA, xa_bf16, ldxa, hint, ctr, sum, s))
         return;
     const int lpr = pv <= 8 ? 8 : (pv <= 16 ? 16 : 32);
@@ -1410,7 +1422,7 @@ void agg_mean_xa(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const in
             cudaMemsetAsync(ctr, 0, sizeof(unsigned), s);                                                      \
             k_agg_mean_xa<TI, TO, LPR><<<grid, 256, sm, s>>>((const TI*)X, ldx, srow, erow, emap, indptr, cnt,    \
                 no_order ? nullptr : otab, Fi, Fp, (TO*)XA, ldxa, hint, pz * pv, std::min(nv, (pz + 1) * pv), ctr, \
-                sum ? 1 : 0); } }))
+                sum ? 1 : 0, sh); } }))
     if (lpr == 8) { AGG_L(8); } else if (lpr == 16) { AGG_L(16); } else { AGG_L(32); }
 #undef AGG_L
 }

@@ -502,6 +502,7 @@ struct betty_plan {
     std::vector<int32_t*> fcsc_tmp;
     bool lean0 = false;           // the step extracts layer 0 lean (extract.h ExtractArgs::lean0)
     SageBufs sb;
+    FeatShards shards;            // layer-0 feature table sharded by rows (betty_plan_set_feature_shards)
     std::vector<BlockView> views;
     // REG inside the step
     bool with_reg = false;
@@ -657,6 +658,73 @@ static betty_status plan_reg_setup(betty_ctx* c, betty_plan* p, const betty_bloc
     p->with_reg = true;
     p->info.reg_nnz = nnz;
     p->info.arena_bytes = p->arena->bytes + A.bytes + p->sb.bytes;
+    return BETTY_OK;
+}
+
+extern "C" betty_status betty_plan_set_feature_shards(betty_ctx* c, betty_plan* p, int32_t R, const void* const* base,
+                                                     int64_t rows_per_shard) {
+    if (!c) return BETTY_EINVAL;
+    if (!p || R < 0 || R > MAX_SHARDS || (R > 0 && (!base || rows_per_shard < 1)))
+        return fail(c, BETTY_EINVAL, "plan_set_feature_shards: bad arguments");
+    if (R > 0 && (p->m.layers[0].kind != KIND_AGG))
+        return fail(c, BETTY_EUNSUPPORTED, "plan_set_feature_shards: only an aggregate-first layer 0 (mean / sum, "
+                                           "F_in <= F_out) gathers from a sharded table");
+    for (int r = 0; r < R; ++r)
+        if (!base[r] || ((uintptr_t)base[r] & 15)) return fail(c, BETTY_EINVAL, "plan_set_feature_shards: bad base");
+    FeatShards sh;
+    sh.R = R;
+    sh.rps = rows_per_shard;
+    for (int r = 0; r < R; ++r) sh.base[r] = base[r];
+    p->shards = sh;
+    p->sb.shards = R > 0 ? &p->shards : nullptr;
+    if (p->gexec) { cudaGraphExecDestroy(p->gexec); p->gexec = nullptr; }     // kernel arguments change
+    return BETTY_OK;
+}
+
+// ------------------------------------------ device buffers shared across processes (CUDA IPC)
+extern "C" betty_status betty_dev_alloc(betty_ctx* c, size_t bytes, void** out) {
+    if (!c || !out) return BETTY_EINVAL;
+    *out = nullptr;
+    cudaSetDevice(c->device);
+    if (cudaMalloc(out, std::max<size_t>(bytes, 16)) != cudaSuccess) {
+        cudaGetLastError();
+        return fail(c, BETTY_ENOMEM, "dev_alloc: cudaMalloc failed");
+    }
+    return BETTY_OK;
+}
+extern "C" betty_status betty_dev_free(betty_ctx* c, void* p) {
+    if (!c) return BETTY_EINVAL;
+    if (p) cudaFree(p);
+    return BETTY_OK;
+}
+extern "C" betty_status betty_ipc_handle(betty_ctx* c, void* dev_ptr, void* handle) {
+    if (!c || !dev_ptr || !handle) return BETTY_EINVAL;
+    cudaIpcMemHandle_t h;
+    if (cudaIpcGetMemHandle(&h, dev_ptr) != cudaSuccess) {
+        cudaGetLastError();
+        return fail(c, BETTY_ECUDA, "ipc_handle: cudaIpcGetMemHandle failed (pointer from betty_dev_alloc?)");
+    }
+    static_assert(sizeof(h) == BETTY_IPC_HANDLE_BYTES, "IPC handle size");
+    memcpy(handle, &h, sizeof(h));
+    return BETTY_OK;
+}
+extern "C" betty_status betty_ipc_open(betty_ctx* c, const void* handle, void** dev_ptr) {
+    if (!c || !handle || !dev_ptr) return BETTY_EINVAL;
+    cudaIpcMemHandle_t h;
+    memcpy(&h, handle, sizeof(h));
+    cudaSetDevice(c->device);
+    if (cudaIpcOpenMemHandle(dev_ptr, h, cudaIpcMemLazyEnablePeerAccess) != cudaSuccess) {
+        cudaGetLastError();
+        return fail(c, BETTY_ECUDA, "ipc_open: cudaIpcOpenMemHandle failed");
+    }
+    return BETTY_OK;
+}
+extern "C" betty_status betty_ipc_close(betty_ctx* c, void* dev_ptr) {
+    if (!c || !dev_ptr) return BETTY_EINVAL;
+    if (cudaIpcCloseMemHandle(dev_ptr) != cudaSuccess) {
+        cudaGetLastError();
+        return fail(c, BETTY_ECUDA, "ipc_close failed");
+    }
     return BETTY_OK;
 }
 

@@ -107,6 +107,7 @@ struct Probe {
 
 struct SageBufs {
     Probe* probe = nullptr;
+    const FeatShards* shards = nullptr;     // layer-0 feature table sharded by rows (or null)
     bool tf32 = false;            // FP32 mode products as 3xTF32 on tcgen05 (else SIMT FFMA)
     std::vector<LayerBufs> l;
     float* logits = nullptr;

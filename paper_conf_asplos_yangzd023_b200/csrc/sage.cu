@@ -268,7 +268,8 @@ void sage_forward(betty_ctx* c, const ModelCfg& m, SageBufs& b, const BlockView*
             const int32_t* erow = (l == 0 && V.egid) ? V.egid : V.indices;
             const int32_t* emap = (l == 0 && !V.egid) ? V.src_gid : nullptr;
             agg_mean_xa(c, X, xbf, ldx, xrow, erow, emap, V.indptr, V.cnt, V.order_tab, V.cap_dst,
-                        V.src_per_mb > 0 ? V.src_per_mb : V.cap_src, L.Fi, L.Fp, B.XA, m.bf16, L.ld_xa, m.sum, s);
+                        V.src_per_mb > 0 ? V.src_per_mb : V.cap_src, L.Fi, L.Fp, B.XA, m.bf16, L.ld_xa, m.sum,
+                        l == 0 ? b.shards : nullptr, s);
             PE(l == 0 ? PROBE_AGG_L0 : PROBE_AGG_L1);
         }
         GemmRow g{};

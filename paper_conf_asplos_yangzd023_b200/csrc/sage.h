@@ -8,11 +8,21 @@ struct betty_ctx;
 namespace betty {
 
 // ---- agg.cu
+// A feature table sharded by rows (BASELINE configs[4]): row g lives in base[g / rps]
+// at local row g % rps (row stride ld of the table); R == 0: one contiguous table (X, ldx).  The bases
+// may be peer-mapped memory of other GPUs (CUDA IPC): the gathers then cross NVLink.
+constexpr int MAX_SHARDS = 64;
+struct FeatShards {
+    int R = 0;
+    int64_t rps = 0;
+    const void* base[MAX_SHARDS] = {};
+};
 // XA[v] = [X[srow v] | mean_e X[row(e)] | 1], row(e) = emap ? emap[erow[e]] : erow[e]
 // otab: optional micro-batch-major row order (extract.h), null = ascending rows
 void agg_mean_xa(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, const int32_t* srow, const int32_t* erow,
                  const int32_t* emap, const int64_t* indptr, const int64_t* cnt, const int64_t* otab, int64_t rows_cap,
-                 int64_t src_per_mb, int Fi, int Fp, void* XA, bool xa_bf16, int64_t ldxa, bool sum, cudaStream_t s);
+                 int64_t src_per_mb, int Fi, int Fp, void* XA, bool xa_bf16, int64_t ldxa, bool sum,
+                 const FeatShards* shards, cudaStream_t s);
 // S[v] = Ys[v] + (1/D_v) sum_u Y[u]  (Y: neighbour half over src rows, Ys: self half over dst rows, same ld)
 // sum: the sum aggregator (no 1/D_v); likewise agg_mean_xa's sum and a null indptr of the CSC kernels
 void agg_mean_pf(betty_ctx* c, const float* Y, const float* Ys, int64_t ldy, const int64_t* indptr, const int32_t* idx,

@@ -319,6 +319,22 @@ def features_device(cfg: Config, ds: "Dataset", bf16: bool, align: int, device, 
     return out
 
 
+def features_fill_rows(cfg: Config, ds: "Dataset", out, row0: int, chunk_rows: int = 1 << 22):
+    """Fill a device tensor out[n, ld] (n <= rows left from row0) with feature rows row0 .. row0+n-1
+    (columns [0, cfg.ld), the rest zero): one shard of a row-sharded table."""
+    import torch
+    n = min(out.shape[0], cfg.n - row0)
+    out.zero_()
+    for r0 in range(row0, row0 + n, chunk_rows):
+        m = min(chunk_rows, row0 + n - r0)
+        if ds.feats is not None:
+            h = ds.feats[r0:r0 + m]
+        else:
+            h = features_rows(ds.graph.comm, cfg.F, cfg.ld, row0=r0, n=m, kind=cfg.feat_kind, seed=cfg.seeds["feat"])
+        out[r0 - row0:r0 - row0 + m, :cfg.ld] = torch.from_numpy(np.ascontiguousarray(h)).to(out.device).to(out.dtype)
+    return out
+
+
 def init_params(dims: Sequence[int], aggr: str, seed: int = 4) -> np.ndarray:
     """Xavier-uniform weights, zero... small uniform biases; flat fp32 in the
     layout of include/betty.h (per layer: [W_pool, b_pool] (pool only),
