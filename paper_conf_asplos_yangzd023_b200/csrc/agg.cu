@@ -1370,11 +1370,14 @@ static bool agg_mean_g4(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, c
     a.stage_bytes = (a.slot_groups + G4_MAXR / 4) * a.grp_bytes;
     const size_t sm = (size_t)G4_STAGES * a.stage_bytes + red_bytes;
     DISPATCH_ACT(x_bf16, TI, DISPATCH_ACT(xa_bf16, TO, {
-        static bool attr = false;
-        if (!attr) {
-            cudaFuncSetAttribute(k_agg_mean_g4<TI, TO>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
-            attr = true;
+        static int max_dyn = -1;
+        if (max_dyn < 0) {       // the opt-in maximum per CTA (227 KB) minus the kernel's static shared memory
+            cudaFuncAttributes fa{};
+            cudaFuncGetAttributes(&fa, k_agg_mean_g4<TI, TO>);
+            max_dyn = 227 * 1024 - (int)fa.sharedSizeBytes;
+            cudaFuncSetAttribute(k_agg_mean_g4<TI, TO>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_dyn);
         }
+        if ((int)sm > max_dyn) return false;
         cudaMemsetAsync(ctr, 0, sizeof(unsigned), s);
         k_agg_mean_g4<TI, TO><<<c->num_sms, G4_THREADS, sm, s>>>(tm, a);
     }))
