@@ -504,6 +504,9 @@ def main():
 
     # ---------------------- paper precision (fp32) beside a bf16 headline
     paper = None
+    if args.config == "C5" and args.mode == "bf16" and not args.no_fp32:
+        args.no_fp32 = True           # a 57 GB fp32 table next to the bf16 plan's arenas does not fit one GPU
+        paper = {"skipped": "C5: the fp32 feature table (57 GB) and fp32 arenas do not fit beside the bf16 run"}
     if args.mode == "bf16" and not args.no_fp32:
         feats32 = synth.features_device(cfg, ds, False, args.feat_align, device)
         if args.feat_layout != "gid":

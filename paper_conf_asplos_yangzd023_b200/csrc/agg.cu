@@ -1363,7 +1363,16 @@ static bool agg_mean_g4(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, c
     a.row_bytes = (uint32_t)nv * 16u;
     a.grp_bytes = (4u * a.row_bytes + 127u) / 128u * 128u;
     const size_t red_bytes = 0;
-    const size_t budget = (size_t)196 * 1024 - red_bytes;            // dynamic smem for the stage ring
+    static int static_smem = -1;                                      // the kernel's static footprint
+    if (static_smem < 0) {
+        cudaFuncAttributes fa{};
+        if (x_bf16) cudaFuncGetAttributes(&fa, xa_bf16 ? k_agg_mean_g4<__nv_bfloat16, __nv_bfloat16>
+                                                       : k_agg_mean_g4<__nv_bfloat16, float>);
+        else cudaFuncGetAttributes(&fa, xa_bf16 ? k_agg_mean_g4<float, __nv_bfloat16> : k_agg_mean_g4<float, float>);
+        static_smem = (int)fa.sharedSizeBytes;
+    }
+    // dynamic smem for the stage ring: up to 196 KB, within the 227 KB opt-in minus the static part
+    const size_t budget = std::min<size_t>((size_t)196 * 1024, (size_t)(227 * 1024 - static_smem - 1024)) - red_bytes;
     const int64_t groups = (int64_t)(budget / G4_STAGES) / a.grp_bytes - G4_MAXR / 4;
     if (groups < 4) return false;
     a.slot_groups = (uint32_t)std::min<int64_t>(groups, 64);     // a producer lane issues <= 2 groups

@@ -1,18 +1,23 @@
-// gemm_tc.cu -- the dense SAGE layers on the 5th-generation tensor cores
-// (tcgen05.mma kind::f16, bf16 operands, fp32 accumulation in TMEM), BF16
-// mode.  Hand-written PTX: TMA (cp.async.bulk.tensor, 128B swizzle) fills a
-// multi-stage shared-memory ring, one elected thread issues tcgen05.mma into
-// TMEM, four epilogue warps drain TMEM with tcgen05.ld and apply the fused
-// epilogue.  Warp roles (192 threads, 1 CTA / SM, persistent):
-//   warp 0: TMA producer   warp 1: TMEM allocator + MMA issuer   warps 2-5: epilogue
+// gemm_tc.cu -- the dense SAGE layers on the 5th-generation tensor cores, hand-written PTX:
+// TMA (cp.async.bulk.tensor, 128B swizzle) fills a multi-stage shared-memory ring, one elected
+// thread issues tcgen05.mma into TMEM, epilogue warps drain TMEM with tcgen05.ld.  Persistent, one
+// CTA per SM.  Two precisions:
+//   BF16 mode: kind::f16 (bf16 operands), fp32 accumulation;
+//   FP32 mode (TF = true): kind::tf32 as 3xTF32 -- converter warps split each landed fp32 stage into an
+//     RN-tf32 hi (in place) and lo, and per k-block the MMA warp issues lo*hi, hi*lo (into a second
+//     accumulator) and hi*hi; see split_tf32 and the k_tc_red drain for why (fp32-level accuracy).
 //
 //   k_tc_row : C[M x N] = A[M x K] B[K x N]   (A, B K-major; M on the device)
-//              epilogues: store / ReLU + ones column / ReLU' mask / residual + mask
-//              two TMEM accumulators so the epilogue of tile i overlaps the MMAs of tile i+1
-//   k_tc_red : P[K1 x N] = A^T B over the node dimension (dW), A and B MN-major
-//              (node rows contiguous in features), a fixed row range per CTA
-//              accumulated in TMEM, partials reduced deterministically by
-//              k_red_final (gemm.cu) into the flat gradient.
+//              warps: 0 TMA producer, 1 TMEM allocator + MMA issuer, 2-9 epilogue (8 warps: warp w
+//              drains TMEM lanes 32*(w%4).. for one half of the columns), + 2 converter warps in TF
+//              (320 / 384 threads).  Epilogues: store / ReLU + ones column (+ ReLU' bits) / ReLU' mask
+//              / residual + mask; each 32-column chunk goes TMEM -> registers -> swizzled smem slot ->
+//              TMA store.  Two TMEM accumulators (BF16 always, TF when 4 * BN <= 512) so the epilogue
+//              of tile i overlaps the MMAs of tile i+1.
+//   k_tc_red : P[K1 x N] = A^T B over the node dimension (dW), A and B MN-major (node rows
+//              contiguous in features), a fixed row range per CTA accumulated in TMEM, partials
+//              reduced deterministically by k_red_final (gemm.cu) into the flat gradient.  Warps: 0
+//              TMA, 1 MMA, 2-5 epilogue (+ 4 converter warps in TF: 192 / 320 threads).
 #include <cuda.h>
 #include <cuda_runtime.h>
 #include <cuda_bf16.h>
@@ -108,6 +113,18 @@ __device__ __forceinline__ void split_tf32(uint32_t x, uint32_t lo) {
     asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};" ::"r"(x), "f"(h.x), "f"(h.y), "f"(h.z), "f"(h.w) : "memory");
     asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};" ::"r"(lo), "f"(l.x), "f"(l.y), "f"(l.z), "f"(l.w) : "memory");
 }
+// hw_hi variant: only lo = x - trunc_tf32(x) is written; the tensor core's own fp32 -> tf32
+// conversion of the untouched x must then be the truncation (BETTY_TF32_HW_HI=1, an experiment)
+__device__ __forceinline__ void split_tf32_lo(uint32_t x, uint32_t lo) {
+    float4 v;
+    asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "r"(x));
+    float4 l;
+    l.x = v.x - __uint_as_float(__float_as_uint(v.x) & 0xFFFFE000u);
+    l.y = v.y - __uint_as_float(__float_as_uint(v.y) & 0xFFFFE000u);
+    l.z = v.z - __uint_as_float(__float_as_uint(v.z) & 0xFFFFE000u);
+    l.w = v.w - __uint_as_float(__float_as_uint(v.w) & 0xFFFFE000u);
+    asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};" ::"r"(lo), "f"(l.x), "f"(l.y), "f"(l.z), "f"(l.w) : "memory");
+}
 __device__ __forceinline__ void zero2_shared(uint32_t x, uint32_t lo) {
     asm volatile("st.shared.v4.u32 [%0], {%1, %1, %1, %1};" ::"r"(x), "r"(0u) : "memory");
     asm volatile("st.shared.v4.u32 [%0], {%1, %1, %1, %1};" ::"r"(lo), "r"(0u) : "memory");
@@ -171,6 +188,7 @@ struct RowArgs {
     int half_cols;           // columns per epilogue half (multiple of 32, <= 32 * MAXCH)
     uint32_t slot_bytes;     // one staging slot: 32 rows x 32 columns
     int bstream;             // 1: B is streamed with A through the ring (B too large to stay resident)
+    int hw_hi;               // TF: converter writes lo only (see split_tf32_lo)
     int64_t cend;            // trailing columns [N, cend) of a row are written (ones column / zeros)
 };
 
@@ -451,9 +469,15 @@ k_tc_row(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtens
             for (int kb = 0; kb < p.nk; ++kb) {
                 mbar_wait(&full[s], ph);
                 const uint32_t a = su32(aring + s * ring_bytes);
+                if (p.hw_hi) {
 #pragma unroll 4
-                for (int i = tid; i < (int)(a_bytes / 16); i += 32 * ROW_CONV_WARPS)
-                    split_tf32(a + 16 * i, a + a_bytes + 16 * i);
+                    for (int i = tid; i < (int)(a_bytes / 16); i += 32 * ROW_CONV_WARPS)
+                        split_tf32_lo(a + 16 * i, a + a_bytes + 16 * i);
+                } else {
+#pragma unroll 4
+                    for (int i = tid; i < (int)(a_bytes / 16); i += 32 * ROW_CONV_WARPS)
+                        split_tf32(a + 16 * i, a + a_bytes + 16 * i);
+                }
                 fence_proxy_async();             // generic-proxy writes -> visible to the tensor core
                 __syncwarp();
                 if ((threadIdx.x & 31) == 0) mbar_arrive(&conv[s]);
@@ -606,6 +630,7 @@ struct RedArgs {
     float* partials;           // [S][K1][N]
     uint32_t tmem_cols;
     uint32_t sbo;              // TF: byte stride between 4-row K atoms (512)
+    int hw_hi;                 // TF: converter writes lo only (see split_tf32_lo)
 };
 
 // TF (FP32 mode, 3xTF32): fp32 operands, k-blocks of 16 nodes (boxes of 32 features x 16 nodes, the
@@ -748,7 +773,10 @@ k_tc_red(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtens
             const uint32_t sa = su32(smem + s * stage_bytes);
             const int64_t valid = M - kb * KN;
             const int n16 = (int)(raw_bytes / 16);
-            if (valid >= KN) {
+            if (valid >= KN && p.hw_hi) {
+#pragma unroll 4
+                for (int i = tid; i < n16; i += 32 * CONV_WARPS) split_tf32_lo(sa + 16 * i, sa + raw_bytes + 16 * i);
+            } else if (valid >= KN) {
 #pragma unroll 4
                 for (int i = tid; i < n16; i += 32 * CONV_WARPS) split_tf32(sa + 16 * i, sa + raw_bytes + 16 * i);
             } else {                                     // the last k-block: rows >= M are zeroed
@@ -921,6 +949,8 @@ bool gemm_row_tc(betty_ctx* c, const GemmRow& g, const void* Bk, const void* Bk_
     p.M_dev = g.M_dev; p.K = g.K; p.N = g.N; p.BN = BN; p.nk = nk;
     p.stages = (int)std::max<size_t>(2, std::min<size_t>(8, (budget - fixed) / ring));
     p.bstream = bstream ? 1 : 0;
+    static const int hw_hi_row = getenv("BETTY_TF32_HW_HI") ? atoi(getenv("BETTY_TF32_HW_HI")) : 0;
+    p.hw_hi = hw_hi_row;
     p.C = g.C; p.ldc = g.ldc; p.cend = g.cend > 0 ? g.cend : g.ldc;
     p.mask = g.mask; p.ldm = g.ldm; p.m_bf16 = g.m_bf16; p.res = g.res; p.ldr = g.ldr; p.nres_dev = g.nres_dev;
     p.mbits = g.mbits; p.ldmb = g.ldmb;
@@ -1011,6 +1041,8 @@ bool gemm_red_tc(betty_ctx* c, const GemmRed& g, int* S_used, cudaStream_t s) {
     p.tmem_cols = tmem_cols_for((TF ? 2 : p.mt_cta) * p.acc_stride);
     static const uint32_t sbo_env = getenv("BETTY_TF_SBO") ? (uint32_t)atoi(getenv("BETTY_TF_SBO")) : 512u;
     p.sbo = sbo_env;
+    static const int hw_hi = getenv("BETTY_TF32_HW_HI") ? atoi(getenv("BETTY_TF32_HW_HI")) : 0;
+    p.hw_hi = hw_hi;
     const size_t smem = (size_t)p.stages * stage_bytes + 1024 + 256;
     const int grid = (p.mt_cta == 1 ? p.mtiles : 1) * p.S;
     if (TF) {
