@@ -23,6 +23,7 @@
 // micro-batch 0] ++ [new of 1] ++ ..., so that dst ids remain a prefix of the
 // src ids (the self term of SAGE needs it).  Per micro-batch this is exactly
 // its canonical block under a renumbering; for c = 1 it IS the canonical block.
+#include <cstring>
 #include "common.cuh"
 #include "internal.h"
 #include "extract.h"
@@ -90,15 +91,6 @@ __global__ void k_sel_offsets(const int64_t* __restrict__ off, int64_t nchunks, 
 }
 
 // ------------------------------------------------------------ per layer
-__global__ void k_deg(const int32_t* __restrict__ dst_pos, const int64_t* __restrict__ findptr, const int64_t* cnt,
-                      int64_t* __restrict__ deg) {
-    const int64_t n = cnt[0];
-    for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < n; r += (int64_t)gridDim.x * blockDim.x) {
-        const int32_t p = dst_pos[r];
-        deg[r] = findptr[p + 1] - findptr[p];
-    }
-}
-
 __global__ void k_mark_dst(const int32_t* __restrict__ dst_pos, const int32_t* __restrict__ row_mb,
                            const int64_t* cnt, uint32_t* dstbits, int64_t W) {
     const int64_t n = cnt[0];
@@ -195,13 +187,6 @@ static void slot_rank(const uint32_t* bits, const uint32_t* mask, int32_t c, int
     k_rank_write<<<g, RANK_THREADS, 0, s>>>(bits, mask, W, csum, out, slot_total);
 }
 
-// {bits, slot-relative popcount prefix} per bitmap word (wordoff: global exclusive scan)
-__global__ void k_pack_rank(const uint32_t* __restrict__ bits, const int64_t* __restrict__ wordoff, int64_t W,
-                            int64_t n, uint2* __restrict__ out) {
-    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
-        out[i] = make_uint2(bits[i], (uint32_t)(wordoff[i] - wordoff[(i / W) * W]));
-}
-
 // Local ids without a map.  Slot j's src list at layer l is [dst rows of layer l] ++ [new
 // sources, ascending position]; its dst rows ARE its src list at layer l+1 (same positions),
 // and at the top layer its outputs in ascending position.  So for a source p of slot j:
@@ -270,7 +255,7 @@ __global__ void __launch_bounds__(256) k_mark_new(const int32_t* __restrict__ ds
                                                   const int64_t* cnt, const int64_t* __restrict__ findptr,
                                                   const int32_t* __restrict__ fnbr, const uint32_t* __restrict__ dstbits,
                                                   uint32_t* newbits, int64_t W, const int64_t* __restrict__ otab,
-                                                  unsigned* ctr) {
+                                                  unsigned* ctr, int claim) {
     __shared__ int64_t s_vs[ORDER_SMEM + 1], s_rs[ORDER_SMEM];
     __shared__ FlatRows s_rows[8];
     const int nseg = order_load(otab, s_vs, s_rs);
@@ -278,18 +263,19 @@ __global__ void __launch_bounds__(256) k_mark_new(const int32_t* __restrict__ ds
     const int64_t n = cnt[0];
     const int lane = lane_id();
     FlatRows& F = s_rows[warp_id()];
-    // dynamic schedule (32-row claims): the rows in flight stay a narrow window of the
-    // micro-batch-major order, so one micro-batch's bitmaps / map stay in L2
+    // dynamic schedule (claims of `claim` <= 32 rows, lane = row): the rows in flight stay a narrow
+    // window of the micro-batch-major order, so one micro-batch's bitmaps / map stay in L2; small
+    // layers use shorter claims so that more warps share the (latency-bound) edge walk
     __shared__ int64_t s_claim[8];
     for (;;) {
-        if (lane == 0) s_claim[warp_id()] = (int64_t)atomicAdd(ctr, 1u) * 32;
+        if (lane == 0) s_claim[warp_id()] = (int64_t)atomicAdd(ctr, 1u) * claim;
         __syncwarp();
         const int64_t v0 = s_claim[warp_id()];
         __syncwarp();
         if (v0 >= n) break;
         const int64_t vv = v0 + lane;
         int d = 0;
-        if (vv < n) {
+        if (lane < claim && vv < n) {
             const int64_t r = order_map(vv, nseg, s_vs, s_rs, seg);
             const int32_t q = dst_pos[r];
             const int64_t b = findptr[q];
@@ -339,7 +325,7 @@ __global__ void __launch_bounds__(256) k_relabel(const int32_t* __restrict__ dst
                                                  const RankSet R, int l, int32_t* __restrict__ indices,
                                                  int64_t cap_e, const int32_t* __restrict__ fsrc_gid,
                                                  int32_t* __restrict__ egid, const int64_t* __restrict__ otab,
-                                                 unsigned* ctr) {
+                                                 unsigned* ctr, int claim, int32_t* __restrict__ tcnt, int64_t cap_src) {
     __shared__ int64_t s_vs[ORDER_SMEM + 1], s_rs[ORDER_SMEM];
     __shared__ FlatRows s_rows[8];
     const int nseg = order_load(otab, s_vs, s_rs);
@@ -347,18 +333,19 @@ __global__ void __launch_bounds__(256) k_relabel(const int32_t* __restrict__ dst
     const int64_t n = cnt[0];
     const int lane = lane_id();
     FlatRows& F = s_rows[warp_id()];
-    // dynamic schedule (32-row claims): the rows in flight stay a narrow window of the
-    // micro-batch-major order, so one micro-batch's bitmaps / map stay in L2
+    // dynamic schedule (claims of `claim` <= 32 rows, lane = row): the rows in flight stay a narrow
+    // window of the micro-batch-major order, so one micro-batch's bitmaps / map stay in L2; small
+    // layers use shorter claims so that more warps share the (latency-bound) edge walk
     __shared__ int64_t s_claim[8];
     for (;;) {
-        if (lane == 0) s_claim[warp_id()] = (int64_t)atomicAdd(ctr, 1u) * 32;
+        if (lane == 0) s_claim[warp_id()] = (int64_t)atomicAdd(ctr, 1u) * claim;
         __syncwarp();
         const int64_t v0 = s_claim[warp_id()];
         __syncwarp();
         if (v0 >= n) break;
         const int64_t vv = v0 + lane;
         int d = 0;
-        if (vv < n) {
+        if (lane < claim && vv < n) {
             const int64_t r = order_map(vv, nseg, s_vs, s_rs, seg);
             const int32_t q = dst_pos[r];
             const int64_t b = findptr[q];
@@ -431,6 +418,8 @@ __global__ void __launch_bounds__(256) k_relabel(const int32_t* __restrict__ dst
                     if (o < cap_e) {
                         indices[o] = id[u];
                         if (egid) egid[o] = gid[u];
+                        // CSC column length of the source (zeroed by the emit kernels)
+                        if (tcnt && id[u] < cap_src) atomicAdd(&tcnt[id[u]], 1);
                     }
                 }
             }
@@ -520,11 +509,6 @@ __global__ void __launch_bounds__(256) k_csc_flat(const int32_t* __restrict__ sr
     }
 }
 
-__global__ void k_popc(const uint32_t* __restrict__ newbits, int64_t n, int32_t* __restrict__ wc) {
-    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
-        wc[i] = __popc(newbits[i]);
-}
-
 // single CTA: per micro-batch src counts and offsets; checks capacities
 __global__ void k_counts(const int64_t* __restrict__ mb_dst_off, const int64_t* __restrict__ slot_total,
                          int32_t c, int64_t* __restrict__ mb_src_off, int64_t* cnt, int64_t cap_src, int64_t cap_e,
@@ -558,7 +542,7 @@ __global__ void k_emit_new(const uint2* __restrict__ nrank, int64_t W, int32_t c
                            const int64_t* __restrict__ mb_dst_off,
                            const int64_t* __restrict__ mb_src_off, const int32_t* __restrict__ fsrc_gid,
                            int32_t* __restrict__ src_pos, int32_t* __restrict__ src_gid, int32_t* __restrict__ src_mb,
-                           int64_t cap_src) {
+                           int64_t cap_src, int32_t* __restrict__ tcnt) {
     const int64_t n = (int64_t)c * W;
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
         const uint2 r = nrank[i];
@@ -572,7 +556,10 @@ __global__ void k_emit_new(const uint2* __restrict__ nrank, int64_t W, int32_t c
             const int b = __ffs(bits) - 1;
             bits &= bits - 1;
             const int32_t p = (int32_t)(w * 32 + b);
-            if (s < cap_src) { src_pos[s] = p; src_gid[s] = fsrc_gid[p]; src_mb[s] = j; }
+            if (s < cap_src) {
+                src_pos[s] = p; src_gid[s] = fsrc_gid[p]; src_mb[s] = j;
+                if (tcnt) tcnt[s] = 0;
+            }
             ++s;
         }
     }
@@ -582,49 +569,16 @@ __global__ void k_emit_dst(const int32_t* __restrict__ dst_pos, const int32_t* _
                            const int64_t* cnt, const int64_t* __restrict__ mb_dst_off,
                            const int64_t* __restrict__ mb_src_off, const int32_t* __restrict__ fsrc_gid,
                            int32_t* __restrict__ src_pos, int32_t* __restrict__ src_gid, int32_t* __restrict__ src_mb,
-                           int64_t cap_src) {
+                           int64_t cap_src, int32_t* __restrict__ tcnt) {
     const int64_t n = cnt[0];
     for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < n; r += (int64_t)gridDim.x * blockDim.x) {
         const int j = row_mb[r];
         const int64_t s = r;                            // dst prefix keeps the row order
         (void)mb_dst_off; (void)mb_src_off;
         const int32_t p = dst_pos[r];
-        if (s < cap_src) { src_pos[s] = p; src_gid[s] = fsrc_gid[p]; src_mb[s] = j; }
-    }
-}
-
-// CSC of a micro-batch layer from the full-batch CSC (no atomics, no sort for the
-// top layer): local src u (full position p, slot j) keeps the full-batch column of p
-// restricted to j's dst rows, relabelled through the dst map.  Top-layer dst ids
-// ascend with the full position, so the columns come out ascending.
-__global__ void k_csc_count(const int32_t* __restrict__ src_pos, const int32_t* __restrict__ src_mb, const int64_t* cnt,
-                            const int64_t* __restrict__ ft_indptr, const int32_t* __restrict__ ft_nbr,
-                            const uint32_t* __restrict__ dstbits, int64_t W, int32_t* __restrict__ tcnt) {
-    const int64_t n = cnt[1];
-    for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < n; u += (int64_t)gridDim.x * blockDim.x) {
-        const int32_t p = src_pos[u];
-        const uint32_t* db = dstbits + (int64_t)src_mb[u] * W;
-        int k = 0;
-        for (int64_t e = ft_indptr[p], ee = ft_indptr[p + 1]; e < ee; ++e) {
-            const int32_t q = ft_nbr[e];
-            k += (db[q >> 5] >> (q & 31)) & 1u;
-        }
-        tcnt[u] = k;
-    }
-}
-__global__ void k_csc_fill(const int32_t* __restrict__ src_pos, const int32_t* __restrict__ src_mb, const int64_t* cnt,
-                           const int64_t* __restrict__ ft_indptr, const int32_t* __restrict__ ft_nbr,
-                           const uint32_t* __restrict__ dstbits, int64_t W, const RankSet R, int l,
-                           const int64_t* __restrict__ t_indptr, int32_t* __restrict__ t_idx) {
-    const int64_t n = cnt[1];
-    for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < n; u += (int64_t)gridDim.x * blockDim.x) {
-        const int32_t p = src_pos[u];
-        const int j = src_mb[u];
-        const uint32_t* db = dstbits + (int64_t)j * W;
-        int64_t o = t_indptr[u];
-        for (int64_t e = ft_indptr[p], ee = ft_indptr[p + 1]; e < ee; ++e) {
-            const int32_t q = ft_nbr[e];
-            if ((db[q >> 5] >> (q & 31)) & 1u) t_idx[o++] = (int32_t)dst_id(R, l, j, q);
+        if (s < cap_src) {
+            src_pos[s] = p; src_gid[s] = fsrc_gid[p]; src_mb[s] = j;
+            if (tcnt) tcnt[s] = 0;
         }
     }
 }
@@ -784,31 +738,43 @@ void extract_group(betty_ctx* ctx, const ExtractArgs& a, cudaStream_t s) {
         if (l == 0 && a.lean0 && F.egid && B.egid) {
             // lean layer 0: the dst prefix (self rows) and the edges' source gids, nothing else
             k_emit_dst<<<grid_for(ctx, cap_d, 256), 256, 0, s>>>(dst_pos, row_mb, B.cnt, dst_off, B.mb_src_off,
-                                                                 F.src_gid, B.src_pos, B.src_gid, B.src_mb, cap_s);
+                                                                 F.src_gid, B.src_pos, B.src_gid, B.src_mb, cap_s,
+                                                                 nullptr);
             k_seg_egid<<<grid_for(ctx, (cap_d + 31) / 32 * 32, 256), 256, 0, s>>>(dst_pos, B.cnt, F.indptr, F.egid,
                                                                                   B.indptr, B.egid, cap_e, ctx->dev_err);
             break;
         }
         // dedupe: dst bitmap + position map, then new-source bitmap
         k_mark_dst<<<grid_for(ctx, cap_d, 256), 256, 0, s>>>(dst_pos, row_mb, B.cnt, a.sc.dstbits, W);
-        const int g_rows = grid_for(ctx, cap_d, 256);       // 32 rows per warp
+        // rows per claim: 32 while the layer fills every resident warp (148 SMs x 64) with 32-row
+        // claims, else fewer (down to 8) so that the edge walk spreads over more warps
+        const int64_t warps_res = (int64_t)ctx->num_sms * 64;
+        int claim = 32;
+        static const bool fixed_claim = getenv("BETTY_CLAIM32") != nullptr;      // A/B switch
+        while (!fixed_claim && claim > 8 && cap_d < warps_res * claim / 2) claim >>= 1;
+        const int g_rows = grid_for(ctx, (cap_d * 32 + claim - 1) / claim, 256);
         unsigned* ctr = ctx->L().counters + CTR_EXTRACT;
         cudaMemsetAsync(ctr, 0, sizeof(unsigned), s);
         // mark_nocheck: mark every neighbour (no dst lookup per edge); the dst rows are masked out of
         // the bitmap words by the rank pass instead
         static const bool mark_nocheck = getenv("BETTY_MARK_NOCHECK") && atoi(getenv("BETTY_MARK_NOCHECK"));
         k_mark_new<<<g_rows, 256, 0, s>>>(dst_pos, row_mb, B.cnt, F.indptr, F.nbr, mark_nocheck ? nullptr : a.sc.dstbits,
-                                          a.sc.newbits, W, otab, ctr);
+                                          a.sc.newbits, W, otab, ctr, claim);
         // ascending order of new sources = popcount scan over the bitmap words
         int64_t* csum = a.sc.wordoff;                   // chunk sums, then slot totals at the end
         int64_t* slot_tot = a.sc.wordoff + (int64_t)c * ((W + RANK_CHUNK - 1) / RANK_CHUNK + 1);
         slot_rank(a.sc.newbits, mark_nocheck ? a.sc.dstbits : nullptr, c, W, csum, a.sc.nrank[l], slot_tot, s);
+        // CSC column lengths of this layer: counted by the relabel pass (a histogram of the local
+        // source ids it writes) unless BETTY_CSC_COUNT=flat (a separate pass over the full-batch CSC)
+        const bool want_csc = B.t_indptr && (a.csc_mask >> l & 1);
+        static const bool flat_count = getenv("BETTY_CSC_COUNT") && !strcmp(getenv("BETTY_CSC_COUNT"), "flat");
+        int32_t* hist = (want_csc && F.t_indptr && !flat_count) ? a.sc.tcnt : nullptr;
         k_counts<<<1, 1024, 0, s>>>(dst_off, slot_tot, c, B.mb_src_off, B.cnt, cap_s, cap_e,
                                     l > 0 ? a.layers[l - 1].cnt : nullptr, ctx->dev_err);
         k_emit_dst<<<grid_for(ctx, cap_d, 256), 256, 0, s>>>(dst_pos, row_mb, B.cnt, dst_off, B.mb_src_off,
-                                                             F.src_gid, B.src_pos, B.src_gid, B.src_mb, cap_s);
+                                                             F.src_gid, B.src_pos, B.src_gid, B.src_mb, cap_s, hist);
         k_emit_new<<<grid_for(ctx, cW, 256), 256, 0, s>>>(a.sc.nrank[l], W, c, B.cnt, dst_off, B.mb_src_off,
-                                                          F.src_gid, B.src_pos, B.src_gid, B.src_mb, cap_s);
+                                                          F.src_gid, B.src_pos, B.src_gid, B.src_mb, cap_s, hist);
         // rank structures of this layer (and of the outputs at the top layer)
         if (l == a.L - 1) slot_rank(a.sc.dstbits, nullptr, c, W, csum, a.sc.drank_top, nullptr, s);
         RankSet R{};
@@ -824,12 +790,12 @@ void extract_group(betty_ctx* ctx, const ExtractArgs& a, cudaStream_t s) {
         R.top_off = a.sc.top_dst_off;
         cudaMemsetAsync(ctr + 1, 0, sizeof(unsigned), s);
         k_relabel<<<g_rows, 256, 0, s>>>(dst_pos, row_mb, B.cnt, F.indptr, F.nbr, B.indptr, R, l, B.indices, cap_e,
-                                         F.src_gid, B.egid, otab, ctr + 1);
-        const bool want_csc = B.t_indptr && (a.csc_mask >> l & 1);
+                                         F.src_gid, B.egid, otab, ctr + 1, claim, hist, cap_s);
         if (want_csc && F.t_indptr) {           // from the full-batch CSC (needs the dst bitmap + map)
             const int g_src = grid_for(ctx, (cap_s + 31) / 32 * 32, 256);
-            k_csc_flat<false><<<g_src, 256, 0, s>>>(B.src_pos, B.src_mb, B.cnt, F.t_indptr, F.t_nbr, a.sc.dstbits, W,
-                                                    R, l, nullptr, nullptr, a.sc.tcnt);
+            if (!hist)
+                k_csc_flat<false><<<g_src, 256, 0, s>>>(B.src_pos, B.src_mb, B.cnt, F.t_indptr, F.t_nbr, a.sc.dstbits,
+                                                        W, R, l, nullptr, nullptr, a.sc.tcnt);
             scan_i32(ctx, a.sc.tcnt, B.t_indptr, B.cnt + 1, 0, cap_s, nullptr, s);
             k_csc_flat<true><<<g_src, 256, 0, s>>>(B.src_pos, B.src_mb, B.cnt, F.t_indptr, F.t_nbr, a.sc.dstbits, W,
                                                    R, l, B.t_indptr, B.t_indices, nullptr);
