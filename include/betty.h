@@ -137,7 +137,10 @@ BETTY_API void betty_csr_free(betty_ctx* ctx, betty_csr* reg);
  * be NULL).  part[n_out] (device) assigns each output position to [0,K).
  * Fills mb[L] with micro-batch k (all arrays allocated, CSC included,
  * sizes written on the host after one stream synchronisation).  part values
- * out of range return EINVAL.  An empty micro-batch yields zero-sized blocks. */
+ * out of range return EINVAL.  An empty micro-batch yields zero-sized blocks.
+ * Limits of the output selection: K <= 16384, n_out < 2^23 - 1 and fewer than
+ * 2^40 top-layer edges, else BETTY_EUNSUPPORTED (also for betty_mb_sizes and
+ * betty_plan_create, whose launch groups hold <= 512 micro-batches). */
 BETTY_API betty_status betty_extract_blocks(betty_ctx* ctx, const betty_block* full, int32_t L, const int32_t* part,
                                   int64_t n_out, int32_t K, int32_t k, betty_block* mb, betty_stream stream);
 BETTY_API void betty_block_free(betty_ctx* ctx, betty_block* blocks, int32_t L);

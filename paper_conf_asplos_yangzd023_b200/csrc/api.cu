@@ -159,7 +159,7 @@ static bool alloc_extract(Arena& A, int L, const ExtractFull* full, int64_t n_ou
                           const std::vector<int64_t>& cap_e, uint32_t csc_mask, ExtractSet* X) {
     X->layers.assign(L, ExtractLayer{});
     X->cnt_all = A.get<int64_t>(L * 4);
-    int64_t max_src = 1, max_dst = 1;
+    int64_t max_src = 1;
     for (int l = 0; l < L; ++l) {
         ExtractLayer& B = X->layers[l];
         B.cap_dst = std::max<int64_t>(cap_dst[l], 1);
@@ -178,22 +178,20 @@ static bool alloc_extract(Arena& A, int L, const ExtractFull* full, int64_t n_ou
         B.mb_src_off = A.get<int64_t>(c + 1);
         if (l + 1 < L) B.order_tab = A.get<int64_t>(2 * (ORDER_TAB_MAX + 1) + 1);
         max_src = std::max(max_src, std::max(full[l].n_src, B.cap_src));
-        max_dst = std::max(max_dst, B.cap_dst);
     }
     int64_t max_full = 1;
     for (int l = 0; l < L; ++l) max_full = std::max(max_full, full[l].n_src);
     const int64_t W = (max_full + 31) / 32 + 1;
-    const int64_t nchunks = (n_out + 1023) / 1024 + 1;
+    const int64_t nchunks = (n_out + SEL_CHUNK - 1) / SEL_CHUNK + 1;
     ExtractScratch& sc = X->sc;
     sc.dstbits = A.get<uint32_t>(c * W);
     sc.newbits = A.get<uint32_t>(c * W);
     for (int l = 0; l < L; ++l) sc.nrank[l] = A.get<uint2>(c * ((full[l].n_src + 31) / 32));
     sc.drank_top = A.get<uint2>(c * ((full[L - 1].n_src + 31) / 32));
-    sc.wordcnt = A.get<int32_t>(c * W);
     sc.wordoff = A.get<int64_t>(c * W + 1);
-    sc.deg = A.get<int64_t>(max_dst);
     sc.tcnt = A.get<int32_t>(max_src);
-    sc.sel_cnt = A.get<int32_t>(c * nchunks);
+    sc.ndeg = A.get<int32_t>(max_src);
+    sc.sel_cnt = A.get<int64_t>(c * nchunks);
     sc.sel_off = A.get<int64_t>(c * nchunks + 1);
     sc.top_dst_pos = A.get<int32_t>(std::max<int64_t>(n_out, 1));
     sc.top_row_mb = A.get<int32_t>(std::max<int64_t>(n_out, 1));
@@ -237,6 +235,8 @@ extern "C" betty_status betty_extract_blocks(betty_ctx* c, const betty_block* fu
     if (st) return st;
     if (!mb || (n_out > 0 && !part) || K < 1 || k < 0 || k >= K || full[L - 1].n_dst != n_out)
         return fail(c, BETTY_EINVAL, "extract: bad part / K / k / n_out");
+    if (!extract_limits_ok(K, 1, n_out, full[L - 1].n_edges))
+        return fail(c, BETTY_EUNSUPPORTED, "extract: K > 16384, n_out >= 2^23 or >= 2^40 top-layer edges");
     std::vector<ExtractFull> F = to_full(full, L);
     std::vector<int64_t> cd(L), cs(L), ce(L);
     for (int l = 0; l < L; ++l) { cd[l] = full[l].n_dst; cs[l] = full[l].n_src; ce[l] = full[l].n_edges; }
@@ -784,6 +784,10 @@ extern "C" betty_status betty_plan_create(betty_ctx* c, const betty_model* model
     p->m = m; p->L = L; p->K = K; p->flags = flags; p->n_out = n_out; p->part = part;
     p->full = to_full(full, L);
     p->c = group <= 0 ? std::max(1, n_my) : std::min(group, std::max(1, n_my));
+    if (!extract_limits_ok(K, p->c, n_out, full[L - 1].n_edges)) {
+        delete p;
+        return fail(c, BETTY_EUNSUPPORTED, "plan: K > 16384, launch group > 512, n_out >= 2^23 or >= 2^40 top-layer edges");
+    }
     for (int i = 0; i < n_my; i += p->c)
         p->groups.emplace_back(my_k + i, my_k + std::min(n_my, i + p->c));
     p->csc_mask = 0;
@@ -882,7 +886,7 @@ extern "C" betty_status betty_plan_create(betty_ctx* c, const betty_model* model
         int64_t maxfull = 1;
         for (int l = 0; l < L; ++l) maxfull = std::max(maxfull, full[l].n_src);
         mx = std::max(mx, (int64_t)p->c * ((maxfull + 31) / 32 + 1));
-        mx = std::max(mx, (int64_t)p->c * ((n_out + 1023) / 1024 + 1));
+        mx = std::max(mx, (int64_t)p->c * ((n_out + SEL_CHUNK - 1) / SEL_CHUNK + 1));
         ensure_scan_scratch(c, mx, s);
     }
     // ---- REG inside the step (once here to size its buffers): all rows until betty_plan_set_reg_rows
@@ -1100,6 +1104,8 @@ extern "C" betty_status betty_mb_sizes(betty_ctx* c, const betty_block* full, in
     if (st) return st;
     if (K < 1 || !sizes || full[L - 1].n_dst != n_out || (n_out > 0 && !part))
         return fail(c, BETTY_EINVAL, "mb_sizes: bad K / sizes / n_out / part");
+    if (!extract_limits_ok(K, 1, n_out, full[L - 1].n_edges))
+        return fail(c, BETTY_EUNSUPPORTED, "mb_sizes: K > 16384, n_out >= 2^23 or >= 2^40 top-layer edges");
     std::vector<ExtractFull> F = to_full(full, L);
     std::vector<int32_t> ks(K);
     for (int k = 0; k < K; ++k) ks[k] = k;

@@ -31,63 +31,129 @@
 namespace betty {
 
 // ----------------------------------------------------------- output select
-constexpr int SEL_CHUNK = 1024;
+// Output selection V_k (Alg. 1 line 9: the outputs of micro-batch k, ascending),
+// for all c slots of a launch group at once, with the top layer's indptr and dst bitmap produced on
+// the way.  Two passes over part[], one CTA per SEL_CHUNK-output chunk; an output's slot comes from
+// a K-entry table in shared memory.  Pass 1 accumulates, per slot, the chunk's selected outputs and
+// their top-layer degrees, packed as count << SEL_SHIFT | degree sum, so that ONE int64 scan gives
+// both the dst positions and the indptr offsets.  Pass 2 (one warp per chunk, SEL_CHUNK / 32 steps
+// of 32 outputs, ascending) writes each selected output's position, slot, indptr entry and dst bit.
+constexpr int SEL_KMAX = 16384, SEL_CMAX = 512, SEL_SHIFT = 40;
+constexpr int64_t SEL_DEG_MASK = (1ll << SEL_SHIFT) - 1;
 
-__global__ void k_sel_count(const int32_t* __restrict__ part, int64_t n_out, int32_t K, const int32_t* __restrict__ ks,
-                            int32_t c, int32_t* __restrict__ chunk_cnt, int64_t nchunks, int* dev_err) {
-    __shared__ int s[32];
-    const int j = blockIdx.y;
-    const int32_t k = ks[j];
-    for (int64_t ch = blockIdx.x; ch < nchunks; ch += gridDim.x) {
-        int local = 0;
-        for (int64_t i = ch * SEL_CHUNK + threadIdx.x; i < mn64((ch + 1) * SEL_CHUNK, n_out); i += blockDim.x) {
-            const int32_t p = part[i];
-            if (j == 0 && (p < 0 || p >= K)) atomicOr(dev_err, DEVERR_BAD_PART);
-            local += (p == k);
-        }
-        int w = warp_sum(local);
-        if (lane_id() == 0) s[warp_id()] = w;
-        __syncthreads();
-        if (threadIdx.x == 0) {
-            int t = 0;
-            for (int i = 0; i < (int)(blockDim.x >> 5); ++i) t += s[i];
-            chunk_cnt[(int64_t)j * nchunks + ch] = t;
-        }
-        __syncthreads();
-    }
+__device__ __forceinline__ void sel_slot_table(int16_t* tab, const int32_t* __restrict__ ks, int c, int K) {
+    for (int k = threadIdx.x; k < K; k += blockDim.x) tab[k] = -1;
+    __syncthreads();
+    for (int j = threadIdx.x; j < c; j += blockDim.x) tab[ks[j]] = (int16_t)j;
+    __syncthreads();
 }
 
-// each thread handles SEL_CHUNK/blockDim.x consecutive outputs of the chunk
-__global__ void __launch_bounds__(256) k_sel_write(const int32_t* __restrict__ part, int64_t n_out,
-                                                   const int32_t* __restrict__ ks, const int64_t* __restrict__ off,
-                                                   int64_t nchunks, int32_t* __restrict__ dst_pos,
-                                                   int32_t* __restrict__ row_mb) {
-    __shared__ int64_t s_warp[9];
-    const int j = blockIdx.y;
-    const int32_t k = ks[j];
+__global__ void __launch_bounds__(256) k_sel_count(const int32_t* __restrict__ part, int64_t n_out, int32_t K,
+                                                   const int32_t* __restrict__ ks, int32_t c,
+                                                   const int64_t* __restrict__ findptr, int64_t* __restrict__ sel_cnt,
+                                                   int64_t nchunks, int* dev_err) {
+    __shared__ int16_t s_tab[SEL_KMAX];
+    __shared__ unsigned long long s_acc[SEL_CMAX];
+    sel_slot_table(s_tab, ks, c, K);
+    for (int j = threadIdx.x; j < c; j += blockDim.x) s_acc[j] = 0ull;
+    __syncthreads();
+    const int64_t ch = blockIdx.x;
+    const int64_t end = mn64((ch + 1) * SEL_CHUNK, n_out);
     constexpr int PER = SEL_CHUNK / 256;
-    for (int64_t ch = blockIdx.x; ch < nchunks; ch += gridDim.x) {
-        const int64_t b = ch * SEL_CHUNK + (int64_t)threadIdx.x * PER;
-        int flags = 0, cnt = 0;
+    int32_t p[PER];
 #pragma unroll
-        for (int t = 0; t < PER; ++t) {
-            const bool f = (b + t < n_out) && part[b + t] == k;
-            flags |= (int)f << t;
-            cnt += f;
-        }
-        int64_t tot;
-        int64_t pos = off[(int64_t)j * nchunks + ch] + block_excl_scan<int64_t>(cnt, s_warp, &tot);
-#pragma unroll
-        for (int t = 0; t < PER; ++t)
-            if (flags >> t & 1) { dst_pos[pos] = (int32_t)(b + t); row_mb[pos] = j; ++pos; }
+    for (int t = 0; t < PER; ++t) {                    // all loads in flight at once
+        const int64_t i = ch * SEL_CHUNK + t * 256 + threadIdx.x;
+        p[t] = i < end ? part[i] : -2;
     }
+    int j[PER];
+    int64_t d[PER];
+#pragma unroll
+    for (int t = 0; t < PER; ++t) {
+        const int64_t i = ch * SEL_CHUNK + t * 256 + threadIdx.x;
+        j[t] = -1;
+        d[t] = 0;
+        if (p[t] == -2) continue;
+        if (p[t] < 0 || p[t] >= K) { atomicOr(dev_err, DEVERR_BAD_PART); continue; }
+        j[t] = s_tab[p[t]];
+        if (j[t] >= 0) d[t] = findptr[i + 1] - findptr[i];
+    }
+#pragma unroll
+    for (int t = 0; t < PER; ++t)
+        if (j[t] >= 0) atomicAdd(&s_acc[j[t]], (1ull << SEL_SHIFT) + (unsigned long long)d[t]);
+    __syncthreads();
+    for (int j = threadIdx.x; j < c; j += blockDim.x) sel_cnt[(int64_t)j * nchunks + ch] = (int64_t)s_acc[j];
 }
 
-// single CTA: per-slot dst offsets of the output layer
-__global__ void k_sel_offsets(const int64_t* __restrict__ off, int64_t nchunks, int32_t c, int64_t* mb_dst_off,
-                              int64_t* cnt) {
-    for (int j = threadIdx.x; j <= c; j += blockDim.x) mb_dst_off[j] = off[(int64_t)j * nchunks];
-    if (threadIdx.x == 0) cnt[0] = off[(int64_t)c * nchunks];
+__global__ void __launch_bounds__(32) k_sel_write(const int32_t* __restrict__ part, int64_t n_out, int32_t K,
+                                                  const int32_t* __restrict__ ks, int32_t c,
+                                                  const int64_t* __restrict__ findptr, const int64_t* __restrict__ off,
+                                                  int64_t nchunks, int32_t* __restrict__ dst_pos,
+                                                  int32_t* __restrict__ row_mb, int64_t* __restrict__ indptr,
+                                                  int64_t cap_d, uint32_t* dstbits, int64_t W,
+                                                  int64_t* __restrict__ mb_dst_off, int64_t* cnt, int* dev_err) {
+    __shared__ int16_t s_tab[SEL_KMAX];
+    __shared__ int64_t s_pos[SEL_CMAX], s_deg[SEL_CMAX];
+    __shared__ int64_t s_d[32];
+    sel_slot_table(s_tab, ks, c, K);
+    const int lane = threadIdx.x;
+    const int64_t ch = blockIdx.x;
+    for (int j = lane; j < c; j += 32) {
+        const int64_t o = off[(int64_t)j * nchunks + ch];
+        s_pos[j] = o >> SEL_SHIFT;
+        s_deg[j] = o & SEL_DEG_MASK;
+    }
+    if (ch == 0) {                                      // per-slot offsets, totals, indptr[n]
+        for (int j = lane; j <= c; j += 32) mb_dst_off[j] = off[(int64_t)j * nchunks] >> SEL_SHIFT;
+        if (lane == 0) {
+            const int64_t t = off[(int64_t)c * nchunks], n = t >> SEL_SHIFT;
+            cnt[0] = n;
+            cnt[2] = t & SEL_DEG_MASK;
+            if (n <= cap_d) indptr[n] = t & SEL_DEG_MASK;
+            else atomicOr(dev_err, DEVERR_OVERFLOW);
+        }
+    }
+    const int64_t base = ch * SEL_CHUNK;
+    const int nloc = (int)mn64(SEL_CHUNK, n_out - base);
+    // the chunk's slots and degrees first, every load in flight at once (lane = output of a step)
+    constexpr int STEPS = SEL_CHUNK / 32;
+    int32_t pp[STEPS], ds[STEPS];
+#pragma unroll
+    for (int t = 0; t < STEPS; ++t) {
+        const int64_t i = base + t * 32 + lane;
+        const bool in = t * 32 + lane < nloc;
+        pp[t] = in ? part[i] : -1;
+        ds[t] = in ? (int32_t)(findptr[i + 1] - findptr[i]) : 0;
+    }
+    int16_t js[STEPS];
+#pragma unroll
+    for (int t = 0; t < STEPS; ++t) js[t] = (pp[t] >= 0 && pp[t] < K) ? s_tab[pp[t]] : (int16_t)-1;
+    __syncwarp();
+#pragma unroll
+    for (int t = 0; t < STEPS; ++t) {
+        if (t * 32 >= nloc) break;
+        const int64_t i = base + t * 32 + lane;
+        const int j = js[t];
+        const int64_t d = j >= 0 ? ds[t] : 0;
+        const unsigned m = __match_any_sync(0xffffffffu, j);
+        const unsigned lower = m & ((1u << lane) - 1u);
+        s_d[lane] = d;
+        __syncwarp();
+        if (j >= 0) {
+            int64_t db = 0;                             // degrees of the same slot's earlier outputs in this step
+            for (unsigned b = lower; b; b &= b - 1u) db += s_d[__ffs(b) - 1];
+            const int64_t pos = s_pos[j] + __popc(lower);
+            if (pos < cap_d) {
+                dst_pos[pos] = (int32_t)i;
+                row_mb[pos] = j;
+                indptr[pos] = s_deg[j] + db;
+            }
+            if (dstbits) atomicOr(&dstbits[(int64_t)j * W + (i >> 5)], 1u << (i & 31));
+            __syncwarp(m);
+            if (lane == 31 - __clz(m)) { s_pos[j] += __popc(m); s_deg[j] += db + d; }
+        }
+        __syncwarp();
+    }
 }
 
 // ------------------------------------------------------------ per layer
@@ -538,11 +604,15 @@ __global__ void k_counts(const int64_t* __restrict__ mb_dst_off, const int64_t* 
     }
 }
 
+// The emit kernels write a layer's src list (dst prefix, then the new sources ascending) and, on
+// the way, zero the CSC column counts (tcnt) and record each source's full-batch degree in the
+// layer below (ndeg: the next layer's dst degrees, so its indptr is a plain scan, not a gather).
 __global__ void k_emit_new(const uint2* __restrict__ nrank, int64_t W, int32_t c, const int64_t* n_dst_tot,
                            const int64_t* __restrict__ mb_dst_off,
                            const int64_t* __restrict__ mb_src_off, const int32_t* __restrict__ fsrc_gid,
                            int32_t* __restrict__ src_pos, int32_t* __restrict__ src_gid, int32_t* __restrict__ src_mb,
-                           int64_t cap_src, int32_t* __restrict__ tcnt) {
+                           int64_t cap_src, int32_t* __restrict__ tcnt, const int64_t* __restrict__ nfindptr,
+                           int32_t* __restrict__ ndeg) {
     const int64_t n = (int64_t)c * W;
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
         const uint2 r = nrank[i];
@@ -559,6 +629,7 @@ __global__ void k_emit_new(const uint2* __restrict__ nrank, int64_t W, int32_t c
             if (s < cap_src) {
                 src_pos[s] = p; src_gid[s] = fsrc_gid[p]; src_mb[s] = j;
                 if (tcnt) tcnt[s] = 0;
+                if (ndeg) ndeg[s] = (int32_t)(nfindptr[p + 1] - nfindptr[p]);
             }
             ++s;
         }
@@ -569,7 +640,8 @@ __global__ void k_emit_dst(const int32_t* __restrict__ dst_pos, const int32_t* _
                            const int64_t* cnt, const int64_t* __restrict__ mb_dst_off,
                            const int64_t* __restrict__ mb_src_off, const int32_t* __restrict__ fsrc_gid,
                            int32_t* __restrict__ src_pos, int32_t* __restrict__ src_gid, int32_t* __restrict__ src_mb,
-                           int64_t cap_src, int32_t* __restrict__ tcnt) {
+                           int64_t cap_src, int32_t* __restrict__ tcnt, const int64_t* __restrict__ nfindptr,
+                           int32_t* __restrict__ ndeg) {
     const int64_t n = cnt[0];
     for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < n; r += (int64_t)gridDim.x * blockDim.x) {
         const int j = row_mb[r];
@@ -579,6 +651,7 @@ __global__ void k_emit_dst(const int32_t* __restrict__ dst_pos, const int32_t* _
         if (s < cap_src) {
             src_pos[s] = p; src_gid[s] = fsrc_gid[p]; src_mb[s] = j;
             if (tcnt) tcnt[s] = 0;
+            if (ndeg) ndeg[s] = (int32_t)(nfindptr[p + 1] - nfindptr[p]);
         }
     }
 }
@@ -695,10 +768,15 @@ static inline int grid_for(betty_ctx* c, int64_t work, int threads, int per_sm =
     return (int)std::max<int64_t>(1, std::min<int64_t>((work + threads - 1) / threads, (int64_t)c->num_sms * per_sm));
 }
 
+bool extract_limits_ok(int32_t K, int32_t c, int64_t n_out, int64_t top_edges) {
+    return K >= 1 && K <= SEL_KMAX && c >= 1 && c <= SEL_CMAX && n_out < (1ll << (63 - SEL_SHIFT)) - 1 &&
+           top_edges < (1ll << SEL_SHIFT);
+}
+
 size_t extract_scratch_bytes(int64_t c, int64_t max_full_src, int64_t sel_nchunks) {
     const int64_t W = (max_full_src + 31) / 32 + 1;
     return (size_t)(c * W * 4 * 2 + c * max_full_src * 4 + (c * W + 1) * 8 + c * W * 4 +
-                    (c * sel_nchunks + 1) * 8 + c * sel_nchunks * 4 + 4096);
+                    (c * sel_nchunks + 1) * 8 + c * sel_nchunks * 8 + 4096);
 }
 
 void extract_group(betty_ctx* ctx, const ExtractArgs& a, cudaStream_t s) {
@@ -707,13 +785,18 @@ void extract_group(betty_ctx* ctx, const ExtractArgs& a, cudaStream_t s) {
     const int64_t nchunks = (n_out + SEL_CHUNK - 1) / SEL_CHUNK;
     ExtractLayer* top = &a.layers[a.L - 1];
 
-    // ---- V_k: outputs with part == ks[j], ascending, for every slot j
+    // ---- V_k: outputs with part == ks[j], ascending, for every slot j (+ the top layer's indptr,
+    // counts and dst bitmap; the bitmap only when the top layer is not extracted lean)
+    const bool top_lean = a.L == 1 && a.lean0 && a.full[0].egid && top->egid;
     {
-        dim3 g((unsigned)std::max<int64_t>(1, std::min<int64_t>(nchunks, 1024)), (unsigned)c);
-        k_sel_count<<<g, 256, 0, s>>>(a.part, n_out, a.K, a.ks, c, a.sc.sel_cnt, nchunks, ctx->dev_err);
-        scan_i32(ctx, a.sc.sel_cnt, a.sc.sel_off, nullptr, (int64_t)c * nchunks, 0, nullptr, s);
-        k_sel_write<<<g, 256, 0, s>>>(a.part, n_out, a.ks, a.sc.sel_off, nchunks, a.sc.top_dst_pos, a.sc.top_row_mb);
-        k_sel_offsets<<<1, 256, 0, s>>>(a.sc.sel_off, nchunks, c, a.sc.top_dst_off, top->cnt);
+        const unsigned g = (unsigned)std::max<int64_t>(1, nchunks);
+        k_sel_count<<<g, 256, 0, s>>>(a.part, n_out, a.K, a.ks, c, a.full[a.L - 1].indptr, a.sc.sel_cnt, nchunks,
+                                      ctx->dev_err);
+        scan_i64(ctx, a.sc.sel_cnt, a.sc.sel_off, nullptr, (int64_t)c * nchunks, 0, nullptr, s);
+        k_sel_write<<<g, 32, 0, s>>>(a.part, n_out, a.K, a.ks, c, a.full[a.L - 1].indptr, a.sc.sel_off, nchunks,
+                                     a.sc.top_dst_pos, a.sc.top_row_mb, top->indptr, top->cap_dst,
+                                     top_lean ? nullptr : a.sc.dstbits, (a.full[a.L - 1].n_src + 31) / 32,
+                                     a.sc.top_dst_off, top->cnt, ctx->dev_err);
     }
 
     const int32_t* dst_pos = a.sc.top_dst_pos;
@@ -734,18 +817,19 @@ void extract_group(betty_ctx* ctx, const ExtractArgs& a, cudaStream_t s) {
             otab = B.order_tab;
         }
         // rows: degree of each dst row in the full batch -> local indptr
-        scan_deg(ctx, dst_pos, F.indptr, B.indptr, B.cnt + 0, cap_d, B.cnt + 2, s);
+        const bool top = l == a.L - 1;                  // its indptr / counts / dst bits come from the selection
+        if (!top) scan_i32(ctx, a.sc.ndeg, B.indptr, B.cnt + 0, 0, cap_d, B.cnt + 2, s);   // degrees: emit kernels above
         if (l == 0 && a.lean0 && F.egid && B.egid) {
             // lean layer 0: the dst prefix (self rows) and the edges' source gids, nothing else
             k_emit_dst<<<grid_for(ctx, cap_d, 256), 256, 0, s>>>(dst_pos, row_mb, B.cnt, dst_off, B.mb_src_off,
                                                                  F.src_gid, B.src_pos, B.src_gid, B.src_mb, cap_s,
-                                                                 nullptr);
+                                                                 nullptr, nullptr, nullptr);
             k_seg_egid<<<grid_for(ctx, (cap_d + 31) / 32 * 32, 256), 256, 0, s>>>(dst_pos, B.cnt, F.indptr, F.egid,
                                                                                   B.indptr, B.egid, cap_e, ctx->dev_err);
             break;
         }
         // dedupe: dst bitmap + position map, then new-source bitmap
-        k_mark_dst<<<grid_for(ctx, cap_d, 256), 256, 0, s>>>(dst_pos, row_mb, B.cnt, a.sc.dstbits, W);
+        if (!top) k_mark_dst<<<grid_for(ctx, cap_d, 256), 256, 0, s>>>(dst_pos, row_mb, B.cnt, a.sc.dstbits, W);
         // rows per claim: 32 while the layer fills every resident warp (148 SMs x 64) with 32-row
         // claims, else fewer (down to 8) so that the edge walk spreads over more warps
         const int64_t warps_res = (int64_t)ctx->num_sms * 64;
@@ -769,12 +853,16 @@ void extract_group(betty_ctx* ctx, const ExtractArgs& a, cudaStream_t s) {
         const bool want_csc = B.t_indptr && (a.csc_mask >> l & 1);
         static const bool flat_count = getenv("BETTY_CSC_COUNT") && !strcmp(getenv("BETTY_CSC_COUNT"), "flat");
         int32_t* hist = (want_csc && F.t_indptr && !flat_count) ? a.sc.tcnt : nullptr;
+        const int64_t* nfi = l > 0 ? a.full[l - 1].indptr : nullptr;     // the layer below's dst degrees
+        int32_t* ndeg = l > 0 ? a.sc.ndeg : nullptr;
         k_counts<<<1, 1024, 0, s>>>(dst_off, slot_tot, c, B.mb_src_off, B.cnt, cap_s, cap_e,
                                     l > 0 ? a.layers[l - 1].cnt : nullptr, ctx->dev_err);
         k_emit_dst<<<grid_for(ctx, cap_d, 256), 256, 0, s>>>(dst_pos, row_mb, B.cnt, dst_off, B.mb_src_off,
-                                                             F.src_gid, B.src_pos, B.src_gid, B.src_mb, cap_s, hist);
+                                                             F.src_gid, B.src_pos, B.src_gid, B.src_mb, cap_s, hist,
+                                                             nfi, ndeg);
         k_emit_new<<<grid_for(ctx, cW, 256), 256, 0, s>>>(a.sc.nrank[l], W, c, B.cnt, dst_off, B.mb_src_off,
-                                                          F.src_gid, B.src_pos, B.src_gid, B.src_mb, cap_s, hist);
+                                                          F.src_gid, B.src_pos, B.src_gid, B.src_mb, cap_s, hist,
+                                                          nfi, ndeg);
         // rank structures of this layer (and of the outputs at the top layer)
         if (l == a.L - 1) slot_rank(a.sc.dstbits, nullptr, c, W, csum, a.sc.drank_top, nullptr, s);
         RankSet R{};

@@ -80,11 +80,10 @@ struct ExtractScratch {
     // local id is then computed (no position -> id map): see src_id() in extract.cu
     uint2* nrank[16];           // [c*W_l]
     uint2* drank_top;           // [c*W_{L-1}]
-    int32_t* wordcnt;           // [c*Wmax]
     int64_t* wordoff;           // [c*Wmax+1]
-    int64_t* deg;               // [max cap_dst]
     int32_t* tcnt;              // [max cap_src]
-    int32_t* sel_cnt;           // [c*nchunks]
+    int32_t* ndeg;              // [max cap_src]: full-batch degrees of the next layer's dst rows
+    int64_t* sel_cnt;           // [c*nchunks] (selection: count << 40 | degree sum, per slot and chunk)
     int64_t* sel_off;           // [c*nchunks+1]
     int32_t* top_dst_pos;       // [n_out]
     int32_t* top_row_mb;        // [n_out]
@@ -110,5 +109,10 @@ struct ExtractArgs {
 };
 
 void extract_group(betty_ctx* ctx, const ExtractArgs& a, cudaStream_t s);
+// outputs per selection chunk (one CTA each; 256: 8 serial steps per warp in the write pass)
+constexpr int SEL_CHUNK = 256;
+// the selection's limits (extract.cu): K <= 16384 micro-batches, launch groups of <= 512, fewer than
+// 2^23 - 1 outputs and 2^40 top-layer edges
+bool extract_limits_ok(int32_t K, int32_t c, int64_t n_out, int64_t top_edges);
 
 }  // namespace betty

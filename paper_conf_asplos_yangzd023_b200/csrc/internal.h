@@ -51,11 +51,6 @@ void scan_i64(betty_ctx* c, const int64_t* in, int64_t* out, const int64_t* n_de
               int64_t* total_dev, cudaStream_t s);
 void scan_i32(betty_ctx* c, const int32_t* in, int64_t* out, const int64_t* n_dev, int64_t n_fixed, int64_t n_cap,
               int64_t* total_dev, cudaStream_t s);
-// exclusive scans with fused element loads: popcounts of bitmap words (n words, fixed) and
-// degrees indptr[rows[i]+1] - indptr[rows[i]] of gathered rows (count on the device)
-void scan_popc(betty_ctx* c, const uint32_t* bits, int64_t* out, int64_t n, cudaStream_t s);
-void scan_deg(betty_ctx* c, const int32_t* rows, const int64_t* indptr, int64_t* out, const int64_t* n_dev,
-              int64_t n_cap, int64_t* total_dev, cudaStream_t s);
 // sort each segment [ptr[i], ptr[i+1]) of keys ascending, i < *nseg_dev (or nseg_fixed)
 void segsort_i32(betty_ctx* c, const int64_t* ptr, int32_t* keys, const int64_t* nseg_dev, int64_t nseg_fixed,
                  int64_t nseg_cap, cudaStream_t s);

@@ -24,21 +24,10 @@ __device__ __forceinline__ void st_release(unsigned long long* p, unsigned long 
     asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
-// element loaders of the scan: plain values, popcounts of bitmap words, degrees of gathered rows
+// element loader of the scan: plain values
 template <typename Tin> struct LdPlain {
     const Tin* in;
     __device__ __forceinline__ int64_t operator()(int64_t i) const { return (int64_t)in[i]; }
-};
-struct LdPopc {
-    const uint32_t* bits;
-    __device__ __forceinline__ int64_t operator()(int64_t i) const { return __popc(bits[i]); }
-};
-struct LdDeg {
-    const int32_t* rows; const int64_t* indptr;
-    __device__ __forceinline__ int64_t operator()(int64_t i) const {
-        const int32_t p = rows[i];
-        return indptr[p + 1] - indptr[p];
-    }
 };
 
 template <typename Ld>
@@ -163,13 +152,6 @@ void scan_i64(betty_ctx* c, const int64_t* in, int64_t* out, const int64_t* n_de
 void scan_i32(betty_ctx* c, const int32_t* in, int64_t* out, const int64_t* n_dev, int64_t n_fixed, int64_t n_cap,
               int64_t* total_dev, cudaStream_t s) {
     scan_impl(c, LdPlain<int32_t>{in}, out, n_dev, n_fixed, n_cap, total_dev, s);
-}
-void scan_popc(betty_ctx* c, const uint32_t* bits, int64_t* out, int64_t n, cudaStream_t s) {
-    scan_impl(c, LdPopc{bits}, out, nullptr, n, 0, nullptr, s);
-}
-void scan_deg(betty_ctx* c, const int32_t* rows, const int64_t* indptr, int64_t* out, const int64_t* n_dev,
-              int64_t n_cap, int64_t* total_dev, cudaStream_t s) {
-    scan_impl(c, LdDeg{rows, indptr}, out, n_dev, 0, n_cap, total_dev, s);
 }
 
 // ---------------------------------------------------------------- memset

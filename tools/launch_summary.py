@@ -31,7 +31,7 @@ def main(path):
         a[2] += d.get("dram__bytes_read.sum", 0.0)
         a[3] += d.get("dram__bytes_write.sum", 0.0)
     tot = sum(a[1] for a in agg.values())
-    print(f"one step: {len(launches)} launches, {tot / 1e3:.3f} ms serialised (ncu, cold-cache)")
+    print(f"one step: {len(launches)} launches, {tot / 1e3:.3f} ms serialised (ncu; cache control as launched: launches.sh CACHE, default all = cold)")
     print(f"{'kernel':34s} {'n':>3s} {'us':>9s} {'share':>6s} {'rd MB':>9s} {'wr MB':>9s}")
     for k, a in sorted(agg.items(), key=lambda x: -x[1][1]):
         print(f"{k[:34]:34s} {a[0]:3d} {a[1]:9.1f} {100 * a[1] / tot:5.1f}% {a[2]:9.1f} {a[3]:9.1f}")
