@@ -2,6 +2,7 @@
 // and the per-step weight layout preparation (fp32 params -> GEMM layouts,
 // cast to bf16 in BF16 mode).
 #include <cmath>
+#include <cstdlib>
 #include "common.cuh"
 #include "internal.h"
 #include "sage.h"
@@ -10,9 +11,10 @@ namespace betty {
 
 // ------------------------------------------------------------------ loss
 // loss_accum += scale * sum_v [logsumexp(S_v) - S_v[y_v]] ;  dS_v = scale * (softmax(S_v) - onehot(y_v))
-// (reading #15: scale = 1 / n_out of the full batch).  One warp per row,
-// C <= 256.  The loss is reduced deterministically: per-CTA partials in a
-// fixed order, summed by the last CTA.
+// (reading #15: scale = 1 / n_out of the full batch).  One warp per row, LOSS_R rows per warp at a
+// time (their loads issued together and their shuffle reductions interleaved: one row's chain of
+// dependent loads and shuffles left the warp stalled, ncu r02r), C <= 256.  The loss is reduced
+// deterministically: per-CTA partials in a fixed order, summed by the last CTA.
 constexpr int LOSS_MAXT_CAP = 8;               // C <= 256
 
 template <typename TA, int LOSS_MAXT>        // LOSS_MAXT = ceil(C / 32) column groups per lane
@@ -22,6 +24,7 @@ __global__ void __launch_bounds__(256) k_loss(const float* __restrict__ logits, 
                                               int64_t ldds, TA* __restrict__ dS_act, int64_t ld_act,
                                               const int64_t* __restrict__ indptr, double* partials, unsigned* ctr,
                                               float* loss_accum) {
+    constexpr int R = LOSS_MAXT <= 2 ? 4 : (LOSS_MAXT <= 4 ? 2 : 1);
     __shared__ double s_w[8];
     __shared__ int s_last;
     const int64_t nd = cnt[0];
@@ -29,61 +32,194 @@ __global__ void __launch_bounds__(256) k_loss(const float* __restrict__ logits, 
     const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
     double wl = 0.0;
-    // the next row's label, degree and logits are loaded while this row is reduced (a row's
-    // arithmetic is a chain of shuffles; its loads would otherwise sit in front of it)
-    int32_t ny = 0;
-    int64_t ndg = 1;
-    float nx[LOSS_MAXT];
-    auto fetch = [&](int64_t vv) {
-        if (vv < nd) {
-            ny = labels[gid[vv]];
-            if (indptr) ndg = indptr[vv + 1] - indptr[vv];
+    for (int64_t v0 = gw * R; v0 < nd; v0 += nw * R) {
+        int32_t gi[R], y[R];
+        int64_t dg[R];
+        float x[R][LOSS_MAXT];
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+            const int64_t v = v0 + r;
+            const bool ok = v < nd;
+            gi[r] = ok ? gid[v] : 0;
+            dg[r] = (ok && indptr) ? indptr[v + 1] - indptr[v] : 1;
 #pragma unroll
             for (int t = 0; t < LOSS_MAXT; ++t) {
                 const int c = lane + 32 * t;
-                nx[t] = c < C ? logits[vv * ldl + c] : -INFINITY;
+                x[r][t] = (ok && c < C) ? logits[v * ldl + c] : -INFINITY;
             }
         }
-    };
-    fetch(gw);
-    for (int64_t v = gw; v < nd; v += nw) {
-        const int32_t y = ny;
-        // indptr (project-first top layer): the fp32 dS is stored pre-scaled by 1/D_v for P^T D+ dS
-        float inv = 1.f;
-        if (indptr) inv = ndg > 0 ? 1.f / (float)ndg : 0.f;
-        float x[LOSS_MAXT];
-        float mx = -INFINITY;
 #pragma unroll
-        for (int t = 0; t < LOSS_MAXT; ++t) {
-            x[t] = nx[t];
-            mx = fmaxf(mx, x[t]);
+        for (int r = 0; r < R; ++r) y[r] = v0 + r < nd ? labels[gi[r]] : -1;
+        float mx[R], se[R], lse[R], xy[R];
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+            mx[r] = -INFINITY;
+#pragma unroll
+            for (int t = 0; t < LOSS_MAXT; ++t) mx[r] = fmaxf(mx[r], x[r][t]);
         }
-        fetch(v + nw);
-        mx = warp_max(mx);
-        float se = 0.f;
 #pragma unroll
-        for (int t = 0; t < LOSS_MAXT; ++t) {
-            const int c = lane + 32 * t;
-            if (c < C) se += expf(x[t] - mx);
+        for (int o = 16; o > 0; o >>= 1)
+#pragma unroll
+            for (int r = 0; r < R; ++r) mx[r] = fmaxf(mx[r], __shfl_xor_sync(0xffffffffu, mx[r], o));
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+            se[r] = 0.f;
+#pragma unroll
+            for (int t = 0; t < LOSS_MAXT; ++t)
+                if (lane + 32 * t < C) se[r] += expf(x[r][t] - mx[r]);
         }
-        se = warp_sum(se);
-        const float lse = mx + logf(se);
-        float xy = 0.f;
 #pragma unroll
-        for (int t = 0; t < LOSS_MAXT; ++t) {
-            const int c = lane + 32 * t;
-            if (c == y) xy = x[t];
-            if (c < C) {
-                const float d = scale * (expf(x[t] - lse) - (c == y ? 1.f : 0.f));
-                dS[v * ldds + c] = d * inv;
-                if (dS_act) st_act(dS_act + v * ld_act + c, d);
+        for (int o = 16; o > 0; o >>= 1)
+#pragma unroll
+            for (int r = 0; r < R; ++r) se[r] += __shfl_xor_sync(0xffffffffu, se[r], o);
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+            const int64_t v = v0 + r;
+            lse[r] = mx[r] + logf(se[r]);
+            xy[r] = 0.f;
+            if (v >= nd) continue;
+            // indptr (project-first top layer): the fp32 dS is stored pre-scaled by 1/D_v for P^T D+ dS
+            const float inv = indptr ? (dg[r] > 0 ? 1.f / (float)dg[r] : 0.f) : 1.f;
+#pragma unroll
+            for (int t = 0; t < LOSS_MAXT; ++t) {
+                const int c = lane + 32 * t;
+                if (c == y[r]) xy[r] = x[r][t];
+                if (c < C) {
+                    const float d = scale * (expf(x[r][t] - lse[r]) - (c == y[r] ? 1.f : 0.f));
+                    dS[v * ldds + c] = d * inv;
+                    if (dS_act) st_act(dS_act + v * ld_act + c, d);
+                }
             }
+            if (dS_act)
+                for (int c = C + lane; c < ld_act; c += 32) st_act(dS_act + v * ld_act + c, 0.f);
         }
-        xy = warp_sum(xy);   // exactly one lane holds y
-        wl += (double)scale * (double)(lse - xy);
-        if (dS_act)
-            for (int c = C + lane; c < ld_act; c += 32) st_act(dS_act + v * ld_act + c, 0.f);
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1)
+#pragma unroll
+            for (int r = 0; r < R; ++r) xy[r] += __shfl_xor_sync(0xffffffffu, xy[r], o);   // one lane holds y
+#pragma unroll
+        for (int r = 0; r < R; ++r)
+            if (v0 + r < nd) wl += (double)scale * (double)(lse[r] - xy[r]);
     }
+    if (lane == 0) s_w[warp_id()] = wl;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double b = 0.0;
+        for (int i = 0; i < (int)(blockDim.x >> 5); ++i) b += s_w[i];
+        partials[blockIdx.x] = b;
+        __threadfence();
+        s_last = (atomicAdd(&ctr[0], 1u) == gridDim.x - 1);
+    }
+    __syncthreads();
+    if (s_last) {                       // fixed-order reduction of the partials by the last CTA
+        __threadfence();
+        double t = 0.0;
+        for (unsigned i = threadIdx.x; i < gridDim.x; i += blockDim.x) t += ((volatile double*)partials)[i];
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) t += __shfl_xor_sync(0xffffffffu, t, o);
+        __syncthreads();
+        if (lane == 0) s_w[warp_id()] = t;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            double tot = 0.0;
+            for (int i = 0; i < (int)(blockDim.x >> 5); ++i) tot += s_w[i];
+            loss_accum[0] += (float)tot;
+            ctr[0] = 0;
+        }
+    }
+}
+
+// C <= 64 (every C1-C5 output layer): half a warp per row, 4 consecutive classes per lane as one
+// 16-byte vector, LOSS_V_R rows per half-warp per step -- a quarter of the instructions per row of
+// k_loss (issue-bound there: ~290 warp-instructions per 47-class row, ncu r02r).  Same arithmetic
+// and reduction structure per row (max, sum of exp, lse), dS / dS_act padding columns written as 0.
+constexpr int LOSS_V_R = 2;
+__device__ __forceinline__ float hmax16(float v) {
+#pragma unroll
+    for (int o = 8; o > 0; o >>= 1) v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, o));
+    return v;
+}
+__device__ __forceinline__ float hsum16(float v) {
+#pragma unroll
+    for (int o = 8; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    return v;
+}
+__device__ __forceinline__ void st_act4z(float* p, const float* v) { st_act4(p, v); }
+__device__ __forceinline__ void st_act4z(__nv_bfloat16* p, const float* v) { st_act4(p, v); }
+
+template <typename TA>
+__global__ void __launch_bounds__(256) k_loss_v(const float* __restrict__ logits, int64_t ldl,
+                                                const int32_t* __restrict__ labels, const int32_t* __restrict__ gid,
+                                                const int64_t* cnt, int C, float scale, float* __restrict__ dS,
+                                                int64_t ldds, TA* __restrict__ dS_act, int64_t ld_act,
+                                                const int64_t* __restrict__ indptr, double* partials, unsigned* ctr,
+                                                float* loss_accum) {
+    constexpr int R = LOSS_V_R;
+    __shared__ double s_w[8];
+    __shared__ int s_last;
+    const int64_t nd = cnt[0];
+    const int lane = lane_id(), hl = lane & 15, hw = lane >> 4;
+    const int c0 = 4 * hl;
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    double wl = 0.0;
+    for (int64_t v0 = gw * 2 * R; v0 < nd; v0 += nw * 2 * R) {
+        int32_t gi[R], y[R];
+        int64_t dg[R];
+        float x[R][4];
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+            const int64_t v = v0 + 2 * r + hw;
+            const bool ok = v < nd;
+            gi[r] = ok ? gid[v] : 0;
+            dg[r] = (ok && indptr) ? indptr[v + 1] - indptr[v] : 1;
+            float4 t = make_float4(-INFINITY, -INFINITY, -INFINITY, -INFINITY);
+            if (ok && c0 < C) t = *(const float4*)(logits + v * ldl + c0);
+            x[r][0] = t.x; x[r][1] = c0 + 1 < C ? t.y : -INFINITY;
+            x[r][2] = c0 + 2 < C ? t.z : -INFINITY; x[r][3] = c0 + 3 < C ? t.w : -INFINITY;
+        }
+#pragma unroll
+        for (int r = 0; r < R; ++r) y[r] = v0 + 2 * r + hw < nd ? labels[gi[r]] : -1;
+        float mx[R], se[R], lse[R], xy[R];
+#pragma unroll
+        for (int r = 0; r < R; ++r) mx[r] = hmax16(fmaxf(fmaxf(x[r][0], x[r][1]), fmaxf(x[r][2], x[r][3])));
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+            float e = 0.f;
+#pragma unroll
+            for (int k = 0; k < 4; ++k)
+                if (c0 + k < C) e += expf(x[r][k] - mx[r]);
+            se[r] = hsum16(e);
+        }
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+            const int64_t v = v0 + 2 * r + hw;
+            lse[r] = mx[r] + logf(se[r]);
+            xy[r] = 0.f;
+            if (v < nd) {
+                const float inv = indptr ? (dg[r] > 0 ? 1.f / (float)dg[r] : 0.f) : 1.f;
+                float d[4];
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                    const int c = c0 + k;
+                    if (c == y[r]) xy[r] = x[r][k];
+                    d[k] = c < C ? scale * (expf(x[r][k] - lse[r]) - (c == y[r] ? 1.f : 0.f)) : 0.f;
+                }
+                if (c0 < ldds)
+                    *(float4*)(dS + v * ldds + c0) = make_float4(d[0] * inv, d[1] * inv, d[2] * inv, d[3] * inv);
+                if (dS_act) {
+                    const float z[4] = {0.f, 0.f, 0.f, 0.f};
+                    for (int cc = c0; cc < ld_act; cc += 64) st_act4z(dS_act + v * ld_act + cc, cc == c0 ? d : z);
+                }
+            }
+            xy[r] = hsum16(xy[r]);                      // one lane of the half holds y
+        }
+        if (hl == 0)
+#pragma unroll
+            for (int r = 0; r < R; ++r)
+                if (v0 + 2 * r + hw < nd) wl += (double)scale * (double)(lse[r] - xy[r]);
+    }
+    wl += __shfl_xor_sync(0xffffffffu, wl, 16);         // the two halves' row sums (lane 0 keeps them)
     if (lane == 0) s_w[warp_id()] = wl;
     __syncthreads();
     if (threadIdx.x == 0) {
@@ -115,9 +251,24 @@ __global__ void __launch_bounds__(256) k_loss(const float* __restrict__ logits, 
 void loss_ce(betty_ctx* c, const float* logits, int64_t ldl, const int32_t* labels, const int32_t* gid,
              const int64_t* cnt, int64_t rows_cap, int C, float scale, float* dS, int64_t ldds, void* dS_act,
              bool act_bf16, int64_t ld_act, const int64_t* prescale_indptr, float* loss_accum, cudaStream_t s) {
-    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((rows_cap * 32 + 255) / 256,
+    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((rows_cap * 8 + 255) / 256,
                                                                  std::min(2048, c->num_sms * 8)));
     double* partials = (double*)(c->L().counters + 64);   // 2048 doubles after the counters
+    static const bool no_vec = getenv("BETTY_LOSS_VEC") && atoi(getenv("BETTY_LOSS_VEC")) == 0;   // A/B switch
+    if (!no_vec && C <= 64 && ldl % 4 == 0 && ldds % 4 == 0 && ld_act % 4 == 0 && ((uintptr_t)logits & 15) == 0 &&
+        ((uintptr_t)dS & 15) == 0 && ((uintptr_t)dS_act & 15) == 0) {
+        const int gv = (int)std::max<int64_t>(1, std::min<int64_t>((rows_cap * 32 / (2 * LOSS_V_R) + 255) / 256,
+                                                                   std::min(2048, c->num_sms * 8)));
+        if (act_bf16)
+            k_loss_v<__nv_bfloat16><<<gv, 256, 0, s>>>(logits, ldl, labels, gid, cnt, C, scale, dS, ldds,
+                                                      (__nv_bfloat16*)dS_act, ld_act, prescale_indptr, partials,
+                                                      c->L().counters + CTR_LOSS, loss_accum);
+        else
+            k_loss_v<float><<<gv, 256, 0, s>>>(logits, ldl, labels, gid, cnt, C, scale, dS, ldds, (float*)dS_act,
+                                              ld_act, prescale_indptr, partials, c->L().counters + CTR_LOSS,
+                                              loss_accum);
+        return;
+    }
     const int T = (C + 31) / 32;               // instantiated for 1, 2, 4 and 8 column groups per lane
 #define LOSS_L(TT) do {                                                                                        \
         if (act_bf16)                                                                                          \

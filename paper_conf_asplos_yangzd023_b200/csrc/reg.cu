@@ -102,6 +102,47 @@ __device__ __forceinline__ void reg_expand(const int64_t* __restrict__ indptr, c
     }
 }
 
+// The same expansion by one warp for a row with ub <= REG_WARP_MAX (so a 32-edge chunk spans at
+// most REG_WARP_MAX + 32 candidates): each lane stamps its edge's index over the edge's flat range
+// in s_seg (a short per-lane loop of shared stores), so a candidate finds its edge with one shared
+// load instead of a binary search over the chunk's prefix (ncu r02r: the search was the kernel's
+// hottest code).
+constexpr int REG_SEG_MAX = REG_WARP_MAX + 32;
+__device__ __forceinline__ void reg_expand_warp(const int64_t* __restrict__ indptr, const int32_t* __restrict__ idx,
+                                                const int64_t* __restrict__ t_indptr,
+                                                const int32_t* __restrict__ t_idx, int64_t i, int64_t row0,
+                                                int32_t* buf, int* s_pre, int64_t* s_cb, uint8_t* s_seg) {
+    const int64_t rb = indptr[i], re = indptr[i + 1];
+    const int32_t gi = (int32_t)(row0 + i);
+    const int lane = lane_id();
+    int64_t o = 0;
+    for (int64_t e0 = rb; e0 < re; e0 += 32) {
+        const int n = (int)mn64(32, re - e0);
+        int d = 0;
+        int64_t cb = 0;
+        if (lane < n) {
+            const int32_t u = idx[e0 + lane];
+            cb = t_indptr[u];
+            d = (int)(t_indptr[u + 1] - cb);
+        }
+        const int incl = warp_incl_scan(d);
+        const int total = __shfl_sync(0xffffffffu, incl, 31);
+        const int start = incl - d;
+        s_pre[lane] = start;
+        s_cb[lane] = cb;
+        for (int k = 0; k < d; ++k) s_seg[start + k] = (uint8_t)lane;
+        __syncwarp();
+        for (int f = lane; f < total; f += 32) {
+            const int k = s_seg[f];
+            const int t = f - s_pre[k];
+            const int32_t j = t_idx[s_cb[k] + t];
+            if (j != gi) buf[o + (s_pre[k] - k) + t - (j > gi ? 1 : 0)] = j;
+        }
+        o += total - n;
+        __syncwarp();
+    }
+}
+
 // run-length encode sorted buf[0, n) -> (col, w) at out offset; returns count (to all threads)
 __device__ __forceinline__ void reg_rle_store(const int32_t* buf, int n, int32_t* __restrict__ ocol,
                                               int32_t* __restrict__ ow, int tid, int nthr, int* s_cnt) {
@@ -232,6 +273,7 @@ __global__ void __launch_bounds__(256) k_reg_rows_warp(const int64_t* __restrict
     __shared__ int32_t buf[8][REG_WARP_MAX + 1];
     __shared__ int s_pre[8][33];
     __shared__ int64_t s_cb[8][32];
+    __shared__ uint8_t s_seg[8][REG_SEG_MAX];
     const int64_t n = *n_rows_dev;
     const int w = warp_id(), lane = lane_id();
     const int64_t gw = blockIdx.x * 8ll + w, nw = gridDim.x * 8ll;
@@ -239,7 +281,7 @@ __global__ void __launch_bounds__(256) k_reg_rows_warp(const int64_t* __restrict
         const int64_t u = ub[i];
         if (u > REG_WARP_MAX) continue;                 // handled by the CTA kernel
         if (u == 0) { if (lane == 0) nnz[i] = 0; continue; }
-        reg_expand(indptr, idx, t_indptr, t_idx, i, row0, buf[w], lane, 32, s_pre[w], s_cb[w]);
+        reg_expand_warp(indptr, idx, t_indptr, t_idx, i, row0, buf[w], s_pre[w], s_cb[w], s_seg[w]);
         if (u <= 32) {               // sort + run-length encode in registers
             int32_t x = lane < u ? buf[w][lane] : INT_MAX;
             x = warp_bitonic32(x);
