@@ -108,22 +108,25 @@ __device__ __forceinline__ void reg_expand(const int64_t* __restrict__ indptr, c
 // load instead of a binary search over the chunk's prefix (ncu r02r: the search was the kernel's
 // hottest code).
 constexpr int REG_SEG_MAX = REG_WARP_MAX + 32;
-__device__ __forceinline__ void reg_expand_warp(const int64_t* __restrict__ indptr, const int32_t* __restrict__ idx,
-                                                const int64_t* __restrict__ t_indptr,
+__device__ __forceinline__ void reg_expand_warp(const int32_t* __restrict__ idx, const int64_t* __restrict__ t_indptr,
                                                 const int32_t* __restrict__ t_idx, int64_t i, int64_t row0,
-                                                int32_t* buf, int* s_pre, int64_t* s_cb, uint8_t* s_seg) {
-    const int64_t rb = indptr[i], re = indptr[i + 1];
+                                                int64_t rb, int64_t re, int64_t cb0, int d0, int32_t* buf,
+                                                int* s_pre, int64_t* s_cb, uint8_t* s_seg) {
     const int32_t gi = (int32_t)(row0 + i);
     const int lane = lane_id();
     int64_t o = 0;
     for (int64_t e0 = rb; e0 < re; e0 += 32) {
         const int n = (int)mn64(32, re - e0);
-        int d = 0;
-        int64_t cb = 0;
-        if (lane < n) {
-            const int32_t u = idx[e0 + lane];
-            cb = t_indptr[u];
-            d = (int)(t_indptr[u + 1] - cb);
+        int d = d0;                                     // the first chunk's columns come prefetched
+        int64_t cb = cb0;
+        if (e0 != rb) {
+            d = 0;
+            cb = 0;
+            if (lane < n) {
+                const int32_t u = idx[e0 + lane];
+                cb = t_indptr[u];
+                d = (int)(t_indptr[u + 1] - cb);
+            }
         }
         const int incl = warp_incl_scan(d);
         const int total = __shfl_sync(0xffffffffu, incl, 31);
@@ -277,11 +280,32 @@ __global__ void __launch_bounds__(256) k_reg_rows_warp(const int64_t* __restrict
     const int64_t n = *n_rows_dev;
     const int w = warp_id(), lane = lane_id();
     const int64_t gw = blockIdx.x * 8ll + w, nw = gridDim.x * 8ll;
+    // Software pipeline over the warp's rows: a row's data is a chain of four dependent loads
+    // (indptr -> idx -> t_indptr -> t_idx).  The next row's first three levels are issued while this
+    // row is expanded and sorted (level 1 at the top, level 2 after the expansion, level 3 after the
+    // sort), so only its t_idx gathers remain on the critical path (ncu r02y: the warps waited on the
+    // chain, with the grid at 4x the resident warps).
+    int64_t pu = 0, prb = 0, pre = 0, poff = 0, pcb = 0;
+    int32_t pidx = 0;
+    int pd = 0;
+    auto lvl1 = [&](int64_t r) {
+        pu = 0; prb = 0; pre = 0; poff = 0;
+        if (r < n) { pu = ub[r]; prb = indptr[r]; pre = indptr[r + 1]; poff = off[r]; }
+    };
+    auto lvl2 = [&]() { pidx = (pu > 0 && pu <= REG_WARP_MAX && lane < pre - prb) ? idx[prb + lane] : -1; };
+    auto lvl3 = [&]() {
+        pcb = 0; pd = 0;
+        if (pidx >= 0) { pcb = t_indptr[pidx]; pd = (int)(t_indptr[pidx + 1] - pcb); }
+    };
+    lvl1(gw); lvl2(); lvl3();
     for (int64_t i = gw; i < n; i += nw) {
-        const int64_t u = ub[i];
-        if (u > REG_WARP_MAX) continue;                 // handled by the CTA kernel
-        if (u == 0) { if (lane == 0) nnz[i] = 0; continue; }
-        reg_expand_warp(indptr, idx, t_indptr, t_idx, i, row0, buf[w], s_pre[w], s_cb[w], s_seg[w]);
+        const int64_t u = pu, rb = prb, re = pre, oi = poff, cb0 = pcb;
+        const int d0 = pd;
+        lvl1(i + nw);
+        if (u > REG_WARP_MAX) { lvl2(); lvl3(); continue; }      // handled by the CTA kernel
+        if (u == 0) { if (lane == 0) nnz[i] = 0; lvl2(); lvl3(); continue; }
+        reg_expand_warp(idx, t_indptr, t_idx, i, row0, rb, re, cb0, d0, buf[w], s_pre[w], s_cb[w], s_seg[w]);
+        lvl2();
         if (u <= 32) {               // sort + run-length encode in registers
             int32_t x = lane < u ? buf[w][lane] : INT_MAX;
             x = warp_bitonic32(x);
@@ -291,16 +315,18 @@ __global__ void __launch_bounds__(256) k_reg_rows_warp(const int64_t* __restrict
             const unsigned above = hm & ~((2u << lane) - 1u);
             const int nxt = above ? __ffs(above) - 1 : (int)u;
             const int pos = __popc(hm & ((1u << lane) - 1u));
-            if (head) { tcol[off[i] + pos] = x; tw[off[i] + pos] = nxt - lane; }
+            if (head) { tcol[oi + pos] = x; tw[oi + pos] = nxt - lane; }
             if (lane == 0) nnz[i] = __popc(hm);
             __syncwarp();
+            lvl3();
             continue;
         }
         int cnt;
-        if (u <= 64) cnt = warp_sort_rle<2>(buf[w], (int)u, tcol + off[i], tw + off[i]);
-        else if (u <= 128) cnt = warp_sort_rle<4>(buf[w], (int)u, tcol + off[i], tw + off[i]);
-        else cnt = warp_sort_rle<8>(buf[w], (int)u, tcol + off[i], tw + off[i]);
+        if (u <= 64) cnt = warp_sort_rle<2>(buf[w], (int)u, tcol + oi, tw + oi);
+        else if (u <= 128) cnt = warp_sort_rle<4>(buf[w], (int)u, tcol + oi, tw + oi);
+        else cnt = warp_sort_rle<8>(buf[w], (int)u, tcol + oi, tw + oi);
         if (lane == 0) nnz[i] = cnt;
+        lvl3();
     }
 }
 
