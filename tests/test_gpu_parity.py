@@ -348,6 +348,47 @@ def test_step_matches_oracle(B, ctx, c, mode, group, graph):
     plan.free()
 
 
+@pytest.mark.parametrize("mode", ["fp32", "bf16"])
+@pytest.mark.parametrize("c", [CASES[0], CASES[4], CASES[11]], ids=lambda c: c["name"])
+def test_step_degenerate_inputs(B, ctx, c, mode):
+    """Degenerate cases of the method through the fused step (graph replay): a sparse graph whose
+    sampled rows are often empty (D_v = 0: h_N = 0, readings #12, #14, S1), micro-batches
+    with no outputs at all (labels 1, 3, 4 of K = 6 unused, reading #10), a ragged last launch group (4 + 2), and
+    a plan whose every micro-batch is empty (zero gradient, zero loss)."""
+    n, pairs, n_out = 600, 150, 60
+    F = c["dims"][0]
+    ld = (F + 7) // 8 * 8
+    g, sd, blocks, feats, _ = tiny(n=n, pairs=pairs, fanouts=c["fanouts"], n_out=n_out, F=F, C=c["dims"][-1],
+                                   seed=5, ld=ld)
+    empty_rows = sum(int(np.sum(np.diff(b.indptr) == 0)) for b in blocks)
+    assert empty_rows > 0                               # the case really has rows with D_v = 0
+    labels = (np.arange(n) * 5 % c["dims"][-1]).astype(np.int32)
+    params = synth.init_params(c["dims"], c["aggr"], seed=5)
+    K = 6
+    part = np.array([(0, 2, 5)[i % 3] for i in range(len(sd))], dtype=np.int32)
+    dev = B.blocks_to_device(blocks)
+    dpart = torch.as_tensor(part).cuda()
+    model = B.Model(c["dims"], c["aggr"], mode, mode)
+    P = torch.as_tensor(params).cuda()
+    X = dev_feats(feats, mode)
+    Y = torch.as_tensor(labels).cuda()
+    scale = 1.0 / len(sd)
+    for ks, group in (([0, 1, 2, 3, 4, 5], 4), ([1, 3], 0)):
+        plan = B.betty_plan_create(ctx, model, dev, dpart, K, ks, group=group, flags=B.PLAN_GRAPH)
+        og, ol = oracle.step(c["dims"], c["aggr"], mode == "bf16", blocks, part, K, ks, params, feats, labels, scale)
+        for rep in range(2):
+            grad = torch.zeros_like(P)
+            loss = torch.zeros(1, device="cuda")
+            B.betty_step(ctx, plan, P, X, Y, scale, grad, loss)
+            B.betty_sync_check(ctx)
+            if not np.any(og):
+                assert not torch.any(grad).item() and loss.item() == 0.0
+            else:
+                assert_grad_close(grad.cpu().numpy(), og, c["dims"], c["aggr"], RTOL[mode], f"ks={ks} rep={rep}")
+                assert loss.item() == pytest.approx(ol, rel=RTOL[mode])
+        plan.free()
+
+
 def test_sum_of_micro_batches_equals_full_batch_on_gpu(B, ctx):
     """Betty's invariant on the GPU path itself: K=8 step == K=1 step (fp32)."""
     c = CASES[1]
