@@ -1388,7 +1388,10 @@ static bool agg_mean_g4(betty_ctx* c, const void* X, bool x_bf16, int64_t ldx, c
         }
         if ((int)sm > max_dyn) return false;
         cudaMemsetAsync(ctr, 0, sizeof(unsigned), s);
-        k_agg_mean_g4<TI, TO><<<c->num_sms, G4_THREADS, sm, s>>>(tm, a);
+        // BETTY_G4_GRID: (study) fewer CTAs than SMs -- the kernel's time scales as 1 / grid
+        // (profiles/r03_agg_bound.txt: its bound is inside each SM, not L2 or HBM)
+        static const int g4_grid = getenv("BETTY_G4_GRID") ? atoi(getenv("BETTY_G4_GRID")) : 0;
+        k_agg_mean_g4<TI, TO><<<g4_grid > 0 ? g4_grid : c->num_sms, G4_THREADS, sm, s>>>(tm, a);
     }))
     return true;
 }
