@@ -916,7 +916,14 @@ extern "C" betty_status betty_plan_create(betty_ctx* c, const betty_model* model
             if (cudaStreamEndCapture(cs2, &gr) == cudaSuccess) {
                 size_t n = 0;
                 cudaGraphGetNodes(gr, nullptr, &n);
-                p->info.kernels_per_step = (int32_t)n;
+                std::vector<cudaGraphNode_t> nodes(n);
+                int32_t nk = 0;                     // kernel nodes only (not memsets / copies / events)
+                if (n && cudaGraphGetNodes(gr, nodes.data(), &n) == cudaSuccess)
+                    for (size_t i = 0; i < n; ++i) {
+                        cudaGraphNodeType t;
+                        if (cudaGraphNodeGetType(nodes[i], &t) == cudaSuccess && t == cudaGraphNodeTypeKernel) ++nk;
+                    }
+                p->info.kernels_per_step = nk;
                 cudaGraphDestroy(gr);
             }
         }
