@@ -113,6 +113,29 @@ __device__ __forceinline__ void split_tf32(uint32_t x, uint32_t lo) {
     asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};" ::"r"(x), "f"(h.x), "f"(h.y), "f"(h.z), "f"(h.w) : "memory");
     asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};" ::"r"(lo), "f"(l.x), "f"(l.y), "f"(l.z), "f"(l.w) : "memory");
 }
+// SPLIT_NB float4 at once: every load issued before any arithmetic or store, so the shared-memory
+// latency is paid once per batch instead of once per float4 (the volatile ld/st of split_tf32 kept
+// the converter warps latency-bound: ncu showed the small-N fp32 GEMMs at 16 % tensor activity)
+constexpr int SPLIT_NB = 4;
+__device__ __forceinline__ void split_tf32_n(uint32_t x, uint32_t lo, uint32_t stride) {
+    float4 v[SPLIT_NB];
+#pragma unroll
+    for (int b = 0; b < SPLIT_NB; ++b)
+        asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];"
+                     : "=f"(v[b].x), "=f"(v[b].y), "=f"(v[b].z), "=f"(v[b].w) : "r"(x + b * stride));
+#pragma unroll
+    for (int b = 0; b < SPLIT_NB; ++b) {
+        float4 h, l;
+        h.x = tf32_rn(v[b].x); l.x = tf32_rn(v[b].x - h.x);
+        h.y = tf32_rn(v[b].y); l.y = tf32_rn(v[b].y - h.y);
+        h.z = tf32_rn(v[b].z); l.z = tf32_rn(v[b].z - h.z);
+        h.w = tf32_rn(v[b].w); l.w = tf32_rn(v[b].w - h.w);
+        asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};" ::"r"(x + b * stride), "f"(h.x), "f"(h.y), "f"(h.z),
+                     "f"(h.w) : "memory");
+        asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};" ::"r"(lo + b * stride), "f"(l.x), "f"(l.y), "f"(l.z),
+                     "f"(l.w) : "memory");
+    }
+}
 // hw_hi variant: only lo = x - trunc_tf32(x) is written; the tensor core's own fp32 -> tf32
 // conversion of the untouched x must then be the truncation (BETTY_TF32_HW_HI=1, an experiment)
 __device__ __forceinline__ void split_tf32_lo(uint32_t x, uint32_t lo) {
@@ -474,9 +497,12 @@ k_tc_row(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtens
                     for (int i = tid; i < (int)(a_bytes / 16); i += 32 * ROW_CONV_WARPS)
                         split_tf32_lo(a + 16 * i, a + a_bytes + 16 * i);
                 } else {
-#pragma unroll 4
-                    for (int i = tid; i < (int)(a_bytes / 16); i += 32 * ROW_CONV_WARPS)
-                        split_tf32(a + 16 * i, a + a_bytes + 16 * i);
+                    constexpr int STEP = 32 * ROW_CONV_WARPS;
+                    const int n16 = (int)(a_bytes / 16);
+                    int i = tid;
+                    for (; i + (SPLIT_NB - 1) * STEP < n16; i += SPLIT_NB * STEP)
+                        split_tf32_n(a + 16 * i, a + a_bytes + 16 * i, 16 * STEP);
+                    for (; i < n16; i += STEP) split_tf32(a + 16 * i, a + a_bytes + 16 * i);
                 }
                 fence_proxy_async();             // generic-proxy writes -> visible to the tensor core
                 __syncwarp();
@@ -777,8 +803,11 @@ k_tc_red(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtens
 #pragma unroll 4
                 for (int i = tid; i < n16; i += 32 * CONV_WARPS) split_tf32_lo(sa + 16 * i, sa + raw_bytes + 16 * i);
             } else if (valid >= KN) {
-#pragma unroll 4
-                for (int i = tid; i < n16; i += 32 * CONV_WARPS) split_tf32(sa + 16 * i, sa + raw_bytes + 16 * i);
+                constexpr int STEP = 32 * CONV_WARPS;
+                int i = tid;
+                for (; i + (SPLIT_NB - 1) * STEP < n16; i += SPLIT_NB * STEP)
+                    split_tf32_n(sa + 16 * i, sa + raw_bytes + 16 * i, 16 * STEP);
+                for (; i < n16; i += STEP) split_tf32(sa + 16 * i, sa + raw_bytes + 16 * i);
             } else {                                     // the last k-block: rows >= M are zeroed
                 for (int i = tid; i < n16; i += 32 * CONV_WARPS) {
                     const int row = (i >> 3) & (KN - 1); // 8 float4 per 128-byte row, KN rows per box
