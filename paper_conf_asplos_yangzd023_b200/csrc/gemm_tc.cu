@@ -668,13 +668,16 @@ struct RedArgs {
 // accumulator into a TMEM running total with round-to-nearest fp32 adds (one feature tile per CTA,
 // TMEM = accumulator + total).
 constexpr int RED_THREADS_TF = THREADS + 32 * CONV_WARPS;
-constexpr int RED_SB = 4;
-template <bool TF>
+// TKN (fp32 mode): nodes per k-block -- 16, or 32 for narrow B (N <= 64: a k-block's MMAs are short,
+// so per-k-block barrier / converter / issue overhead dominated; C3 fp32 step 10.57 -> 10.31 ms with
+// 32 everywhere, while the N = 256 dW0 was faster with 16); RED_SB k-blocks = 64 nodes per drain
+template <bool TF, int TKN>
 __global__ void __launch_bounds__(TF ? RED_THREADS_TF : THREADS, 1)
 k_tc_red(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB, RedArgs p) {
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
-    constexpr int KN = TF ? 16 : BK;                  // nodes (reduction rows) per k-block
+    constexpr int KN = TF ? TKN : BK;                 // nodes (reduction rows) per k-block
+    constexpr int RED_SB = 64 / TKN;
     const int S = p.stages;
     const uint32_t box = KN * 128;                    // KN rows x 128 B (64 bf16 / 32 fp32 features)
     const int nbA_cta = p.nbA * p.mt_cta;             // A boxes per stage
@@ -1043,7 +1046,8 @@ bool gemm_red_tc(betty_ctx* c, const GemmRed& g, int* S_used, cudaStream_t s) {
     if (TF && (g.b_bf16 || (g.lda & 3) || (g.ldb & 3))) return false;
     if (!TF && (!g.a_bf16 || !g.b_bf16 || (g.lda & 7) || (g.ldb & 7))) return false;
     if (g.N > 256) return false;
-    const int KN = TF ? 16 : BK, fbox = TF ? 32 : 64;
+    const int tkn = g.N <= 64 ? 32 : 16;        // fp32 mode: nodes per k-block (see k_tc_red)
+    const int KN = TF ? tkn : BK, fbox = TF ? 32 : 64;
     const int BN = (g.N + 15) / 16 * 16;
     CUtensorMap ma, mb;
     const CUtensorMapSwizzle sw = TF ? CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B : CU_TENSOR_MAP_SWIZZLE_128B;
@@ -1077,17 +1081,19 @@ bool gemm_red_tc(betty_ctx* c, const GemmRed& g, int* S_used, cudaStream_t s) {
     if (TF) {
         static bool attr = false;
         if (!attr) {
-            cudaFuncSetAttribute(k_tc_red<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+            cudaFuncSetAttribute(k_tc_red<true, 16>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+            cudaFuncSetAttribute(k_tc_red<true, 32>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
             attr = true;
         }
-        k_tc_red<true><<<grid, RED_THREADS_TF, smem, s>>>(ma, mb, p);
+        if (tkn == 32) k_tc_red<true, 32><<<grid, RED_THREADS_TF, smem, s>>>(ma, mb, p);
+        else k_tc_red<true, 16><<<grid, RED_THREADS_TF, smem, s>>>(ma, mb, p);
     } else {
         static bool attr = false;
         if (!attr) {
-            cudaFuncSetAttribute(k_tc_red<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+            cudaFuncSetAttribute(k_tc_red<false, 16>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
             attr = true;
         }
-        k_tc_red<false><<<grid, THREADS, smem, s>>>(ma, mb, p);
+        k_tc_red<false, 16><<<grid, THREADS, smem, s>>>(ma, mb, p);
     }
     return true;
 }
