@@ -213,6 +213,8 @@ struct RowArgs {
     int bstream;             // 1: B is streamed with A through the ring (B too large to stay resident)
     int hw_hi;               // TF: converter writes lo only (see split_tf32_lo)
     int64_t cend;            // trailing columns [N, cend) of a row are written (ones column / zeros)
+    int kbb;                 // bytes per row of one k-block: 128 (SWIZZLE_128B), or 64 (TF: SWIZZLE_64B,
+                             // half the ring stage -> twice the stages when B streams or sits resident)
 };
 
 __device__ __forceinline__ uint32_t pack_bf16x2(float a, float b) {
@@ -369,8 +371,8 @@ k_tc_row(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtens
     constexpr int ES = TF ? ESLOTS_TF : ESLOTS;
     constexpr int NSPLIT = TF ? 2 : 1;                       // hi (+ lo) copies of each operand block
     const int S = p.stages;
-    const uint32_t a_bytes = BM * 128;                       // one A k-block: 128 rows x 128 B
-    const uint32_t bblk = (uint32_t)p.BN * 128;              // one K-block of B
+    const uint32_t a_bytes = BM * p.kbb;                     // one A k-block: 128 rows x kbb bytes
+    const uint32_t bblk = (uint32_t)p.BN * p.kbb;            // one K-block of B
     // one ring stage: A (+ A lo) (+ B (+ B lo) when streamed)
     const uint32_t ring_bytes = NSPLIT * (a_bytes + (p.bstream ? bblk : 0u));
     uint8_t* bres = smem;                                    // NSPLIT * nk * bblk (resident B) or nothing
@@ -407,7 +409,7 @@ k_tc_row(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtens
 
     if (warp == 0) {
         if (elect_lane0() && blockIdx.x < tiles) {
-            constexpr int KE = TF ? 32 : BK;                 // elements per k-block
+            const int KE = TF ? p.kbb / 4 : BK;              // elements per k-block
             if (!p.bstream) {
                 mbar_expect_tx(bfull, NSPLIT * p.nk * bblk);
                 for (int kb = 0; kb < p.nk; ++kb) {
@@ -459,15 +461,17 @@ k_tc_row(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtens
                         const uint32_t alo = a0 + a_bytes;
                         const uint32_t blo = p.bstream ? b0 + bblk : su32(bres + (p.nk + kb) * bblk);
                         const uint32_t dl = d + p.acc_stride;
-#pragma unroll
-                        for (int k = 0; k < 4; ++k)
-                            umma_tf32(dl, sdesc(alo + k * 32, 0, 1024), sdesc(b0 + k * 32, 0, 1024), idesc, (kb | k) != 0);
-#pragma unroll
-                        for (int k = 0; k < 4; ++k)
-                            umma_tf32(dl, sdesc(a0 + k * 32, 0, 1024), sdesc(blo + k * 32, 0, 1024), idesc, 1);
-#pragma unroll
-                        for (int k = 0; k < 4; ++k)
-                            umma_tf32(d, sdesc(a0 + k * 32, 0, 1024), sdesc(b0 + k * 32, 0, 1024), idesc, (kb | k) != 0);
+                        // K = 8 fp32 (32 B) per MMA; 8-row swizzle atoms of kbb bytes per row (SBO = 8 kbb)
+                        const int nks = p.kbb / 32;
+                        const uint32_t sbo = 8u * (uint32_t)p.kbb, lay = p.kbb == 128 ? 2u : 4u;
+                        for (int k = 0; k < nks; ++k)
+                            umma_tf32(dl, sdesc(alo + k * 32, 0, sbo, lay), sdesc(b0 + k * 32, 0, sbo, lay), idesc,
+                                      (kb | k) != 0);
+                        for (int k = 0; k < nks; ++k)
+                            umma_tf32(dl, sdesc(a0 + k * 32, 0, sbo, lay), sdesc(blo + k * 32, 0, sbo, lay), idesc, 1);
+                        for (int k = 0; k < nks; ++k)
+                            umma_tf32(d, sdesc(a0 + k * 32, 0, sbo, lay), sdesc(b0 + k * 32, 0, sbo, lay), idesc,
+                                      (kb | k) != 0);
                     } else {
 #pragma unroll
                         for (int k = 0; k < BK / UK; ++k) {
@@ -953,32 +957,46 @@ bool gemm_row_tc(betty_ctx* c, const GemmRow& g, const void* Bk, const void* Bk_
     if (!TF && (!g.a_bf16 || !g.b_bf16 || (g.lda & 7) || (ldbk & 7))) return false;
     if (g.N > 256 || g.N < 1) return false;
     if ((g.epi == EPI_MASK || g.epi == EPI_RES_MASK) && !g.mbits && (g.ldm & (g.m_bf16 ? 7 : 3))) return false;
-    const int KE = TF ? 32 : BK;                // elements per 128-byte k-block
     const int NS = TF ? 2 : 1;                  // hi (+ lo) copies
     const int BN = (g.N + 15) / 16 * 16;
-    const int nk = (g.K + KE - 1) / KE;
-    const size_t bblk = (size_t)BN * 128;
-    const size_t b_bytes = (size_t)nk * bblk * NS;
-    const size_t a_bytes = (size_t)BM * 128 * NS;
     const uint32_t slot_bytes = 32 * 32 * (g.c_bf16 ? 2 : 4);
     const size_t stage_bytes = (size_t)EPI_WARPS * (TF ? ESLOTS_TF : ESLOTS) * slot_bytes;
     const size_t budget = 227 * 1024;           // the sm_100 opt-in maximum of dynamic shared memory per CTA
-    // B resident when it fits next to a 2-stage A ring, else streamed with A
-    const bool bstream = b_bytes + stage_bytes + 2 * a_bytes + 1024 + 256 > budget;
-    const size_t ring = a_bytes + (bstream ? bblk * NS : 0);
-    const size_t fixed = (bstream ? 0 : b_bytes) + stage_bytes + 1024 + 256;
+    // k-block row bytes: 128; in fp32 (TF) mode 64 when the 128-byte layout leaves fewer than 3 ring
+    // stages (B hi + lo resident or streamed, the A lo copy: the narrow / wide fp32 GEMMs were stuck at
+    // a 2-deep ring).  BETTY_TF_KBB=128/64 forces one.
+    static const int kbb_env = getenv("BETTY_TF_KBB") ? atoi(getenv("BETTY_TF_KBB")) : 0;
+    int kbb = 128;
+    int KE = 0, nk = 0;
+    size_t bblk = 0, b_bytes = 0, a_bytes = 0, ring = 0, fixed = 0;
+    bool bstream = false;
+    for (int pass = 0; pass < 2; ++pass) {
+        KE = TF ? kbb / 4 : BK;                 // elements per k-block
+        nk = (g.K + KE - 1) / KE;
+        bblk = (size_t)BN * kbb;
+        b_bytes = (size_t)nk * bblk * NS;
+        a_bytes = (size_t)BM * kbb * NS;
+        // B resident when it fits next to a 2-stage A ring, else streamed with A
+        bstream = b_bytes + stage_bytes + 2 * a_bytes + 1024 + 256 > budget;
+        ring = a_bytes + (bstream ? bblk * NS : 0);
+        fixed = (bstream ? 0 : b_bytes) + stage_bytes + 1024 + 256;
+        const bool want64 = TF && (kbb_env == 64 || (kbb_env != 128 && (budget - fixed) / ring < 3));
+        if (pass == 0 && want64) { kbb = 64; continue; }
+        break;
+    }
     if (fixed + 2 * ring > budget) return false;
+    const CUtensorMapSwizzle swz = kbb == 128 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B;
     CUtensorMap ma, mb, mc, mbl;
-    if (!make_map_t(&ma, g.A, TF, g.K, g.M_cap, g.lda, KE, BM, CU_TENSOR_MAP_SWIZZLE_128B) ||
-        !make_map_t(&mb, Bk, TF, g.K, g.N, ldbk, KE, BN, CU_TENSOR_MAP_SWIZZLE_128B))
+    if (!make_map_t(&ma, g.A, TF, g.K, g.M_cap, g.lda, KE, BM, swz) ||
+        !make_map_t(&mb, Bk, TF, g.K, g.N, ldbk, KE, BN, swz))
         return false;
-    if (TF && !make_map_t(&mbl, Bk_lo, true, g.K, g.N, ldbk, KE, BN, CU_TENSOR_MAP_SWIZZLE_128B)) return false;
+    if (TF && !make_map_t(&mbl, Bk_lo, true, g.K, g.N, ldbk, KE, BN, swz)) return false;
     if (!TF) mbl = mb;
     if (!make_map_t(&mc, g.C, !g.c_bf16, g.N, g.M_cap, g.ldc, 32, 32,
                     g.c_bf16 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_128B))
         return false;
     RowArgs p{};
-    p.M_dev = g.M_dev; p.K = g.K; p.N = g.N; p.BN = BN; p.nk = nk;
+    p.M_dev = g.M_dev; p.K = g.K; p.N = g.N; p.BN = BN; p.nk = nk; p.kbb = kbb;
     p.stages = (int)std::max<size_t>(2, std::min<size_t>(8, (budget - fixed) / ring));
     p.bstream = bstream ? 1 : 0;
     static const int hw_hi_row = getenv("BETTY_TF32_HW_HI") ? atoi(getenv("BETTY_TF32_HW_HI")) : 0;
