@@ -962,9 +962,10 @@ bool gemm_row_tc(betty_ctx* c, const GemmRow& g, const void* Bk, const void* Bk_
     const uint32_t slot_bytes = 32 * 32 * (g.c_bf16 ? 2 : 4);
     const size_t stage_bytes = (size_t)EPI_WARPS * (TF ? ESLOTS_TF : ESLOTS) * slot_bytes;
     const size_t budget = 227 * 1024;           // the sm_100 opt-in maximum of dynamic shared memory per CTA
-    // k-block row bytes: 128; in fp32 (TF) mode 64 when the 128-byte layout leaves fewer than 3 ring
-    // stages (B hi + lo resident or streamed, the A lo copy: the narrow / wide fp32 GEMMs were stuck at
-    // a 2-deep ring).  BETTY_TF_KBB=128/64 forces one.
+    // k-block row bytes: 128 for bf16; 64 in fp32 (TF) mode, where B hi + lo (resident or streamed) and
+    // the lo copy of every A stage left room for a 2-deep ring only (the wide fp32 forward: 1.73 -> 1.57
+    // ms).  C3 fp32 step, two runs each: 64 everywhere 10.14 / 10.09 ms, 64 only where B streams
+    // 10.27 / 10.22, 128 everywhere 10.31 / 10.32.  BETTY_TF_KBB=128 restores the 128-byte layout.
     static const int kbb_env = getenv("BETTY_TF_KBB") ? atoi(getenv("BETTY_TF_KBB")) : 0;
     int kbb = 128;
     int KE = 0, nk = 0;
@@ -980,7 +981,7 @@ bool gemm_row_tc(betty_ctx* c, const GemmRow& g, const void* Bk, const void* Bk_
         bstream = b_bytes + stage_bytes + 2 * a_bytes + 1024 + 256 > budget;
         ring = a_bytes + (bstream ? bblk * NS : 0);
         fixed = (bstream ? 0 : b_bytes) + stage_bytes + 1024 + 256;
-        const bool want64 = TF && (kbb_env == 64 || (kbb_env != 128 && (budget - fixed) / ring < 3));
+        const bool want64 = TF && kbb_env != 128;
         if (pass == 0 && want64) { kbb = 64; continue; }
         break;
     }
