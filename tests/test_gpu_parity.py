@@ -234,6 +234,31 @@ def test_group_extraction(B, ctx, group):
     plan.free()
 
 
+def test_wide_launch_group_and_many_parts(B, ctx):
+    """The output selection at its limits: K = 700 parts over 600 outputs (most parts empty), a launch
+    group of 512 micro-batches (the largest one pass handles) holding every non-empty and many empty
+    ones, bit-exact against the oracle's union; K beyond 16384 is refused (EUNSUPPORTED)."""
+    g, sd, blocks, feats, labels = tiny(n=3000, pairs=9000, fanouts=(3, 4), n_out=600, seed=9)
+    K = 700
+    part = synth.random_partition(len(sd), K, 4)
+    ks = list(range(0, K, 1))[:512]
+    dev = B.blocks_to_device(blocks)
+    dpart = torch.as_tensor(part).cuda()
+    model = B.Model([8, 12, 3], "mean", "fp32")
+    plan = B.betty_plan_create(ctx, model, dev, dpart, K, ks, group=512, flags=0)
+    got = plan.group_blocks(0)
+    want = concat_oracle(blocks, part, K, ks)
+    for l, (a, b) in enumerate(zip(got, want)):
+        assert (a.n_dst, a.n_src, a.n_edges) == (b.n_dst, b.n_src, b.n_edges), l
+        for name in ("indptr", "indices", "src_pos", "src_gid"):
+            np.testing.assert_array_equal(getattr(a, name).cpu().numpy(), getattr(b, name), err_msg=f"l{l} {name}")
+    plan.free()
+    with pytest.raises(B.BettyError, match="EUNSUPPORTED"):
+        B.betty_extract_blocks(ctx, dev, torch.zeros(len(sd), dtype=torch.int32, device="cuda"), 20000, 0)
+    with pytest.raises(B.BettyError, match="EUNSUPPORTED"):
+        B.betty_plan_create(ctx, model, dev, dpart, K, list(range(K)), group=600, flags=0)
+
+
 def test_extract_bad_input(B, ctx):
     g, sd, blocks, feats, labels = tiny(seed=5)
     dev = B.blocks_to_device(blocks)
