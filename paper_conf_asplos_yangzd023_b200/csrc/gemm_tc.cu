@@ -189,7 +189,7 @@ __device__ __forceinline__ bool elect_lane0() { return (threadIdx.x & 31) == 0; 
 // instead of re-reading the bf16 activations.  The kernel is templated on the
 // epilogue so each 32-column chunk is straight-line code (~150 instructions).
 constexpr int EPI_WARPS = 8;
-constexpr int ESLOTS = 2;                       // staging slots per epilogue warp (bf16 operands)
+constexpr int ESLOTS = 1;                       // staging slots (4 KB) per epilogue warp (bf16 operands)
 constexpr int ESLOTS_TF = 1;                    // ... FP32 mode (the 3xTF32 ring needs the room)
 constexpr int ROW_THREADS = 64 + 32 * EPI_WARPS;
 constexpr int CONV_WARPS = 4;                   // FP32 mode: hi/lo split of each stage (k_tc_red)
@@ -300,9 +300,11 @@ __device__ __forceinline__ uint32_t mask_word_from_act(const RowArgs& p, int64_t
 
 // one 32-column chunk: epilogue math on v (fp32 bits in r), staged for the TMA store.
 // Returns the ReLU bits (EPI_RELU_ONES).
+// bf16 (CBF): `part` 1 / 2 = first / second 32 columns of a 64-column pair staged as 128-byte rows
+// (SWIZZLE_128B, one TMA store per pair), 0 = a lone chunk as 64-byte rows (SWIZZLE_64B)
 template <int EPI, bool CBF>
 __device__ __forceinline__ uint32_t chunk_epilogue(const RowArgs& p, const uint32_t* r, int64_t m, int c0, bool ok,
-                                                   uint32_t mword, int64_t nres, uint8_t* slot, int lane) {
+                                                   uint32_t mword, int64_t nres, uint8_t* slot, int lane, int part) {
     float v[32];
 #pragma unroll
     for (int j = 0; j < 32; ++j) v[j] = __uint_as_float(r[j]);
@@ -339,11 +341,20 @@ __device__ __forceinline__ uint32_t chunk_epilogue(const RowArgs& p, const uint3
             for (int k = 0; k < 16; ++k)
                 bits |= (uint32_t)((w[k] & 0x7fffu) != 0u) << (2 * k) | (uint32_t)((w[k] & 0x7fff0000u) != 0u) << (2 * k + 1);
         }
-        // 64 B rows, SWIZZLE_64B: 16-B chunk c of row r at c ^ ((r >> 1) & 3)
-        uint8_t* row = slot + lane * 64;
+        if (part == 0) {
+            // 64 B rows, SWIZZLE_64B: 16-B chunk c of row r at c ^ ((r >> 1) & 3)
+            uint8_t* row = slot + lane * 64;
 #pragma unroll
-        for (int c = 0; c < 4; ++c)
-            *(uint4*)(row + ((c ^ ((lane >> 1) & 3)) << 4)) = make_uint4(w[4 * c], w[4 * c + 1], w[4 * c + 2], w[4 * c + 3]);
+            for (int c = 0; c < 4; ++c)
+                *(uint4*)(row + ((c ^ ((lane >> 1) & 3)) << 4)) = make_uint4(w[4 * c], w[4 * c + 1], w[4 * c + 2], w[4 * c + 3]);
+        } else {
+            // 128 B rows, SWIZZLE_128B: 16-B chunk cc = 4 (part - 1) + c of row r at cc ^ (r & 7)
+            uint8_t* row = slot + lane * 128;
+#pragma unroll
+            for (int c = 0; c < 4; ++c)
+                *(uint4*)(row + (((4 * (part - 1) + c) ^ (lane & 7)) << 4)) =
+                    make_uint4(w[4 * c], w[4 * c + 1], w[4 * c + 2], w[4 * c + 3]);
+        }
     } else {
         if (EPI == EPI_RELU_ONES) {
 #pragma unroll
@@ -365,7 +376,8 @@ __device__ __forceinline__ uint32_t chunk_epilogue(const RowArgs& p, const uint3
 template <int EPI, bool CBF, bool MBITS, bool TF>
 __global__ void __launch_bounds__(TF ? ROW_THREADS_TF : ROW_THREADS, 1)
 k_tc_row(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
-         const __grid_constant__ CUtensorMap tmC, const __grid_constant__ CUtensorMap tmBlo, RowArgs p) {
+         const __grid_constant__ CUtensorMap tmC, const __grid_constant__ CUtensorMap tmBlo,
+         const __grid_constant__ CUtensorMap tmC2, RowArgs p) {
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
     constexpr int ES = TF ? ESLOTS_TF : ESLOTS;
@@ -399,6 +411,7 @@ k_tc_row(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtens
         asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmA) : "memory");
         asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmB) : "memory");
         asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmC) : "memory");
+        if (CBF) asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmC2) : "memory");
         if (TF) asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmBlo) : "memory");
     }
     if (warp == 1) tmem_alloc_warp(tslot, p.tmem_cols);
@@ -582,7 +595,7 @@ k_tc_row(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtens
                         uint8_t* sl = my_stage + slot * p.slot_bytes;
                         if (lane == 0) bulk_wait_read<ES - 1>();
                         __syncwarp();
-                        obits[ci] = chunk_epilogue<EPI, CBF>(p, ra, m, c0, ok, mw[ci], nres, sl, lane);
+                        obits[ci] = chunk_epilogue<EPI, CBF>(p, ra, m, c0, ok, mw[ci], nres, sl, lane, 0);
                         fence_proxy_async();
                         __syncwarp();
                         if (lane == 0) {
@@ -602,17 +615,26 @@ k_tc_row(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtens
                     uint32_t* nxt = (ci & 1) ? ra : rb;
                     const int c0 = cbeg + 32 * ci;
                     if (ci + 1 < nch) tmem_ld32_nowait(tbase + c0 + 32, nxt);   // next chunk in flight
+                    // bf16: chunks (0,1), (2,3) of the half share a slot and one 64-column store
+                    const bool second = CBF && (ci & 1) != 0;
+                    const bool paired = CBF && (second || ci + 1 < nch);
+                    const int part = paired ? (second ? 2 : 1) : 0;
                     uint8_t* sl = my_stage + slot * p.slot_bytes;
-                    if (lane == 0) bulk_wait_read<ES - 1>();        // the store that used this slot has read it
-                    __syncwarp();
-                    obits[ci] = chunk_epilogue<EPI, CBF>(p, cur, m, c0, ok, mw[ci], nres, sl, lane);
-                    fence_proxy_async();
-                    __syncwarp();
-                    if (lane == 0) {
-                        tma_store_2d(&tmC, sl, c0, (int)row0);
-                        bulk_commit();
+                    if (!second) {
+                        if (lane == 0) bulk_wait_read<ES - 1>();    // the store that used this slot has read it
+                        __syncwarp();
                     }
-                    if (++slot == ES) slot = 0;
+                    obits[ci] = chunk_epilogue<EPI, CBF>(p, cur, m, c0, ok, mw[ci], nres, sl, lane, part);
+                    if (second || !paired) {
+                        fence_proxy_async();
+                        __syncwarp();
+                        if (lane == 0) {
+                            if (part == 2) tma_store_2d(&tmC2, sl, c0 - 32, (int)row0);
+                            else tma_store_2d(&tmC, sl, c0, (int)row0);
+                            bulk_commit();
+                        }
+                        if (++slot == ES) slot = 0;
+                    }
                     if (ci + 1 < nch) tmem_wait_regs(nxt);
                 }
             }
@@ -959,7 +981,7 @@ bool gemm_row_tc(betty_ctx* c, const GemmRow& g, const void* Bk, const void* Bk_
     if ((g.epi == EPI_MASK || g.epi == EPI_RES_MASK) && !g.mbits && (g.ldm & (g.m_bf16 ? 7 : 3))) return false;
     const int NS = TF ? 2 : 1;                  // hi (+ lo) copies
     const int BN = (g.N + 15) / 16 * 16;
-    const uint32_t slot_bytes = 32 * 32 * (g.c_bf16 ? 2 : 4);
+    const uint32_t slot_bytes = 32 * 128;       // 32 rows x 128 B (bf16: a 64-column pair; fp32: 32 columns)
     const size_t stage_bytes = (size_t)EPI_WARPS * (TF ? ESLOTS_TF : ESLOTS) * slot_bytes;
     const size_t budget = 227 * 1024;           // the sm_100 opt-in maximum of dynamic shared memory per CTA
     // k-block row bytes: 128 for bf16; 64 in fp32 (TF) mode, where B hi + lo (resident or streamed) and
@@ -987,7 +1009,7 @@ bool gemm_row_tc(betty_ctx* c, const GemmRow& g, const void* Bk, const void* Bk_
     }
     if (fixed + 2 * ring > budget) return false;
     const CUtensorMapSwizzle swz = kbb == 128 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B;
-    CUtensorMap ma, mb, mc, mbl;
+    CUtensorMap ma, mb, mc, mbl, mc2;
     if (!make_map_t(&ma, g.A, TF, g.K, g.M_cap, g.lda, KE, BM, swz) ||
         !make_map_t(&mb, Bk, TF, g.K, g.N, ldbk, KE, BN, swz))
         return false;
@@ -996,6 +1018,13 @@ bool gemm_row_tc(betty_ctx* c, const GemmRow& g, const void* Bk, const void* Bk_
     if (!make_map_t(&mc, g.C, !g.c_bf16, g.N, g.M_cap, g.ldc, 32, 32,
                     g.c_bf16 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_128B))
         return false;
+    // bf16 C: 64-column boxes of 128-byte rows for paired chunks (half the store row segments; the
+    // bf16-storing GEMMs ran at ~4.7 TB/s against 6.5 for the fp32-storing one, ncu r03)
+    if (g.c_bf16) {
+        if (!make_map_t(&mc2, g.C, false, g.N, g.M_cap, g.ldc, 64, 32, CU_TENSOR_MAP_SWIZZLE_128B)) return false;
+    } else {
+        mc2 = mc;
+    }
     RowArgs p{};
     p.M_dev = g.M_dev; p.K = g.K; p.N = g.N; p.BN = BN; p.nk = nk; p.kbb = kbb;
     p.stages = (int)std::max<size_t>(2, std::min<size_t>(8, (budget - fixed) / ring));
@@ -1024,7 +1053,7 @@ bool gemm_row_tc(betty_ctx* c, const GemmRow& g, const void* Bk, const void* Bk_
             cudaFuncSetAttribute(k_tc_row<E, CB, MB, T>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024); \
             attr = true;                                                                           \
         }                                                                                          \
-        k_tc_row<E, CB, MB, T><<<grid, T ? ROW_THREADS_TF : ROW_THREADS, smem, s>>>(ma, mb, mc, mbl, p); \
+        k_tc_row<E, CB, MB, T><<<grid, T ? ROW_THREADS_TF : ROW_THREADS, smem, s>>>(ma, mb, mc, mbl, mc2, p); \
     } while (0)
     if (TF) {
         switch (g.epi) {
