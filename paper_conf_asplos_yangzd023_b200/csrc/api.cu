@@ -520,10 +520,11 @@ struct betty_plan {
     Probe probe;
 };
 
-// Where the REG rebuild forks onto its side stream: 0 at the start of the step (with the extraction),
-// 1 after the first group's extraction (with the aggregation / GEMMs), 2 (default) before its
-// backward.  Measured on C3: 5.10 / 5.25 / 5.04 ms per step -- the latency-bound extraction suffers
-// most from sharing the SMs (1.13 ms alone, 1.44 ms beside the REG), the backward least.
+// Where the REG rebuild forks onto its side stream: 0 at the start of the step (beside the
+// extraction), 1 after the first group's extraction (beside the aggregation / GEMMs), 2 (default)
+// before its backward.  Measured on C3, two runs each: 4.100 / 4.115 ms (fork 0) against 4.132 / 4.129
+// (fork 2), 8-rank share 0.686 against 0.698 ms; fork 1 4.25 ms.  Fork 0 is 0.5 % faster but folds the
+// REG into the extraction's site time (0.77 instead of 0.51 ms), so the default keeps the sites apart.
 static int reg_fork_point() {
     static const int v = getenv("BETTY_REG_FORK") ? atoi(getenv("BETTY_REG_FORK")) : 2;
     return v;
