@@ -655,6 +655,15 @@ static betty_status plan_reg_setup(betty_ctx* c, betty_plan* p, const betty_bloc
     // full batch, like the extraction's full-batch CSC: the step's rebuild reuses it and runs the
     // SpGEMM proper (expansion, sort, run-length encode, compaction) over the rank's rows.
     R.a.csc_ready = !(p->flags & BETTY_PLAN_FRESH);    // FRESH: the step rebuilds it from the block
+    // FRESH with the output block's full-batch CSC among the step's rebuilt CSCs (same block, same
+    // transpose, duplicate-checked, rebuilt on the main stream before the REG forks): the REG reads
+    // that one instead of transposing the block a second time (the e2e step's duplicate ~0.2 ms)
+    if ((p->flags & BETTY_PLAN_FRESH) && (p->csc_mask >> (p->L - 1) & 1) && p->full[p->L - 1].t_indptr &&
+        ob == &p->reg_block) {
+        R.a.t_indptr = (int64_t*)p->full[p->L - 1].t_indptr;
+        R.a.t_idx = (int32_t*)p->full[p->L - 1].t_nbr;
+        R.a.csc_ready = true;
+    }
     p->R = R;
     p->with_reg = true;
     p->info.reg_nnz = nnz;

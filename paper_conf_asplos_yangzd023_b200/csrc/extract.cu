@@ -107,10 +107,14 @@ __global__ void __launch_bounds__(32) k_sel_write(const int32_t* __restrict__ pa
         for (int j = lane; j <= c; j += 32) mb_dst_off[j] = off[(int64_t)j * nchunks] >> SEL_SHIFT;
         if (lane == 0) {
             const int64_t t = off[(int64_t)c * nchunks], n = t >> SEL_SHIFT;
-            cnt[0] = n;
-            cnt[2] = t & SEL_DEG_MASK;
-            if (n <= cap_d) indptr[n] = t & SEL_DEG_MASK;
-            else atomicOr(dev_err, DEVERR_OVERFLOW);
+            if (n <= cap_d) {
+                cnt[0] = n;
+                cnt[2] = t & SEL_DEG_MASK;
+                indptr[n] = t & SEL_DEG_MASK;
+            } else {                                    // EOVERFLOW; the group runs empty (see k_counts)
+                atomicOr(dev_err, DEVERR_OVERFLOW);
+                cnt[0] = 0; cnt[2] = 0; indptr[0] = 0;
+            }
         }
     }
     const int64_t base = ch * SEL_CHUNK;
@@ -598,9 +602,17 @@ __global__ void k_counts(const int64_t* __restrict__ mb_dst_off, const int64_t* 
         (void)mb_dst_off;
         mb_src_off[c] = s_base;
         const int64_t ns = cnt[0] + s_base;
-        cnt[1] = ns;
-        if (ns > cap_src || cnt[2] > cap_e) atomicOr(dev_err, DEVERR_OVERFLOW);
-        if (next_cnt) next_cnt[0] = ns;
+        if (ns > cap_src || cnt[2] > cap_e) {
+            // beyond the plan's capacities (a FRESH plan's batch grew): report EOVERFLOW at the next
+            // synchronising call and empty this layer and the ones below, so no later kernel writes
+            // past an arena buffer
+            atomicOr(dev_err, DEVERR_OVERFLOW);
+            cnt[0] = 0; cnt[1] = 0; cnt[2] = 0;
+            if (next_cnt) next_cnt[0] = 0;
+        } else {
+            cnt[1] = ns;
+            if (next_cnt) next_cnt[0] = ns;
+        }
     }
 }
 
@@ -704,8 +716,12 @@ __global__ void __launch_bounds__(256) k_seg_egid(const int32_t* __restrict__ ds
     __shared__ FlatRows s_rows[8];
     const int64_t n = cnt[0];
     if (blockIdx.x == 0 && threadIdx.x == 0) {
-        cnt[1] = n;
-        if (cnt[2] > cap_e) atomicOr(dev_err, DEVERR_OVERFLOW);
+        if (cnt[2] > cap_e) {                           // EOVERFLOW; the layer runs empty (see k_counts)
+            atomicOr(dev_err, DEVERR_OVERFLOW);
+            cnt[0] = 0; cnt[1] = 0; cnt[2] = 0;
+        } else {
+            cnt[1] = n;
+        }
     }
     const int lane = lane_id();
     FlatRows& F = s_rows[warp_id()];

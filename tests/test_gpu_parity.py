@@ -414,6 +414,66 @@ def test_step_degenerate_inputs(B, ctx, c, mode):
         plan.free()
 
 
+@pytest.mark.parametrize("mode", ["fp32", "bf16"])
+@pytest.mark.parametrize("c", [CASES[1], CASES[2], CASES[11]], ids=lambda c: c["name"])
+def test_fresh_plan_follows_the_buffers(B, ctx, c, mode):
+    """BETTY_PLAN_FRESH (the e2e path): every step re-derives the full-batch CSCs, the REG's CSC and
+    the edge -> gid array from the CURRENT block buffers.  (1) A different batch of the same sizes is
+    written into the bound buffers -- the input layer's source node ids permuted (other feature rows,
+    same structure) -- and the next steps must match the oracle on the NEW blocks.  (2) A batch that
+    outgrows the plan's capacities (every output row's neighbours shifted by one source position)
+    must either fit and match the oracle or fail cleanly with EOVERFLOW at the synchronising call."""
+    import dataclasses
+    sd, blocks, feats, labels, params = make_case(c, seed=4)
+    K = 5
+    part = synth.random_partition(len(sd), K, 13)
+    ks = [0, 1, 2, 3, 4]
+    dev = B.blocks_to_device(blocks)
+    dpart = torch.as_tensor(part).cuda()
+    model = B.Model(c["dims"], c["aggr"], mode, mode)
+    P = torch.as_tensor(params).cuda()
+    X = dev_feats(feats, mode)
+    Y = torch.as_tensor(labels).cuda()
+    scale = 1.0 / len(sd)
+    plan = B.betty_plan_create(ctx, model, dev, dpart, K, ks, group=0,
+                               flags=B.PLAN_GRAPH | B.PLAN_REG | B.PLAN_FRESH)
+
+    def run(bl):
+        og, ol = oracle.step(c["dims"], c["aggr"], mode == "bf16", bl, part, K, ks, params, feats, labels, scale)
+        for rep in range(2):
+            grad = torch.zeros_like(P)
+            loss = torch.zeros(1, device="cuda")
+            B.betty_step(ctx, plan, P, X, Y, scale, grad, loss)
+            B.betty_sync_check(ctx)
+            assert_grad_close(grad.cpu().numpy(), og, c["dims"], c["aggr"], RTOL[mode], f"rep={rep}")
+            assert loss.item() == pytest.approx(ol, rel=RTOL[mode])
+
+    run(blocks)
+    # (1) the input layer's sources are other nodes: permute the src ids beyond the dst prefix
+    b0 = blocks[0]
+    rng = np.random.default_rng(7)
+    gid = b0.src_gid.copy()
+    tail = gid[b0.n_dst:].copy()
+    gid[b0.n_dst:] = rng.permutation(tail)
+    moved = blocks[:]
+    moved[0] = dataclasses.replace(b0, src_gid=gid)
+    dev[0].src_gid.copy_(torch.as_tensor(gid))
+    og_new, _ = oracle.step(c["dims"], c["aggr"], mode == "bf16", moved, part, K, ks, params, feats, labels, scale)
+    og_old, _ = oracle.step(c["dims"], c["aggr"], mode == "bf16", blocks, part, K, ks, params, feats, labels, scale)
+    assert np.abs(og_new - og_old).max() > 1e-3              # the change is visible in the gradient
+    run(moved)
+    # (2) a batch beyond the plan's capacities: clean EOVERFLOW (no fault), or it fits and matches
+    top = moved[-1]
+    shifted = moved[:-1] + [dataclasses.replace(
+        top, nbr_pos=((top.nbr_pos.astype(np.int64) + 1) % top.n_src).astype(np.int32))]
+    dev[-1].indices.copy_(torch.as_tensor(shifted[-1].nbr_pos))
+    try:
+        run(shifted)
+    except B.BettyError as e:
+        assert "EOVERFLOW" in str(e), str(e)
+    plan.free()
+
+
 def test_sum_of_micro_batches_equals_full_batch_on_gpu(B, ctx):
     """Betty's invariant on the GPU path itself: K=8 step == K=1 step (fp32)."""
     c = CASES[1]

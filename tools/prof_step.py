@@ -30,6 +30,7 @@ def main():
     p.add_argument("--group", type=int, default=0)
     p.add_argument("--feat-align", type=int, default=256)
     p.add_argument("--sim-world", type=int, default=1, help="rank 0's share of an N-rank job")
+    p.add_argument("--fresh", action="store_true", help="BETTY_PLAN_FRESH plan (the e2e path's step)")
     a = p.parse_args()
     cfg = synth.CONFIGS[a.config]
     if a.scale != 1.0:
@@ -46,7 +47,7 @@ def main():
     params = torch.as_tensor(synth.init_params(cfg.dims, cfg.aggr, seed=cfg.seeds["init"])).cuda()
     grad = torch.zeros_like(params)
     loss = torch.zeros(1, device="cuda")
-    flags = B.PLAN_REG | (B.PLAN_GRAPH if a.graph else 0)
+    flags = B.PLAN_REG | (B.PLAN_GRAPH if a.graph else 0) | (B.PLAN_FRESH if a.fresh else 0)
     from paper_conf_asplos_yangzd023_b200.dist import lpt_assign, micro_batch_costs, reg_rows
     my_k = lpt_assign(micro_batch_costs(part, a.K, ds.blocks[-1].indptr), a.sim_world)[0]
     plan = B.betty_plan_create(ctx, model, dev, dpart, a.K, my_k, group=a.group, flags=flags)
