@@ -132,7 +132,9 @@ __global__ void __launch_bounds__(256) k_loss(const float* __restrict__ logits, 
 // C <= 64 (every C1-C5 output layer): half a warp per row, 4 consecutive classes per lane as one
 // 16-byte vector, LOSS_V_R rows per half-warp per step -- a quarter of the instructions per row of
 // k_loss (issue-bound there: ~290 warp-instructions per 47-class row, ncu r02r).  Same arithmetic
-// and reduction structure per row (max, sum of exp, lse), dS / dS_act padding columns written as 0.
+// and reduction structure per row (max, sum of exp, lse), dS / dS_act padding columns written as 0;
+// exp / log through the SFU approximations (ex2 / lg2: ~2^-22 relative for the non-positive
+// arguments here, far inside the 1e-5 gradient budget of reading #18).
 constexpr int LOSS_V_R = 2;
 __device__ __forceinline__ float hmax16(float v) {
 #pragma unroll
@@ -188,13 +190,13 @@ __global__ void __launch_bounds__(256) k_loss_v(const float* __restrict__ logits
             float e = 0.f;
 #pragma unroll
             for (int k = 0; k < 4; ++k)
-                if (c0 + k < C) e += expf(x[r][k] - mx[r]);
+                if (c0 + k < C) e += __expf(x[r][k] - mx[r]);
             se[r] = hsum16(e);
         }
 #pragma unroll
         for (int r = 0; r < R; ++r) {
             const int64_t v = v0 + 2 * r + hw;
-            lse[r] = mx[r] + logf(se[r]);
+            lse[r] = mx[r] + __logf(se[r]);
             xy[r] = 0.f;
             if (v < nd) {
                 const float inv = indptr ? (dg[r] > 0 ? 1.f / (float)dg[r] : 0.f) : 1.f;
@@ -203,7 +205,7 @@ __global__ void __launch_bounds__(256) k_loss_v(const float* __restrict__ logits
                 for (int k = 0; k < 4; ++k) {
                     const int c = c0 + k;
                     if (c == y[r]) xy[r] = x[r][k];
-                    d[k] = c < C ? scale * (expf(x[r][k] - lse[r]) - (c == y[r] ? 1.f : 0.f)) : 0.f;
+                    d[k] = c < C ? scale * (__expf(x[r][k] - lse[r]) - (c == y[r] ? 1.f : 0.f)) : 0.f;
                 }
                 if (c0 < ldds)
                     *(float4*)(dS + v * ldds + c0) = make_float4(d[0] * inv, d[1] * inv, d[2] * inv, d[3] * inv);
