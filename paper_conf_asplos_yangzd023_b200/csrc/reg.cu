@@ -478,10 +478,9 @@ void reg_phase2(betty_ctx* c, const RegArgs& a, cudaStream_t s) {
     const int gw = (int)std::max<int64_t>(1, std::min<int64_t>((a.rows_cap * 32 + 255) / 256, (int64_t)c->num_sms * 16));
     k_reg_rows_warp<<<gw, 256, 0, s>>>(a.indptr, a.idx, a.t_indptr, a.t_idx, a.n_rows_dev, a.row0, a.ub, a.off, a.tcol,
                                        a.tw, a.row_nnz);
-    // rows with more than REG_WARP_MAX candidates are rare (C3: a few hundred of 196 K): a few CTAs
-    // (each needs 1024 threads and 128 KB of shared memory, i.e. a whole SM) sweep them
-    static const int cta_grid = getenv("BETTY_REG_CTA_GRID") ? atoi(getenv("BETTY_REG_CTA_GRID")) : 16;
-    k_reg_rows_cta<<<std::max(1, std::min(cta_grid, c->num_sms)), 1024, REG_CTA_MAX * 4, s>>>(a.indptr, a.idx, a.t_indptr, a.t_idx, a.row0, a.ub, a.off,
+    // one CTA per SM over the rows with more than REG_WARP_MAX candidates (a few hundred of 196 K on C3,
+    // but most rows of a full-neighbourhood batch such as C2: a 16-CTA grid took C2 from 8.3 to 17.7 ms)
+    k_reg_rows_cta<<<c->num_sms, 1024, REG_CTA_MAX * 4, s>>>(a.indptr, a.idx, a.t_indptr, a.t_idx, a.row0, a.ub, a.off,
                                                             c->L().big_list, c->L().big_count, a.tcol, a.tw, a.row_nnz,
                                                             a.hub_bits, a.hub_pre, a.hub_words, c->dev_err);
     scan_i64(c, a.row_nnz, a.out_indptr, a.n_rows_dev, 0, a.rows_cap, a.nnz_total_dev, s);
