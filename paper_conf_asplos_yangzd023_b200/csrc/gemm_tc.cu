@@ -192,8 +192,14 @@ constexpr int EPI_WARPS = 8;
 constexpr int ESLOTS = 1;                       // staging slots (4 KB) per epilogue warp (bf16 operands)
 constexpr int ESLOTS_TF = 1;                    // ... FP32 mode (the 3xTF32 ring needs the room)
 constexpr int ROW_THREADS = 64 + 32 * EPI_WARPS;
-constexpr int CONV_WARPS = 4;                   // FP32 mode: hi/lo split of each stage (k_tc_red)
-constexpr int ROW_CONV_WARPS = 2;               // ... of each A stage (k_tc_row; keeps the epilogue unspilled)
+#ifndef BETTY_RED_CONV
+#define BETTY_RED_CONV 4
+#endif
+#ifndef BETTY_ROW_CONV
+#define BETTY_ROW_CONV 2
+#endif
+constexpr int CONV_WARPS = BETTY_RED_CONV;      // FP32 mode: hi/lo split of each stage (k_tc_red)
+constexpr int ROW_CONV_WARPS = BETTY_ROW_CONV;  // ... of each A stage (k_tc_row; keeps the epilogue unspilled)
 constexpr int ROW_THREADS_TF = ROW_THREADS + 32 * ROW_CONV_WARPS;
 constexpr int MAXCH = 4;                        // 32-column chunks per epilogue half (N <= 256)
 struct RowArgs {

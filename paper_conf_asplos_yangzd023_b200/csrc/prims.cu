@@ -1,6 +1,6 @@
 // prims.cu -- device-wide primitives with DEVICE-resident sizes, so that a
 // whole training step runs without host synchronisation (graph-capturable):
-//   * single-pass exclusive scan (decoupled look-back, persistent CTAs)
+//   * single-pass exclusive scan (one chunk per CTA, aggregates exchanged through flags)
 //   * segmented sort of short int32 segments (warp / CTA bitonic)
 //   * CSR -> CSC transpose with ascending row ids per column
 #include <climits>
@@ -11,8 +11,6 @@ namespace betty {
 
 // ------------------------------------------------------------------ scan
 constexpr int SCAN_THREADS = 256;
-constexpr int SCAN_ITEMS = 16;
-constexpr int SCAN_TILE = SCAN_THREADS * SCAN_ITEMS;
 constexpr unsigned long long ST_AGG = 1ull << 62, ST_PRE = 2ull << 62, ST_VAL = (1ull << 62) - 1;
 
 __device__ __forceinline__ unsigned long long ld_acquire(const unsigned long long* p) {
@@ -24,103 +22,121 @@ __device__ __forceinline__ void st_release(unsigned long long* p, unsigned long 
     asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
-// element loader of the scan: plain values
-template <typename Tin> struct LdPlain {
-    const Tin* in;
-    __device__ __forceinline__ int64_t operator()(int64_t i) const { return (int64_t)in[i]; }
-};
+// Chunked single-pass scan: one contiguous chunk per CTA (grid <= 2 x SMs, chunk >= SCAN_CHUNK_MIN
+// elements).  A CTA claims its chunk by ticket (so every lower chunk belongs to a CTA that is already
+// running), reduces it with coalesced vector loads, publishes the aggregate, sums ALL lower chunks'
+// aggregates in one warp-parallel pass (<= 2 x SMs flags, no chain of inclusive prefixes), then
+// scans its chunk (second read from L2) with a running carry.  The earlier tile-by-tile decoupled
+// look-back (4096-element tiles, prefixes propagated 32 tiles per hop) took 35 us for 2.4 M int32
+// and 13 us for 7 tiles -- the hop chain, not the bytes (r05 launch list).
+constexpr int SCAN_CHUNK_MIN = 4096;
+template <typename Tin>
+__device__ __forceinline__ void scan_ld4(const Tin* __restrict__ in, int64_t i, int64_t hi, bool vec, int64_t (&v)[4]) {
+    if (vec && i + 4 <= hi) {
+        if constexpr (sizeof(Tin) == 4) {
+            const int4 x = __ldg(reinterpret_cast<const int4*>(in + i));
+            v[0] = x.x; v[1] = x.y; v[2] = x.z; v[3] = x.w;
+        } else {
+            const longlong2 x = __ldg(reinterpret_cast<const longlong2*>(in + i));
+            const longlong2 y = __ldg(reinterpret_cast<const longlong2*>(in + i) + 1);
+            v[0] = x.x; v[1] = x.y; v[2] = y.x; v[3] = y.y;
+        }
+    } else {
+#pragma unroll
+        for (int q = 0; q < 4; ++q) v[q] = i + q < hi ? (int64_t)in[i + q] : 0;
+    }
+}
 
-template <typename Ld>
-__global__ void __launch_bounds__(SCAN_THREADS) k_scan(const Ld in, int64_t* __restrict__ out,
+template <typename Tin>
+__global__ void __launch_bounds__(SCAN_THREADS) k_scan(const Tin* __restrict__ in, int64_t* __restrict__ out,
                                                        const int64_t* n_dev, int64_t n_fixed, int64_t* total_dev,
                                                        unsigned long long* status, unsigned* ctr) {
     __shared__ int64_t s_warp[SCAN_THREADS / 32 + 1];
-    __shared__ int64_t s_tile, s_prefix;
+    __shared__ int64_t s_prefix;
+    __shared__ unsigned s_c;
     __shared__ int s_last;
     const int64_t n = n_dev ? *n_dev : n_fixed;
-    const int64_t n_tiles = (n + SCAN_TILE - 1) / SCAN_TILE;
-    for (;;) {
-        if (threadIdx.x == 0) s_tile = atomicAdd(&ctr[0], 1u);
-        __syncthreads();
-        const int64_t t = s_tile;
-        if (t >= n_tiles) break;
-        const int64_t base = t * SCAN_TILE + (int64_t)threadIdx.x * SCAN_ITEMS;
-        int64_t v[SCAN_ITEMS];
-        int64_t sum = 0;
-#pragma unroll
-        for (int i = 0; i < SCAN_ITEMS; ++i) {
-            const int64_t idx = base + i;
-            v[i] = idx < n ? in(idx) : 0;
-            sum += v[i];
-        }
-        int64_t agg;
-        const int64_t ex = block_excl_scan(sum, s_warp, &agg);
-        if (threadIdx.x < 32) {
-            // warp-parallel decoupled look-back: inspect the 32 predecessor tiles at
-            // once, add the aggregates after the nearest inclusive prefix, repeat
-            // further back only while no prefix is found
-            const int lane = threadIdx.x;
-            int64_t prefix = 0;
-            if (t == 0) {
-                if (lane == 0) st_release(&status[0], ST_PRE | (unsigned long long)agg);
-            } else {
-                if (lane == 0) st_release(&status[t], ST_AGG | (unsigned long long)agg);
-                int64_t hi = t - 1;                          // window [hi-31, hi]
-                for (;;) {
-                    const int64_t j = hi - lane;
-                    unsigned long long st = j >= 0 ? ld_acquire(&status[j]) : (ST_PRE | 0ull);
-                    // wait until every tile of the window has published something
-                    while (__any_sync(0xffffffffu, (st >> 62) == 0)) {
-                        if ((st >> 62) == 0) st = ld_acquire(&status[j]);
-                    }
-                    const unsigned pre = __ballot_sync(0xffffffffu, (st >> 62) == 2);
-                    // lanes up to and including the nearest PRE (lowest lane index with PRE) contribute
-                    const int stop = pre ? __ffs(pre) - 1 : 31;
-                    int64_t v = lane <= stop ? (int64_t)(st & ST_VAL) : 0;
-#pragma unroll
-                    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
-                    prefix += v;
-                    if (pre) break;
-                    hi -= 32;
-                }
-                if (lane == 0) st_release(&status[t], ST_PRE | (unsigned long long)(prefix + agg));
-            }
-            if (lane == 0) {
-                s_prefix = prefix;
-                if (t == n_tiles - 1 && total_dev) *total_dev = prefix + agg;
-                if (t == 0) out[0] = 0;
-            }
+    const int G = (int)gridDim.x;
+    if (threadIdx.x == 0) s_c = atomicAdd(&ctr[0], 1u);
+    __syncthreads();
+    const int c = (int)s_c;
+    // chunks in use: <= the grid, >= SCAN_CHUNK_MIN elements each (a small n uses few CTAs)
+    const int nch = (int)max((int64_t)1, min((int64_t)G, (n + SCAN_CHUNK_MIN - 1) / SCAN_CHUNK_MIN));
+    const int64_t cs = ((n + nch - 1) / nch + 3) & ~(int64_t)3;     // chunk size, a multiple of 4
+    if (c >= nch) {                                                  // idle CTA: only the cleanup count
+        if (threadIdx.x == 0) {
+            __threadfence();
+            s_last = (atomicAdd(&ctr[1], 1u) == (unsigned)G - 1);
         }
         __syncthreads();
-        int64_t run = s_prefix + ex;
-#pragma unroll
-        for (int i = 0; i < SCAN_ITEMS; ++i) {
-            const int64_t idx = base + i;
-            run += v[i];
-            if (idx < n) out[idx + 1] = run;
+        if (s_last) {
+            for (int j = threadIdx.x; j < nch; j += blockDim.x) status[j] = 0;
+            if (threadIdx.x == 0) { ctr[0] = 0; ctr[1] = 0; }
+            __threadfence();
         }
-        __syncthreads();
+        return;
     }
-    if (n_tiles == 0 && blockIdx.x == 0 && threadIdx.x == 0) {
-        out[0] = 0;
-        if (total_dev) *total_dev = 0;
+    const int64_t lo = min(n, (int64_t)c * cs), hi = min(n, lo + cs);
+    const bool vec = ((uintptr_t)in & 15) == 0;                     // lo is a multiple of 4 elements
+    // 1. the chunk's aggregate
+    int64_t sum = 0;
+    for (int64_t i = lo + 4 * (int64_t)threadIdx.x; i < hi; i += 4 * SCAN_THREADS) {
+        int64_t v[4];
+        scan_ld4(in, i, hi, vec, v);
+        sum += v[0] + v[1] + v[2] + v[3];
     }
-    // the last CTA to finish clears the tile status and the counters
+    int64_t agg;
+    block_excl_scan(sum, s_warp, &agg);
+    // 2. publish it, then sum every lower chunk's aggregate
+    if (threadIdx.x < 32) {
+        const int lane = threadIdx.x;
+        if (lane == 0) st_release(&status[c], ST_AGG | (unsigned long long)agg);
+        int64_t p = 0;
+        for (int j = lane; j < c; j += 32) {
+            unsigned long long st = ld_acquire(&status[j]);
+            while ((st >> 62) == 0) st = ld_acquire(&status[j]);
+            p += (int64_t)(st & ST_VAL);
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) p += __shfl_xor_sync(0xffffffffu, p, o);
+        if (lane == 0) {
+            s_prefix = p;
+            if (c == nch - 1 && total_dev) *total_dev = p + agg;
+            if (c == 0) out[0] = 0;
+        }
+    }
+    __syncthreads();
+    // 3. the chunk's inclusive sums, written to out[i + 1]
+    int64_t run = s_prefix;
+    for (int64_t base = lo; base < hi; base += 4 * SCAN_THREADS) {
+        const int64_t i = base + 4 * (int64_t)threadIdx.x;
+        int64_t v[4];
+        scan_ld4(in, i, hi, vec, v);
+        int64_t tot;
+        int64_t r = run + block_excl_scan(v[0] + v[1] + v[2] + v[3], s_warp, &tot);
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+            r += v[q];
+            if (i + q < hi) out[i + q + 1] = r;
+        }
+        run += tot;
+    }
+    // the last CTA to finish clears the chunk flags and the counters
     __syncthreads();
     if (threadIdx.x == 0) {
         __threadfence();
-        s_last = (atomicAdd(&ctr[1], 1u) == gridDim.x - 1);
+        s_last = (atomicAdd(&ctr[1], 1u) == (unsigned)G - 1);
     }
     __syncthreads();
     if (s_last) {
-        for (int64_t j = threadIdx.x; j < n_tiles; j += blockDim.x) status[j] = 0;
+        for (int j = threadIdx.x; j < nch; j += blockDim.x) status[j] = 0;
         if (threadIdx.x == 0) { ctr[0] = 0; ctr[1] = 0; }
         __threadfence();
     }
 }
 
 void ensure_scan_scratch(betty_ctx* c, int64_t n_cap, cudaStream_t s) {
-    const int64_t tiles = (n_cap + SCAN_TILE - 1) / SCAN_TILE + 1;
+    const int64_t tiles = (n_cap + SCAN_CHUNK_MIN - 1) / SCAN_CHUNK_MIN + 1;   // >= the grid
     if (tiles > c->L().scan_status_cap) {
         // growing is only legal outside graph capture; plan creation sizes it first.  A plan's
         // instantiated CUDA graph holds the old pointer by value, so the old buffer is retired (kept
@@ -134,24 +150,24 @@ void ensure_scan_scratch(betty_ctx* c, int64_t n_cap, cudaStream_t s) {
     }
 }
 
-template <typename Ld>
-static void scan_impl(betty_ctx* c, const Ld in, int64_t* out, const int64_t* n_dev, int64_t n_fixed, int64_t n_cap,
+template <typename Tin>
+static void scan_impl(betty_ctx* c, const Tin* in, int64_t* out, const int64_t* n_dev, int64_t n_fixed, int64_t n_cap,
                       int64_t* total_dev, cudaStream_t s) {
     if (!n_dev) n_cap = n_fixed;
     ensure_scan_scratch(c, n_cap, s);
-    int64_t tiles = (n_cap + SCAN_TILE - 1) / SCAN_TILE;
-    int grid = (int)std::min<int64_t>(std::max<int64_t>(tiles, 1), (int64_t)c->num_sms * 2);
-    k_scan<Ld><<<grid, SCAN_THREADS, 0, s>>>(in, out, n_dev, n_fixed, total_dev, c->L().scan_status,
-                                             c->L().counters + CTR_SCAN);
+    const int64_t chunks = (n_cap + SCAN_CHUNK_MIN - 1) / SCAN_CHUNK_MIN;
+    const int grid = (int)std::min<int64_t>(std::max<int64_t>(chunks, 1), (int64_t)c->num_sms * 2);
+    k_scan<Tin><<<grid, SCAN_THREADS, 0, s>>>(in, out, n_dev, n_fixed, total_dev, c->L().scan_status,
+                                              c->L().counters + CTR_SCAN);
 }
 
 void scan_i64(betty_ctx* c, const int64_t* in, int64_t* out, const int64_t* n_dev, int64_t n_fixed, int64_t n_cap,
               int64_t* total_dev, cudaStream_t s) {
-    scan_impl(c, LdPlain<int64_t>{in}, out, n_dev, n_fixed, n_cap, total_dev, s);
+    scan_impl(c, in, out, n_dev, n_fixed, n_cap, total_dev, s);
 }
 void scan_i32(betty_ctx* c, const int32_t* in, int64_t* out, const int64_t* n_dev, int64_t n_fixed, int64_t n_cap,
               int64_t* total_dev, cudaStream_t s) {
-    scan_impl(c, LdPlain<int32_t>{in}, out, n_dev, n_fixed, n_cap, total_dev, s);
+    scan_impl(c, in, out, n_dev, n_fixed, n_cap, total_dev, s);
 }
 
 // ---------------------------------------------------------------- memset
