@@ -588,7 +588,11 @@ def main():
     if not plans:                                  # no room for a FRESH plan: re-copy into the timed plan
         plans, bufs = [plan], [dev_list(dev_blocks, dpart)]
     h2d = sum(x.numel() * x.element_size() for x in host)
-    loss_host = torch.zeros(1).pin_memory()
+    # every step's loss is read on the host inside the timed region, one step behind the device (the
+    # host waits for step i-1's loss while step i runs, so no step waits on a host round trip)
+    loss_host = [torch.zeros(1).pin_memory() for _ in range(2)]
+    ev_loss = [torch.cuda.Event() for _ in range(2)]
+    losses = []
     cs = torch.cuda.Stream(device=device)
     ev_copied = [torch.cuda.Event() for _ in bufs]
     ev_used = [torch.cuda.Event() for _ in bufs]
@@ -616,12 +620,16 @@ def main():
             copy_in(1 - b)
         step(plans[b])
         ev_used[b].record(stream)
-        loss_host.copy_(loss, non_blocking=True)
-        stream.synchronize()
-        _ = float(loss_host[0])
+        loss_host[i % 2].copy_(loss, non_blocking=True)
+        ev_loss[i % 2].record(stream)
         if nb == 1 and i + 1 < e2e_steps:
             cs.wait_stream(stream)
             copy_in(0)
+        if i >= 1:                                  # step i-1's loss on the host
+            ev_loss[(i - 1) % 2].synchronize()
+            losses.append(float(loss_host[(i - 1) % 2][0]))
+    ev_loss[(e2e_steps - 1) % 2].synchronize()
+    losses.append(float(loss_host[(e2e_steps - 1) % 2][0]))
     f1.record(stream)
     torch.cuda.synchronize()
     e2e_ms = f0.elapsed_time(f1) / e2e_steps
@@ -666,7 +674,9 @@ def main():
                 if roof else None},
             "e2e": {"value": edges_all / (e2e_ms * 1e-3), "unit": "edges/s", "ms_per_step": e2e_ms,
                     "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": 4,
-                    "input_buffers": nb, "fresh_inputs": plans[0] is not plan},
+                    "input_buffers": nb, "fresh_inputs": plans[0] is not plan, "loss_reads": len(losses),
+                    "loss_read": "every step's loss copied to pinned host memory and read on the host, one "
+                                 "step behind the device"},
             "gpu_launches": launches,
             "clocks": clk,
             "roofline": roof,
