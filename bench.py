@@ -286,6 +286,8 @@ def alg_bytes(site: str, info: dict, cfg, mode: str, n_groups: int):
     elif site == "gemm_fwd_l0":
         H = cfg.hidden
         b = s_act * ld_xa * nd[0] + s_act * (2 * Fp + 1) * H + s_act * ((H + 1 + 7) // 8 * 8) * nd[0]
+    elif site == "agg_l0_stream":        # the same formula with every edge's row gathered (no reuse)
+        b = 4 * E[0] + 8 * (nd[0] + 1) + s_feat * F * E[0] + s_act * F * nd[0]
     else:
         return None
     return b / max(n_groups, 1)
@@ -795,12 +797,25 @@ def roofline(plan, step, info, cfg, mode, ms, peaks, peak_src, key):
     if ab is None:
         return None
     achieved = ab / (per_launch_ms * 1e-3) / 1e9
+    sb = alg_bytes("agg_l0_stream", info, cfg, mode, info["n_groups"])
+    rows = (info["edges"][0] + info["n_dst"][0]) / max(info["n_groups"], 1)   # neighbour + self rows fetched
     return {"kernel": "k_agg_mean_g4 (layer-0 mean aggregation)", "bound": "hbm", "achieved": achieved,
             "peak": peaks["hbm_gbs"], "unit": "GB/s", "frac": achieved / peaks["hbm_gbs"],
             "traffic": load_traffic(dom, key), "alg_bytes_per_launch": ab,
             "alg_bytes_formula": "4E + 8(n_dst+1) + s*F*n_src + s*F*n_dst (SURVEY §8(d), distinct sources)",
             "avg_launch_ms": per_launch_ms, "launches_per_step": launches_per_step, "peak_source": peak_src,
             "share_of_step": per_launch_ms * launches_per_step / ms,
+            # context (frac above is the official, compulsory-bytes figure): SURVEY §8(d)'s stream form
+            # of the same formula, s*F*E gathered, and the row-fetch rate against the measured random-row
+            # ceiling of a table larger than L2 (profiles/r03_gather_l2.txt, r03_agg_bound.txt)
+            "stream": {"alg_bytes_per_launch": sb,
+                       "achieved": sb / (per_launch_ms * 1e-3) / 1e9,
+                       "frac": sb / (per_launch_ms * 1e-3) / 1e9 / peaks["hbm_gbs"],
+                       "formula": "4E + 8(n_dst+1) + s*F*E + s*F*n_dst (SURVEY §8(d) AGG-MEAN fwd)"},
+            "row_fetches_per_ns": rows / (per_launch_ms * 1e6),
+            "row_fetch_ceiling_per_ns": {"value": 24.9, "what": "random 208-byte rows from a 0.52 GB table, "
+                                         "LDG at full occupancy (tools/micro/gather_l2.cu); TMA gather4 22.9"}
+            if mode == "bf16" and cfg.F == 100 else None,
             "other_sites_ms_per_step": {k: v[0] * v[1] for k, v in probe_ms.items()}}
 
 
