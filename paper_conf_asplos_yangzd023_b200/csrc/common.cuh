@@ -83,6 +83,10 @@ __host__ __device__ __forceinline__ int64_t mn64(int64_t a, int64_t b) { return 
 
 // ------------------------------------------------------------ warp / block
 __device__ __forceinline__ int lane_id() { return threadIdx.x & 31; }
+// GPU-scope acquire-release fence for the "last CTA reduces" and flag patterns.  __threadfence() is
+// fence.sc.gpu (MEMBAR.SC.GPU), a sequentially-consistent fence that cost the small scans ~10 us each
+// (ncu r06: a 7-CTA scan of 28 K elements ran 15 us with 1 K active cycles per SM)
+__device__ __forceinline__ void fence_gpu() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
 __device__ __forceinline__ int warp_id() { return threadIdx.x >> 5; }
 
 // ascending bitonic sort of one int32 per lane across the warp

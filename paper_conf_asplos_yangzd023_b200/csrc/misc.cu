@@ -107,12 +107,12 @@ __global__ void __launch_bounds__(256) k_loss(const float* __restrict__ logits, 
         double b = 0.0;
         for (int i = 0; i < (int)(blockDim.x >> 5); ++i) b += s_w[i];
         partials[blockIdx.x] = b;
-        __threadfence();
+        fence_gpu();
         s_last = (atomicAdd(&ctr[0], 1u) == gridDim.x - 1);
     }
     __syncthreads();
     if (s_last) {                       // fixed-order reduction of the partials by the last CTA
-        __threadfence();
+        fence_gpu();
         double t = 0.0;
         for (unsigned i = threadIdx.x; i < gridDim.x; i += blockDim.x) t += ((volatile double*)partials)[i];
 #pragma unroll
@@ -228,12 +228,12 @@ __global__ void __launch_bounds__(256) k_loss_v(const float* __restrict__ logits
         double b = 0.0;
         for (int i = 0; i < (int)(blockDim.x >> 5); ++i) b += s_w[i];
         partials[blockIdx.x] = b;
-        __threadfence();
+        fence_gpu();
         s_last = (atomicAdd(&ctr[0], 1u) == gridDim.x - 1);
     }
     __syncthreads();
     if (s_last) {                       // fixed-order reduction of the partials by the last CTA
-        __threadfence();
+        fence_gpu();
         double t = 0.0;
         for (unsigned i = threadIdx.x; i < gridDim.x; i += blockDim.x) t += ((volatile double*)partials)[i];
 #pragma unroll

@@ -22,28 +22,37 @@ __device__ __forceinline__ void st_release(unsigned long long* p, unsigned long 
     asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
-// Chunked single-pass scan: one contiguous chunk per CTA (grid <= 2 x SMs, chunk >= SCAN_CHUNK_MIN
-// elements).  A CTA claims its chunk by ticket (so every lower chunk belongs to a CTA that is already
-// running), reduces it with coalesced vector loads, publishes the aggregate, sums ALL lower chunks'
-// aggregates in one warp-parallel pass (<= 2 x SMs flags, no chain of inclusive prefixes), then
-// scans its chunk (second read from L2) with a running carry.  The earlier tile-by-tile decoupled
-// look-back (4096-element tiles, prefixes propagated 32 tiles per hop) took 35 us for 2.4 M int32
-// and 13 us for 7 tiles -- the hop chain, not the bytes (r05 launch list).
-constexpr int SCAN_CHUNK_MIN = 4096;
+// Chunked single-pass scan: one contiguous run of 4096-element tiles per CTA (grid <= 2 x SMs; a small
+// n uses fewer CTAs), claimed by ticket (so every lower chunk belongs to a CTA that is already running).
+// A thread holds 16 consecutive elements of a tile in registers, loaded by independent 16-byte loads
+// (one memory round trip per tile); the chunk's aggregate is published as a flag word, warp 0 sums ALL
+// lower chunks' aggregates in one warp-parallel pass (no chain of inclusive prefixes), and the chunk is
+// scanned with a running carry (a one-tile chunk -- n <= 1.2 M -- straight from the registers it was
+// reduced from).  ncu r06: the tile-by-tile decoupled look-back took 35 us for 2.4 M int32 (prefixes
+// propagated <= 32 tiles per hop) and a chunk loop with one 4-element load per thread and round trip
+// 15 us for 28 K elements -- latency chains, not bytes.
+constexpr int SCAN_ITEMS = 16;
+constexpr int SCAN_TILE = SCAN_THREADS * SCAN_ITEMS;
 template <typename Tin>
-__device__ __forceinline__ void scan_ld4(const Tin* __restrict__ in, int64_t i, int64_t hi, bool vec, int64_t (&v)[4]) {
-    if (vec && i + 4 <= hi) {
+__device__ __forceinline__ void scan_ld16(const Tin* __restrict__ in, int64_t i, int64_t hi, bool vec,
+                                          int64_t (&v)[SCAN_ITEMS]) {
+    if (vec && i + SCAN_ITEMS <= hi) {
         if constexpr (sizeof(Tin) == 4) {
-            const int4 x = __ldg(reinterpret_cast<const int4*>(in + i));
-            v[0] = x.x; v[1] = x.y; v[2] = x.z; v[3] = x.w;
+            int4 x[4];
+#pragma unroll
+            for (int q = 0; q < 4; ++q) x[q] = __ldg(reinterpret_cast<const int4*>(in + i) + q);
+#pragma unroll
+            for (int q = 0; q < 4; ++q) { v[4 * q] = x[q].x; v[4 * q + 1] = x[q].y; v[4 * q + 2] = x[q].z; v[4 * q + 3] = x[q].w; }
         } else {
-            const longlong2 x = __ldg(reinterpret_cast<const longlong2*>(in + i));
-            const longlong2 y = __ldg(reinterpret_cast<const longlong2*>(in + i) + 1);
-            v[0] = x.x; v[1] = x.y; v[2] = y.x; v[3] = y.y;
+            longlong2 x[8];
+#pragma unroll
+            for (int q = 0; q < 8; ++q) x[q] = __ldg(reinterpret_cast<const longlong2*>(in + i) + q);
+#pragma unroll
+            for (int q = 0; q < 8; ++q) { v[2 * q] = x[q].x; v[2 * q + 1] = x[q].y; }
         }
     } else {
 #pragma unroll
-        for (int q = 0; q < 4; ++q) v[q] = i + q < hi ? (int64_t)in[i + q] : 0;
+        for (int q = 0; q < SCAN_ITEMS; ++q) v[q] = i + q < hi ? (int64_t)in[i + q] : 0;
     }
 }
 
@@ -57,86 +66,96 @@ __global__ void __launch_bounds__(SCAN_THREADS) k_scan(const Tin* __restrict__ i
     __shared__ int s_last;
     const int64_t n = n_dev ? *n_dev : n_fixed;
     const int G = (int)gridDim.x;
-    if (threadIdx.x == 0) s_c = atomicAdd(&ctr[0], 1u);
-    __syncthreads();
-    const int c = (int)s_c;
-    // chunks in use: <= the grid, >= SCAN_CHUNK_MIN elements each (a small n uses few CTAs)
-    const int nch = (int)max((int64_t)1, min((int64_t)G, (n + SCAN_CHUNK_MIN - 1) / SCAN_CHUNK_MIN));
-    const int64_t cs = ((n + nch - 1) / nch + 3) & ~(int64_t)3;     // chunk size, a multiple of 4
-    if (c >= nch) {                                                  // idle CTA: only the cleanup count
-        if (threadIdx.x == 0) {
-            __threadfence();
-            s_last = (atomicAdd(&ctr[1], 1u) == (unsigned)G - 1);
+    const int64_t ntiles = (n + SCAN_TILE - 1) / SCAN_TILE;
+    const int nch = (int)max((int64_t)1, min((int64_t)G, ntiles));     // chunks in use
+    const int64_t tpc = (ntiles + nch - 1) / nch;                        // tiles per chunk
+    const bool solo = G == 1;                        // one CTA: no ticket, no flags, no cleanup
+    if (!solo) {
+        if (threadIdx.x == 0) s_c = atomicAdd(&ctr[0], 1u);
+        __syncthreads();
+    }
+    const int c = solo ? 0 : (int)s_c;
+    if (c < nch) {
+        const int64_t lo = min(n, (int64_t)c * tpc * SCAN_TILE), hi = min(n, lo + tpc * SCAN_TILE);
+        const bool vec = ((uintptr_t)in & 15) == 0;                      // tiles start 64-byte aligned
+        const int64_t toff = (int64_t)threadIdx.x * SCAN_ITEMS;
+        // 1. the chunk's aggregate (a one-tile chunk keeps its values for step 3)
+        int64_t v[SCAN_ITEMS];
+        int64_t sum = 0;
+        scan_ld16(in, lo + toff, hi, vec, v);
+#pragma unroll
+        for (int q = 0; q < SCAN_ITEMS; ++q) sum += v[q];
+#pragma unroll 2
+        for (int64_t base = lo + SCAN_TILE; !solo && base < hi; base += SCAN_TILE) {
+            int64_t w[SCAN_ITEMS];
+            scan_ld16(in, base + toff, hi, vec, w);
+#pragma unroll
+            for (int q = 0; q < SCAN_ITEMS; ++q) sum += w[q];
+        }
+        int64_t agg = 0;
+        if (!solo) block_excl_scan(sum, s_warp, &agg);
+        else if (threadIdx.x == 0) { s_prefix = 0; out[0] = 0; }
+        // 2. publish it, then sum every lower chunk's aggregate
+        if (!solo && threadIdx.x < 32) {
+            const int lane = threadIdx.x;
+            if (lane == 0) st_release(&status[c], ST_AGG | (unsigned long long)agg);
+            int64_t p = 0;
+            for (int j = lane; j < c; j += 32) {
+                unsigned long long st = ld_acquire(&status[j]);
+                while ((st >> 62) == 0) st = ld_acquire(&status[j]);
+                p += (int64_t)(st & ST_VAL);
+            }
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) p += __shfl_xor_sync(0xffffffffu, p, o);
+            if (lane == 0) {
+                s_prefix = p;
+                if (c == nch - 1 && total_dev) *total_dev = p + agg;
+                if (c == 0) out[0] = 0;
+            }
         }
         __syncthreads();
-        if (s_last) {
-            for (int j = threadIdx.x; j < nch; j += blockDim.x) status[j] = 0;
-            if (threadIdx.x == 0) { ctr[0] = 0; ctr[1] = 0; }
-            __threadfence();
-        }
-        return;
-    }
-    const int64_t lo = min(n, (int64_t)c * cs), hi = min(n, lo + cs);
-    const bool vec = ((uintptr_t)in & 15) == 0;                     // lo is a multiple of 4 elements
-    // 1. the chunk's aggregate
-    int64_t sum = 0;
-    for (int64_t i = lo + 4 * (int64_t)threadIdx.x; i < hi; i += 4 * SCAN_THREADS) {
-        int64_t v[4];
-        scan_ld4(in, i, hi, vec, v);
-        sum += v[0] + v[1] + v[2] + v[3];
-    }
-    int64_t agg;
-    block_excl_scan(sum, s_warp, &agg);
-    // 2. publish it, then sum every lower chunk's aggregate
-    if (threadIdx.x < 32) {
-        const int lane = threadIdx.x;
-        if (lane == 0) st_release(&status[c], ST_AGG | (unsigned long long)agg);
-        int64_t p = 0;
-        for (int j = lane; j < c; j += 32) {
-            unsigned long long st = ld_acquire(&status[j]);
-            while ((st >> 62) == 0) st = ld_acquire(&status[j]);
-            p += (int64_t)(st & ST_VAL);
-        }
+        // 3. the chunk's inclusive sums, written to out[i + 1]; the next tile's loads are issued before
+        // this tile's block scan (a solo CTA walks many tiles)
+        int64_t run = s_prefix;
+        for (int64_t base = lo; base < hi; base += SCAN_TILE) {
+            const int64_t i = base + toff;
+            int64_t nx[SCAN_ITEMS];
+            if (base + SCAN_TILE < hi) scan_ld16(in, i + SCAN_TILE, hi, vec, nx);
+            int64_t ts = 0;
 #pragma unroll
-        for (int o = 16; o > 0; o >>= 1) p += __shfl_xor_sync(0xffffffffu, p, o);
-        if (lane == 0) {
-            s_prefix = p;
-            if (c == nch - 1 && total_dev) *total_dev = p + agg;
-            if (c == 0) out[0] = 0;
-        }
-    }
-    __syncthreads();
-    // 3. the chunk's inclusive sums, written to out[i + 1]
-    int64_t run = s_prefix;
-    for (int64_t base = lo; base < hi; base += 4 * SCAN_THREADS) {
-        const int64_t i = base + 4 * (int64_t)threadIdx.x;
-        int64_t v[4];
-        scan_ld4(in, i, hi, vec, v);
-        int64_t tot;
-        int64_t r = run + block_excl_scan(v[0] + v[1] + v[2] + v[3], s_warp, &tot);
+            for (int q = 0; q < SCAN_ITEMS; ++q) ts += v[q];
+            int64_t tot;
+            int64_t r = run + block_excl_scan(ts, s_warp, &tot);
 #pragma unroll
-        for (int q = 0; q < 4; ++q) {
-            r += v[q];
-            if (i + q < hi) out[i + q + 1] = r;
+            for (int q = 0; q < SCAN_ITEMS; ++q) {
+                r += v[q];
+                if (i + q < hi) out[i + q + 1] = r;
+            }
+            run += tot;
+            if (base + SCAN_TILE < hi) {
+#pragma unroll
+                for (int q = 0; q < SCAN_ITEMS; ++q) v[q] = nx[q];
+            }
         }
-        run += tot;
+        if (solo && threadIdx.x == 0 && total_dev) *total_dev = run;
     }
+    if (solo) return;
     // the last CTA to finish clears the chunk flags and the counters
     __syncthreads();
     if (threadIdx.x == 0) {
-        __threadfence();
+        fence_gpu();
         s_last = (atomicAdd(&ctr[1], 1u) == (unsigned)G - 1);
     }
     __syncthreads();
     if (s_last) {
         for (int j = threadIdx.x; j < nch; j += blockDim.x) status[j] = 0;
         if (threadIdx.x == 0) { ctr[0] = 0; ctr[1] = 0; }
-        __threadfence();
+        fence_gpu();
     }
 }
 
 void ensure_scan_scratch(betty_ctx* c, int64_t n_cap, cudaStream_t s) {
-    const int64_t tiles = (n_cap + SCAN_CHUNK_MIN - 1) / SCAN_CHUNK_MIN + 1;   // >= the grid
+    const int64_t tiles = (n_cap + SCAN_TILE - 1) / SCAN_TILE + 1;   // >= the grid
     if (tiles > c->L().scan_status_cap) {
         // growing is only legal outside graph capture; plan creation sizes it first.  A plan's
         // instantiated CUDA graph holds the old pointer by value, so the old buffer is retired (kept
@@ -155,7 +174,9 @@ static void scan_impl(betty_ctx* c, const Tin* in, int64_t* out, const int64_t* 
                       int64_t* total_dev, cudaStream_t s) {
     if (!n_dev) n_cap = n_fixed;
     ensure_scan_scratch(c, n_cap, s);
-    const int64_t chunks = (n_cap + SCAN_CHUNK_MIN - 1) / SCAN_CHUNK_MIN;
+    // one chunk of tiles per CTA; a one-tile scan runs on one CTA without flags or atomics (one CTA
+    // walking up to 16 tiles alone was measured slower: C3 step 4.087 -> 4.117 ms)
+    const int64_t chunks = (n_cap + SCAN_TILE - 1) / SCAN_TILE;
     const int grid = (int)std::min<int64_t>(std::max<int64_t>(chunks, 1), (int64_t)c->num_sms * 2);
     k_scan<Tin><<<grid, SCAN_THREADS, 0, s>>>(in, out, n_dev, n_fixed, total_dev, c->L().scan_status,
                                               c->L().counters + CTR_SCAN);
