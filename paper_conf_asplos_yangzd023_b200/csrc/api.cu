@@ -546,8 +546,8 @@ static void step_body(betty_ctx* c, betty_plan* p, const float* params, const vo
         c->lane = 0;
         cudaEventRecord(p->ev_join, p->side);
     };
-    if ((p->flags & BETTY_PLAN_FRESH) && p->lean0)      // full-batch edge -> gid of layer 0
-        full_egid(c, p->full[0].nbr, p->full[0].src_gid, p->full[0].n_edges, (int32_t*)p->full[0].egid, s);
+    // FRESH: the lean layer 0 reads src_gid[nbr[e]] directly (ExtractArgs::egid_direct) instead of a
+    // rebuilt full-batch edge -> gid array (one pass over the full batch's 20 M edges less per step)
     if (p->flags & BETTY_PLAN_FRESH) {        // full-batch CSCs from the current block buffers
         for (int l = 0; l < p->L; ++l) {
             if (!(p->csc_mask >> l & 1)) continue;
@@ -567,6 +567,7 @@ static void step_body(betty_ctx* c, betty_plan* p, const float* params, const vo
         a.ks = p->d_ks + g * p->c; a.c = (int32_t)p->groups[g].size();
         a.layers = p->X.layers.data(); a.sc = p->X.sc; a.csc_mask = p->csc_mask;
         a.lean0 = p->lean0;
+        a.egid_direct = (p->flags & BETTY_PLAN_FRESH) != 0;
         if (pr) pr->begin(PROBE_EXTRACT, s);
         extract_group(c, a, s);
         if (pr) pr->end(PROBE_EXTRACT, s);

@@ -708,9 +708,12 @@ __global__ void k_order_tab(int32_t c, int L, int l, const int64_t* __restrict__
 
 // lean layer 0: each dst row's full-batch edge segment of source gids -> the group's egid (rows in
 // their group order; warp-flattened like the relabel, coalesced within a row); n_src := n_dst
+// (fnbr, fsrc_gid non-null: the gid of edge f is fsrc_gid[fnbr[f]], read directly -- a FRESH step)
 __global__ void __launch_bounds__(256) k_seg_egid(const int32_t* __restrict__ dst_pos, int64_t* cnt,
                                                   const int64_t* __restrict__ findptr,
                                                   const int32_t* __restrict__ fegid,
+                                                  const int32_t* __restrict__ fnbr,
+                                                  const int32_t* __restrict__ fsrc_gid,
                                                   const int64_t* __restrict__ indptr, int32_t* __restrict__ egid,
                                                   int64_t cap_e, int* dev_err) {
     __shared__ FlatRows s_rows[8];
@@ -751,9 +754,13 @@ __global__ void __launch_bounds__(256) k_seg_egid(const int32_t* __restrict__ ds
                 o[u] = -1;
                 if (f < total) {
                     const int k = flat_row(F, f);
-                    g[u] = fegid[F.fb[k] + (f - F.pre[k])];
+                    g[u] = fnbr ? fnbr[F.fb[k] + (f - F.pre[k])] : fegid[F.fb[k] + (f - F.pre[k])];
                     o[u] = F.ob[k] + (f - F.pre[k]);
                 }
+            }
+            if (fnbr) {
+#pragma unroll
+                for (int u = 0; u < FLAT_UNR; ++u) if (o[u] >= 0) g[u] = fsrc_gid[g[u]];
             }
 #pragma unroll
             for (int u = 0; u < FLAT_UNR; ++u) if (o[u] >= 0 && o[u] < cap_e) egid[o[u]] = g[u];
@@ -840,8 +847,9 @@ void extract_group(betty_ctx* ctx, const ExtractArgs& a, cudaStream_t s) {
             k_emit_dst<<<grid_for(ctx, cap_d, 256), 256, 0, s>>>(dst_pos, row_mb, B.cnt, dst_off, B.mb_src_off,
                                                                  F.src_gid, B.src_pos, B.src_gid, B.src_mb, cap_s,
                                                                  nullptr, nullptr, nullptr);
-            k_seg_egid<<<grid_for(ctx, (cap_d + 31) / 32 * 32, 256), 256, 0, s>>>(dst_pos, B.cnt, F.indptr, F.egid,
-                                                                                  B.indptr, B.egid, cap_e, ctx->dev_err);
+            k_seg_egid<<<grid_for(ctx, (cap_d + 31) / 32 * 32, 256), 256, 0, s>>>(
+                dst_pos, B.cnt, F.indptr, F.egid, a.egid_direct ? F.nbr : nullptr, a.egid_direct ? F.src_gid : nullptr,
+                B.indptr, B.egid, cap_e, ctx->dev_err);
             break;
         }
         // dedupe: dst bitmap + position map, then new-source bitmap

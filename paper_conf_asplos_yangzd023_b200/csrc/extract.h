@@ -106,6 +106,10 @@ struct ExtractArgs {
     // gathered by global id from the resident table, no kernel reads the layer's src list, local
     // indices or CSC.  The plan's step sets it; standalone / inspection extractions never do.
     bool lean0 = false;
+    // egid_direct: the lean layer 0 reads each edge's source gid as src_gid[nbr[e]] of the full batch
+    // instead of the per-plan full[0].egid array (a FRESH step: its blocks change every step, so the
+    // array would be rebuilt first -- one more pass over the full batch's edges)
+    bool egid_direct = false;
 };
 
 void extract_group(betty_ctx* ctx, const ExtractArgs& a, cudaStream_t s);

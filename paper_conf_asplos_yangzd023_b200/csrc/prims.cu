@@ -225,9 +225,11 @@ __device__ void smem_bitonic(int32_t* s, int P, int tid, int nthreads, bool warp
     }
 }
 
+// dup: also flag a repeated key inside a segment (DEVERR_DUP_EDGE; the transpose's repeated-edge check,
+// folded into the sort instead of a separate pass over the CSC)
 __global__ void __launch_bounds__(256) k_segsort_warp(const int64_t* __restrict__ ptr, int32_t* __restrict__ keys,
                                                       const int64_t* nseg_dev, int64_t nseg_fixed, int64_t* big,
-                                                      int* big_cnt, int64_t big_cap, int* dev_err) {
+                                                      int* big_cnt, int64_t big_cap, int* dev_err, int dup) {
     __shared__ int32_t buf[8][SEG_WARP_MAX];
     const int64_t nseg = nseg_dev ? *nseg_dev : nseg_fixed;
     const int w = warp_id(), lane = lane_id();
@@ -251,6 +253,12 @@ __global__ void __launch_bounds__(256) k_segsort_warp(const int64_t* __restrict_
                     if (k[j] < k[j - 1]) { const int32_t t = k[j]; k[j] = k[j - 1]; k[j - 1] = t; }
 #pragma unroll
             for (int i = 0; i < SEG_THREAD_MAX; ++i) if (i < ml) keys[mb + i] = k[i];
+            if (dup) {
+                bool rep = false;
+#pragma unroll
+                for (int i = 1; i < SEG_THREAD_MAX; ++i) rep |= i < ml && k[i] == k[i - 1];
+                if (rep) atomicOr(dev_err, DEVERR_DUP_EDGE);
+            }
         }
         unsigned long_mask = __ballot_sync(0xffffffffu, ml > SEG_THREAD_MAX);
         while (long_mask) {
@@ -262,13 +270,18 @@ __global__ void __launch_bounds__(256) k_segsort_warp(const int64_t* __restrict_
                 int32_t x = lane < len ? keys[b + lane] : INT_MAX;
                 x = warp_bitonic32(x);
                 if (lane < len) keys[b + lane] = x;
+                const int32_t prev = __shfl_up_sync(0xffffffffu, x, 1);
+                if (dup && lane > 0 && lane < len && x == prev) atomicOr(dev_err, DEVERR_DUP_EDGE);
             } else if (len <= SEG_WARP_MAX) {
                 int P = 64;
                 while (P < len) P <<= 1;
                 for (int i = lane; i < P; i += 32) buf[w][i] = i < len ? keys[b + i] : INT_MAX;
                 __syncwarp();
                 smem_bitonic(buf[w], P, lane, 32, true);
-                for (int i = lane; i < len; i += 32) keys[b + i] = buf[w][i];
+                for (int i = lane; i < len; i += 32) {
+                    keys[b + i] = buf[w][i];
+                    if (dup && i > 0 && buf[w][i] == buf[w][i - 1]) atomicOr(dev_err, DEVERR_DUP_EDGE);
+                }
                 __syncwarp();
             } else if (lane == 0) {
                 const int i = atomicAdd(big_cnt, 1);
@@ -279,7 +292,7 @@ __global__ void __launch_bounds__(256) k_segsort_warp(const int64_t* __restrict_
 }
 
 __global__ void __launch_bounds__(1024) k_segsort_big(const int64_t* __restrict__ ptr, int32_t* __restrict__ keys,
-                                                      const int64_t* big, int* big_cnt, int* dev_err) {
+                                                      const int64_t* big, int* big_cnt, int* dev_err, int dup) {
     extern __shared__ int32_t sbuf[];
     const int n_big = *big_cnt;
     for (int t = blockIdx.x; t < n_big; t += gridDim.x) {
@@ -294,7 +307,10 @@ __global__ void __launch_bounds__(1024) k_segsort_big(const int64_t* __restrict_
         for (int i = threadIdx.x; i < P; i += blockDim.x) sbuf[i] = i < len ? keys[b + i] : INT_MAX;
         __syncthreads();
         smem_bitonic(sbuf, P, threadIdx.x, blockDim.x, false);
-        for (int i = threadIdx.x; i < len; i += blockDim.x) keys[b + i] = sbuf[i];
+        for (int i = threadIdx.x; i < len; i += blockDim.x) {
+            keys[b + i] = sbuf[i];
+            if (dup && i > 0 && sbuf[i] == sbuf[i - 1]) atomicOr(dev_err, DEVERR_DUP_EDGE);
+        }
         __syncthreads();
     }
 }
@@ -305,14 +321,19 @@ void init_prims_attrs() {
     cudaFuncSetAttribute(k_segsort_big, cudaFuncAttributeMaxDynamicSharedMemorySize, SEG_CTA_MAX * 4);
 }
 
-void segsort_i32(betty_ctx* c, const int64_t* ptr, int32_t* keys, const int64_t* nseg_dev, int64_t nseg_fixed,
-                 int64_t nseg_cap, cudaStream_t s) {
+static void segsort_impl(betty_ctx* c, const int64_t* ptr, int32_t* keys, const int64_t* nseg_dev, int64_t nseg_fixed,
+                         int64_t nseg_cap, bool dup, cudaStream_t s) {
     if (!nseg_dev) nseg_cap = nseg_fixed;
     int grid = (int)std::min<int64_t>((nseg_cap + 255) / 256 + 1, (int64_t)c->num_sms * 8);
     k_reset_int<<<1, 1, 0, s>>>(c->L().big_count);
     k_segsort_warp<<<grid, 256, 0, s>>>(ptr, keys, nseg_dev, nseg_fixed, c->L().big_list, c->L().big_count, c->L().big_list_cap,
-                                        c->dev_err);
-    k_segsort_big<<<c->num_sms, 1024, SEG_CTA_MAX * 4, s>>>(ptr, keys, c->L().big_list, c->L().big_count, c->dev_err);
+                                        c->dev_err, dup ? 1 : 0);
+    k_segsort_big<<<c->num_sms, 1024, SEG_CTA_MAX * 4, s>>>(ptr, keys, c->L().big_list, c->L().big_count, c->dev_err,
+                                                            dup ? 1 : 0);
+}
+void segsort_i32(betty_ctx* c, const int64_t* ptr, int32_t* keys, const int64_t* nseg_dev, int64_t nseg_fixed,
+                 int64_t nseg_cap, cudaStream_t s) {
+    segsort_impl(c, ptr, keys, nseg_dev, nseg_fixed, nseg_cap, false, s);
 }
 
 // ------------------------------------------------------------- transpose
@@ -333,18 +354,10 @@ __global__ void k_scatter_t(const int64_t* __restrict__ indptr, const int32_t* _
         const int64_t b = indptr[r], e = indptr[r + 1];
         for (int64_t i = b + lane; i < e; i += 32) {
             const int32_t col = idx[i];
-            const int32_t k = atomicAdd(&cursor[col], 1);
+            const int32_t k = atomicSub(&cursor[col], 1) - 1;     // the histogram counts down to 0
             t_idx[t_indptr[col] + k] = (int32_t)r;
         }
     }
-}
-
-__global__ void k_dup_check(const int64_t* __restrict__ t_indptr, const int32_t* __restrict__ t_idx,
-                            const int64_t* n_cols_dev, int* dev_err) {
-    const int64_t n = *n_cols_dev;
-    for (int64_t col = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; col < n; col += (int64_t)gridDim.x * blockDim.x)
-        for (int64_t i = t_indptr[col] + 1; i < t_indptr[col + 1]; ++i)
-            if (t_idx[i] == t_idx[i - 1]) { atomicOr(dev_err, DEVERR_DUP_EDGE); break; }
 }
 
 void csr_transpose(betty_ctx* c, const int64_t* indptr, const int32_t* idx, const int64_t* n_rows_dev,
@@ -356,13 +369,8 @@ void csr_transpose(betty_ctx* c, const int64_t* indptr, const int32_t* idx, cons
     memset_dev(cnt, 0, n_cols_dev, 4, cols_cap, s);
     k_hist<<<g_e, 256, 0, s>>>(idx, n_edges_dev, cnt);
     scan_i32(c, cnt, t_indptr, n_cols_dev, 0, cols_cap, nullptr, s);
-    memset_dev(cnt, 0, n_cols_dev, 4, cols_cap, s);
     k_scatter_t<<<g_r, 256, 0, s>>>(indptr, idx, n_rows_dev, t_indptr, cnt, t_idx);
-    segsort_i32(c, t_indptr, t_idx, n_cols_dev, 0, cols_cap, s);
-    if (dup_check) {
-        const int g_c = (int)std::min<int64_t>((cols_cap + 255) / 256 + 1, (int64_t)c->num_sms * 8);
-        k_dup_check<<<g_c, 256, 0, s>>>(t_indptr, t_idx, n_cols_dev, c->dev_err);
-    }
+    segsort_impl(c, t_indptr, t_idx, n_cols_dev, 0, cols_cap, dup_check, s);   // (+ the repeated-edge check)
 }
 
 }  // namespace betty
