@@ -202,6 +202,7 @@ constexpr int CONV_WARPS = BETTY_RED_CONV;      // FP32 mode: hi/lo split of eac
 constexpr int ROW_CONV_WARPS = BETTY_ROW_CONV;  // ... of each A stage (k_tc_row; keeps the epilogue unspilled)
 constexpr int ROW_THREADS_TF = ROW_THREADS + 32 * ROW_CONV_WARPS;
 constexpr int MAXCH = 4;                        // 32-column chunks per epilogue half (N <= 256)
+constexpr int TQ = 4;                           // tile queue entries (producer -> MMA / epilogue / converters)
 struct RowArgs {
     const int64_t* M_dev;
     int K, N, BN, nk, stages;
@@ -219,6 +220,8 @@ struct RowArgs {
     int bstream;             // 1: B is streamed with A through the ring (B too large to stay resident)
     int hw_hi;               // TF: converter writes lo only (see split_tf32_lo)
     int64_t cend;            // trailing columns [N, cend) of a row are written (ones column / zeros)
+    unsigned* tctr;          // [2] dynamic tile claims (next tile, CTAs done; zero between launches), or
+                             // null: static round-robin tiles
     int kbb;                 // bytes per row of one k-block: 128 (SWIZZLE_128B), or 64 (TF: SWIZZLE_64B,
                              // half the ring stage -> twice the stages when B streams or sits resident)
 };
@@ -402,17 +405,34 @@ k_tc_row(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtens
     uint64_t* tempty = tfull + 2;     // [2]
     uint64_t* bfull = tempty + 2;     // [1]
     uint64_t* conv = bfull + 1;       // [S] (TF) A stage split into hi / lo
-    uint32_t* tslot = (uint32_t*)(conv + (TF ? S : 0));
+    uint64_t* tqf = conv + (TF ? S : 0);   // [TQ] tile queue: entry published by the producer
+    uint64_t* tqe = tqf + TQ;              // [TQ] ... read by every consumer warp
+    int32_t* tq = (int32_t*)(tqe + TQ);    // [TQ] tile ids (-1: no more tiles)
+    uint32_t* tslot = (uint32_t*)(tq + TQ);
 
     const int warp = threadIdx.x >> 5;
     const int64_t M = *p.M_dev;
     const int64_t tiles = (M + BM - 1) / BM;
+    // consumers of a queue entry: the MMA warp, the epilogue warps (+ the converter warps)
+    constexpr int TQ_READERS = 1 + EPI_WARPS + (TF ? ROW_CONV_WARPS : 0);
+    // one warp's read of the next queue entry (every lane gets the tile id)
+    int tq_i = 0;
+    uint32_t tq_ph = 0;
+    auto tq_pop = [&]() -> int64_t {
+        mbar_wait(&tqf[tq_i], tq_ph);
+        const int32_t t = tq[tq_i];
+        __syncwarp();
+        if ((threadIdx.x & 31) == 0) mbar_arrive(&tqe[tq_i]);
+        if (++tq_i == TQ) { tq_i = 0; tq_ph ^= 1; }
+        return t;
+    };
 
     if (threadIdx.x == 0) {
         for (int s = 0; s < S; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
         for (int a = 0; a < 2; ++a) { mbar_init(&tfull[a], 1); mbar_init(&tempty[a], 32 * EPI_WARPS); }
         mbar_init(bfull, 1);
         if (TF) for (int s = 0; s < S; ++s) mbar_init(&conv[s], ROW_CONV_WARPS);
+        for (int i = 0; i < TQ; ++i) { mbar_init(&tqf[i], 1); mbar_init(&tqe[i], TQ_READERS); }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
         asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmA) : "memory");
         asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmB) : "memory");
@@ -427,20 +447,38 @@ k_tc_row(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtens
     const uint32_t tmem = *tslot;
 
     if (warp == 0) {
-        if (elect_lane0() && blockIdx.x < tiles) {
+        if (elect_lane0()) {
             const int KE = TF ? p.kbb / 4 : BK;              // elements per k-block
-            if (!p.bstream) {
-                mbar_expect_tx(bfull, NSPLIT * p.nk * bblk);
-                for (int kb = 0; kb < p.nk; ++kb) {
-                    tma_2d(bres + kb * bblk, &tmB, kb * KE, 0, bfull);
-                    if (TF) tma_2d(bres + (p.nk + kb) * bblk, &tmBlo, kb * KE, 0, bfull);
-                }
-            }
             // TF stage: [A | A lo | B | B lo]; TMA fills A, B, B lo (the converter writes A lo)
             const uint32_t land = ring_bytes - (TF ? a_bytes : 0u);
             int s = 0;
             uint32_t ph = 0;
-            for (int64_t t = blockIdx.x; t < tiles; t += gridDim.x) {
+            int q = 0;
+            uint32_t qph = 0;
+            bool bload = !p.bstream;
+            // Tiles are claimed one at a time from a global counter (p.tctr) and queued for the other
+            // roles, so a CTA that starts late (its SM still held by a concurrent kernel, e.g. the REG
+            // on the side stream) takes fewer tiles instead of delaying the whole GEMM; each output
+            // row is still computed by exactly one CTA, so the result does not depend on the order.
+            int64_t tn = p.tctr ? (int64_t)atomicAdd(p.tctr, 1u) : (int64_t)blockIdx.x;
+            for (;;) {
+                const int64_t t = tn;
+                const bool end = t >= tiles;
+                mbar_wait(&tqe[q], qph ^ 1);
+                tq[q] = end ? -1 : (int32_t)t;
+                mbar_arrive(&tqf[q]);
+                if (++q == TQ) { q = 0; qph ^= 1; }
+                if (end) break;
+                // the next claim's round trip overlaps this tile's loads
+                tn = p.tctr ? (int64_t)atomicAdd(p.tctr, 1u) : t + gridDim.x;
+                if (bload) {                                 // B resident: loaded before the first tile
+                    bload = false;
+                    mbar_expect_tx(bfull, NSPLIT * p.nk * bblk);
+                    for (int kb = 0; kb < p.nk; ++kb) {
+                        tma_2d(bres + kb * bblk, &tmB, kb * KE, 0, bfull);
+                        if (TF) tma_2d(bres + (p.nk + kb) * bblk, &tmBlo, kb * KE, 0, bfull);
+                    }
+                }
                 for (int kb = 0; kb < p.nk; ++kb) {
                     mbar_wait(&empty[s], ph ^ 1);
                     mbar_expect_tx(&full[s], land);
@@ -459,8 +497,10 @@ k_tc_row(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtens
         int s = 0;
         uint32_t ph = 0;
         int it = 0;
-        if (blockIdx.x < tiles && !p.bstream) mbar_wait(bfull, 0);
-        for (int64_t t = blockIdx.x; t < tiles; t += gridDim.x, ++it) {
+        bool bready = p.bstream;
+        for (;; ++it) {
+            if (tq_pop() < 0) break;
+            if (!bready) { mbar_wait(bfull, 0); bready = true; }
             const int acc = it % p.nbuf;
             const uint32_t aph = (it / p.nbuf) & 1;
             mbar_wait(&tempty[acc], aph ^ 1);
@@ -511,7 +551,7 @@ k_tc_row(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtens
         const int tid = (warp - 2 - EPI_WARPS) * 32 + (threadIdx.x & 31);
         int s = 0;
         uint32_t ph = 0;
-        for (int64_t t = blockIdx.x; t < tiles; t += gridDim.x) {
+        while (tq_pop() >= 0) {
             for (int kb = 0; kb < p.nk; ++kb) {
                 mbar_wait(&full[s], ph);
                 const uint32_t a = su32(aring + s * ring_bytes);
@@ -553,14 +593,17 @@ k_tc_row(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtens
         for (int ci = 0; ci < MAXCH; ++ci) mw_next[ci] = 0u;
         auto load_bits = [&](int64_t tt, uint32_t (&dst)[MAXCH]) {
             const int64_t mm = tt * BM + q * 32 + lane;
-            if (tt < tiles && mm < M) {
+            if (tt >= 0 && tt < tiles && mm < M) {
                 const uint32_t* wb = p.mbits + mm * p.ldmb + cbeg / 32;
 #pragma unroll
                 for (int ci = 0; ci < MAXCH; ++ci) if (ci < nch) dst[ci] = wb[ci];
             }
         };
-        if (HAS_MASK && MBITS) load_bits(blockIdx.x, mw_next);
-        for (int64_t t = blockIdx.x; t < tiles; t += gridDim.x, ++it) {
+        // the queue is read one entry ahead: the next tile's ReLU' bits are prefetched during this one
+        int64_t t_next = tq_pop();
+        if (HAS_MASK && MBITS) load_bits(t_next, mw_next);
+        for (int64_t t = t_next; t >= 0; t = t_next, ++it) {
+            t_next = tq_pop();
             const int acc = it % p.nbuf;
             const uint32_t aph = (it / p.nbuf) & 1;
             const int64_t row0 = t * BM + q * 32;
@@ -574,7 +617,7 @@ k_tc_row(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtens
                 if (MBITS) {
 #pragma unroll
                     for (int ci = 0; ci < MAXCH; ++ci) { mw[ci] = ok ? mw_next[ci] : 0u; mw_next[ci] = 0u; }
-                    load_bits(t + gridDim.x, mw_next);
+                    load_bits(t_next, mw_next);
                 } else {
 #pragma unroll
                     for (int ci = 0; ci < MAXCH; ++ci) if (ci < nch) mw[ci] = mask_word_from_act(p, m, cbeg + 32 * ci, ok);
@@ -676,6 +719,16 @@ k_tc_row(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtens
     if (warp == 1) {
         fence_after();
         tmem_free_warp(tmem, p.tmem_cols);
+    }
+    // the last CTA to finish resets the tile counter for the next launch (every claim, the one past
+    // the last tile included, happened before its CTA got here)
+    if (p.tctr && threadIdx.x == 0) {
+        fence_gpu();
+        if (atomicAdd(&p.tctr[1], 1u) == gridDim.x - 1) {
+            p.tctr[0] = 0;
+            p.tctr[1] = 0;
+            fence_gpu();
+        }
     }
 }
 
@@ -1006,9 +1059,9 @@ bool gemm_row_tc(betty_ctx* c, const GemmRow& g, const void* Bk, const void* Bk_
         b_bytes = (size_t)nk * bblk * NS;
         a_bytes = (size_t)BM * kbb * NS;
         // B resident when it fits next to a 2-stage A ring, else streamed with A
-        bstream = b_bytes + stage_bytes + 2 * a_bytes + 1024 + 256 > budget;
+        bstream = b_bytes + stage_bytes + 2 * a_bytes + 1024 + 512 > budget;   // 512: barriers, tile queue
         ring = a_bytes + (bstream ? bblk * NS : 0);
-        fixed = (bstream ? 0 : b_bytes) + stage_bytes + 1024 + 256;
+        fixed = (bstream ? 0 : b_bytes) + stage_bytes + 1024 + 512;
         const bool want64 = TF && kbb_env != 128;
         if (pass == 0 && want64) { kbb = 64; continue; }
         break;
@@ -1033,6 +1086,9 @@ bool gemm_row_tc(betty_ctx* c, const GemmRow& g, const void* Bk, const void* Bk_
     }
     RowArgs p{};
     p.M_dev = g.M_dev; p.K = g.K; p.N = g.N; p.BN = BN; p.nk = nk; p.kbb = kbb;
+    // dynamic tile claims (BETTY_GEMM_STATIC=1: the round-robin assignment, for A/B runs)
+    static const bool gemm_static = getenv("BETTY_GEMM_STATIC") && atoi(getenv("BETTY_GEMM_STATIC")) != 0;
+    p.tctr = gemm_static ? nullptr : c->L().counters + CTR_GEMM;
     p.stages = (int)std::max<size_t>(2, std::min<size_t>(8, (budget - fixed) / ring));
     p.bstream = bstream ? 1 : 0;
     static const int hw_hi_row = getenv("BETTY_TF32_HW_HI") ? atoi(getenv("BETTY_TF32_HW_HI")) : 0;

@@ -35,7 +35,7 @@ struct betty_ctx {
 namespace betty {
 
 enum { DEVERR_OVERFLOW = 1, DEVERR_DUP_EDGE = 2, DEVERR_BAD_PART = 4 };
-enum { CTR_SCAN = 0, CTR_SCAN_DONE = 1, CTR_LOSS = 4, CTR_LOSS_DONE = 5, CTR_AGG = 8, CTR_EXTRACT = 10 };
+enum { CTR_SCAN = 0, CTR_SCAN_DONE = 1, CTR_LOSS = 4, CTR_LOSS_DONE = 5, CTR_AGG = 8, CTR_EXTRACT = 10, CTR_GEMM = 32 };
 
 void* ctx_alloc(betty_ctx* c, size_t bytes, cudaStream_t s);
 void ensure_scan_scratch(betty_ctx* c, int64_t n_cap, cudaStream_t s);
