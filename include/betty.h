@@ -51,7 +51,12 @@ typedef void (*betty_free_fn)(void* ptr, betty_stream stream, void* user);
 /* One context per device (per rank).  alloc/free may be NULL: the library
  * then uses the CUDA stream-ordered allocator (cudaMallocAsync).  Outputs of
  * betty_extract_blocks / betty_reg_build / betty_sage_fwd and plan arenas come
- * from this allocator and are released with the matching *_free call. */
+ * from this allocator and are released with the matching *_free call.
+ * Calls on one context must be ordered on ONE stream (or otherwise serialised):
+ * the context's device scratch -- scan flags, work-claim counters (aggregation,
+ * extraction, row-GEMM tile claims), loss partials -- is shared by its calls and
+ * reset by each kernel for the next one.  A plan's in-step REG rebuild uses its
+ * own side-stream scratch.  Concurrent work needs one context per stream. */
 BETTY_API betty_status betty_ctx_create(int device, betty_alloc_fn alloc, betty_free_fn dealloc, void* user, betty_ctx** out);
 BETTY_API void betty_ctx_destroy(betty_ctx* ctx);
 BETTY_API const char* betty_last_error(const betty_ctx* ctx);
