@@ -7,8 +7,9 @@
 //             deterministic ordered reduction that ADDS into the flat gradient
 //             (fused accumulation across micro-batches, a6) with the GEMM ->
 //             parameter layout mapping.
-// The tcgen05 tensor-core path (gemm_tc.cu) replaces these in BF16 mode for
-// the large shapes; these stay the FP32-mode path and the small-shape path.
+// The tcgen05 tensor-core path (gemm_tc.cu: bf16, and fp32 as 3xTF32) takes
+// every shape it supports in both modes; these kernels remain for the shapes
+// it rejects (and k_red_final serves both paths).
 #include <algorithm>
 #include "common.cuh"
 #include "internal.h"
