@@ -115,7 +115,7 @@ __global__ void __launch_bounds__(SCAN_THREADS) k_scan(const Tin* __restrict__ i
         }
         __syncthreads();
         // 3. the chunk's inclusive sums, written to out[i + 1]; the next tile's loads are issued before
-        // this tile's block scan (a solo CTA walks many tiles)
+        // this tile's block scan (chunks of several tiles: n > 1.2 M)
         int64_t run = s_prefix;
         for (int64_t base = lo; base < hi; base += SCAN_TILE) {
             const int64_t i = base + toff;
