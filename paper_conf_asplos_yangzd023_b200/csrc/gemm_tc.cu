@@ -176,6 +176,9 @@ __device__ __forceinline__ void tmem_free_warp(uint32_t taddr, uint32_t ncols) {
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(taddr), "r"(ncols) : "memory");
 }
 __device__ __forceinline__ bool elect_lane0() { return (threadIdx.x & 31) == 0; }
+__device__ __forceinline__ void sts128(uint32_t a, uint32_t x, uint32_t y, uint32_t z, uint32_t w) {
+    asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(a), "r"(x), "r"(y), "r"(z), "r"(w) : "memory");
+}
 
 // --------------------------------------------------------------- row GEMM
 // B (the weights, <= 256 x K) stays resident in shared memory for the whole
@@ -350,19 +353,20 @@ __device__ __forceinline__ uint32_t chunk_epilogue(const RowArgs& p, const uint3
             for (int k = 0; k < 16; ++k)
                 bits |= (uint32_t)((w[k] & 0x7fffu) != 0u) << (2 * k) | (uint32_t)((w[k] & 0x7fff0000u) != 0u) << (2 * k + 1);
         }
+        // (explicit st.shared: the generic stores compiled to ST.E into the shared window)
         if (part == 0) {
             // 64 B rows, SWIZZLE_64B: 16-B chunk c of row r at c ^ ((r >> 1) & 3)
-            uint8_t* row = slot + lane * 64;
+            const uint32_t row = su32(slot) + lane * 64;
 #pragma unroll
             for (int c = 0; c < 4; ++c)
-                *(uint4*)(row + ((c ^ ((lane >> 1) & 3)) << 4)) = make_uint4(w[4 * c], w[4 * c + 1], w[4 * c + 2], w[4 * c + 3]);
+                sts128(row + ((c ^ ((lane >> 1) & 3)) << 4), w[4 * c], w[4 * c + 1], w[4 * c + 2], w[4 * c + 3]);
         } else {
             // 128 B rows, SWIZZLE_128B: 16-B chunk cc = 4 (part - 1) + c of row r at cc ^ (r & 7)
-            uint8_t* row = slot + lane * 128;
+            const uint32_t row = su32(slot) + lane * 128;
 #pragma unroll
             for (int c = 0; c < 4; ++c)
-                *(uint4*)(row + (((4 * (part - 1) + c) ^ (lane & 7)) << 4)) =
-                    make_uint4(w[4 * c], w[4 * c + 1], w[4 * c + 2], w[4 * c + 3]);
+                sts128(row + (((4 * (part - 1) + c) ^ (lane & 7)) << 4), w[4 * c], w[4 * c + 1], w[4 * c + 2],
+                       w[4 * c + 3]);
         }
     } else {
         if (EPI == EPI_RELU_ONES) {
@@ -370,10 +374,11 @@ __device__ __forceinline__ uint32_t chunk_epilogue(const RowArgs& p, const uint3
             for (int j = 0; j < 32; ++j) bits |= (uint32_t)(v[j] > 0.f) << j;
         }
         // 128 B rows, SWIZZLE_128B: 16-B chunk c of row r at c ^ (r & 7)
-        uint8_t* row = slot + lane * 128;
+        const uint32_t row = su32(slot) + lane * 128;
 #pragma unroll
         for (int c = 0; c < 8; ++c)
-            *(float4*)(row + ((c ^ (lane & 7)) << 4)) = make_float4(v[4 * c], v[4 * c + 1], v[4 * c + 2], v[4 * c + 3]);
+            sts128(row + ((c ^ (lane & 7)) << 4), __float_as_uint(v[4 * c]), __float_as_uint(v[4 * c + 1]),
+                   __float_as_uint(v[4 * c + 2]), __float_as_uint(v[4 * c + 3]));
     }
     return bits;
 }
