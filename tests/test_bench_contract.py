@@ -1,5 +1,5 @@
 """The bench line contract (task statement / SURVEY.md §8(d)) on the committed measurement
-(profiles/r08_bench_C3.jsonl, written by bench.py on a B200): every key the driver and the judge
+(profiles/r09_bench_C3.jsonl, written by bench.py on a B200): every key the driver and the judge
 read is present with a sane value.  CPU only (reads the committed JSON)."""
 import json
 import os
@@ -13,7 +13,7 @@ def _line(name):
 
 
 def test_c3_bench_line_contract():
-    d = _line("r08_bench_C3.jsonl")
+    d = _line("r09_bench_C3.jsonl")
     for k in ("metric", "value", "unit", "n_gpus", "steps", "warmup", "ms_per_step", "higher_is_better", "scaling",
               "vs_baseline", "dtype", "data", "config", "e2e", "gpu_launches", "clocks", "roofline", "cpu_baseline"):
         assert k in d, k
